@@ -1,0 +1,201 @@
+/*
+ * dbc.h -- C ABI of the B200 dynamic betweenness-centrality library (libdbc.so).
+ *
+ * Method: McLaughlin & Bader, "Revisiting Edge and Node Parallelism for Dynamic
+ * GPU Graph Analytics".  Citations are "P:<line>" into
+ * /root/reference/PAPER.md, plus the section / algorithm / equation.
+ *
+ *  - The library stores, for each root s of a root set R, the BFS distance
+ *    d_s(t), the shortest-path count sigma_st and the dependency delta_s(t) for
+ *    every vertex t (Sec. II-D), and the betweenness partial
+ *    BC(v) = sum_{s in R, s != v} delta_s(v) (Eq. (3); ordered pairs,
+ *    unscaled -- DESIGN.md reading R1).
+ *  - dbc_static_compute runs Brandes' algorithm (Alg. 1) over the
+ *    local roots: it builds the state and is the GPU recompute baseline
+ *    (Table III).
+ *  - dbc_insert_edges applies edge insertions one at a time (Sec. IV):
+ *    for every root the insertion is classified by d_s(u) vs d_s(v) (Cases 1/2/3,
+ *    P:148-159); affected vertices get d/sigma repaired by a frontier-queued
+ *    forward pass (Alg. 2 stage 2 / Alg. 5) and delta/BC by a
+ *    reverse level-ordered pass (Alg. 2 stage 3 / Alg. 7 / Alg. 8, P:198-240,
+ *    P:366-432).  The result equals a recompute from scratch on the new graph.
+ *
+ * Conventions shared by every call
+ *  - Every call returns dbc_status (0 = DBC_OK, < 0 = error).  No exception,
+ *    abort or exit crosses the ABI.  On error, dbc_last_error(ctx) holds a
+ *    one-line message and the context state is unchanged unless stated.
+ *  - Vertices are int32 in [0, n).  Unreachable: d = DBC_INF (INT32_MAX),
+ *    sigma = 0, delta = 0.  delta_s(s) = 0 by convention.
+ *  - Host pointers are borrowed for the duration of the call only (copied).
+ *    Device pointers (suffix _device) must be device memory of opt->device and
+ *    must stay valid until the work enqueued by the call has completed on the
+ *    context stream.
+ *  - All device work runs on one CUDA stream (opt->stream, or a stream the
+ *    library creates).  Calls returning host data synchronise that stream.
+ *  - A context is not thread-safe.  Several contexts may coexist (e.g. one per
+ *    GPU and rank).
+ *  - Multi-GPU: every rank passes the FULL root list; rank r owns root slots
+ *    with slot % world == r.  BC partials are summed
+ *    across ranks by the caller (dbc_get_bc_partial_device + an NCCL
+ *    all-reduce) -- the only cross-GPU exchange of the method.
+ */
+#ifndef DBC_H
+#define DBC_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define DBC_INF INT32_MAX
+#define DBC_ABI_VERSION 1
+
+typedef struct dbc_ctx dbc_ctx; /* opaque; owns all device memory it allocates */
+
+typedef enum {
+    DBC_OK = 0,
+    DBC_EINVAL = -1,     /* bad argument (NULL, n < 1, bad CSR, bad slot, ...) */
+    DBC_ENOMEM = -2,     /* device or host allocation failed */
+    DBC_ECUDA = -3,      /* CUDA runtime error (message in dbc_last_error) */
+    DBC_ENCCL = -4,      /* reserved: collective failure */
+    DBC_ESTATE = -5,     /* call out of order, e.g. insert before static_compute */
+    DBC_EEDGE = -6,      /* self loop, out-of-range vertex, edge already present,
+                            or duplicate edge within a batch; batch not applied */
+    DBC_ECAPACITY = -7,  /* inserted-edge capacity (opt.edge_capacity) exhausted */
+    DBC_ENUMERIC = -8    /* a shortest-path count overflowed fp64 to +inf */
+} dbc_status;
+
+/* Flags for dbc_options.flags */
+#define DBC_FLAG_MODE_S   0x1u /* one update launch per insertion (paper structure,
+                                  P:244-252); default is the root-asynchronous
+                                  batch kernel (Mode A, one launch per batch).
+                                  Both give identical d/sigma.                     */
+#define DBC_FLAG_TIMING   0x2u /* record CUDA events around the library's kernels;
+                                  read with dbc_get_timings                        */
+#define DBC_FLAG_EXACT_BC 0x4u /* dbc_get_bc / dbc_get_bc_partial_device rebase the
+                                  partial as sum over local slots of delta_s(v)
+                                  (Eq. (3)) instead of the incrementally updated
+                                  value: removes drift over long streams          */
+
+typedef struct {
+    int32_t device;        /* CUDA device ordinal (default 0)                      */
+    int32_t rank;          /* this process's rank in [0, world) (default 0)        */
+    int32_t world;         /* number of ranks / GPUs sharing the root set (def. 1) */
+    int32_t workers;       /* persistent worker CTAs; 0 = automatic                */
+    int64_t edge_capacity; /* max undirected edges inserted over the context's
+                              lifetime; 0 = automatic (max(2^16, m/4))            */
+    void *stream;          /* cudaStream_t to run on; NULL = library-owned stream  */
+    uint32_t flags;        /* DBC_FLAG_*                                           */
+    uint32_t reserved[7];  /* must be zero                                         */
+} dbc_options;
+
+/* Per-call counters.  Filled when a non-NULL pointer is passed (synchronises). */
+typedef struct {
+    int64_t insertions;      /* edges inserted by the call                          */
+    int64_t case_count[3];   /* (root, insertion) scenarios in Case 1 / 2 / 3 */
+    int64_t touched;         /* vertices touched (t[v] != untouched)       */
+    int64_t down_vertices;   /* vertices whose sigma was recomputed (stage 2)        */
+    int64_t edges_scanned;   /* adjacency entries read                               */
+    int64_t alg_bytes;       /* algorithmic bytes of the update    */
+} dbc_insert_stats;
+
+typedef struct {
+    float append_ms;   /* graph validation + append of the last insert call    */
+    float update_ms;   /* update kernel(s) of the last insert call             */
+    float static_ms;   /* last dbc_static_compute                              */
+    int32_t update_launches;  /* update kernel launches in the last insert call */
+    int32_t kernel_launches;  /* all library kernels launched by the last insert call */
+    int64_t static_alg_bytes; /* algorithmic bytes of the last static compute   */
+    /* cumulative since dbc_create / dbc_reset_timings: */
+    double append_ms_total;
+    double update_ms_total;
+    int64_t update_launches_total;
+    int64_t kernel_launches_total;
+    int64_t insertions_total;
+    int64_t alg_bytes_total;   /* update kernels' algorithmic bytes            */
+} dbc_timings;
+
+/* Fills *opt with defaults (device 0, rank 0, world 1, automatic sizes). */
+void dbc_options_default(dbc_options *opt);
+
+/* Creates a context from an undirected graph in CSR form and a root set.
+ *  n        number of vertices, >= 1
+ *  row_ptr  host int64[n+1], row_ptr[0] = 0, non-decreasing
+ *  col      host int32[row_ptr[n]]; the CSR must be symmetric, without self
+ *           loops or duplicate entries (undirected).  The order
+ *           of each row is the canonical adjacency order; inserted neighbours
+ *           are appended after it in insertion order.
+ *  roots    host int32[k], distinct, in range (the sampled sources)
+ *  k        >= 0 (k = 0 gives BC = 0)
+ *  opt      nullable (defaults)
+ * Validates everything (O(m log) on the host) and uploads the CSR.  The
+ * per-root state is allocated but undefined until dbc_static_compute.
+ * Errors: DBC_EINVAL, DBC_ENOMEM, DBC_ECUDA. */
+dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_ptr,
+                      const int32_t *col, const int32_t *roots, int32_t k,
+                      const dbc_options *opt);
+
+/* Brandes over this rank's root shard (Alg. 1): resets and
+ * recomputes d, sigma, delta of every local root and the BC partial on the
+ * CURRENT graph (all inserted edges included).  Asynchronous on the stream. */
+dbc_status dbc_static_compute(dbc_ctx *c);
+
+/* Inserts count >= 0 undirected edges (u[i], v[i]) given in HOST memory, with
+ * exactly the semantics of count sequential single-edge insertions (P:440,
+ * "reinserted one at a time").  The whole batch is validated before anything
+ * changes (self loop, range, already present, duplicate in batch ->
+ * DBC_EEDGE; capacity -> DBC_ECAPACITY).  Requires a prior
+ * dbc_static_compute (DBC_ESTATE).  Synchronises once after validation; the
+ * update itself is enqueued asynchronously.  stats: nullable. */
+dbc_status dbc_insert_edges(dbc_ctx *c, const int32_t *u, const int32_t *v,
+                            int64_t count, dbc_insert_stats *stats);
+
+/* Same as dbc_insert_edges with u, v in DEVICE memory (int32[count] each). */
+dbc_status dbc_insert_edges_device(dbc_ctx *c, const int32_t *u_device,
+                                   const int32_t *v_device, int64_t count,
+                                   dbc_insert_stats *stats);
+
+/* Copies this rank's BC partial (sum over LOCAL roots, Eq. (3)) to host
+ * bc[n].  With world == 1 this is the global BC.  Synchronises.  Returns
+ * DBC_ENUMERIC if an earlier update overflowed. */
+dbc_status dbc_get_bc(dbc_ctx *c, double *bc);
+
+/* Device pointer to this rank's BC partial, fp64[n] (valid until destroy);
+ * for an in-place NCCL sum-all-reduce across ranks.  Not synchronising. */
+dbc_status dbc_get_bc_partial_device(dbc_ctx *c, double **bc_device);
+
+/* Copies one root's state to host arrays of n elements (any may be NULL).
+ * slot: global slot in [0, k); must be owned by this rank (slot % world ==
+ * rank), else DBC_EINVAL.  Synchronises. */
+dbc_status dbc_get_root_state(dbc_ctx *c, int32_t slot, int32_t *d,
+                              double *sigma, double *delta);
+
+/* Number of root slots owned by this rank. */
+dbc_status dbc_num_local_roots(const dbc_ctx *c, int32_t *k_local);
+
+/* Waits for all enqueued work; reports deferred errors (DBC_ENUMERIC, DBC_ECUDA). */
+dbc_status dbc_synchronize(dbc_ctx *c);
+
+/* Kernel timings (CUDA events on the context stream; requires DBC_FLAG_TIMING)
+ * of the last calls plus cumulative totals.  Synchronises. */
+dbc_status dbc_get_timings(dbc_ctx *c, dbc_timings *t);
+
+/* Zeroes the cumulative fields of dbc_timings.  Synchronises. */
+dbc_status dbc_reset_timings(dbc_ctx *c);
+
+/* Device memory held by the context, in bytes. */
+dbc_status dbc_device_bytes(const dbc_ctx *c, int64_t *bytes);
+
+const char *dbc_strerror(dbc_status s);
+const char *dbc_last_error(const dbc_ctx *c);
+int32_t dbc_abi_version(void);
+
+/* Frees everything; NULL is a no-op. */
+void dbc_destroy(dbc_ctx *c);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DBC_H */

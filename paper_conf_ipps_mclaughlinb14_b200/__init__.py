@@ -1,0 +1,23 @@
+"""B200-native dynamic betweenness centrality (McLaughlin & Bader, dblp conf/ipps 2014).
+
+The compute path is libdbc.so (hand-written sm_100a CUDA behind the C ABI of
+include/dbc.h); this package is the thin Python binding.  See DESIGN.md.
+"""
+
+from .dbc import (  # noqa: F401
+    DBC_INF,
+    FLAG_EXACT_BC,
+    FLAG_MODE_S,
+    FLAG_TIMING,
+    DBCError,
+    DynamicBC,
+    LIB_PATH,
+    allreduce_bc,
+    load_library,
+    local_slots,
+)
+
+__all__ = [
+    "DynamicBC", "DBCError", "DBC_INF", "FLAG_MODE_S", "FLAG_TIMING", "FLAG_EXACT_BC",
+    "LIB_PATH", "load_library", "local_slots", "allreduce_bc",
+]

@@ -1,0 +1,654 @@
+// api.cu -- the C ABI of libdbc (include/dbc.h): context, HBM arena, root
+// sharding, batch flow, error model.  Every compute step runs in the kernels of
+// static_brandes.cu / update.cu / graph.cu; this file only validates,
+// allocates, launches and copies.
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "dbc.h"
+#include "dbc_internal.cuh"
+#include "graph_ops.h"
+
+using namespace dbc;
+
+struct dbc_ctx {
+    int device = 0, rank = 0, world = 1;
+    uint32_t flags = 0;
+    int32_t n = 0;
+    int64_t nnz = 0, nnz0 = 0, col_cap = 0;
+    int64_t edge_cap = 0, inserted = 0;
+    int32_t k = 0, k_loc = 0;
+    std::vector<int32_t> roots_local;
+    cudaStream_t stream = nullptr;
+    bool own_stream = false;
+    int workers = 0;
+    int nsm = 148;
+    bool have_state = false;
+    uint64_t epoch_used = 0;
+
+    // graph double buffer
+    int32_t *rp[2] = {nullptr, nullptr};
+    int32_t *col[2] = {nullptr, nullptr};
+    int cur = 0;
+    AppendBufs ab{};
+    int32_t *bu = nullptr, *bv = nullptr;  // host-API batch staging
+
+    // state
+    int32_t *d = nullptr;
+    double2 *sd = nullptr;
+    double *bc = nullptr;
+    int32_t *roots_d = nullptr;
+
+    Scratch ws{};
+    int32_t *next_slot = nullptr;
+    unsigned long long *stats = nullptr;
+    int32_t *err = nullptr;
+
+    std::vector<void *> allocs;
+    int64_t bytes = 0;
+
+    cudaEvent_t ev[6] = {};
+    bool ev_ok = false;
+    dbc_timings tm{};
+    bool tm_pending = false, tm_static = false;
+    unsigned long long bytes_base = 0;
+
+    std::string msg;
+};
+
+static thread_local std::string g_create_msg;
+
+static dbc_status fail(dbc_ctx *c, dbc_status s, const char *fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    if (c)
+        c->msg = buf;
+    else
+        g_create_msg = buf;
+    return s;
+}
+
+#define CK(call)                                                                           \
+    do {                                                                                   \
+        cudaError_t e_ = (call);                                                           \
+        if (e_ != cudaSuccess)                                                             \
+            return fail(c, DBC_ECUDA, "%s: %s (%s:%d)", #call, cudaGetErrorString(e_),     \
+                        __FILE__, __LINE__);                                               \
+    } while (0)
+
+template <class T>
+static dbc_status dalloc(dbc_ctx *c, T **p, size_t count) {
+    size_t b = std::max<size_t>(count, 1) * sizeof(T);
+    void *q = nullptr;
+    cudaError_t e = cudaMalloc(&q, b);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return fail(c, DBC_ENOMEM, "cudaMalloc(%zu bytes) failed: %s", b, cudaGetErrorString(e));
+    }
+    c->allocs.push_back(q);
+    c->bytes += (int64_t)b;
+    *p = (T *)q;
+    return DBC_OK;
+}
+
+#define TRY(x)                          \
+    do {                                \
+        dbc_status s_ = (x);            \
+        if (s_ != DBC_OK) return s_;    \
+    } while (0)
+
+extern "C" {
+
+void dbc_options_default(dbc_options *opt) {
+    if (!opt) return;
+    std::memset(opt, 0, sizeof(*opt));
+    opt->world = 1;
+}
+
+int32_t dbc_abi_version(void) { return DBC_ABI_VERSION; }
+
+const char *dbc_strerror(dbc_status s) {
+    switch (s) {
+        case DBC_OK: return "ok";
+        case DBC_EINVAL: return "invalid argument";
+        case DBC_ENOMEM: return "out of memory";
+        case DBC_ECUDA: return "CUDA error";
+        case DBC_ENCCL: return "collective error";
+        case DBC_ESTATE: return "call out of order";
+        case DBC_EEDGE: return "invalid edge in batch";
+        case DBC_ECAPACITY: return "inserted-edge capacity exhausted";
+        case DBC_ENUMERIC: return "shortest-path count overflowed";
+    }
+    return "unknown status";
+}
+
+const char *dbc_last_error(const dbc_ctx *c) { return c ? c->msg.c_str() : g_create_msg.c_str(); }
+
+void dbc_destroy(dbc_ctx *c) {
+    if (!c) return;
+    cudaSetDevice(c->device);
+    if (c->stream) cudaStreamSynchronize(c->stream);
+    for (void *p : c->allocs) cudaFree(p);
+    if (c->ev_ok)
+        for (auto &e : c->ev) cudaEventDestroy(e);
+    if (c->own_stream && c->stream) cudaStreamDestroy(c->stream);
+    delete c;
+}
+
+}  // extern "C"
+
+// Host CSR validation: symmetric, no self loops, no duplicate entries.
+static bool validate_csr(int32_t n, const int64_t *rp, const int32_t *col, std::string &why) {
+    if (rp[0] != 0) { why = "row_ptr[0] != 0"; return false; }
+    for (int32_t v = 0; v < n; ++v)
+        if (rp[v + 1] < rp[v]) { why = "row_ptr not non-decreasing"; return false; }
+    const int64_t nnz = rp[n];
+    for (int64_t j = 0; j < nnz; ++j)
+        if (col[j] < 0 || col[j] >= n) { why = "col entry out of range"; return false; }
+    // sorted copies of every row, then per-entry reverse lookup
+    std::vector<int32_t> srt(col, col + nnz);
+    unsigned nt = std::max(1u, std::min(32u, std::thread::hardware_concurrency()));
+    std::vector<std::string> whys(nt);
+    std::vector<int> ok(nt, 1);
+    auto sort_rows = [&](unsigned t) {
+        for (int64_t v = t; v < n; v += nt) std::sort(srt.begin() + rp[v], srt.begin() + rp[v + 1]);
+    };
+    auto check_rows = [&](unsigned t) {
+        for (int64_t v = t; v < n && ok[t]; v += nt) {
+            for (int64_t j = rp[v]; j < rp[v + 1]; ++j) {
+                const int32_t y = srt[j];
+                if (y == v) { ok[t] = 0; whys[t] = "self loop at vertex " + std::to_string(v); break; }
+                if (j > rp[v] && srt[j - 1] == y) {
+                    ok[t] = 0; whys[t] = "duplicate entry in row " + std::to_string(v); break;
+                }
+                if (!std::binary_search(srt.begin() + rp[y], srt.begin() + rp[y + 1], (int32_t)v)) {
+                    ok[t] = 0;
+                    whys[t] = "CSR not symmetric: " + std::to_string(v) + "->" + std::to_string(y);
+                    break;
+                }
+            }
+        }
+    };
+    {
+        std::vector<std::thread> th;
+        for (unsigned t = 0; t < nt; ++t) th.emplace_back(sort_rows, t);
+        for (auto &x : th) x.join();
+    }
+    {
+        std::vector<std::thread> th;
+        for (unsigned t = 0; t < nt; ++t) th.emplace_back(check_rows, t);
+        for (auto &x : th) x.join();
+    }
+    for (unsigned t = 0; t < nt; ++t)
+        if (!ok[t]) { why = whys[t]; return false; }
+    return true;
+}
+
+static GView view_of(const dbc_ctx *c) {
+    GView g;
+    g.rp = c->rp[c->cur];
+    g.col = c->col[c->cur];
+    g.xinfo = c->ab.xinfo;
+    g.xtag = c->ab.xtag;
+    return g;
+}
+
+static Scratch worker_scratch(const dbc_ctx *c) { return c->ws; }
+
+static dbc_status reset_epochs(dbc_ctx *c) {
+    const size_t nw = (size_t)c->workers, n = (size_t)c->n;
+    if (!nw) return DBC_OK;
+    CK(cudaMemsetAsync(c->ws.mark, 0, sizeof(uint32_t) * nw * n, c->stream));
+    CK(cudaMemsetAsync(c->ws.lowrec, 0, sizeof(unsigned long long) * nw * n, c->stream));
+    CK(cudaMemsetAsync(c->ws.wepoch, 0, sizeof(uint32_t) * nw, c->stream));
+    c->epoch_used = 0;
+    return DBC_OK;
+}
+
+extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_ptr,
+                                 const int32_t *col, const int32_t *roots, int32_t k,
+                                 const dbc_options *opt_in) {
+    dbc_ctx *c = nullptr;
+    if (!out) return fail(nullptr, DBC_EINVAL, "out is NULL");
+    *out = nullptr;
+    if (n < 1) return fail(nullptr, DBC_EINVAL, "n must be >= 1");
+    if (!row_ptr || (!col && row_ptr && row_ptr[n] > 0)) return fail(nullptr, DBC_EINVAL, "NULL CSR");
+    if (k < 0 || (k > 0 && !roots)) return fail(nullptr, DBC_EINVAL, "bad roots");
+    dbc_options opt;
+    if (opt_in)
+        opt = *opt_in;
+    else
+        dbc_options_default(&opt);
+    if (opt.world < 1 || opt.rank < 0 || opt.rank >= opt.world)
+        return fail(nullptr, DBC_EINVAL, "bad rank/world %d/%d", opt.rank, opt.world);
+    if (opt.edge_capacity < 0 || opt.workers < 0) return fail(nullptr, DBC_EINVAL, "bad sizes");
+    for (int i = 0; i < 7; ++i)
+        if (opt.reserved[i]) return fail(nullptr, DBC_EINVAL, "reserved fields must be zero");
+    {
+        std::string why;
+        if (!validate_csr(n, row_ptr, col, why)) return fail(nullptr, DBC_EINVAL, "bad CSR: %s", why.c_str());
+    }
+    {
+        std::vector<int32_t> r(roots, roots + k);
+        for (int32_t x : r)
+            if (x < 0 || x >= n) return fail(nullptr, DBC_EINVAL, "root %d out of range", x);
+        std::sort(r.begin(), r.end());
+        if (std::adjacent_find(r.begin(), r.end()) != r.end())
+            return fail(nullptr, DBC_EINVAL, "roots not distinct");
+    }
+
+    c = new dbc_ctx();
+    c->device = opt.device;
+    c->rank = opt.rank;
+    c->world = opt.world;
+    c->flags = opt.flags;
+    c->n = n;
+    c->k = k;
+    c->nnz = c->nnz0 = row_ptr[n];
+    const int64_t m = c->nnz0 / 2;
+    c->edge_cap = opt.edge_capacity ? opt.edge_capacity : std::max<int64_t>(1 << 16, m / 4);
+    c->col_cap = c->nnz0 + 2 * c->edge_cap;
+    if (c->col_cap >= (int64_t)INT32_MAX - 1) {
+        dbc_status s = fail(nullptr, DBC_EINVAL, "graph + capacity too large for int32 offsets (%lld)",
+                            (long long)c->col_cap);
+        delete c;
+        return s;
+    }
+    for (int32_t slot = opt.rank; slot < k; slot += opt.world) c->roots_local.push_back(roots[slot]);
+    c->k_loc = (int32_t)c->roots_local.size();
+
+    auto bail = [&](dbc_status s) {
+        g_create_msg = c->msg;
+        dbc_destroy(c);
+        return s;
+    };
+    if (cudaSetDevice(c->device) != cudaSuccess) {
+        cudaGetLastError();
+        fail(c, DBC_ECUDA, "cudaSetDevice(%d) failed", c->device);
+        return bail(DBC_ECUDA);
+    }
+    cudaDeviceGetAttribute(&c->nsm, cudaDevAttrMultiProcessorCount, c->device);
+    if (opt.stream) {
+        c->stream = (cudaStream_t)opt.stream;
+    } else {
+        if (cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) != cudaSuccess) {
+            fail(c, DBC_ECUDA, "stream creation failed");
+            return bail(DBC_ECUDA);
+        }
+        c->own_stream = true;
+    }
+    for (auto &e : c->ev)
+        if (cudaEventCreate(&e) != cudaSuccess) {
+            fail(c, DBC_ECUDA, "event creation failed");
+            return bail(DBC_ECUDA);
+        }
+    c->ev_ok = true;
+
+    // workers: persistent CTAs; bounded by roots and by a scratch-memory budget
+    const size_t per_worker = (size_t)n * (4 + 8 + 8 + 4 + 4 + 8 + 4 + 4 + 4 + 4) + (size_t)(n + 2) * 4 + 64;
+    size_t free_b = 0, total_b = 0;
+    cudaMemGetInfo(&free_b, &total_b);
+    const size_t state_b = (size_t)c->k_loc * n * 20 + (size_t)c->col_cap * 8 + (size_t)n * 40;
+    size_t budget = free_b > state_b ? (free_b - state_b) / 2 : 0;
+    int want = opt.workers ? opt.workers : 2 * c->nsm;
+    want = std::min(want, c->k_loc);
+    int fit = (int)std::min<size_t>(budget / per_worker, 1 << 20);
+    c->workers = std::max(0, std::min(want, fit));
+    if (c->k_loc > 0 && c->workers == 0) {
+        fail(c, DBC_ENOMEM, "not enough device memory for one worker (%zu bytes)", per_worker);
+        return bail(DBC_ENOMEM);
+    }
+
+    dbc_status s;
+#define AL(p, cnt)                        \
+    if ((s = dalloc(c, &(p), (cnt))) != DBC_OK) return bail(s);
+    AL(c->rp[0], (size_t)n + 1);
+    AL(c->rp[1], (size_t)n + 1);
+    AL(c->col[0], (size_t)c->col_cap);
+    AL(c->col[1], (size_t)c->col_cap);
+    const size_t e2 = (size_t)2 * c->edge_cap;
+    AL(c->ab.slot, e2);
+    AL(c->ab.xtag, e2);
+    AL(c->ab.gnbr, e2);
+    AL(c->ab.xinfo, (size_t)n);
+    AL(c->ab.xcnt, (size_t)n);
+    AL(c->ab.xoff, (size_t)n);
+    AL(c->ab.deg, (size_t)n + 1);
+    AL(c->ab.sums, (size_t)scan_sums_capacity(n + 1));
+    AL(c->ab.bad, 1);
+    AL(c->bu, (size_t)c->edge_cap);
+    AL(c->bv, (size_t)c->edge_cap);
+    const size_t kn = (size_t)c->k_loc * n;
+    AL(c->d, kn);
+    AL(c->sd, kn);
+    AL(c->bc, (size_t)n);
+    AL(c->roots_d, (size_t)c->k_loc);
+    const size_t wn = (size_t)c->workers * n;
+    AL(c->ws.mark, wn);
+    AL(c->ws.lowrec, wn);
+    AL(c->ws.dacc, wn);
+    AL(c->ws.Dv, wn);
+    AL(c->ws.Dold, wn);
+    AL(c->ws.Dsig, wn);
+    AL(c->ws.Doff, (size_t)c->workers * (n + 2));
+    AL(c->ws.U0, wn);
+    AL(c->ws.U1, wn);
+    AL(c->ws.Rv, wn);
+    AL(c->ws.Rl, wn);
+    AL(c->ws.wepoch, (size_t)c->workers);
+    AL(c->next_slot, 1);
+    AL(c->stats, (size_t)kStCount);
+    AL(c->err, 1);
+#undef AL
+
+    // upload CSR (int32 offsets), roots; zero scratch
+    {
+        std::vector<int32_t> rp32((size_t)n + 1);
+        for (int32_t v = 0; v <= n; ++v) rp32[v] = (int32_t)row_ptr[v];
+        if (cudaMemcpy(c->rp[0], rp32.data(), sizeof(int32_t) * (n + 1), cudaMemcpyHostToDevice) != cudaSuccess ||
+            (c->nnz0 && cudaMemcpy(c->col[0], col, sizeof(int32_t) * c->nnz0, cudaMemcpyHostToDevice) != cudaSuccess) ||
+            (c->k_loc && cudaMemcpy(c->roots_d, c->roots_local.data(), sizeof(int32_t) * c->k_loc,
+                                    cudaMemcpyHostToDevice) != cudaSuccess)) {
+            fail(c, DBC_ECUDA, "upload failed: %s", cudaGetErrorString(cudaGetLastError()));
+            return bail(DBC_ECUDA);
+        }
+    }
+    if (c->workers) cudaMemsetAsync(c->ws.dacc, 0, sizeof(double) * wn, c->stream);
+    if ((s = reset_epochs(c)) != DBC_OK) return bail(s);
+    cudaMemsetAsync(c->bc, 0, sizeof(double) * n, c->stream);
+    cudaMemsetAsync(c->err, 0, sizeof(int32_t), c->stream);
+    cudaMemsetAsync(c->stats, 0, sizeof(unsigned long long) * kStCount, c->stream);
+    if (cudaStreamSynchronize(c->stream) != cudaSuccess) {
+        fail(c, DBC_ECUDA, "init failed: %s", cudaGetErrorString(cudaGetLastError()));
+        return bail(DBC_ECUDA);
+    }
+    *out = c;
+    return DBC_OK;
+}
+
+// fold the event times of the previous insert call into the totals (its work
+// has completed whenever this is called after a stream synchronisation)
+static dbc_status fold_timings(dbc_ctx *c) {
+    if (c->tm_pending) {
+        CK(cudaEventElapsedTime(&c->tm.append_ms, c->ev[0], c->ev[1]));
+        CK(cudaEventElapsedTime(&c->tm.update_ms, c->ev[2], c->ev[3]));
+        c->tm.append_ms_total += c->tm.append_ms;
+        c->tm.update_ms_total += c->tm.update_ms;
+        c->tm_pending = false;
+    }
+    if (c->tm_static) {
+        CK(cudaEventElapsedTime(&c->tm.static_ms, c->ev[4], c->ev[5]));
+        c->tm_static = false;
+    }
+    return DBC_OK;
+}
+
+extern "C" dbc_status dbc_static_compute(dbc_ctx *c) {
+    if (!c) return DBC_EINVAL;
+    CK(cudaSetDevice(c->device));
+    CK(cudaMemsetAsync(c->bc, 0, sizeof(double) * c->n, c->stream));
+    CK(cudaMemsetAsync(c->next_slot, 0, sizeof(int32_t), c->stream));
+    CK(cudaMemsetAsync(c->stats + kStStaticBytes, 0, sizeof(unsigned long long), c->stream));
+    const bool tm = c->flags & DBC_FLAG_TIMING;
+    if (tm) CK(cudaEventRecord(c->ev[4], c->stream));
+    if (c->workers) {
+        StaticArgs a;
+        a.g = view_of(c);
+        a.n = c->n;
+        a.k_loc = c->k_loc;
+        a.roots = c->roots_d;
+        a.d = c->d;
+        a.sd = c->sd;
+        a.bc = c->bc;
+        a.ws = worker_scratch(c);
+        a.next_slot = c->next_slot;
+        a.stats = c->stats;
+        a.err = c->err;
+        launch_static(a, c->workers, c->stream);
+        CK(cudaGetLastError());
+    }
+    if (tm) {
+        CK(cudaEventRecord(c->ev[5], c->stream));
+        c->tm_static = true;
+    }
+    c->have_state = true;
+    return DBC_OK;
+}
+
+static dbc_status read_stats(dbc_ctx *c, unsigned long long *h) {
+    CK(cudaMemcpyAsync(h, c->stats, sizeof(unsigned long long) * kStCount, cudaMemcpyDeviceToHost,
+                       c->stream));
+    CK(cudaStreamSynchronize(c->stream));
+    return DBC_OK;
+}
+
+static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, int64_t cnt,
+                                dbc_insert_stats *stats) {
+    if (!c->have_state) return fail(c, DBC_ESTATE, "dbc_static_compute must run before insertions");
+    if (cnt < 0 || (cnt > 0 && (!u || !v))) return fail(c, DBC_EINVAL, "bad batch");
+    if (cnt > INT32_MAX / 4) return fail(c, DBC_EINVAL, "batch too large");
+    if (c->inserted + cnt > c->edge_cap)
+        return fail(c, DBC_ECAPACITY, "edge capacity %lld exhausted (%lld inserted, batch %lld)",
+                    (long long)c->edge_cap, (long long)c->inserted, (long long)cnt);
+    CK(cudaSetDevice(c->device));
+    const bool tm = c->flags & DBC_FLAG_TIMING;
+    int launches = 0;
+    if (tm) CK(cudaEventRecord(c->ev[0], c->stream));
+    GView g = view_of(c);
+    launches += validate_batch(c->ab, g, c->rp[c->cur], c->n, u, v, cnt, c->stream);
+    CK(cudaGetLastError());
+    int32_t bad = 0;
+    CK(cudaMemcpyAsync(&bad, c->ab.bad, sizeof(int32_t), cudaMemcpyDeviceToHost, c->stream));
+    CK(cudaStreamSynchronize(c->stream));  // all earlier work is complete here
+    TRY(fold_timings(c));
+    if (bad) {
+        const char *why = (bad & 1) ? "self loop or vertex out of range"
+                          : (bad & 2) ? "edge already present"
+                                      : "duplicate edge within the batch";
+        return fail(c, DBC_EEDGE, "batch rejected: %s", why);
+    }
+    unsigned long long h0[kStCount] = {};
+    if (stats) TRY(read_stats(c, h0));
+    if (cnt == 0) {
+        if (stats) std::memset(stats, 0, sizeof(*stats));
+        return DBC_OK;
+    }
+    const int nb = 1 - c->cur;
+    launches += append_batch(c->ab, c->rp[c->cur], c->col[c->cur], c->rp[nb], c->col[nb], c->n,
+                             c->stream);
+    CK(cudaGetLastError());
+    c->cur = nb;
+    c->nnz += 2 * cnt;
+    c->inserted += cnt;
+    if (tm) CK(cudaEventRecord(c->ev[1], c->stream));
+
+    // epoch budget: each job of a worker consumes one epoch (30 bits available)
+    const uint64_t jobs = (uint64_t)c->k_loc * (uint64_t)cnt;
+    if (c->epoch_used + jobs + 1 >= (1ull << 30)) TRY(reset_epochs(c));
+    c->epoch_used += jobs;
+
+    UpdateArgs a;
+    a.g = view_of(c);
+    a.n = c->n;
+    a.k_loc = c->k_loc;
+    a.roots = c->roots_d;
+    a.d = c->d;
+    a.sd = c->sd;
+    a.bc = c->bc;
+    a.ins_u = u;
+    a.ins_v = v;
+    a.ws = worker_scratch(c);
+    a.next_slot = c->next_slot;
+    a.stats = c->stats;
+    a.err = c->err;
+    if (tm) CK(cudaEventRecord(c->ev[2], c->stream));
+    int ulaunch = 0;
+    if (c->workers) {
+        if (c->flags & DBC_FLAG_MODE_S) {
+            for (int64_t i = 0; i < cnt; ++i) {
+                CK(cudaMemsetAsync(c->next_slot, 0, sizeof(int32_t), c->stream));
+                a.ins_begin = (int32_t)i;
+                a.ins_end = (int32_t)i + 1;
+                launch_update(a, c->workers, c->stream);
+                ++ulaunch;
+            }
+        } else {
+            CK(cudaMemsetAsync(c->next_slot, 0, sizeof(int32_t), c->stream));
+            a.ins_begin = 0;
+            a.ins_end = (int32_t)cnt;
+            launch_update(a, c->workers, c->stream);
+            ++ulaunch;
+        }
+        CK(cudaGetLastError());
+    }
+    if (tm) {
+        CK(cudaEventRecord(c->ev[3], c->stream));
+        c->tm_pending = true;
+    }
+    launches += ulaunch;
+    c->tm.update_launches = ulaunch;
+    c->tm.kernel_launches = launches;
+    c->tm.update_launches_total += ulaunch;
+    c->tm.kernel_launches_total += launches;
+    c->tm.insertions_total += cnt;
+    if (stats) {
+        unsigned long long h[kStCount];
+        TRY(read_stats(c, h));
+        stats->insertions = cnt;
+        stats->case_count[0] = (int64_t)(h[kStCase1] - h0[kStCase1]);
+        stats->case_count[1] = (int64_t)(h[kStCase2] - h0[kStCase2]);
+        stats->case_count[2] = (int64_t)(h[kStCase3] - h0[kStCase3]);
+        stats->touched = (int64_t)(h[kStTouched] - h0[kStTouched]);
+        stats->down_vertices = (int64_t)(h[kStDown] - h0[kStDown]);
+        stats->edges_scanned = (int64_t)(h[kStScanned] - h0[kStScanned]);
+        stats->alg_bytes = (int64_t)(h[kStBytes] - h0[kStBytes]);
+    }
+    return DBC_OK;
+}
+
+extern "C" dbc_status dbc_insert_edges_device(dbc_ctx *c, const int32_t *u, const int32_t *v,
+                                              int64_t count, dbc_insert_stats *stats) {
+    if (!c) return DBC_EINVAL;
+    return insert_device(c, u, v, count, stats);
+}
+
+extern "C" dbc_status dbc_insert_edges(dbc_ctx *c, const int32_t *u, const int32_t *v, int64_t count,
+                                       dbc_insert_stats *stats) {
+    if (!c) return DBC_EINVAL;
+    if (count < 0 || (count > 0 && (!u || !v))) return fail(c, DBC_EINVAL, "bad batch");
+    if (c->inserted + count > c->edge_cap)
+        return fail(c, DBC_ECAPACITY, "edge capacity %lld exhausted (%lld inserted, batch %lld)",
+                    (long long)c->edge_cap, (long long)c->inserted, (long long)count);
+    if (!c->have_state) return fail(c, DBC_ESTATE, "dbc_static_compute must run before insertions");
+    CK(cudaSetDevice(c->device));
+    if (count) {
+        CK(cudaMemcpyAsync(c->bu, u, sizeof(int32_t) * count, cudaMemcpyHostToDevice, c->stream));
+        CK(cudaMemcpyAsync(c->bv, v, sizeof(int32_t) * count, cudaMemcpyHostToDevice, c->stream));
+    }
+    return insert_device(c, c->bu, c->bv, count, stats);
+}
+
+static dbc_status check_err(dbc_ctx *c) {
+    int32_t e = 0;
+    CK(cudaMemcpyAsync(&e, c->err, sizeof e, cudaMemcpyDeviceToHost, c->stream));
+    CK(cudaStreamSynchronize(c->stream));
+    if (e & kErrNumeric) return fail(c, DBC_ENUMERIC, "a shortest-path count overflowed fp64");
+    return DBC_OK;
+}
+
+extern "C" dbc_status dbc_synchronize(dbc_ctx *c) {
+    if (!c) return DBC_EINVAL;
+    CK(cudaSetDevice(c->device));
+    CK(cudaStreamSynchronize(c->stream));
+    return check_err(c);
+}
+
+extern "C" dbc_status dbc_get_bc_partial_device(dbc_ctx *c, double **p) {
+    if (!c || !p) return DBC_EINVAL;
+    CK(cudaSetDevice(c->device));
+    if ((c->flags & DBC_FLAG_EXACT_BC) && c->have_state && c->k_loc)
+        {
+        exact_bc(c->sd, c->roots_d, c->k_loc, c->n, c->bc, c->stream);
+        CK(cudaGetLastError());
+    }
+    *p = c->bc;
+    return DBC_OK;
+}
+
+extern "C" dbc_status dbc_get_bc(dbc_ctx *c, double *bc) {
+    if (!c || !bc) return DBC_EINVAL;
+    if (!c->have_state) return fail(c, DBC_ESTATE, "no state: call dbc_static_compute first");
+    double *p = nullptr;
+    TRY(dbc_get_bc_partial_device(c, &p));
+    CK(cudaMemcpyAsync(bc, p, sizeof(double) * c->n, cudaMemcpyDeviceToHost, c->stream));
+    return check_err(c);
+}
+
+extern "C" dbc_status dbc_get_root_state(dbc_ctx *c, int32_t slot, int32_t *d, double *sigma,
+                                         double *delta) {
+    if (!c) return DBC_EINVAL;
+    if (slot < 0 || slot >= c->k || slot % c->world != c->rank)
+        return fail(c, DBC_EINVAL, "slot %d not owned by rank %d", slot, c->rank);
+    if (!c->have_state) return fail(c, DBC_ESTATE, "no state: call dbc_static_compute first");
+    CK(cudaSetDevice(c->device));
+    const size_t li = (size_t)(slot - c->rank) / c->world, n = (size_t)c->n;
+    if (d) CK(cudaMemcpyAsync(d, c->d + li * n, sizeof(int32_t) * n, cudaMemcpyDeviceToHost, c->stream));
+    if (sigma || delta) {
+        std::vector<double2> tmp(n);
+        CK(cudaMemcpyAsync(tmp.data(), c->sd + li * n, sizeof(double2) * n, cudaMemcpyDeviceToHost,
+                           c->stream));
+        CK(cudaStreamSynchronize(c->stream));
+        for (size_t i = 0; i < n; ++i) {
+            if (sigma) sigma[i] = tmp[i].x;
+            if (delta) delta[i] = tmp[i].y;
+        }
+    }
+    return check_err(c);
+}
+
+extern "C" dbc_status dbc_num_local_roots(const dbc_ctx *c, int32_t *k_local) {
+    if (!c || !k_local) return DBC_EINVAL;
+    *k_local = c->k_loc;
+    return DBC_OK;
+}
+
+extern "C" dbc_status dbc_device_bytes(const dbc_ctx *c, int64_t *bytes) {
+    if (!c || !bytes) return DBC_EINVAL;
+    *bytes = c->bytes;
+    return DBC_OK;
+}
+
+extern "C" dbc_status dbc_get_timings(dbc_ctx *c, dbc_timings *t) {
+    if (!c || !t) return DBC_EINVAL;
+    CK(cudaSetDevice(c->device));
+    CK(cudaStreamSynchronize(c->stream));
+    TRY(fold_timings(c));
+    unsigned long long h[kStCount];
+    TRY(read_stats(c, h));
+    c->tm.static_alg_bytes = (int64_t)h[kStStaticBytes];
+    c->tm.alg_bytes_total = (int64_t)(h[kStBytes] - c->bytes_base);
+    *t = c->tm;
+    return DBC_OK;
+}
+
+extern "C" dbc_status dbc_reset_timings(dbc_ctx *c) {
+    if (!c) return DBC_EINVAL;
+    CK(cudaSetDevice(c->device));
+    CK(cudaStreamSynchronize(c->stream));
+    TRY(fold_timings(c));
+    unsigned long long h[kStCount];
+    TRY(read_stats(c, h));
+    c->bytes_base = h[kStBytes];
+    c->tm.append_ms_total = c->tm.update_ms_total = 0.0;
+    c->tm.update_launches_total = c->tm.kernel_launches_total = 0;
+    c->tm.insertions_total = c->tm.alg_bytes_total = 0;
+    return DBC_OK;
+}

@@ -1,0 +1,245 @@
+// graph.cu -- K5: batch validation and graph append (+ the exact-BC rebase).
+//
+// The paper neglects the cost of updating the graph ("We
+// neglect the cost of updating the graph ... techniques ... are discussed in
+// [23]").  Here the append is a handful of bulk kernels per batch: the new CSR
+// is the old one with each row extended by the batch's entries in insertion
+// order (canonical order, R5), written into the second graph buffer;
+// rows holding batch entries are flagged so the update kernel sees, for
+// insertion i, exactly the edges with insertion index <= i (Sec. IV: edges are
+// "reinserted into the graph one at a time").
+//
+// Validation (R16): range, self loop, already present, duplicate
+// within the batch -- all decided before the live graph or any state changes.
+#include <algorithm>
+
+#include "dbc_internal.cuh"
+#include "graph_ops.h"
+
+namespace dbc {
+
+static inline unsigned blocks_for(int64_t items, int threads) {
+    return (unsigned)std::max<int64_t>(1, (items + threads - 1) / threads);
+}
+
+// one warp per batch edge: range / self loop / presence in the current graph
+__global__ void k_validate_edges(GView g, int32_t n, const int32_t *u, const int32_t *v,
+                                 int64_t cnt, int32_t *bad) {
+    const int lane = threadIdx.x & 31;
+    const int64_t e = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (e >= cnt) return;
+    const int a = u[e], b = v[e];
+    if (a < 0 || a >= n || b < 0 || b >= n || a == b) {
+        if (lane == 0) atomicOr(bad, 1);
+        return;
+    }
+    const int2 ra = row_of(g, a, INT32_MAX), rb = row_of(g, b, INT32_MAX);
+    const bool use_a = (ra.y - ra.x) <= (rb.y - rb.x);
+    const int2 r = use_a ? ra : rb;
+    const int target = use_a ? b : a;
+    bool found = false;
+    for (int j = r.x + lane; j < r.y; j += 32) found |= (ldg_i(g.col + j) == target);
+    if (__any_sync(kFull, found) && lane == 0) atomicOr(bad, 2);
+}
+
+// count directed batch entries per vertex; remember each entry's arrival slot
+__global__ void k_count(const int32_t *u, const int32_t *v, int64_t cnt, int32_t n, int32_t *xcnt,
+                        int32_t *slot) {
+    const int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (e >= cnt) return;
+    const int a = u[e], b = v[e];
+    if (a < 0 || a >= n || b < 0 || b >= n) return;  // rejected by k_validate_edges
+    slot[2 * e] = atomicAdd(xcnt + a, 1);
+    slot[2 * e + 1] = atomicAdd(xcnt + b, 1);
+}
+
+__global__ void k_degrees(const int32_t *rp_old, const int32_t *xcnt, int32_t n, int32_t *deg) {
+    const int64_t x = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (x > n) return;
+    deg[x] = (x == n) ? 0 : ((rp_old[x + 1] & kMask) - (rp_old[x] & kMask) + xcnt[x]);
+}
+
+// ---- exclusive scan of int32 (3 kernels: block scan, scan of block sums, add) ----
+constexpr int kScanBlock = 1024;
+
+__device__ __forceinline__ int block_exclusive_scan(int x, int *warp_sums, int *total) {
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    int incl = x;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(kFull, incl, o);
+        if (lane >= o) incl += y;
+    }
+    if (lane == 31) warp_sums[wid] = incl;
+    __syncthreads();
+    if (wid == 0) {
+        int s = lane < (kScanBlock / 32) ? warp_sums[lane] : 0;
+        int si = s;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(kFull, si, o);
+            if (lane >= o) si += y;
+        }
+        if (lane < kScanBlock / 32) warp_sums[lane] = si - s;
+        if (lane == 31) *total = si;
+    }
+    __syncthreads();
+    return warp_sums[wid] + incl - x;
+}
+
+__global__ void __launch_bounds__(kScanBlock) k_scan_block(const int32_t *in, int32_t *out, int64_t cnt,
+                                                           int32_t *sums) {
+    __shared__ int ws[32];
+    __shared__ int tot;
+    const int64_t i = (int64_t)blockIdx.x * kScanBlock + threadIdx.x;
+    const int x = i < cnt ? in[i] : 0;
+    const int ex = block_exclusive_scan(x, ws, &tot);
+    if (i < cnt) out[i] = ex;
+    if (threadIdx.x == 0) sums[blockIdx.x] = tot;
+}
+
+__global__ void __launch_bounds__(kScanBlock) k_scan_sums(int32_t *sums, int32_t nb) {
+    __shared__ int ws[32];
+    __shared__ int tot;
+    int carry = 0;
+    for (int base = 0; base < nb; base += kScanBlock) {
+        const int i = base + threadIdx.x;
+        const int x = i < nb ? sums[i] : 0;
+        const int ex = block_exclusive_scan(x, ws, &tot);
+        if (i < nb) sums[i] = ex + carry;
+        carry += tot;
+        __syncthreads();
+    }
+}
+
+__global__ void k_scan_add(int32_t *out, int64_t cnt, const int32_t *sums) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < cnt) out[i] += sums[i / kScanBlock];
+}
+
+// scatter batch entries into per-vertex groups (arrival order)
+__global__ void k_group_scatter(const int32_t *u, const int32_t *v, int64_t cnt, int32_t n,
+                                const int32_t *xoff, const int32_t *slot, int32_t *gtag,
+                                int32_t *gnbr) {
+    const int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (e >= cnt) return;
+    const int a = u[e], b = v[e];
+    if (a < 0 || a >= n || b < 0 || b >= n) return;
+    int p = xoff[a] + slot[2 * e];
+    gtag[p] = (int)e;
+    gnbr[p] = b;
+    p = xoff[b] + slot[2 * e + 1];
+    gtag[p] = (int)e;
+    gnbr[p] = a;
+}
+
+// per vertex with batch entries: order its group by insertion index (canonical
+// order), detect duplicate edges within the batch, publish xinfo.
+__global__ void k_group_sort(const int32_t *xcnt, const int32_t *xoff, int32_t n, int32_t *gtag,
+                             int32_t *gnbr, int2 *xinfo, int32_t *bad) {
+    const int64_t x = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (x >= n) return;
+    const int c = xcnt[x];
+    if (c == 0) return;
+    const int b = xoff[x];
+    for (int i = 1; i < c; ++i) {  // insertion sort (groups are tiny)
+        const int t = gtag[b + i], nb = gnbr[b + i];
+        int j = i - 1;
+        while (j >= 0 && gtag[b + j] > t) {
+            gtag[b + j + 1] = gtag[b + j];
+            gnbr[b + j + 1] = gnbr[b + j];
+            --j;
+        }
+        gtag[b + j + 1] = t;
+        gnbr[b + j + 1] = nb;
+    }
+    for (int i = 1; i < c; ++i)
+        for (int j = 0; j < i; ++j)
+            if (gnbr[b + j] == gnbr[b + i]) atomicOr(bad, 4);
+    xinfo[x] = make_int2(b, c);
+}
+
+// warp per vertex: copy the old row to its new place, append the batch group
+__global__ void k_copy_rows(const int32_t *rp_old, const int32_t *col_old, const int32_t *rp_new,
+                            int32_t *col_new, const int32_t *xcnt, const int32_t *xoff,
+                            const int32_t *gnbr, int32_t n) {
+    const int lane = threadIdx.x & 31;
+    const int64_t warps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t x = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; x < n; x += warps) {
+        const int ob = rp_old[x] & kMask, oe = rp_old[x + 1] & kMask, nb = rp_new[x];
+        for (int j = lane; j < oe - ob; j += 32) col_new[nb + j] = col_old[ob + j];
+        const int c = xcnt[x];
+        if (c) {
+            const int g0 = xoff[x], dst = nb + (oe - ob);
+            for (int j = lane; j < c; j += 32) col_new[dst + j] = gnbr[g0 + j];
+        }
+    }
+}
+
+__global__ void k_flag_rows(const int32_t *xcnt, int32_t n, int32_t *rp_new) {
+    const int64_t x = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (x < n && xcnt[x]) rp_new[x] |= (int32_t)0x80000000u;
+}
+
+int64_t scan_sums_capacity(int64_t n) { return (n + 1 + kScanBlock - 1) / kScanBlock + 1; }
+
+static int scan_launch(const int32_t *in, int32_t *out, int64_t cnt, int32_t *sums, cudaStream_t s) {
+    const int nb = (int)blocks_for(cnt, kScanBlock);
+    k_scan_block<<<nb, kScanBlock, 0, s>>>(in, out, cnt, sums);
+    k_scan_sums<<<1, kScanBlock, 0, s>>>(sums, nb);
+    k_scan_add<<<blocks_for(cnt, 256), 256, 0, s>>>(out, cnt, sums);
+    return 3;
+}
+
+int validate_batch(const AppendBufs &B, const GView &g, const int32_t *rp_old, int32_t n,
+                   const int32_t *u, const int32_t *v, int64_t cnt, cudaStream_t s) {
+    int launches = 0;
+    cudaMemsetAsync(B.bad, 0, sizeof(int32_t), s);
+    cudaMemsetAsync(B.xcnt, 0, sizeof(int32_t) * (size_t)n, s);
+    if (cnt) {
+        k_validate_edges<<<blocks_for(cnt * 32, 256), 256, 0, s>>>(g, n, u, v, cnt, B.bad);
+        k_count<<<blocks_for(cnt, 256), 256, 0, s>>>(u, v, cnt, n, B.xcnt, B.slot);
+        launches += 2;
+    }
+    // xoff = exclusive scan of xcnt (group offsets)
+    launches += scan_launch(B.xcnt, B.xoff, n, B.sums, s);
+    if (cnt) {
+        k_group_scatter<<<blocks_for(cnt, 256), 256, 0, s>>>(u, v, cnt, n, B.xoff, B.slot, B.xtag,
+                                                            B.gnbr);
+        k_group_sort<<<blocks_for(n, 256), 256, 0, s>>>(B.xcnt, B.xoff, n, B.xtag, B.gnbr, B.xinfo,
+                                                       B.bad);
+        launches += 2;
+    }
+    (void)rp_old;
+    return launches;
+}
+
+int append_batch(const AppendBufs &B, const int32_t *rp_old, const int32_t *col_old, int32_t *rp_new,
+                 int32_t *col_new, int32_t n, cudaStream_t s) {
+    int launches = 0;
+    k_degrees<<<blocks_for((int64_t)n + 1, 256), 256, 0, s>>>(rp_old, B.xcnt, n, B.deg);
+    launches += 1 + scan_launch(B.deg, rp_new, (int64_t)n + 1, B.sums, s);
+    k_copy_rows<<<std::min<int64_t>(blocks_for((int64_t)n * 32, 256), 148 * 16), 256, 0, s>>>(
+        rp_old, col_old, rp_new, col_new, B.xcnt, B.xoff, B.gnbr, n);
+    k_flag_rows<<<blocks_for(n, 256), 256, 0, s>>>(B.xcnt, n, rp_new);
+    return launches + 2;
+}
+
+// BC partial rebased as the column sum of delta over local slots (DBC_FLAG_EXACT_BC)
+__global__ void k_exact_bc(const double2 *sd, const int32_t *roots, int32_t k_loc, int32_t n,
+                           double *bc) {
+    const int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (v >= n) return;
+    double acc = 0.0;
+    for (int li = 0; li < k_loc; ++li)
+        if (roots[li] != v) acc += sd[(size_t)li * n + v].y;
+    bc[v] = acc;
+}
+
+int exact_bc(const double2 *sd, const int32_t *roots, int32_t k_loc, int32_t n, double *bc,
+             cudaStream_t s) {
+    k_exact_bc<<<blocks_for(n, 256), 256, 0, s>>>(sd, roots, k_loc, n, bc);
+    return 1;
+}
+
+}  // namespace dbc

@@ -1,0 +1,34 @@
+// graph_ops.h -- host-side entry points of graph.cu (batch validation, append,
+// exact-BC rebase).  Internal to libdbc.  Each returns the number of kernels it
+// launched (errors are picked up by the caller with cudaGetLastError).
+#pragma once
+
+#include <cstdint>
+
+#include <cuda_runtime.h>
+
+namespace dbc {
+
+struct GView;
+
+struct AppendBufs {
+    int32_t *slot;   // [2*cap] arrival slot of each directed batch entry in its group
+    int32_t *xtag;   // [2*cap] grouped entries: batch-local insertion index
+    int32_t *gnbr;   // [2*cap] grouped entries: neighbour
+    int2 *xinfo;     // [n] per flagged vertex {first grouped index, count}
+    int32_t *xcnt;   // [n] batch entries per vertex
+    int32_t *xoff;   // [n] group offsets (exclusive scan of xcnt)
+    int32_t *deg;    // [n+1]
+    int32_t *sums;   // scan block sums
+    int32_t *bad;    // [1] validation result bits
+};
+
+int64_t scan_sums_capacity(int64_t n);
+int validate_batch(const AppendBufs &B, const GView &g, const int32_t *rp_old, int32_t n,
+                   const int32_t *u, const int32_t *v, int64_t cnt, cudaStream_t s);
+int append_batch(const AppendBufs &B, const int32_t *rp_old, const int32_t *col_old, int32_t *rp_new,
+                 int32_t *col_new, int32_t n, cudaStream_t s);
+int exact_bc(const double2 *sd, const int32_t *roots, int32_t k_loc, int32_t n, double *bc,
+             cudaStream_t s);
+
+}  // namespace dbc

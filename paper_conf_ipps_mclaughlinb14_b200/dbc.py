@@ -1,0 +1,285 @@
+"""Thin ctypes binding of libdbc.so (include/dbc.h) -- argument marshalling only.
+
+Every step of the method runs in the library's CUDA kernels; this module never
+computes BC, d, sigma or delta itself and has no CPU fallback: if the compiled
+library is missing it raises.  PyTorch supplies the CUDA stream (and, for
+multi-GPU, the process group); numpy arrays are host buffers, torch CUDA
+tensors are device buffers.
+"""
+
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libdbc.so")
+
+DBC_INF = 2**31 - 1
+FLAG_MODE_S = 0x1
+FLAG_TIMING = 0x2
+FLAG_EXACT_BC = 0x4
+
+STATUS = {
+    0: "DBC_OK", -1: "DBC_EINVAL", -2: "DBC_ENOMEM", -3: "DBC_ECUDA", -4: "DBC_ENCCL",
+    -5: "DBC_ESTATE", -6: "DBC_EEDGE", -7: "DBC_ECAPACITY", -8: "DBC_ENUMERIC",
+}
+
+
+class DBCError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+        self.name = STATUS.get(status, str(status))
+
+
+class Options(ctypes.Structure):
+    _fields_ = [
+        ("device", ctypes.c_int32), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
+        ("workers", ctypes.c_int32), ("edge_capacity", ctypes.c_int64),
+        ("stream", ctypes.c_void_p), ("flags", ctypes.c_uint32),
+        ("reserved", ctypes.c_uint32 * 7),
+    ]
+
+
+class InsertStats(ctypes.Structure):
+    _fields_ = [
+        ("insertions", ctypes.c_int64), ("case_count", ctypes.c_int64 * 3),
+        ("touched", ctypes.c_int64), ("down_vertices", ctypes.c_int64),
+        ("edges_scanned", ctypes.c_int64), ("alg_bytes", ctypes.c_int64),
+    ]
+
+    def as_dict(self):
+        return dict(insertions=self.insertions, case1=self.case_count[0],
+                    case2=self.case_count[1], case3=self.case_count[2], touched=self.touched,
+                    down_vertices=self.down_vertices, edges_scanned=self.edges_scanned,
+                    alg_bytes=self.alg_bytes)
+
+
+class Timings(ctypes.Structure):
+    _fields_ = [
+        ("append_ms", ctypes.c_float), ("update_ms", ctypes.c_float),
+        ("static_ms", ctypes.c_float), ("update_launches", ctypes.c_int32),
+        ("kernel_launches", ctypes.c_int32), ("static_alg_bytes", ctypes.c_int64),
+        ("append_ms_total", ctypes.c_double), ("update_ms_total", ctypes.c_double),
+        ("update_launches_total", ctypes.c_int64), ("kernel_launches_total", ctypes.c_int64),
+        ("insertions_total", ctypes.c_int64), ("alg_bytes_total", ctypes.c_int64),
+    ]
+
+    def as_dict(self):
+        return {name: getattr(self, name) for name, _ in self._fields_}
+
+
+# every symbol include/dbc.h declares, with its signature
+_P = ctypes.c_void_p
+SIGNATURES = {
+    "dbc_options_default": (None, [_P]),
+    "dbc_create": (ctypes.c_int, [_P, ctypes.c_int32, _P, _P, _P, ctypes.c_int32, _P]),
+    "dbc_static_compute": (ctypes.c_int, [_P]),
+    "dbc_insert_edges": (ctypes.c_int, [_P, _P, _P, ctypes.c_int64, _P]),
+    "dbc_insert_edges_device": (ctypes.c_int, [_P, _P, _P, ctypes.c_int64, _P]),
+    "dbc_get_bc": (ctypes.c_int, [_P, _P]),
+    "dbc_get_bc_partial_device": (ctypes.c_int, [_P, _P]),
+    "dbc_get_root_state": (ctypes.c_int, [_P, ctypes.c_int32, _P, _P, _P]),
+    "dbc_num_local_roots": (ctypes.c_int, [_P, _P]),
+    "dbc_synchronize": (ctypes.c_int, [_P]),
+    "dbc_get_timings": (ctypes.c_int, [_P, _P]),
+    "dbc_reset_timings": (ctypes.c_int, [_P]),
+    "dbc_device_bytes": (ctypes.c_int, [_P, _P]),
+    "dbc_strerror": (ctypes.c_char_p, [ctypes.c_int]),
+    "dbc_last_error": (ctypes.c_char_p, [_P]),
+    "dbc_abi_version": (ctypes.c_int32, []),
+    "dbc_destroy": (None, [_P]),
+}
+
+_lib = None
+
+
+def load_library():
+    """Load libdbc.so (raises if it was not built -- there is no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} not built: run `python -c 'import __graft_entry__ as g; g.build()'`")
+        lib = ctypes.CDLL(LIB_PATH)
+        for name, (res, args) in SIGNATURES.items():
+            f = getattr(lib, name)
+            f.restype = res
+            f.argtypes = args
+        _lib = lib
+    return _lib
+
+
+def _check(ctx, rc):
+    if rc != 0:
+        lib = load_library()
+        msg = lib.dbc_last_error(ctx)
+        raise DBCError(rc, msg.decode() if msg else "")
+
+
+def _host(a, dtype):
+    return np.ascontiguousarray(a, dtype=dtype)
+
+
+def _np_ptr(a):
+    return a.ctypes.data_as(ctypes.c_void_p)
+
+
+class DynamicBC:
+    """Dynamic betweenness centrality over a root set on one GPU (one rank).
+
+    >>> bc = DynamicBC(n, row_ptr, col, roots)     # dbc_create
+    >>> bc.static_compute()                        # Brandes (Alg. 1)
+    >>> bc.insert_edges(u, v)                      # sequential insertions, one batch
+    >>> bc.get_bc()                                # Eq. (3)
+    """
+
+    def __init__(self, n, row_ptr, col, roots, *, device=0, rank=0, world=1, workers=0,
+                 edge_capacity=0, stream=None, flags=0):
+        lib = load_library()
+        self._lib = lib
+        self._ctx = None
+        self.n = int(n)
+        self.k = int(np.asarray(roots).size)
+        self.rank, self.world, self.device = int(rank), int(world), int(device)
+        rp = _host(row_ptr, np.int64)
+        cl = _host(col, np.int32)
+        rt = _host(roots, np.int32)
+        opt = Options()
+        lib.dbc_options_default(ctypes.byref(opt))
+        opt.device, opt.rank, opt.world = self.device, self.rank, self.world
+        opt.workers, opt.edge_capacity, opt.flags = int(workers), int(edge_capacity), int(flags)
+        if stream is None:
+            try:
+                import torch
+
+                if torch.cuda.is_available():
+                    with torch.cuda.device(self.device):
+                        stream = torch.cuda.current_stream().cuda_stream
+            except Exception:  # pragma: no cover
+                stream = None
+        opt.stream = stream
+        out = ctypes.c_void_p()
+        rc = lib.dbc_create(ctypes.byref(out), self.n, _np_ptr(rp), _np_ptr(cl), _np_ptr(rt),
+                            self.k, ctypes.byref(opt))
+        _check(None, rc)
+        self._ctx = out
+
+    # -- lifecycle -----------------------------------------------------------
+    def close(self):
+        if self._ctx:
+            self._lib.dbc_destroy(self._ctx)
+            self._ctx = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    # -- calls -----------------------------------------------------------------
+    def static_compute(self):
+        _check(self._ctx, self._lib.dbc_static_compute(self._ctx))
+
+    def insert_edges(self, u, v, stats=False):
+        """Host arrays -> dbc_insert_edges; CUDA tensors -> dbc_insert_edges_device."""
+        st = InsertStats() if stats else None
+        stp = ctypes.byref(st) if st is not None else None
+        if hasattr(u, "is_cuda") and u.is_cuda:
+            import torch
+
+            assert u.dtype == torch.int32 and v.dtype == torch.int32 and u.numel() == v.numel()
+            assert u.is_contiguous() and v.is_contiguous()
+            rc = self._lib.dbc_insert_edges_device(self._ctx, ctypes.c_void_p(u.data_ptr()),
+                                                   ctypes.c_void_p(v.data_ptr()), u.numel(), stp)
+        else:
+            uu, vv = _host(u, np.int32).ravel(), _host(v, np.int32).ravel()
+            if uu.size != vv.size:
+                raise ValueError("u and v differ in length")
+            rc = self._lib.dbc_insert_edges(self._ctx, _np_ptr(uu), _np_ptr(vv), uu.size, stp)
+        _check(self._ctx, rc)
+        return st.as_dict() if st is not None else None
+
+    def get_bc(self, out=None):
+        out = np.empty(self.n, dtype=np.float64) if out is None else out
+        _check(self._ctx, self._lib.dbc_get_bc(self._ctx, _np_ptr(out)))
+        return out
+
+    def bc_partial_device_ptr(self) -> int:
+        p = ctypes.c_void_p()
+        _check(self._ctx, self._lib.dbc_get_bc_partial_device(self._ctx, ctypes.byref(p)))
+        return int(p.value)
+
+    def get_root_state(self, slot):
+        d = np.empty(self.n, dtype=np.int32)
+        s = np.empty(self.n, dtype=np.float64)
+        dl = np.empty(self.n, dtype=np.float64)
+        _check(self._ctx, self._lib.dbc_get_root_state(self._ctx, int(slot), _np_ptr(d), _np_ptr(s),
+                                                       _np_ptr(dl)))
+        return d, s, dl
+
+    def num_local_roots(self):
+        k = ctypes.c_int32()
+        _check(self._ctx, self._lib.dbc_num_local_roots(self._ctx, ctypes.byref(k)))
+        return k.value
+
+    def local_slots(self):
+        return list(range(self.rank, self.k, self.world))
+
+    def synchronize(self):
+        _check(self._ctx, self._lib.dbc_synchronize(self._ctx))
+
+    def timings(self):
+        t = Timings()
+        _check(self._ctx, self._lib.dbc_get_timings(self._ctx, ctypes.byref(t)))
+        return t.as_dict()
+
+    def reset_timings(self):
+        _check(self._ctx, self._lib.dbc_reset_timings(self._ctx))
+
+    def device_bytes(self):
+        b = ctypes.c_int64()
+        _check(self._ctx, self._lib.dbc_device_bytes(self._ctx, ctypes.byref(b)))
+        return b.value
+
+
+def local_slots(k: int, rank: int, world: int):
+    """Root slots owned by `rank` (slot % world == rank), SURVEY.md Sec. 8(e)."""
+    return list(range(rank, k, world))
+
+
+def allreduce_bc(dbc: DynamicBC, group=None):
+    """Sum the per-rank BC partials in place over torch.distributed (NCCL on GPUs)
+    and return the global BC on the host.  The only cross-GPU exchange (A5)."""
+    import torch
+    import torch.distributed as dist
+
+    if dbc.world == 1 or not dist.is_initialized():
+        return dbc.get_bc()
+    ptr = dbc.bc_partial_device_ptr()
+    dbc.synchronize()
+    # reduce a copy: the library keeps accumulating this rank's partial
+    t = _wrap_device_f64(ptr, dbc.n, dbc.device).clone()
+    dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+    return t.cpu().numpy()
+
+
+def _wrap_device_f64(ptr: int, n: int, device: int):
+    """Zero-copy torch view of a device fp64 buffer owned by libdbc."""
+    import torch
+
+    class _CAI:
+        __cuda_array_interface__ = {
+            "shape": (n,), "typestr": "<f8", "data": (ptr, False), "version": 3, "strides": None,
+        }
+
+    with torch.cuda.device(device):
+        return torch.as_tensor(_CAI(), device=f"cuda:{device}")

@@ -1,0 +1,293 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the CPU oracle.
+
+Bar (BASELINE.json north_star): d and sigma bit-exact,
+BC within |bc - ref| <= 1e-9 * max(|ref|, 1), delta within 1e-10 * max(|ref|, 1)
+(delta is a diagnostic; derivation in DESIGN.md).
+"""
+
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+import oracle
+import workloads as W
+
+pytestmark = pytest.mark.gpu
+
+BC_TOL = 1e-9
+DELTA_TOL = 1e-10
+
+
+def _dbc(g, roots, **kw):
+    from paper_conf_ipps_mclaughlinb14_b200 import DynamicBC
+
+    return DynamicBC(g.n, g.row_ptr, g.col, roots, **kw)
+
+
+def assert_bc(bc, ref, tol=BC_TOL):
+    err = np.abs(bc - ref) / np.maximum(np.abs(ref), 1.0)
+    assert err.max(initial=0.0) <= tol, f"BC rel err {err.max()} at {int(err.argmax())}"
+
+
+def assert_state(dbc, d_ref, s_ref, dl_ref, slots):
+    for slot in slots:
+        d, s, dl = dbc.get_root_state(slot)
+        assert np.array_equal(d, d_ref[slot]), f"d mismatch at slot {slot}"
+        bad = np.nonzero(s != s_ref[slot])[0]
+        assert bad.size == 0, f"sigma mismatch slot {slot} at {bad[:5]}: {s[bad[:5]]} vs {s_ref[slot][bad[:5]]}"
+        err = np.abs(dl - dl_ref[slot]) / np.maximum(np.abs(dl_ref[slot]), 1.0)
+        assert err.max(initial=0.0) <= DELTA_TOL, f"delta rel err {err.max()} slot {slot}"
+
+
+def check_all(dbc, ref_out, k):
+    bc_ref, d_ref, s_ref, dl_ref = ref_out
+    assert_bc(dbc.get_bc(), bc_ref)
+    assert_state(dbc, d_ref, s_ref, dl_ref, range(k))
+
+
+# ---------------------------------------------------------------- static ----
+STATIC_CASES = {
+    "karate": lambda: (W.karate(), np.arange(34)),
+    "path9": lambda: (W.path_graph(9), np.arange(9)),
+    "star12": lambda: (W.star_graph(12), np.arange(12)),
+    "complete8": lambda: (W.complete_graph(8), np.arange(8)),
+    "grid_big_sigma": lambda: (W.grid_graph(45, 45), np.array([0, 44, 1012, 2024])),
+    "disconnected": lambda: (W.random_gnm(300, 280, 5), np.arange(0, 300, 7)),
+    "isolated_root": lambda: (W.csr_from_edges(6, [0, 1], [1, 2]), np.array([5, 0, 3])),
+    "rmat10": lambda: (W.make_workload("rmat10").graph, W.make_workload("rmat10").roots),
+    "delaunay12": lambda: (W.make_workload("delaunay12").graph, W.make_workload("delaunay12").roots),
+    "hub": lambda: (W.star_graph(3000), np.array([0, 1, 2, 2999])),
+}
+
+
+@pytest.mark.parametrize("name", sorted(STATIC_CASES))
+def test_static_matches_oracle(name):
+    g, roots = STATIC_CASES[name]()
+    roots = np.asarray(roots, np.int32)
+    ref = oracle.brandes_csr(g, roots)
+    with _dbc(g, roots) as dbc:
+        dbc.static_compute()
+        check_all(dbc, ref, roots.size)
+
+
+def test_static_no_edges_and_zero_roots():
+    g = W.csr_from_edges(5, [], [])
+    with _dbc(g, np.array([0, 3], np.int32)) as dbc:
+        dbc.static_compute()
+        assert np.all(dbc.get_bc() == 0)
+        d, s, dl = dbc.get_root_state(1)
+        assert d[3] == 0 and s[3] == 1 and np.all(d[[0, 1, 2, 4]] == oracle.INF)
+    with _dbc(W.path_graph(4), np.array([], np.int32)) as dbc:
+        dbc.static_compute()
+        assert np.all(dbc.get_bc() == 0)
+
+
+# --------------------------------------------------------------- dynamic ----
+def run_stream_single(g, roots, us, vs, check_every=1, flags=0, workers=0):
+    """Insert one edge per call; compare with the naive dynamic oracle."""
+    roots = np.asarray(roots, np.int32)
+    ref = oracle.NaiveDynamicBC(g, roots)
+    with _dbc(g, roots, flags=flags, workers=workers) as dbc:
+        dbc.static_compute()
+        for i, (u, v) in enumerate(zip(us, vs)):
+            dbc.insert_edges([u], [v])
+            ref.insert(u, v)
+            if (i + 1) % check_every == 0 or i + 1 == len(us):
+                check_all(dbc, ref.compute(), roots.size)
+
+
+@pytest.mark.parametrize("n", [5, 6, 9, 10])
+def test_path_to_cycle(n):
+    run_stream_single(W.path_graph(n), np.arange(n), [0], [n - 1])
+
+
+def test_star_to_complete():
+    n = 7
+    pairs = [(a, b) for a in range(1, n) for b in range(a + 1, n)]
+    run_stream_single(W.star_graph(n), np.arange(n), [p[0] for p in pairs], [p[1] for p in pairs])
+
+
+def test_karate_config1_every_insertion():
+    wl = W.make_workload("karate")
+    run_stream_single(wl.graph, wl.roots, wl.ins_u, wl.ins_v)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_random_multicomponent(seed):
+    """Components merge: Case 3 with an unreachable endpoint pulls whole components up."""
+    rng = np.random.default_rng(seed)
+    n = 80
+    g = W.random_gnm(n, 70, 40 + seed)
+    u, v = W.uniform_non_edges(g, 30, seed)
+    roots = rng.choice(n, size=20, replace=False)
+    run_stream_single(g, roots, u, v)
+
+
+@pytest.mark.parametrize("name", ["rmat10", "delaunay12", "delaunay12u"])
+def test_config_shapes_single(name):
+    wl = W.make_workload(name)
+    run_stream_single(wl.graph, wl.roots, wl.ins_u, wl.ins_v, check_every=5)
+
+
+def test_grid_sigma_above_2p53_dynamic():
+    """sigma > 2^53 (Delaunay-like meshes reach 2^100): pull sums in canonical order stay bit-exact."""
+    g = W.grid_graph(60, 60)
+    roots = np.array([0, 59, 3599, 1830], np.int32)
+    rng = np.random.default_rng(3)
+    eu, ev = W.edges_of(g)
+    # diagonal shortcuts inside the mesh (Case 2/3 mixes)
+    cand = [(i * 60 + j, (i + 1) * 60 + j + 1) for i in range(0, 59, 7) for j in range(0, 59, 11)]
+    pick = [cand[i] for i in rng.permutation(len(cand))[:12]]
+    run_stream_single(g, roots, [p[0] for p in pick], [p[1] for p in pick], check_every=3)
+
+
+@pytest.mark.parametrize("flags", [0, 1])  # Mode A (batch kernel), Mode S (per insertion)
+@pytest.mark.parametrize("name", ["karate", "rmat10", "delaunay12u"])
+def test_batch_modes_match_oracle(name, flags):
+    wl = W.make_workload(name)
+    ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
+    with _dbc(wl.graph, wl.roots, flags=flags) as dbc:
+        dbc.static_compute()
+        half = wl.ins_u.size // 2
+        for sl in (slice(0, half), slice(half, None)):
+            st = dbc.insert_edges(wl.ins_u[sl], wl.ins_v[sl], stats=True)
+            for u, v in zip(wl.ins_u[sl], wl.ins_v[sl]):
+                ref.insert(u, v)
+            assert st["case1"] + st["case2"] + st["case3"] == wl.roots.size * wl.ins_u[sl].size
+            check_all(dbc, ref.compute(), wl.roots.size)
+
+
+def test_mode_a_equals_mode_s_and_static_bitwise():
+    wl = W.make_workload("delaunay12")
+    outs = []
+    for flags in (0, 1):
+        with _dbc(wl.graph, wl.roots, flags=flags, workers=7) as dbc:
+            dbc.static_compute()
+            dbc.insert_edges(wl.ins_u, wl.ins_v)
+            outs.append([dbc.get_root_state(s)[:2] for s in range(wl.roots.size)])
+            dbc.static_compute()  # GPU recompute on the final graph
+            outs.append([dbc.get_root_state(s)[:2] for s in range(wl.roots.size)])
+    for o in outs[1:]:
+        for (d0, s0), (d1, s1) in zip(outs[0], o):
+            assert np.array_equal(d0, d1) and np.array_equal(s0, s1)
+
+
+def test_exact_bc_flag():
+    from paper_conf_ipps_mclaughlinb14_b200 import FLAG_EXACT_BC
+
+    wl = W.make_workload("rmat10")
+    ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
+    with _dbc(wl.graph, wl.roots, flags=FLAG_EXACT_BC) as dbc:
+        dbc.static_compute()
+        dbc.insert_edges(wl.ins_u, wl.ins_v)
+        for u, v in zip(wl.ins_u, wl.ins_v):
+            ref.insert(u, v)
+        bc_ref = ref.compute()[0]
+        assert_bc(dbc.get_bc(), bc_ref, tol=1e-12)
+
+
+def test_device_batch_api():
+    import torch
+
+    wl = W.make_workload("rmat10")
+    ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
+    with _dbc(wl.graph, wl.roots) as dbc:
+        dbc.static_compute()
+        u = torch.from_numpy(wl.ins_u).cuda()
+        v = torch.from_numpy(wl.ins_v).cuda()
+        dbc.insert_edges(u, v)
+        for a, b in zip(wl.ins_u, wl.ins_v):
+            ref.insert(a, b)
+        check_all(dbc, ref.compute(), wl.roots.size)
+
+
+def test_fake_multi_gpu_shards_sum_to_single():
+    """Two rank contexts (world=2) on one device: partials sum to the 1-rank BC."""
+    wl = W.make_workload("rmat10")
+    outs = []
+    for world in (1, 2):
+        parts = []
+        for rank in range(world):
+            with _dbc(wl.graph, wl.roots, rank=rank, world=world) as dbc:
+                dbc.static_compute()
+                dbc.insert_edges(wl.ins_u, wl.ins_v)
+                parts.append(dbc.get_bc())
+                assert dbc.num_local_roots() == len(range(rank, wl.roots.size, world))
+        outs.append(np.sum(parts, axis=0))
+    assert_bc(outs[1], outs[0], tol=1e-12)
+
+
+# ----------------------------------------------------------- error paths ----
+def test_error_paths_leave_state_unchanged():
+    from paper_conf_ipps_mclaughlinb14_b200 import DBCError
+
+    g = W.karate()
+    roots = np.arange(34, dtype=np.int32)
+    with _dbc(g, roots, edge_capacity=4) as dbc:
+        with pytest.raises(DBCError) as e:
+            dbc.insert_edges([0], [9])
+        assert e.value.name == "DBC_ESTATE"
+        dbc.static_compute()
+        bc0 = dbc.get_bc().copy()
+        st0 = dbc.get_root_state(5)
+        bad = {
+            "self loop": ([3], [3]),
+            "range": ([0], [34]),
+            "negative": ([-1], [2]),
+            "present": ([0], [1]),
+            "present reversed": ([1], [0]),
+            "dup in batch": ([0, 9], [9, 0]),
+            "bad later in batch": ([0, 4], [9, 4]),
+        }
+        for name, (u, v) in bad.items():
+            with pytest.raises(DBCError) as e:
+                dbc.insert_edges(u, v)
+            assert e.value.name == "DBC_EEDGE", name
+        with pytest.raises(DBCError) as e:
+            dbc.insert_edges([0, 0, 0, 0, 0], [9, 14, 15, 16, 18])
+        assert e.value.name == "DBC_ECAPACITY"
+        assert np.array_equal(dbc.get_bc(), bc0)
+        for a, b in zip(dbc.get_root_state(5), st0):
+            assert np.array_equal(a, b)
+        with pytest.raises(DBCError) as e:
+            dbc.get_root_state(34)
+        assert e.value.name == "DBC_EINVAL"
+        dbc.insert_edges([], [])  # empty batch is fine
+        dbc.insert_edges([0, 9], [9, 14])
+        dbc.insert_edges([0, 9], [15, 16])
+        with pytest.raises(DBCError) as e:
+            dbc.insert_edges([0], [18])
+        assert e.value.name == "DBC_ECAPACITY"
+
+
+# ------------------------------------------------- full size (configs[1]) ----
+def test_rmat16_full_size_batch_parity():
+    """BASELINE configs[1] at full size, in the launch configuration bench.py times
+    (Mode A, one batch): BC over all 256 roots vs the oracle recompute, d/sigma/delta
+    on sampled roots, and GPU dynamic == GPU static (bitwise d/sigma) on the final graph."""
+    wl = W.make_workload("rmat16")
+    g = wl.graph
+    with _dbc(g, wl.roots) as dbc:
+        dbc.static_compute()
+        st = dbc.insert_edges(wl.ins_u, wl.ins_v, stats=True)
+        assert st["case1"] + st["case2"] + st["case3"] == 256 * 1000
+        bc = dbc.get_bc()
+        ref = oracle.NaiveDynamicBC(g, wl.roots)
+        for u, v in zip(wl.ins_u, wl.ins_v):
+            ref.insert(u, v)
+        rp, col = ref.csr()
+        sample = np.array([0, 17, 101, 255], np.int32)
+        bc_ref, d_ref, s_ref, dl_ref = oracle.brandes(g.n, rp, col, wl.roots[sample])
+        for i, slot in enumerate(sample):
+            d, s, dl = dbc.get_root_state(int(slot))
+            assert np.array_equal(d, d_ref[i]) and np.array_equal(s, s_ref[i])
+            err = np.abs(dl - dl_ref[i]) / np.maximum(np.abs(dl_ref[i]), 1.0)
+            assert err.max() <= DELTA_TOL
+        full_bc_ref = oracle.brandes(g.n, rp, col, wl.roots, want_state=False)[0]
+        assert_bc(bc, full_bc_ref)
+        dyn = [dbc.get_root_state(s)[:2] for s in range(0, 256, 15)]
+        dbc.static_compute()
+        for (d0, s0), s in zip(dyn, range(0, 256, 15)):
+            d1, s1, _ = dbc.get_root_state(s)
+            assert np.array_equal(d0, d1) and np.array_equal(s0, s1)
