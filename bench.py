@@ -238,7 +238,8 @@ def run_ours(args):
     wl = W.make_workload(args.config, seed=args.seed, insertions=B * nb, k=k)
     g = wl.graph
     flags = FLAG_TIMING | (FLAG_MODE_S if args.mode == "S" else 0)
-    stream = torch.cuda.current_stream()
+    stream = torch.cuda.Stream(device=dev)  # the library and the timing events share it
+    torch.cuda.set_stream(stream)
     dbc = DynamicBC(g.n, g.row_ptr, g.col, wl.roots, device=dev, rank=rank, world=world,
                     workers=args.workers, edge_capacity=B * nb, flags=flags,
                     stream=stream.cuda_stream)

@@ -86,7 +86,8 @@ typedef struct {
     int32_t workers;       /* persistent worker CTAs; 0 = automatic                */
     int64_t edge_capacity; /* max undirected edges inserted over the context's
                               lifetime; 0 = automatic (max(2^16, m/4))            */
-    void *stream;          /* cudaStream_t to run on; NULL = library-owned stream  */
+    void *stream;          /* cudaStream_t to run on; NULL = library-owned stream;
+                              cudaStreamLegacy ((void*)1) = the legacy default stream */
     uint32_t flags;        /* DBC_FLAG_*                                           */
     uint32_t reserved[7];  /* must be zero                                         */
 } dbc_options;

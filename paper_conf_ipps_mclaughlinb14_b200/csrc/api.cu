@@ -293,7 +293,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     c->ev_ok = true;
 
     // workers: persistent CTAs; bounded by roots and by a scratch-memory budget
-    const size_t per_worker = (size_t)n * (4 + 8 + 8 + 4 + 4 + 8 + 4 + 4 + 4 + 4) + (size_t)(n + 2) * 4 + 64;
+    const size_t per_worker = (size_t)n * (4 + 8 + 8 + 4 + 4 + 8 + 4 + 4 + 4 + 4 + 4) + (size_t)(n + 2) * 4 + 64;
     size_t free_b = 0, total_b = 0;
     cudaMemGetInfo(&free_b, &total_b);
     const size_t state_b = (size_t)c->k_loc * n * 20 + (size_t)c->col_cap * 8 + (size_t)n * 40;
@@ -343,6 +343,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->ws.U1, wn);
     AL(c->ws.Rv, wn);
     AL(c->ws.Rl, wn);
+    AL(c->ws.Bq, wn);
     AL(c->ws.wepoch, (size_t)c->workers);
     AL(c->next_slot, 1);
     AL(c->stats, (size_t)kStCount);

@@ -57,6 +57,7 @@ struct Scratch {
     int32_t *Doff;             // level offsets of D (also static level offsets), n+2
     int32_t *U0, *U1;          // up frontier ping-pong
     int32_t *Rv, *Rl;          // removal-push targets and their levels (Case 3)
+    int32_t *Bq;               // big-row queue of the current level (2 ends)
     uint32_t *wepoch;          // per-worker epoch counter
 };
 
@@ -102,38 +103,146 @@ __device__ __forceinline__ void group_sync() {
 using G1 = std::integral_constant<int, 1>;
 using G32 = std::integral_constant<int, 32>;
 
-// Two-tier node-parallel mapping of a vertex list onto a CTA (the paper's
-// node-based parallelism, Sec. III, re-mapped for 32-wide warps):
-// each warp takes 32 consecutive items, one per lane; rows of <= kSmallDeg
-// entries are walked sequentially by their lane (canonical order for free),
-// longer rows are walked by the whole warp, one row at a time.
-//   get(idx, &v) -> bool   : item idx is active, vertex v
-//   need_row(idx, v) -> bool: whether the body needs the adjacency row
-//   body(G, idx, v, row, gl): gl = lane within the group (0 for G1)
-template <class Get, class NeedRow, class Body>
-__device__ __forceinline__ void two_tier(int count, const GView &g, int limit, Get get,
-                                         NeedRow need_row, Body body) {
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    for (int base = warp * 32; base < count; base += kWarps * 32) {
-        const int idx = base + lane;
+// ---------------------------------------------------------------------------
+// Level processing (the paper's node-based parallelism, Sec. III, P:272-274,
+// re-mapped for B200): the vertices of one BFS level are split by row length.
+//  * small rows (<= kSmallDeg entries): one lane walks the whole row in
+//    canonical order (bit-exact pull sums for free, 32 independent rows per
+//    warp in flight);
+//  * big rows (hubs): queued, then processed in rounds of <= kBig rows whose
+//    entries are flattened across the whole CTA (every thread takes entries
+//    e = tid, tid + kBlock, ..., kUnroll of them per step with the column and
+//    distance gathers hoisted), per-row reductions going through warp-
+//    aggregated shared-memory fp64 atomics.  This is the load-balanced
+//    "advance" Merrill et al. [19] (cited at P:322) describe, restricted to the
+//    rows that need it.
+
+constexpr int kBig = 128;     // big rows per round
+constexpr int kUnroll = 4;    // entries per thread in flight
+
+struct BigSmem {
+    int idx[kBig];    // item index (caller's list) of each big row
+    int v[kBig];      // vertex
+    int b[kBig];      // row begin
+    int off[kBig + 1];  // exclusive scan of row lengths; off[m] = total
+    double acc[kBig];   // per-row reduction
+    double c0[kBig], c1[kBig];  // per-row constants of the caller
+    int m;            // rows in this round
+};
+
+// Pass over `count` items: small rows processed inline by their lane; big rows
+// handed (as item indices) to enqueue().
+//   get(idx, &v) -> bool : item idx is active, vertex v
+//   need_row(idx, v)     : whether the row is needed at all
+//   small(idx, v, row)   : process one small row sequentially
+template <class Get, class NeedRow, class Small, class Enq>
+__device__ __forceinline__ void split_pass(int count, const GView &g, int limit, Get get,
+                                           NeedRow need_row, Small small, Enq enqueue) {
+    for (int idx = threadIdx.x; idx < count; idx += kBlock) {
         int v = 0;
-        bool valid = idx < count && get(idx, v);
+        if (!get(idx, v)) continue;
         int2 r = make_int2(0, 0);
-        if (valid && need_row(idx, v)) r = row_of(g, v, limit);
-        const bool big = valid && (r.y - r.x) > kSmallDeg;
-        if (valid && !big) body(G1{}, idx, v, r, 0);
-        unsigned bm = __ballot_sync(kFull, big);
-        while (bm) {
-            const int src = __ffs(bm) - 1;
-            bm &= bm - 1;
-            const int bidx = __shfl_sync(kFull, idx, src);
-            const int bv = __shfl_sync(kFull, v, src);
-            int2 br;
-            br.x = __shfl_sync(kFull, r.x, src);
-            br.y = __shfl_sync(kFull, r.y, src);
-            body(G32{}, bidx, bv, br, lane);
+        if (need_row(idx, v)) r = row_of(g, v, limit);
+        if (r.y - r.x > kSmallDeg) {
+            enqueue(idx);
+        } else {
+            small(idx, v, r);
         }
     }
+}
+
+// Load a round of m <= kBig queued big rows into shared memory (rows, offsets).
+// fetch(t) -> item index of the t-th row of the round; getv(idx) -> vertex.
+// Caller must __syncthreads() before (queue complete) -- this ends with a barrier.
+template <class Fetch, class GetV>
+__device__ __forceinline__ void big_load(BigSmem &S, int m, Fetch fetch, GetV getv,
+                                         const GView &g, int limit) {
+    const int tid = threadIdx.x;
+    if (tid < m) {
+        const int idx = fetch(tid);
+        const int v = getv(idx);
+        const int2 r = row_of(g, v, limit);
+        S.idx[tid] = idx;
+        S.v[tid] = v;
+        S.b[tid] = r.x;
+        S.off[tid + 1] = r.y - r.x;
+        S.acc[tid] = 0.0;
+    }
+    if (tid == 0) {
+        S.off[0] = 0;
+        S.m = m;
+    }
+    __syncthreads();
+    if (tid < 32) {  // inclusive scan of off[1..m] by warp 0 (m <= kBig = 4*32)
+        int vals[kBig / 32];
+        int run = 0;
+#pragma unroll
+        for (int q = 0; q < kBig / 32; ++q) {
+            const int i = tid * (kBig / 32) + q;
+            vals[q] = (i < m) ? S.off[i + 1] : 0;
+            run += vals[q];
+        }
+        int incl = run;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(kFull, incl, o);
+            if (tid >= o) incl += y;
+        }
+        int ex = incl - run;
+#pragma unroll
+        for (int q = 0; q < kBig / 32; ++q) {
+            const int i = tid * (kBig / 32) + q;
+            ex += vals[q];
+            if (i < m) S.off[i + 1] = ex;
+        }
+    }
+    __syncthreads();
+}
+
+// Flattened pass over all entries of the loaded round.  f(t, y, dy) is called
+// for every entry (t = row slot, y = neighbour, dy = d[y] gathered up front)
+// and returns a contribution that is summed into S.acc[t].  Ends with a barrier.
+template <class F>
+__device__ __forceinline__ void big_entries(BigSmem &S, const GView &g, const int32_t *dr, F f) {
+    const int tid = threadIdx.x, lane = tid & 31;
+    const int m = S.m, E = S.off[m];
+    for (int base = 0; base < E; base += kUnroll * kBlock) {
+        int t[kUnroll], y[kUnroll], dy[kUnroll];
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u) {
+            const int e = base + u * kBlock + tid;
+            t[u] = -1;
+            if (e < E) {
+                int lo = 0, hi = m - 1;  // last t with off[t] <= e
+                while (lo < hi) {
+                    const int mid = (lo + hi + 1) >> 1;
+                    if (S.off[mid] <= e) lo = mid; else hi = mid - 1;
+                }
+                t[u] = lo;
+                y[u] = ldg_i(g.col + S.b[lo] + (e - S.off[lo]));
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u)
+            if (t[u] >= 0) dy[u] = ldcg_i(dr + y[u]);
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u) {
+            double c = 0.0;
+            if (t[u] >= 0) c = f(t[u], y[u], dy[u]);
+            const int t0 = __shfl_sync(kFull, t[u], 0);
+            const bool uni = __all_sync(kFull, t[u] == t0 || t[u] < 0);
+            if (uni) {
+                if (t0 >= 0) {
+#pragma unroll
+                    for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(kFull, c, o);
+                    if (lane == 0 && c != 0.0) atomicAdd(&S.acc[t0], c);
+                }
+            } else if (c != 0.0) {
+                atomicAdd(&S.acc[t[u]], c);
+            }
+        }
+    }
+    __syncthreads();
 }
 
 // ---------------------------------------------------------------------------

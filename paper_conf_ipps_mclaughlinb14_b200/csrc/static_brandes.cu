@@ -16,15 +16,21 @@
 
 namespace dbc {
 
-__global__ void __launch_bounds__(kBlock) static_kernel(StaticArgs a) {
+__global__ void __launch_bounds__(kBlock, 2) static_kernel(StaticArgs a) {
     __shared__ int s_slot;
     __shared__ int s_tail;
+    __shared__ int s_nbig;
+    __shared__ BigSmem S;
     const int tid = threadIdx.x;
     const int w = blockIdx.x;
     const size_t n = (size_t)a.n;
     int32_t *order = a.ws.Dv + (size_t)w * n;
     int32_t *loff = a.ws.Doff + (size_t)w * (n + 2);
+    int32_t *Bq = a.ws.Bq + (size_t)w * n;
+    const GView &g = a.g;
     unsigned long long bytes = 0;
+    auto enq = [&](int idx) { Bq[atomicAdd(&s_nbig, 1)] = idx; };
+    if (tid == 0) s_nbig = 0;
 
     for (;;) {
         if (tid == 0) s_slot = atomicAdd(a.next_slot, 1);
@@ -36,10 +42,13 @@ __global__ void __launch_bounds__(kBlock) static_kernel(StaticArgs a) {
         int32_t *dr = a.d + (size_t)slot * n;
         double2 *sdr = a.sd + (size_t)slot * n;
 
-        // Stage 1 (Alg. 1 lines 3-9): d = INF, sigma = delta = 0.
-        for (size_t v = tid; v < n; v += kBlock) {
-            dr[v] = kInf;
-            sdr[v] = make_double2(0.0, 0.0);
+        // Stage 1 (Alg. 1 lines 3-9): d = INF, sigma = delta = 0 (vectorised stores).
+        {
+            int4 *d4 = reinterpret_cast<int4 *>(dr);
+            const size_t n4 = ((size_t)slot * n) % 4 == 0 ? n / 4 : 0;
+            for (size_t v = tid; v < n4; v += kBlock) d4[v] = make_int4(kInf, kInf, kInf, kInf);
+            for (size_t v = n4 * 4 + tid; v < n; v += kBlock) dr[v] = kInf;
+            for (size_t v = tid; v < n; v += kBlock) sdr[v] = make_double2(0.0, 0.0);
         }
         if (tid == 0) bytes += 20ull * n;
         __syncthreads();
@@ -54,98 +63,126 @@ __global__ void __launch_bounds__(kBlock) static_kernel(StaticArgs a) {
         __syncthreads();
 
         // Stage 2: level-synchronous BFS; level L's sigma pull fused with the
-        // discovery of level L+1.
+        // discovery of level L+1 (one scan of each row).
         int L = 0, lb = 0, le = 1, nl = 1;
+        auto fwd_visit = [&](int x, int dx) -> double {
+            if (dx == L - 1) {
+                bytes += 8;
+                return ldcg_d2(sdr + x).x;
+            }
+            if (dx == kInf && atomicCAS(dr + x, kInf, L + 1) == kInf) {
+                order[atomicAdd(&s_tail, 1)] = x;
+                bytes += 4;
+            }
+            return 0.0;
+        };
+        auto fwd_finish = [&](int v, double sum) {
+            bytes += 8;
+            if (L > 0) {
+                sdr[v].x = sum;
+                bytes += 8;
+                if (!(sum <= 1.7976931348623157e308)) atomicOr(a.err, kErrNumeric);
+            }
+        };
         while (lb < le) {
-            const int cnt = le - lb;
-            two_tier(
-                cnt, a.g, INT32_MAX,
-                [&](int i, int &v) { v = order[lb + i]; return true; },
+            split_pass(
+                le - lb, g, INT32_MAX, [&](int i, int &v) { v = order[lb + i]; return true; },
                 [&](int, int) { return true; },
-                [&](auto Gc, int, int wv, int2 r, int gl) {
-                    constexpr int G = decltype(Gc)::value;
-                    double sum = 0.0;
-                    unsigned long long by = 0;
-                    for (int j = r.x + gl; j < r.y; j += G) {
-                        const int x = ldg_i(a.g.col + j);
-                        int dx = ldcg_i(dr + x);
-                        by += 8;
-                        if (dx == L - 1) {
-                            sum += ldcg_d2(sdr + x).x;
-                            by += 8;
-                        } else if (dx == kInf) {
-                            if (atomicCAS(dr + x, kInf, L + 1) == kInf) {
-                                const int pos = atomicAdd(&s_tail, 1);
-                                order[pos] = x;
-                                by += 4;
-                            }
-                        }
+                [&](int, int v, int2 r) {
+                    double sum = 0.0;  // canonical order
+                    for (int j = r.x; j < r.y; ++j) {
+                        const int x = ldg_i(g.col + j);
+                        sum += fwd_visit(x, ldcg_i(dr + x));
                     }
-                    sum = group_sum<G>(sum);
-                    if constexpr (G == 32) {
-                        if (sum >= kExact) {  // order-dependent rounding: canonical sum
-                            if (gl == 0) {
-                                sum = 0.0;
-                                for (int j = r.x; j < r.y; ++j) {
-                                    const int x = ldg_i(a.g.col + j);
-                                    if (ldcg_i(dr + x) == L - 1) sum += ldcg_d2(sdr + x).x;
-                                }
-                            }
-                            sum = __shfl_sync(kFull, sum, 0);
-                        }
-                    }
-                    if (gl == 0) {
-                        by += 8;
-                        if (L > 0) {
-                            sdr[wv].x = sum;
-                            by += 8;
-                            if (!(sum <= 1.7976931348623157e308)) atomicOr(a.err, kErrNumeric);
-                        }
-                    }
-                    bytes += by;
-                });
+                    bytes += 8ull * (r.y - r.x);
+                    fwd_finish(v, sum);
+                },
+                enq);
             __syncthreads();
+            const int nbig = s_nbig;
+            for (int r0 = 0; r0 < nbig; r0 += kBig) {
+                const int m = min(kBig, nbig - r0);
+                big_load(S, m, [&](int t) { return Bq[r0 + t]; }, [&](int i) { return order[lb + i]; },
+                         g, INT32_MAX);
+                big_entries(S, g, dr, [&](int, int x, int dx) {
+                    bytes += 8;
+                    return fwd_visit(x, dx);
+                });
+                if (tid < m) {
+                    double sum = S.acc[tid];
+                    const int v = S.v[tid];
+                    if (sum >= kExact) {  // order-dependent rounding: canonical sum
+                        const int2 r = row_of(g, v, INT32_MAX);
+                        sum = 0.0;
+                        for (int j = r.x; j < r.y; ++j) {
+                            const int x = ldg_i(g.col + j);
+                            if (ldcg_i(dr + x) == L - 1) sum += ldcg_d2(sdr + x).x;
+                        }
+                    }
+                    fwd_finish(v, sum);
+                }
+                __syncthreads();
+            }
             const int ne = s_tail;
+            __syncthreads();
+            if (tid == 0) {
+                s_nbig = 0;
+                loff[nl + 1] = ne;
+            }
             __syncthreads();
             lb = le;
             le = ne;
-            if (tid == 0) loff[nl + 1] = le;
             ++nl;
             ++L;
         }
-        __syncthreads();
         // levels 0 .. nl-2 are non-empty; loff[j] .. loff[j+1] is level j.
 
         // Stage 3: dependency accumulation in reverse level order (Eq. (2)),
         // BC partial += delta (Eq. (3)), root excluded (delta_s(s) = 0).
         for (int lev = nl - 2; lev >= 1; --lev) {
             const int b0 = loff[lev], b1 = loff[lev + 1];
-            two_tier(
-                b1 - b0, a.g, INT32_MAX,
-                [&](int i, int &v) { v = order[b0 + i]; return true; },
+            auto bwd_visit = [&](double sv, int y, int dy) -> double {
+                if (dy != lev + 1) return 0.0;
+                const double2 t = ldcg_d2(sdr + y);
+                bytes += 16;
+                return __dmul_rn(__ddiv_rn(sv, t.x), __dadd_rn(1.0, t.y));
+            };
+            auto bwd_finish = [&](int v, double acc) {
+                sdr[v].y = acc;
+                atomicAdd(a.bc + v, acc);
+                bytes += 8 + 8 + 16;
+            };
+            split_pass(
+                b1 - b0, g, INT32_MAX, [&](int i, int &v) { v = order[b0 + i]; return true; },
                 [&](int, int) { return true; },
-                [&](auto Gc, int, int v, int2 r, int gl) {
-                    constexpr int G = decltype(Gc)::value;
+                [&](int, int v, int2 r) {
                     const double sv = ldcg_d2(sdr + v).x;
                     double acc = 0.0;
-                    unsigned long long by = 0;
-                    for (int j = r.x + gl; j < r.y; j += G) {
-                        const int y = ldg_i(a.g.col + j);
-                        by += 8;
-                        if (ldcg_i(dr + y) == lev + 1) {
-                            const double2 t = ldcg_d2(sdr + y);
-                            acc += __dmul_rn(__ddiv_rn(sv, t.x), __dadd_rn(1.0, t.y));
-                            by += 16;
-                        }
+                    for (int j = r.x; j < r.y; ++j) {
+                        const int y = ldg_i(g.col + j);
+                        acc += bwd_visit(sv, y, ldcg_i(dr + y));
                     }
-                    acc = group_sum<G>(acc);
-                    if (gl == 0) {
-                        sdr[v].y = acc;
-                        atomicAdd(a.bc + v, acc);
-                        by += 8 + 8 + 16;
-                    }
-                    bytes += by;
+                    bytes += 8ull * (r.y - r.x);
+                    bwd_finish(v, acc);
+                },
+                enq);
+            __syncthreads();
+            const int nbig = s_nbig;
+            for (int r0 = 0; r0 < nbig; r0 += kBig) {
+                const int m = min(kBig, nbig - r0);
+                big_load(S, m, [&](int t) { return Bq[r0 + t]; }, [&](int i) { return order[b0 + i]; },
+                         g, INT32_MAX);
+                if (tid < m) S.c0[tid] = ldcg_d2(sdr + S.v[tid]).x;
+                __syncthreads();
+                big_entries(S, g, dr, [&](int t, int y, int dy) {
+                    bytes += 8;
+                    return bwd_visit(S.c0[t], y, dy);
                 });
+                if (tid < m) bwd_finish(S.v[tid], S.acc[tid]);
+                __syncthreads();
+            }
+            __syncthreads();
+            if (tid == 0) s_nbig = 0;
             __syncthreads();
         }
     }

@@ -37,16 +37,21 @@
 
 namespace dbc {
 
-__device__ __forceinline__ int append_smem(int *ctr) { return atomicAdd(ctr, 1); }
+constexpr int kSrcR = 0x40000000;  // back-queue tag: item is a removal-push target
 
-__global__ void __launch_bounds__(kBlock) update_kernel(UpdateArgs a) {
+__global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
     __shared__ int s_slot;
     __shared__ int s_dcnt;   // |D| (absolute positions in Dv)
     __shared__ int s_ucnt;   // next up frontier size
     __shared__ int s_rcnt;   // |R|
     __shared__ int s_rmax;   // deepest removal-push target level
+    __shared__ int s_nbig, s_nbig2;      // big-row queue (front: D rows, back: U/R rows)
     __shared__ uint32_t s_work[kWarps];  // window classification bits (1 = Case 2/3)
     __shared__ int s_job[4];             // uh, ul, L0, case3 of the current job
+    __shared__ BigSmem S;
+    __shared__ double s_c2[kBig];
+    __shared__ int s_f0[kBig];
+
     const int tid = threadIdx.x;
     const int wk = blockIdx.x;
     const size_t n = (size_t)a.n;
@@ -62,10 +67,21 @@ __global__ void __launch_bounds__(kBlock) update_kernel(UpdateArgs a) {
     int32_t *Ub = a.ws.U1 + (size_t)wk * n;
     int32_t *Rv = a.ws.Rv + (size_t)wk * n;
     int32_t *Rl = a.ws.Rl + (size_t)wk * n;
+    int32_t *Bq = a.ws.Bq + (size_t)wk * n;
     uint32_t epoch = a.ws.wepoch[wk];
+    const GView &g = a.g;
 
     unsigned long long st_bytes = 0, st_scanned = 0, st_touched = 0, st_down = 0;
-    unsigned long long st_case[3] = {0, 0, 0};
+    unsigned long long st_c1 = 0, st_c2 = 0, st_c3 = 0;
+
+    auto enq_front = [&](int idx) { Bq[atomicAdd(&s_nbig, 1)] = idx; };
+    auto enq_back = [&](int idx) { Bq[n - 1 - atomicAdd(&s_nbig2, 1)] = idx; };
+    auto fetch_front = [&](int r0) { return [=](int t) { return Bq[r0 + t]; }; };
+
+    if (tid == 0) {
+        s_nbig = 0;
+        s_nbig2 = 0;
+    }
 
     for (;;) {
         if (tid == 0) s_slot = atomicAdd(a.next_slot, 1);
@@ -73,7 +89,6 @@ __global__ void __launch_bounds__(kBlock) update_kernel(UpdateArgs a) {
         const int slot = s_slot;
         __syncthreads();
         if (slot >= a.k_loc) break;
-        (void)a.roots;
         int32_t *dr = a.d + (size_t)slot * n;
         double2 *sdr = a.sd + (size_t)slot * n;
 
@@ -100,7 +115,7 @@ __global__ void __launch_bounds__(kBlock) update_kernel(UpdateArgs a) {
                 const int off = p - ins;
                 if (!((s_work[off >> 5] >> (off & 31)) & 1u)) {  // Case 1: no work
                     if (tid == 0) {
-                        st_case[0]++;
+                        st_c1++;
                         st_bytes += 8;
                     }
                     continue;
@@ -117,7 +132,10 @@ __global__ void __launch_bounds__(kBlock) update_kernel(UpdateArgs a) {
                     const int dh = u_is_high ? du : dv, dlo = u_is_high ? dv : du;
                     const int L0 = dh + 1;
                     const bool c3 = dlo > L0;
-                    st_case[c3 ? 2 : 1]++;
+                    if (c3)
+                        st_c3++;
+                    else
+                        st_c2++;
                     st_bytes += 8;
                     if (c3) {
                         lowrec[ul] = ((unsigned long long)epoch << 32) | (uint32_t)dlo;
@@ -141,72 +159,88 @@ __global__ void __launch_bounds__(kBlock) update_kernel(UpdateArgs a) {
                 const bool case3 = s_job[3] != 0;
                 const int lim = p;  // graph as of this insertion (edge p included)
 
-                // ---------------- down phase (K3) ----------------
+                // ================= down phase (K3) =================
                 int L = L0, lb = 0, le = 1, nlev = 1;
+                // per-D-entry epilogue: record old d / sigma, store the new sigma
+                auto down_finish = [&](int idx, int w, double sum) {
+                    const unsigned long long lr = ldcg_ull(lowrec + w);
+                    const int od = ((uint32_t)(lr >> 32) == epoch) ? (int)(uint32_t)lr : L;
+                    Dold[idx] = od;
+                    Dsig[idx] = ldcg_d2(sdr + w).x;
+                    sdr[w].x = sum;
+                    if (!(sum <= 1.7976931348623157e308)) atomicOr(a.err, kErrNumeric);
+                    st_bytes += 8 + 8 + 20;
+                };
+                // one neighbour y of a level-L vertex; returns sigma[y] if y is a predecessor
+                auto down_visit = [&](int y, int dy) -> double {
+                    if (dy == L - 1) {
+                        st_bytes += 8;
+                        return ldcg_d2(sdr + y).x;
+                    }
+                    if (dy > L + 1) {  // Case 3 pull-up
+                        const int old = atomicMin(dr + y, L + 1);
+                        if (old > L + 1) {
+                            lowrec[y] = ((unsigned long long)epoch << 32) | (uint32_t)old;
+                            st_bytes += 4;
+                        }
+                        dy = L + 1;
+                    }
+                    if (dy == L + 1 && atomicMax(mark + y, mD) < mD)
+                        Dv[atomicAdd(&s_dcnt, 1)] = y;
+                    return 0.0;
+                };
                 while (true) {
-                    two_tier(
-                        le - lb, a.g, lim,
-                        [&](int i, int &w) { w = Dv[lb + i]; return true; },
+                    split_pass(
+                        le - lb, g, lim, [&](int i, int &w) { w = Dv[lb + i]; return true; },
                         [&](int, int) { return true; },
-                        [&](auto Gc, int i, int w, int2 r, int gl) {
-                            constexpr int G = decltype(Gc)::value;
-                            const int idx = lb + i;
-                            double sum = 0.0;
-                            unsigned long long by = 0, sc = 0;
-                            for (int j = r.x + gl; j < r.y; j += G) {
-                                const int y = ldg_i(a.g.col + j);
-                                int dy = ldcg_i(dr + y);
-                                ++sc;
-                                if (dy == L - 1) {
-                                    sum += ldcg_d2(sdr + y).x;
-                                    by += 8;
-                                } else if (dy > L + 1) {
-                                    const int old = atomicMin(dr + y, L + 1);
-                                    if (old > L + 1) {
-                                        lowrec[y] = ((unsigned long long)epoch << 32) | (uint32_t)old;
-                                        by += 4;
-                                    }
-                                    dy = L + 1;
-                                }
-                                if (dy == L + 1) {
-                                    if (atomicMax(mark + y, mD) < mD) {
-                                        Dv[append_smem(&s_dcnt)] = y;
-                                    }
-                                }
+                        [&](int i, int w, int2 r) {
+                            double sum = 0.0;  // canonical order: bit-exact
+                            for (int j = r.x; j < r.y; ++j) {
+                                const int y = ldg_i(g.col + j);
+                                sum += down_visit(y, ldcg_i(dr + y));
                             }
-                            sum = group_sum<G>(sum);
-                            if constexpr (G == 32) {
-                                if (sum >= kExact) {  // not provably exact: canonical-order sum
-                                    if (gl == 0) {
-                                        sum = 0.0;
-                                        for (int j = r.x; j < r.y; ++j) {
-                                            const int y = ldg_i(a.g.col + j);
-                                            if (ldcg_i(dr + y) == L - 1) sum += ldcg_d2(sdr + y).x;
-                                        }
-                                    }
-                                    sum = __shfl_sync(kFull, sum, 0);
-                                }
-                            }
-                            if (gl == 0) {
-                                const unsigned long long lr = ldcg_ull(lowrec + w);
-                                const int od = ((uint32_t)(lr >> 32) == epoch) ? (int)(uint32_t)lr : L;
-                                Dold[idx] = od;
-                                Dsig[idx] = ldcg_d2(sdr + w).x;
-                                sdr[w].x = sum;
-                                if (!(sum <= 1.7976931348623157e308)) atomicOr(a.err, kErrNumeric);
-                                by += 8 + 8 + 20;
-                            }
-                            st_bytes += by + 8 * sc;
-                            st_scanned += sc;
+                            st_bytes += 8 + 8ull * (r.y - r.x);
+                            st_scanned += r.y - r.x;
+                            down_finish(lb + i, w, sum);
+                        },
+                        enq_front);
+                    __syncthreads();
+                    const int nbig = s_nbig;
+                    for (int r0 = 0; r0 < nbig; r0 += kBig) {
+                        const int m = min(kBig, nbig - r0);
+                        big_load(S, m, fetch_front(r0), [&](int i) { return Dv[lb + i]; }, g, lim);
+                        big_entries(S, g, dr, [&](int, int y, int dy) {
+                            st_bytes += 8;
+                            st_scanned++;
+                            return down_visit(y, dy);
                         });
-                    __syncthreads();
+                        if (tid < m) {
+                            double sum = S.acc[tid];
+                            const int w = S.v[tid];
+                            if (sum >= kExact) {  // order-dependent rounding: canonical sum
+                                const int2 r = row_of(g, w, lim);
+                                sum = 0.0;
+                                for (int j = r.x; j < r.y; ++j) {
+                                    const int y = ldg_i(g.col + j);
+                                    if (ldcg_i(dr + y) == L - 1) sum += ldcg_d2(sdr + y).x;
+                                }
+                            }
+                            st_bytes += 8;
+                            down_finish(lb + S.idx[tid], w, sum);
+                        }
+                        __syncthreads();
+                    }
                     const int ne = s_dcnt;
-                    __syncthreads();
+                    __syncthreads();  // everyone has read nbig / ne
+                    if (tid == 0) {
+                        s_nbig = 0;
+                        if (ne != le) Doff[nlev + 1] = ne;
+                    }
+                    __syncthreads();  // reset visible before the next level enqueues
                     if (ne == le) break;
                     lb = le;
                     le = ne;
                     ++nlev;
-                    if (tid == 0) Doff[nlev] = le;
                     ++L;
                 }
                 // D levels: level L0 + j occupies Dv[Doff[j] .. Doff[j+1]), j < nlev
@@ -216,182 +250,240 @@ __global__ void __launch_bounds__(kBlock) update_kernel(UpdateArgs a) {
                     st_down += dtotal;
                     st_touched += dtotal;
                 }
+                __syncthreads();
 
-                // ---------------- (0) Case-3 removal pushes ----------------
+                // ================= (0) Case-3 removal pushes =================
                 if (case3) {
-                    for (int j = 0; j < nlev; ++j) {
-                        const int b0 = Doff[j], b1 = Doff[j + 1];
-                        const int lev = L0 + j;
-                        two_tier(
-                            b1 - b0, a.g, lim,
-                            [&](int i, int &w) {
-                                const int od = Dold[b0 + i];
-                                w = Dv[b0 + i];
-                                return od != lev && od != kInf;
-                            },
-                            [&](int, int) { return true; },
-                            [&](auto Gc, int i, int w, int2 r, int gl) {
-                                constexpr int G = decltype(Gc)::value;
-                                const int idx = b0 + i;
-                                const int od = Dold[idx];
-                                const double osig = Dsig[idx];
-                                const double coef = 1.0 + ldcg_d2(sdr + w).y;  // delta still old
-                                unsigned long long by = 0, sc = 0;
-                                for (int j2 = r.x + gl; j2 < r.y; j2 += G) {
-                                    const int x = ldg_i(a.g.col + j2);
-                                    ++sc;
-                                    if (ldcg_i(dr + x) != od - 1) continue;
-                                    if (x == uh && w == ul) continue;
-                                    const uint32_t mx = ldcg_u(mark + x);
-                                    if (mx == mD) continue;
-                                    const double sx = ldcg_d2(sdr + x).x;
-                                    atomicAdd(dacc + x, -__dmul_rn(__ddiv_rn(sx, osig), coef));
-                                    by += 24;
-                                    if (atomicMax(mark + x, mU) < E) {
-                                        const int pos = append_smem(&s_rcnt);
-                                        Rv[pos] = x;
-                                        Rl[pos] = od - 1;
-                                        atomicMax(&s_rmax, od - 1);
-                                    }
-                                }
-                                if (gl == 0) by += 8 + 8;
-                                st_bytes += by + 8 * sc;
-                                st_scanned += sc;
-                            });
+                    // a pulled-up w (finite old level od) loses its old predecessors x
+                    auto rem_visit = [&](int w, int od, double osig, double coef, int x, int dx) {
+                        if (dx != od - 1 || (x == uh && w == ul)) return;
+                        if (ldcg_u(mark + x) == mD) return;
+                        const double sx = ldcg_d2(sdr + x).x;
+                        atomicAdd(dacc + x, -__dmul_rn(__ddiv_rn(sx, osig), coef));
+                        st_bytes += 24;
+                        if (atomicMax(mark + x, mU) < E) {
+                            const int pos = atomicAdd(&s_rcnt, 1);
+                            Rv[pos] = x;
+                            Rl[pos] = od - 1;
+                            atomicMax(&s_rmax, od - 1);
+                        }
+                    };
+                    split_pass(
+                        dtotal, g, lim,
+                        [&](int i, int &w) {
+                            const int od = Dold[i];
+                            w = Dv[i];
+                            return od != kInf && od != ldcg_i(dr + w);
+                        },
+                        [&](int, int) { return true; },
+                        [&](int i, int w, int2 r) {
+                            const int od = Dold[i];
+                            const double osig = Dsig[i];
+                            const double coef = 1.0 + ldcg_d2(sdr + w).y;  // delta still old
+                            for (int j = r.x; j < r.y; ++j) {
+                                const int x = ldg_i(g.col + j);
+                                rem_visit(w, od, osig, coef, x, ldcg_i(dr + x));
+                            }
+                            st_bytes += 16 + 8ull * (r.y - r.x);
+                            st_scanned += r.y - r.x;
+                        },
+                        enq_front);
+                    __syncthreads();
+                    const int nbig = s_nbig;
+                    for (int r0 = 0; r0 < nbig; r0 += kBig) {
+                        const int m = min(kBig, nbig - r0);
+                        big_load(S, m, fetch_front(r0), [&](int i) { return Dv[i]; }, g, lim);
+                        if (tid < m) {
+                            const int i = S.idx[tid];
+                            s_f0[tid] = Dold[i];
+                            S.c0[tid] = Dsig[i];
+                            S.c1[tid] = 1.0 + ldcg_d2(sdr + S.v[tid]).y;
+                            st_bytes += 16;
+                        }
+                        __syncthreads();
+                        big_entries(S, g, dr, [&](int t, int x, int dx) {
+                            st_bytes += 8;
+                            st_scanned++;
+                            rem_visit(S.v[t], s_f0[t], S.c0[t], S.c1[t], x, dx);
+                            return 0.0;
+                        });
                     }
+                    __syncthreads();
+                    if (tid == 0) s_nbig = 0;
                     __syncthreads();
                 }
                 const int rcnt = s_rcnt;
                 const int Lmax = max(LmaxD, s_rmax);
                 if (tid == 0) st_touched += rcnt;
 
-                // ---------------- up phase (K4 + Alg. 8) ----------------
+                // ================= up phase (K4 + Alg. 8) =================
                 int *Ucur = Ua, *Unext = Ub;
                 int ucnt = 0;
                 for (int l = Lmax; l >= 1; --l) {
                     if (l < L0 && ucnt == 0) break;  // nothing left above the insertion
-                    // down vertices at level l
+                    const bool push = l >= 2;          // level-1 vertices only feed the root
+                    auto claim_up = [&](int y) {
+                        if (atomicMax(mark + y, mU) < E) Unext[atomicAdd(&s_ucnt, 1)] = y;
+                    };
+                    // up vertex x (not in D): push sigma[p]/sigma[x] * Ddelta[x] upwards
+                    auto up_visit = [&](double gx, double sx, int pp, int dp) {
+                        if (dp != l - 1) return;
+                        const double sp = ldcg_d2(sdr + pp).x;
+                        atomicAdd(dacc + pp, __dmul_rn(__ddiv_rn(sp, sx), gx));
+                        st_bytes += 24;
+                        claim_up(pp);
+                    };
+                    auto up_finish = [&](int x, double gx) {
+                        dacc[x] = 0.0;
+                        sdr[x].y = ldcg_d2(sdr + x).y + gx;
+                        atomicAdd(a.bc + x, gx);
+                        st_bytes += 8 + 8 + 16 + 16;
+                    };
+                    auto up_small = [&](int, int x, int2 r) {
+                        const double gx = ldcg_d(dacc + x);
+                        if (gx != 0.0 && r.y > r.x) {
+                            const double sx = ldcg_d2(sdr + x).x;
+                            for (int j = r.x; j < r.y; ++j) {
+                                const int pp = ldg_i(g.col + j);
+                                up_visit(gx, sx, pp, ldcg_i(dr + pp));
+                            }
+                            st_bytes += 16 + 8ull * (r.y - r.x);
+                            st_scanned += r.y - r.x;
+                        }
+                        up_finish(x, gx);
+                    };
+                    // down vertex x: pull delta (Eq. (2)), then push new-minus-old contributions
+                    auto dpull_visit = [&](double sx, int y, int dy) -> double {
+                        if (dy != l + 1) return 0.0;
+                        const double2 t = ldcg_d2(sdr + y);
+                        st_bytes += 16;
+                        return __dmul_rn(__ddiv_rn(sx, t.x), __dadd_rn(1.0, t.y));
+                    };
+                    auto dpush_visit = [&](int x, double sx, double dn, double odel, double osig,
+                                           bool not_pulled, int pp, int dp) {
+                        if (dp != l - 1) return;
+                        if (ldcg_u(mark + pp) == mD) return;
+                        const double sp = ldcg_d2(sdr + pp).x;
+                        double dlt = __dmul_rn(__ddiv_rn(sp, sx), 1.0 + dn);
+                        if (not_pulled && !(pp == uh && x == ul))
+                            dlt = __dsub_rn(dlt, __dmul_rn(__ddiv_rn(sp, osig), 1.0 + odel));
+                        atomicAdd(dacc + pp, dlt);
+                        st_bytes += 24;
+                        claim_up(pp);
+                    };
+                    auto d_finish = [&](int x, double dn, double odel) {
+                        sdr[x].y = dn;
+                        atomicAdd(a.bc + x, dn - odel);
+                        st_bytes += 8 + 16 + 16;
+                    };
+
+                    int b0 = 0, b1 = 0;
                     if (l >= L0 && l <= LmaxD) {
-                        const int b0 = Doff[l - L0], b1 = Doff[l - L0 + 1];
-                        two_tier(
-                            b1 - b0, a.g, lim,
-                            [&](int i, int &x) { x = Dv[b0 + i]; return true; },
-                            [&](int, int) { return true; },
-                            [&](auto Gc, int i, int x, int2 r, int gl) {
-                                constexpr int G = decltype(Gc)::value;
+                        b0 = Doff[l - L0];
+                        b1 = Doff[l - L0 + 1];
+                    }
+                    // --- small rows of the three sources; big rows queued ---
+                    split_pass(
+                        b1 - b0, g, lim, [&](int i, int &x) { x = Dv[b0 + i]; return true; },
+                        [&](int, int) { return true; },
+                        [&](int i, int x, int2 r) {
+                            const double2 s2 = ldcg_d2(sdr + x);
+                            double dn = 0.0;
+                            for (int j = r.x; j < r.y; ++j) {
+                                const int y = ldg_i(g.col + j);
+                                dn += dpull_visit(s2.x, y, ldcg_i(dr + y));
+                            }
+                            st_scanned += r.y - r.x;
+                            st_bytes += 16 + 8ull * (r.y - r.x);
+                            if (push) {
                                 const int idx = b0 + i;
-                                const double2 sx2 = ldcg_d2(sdr + x);
-                                const double sx = sx2.x, odel = sx2.y;
-                                double acc = 0.0;
-                                unsigned long long by = 0, sc = 0;
-                                for (int j = r.x + gl; j < r.y; j += G) {
-                                    const int y = ldg_i(a.g.col + j);
-                                    ++sc;
-                                    if (ldcg_i(dr + y) == l + 1) {
-                                        const double2 t = ldcg_d2(sdr + y);
-                                        acc += __dmul_rn(__ddiv_rn(sx, t.x), __dadd_rn(1.0, t.y));
-                                        by += 16;
-                                    }
+                                const bool np = Dold[idx] == l;
+                                const double osig = Dsig[idx];
+                                for (int j = r.x; j < r.y; ++j) {
+                                    const int pp = ldg_i(g.col + j);
+                                    dpush_visit(x, s2.x, dn, s2.y, osig, np, pp, ldcg_i(dr + pp));
                                 }
-                                acc = group_sum<G>(acc);
-                                if (l >= 2) {
-                                    const bool not_pulled = Dold[idx] == l;
-                                    const double osig = Dsig[idx];
-                                    const double cnew = 1.0 + acc, cold = 1.0 + odel;
-                                    for (int j = r.x + gl; j < r.y; j += G) {
-                                        const int p = ldg_i(a.g.col + j);
-                                        ++sc;
-                                        if (ldcg_i(dr + p) != l - 1) continue;
-                                        const uint32_t mp = ldcg_u(mark + p);
-                                        if (mp == mD) continue;
-                                        const double sp = ldcg_d2(sdr + p).x;
-                                        double dlt = __dmul_rn(__ddiv_rn(sp, sx), cnew);
-                                        if (not_pulled && !(p == uh && x == ul))
-                                            dlt = __dsub_rn(dlt, __dmul_rn(__ddiv_rn(sp, osig), cold));
-                                        atomicAdd(dacc + p, dlt);
-                                        by += 24;
-                                        if (atomicMax(mark + p, mU) < E) Unext[append_smem(&s_ucnt)] = p;
-                                    }
-                                }
-                                group_sync<G>();
-                                if (gl == 0) {
-                                    sdr[x].y = acc;
-                                    atomicAdd(a.bc + x, acc - odel);
-                                    by += 8 + 16 + 16;
-                                }
-                                st_bytes += by + 8 * sc;
-                                st_scanned += sc;
-                            });
-                    }
-                    // up vertices at level l found by level l+1
-                    two_tier(
-                        ucnt, a.g, lim,
-                        [&](int i, int &x) { x = Ucur[i]; return true; },
-                        [&](int, int) { return l >= 2; },
-                        [&](auto Gc, int, int x, int2 r, int gl) {
-                            constexpr int G = decltype(Gc)::value;
-                            const double g = ldcg_d(dacc + x);
-                            unsigned long long by = 0, sc = 0;
-                            if (g != 0.0) {
-                                const double sx = ldcg_d2(sdr + x).x;
-                                for (int j = r.x + gl; j < r.y; j += G) {
-                                    const int p = ldg_i(a.g.col + j);
-                                    ++sc;
-                                    if (ldcg_i(dr + p) != l - 1) continue;
-                                    const double sp = ldcg_d2(sdr + p).x;
-                                    atomicAdd(dacc + p, __dmul_rn(__ddiv_rn(sp, sx), g));
-                                    by += 24;
-                                    if (atomicMax(mark + p, mU) < E) Unext[append_smem(&s_ucnt)] = p;
-                                }
+                                st_scanned += r.y - r.x;
+                                st_bytes += 16 + 8ull * (r.y - r.x);
                             }
-                            group_sync<G>();
-                            if (gl == 0) {
-                                dacc[x] = 0.0;
-                                sdr[x].y = ldcg_d2(sdr + x).y + g;
-                                atomicAdd(a.bc + x, g);
-                                by += 8 + 8 + 16 + 16 + (r.y > r.x ? 8 : 0);
-                            }
-                            st_bytes += by + 8 * sc;
-                            st_scanned += sc;
-                        });
-                    // removal-push targets at level l
-                    if (rcnt) {
-                        two_tier(
-                            rcnt, a.g, lim,
-                            [&](int i, int &x) { x = Rv[i]; return Rl[i] == l; },
-                            [&](int, int) { return l >= 2; },
-                            [&](auto Gc, int, int x, int2 r, int gl) {
-                                constexpr int G = decltype(Gc)::value;
-                                const double g = ldcg_d(dacc + x);
-                                unsigned long long by = 0, sc = 0;
-                                if (g != 0.0) {
-                                    const double sx = ldcg_d2(sdr + x).x;
-                                    for (int j = r.x + gl; j < r.y; j += G) {
-                                        const int p = ldg_i(a.g.col + j);
-                                        ++sc;
-                                        if (ldcg_i(dr + p) != l - 1) continue;
-                                        const double sp = ldcg_d2(sdr + p).x;
-                                        atomicAdd(dacc + p, __dmul_rn(__ddiv_rn(sp, sx), g));
-                                        by += 24;
-                                        if (atomicMax(mark + p, mU) < E) Unext[append_smem(&s_ucnt)] = p;
-                                    }
-                                }
-                                group_sync<G>();
-                                if (gl == 0) {
-                                    dacc[x] = 0.0;
-                                    sdr[x].y = ldcg_d2(sdr + x).y + g;
-                                    atomicAdd(a.bc + x, g);
-                                    by += 8 + 8 + 16 + 16 + (r.y > r.x ? 8 : 0);
-                                }
-                                st_bytes += by + 8 * sc;
-                                st_scanned += sc;
-                            });
-                    }
+                            d_finish(x, dn, s2.y);
+                        },
+                        enq_front);
+                    split_pass(
+                        ucnt, g, lim, [&](int i, int &x) { x = Ucur[i]; return true; },
+                        [&](int, int) { return push; }, up_small, enq_back);
+                    if (rcnt)
+                        split_pass(
+                            rcnt, g, lim,
+                            [&](int i, int &x) {
+                                x = Rv[i];
+                                return Rl[i] == l;
+                            },
+                            [&](int, int) { return push; }, up_small,
+                            [&](int idx) { enq_back(idx | kSrcR); });
                     __syncthreads();
+                    const int nD = s_nbig, nU = s_nbig2;
+                    // --- big down rows: pull pass, push pass, epilogue ---
+                    for (int r0 = 0; r0 < nD; r0 += kBig) {
+                        const int m = min(kBig, nD - r0);
+                        big_load(S, m, fetch_front(r0), [&](int i) { return Dv[b0 + i]; }, g, lim);
+                        if (tid < m) {
+                            const int idx = b0 + S.idx[tid];
+                            const double2 s2 = ldcg_d2(sdr + S.v[tid]);
+                            S.c0[tid] = s2.x;
+                            S.c1[tid] = s2.y;
+                            s_c2[tid] = Dsig[idx];
+                            s_f0[tid] = Dold[idx] == l;
+                            st_bytes += 16 + 16;
+                        }
+                        __syncthreads();
+                        big_entries(S, g, dr, [&](int t, int y, int dy) {
+                            st_bytes += 8;
+                            st_scanned++;
+                            return dpull_visit(S.c0[t], y, dy);
+                        });
+                        if (push)
+                            big_entries(S, g, dr, [&](int t, int pp, int dp) {
+                                st_bytes += 8;
+                                st_scanned++;
+                                dpush_visit(S.v[t], S.c0[t], S.acc[t], S.c1[t], s_c2[t], s_f0[t] != 0,
+                                            pp, dp);
+                                return 0.0;
+                            });
+                        if (tid < m) d_finish(S.v[tid], S.acc[tid], S.c1[tid]);
+                        __syncthreads();
+                    }
+                    // --- big up rows (U and R) ---
+                    for (int r0 = 0; r0 < nU; r0 += kBig) {
+                        const int m = min(kBig, nU - r0);
+                        big_load(
+                            S, m, [&](int t) { return Bq[n - 1 - (r0 + t)]; },
+                            [&](int idx) { return (idx & kSrcR) ? Rv[idx & ~kSrcR] : Ucur[idx]; }, g, lim);
+                        if (tid < m) {
+                            const int x = S.v[tid];
+                            S.c0[tid] = ldcg_d(dacc + x);
+                            S.c1[tid] = ldcg_d2(sdr + x).x;
+                            st_bytes += 16;
+                        }
+                        __syncthreads();
+                        big_entries(S, g, dr, [&](int t, int pp, int dp) {
+                            const double gx = S.c0[t];
+                            if (gx != 0.0) {
+                                st_bytes += 8;
+                                st_scanned++;
+                                up_visit(gx, S.c1[t], pp, dp);
+                            }
+                            return 0.0;
+                        });
+                        if (tid < m) up_finish(S.v[tid], S.c0[tid]);
+                        __syncthreads();
+                    }
                     ucnt = s_ucnt;
                     __syncthreads();
                     if (tid == 0) {
                         s_ucnt = 0;
+                        s_nbig = 0;
+                        s_nbig2 = 0;
                         st_touched += ucnt;
                     }
                     int *t = Ucur;
@@ -411,9 +503,9 @@ __global__ void __launch_bounds__(kBlock) update_kernel(UpdateArgs a) {
     }
     if (tid == 0) {
         a.ws.wepoch[wk] = epoch;
-        if (st_case[0]) atomicAdd(a.stats + kStCase1, st_case[0]);
-        if (st_case[1]) atomicAdd(a.stats + kStCase2, st_case[1]);
-        if (st_case[2]) atomicAdd(a.stats + kStCase3, st_case[2]);
+        if (st_c1) atomicAdd(a.stats + kStCase1, st_c1);
+        if (st_c2) atomicAdd(a.stats + kStCase2, st_c2);
+        if (st_c3) atomicAdd(a.stats + kStCase3, st_c3);
         if (st_touched) atomicAdd(a.stats + kStTouched, st_touched);
         if (st_down) atomicAdd(a.stats + kStDown, st_down);
     }

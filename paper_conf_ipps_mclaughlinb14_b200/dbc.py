@@ -160,6 +160,8 @@ class DynamicBC:
                         stream = torch.cuda.current_stream().cuda_stream
             except Exception:  # pragma: no cover
                 stream = None
+        if stream == 0:
+            stream = 1  # torch's default stream is the legacy stream: cudaStreamLegacy
         opt.stream = stream
         out = ctypes.c_void_p()
         rc = lib.dbc_create(ctypes.byref(out), self.n, _np_ptr(rp), _np_ptr(cl), _np_ptr(rt),
