@@ -186,6 +186,19 @@ dbc_status dbc_get_timings(dbc_ctx *c, dbc_timings *t);
 /* Zeroes the cumulative fields of dbc_timings.  Synchronises. */
 dbc_status dbc_reset_timings(dbc_ctx *c);
 
+/* Diagnostic counters (cumulative since create; layout is internal and may
+ * change): case counts, touched, down vertices, scanned entries, algorithmic
+ * bytes, static bytes, then scanned entries per update phase (down, removal,
+ * down-vertex pull, down-vertex push, up vertices at level 2, at level >= 3).
+ * Fills min(count, available) values.  Synchronises. */
+dbc_status dbc_debug_counters(dbc_ctx *c, int64_t *out, int32_t count);
+
+/* Diagnostic per-root profile of the update kernel: enable != 0 turns recording
+ * on for later insert calls; out (nullable, int64[4 * k_local]) receives, per
+ * local root slot of the last update launch, {start ns, end ns, working
+ * (Case 2/3) insertions, touched vertices}.  Synchronises when out != NULL. */
+dbc_status dbc_debug_root_profile(dbc_ctx *c, int32_t enable, int64_t *out);
+
 /* Device memory held by the context, in bytes. */
 dbc_status dbc_device_bytes(const dbc_ctx *c, int64_t *bytes);
 

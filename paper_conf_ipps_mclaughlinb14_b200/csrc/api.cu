@@ -34,6 +34,7 @@ struct dbc_ctx {
     // graph double buffer
     int32_t *rp[2] = {nullptr, nullptr};
     int32_t *col[2] = {nullptr, nullptr};
+    int32_t *scol[2] = {nullptr, nullptr};  // rows sorted by neighbour id
     int cur = 0;
     AppendBufs ab{};
     int32_t *bu = nullptr, *bv = nullptr;  // host-API batch staging
@@ -48,6 +49,8 @@ struct dbc_ctx {
     int32_t *next_slot = nullptr;
     unsigned long long *stats = nullptr;
     int32_t *err = nullptr;
+    unsigned long long *root_prof = nullptr;  // [k_loc][4], filled when profiling is on
+    bool prof_on = false;
 
     std::vector<void *> allocs;
     int64_t bytes = 0;
@@ -196,8 +199,10 @@ static GView view_of(const dbc_ctx *c) {
     GView g;
     g.rp = c->rp[c->cur];
     g.col = c->col[c->cur];
+    g.scol = c->scol[c->cur];
     g.xinfo = c->ab.xinfo;
     g.xtag = c->ab.xtag;
+    g.xnbr = c->ab.gnbr;
     return g;
 }
 
@@ -293,7 +298,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     c->ev_ok = true;
 
     // workers: persistent CTAs; bounded by roots and by a scratch-memory budget
-    const size_t per_worker = (size_t)n * (4 + 8 + 8 + 4 + 4 + 8 + 4 + 4 + 4 + 4 + 4) + (size_t)(n + 2) * 4 + 64;
+    const size_t per_worker = (size_t)n * (4 + 8 + 8 + 4 + 4 + 8 + 4 + 4 + 4 + 4 + 8) + (size_t)(n + 2) * 4 + 64;
     size_t free_b = 0, total_b = 0;
     cudaMemGetInfo(&free_b, &total_b);
     const size_t state_b = (size_t)c->k_loc * n * 20 + (size_t)c->col_cap * 8 + (size_t)n * 40;
@@ -314,6 +319,8 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->rp[1], (size_t)n + 1);
     AL(c->col[0], (size_t)c->col_cap);
     AL(c->col[1], (size_t)c->col_cap);
+    AL(c->scol[0], (size_t)c->col_cap);
+    AL(c->scol[1], (size_t)c->col_cap);
     const size_t e2 = (size_t)2 * c->edge_cap;
     AL(c->ab.slot, e2);
     AL(c->ab.xtag, e2);
@@ -343,17 +350,34 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->ws.U1, wn);
     AL(c->ws.Rv, wn);
     AL(c->ws.Rl, wn);
-    AL(c->ws.Bq, wn);
+    AL(c->ws.Bq, 2 * wn);
     AL(c->ws.wepoch, (size_t)c->workers);
     AL(c->next_slot, 1);
     AL(c->stats, (size_t)kStCount);
     AL(c->err, 1);
+    AL(c->root_prof, (size_t)4 * std::max(c->k_loc, 1));
 #undef AL
 
     // upload CSR (int32 offsets), roots; zero scratch
     {
         std::vector<int32_t> rp32((size_t)n + 1);
         for (int32_t v = 0; v <= n; ++v) rp32[v] = (int32_t)row_ptr[v];
+        std::vector<int32_t> srt(col, col + c->nnz0);
+        {
+            unsigned nt = std::max(1u, std::min(32u, std::thread::hardware_concurrency()));
+            std::vector<std::thread> th;
+            for (unsigned t = 0; t < nt; ++t)
+                th.emplace_back([&, t] {
+                    for (int64_t v = t; v < n; v += nt)
+                        std::sort(srt.begin() + row_ptr[v], srt.begin() + row_ptr[v + 1]);
+                });
+            for (auto &x : th) x.join();
+        }
+        if (c->nnz0 && cudaMemcpy(c->scol[0], srt.data(), sizeof(int32_t) * c->nnz0,
+                                  cudaMemcpyHostToDevice) != cudaSuccess) {
+            fail(c, DBC_ECUDA, "upload failed: %s", cudaGetErrorString(cudaGetLastError()));
+            return bail(DBC_ECUDA);
+        }
         if (cudaMemcpy(c->rp[0], rp32.data(), sizeof(int32_t) * (n + 1), cudaMemcpyHostToDevice) != cudaSuccess ||
             (c->nnz0 && cudaMemcpy(c->col[0], col, sizeof(int32_t) * c->nnz0, cudaMemcpyHostToDevice) != cudaSuccess) ||
             (c->k_loc && cudaMemcpy(c->roots_d, c->roots_local.data(), sizeof(int32_t) * c->k_loc,
@@ -463,8 +487,8 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
         return DBC_OK;
     }
     const int nb = 1 - c->cur;
-    launches += append_batch(c->ab, c->rp[c->cur], c->col[c->cur], c->rp[nb], c->col[nb], c->n,
-                             c->stream);
+    launches += append_batch(c->ab, c->rp[c->cur], c->col[c->cur], c->scol[c->cur], c->rp[nb],
+                             c->col[nb], c->scol[nb], c->n, c->stream);
     CK(cudaGetLastError());
     c->cur = nb;
     c->nnz += 2 * cnt;
@@ -490,6 +514,7 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     a.next_slot = c->next_slot;
     a.stats = c->stats;
     a.err = c->err;
+    a.root_prof = c->prof_on ? c->root_prof : nullptr;
     if (tm) CK(cudaEventRecord(c->ev[2], c->stream));
     int ulaunch = 0;
     if (c->workers) {
@@ -637,6 +662,27 @@ extern "C" dbc_status dbc_get_timings(dbc_ctx *c, dbc_timings *t) {
     c->tm.static_alg_bytes = (int64_t)h[kStStaticBytes];
     c->tm.alg_bytes_total = (int64_t)(h[kStBytes] - c->bytes_base);
     *t = c->tm;
+    return DBC_OK;
+}
+
+extern "C" dbc_status dbc_debug_counters(dbc_ctx *c, int64_t *out, int32_t count) {
+    if (!c || !out || count < 0) return DBC_EINVAL;
+    CK(cudaSetDevice(c->device));
+    unsigned long long h[kStCount];
+    TRY(read_stats(c, h));
+    for (int i = 0; i < count && i < kStCount; ++i) out[i] = (int64_t)h[i];
+    return DBC_OK;
+}
+
+extern "C" dbc_status dbc_debug_root_profile(dbc_ctx *c, int32_t enable, int64_t *out) {
+    if (!c) return DBC_EINVAL;
+    CK(cudaSetDevice(c->device));
+    c->prof_on = enable != 0;
+    if (out) {
+        CK(cudaMemcpyAsync(out, c->root_prof, sizeof(int64_t) * 4 * c->k_loc, cudaMemcpyDeviceToHost,
+                           c->stream));
+        CK(cudaStreamSynchronize(c->stream));
+    }
     return DBC_OK;
 }
 

@@ -35,14 +35,19 @@ enum ErrBits : int { kErrNumeric = 1, kErrOverflow = 2 };
 // Counters accumulated by the kernels (device, u64).
 enum StatIdx : int {
     kStCase1 = 0, kStCase2, kStCase3, kStTouched, kStDown, kStScanned, kStBytes,
-    kStStaticBytes, kStCount
+    kStStaticBytes,
+    kStPhase0,  // 6 counters: entries scanned by down / removal / D-pull / D-push / up@2 / up@>=3
+    kStTime0 = kStPhase0 + 6,  // 10 timers (ns, thread 0): down, removal, up-setup, up-rest, -, up-end, up-prep, up-scan, up-pull, up-push
+    kStCount = kStTime0 + 10
 };
 
 struct GView {
     const int32_t *__restrict__ rp;
-    const int32_t *__restrict__ col;
+    const int32_t *__restrict__ col;   // rows in canonical order
+    const int32_t *__restrict__ scol;  // the same rows sorted by neighbour id
     const int2 *__restrict__ xinfo;
     const int32_t *__restrict__ xtag;
+    const int32_t *__restrict__ xnbr;  // neighbour of each batch entry (parallel to xtag)
 };
 
 // Scratch of the persistent workers (one CTA = one worker), each array
@@ -57,19 +62,25 @@ struct Scratch {
     int32_t *Doff;             // level offsets of D (also static level offsets), n+2
     int32_t *U0, *U1;          // up frontier ping-pong
     int32_t *Rv, *Rl;          // removal-push targets and their levels (Case 3)
-    int32_t *Bq;               // big-row queue of the current level (2 ends)
+    int32_t *Bq;               // big-row queues of the current level, 2n per worker
     uint32_t *wepoch;          // per-worker epoch counter
 };
 
 // ---------------------------------------------------------------------------
-// loads: immutable graph via the read-only path, mutable state via L2 (.cg) so
-// values written by atomics of the same kernel are never served stale from L1.
+// loads: the immutable graph through the read-only path; mutable state with
+// plain (L1-cacheable) loads.  A worker CTA is the only writer of its root's
+// arrays and of its scratch during a launch, every cross-thread dependency is
+// ordered by __syncthreads() -- which makes all earlier global writes and
+// atomics of the block visible to it -- and the same-level races the
+// algorithm tolerates (lowering, claims) are resolved by atomics, so a stale
+// line can only cost a redundant atomic, never a wrong value.  L1 is
+// invalidated between launches.
 __device__ __forceinline__ int ldg_i(const int32_t *p) { return __ldg(p); }
-__device__ __forceinline__ int ldcg_i(const int32_t *p) { return __ldcg(p); }
-__device__ __forceinline__ double ldcg_d(const double *p) { return __ldcg(p); }
-__device__ __forceinline__ double2 ldcg_d2(const double2 *p) { return __ldcg(p); }
-__device__ __forceinline__ uint32_t ldcg_u(const uint32_t *p) { return __ldcg(p); }
-__device__ __forceinline__ unsigned long long ldcg_ull(const unsigned long long *p) { return __ldcg(p); }
+__device__ __forceinline__ int ldcg_i(const int32_t *p) { return *p; }
+__device__ __forceinline__ double ldcg_d(const double *p) { return *p; }
+__device__ __forceinline__ double2 ldcg_d2(const double2 *p) { return *p; }
+__device__ __forceinline__ uint32_t ldcg_u(const uint32_t *p) { return *p; }
+__device__ __forceinline__ unsigned long long ldcg_ull(const unsigned long long *p) { return *p; }
 
 // Adjacency row of v, restricted to batch entries with insertion index <= limit
 // (canonical order: base row, then inserted neighbours in insertion order).
@@ -84,6 +95,159 @@ __device__ __forceinline__ int2 row_of(const GView &g, int v, int limit) {
         re -= xi.y - vis;
     }
     return make_int2(rb, re);
+}
+
+// Is p a neighbour of x in the graph as of insertion `limit`?  Binary search in
+// x's sorted row (all entries), then a batch-entry visibility check.
+__device__ __forceinline__ bool adjacent_visible(const GView &g, int x, int p, int limit) {
+    const int rb = ldg_i(g.rp + x);
+    int lo = rb & kMask, hi = (ldg_i(g.rp + x + 1) & kMask) - 1;
+    bool found = false;
+    while (lo <= hi) {
+        const int mid = (lo + hi) >> 1;
+        const int q = ldg_i(g.scol + mid);
+        if (q == p) {
+            found = true;
+            break;
+        }
+        if (q < p) lo = mid + 1; else hi = mid - 1;
+    }
+    if (!found) return false;
+    if (rb < 0) {  // x has entries of the current batch: is (x, p) one of them, and visible?
+        const int2 xi = __ldg(g.xinfo + x);
+        for (int k = 0; k < xi.y; ++k)
+            if (ldg_i(g.xnbr + xi.x + k) == p) return ldg_i(g.xtag + xi.x + k) <= limit;
+    }
+    return true;
+}
+
+// ---------------------------------------------------------------------------
+// Chunked flattened level pass (up phase): up to kChunk items per chunk held in
+// shared memory; all of their row entries are spread over the CTA.
+constexpr int kChunk = 512;
+constexpr int kUcap = 1024;  // up-frontier entries kept in shared memory
+constexpr int kMetaUp = 1, kMetaNotPulled = 2;
+constexpr int kFlatU = 4;  // contiguous entries per thread per step
+
+struct ChunkSmem {
+    int v[kChunk];
+    int meta[kChunk];
+    int beg[kChunk];
+    int off[kChunk + 1];
+    double acc[kChunk], c0[kChunk], c1[kChunk], c2[kChunk];
+};
+
+// exclusive scan in place of off[1..cnt] (lengths) -> off[0..cnt]; ends with a barrier
+__device__ __forceinline__ void chunk_scan(int *off, int cnt) {
+    __shared__ int ws[kWarps];
+    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+    constexpr int per = kChunk / kBlock;  // items per thread
+    int vals[per];
+    int run = 0;
+#pragma unroll
+    for (int q = 0; q < per; ++q) {
+        const int i = tid * per + q;
+        vals[q] = (i < cnt) ? off[i + 1] : 0;
+        run += vals[q];
+    }
+    int incl = run;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(kFull, incl, o);
+        if (lane >= o) incl += y;
+    }
+    if (lane == 31) ws[wid] = incl;
+    __syncthreads();
+    int wbase = 0;
+    for (int w = 0; w < wid; ++w) wbase += ws[w];
+    int ex = wbase + incl - run;
+#pragma unroll
+    for (int q = 0; q < per; ++q) {
+        const int i = tid * per + q;
+        ex += vals[q];
+        if (i < cnt) off[i + 1] = ex;
+    }
+    if (tid == 0) off[0] = 0;
+    __syncthreads();
+}
+
+// Flattened entries [0, E) of the chunk's rows (off = exclusive offsets of cnt
+// rows): thread tid takes kFlatU consecutive entries per step (one binary
+// search, then linear advance), gathers column + distance up front, and calls
+// f(t, y, dy); if acc != nullptr the returned contribution is summed into
+// acc[t] (warp-aggregated shared-memory atomics).  Ends with a barrier.
+template <class Col, class F>
+__device__ __forceinline__ void flat_entries(const int *off, int cnt, int E, Col colf,
+                                             const int32_t *dr, double *acc, F f) {
+    const int tid = threadIdx.x, lane = tid & 31;
+    for (int base = 0; base < E; base += kBlock * kFlatU) {
+        const int e0 = base + tid * kFlatU;
+        int t[kFlatU], y[kFlatU], dy[kFlatU];
+        int cur = -1;
+        if (e0 < E) {
+            int lo = 0, hi = cnt - 1;  // last row with off[row] <= e0
+            while (lo < hi) {
+                const int mid = (lo + hi + 1) >> 1;
+                if (off[mid] <= e0) lo = mid; else hi = mid - 1;
+            }
+            cur = lo;
+        }
+#pragma unroll
+        for (int u = 0; u < kFlatU; ++u) {
+            const int e = e0 + u;
+            t[u] = -1;
+            if (e < E) {
+                while (off[cur + 1] <= e) ++cur;
+                t[u] = cur;
+                y[u] = colf(cur, e);
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < kFlatU; ++u)
+            if (t[u] >= 0) dy[u] = ldcg_i(dr + y[u]);
+#pragma unroll
+        for (int u = 0; u < kFlatU; ++u) {
+            double c = 0.0;
+            if (t[u] >= 0) c = f(t[u], y[u], dy[u]);
+            if (acc) {
+                const int t0 = __shfl_sync(kFull, t[u], 0);
+                const bool uni = __all_sync(kFull, t[u] == t0 || t[u] < 0);
+                if (uni) {
+                    if (t0 >= 0) {
+#pragma unroll
+                        for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(kFull, c, o);
+                        if (lane == 0 && c != 0.0) atomicAdd(acc + t0, c);
+                    }
+                } else if (c != 0.0) {
+                    atomicAdd(acc + t[u], c);
+                }
+            }
+        }
+    }
+    __syncthreads();
+}
+
+// Sequential walk of one (small) row in canonical order with kRowUnroll entries
+// in flight: column, distance and -- for entries passing want(dy) -- the
+// (sigma, delta) pair are gathered up front, then f(y, dy, sd) runs in order.
+constexpr int kRowUnroll = 8;
+template <class Want, class F>
+__device__ __forceinline__ void row_walk(const GView &g, const int32_t *dr, const double2 *sdr,
+                                         int2 r, Want want, F f) {
+    for (int j = r.x; j < r.y; j += kRowUnroll) {
+        int y[kRowUnroll], dy[kRowUnroll];
+        double2 sv[kRowUnroll];
+#pragma unroll
+        for (int u = 0; u < kRowUnroll; ++u) y[u] = (j + u < r.y) ? ldg_i(g.col + j + u) : -1;
+#pragma unroll
+        for (int u = 0; u < kRowUnroll; ++u) dy[u] = (y[u] >= 0) ? ldcg_i(dr + y[u]) : kInf;
+#pragma unroll
+        for (int u = 0; u < kRowUnroll; ++u)
+            sv[u] = (y[u] >= 0 && want(dy[u])) ? ldcg_d2(sdr + y[u]) : make_double2(0.0, 0.0);
+#pragma unroll
+        for (int u = 0; u < kRowUnroll; ++u)
+            if (y[u] >= 0) f(y[u], dy[u], sv[u]);
+    }
 }
 
 template <int G>
@@ -119,6 +283,7 @@ using G32 = std::integral_constant<int, 32>;
 
 constexpr int kBig = 128;     // big rows per round
 constexpr int kUnroll = 4;    // entries per thread in flight
+constexpr int kAdjCap = 512;  // longest root row kept in shared memory (level-2 shortcut)
 
 struct BigSmem {
     int idx[kBig];    // item index (caller's list) of each big row
@@ -144,7 +309,7 @@ __device__ __forceinline__ void split_pass(int count, const GView &g, int limit,
         int2 r = make_int2(0, 0);
         if (need_row(idx, v)) r = row_of(g, v, limit);
         if (r.y - r.x > kSmallDeg) {
-            enqueue(idx);
+            enqueue(idx, v, r);
         } else {
             small(idx, v, r);
         }
@@ -261,6 +426,7 @@ struct UpdateArgs {
     int32_t *next_slot;            // work counter (zeroed before launch)
     unsigned long long *stats;     // kStCount counters
     int32_t *err;
+    unsigned long long *root_prof; // nullable: per local slot {t_begin, t_end, jobs, touched}
 };
 
 struct StaticArgs {

@@ -176,6 +176,41 @@ __global__ void k_copy_rows(const int32_t *rp_old, const int32_t *col_old, const
     }
 }
 
+// warp per vertex: the sorted copy of each row -- old sorted row merged with
+// the batch group (both sides locate their slot by counting the other side)
+__global__ void k_copy_rows_sorted(const int32_t *rp_old, const int32_t *scol_old,
+                                   const int32_t *rp_new, int32_t *scol_new, const int32_t *xcnt,
+                                   const int32_t *xoff, const int32_t *gnbr, int32_t n) {
+    const int lane = threadIdx.x & 31;
+    const int64_t warps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t x = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; x < n; x += warps) {
+        const int ob = rp_old[x] & kMask, oe = rp_old[x + 1] & kMask, nb = rp_new[x];
+        const int c = xcnt[x];
+        if (c == 0) {
+            for (int j = lane; j < oe - ob; j += 32) scol_new[nb + j] = scol_old[ob + j];
+            continue;
+        }
+        const int g0 = xoff[x];
+        for (int j = lane; j < oe - ob; j += 32) {
+            const int val = scol_old[ob + j];
+            int less = 0;
+            for (int k = 0; k < c; ++k) less += gnbr[g0 + k] < val;
+            scol_new[nb + j + less] = val;
+        }
+        for (int k = lane; k < c; k += 32) {
+            const int val = gnbr[g0 + k];
+            int lo = 0, hi = oe - ob;  // old entries < val
+            while (lo < hi) {
+                const int mid = (lo + hi) >> 1;
+                if (scol_old[ob + mid] < val) lo = mid + 1; else hi = mid;
+            }
+            int less = 0;
+            for (int q = 0; q < c; ++q) less += gnbr[g0 + q] < val;
+            scol_new[nb + lo + less] = val;
+        }
+    }
+}
+
 __global__ void k_flag_rows(const int32_t *xcnt, int32_t n, int32_t *rp_new) {
     const int64_t x = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (x < n && xcnt[x]) rp_new[x] |= (int32_t)0x80000000u;
@@ -214,15 +249,18 @@ int validate_batch(const AppendBufs &B, const GView &g, const int32_t *rp_old, i
     return launches;
 }
 
-int append_batch(const AppendBufs &B, const int32_t *rp_old, const int32_t *col_old, int32_t *rp_new,
-                 int32_t *col_new, int32_t n, cudaStream_t s) {
+int append_batch(const AppendBufs &B, const int32_t *rp_old, const int32_t *col_old,
+                 const int32_t *scol_old, int32_t *rp_new, int32_t *col_new, int32_t *scol_new,
+                 int32_t n, cudaStream_t s) {
     int launches = 0;
     k_degrees<<<blocks_for((int64_t)n + 1, 256), 256, 0, s>>>(rp_old, B.xcnt, n, B.deg);
     launches += 1 + scan_launch(B.deg, rp_new, (int64_t)n + 1, B.sums, s);
     k_copy_rows<<<std::min<int64_t>(blocks_for((int64_t)n * 32, 256), 148 * 16), 256, 0, s>>>(
         rp_old, col_old, rp_new, col_new, B.xcnt, B.xoff, B.gnbr, n);
+    k_copy_rows_sorted<<<std::min<int64_t>(blocks_for((int64_t)n * 32, 256), 148 * 16), 256, 0, s>>>(
+        rp_old, scol_old, rp_new, scol_new, B.xcnt, B.xoff, B.gnbr, n);
     k_flag_rows<<<blocks_for(n, 256), 256, 0, s>>>(B.xcnt, n, rp_new);
-    return launches + 2;
+    return launches + 3;
 }
 
 // BC partial rebased as the column sum of delta over local slots (DBC_FLAG_EXACT_BC)

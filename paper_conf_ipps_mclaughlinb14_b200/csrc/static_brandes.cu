@@ -26,10 +26,10 @@ __global__ void __launch_bounds__(kBlock, 2) static_kernel(StaticArgs a) {
     const size_t n = (size_t)a.n;
     int32_t *order = a.ws.Dv + (size_t)w * n;
     int32_t *loff = a.ws.Doff + (size_t)w * (n + 2);
-    int32_t *Bq = a.ws.Bq + (size_t)w * n;
+    int32_t *Bq = a.ws.Bq + (size_t)w * 2 * n;
     const GView &g = a.g;
     unsigned long long bytes = 0;
-    auto enq = [&](int idx) { Bq[atomicAdd(&s_nbig, 1)] = idx; };
+    auto enq = [&](int idx, int, int2) { Bq[atomicAdd(&s_nbig, 1)] = idx; };
     if (tid == 0) s_nbig = 0;
 
     for (;;) {
@@ -65,10 +65,10 @@ __global__ void __launch_bounds__(kBlock, 2) static_kernel(StaticArgs a) {
         // Stage 2: level-synchronous BFS; level L's sigma pull fused with the
         // discovery of level L+1 (one scan of each row).
         int L = 0, lb = 0, le = 1, nl = 1;
-        auto fwd_visit = [&](int x, int dx) -> double {
+        auto fwd_visit = [&](int x, int dx, double2 sv) -> double {
             if (dx == L - 1) {
                 bytes += 8;
-                return ldcg_d2(sdr + x).x;
+                return sv.x;
             }
             if (dx == kInf && atomicCAS(dr + x, kInf, L + 1) == kInf) {
                 order[atomicAdd(&s_tail, 1)] = x;
@@ -90,10 +90,8 @@ __global__ void __launch_bounds__(kBlock, 2) static_kernel(StaticArgs a) {
                 [&](int, int) { return true; },
                 [&](int, int v, int2 r) {
                     double sum = 0.0;  // canonical order
-                    for (int j = r.x; j < r.y; ++j) {
-                        const int x = ldg_i(g.col + j);
-                        sum += fwd_visit(x, ldcg_i(dr + x));
-                    }
+                    row_walk(g, dr, sdr, r, [&](int dx) { return dx == L - 1; },
+                             [&](int x, int dx, double2 sv) { sum += fwd_visit(x, dx, sv); });
                     bytes += 8ull * (r.y - r.x);
                     fwd_finish(v, sum);
                 },
@@ -106,7 +104,8 @@ __global__ void __launch_bounds__(kBlock, 2) static_kernel(StaticArgs a) {
                          g, INT32_MAX);
                 big_entries(S, g, dr, [&](int, int x, int dx) {
                     bytes += 8;
-                    return fwd_visit(x, dx);
+                    const double2 sv = (dx == L - 1) ? ldcg_d2(sdr + x) : make_double2(0.0, 0.0);
+                    return fwd_visit(x, dx, sv);
                 });
                 if (tid < m) {
                     double sum = S.acc[tid];
@@ -141,9 +140,8 @@ __global__ void __launch_bounds__(kBlock, 2) static_kernel(StaticArgs a) {
         // BC partial += delta (Eq. (3)), root excluded (delta_s(s) = 0).
         for (int lev = nl - 2; lev >= 1; --lev) {
             const int b0 = loff[lev], b1 = loff[lev + 1];
-            auto bwd_visit = [&](double sv, int y, int dy) -> double {
+            auto bwd_visit = [&](double sv, int y, int dy, double2 t) -> double {
                 if (dy != lev + 1) return 0.0;
-                const double2 t = ldcg_d2(sdr + y);
                 bytes += 16;
                 return __dmul_rn(__ddiv_rn(sv, t.x), __dadd_rn(1.0, t.y));
             };
@@ -158,10 +156,8 @@ __global__ void __launch_bounds__(kBlock, 2) static_kernel(StaticArgs a) {
                 [&](int, int v, int2 r) {
                     const double sv = ldcg_d2(sdr + v).x;
                     double acc = 0.0;
-                    for (int j = r.x; j < r.y; ++j) {
-                        const int y = ldg_i(g.col + j);
-                        acc += bwd_visit(sv, y, ldcg_i(dr + y));
-                    }
+                    row_walk(g, dr, sdr, r, [&](int dy) { return dy == lev + 1; },
+                             [&](int y, int dy, double2 t) { acc += bwd_visit(sv, y, dy, t); });
                     bytes += 8ull * (r.y - r.x);
                     bwd_finish(v, acc);
                 },
@@ -176,7 +172,8 @@ __global__ void __launch_bounds__(kBlock, 2) static_kernel(StaticArgs a) {
                 __syncthreads();
                 big_entries(S, g, dr, [&](int t, int y, int dy) {
                     bytes += 8;
-                    return bwd_visit(S.c0[t], y, dy);
+                    const double2 sv = (dy == lev + 1) ? ldcg_d2(sdr + y) : make_double2(0.0, 0.0);
+                    return bwd_visit(S.c0[t], y, dy, sv);
                 });
                 if (tid < m) bwd_finish(S.v[tid], S.acc[tid]);
                 __syncthreads();

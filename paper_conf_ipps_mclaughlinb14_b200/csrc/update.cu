@@ -46,6 +46,14 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
     __shared__ int s_rcnt;   // |R|
     __shared__ int s_rmax;   // deepest removal-push target level
     __shared__ int s_nbig, s_nbig2;      // big-row queue (front: D rows, back: U/R rows)
+    __shared__ int s_nbig3;              // level-2 up rows resolved against adj(root)
+    __shared__ int s_ds;                 // |adj(root)| as of the insertion (-1: too long)
+    __shared__ int s_adjs[kAdjCap];      // adj(root) = the level-1 vertices
+    __shared__ int s_adjdeg[kAdjCap];    // their degrees
+    __shared__ ChunkSmem I;              // items of the current up-phase chunk
+    __shared__ int s_l1[kChunk];         // chunk slots resolved against adj(root)
+    __shared__ int s_nl1;
+    __shared__ int s_un[2][kUcap];       // up frontier ping-pong (overflow: Ua / Ub)
     __shared__ uint32_t s_work[kWarps];  // window classification bits (1 = Case 2/3)
     __shared__ int s_job[4];             // uh, ul, L0, case3 of the current job
     __shared__ BigSmem S;
@@ -67,20 +75,34 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
     int32_t *Ub = a.ws.U1 + (size_t)wk * n;
     int32_t *Rv = a.ws.Rv + (size_t)wk * n;
     int32_t *Rl = a.ws.Rl + (size_t)wk * n;
-    int32_t *Bq = a.ws.Bq + (size_t)wk * n;
+    int32_t *Bq = a.ws.Bq + (size_t)wk * 2 * n;
     uint32_t epoch = a.ws.wepoch[wk];
     const GView &g = a.g;
 
-    unsigned long long st_bytes = 0, st_scanned = 0, st_touched = 0, st_down = 0;
+    unsigned long long st_bytes = 0, st_touched = 0, st_down = 0;
+    unsigned long long sc_down = 0, sc_rem = 0, sc_dpull = 0, sc_dpush = 0, sc_up2 = 0, sc_up3 = 0;
     unsigned long long st_c1 = 0, st_c2 = 0, st_c3 = 0;
+    // per-phase wall time seen by thread 0 (diagnostic): down, removal, up-split, up-big, up-L1, up-level-end
+    unsigned long long tm_ph[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
+    unsigned long long tclk = 0;
+    auto tick = [&](int ph) {
+        if (tid == 0) {
+            unsigned long long t;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+            if (ph >= 0) tm_ph[ph] += t - tclk;
+            tclk = t;
+        }
+    };
 
-    auto enq_front = [&](int idx) { Bq[atomicAdd(&s_nbig, 1)] = idx; };
+    auto enq_front = [&](int idx, int, int2) { Bq[atomicAdd(&s_nbig, 1)] = idx; };
     auto enq_back = [&](int idx) { Bq[n - 1 - atomicAdd(&s_nbig2, 1)] = idx; };
+    auto enq_l1 = [&](int idx) { Bq[n + atomicAdd(&s_nbig3, 1)] = idx; };
     auto fetch_front = [&](int r0) { return [=](int t) { return Bq[r0 + t]; }; };
 
     if (tid == 0) {
         s_nbig = 0;
         s_nbig2 = 0;
+        s_nbig3 = 0;
     }
 
     for (;;) {
@@ -91,6 +113,9 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
         if (slot >= a.k_loc) break;
         int32_t *dr = a.d + (size_t)slot * n;
         double2 *sdr = a.sd + (size_t)slot * n;
+        const int sroot = a.roots[slot];
+        unsigned long long prof_t0 = 0, prof_jobs = 0, prof_touch0 = st_touched;
+        if (a.root_prof && tid == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(prof_t0));
 
         // Insertions are walked in order.  Classification (K2) of a window of
         // kBlock insertions runs in parallel against the current d; a Case-2
@@ -122,6 +147,7 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                 }
                 // ---------------- classify + seed (tid 0, broadcast) ----------------
                 ++epoch;
+                ++prof_jobs;
                 const uint32_t E = epoch << 2;
                 const uint32_t mD = E | kDown, mU = E | kUp;
                 if (tid == 0) {
@@ -159,6 +185,7 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                 const bool case3 = s_job[3] != 0;
                 const int lim = p;  // graph as of this insertion (edge p included)
 
+                tick(-1);
                 // ================= down phase (K3) =================
                 int L = L0, lb = 0, le = 1, nlev = 1;
                 // per-D-entry epilogue: record old d / sigma, store the new sigma
@@ -172,10 +199,10 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                     st_bytes += 8 + 8 + 20;
                 };
                 // one neighbour y of a level-L vertex; returns sigma[y] if y is a predecessor
-                auto down_visit = [&](int y, int dy) -> double {
+                auto down_visit = [&](int y, int dy, double2 sv) -> double {
                     if (dy == L - 1) {
                         st_bytes += 8;
-                        return ldcg_d2(sdr + y).x;
+                        return sv.x;
                     }
                     if (dy > L + 1) {  // Case 3 pull-up
                         const int old = atomicMin(dr + y, L + 1);
@@ -195,12 +222,10 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                         [&](int, int) { return true; },
                         [&](int i, int w, int2 r) {
                             double sum = 0.0;  // canonical order: bit-exact
-                            for (int j = r.x; j < r.y; ++j) {
-                                const int y = ldg_i(g.col + j);
-                                sum += down_visit(y, ldcg_i(dr + y));
-                            }
+                            row_walk(g, dr, sdr, r, [&](int dy) { return dy == L - 1; },
+                                     [&](int y, int dy, double2 sv) { sum += down_visit(y, dy, sv); });
                             st_bytes += 8 + 8ull * (r.y - r.x);
-                            st_scanned += r.y - r.x;
+                            sc_down += r.y - r.x;
                             down_finish(lb + i, w, sum);
                         },
                         enq_front);
@@ -211,8 +236,9 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                         big_load(S, m, fetch_front(r0), [&](int i) { return Dv[lb + i]; }, g, lim);
                         big_entries(S, g, dr, [&](int, int y, int dy) {
                             st_bytes += 8;
-                            st_scanned++;
-                            return down_visit(y, dy);
+                            sc_down++;
+                            const double2 sv = (dy == L - 1) ? ldcg_d2(sdr + y) : make_double2(0.0, 0.0);
+                            return down_visit(y, dy, sv);
                         });
                         if (tid < m) {
                             double sum = S.acc[tid];
@@ -252,13 +278,15 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                 }
                 __syncthreads();
 
+                tick(0);
                 // ================= (0) Case-3 removal pushes =================
                 if (case3) {
                     // a pulled-up w (finite old level od) loses its old predecessors x
-                    auto rem_visit = [&](int w, int od, double osig, double coef, int x, int dx) {
+                    auto rem_visit = [&](int w, int od, double osig, double coef, int x, int dx,
+                                         double2 sv) {
                         if (dx != od - 1 || (x == uh && w == ul)) return;
                         if (ldcg_u(mark + x) == mD) return;
-                        const double sx = ldcg_d2(sdr + x).x;
+                        const double sx = sv.x;
                         atomicAdd(dacc + x, -__dmul_rn(__ddiv_rn(sx, osig), coef));
                         st_bytes += 24;
                         if (atomicMax(mark + x, mU) < E) {
@@ -280,12 +308,10 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                             const int od = Dold[i];
                             const double osig = Dsig[i];
                             const double coef = 1.0 + ldcg_d2(sdr + w).y;  // delta still old
-                            for (int j = r.x; j < r.y; ++j) {
-                                const int x = ldg_i(g.col + j);
-                                rem_visit(w, od, osig, coef, x, ldcg_i(dr + x));
-                            }
+                            row_walk(g, dr, sdr, r, [&](int dx) { return dx == od - 1; },
+                                     [&](int x, int dx, double2 sv) { rem_visit(w, od, osig, coef, x, dx, sv); });
                             st_bytes += 16 + 8ull * (r.y - r.x);
-                            st_scanned += r.y - r.x;
+                            sc_rem += r.y - r.x;
                         },
                         enq_front);
                     __syncthreads();
@@ -303,8 +329,9 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                         __syncthreads();
                         big_entries(S, g, dr, [&](int t, int x, int dx) {
                             st_bytes += 8;
-                            st_scanned++;
-                            rem_visit(S.v[t], s_f0[t], S.c0[t], S.c1[t], x, dx);
+                            sc_rem++;
+                            const double2 sv = (dx == s_f0[t] - 1) ? ldcg_d2(sdr + x) : make_double2(0.0, 0.0);
+                            rem_visit(S.v[t], s_f0[t], S.c0[t], S.c1[t], x, dx, sv);
                             return 0.0;
                         });
                     }
@@ -316,60 +343,56 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                 const int Lmax = max(LmaxD, s_rmax);
                 if (tid == 0) st_touched += rcnt;
 
+                tick(1);
                 // ================= up phase (K4 + Alg. 8) =================
-                int *Ucur = Ua, *Unext = Ub;
+                int *Ucur = Ua, *Unext = Ub;  // overflow beyond kUcap entries
+                int ucur_sel = 0;
                 int ucnt = 0;
                 for (int l = Lmax; l >= 1; --l) {
                     if (l < L0 && ucnt == 0) break;  // nothing left above the insertion
                     const bool push = l >= 2;          // level-1 vertices only feed the root
-                    auto claim_up = [&](int y) {
-                        if (atomicMax(mark + y, mU) < E) Unext[atomicAdd(&s_ucnt, 1)] = y;
+                    // queue p for level l-1 unless already queued (plain flag store; a
+                    // rare duplicate from a race is dropped when the list is processed)
+                    auto claim_up = [&](int y, uint32_t my) {
+                        if (my >= E) return;
+                        mark[y] = mU;
+                        const int pos = atomicAdd(&s_ucnt, 1);
+                        if (pos < kUcap)
+                            s_un[ucur_sel ^ 1][pos] = y;
+                        else
+                            Unext[pos - kUcap] = y;
                     };
                     // up vertex x (not in D): push sigma[p]/sigma[x] * Ddelta[x] upwards
-                    auto up_visit = [&](double gx, double sx, int pp, int dp) {
+                    auto up_visit = [&](double gx, double sx, int pp, int dp, double2 sv, uint32_t mp) {
                         if (dp != l - 1) return;
-                        const double sp = ldcg_d2(sdr + pp).x;
+                        const double sp = sv.x;
                         atomicAdd(dacc + pp, __dmul_rn(__ddiv_rn(sp, sx), gx));
                         st_bytes += 24;
-                        claim_up(pp);
+                        claim_up(pp, mp);
                     };
-                    auto up_finish = [&](int x, double gx) {
+                    auto up_finish = [&](int x, double gx, double odel) {
                         dacc[x] = 0.0;
-                        sdr[x].y = ldcg_d2(sdr + x).y + gx;
+                        sdr[x].y = odel + gx;
                         atomicAdd(a.bc + x, gx);
                         st_bytes += 8 + 8 + 16 + 16;
                     };
-                    auto up_small = [&](int, int x, int2 r) {
-                        const double gx = ldcg_d(dacc + x);
-                        if (gx != 0.0 && r.y > r.x) {
-                            const double sx = ldcg_d2(sdr + x).x;
-                            for (int j = r.x; j < r.y; ++j) {
-                                const int pp = ldg_i(g.col + j);
-                                up_visit(gx, sx, pp, ldcg_i(dr + pp));
-                            }
-                            st_bytes += 16 + 8ull * (r.y - r.x);
-                            st_scanned += r.y - r.x;
-                        }
-                        up_finish(x, gx);
-                    };
                     // down vertex x: pull delta (Eq. (2)), then push new-minus-old contributions
-                    auto dpull_visit = [&](double sx, int y, int dy) -> double {
+                    auto dpull_visit = [&](double sx, int y, int dy, double2 t) -> double {
                         if (dy != l + 1) return 0.0;
-                        const double2 t = ldcg_d2(sdr + y);
                         st_bytes += 16;
                         return __dmul_rn(__ddiv_rn(sx, t.x), __dadd_rn(1.0, t.y));
                     };
                     auto dpush_visit = [&](int x, double sx, double dn, double odel, double osig,
-                                           bool not_pulled, int pp, int dp) {
+                                           bool not_pulled, int pp, int dp, double2 sv, uint32_t mp) {
                         if (dp != l - 1) return;
-                        if (ldcg_u(mark + pp) == mD) return;
-                        const double sp = ldcg_d2(sdr + pp).x;
+                        if (mp == mD) return;
+                        const double sp = sv.x;
                         double dlt = __dmul_rn(__ddiv_rn(sp, sx), 1.0 + dn);
                         if (not_pulled && !(pp == uh && x == ul))
                             dlt = __dsub_rn(dlt, __dmul_rn(__ddiv_rn(sp, osig), 1.0 + odel));
                         atomicAdd(dacc + pp, dlt);
                         st_bytes += 24;
-                        claim_up(pp);
+                        claim_up(pp, mp);
                     };
                     auto d_finish = [&](int x, double dn, double odel) {
                         sdr[x].y = dn;
@@ -382,114 +405,165 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                         b0 = Doff[l - L0];
                         b1 = Doff[l - L0 + 1];
                     }
-                    // --- small rows of the three sources; big rows queued ---
-                    split_pass(
-                        b1 - b0, g, lim, [&](int i, int &x) { x = Dv[b0 + i]; return true; },
-                        [&](int, int) { return true; },
-                        [&](int i, int x, int2 r) {
-                            const double2 s2 = ldcg_d2(sdr + x);
-                            double dn = 0.0;
-                            for (int j = r.x; j < r.y; ++j) {
-                                const int y = ldg_i(g.col + j);
-                                dn += dpull_visit(s2.x, y, ldcg_i(dr + y));
+                    const int nDl = b1 - b0;
+                    if (l == 2) {  // level-1 set = the root's row as of this insertion
+                        if (tid == 0) {
+                            const int2 rr = row_of(g, sroot, lim);
+                            s_ds = (rr.y - rr.x <= kAdjCap) ? rr.y - rr.x : -1;
+                        }
+                        __syncthreads();
+                        if (s_ds > 0) {
+                            const int2 rr = row_of(g, sroot, lim);
+                            for (int j = tid; j < s_ds; j += kBlock) {
+                                const int pj = ldg_i(g.col + rr.x + j);
+                                s_adjs[j] = pj;
+                                s_adjdeg[j] = (ldg_i(g.rp + pj + 1) & kMask) - (ldg_i(g.rp + pj) & kMask);
                             }
-                            st_scanned += r.y - r.x;
-                            st_bytes += 16 + 8ull * (r.y - r.x);
-                            if (push) {
-                                const int idx = b0 + i;
-                                const bool np = Dold[idx] == l;
-                                const double osig = Dsig[idx];
-                                for (int j = r.x; j < r.y; ++j) {
-                                    const int pp = ldg_i(g.col + j);
-                                    dpush_visit(x, s2.x, dn, s2.y, osig, np, pp, ldcg_i(dr + pp));
+                        }
+                        __syncthreads();
+                    }
+                    tick(2);
+                    // One flattened pass per chunk of the level's items: the down
+                    // segment first, then the up frontier, then removal targets.
+                    const int total = nDl + ucnt + rcnt;
+                    for (int base = 0; base < total; base += kChunk) {
+                        const int cnt = min(kChunk, total - base);
+                        const int nDc = max(0, min(cnt, nDl - base));
+                        if (tid == 0) s_nl1 = 0;
+                        __syncthreads();
+                        // --- A: per-item prep (independent loads) ---
+                        for (int t = tid; t < cnt; t += kBlock) {
+                            const int q = base + t;
+                            int x = -1, meta = 0, beg = 0, len = 0;
+                            double c0 = 0.0, c1 = 0.0, c2 = 0.0;
+                            if (q < nDl) {
+                                const int idx = b0 + q;
+                                x = Dv[idx];
+                                const double2 s2 = ldcg_d2(sdr + x);
+                                c0 = s2.x;  // sigma (new)
+                                c1 = s2.y;  // delta (old)
+                                c2 = Dsig[idx];
+                                meta = (Dold[idx] == l) ? kMetaNotPulled : 0;
+                                const int2 r = row_of(g, x, lim);
+                                beg = r.x;
+                                len = r.y - r.x;
+                                st_bytes += 8 + 16 + 8 + 4;
+                            } else {
+                                const int qi = q - nDl;
+                                if (qi < ucnt) {
+                                    x = (qi < kUcap) ? s_un[ucur_sel][qi] : Ucur[qi - kUcap];
+                                } else if (Rl[qi - ucnt] == l) {
+                                    x = Rv[qi - ucnt];
                                 }
-                                st_scanned += r.y - r.x;
-                                st_bytes += 16 + 8ull * (r.y - r.x);
+                                // first claimant processes the vertex (drops duplicates)
+                                if (x >= 0 && atomicMax(mark + x, E | 3u) != mU) x = -1;
+                                if (x >= 0) {
+                                    meta = kMetaUp;
+                                    c1 = ldcg_d(dacc + x);  // Ddelta (complete: level l+1 is done)
+                                    const double2 s2 = ldcg_d2(sdr + x);
+                                    c0 = s2.x;
+                                    c2 = s2.y;
+                                    st_bytes += 24;
+                                    if (push && c1 != 0.0) {
+                                        const int2 r = row_of(g, x, lim);
+                                        beg = r.x;
+                                        len = r.y - r.x;
+                                        st_bytes += 8;
+                                        // level 2: resolve against adj(root) when cheaper
+                                        if (l == 2 && len > kSmallDeg && s_ds >= 0 &&
+                                            s_ds * (33 - __clz(len)) < len) {
+                                            s_l1[atomicAdd(&s_nl1, 1)] = t;
+                                            len = 0;
+                                        }
+                                    }
+                                }
                             }
-                            d_finish(x, dn, s2.y);
-                        },
-                        enq_front);
-                    split_pass(
-                        ucnt, g, lim, [&](int i, int &x) { x = Ucur[i]; return true; },
-                        [&](int, int) { return push; }, up_small, enq_back);
-                    if (rcnt)
-                        split_pass(
-                            rcnt, g, lim,
-                            [&](int i, int &x) {
-                                x = Rv[i];
-                                return Rl[i] == l;
-                            },
-                            [&](int, int) { return push; }, up_small,
-                            [&](int idx) { enq_back(idx | kSrcR); });
-                    __syncthreads();
-                    const int nD = s_nbig, nU = s_nbig2;
-                    // --- big down rows: pull pass, push pass, epilogue ---
-                    for (int r0 = 0; r0 < nD; r0 += kBig) {
-                        const int m = min(kBig, nD - r0);
-                        big_load(S, m, fetch_front(r0), [&](int i) { return Dv[b0 + i]; }, g, lim);
-                        if (tid < m) {
-                            const int idx = b0 + S.idx[tid];
-                            const double2 s2 = ldcg_d2(sdr + S.v[tid]);
-                            S.c0[tid] = s2.x;
-                            S.c1[tid] = s2.y;
-                            s_c2[tid] = Dsig[idx];
-                            s_f0[tid] = Dold[idx] == l;
-                            st_bytes += 16 + 16;
+                            I.v[t] = x;
+                            I.meta[t] = meta;
+                            I.beg[t] = beg;
+                            I.off[t + 1] = len;
+                            I.acc[t] = 0.0;
+                            I.c0[t] = c0;
+                            I.c1[t] = c1;
+                            I.c2[t] = c2;
                         }
                         __syncthreads();
-                        big_entries(S, g, dr, [&](int t, int y, int dy) {
-                            st_bytes += 8;
-                            st_scanned++;
-                            return dpull_visit(S.c0[t], y, dy);
-                        });
-                        if (push)
-                            big_entries(S, g, dr, [&](int t, int pp, int dp) {
-                                st_bytes += 8;
-                                st_scanned++;
-                                dpush_visit(S.v[t], S.c0[t], S.acc[t], S.c1[t], s_c2[t], s_f0[t] != 0,
-                                            pp, dp);
-                                return 0.0;
-                            });
-                        if (tid < m) d_finish(S.v[tid], S.acc[tid], S.c1[tid]);
-                        __syncthreads();
-                    }
-                    // --- big up rows (U and R) ---
-                    for (int r0 = 0; r0 < nU; r0 += kBig) {
-                        const int m = min(kBig, nU - r0);
-                        big_load(
-                            S, m, [&](int t) { return Bq[n - 1 - (r0 + t)]; },
-                            [&](int idx) { return (idx & kSrcR) ? Rv[idx & ~kSrcR] : Ucur[idx]; }, g, lim);
-                        if (tid < m) {
-                            const int x = S.v[tid];
-                            S.c0[tid] = ldcg_d(dacc + x);
-                            S.c1[tid] = ldcg_d2(sdr + x).x;
-                            st_bytes += 16;
+                        tick(6);
+                        chunk_scan(I.off, cnt);  // off[0..cnt], ends with a barrier
+                        tick(7);
+                        // --- C1: delta pull of the down vertices (Eq. (2)) ---
+                        const int E1 = I.off[nDc], E = I.off[cnt];
+                        if (E1 > 0)
+                            flat_entries(I.off, cnt, E1, [&](int t, int e) { return ldg_i(g.col + I.beg[t] + e - I.off[t]); },
+                                         dr, I.acc, [&](int t, int y, int dy) -> double {
+                                             sc_dpull++;
+                                             st_bytes += 8;
+                                             if (dy != l + 1) return 0.0;
+                                             return dpull_visit(I.c0[t], y, dy, ldcg_d2(sdr + y));
+                                         });
+                        tick(8);
+                        // --- C2: pushes towards level l-1 (down: new - old, up: sigma ratio * Ddelta) ---
+                        if (push && E > 0)
+                            flat_entries(I.off, cnt, E, [&](int t, int e) { return ldg_i(g.col + I.beg[t] + e - I.off[t]); },
+                                         dr, nullptr, [&](int t, int pp, int dp) -> double {
+                                             (l == 2 ? sc_up2 : sc_up3)++;
+                                             st_bytes += 8;
+                                             if (dp != l - 1) return 0.0;
+                                             const double2 sv = ldcg_d2(sdr + pp);
+                                             const uint32_t mp = ldcg_u(mark + pp);
+                                             const int meta = I.meta[t];
+                                             if (meta & kMetaUp)
+                                                 up_visit(I.c1[t], I.c0[t], pp, dp, sv, mp);
+                                             else
+                                                 dpush_visit(I.v[t], I.c0[t], I.acc[t], I.c1[t], I.c2[t],
+                                                             (meta & kMetaNotPulled) != 0, pp, dp, sv, mp);
+                                             return 0.0;
+                                         });
+                        tick(9);
+                        // --- C3: level-2 rows resolved against adj(root) ---
+                        const int nl1 = s_nl1;
+                        if (nl1 > 0) {
+                            const int ds = s_ds, npairs = nl1 * ds;
+                            for (int qq = tid; qq < npairs; qq += kBlock) {
+                                const int li = qq / ds, j = qq - li * ds;
+                                const int t = s_l1[li];
+                                const int x = I.v[t], pp = s_adjs[j];
+                                const int degx = (ldg_i(g.rp + x + 1) & kMask) - (ldg_i(g.rp + x) & kMask);
+                                const bool adj = (s_adjdeg[j] < degx) ? adjacent_visible(g, pp, x, lim)
+                                                                      : adjacent_visible(g, x, pp, lim);
+                                st_bytes += 32;
+                                if (adj) up_visit(I.c1[t], I.c0[t], pp, 1, ldcg_d2(sdr + pp), ldcg_u(mark + pp));
+                            }
+                            __syncthreads();
+                        }
+                        // --- D: per-item epilogue (Alg. 8 fused) ---
+                        for (int t = tid; t < cnt; t += kBlock) {
+                            const int x = I.v[t];
+                            if (x < 0) continue;
+                            if (I.meta[t] & kMetaUp)
+                                up_finish(x, I.c1[t], I.c2[t]);
+                            else
+                                d_finish(x, I.acc[t], I.c1[t]);
                         }
                         __syncthreads();
-                        big_entries(S, g, dr, [&](int t, int pp, int dp) {
-                            const double gx = S.c0[t];
-                            if (gx != 0.0) {
-                                st_bytes += 8;
-                                st_scanned++;
-                                up_visit(gx, S.c1[t], pp, dp);
-                            }
-                            return 0.0;
-                        });
-                        if (tid < m) up_finish(S.v[tid], S.c0[tid]);
-                        __syncthreads();
                     }
+                    tick(3);
+                    tick(4);
                     ucnt = s_ucnt;
                     __syncthreads();
                     if (tid == 0) {
                         s_ucnt = 0;
                         s_nbig = 0;
                         s_nbig2 = 0;
+                        s_nbig3 = 0;
                         st_touched += ucnt;
                     }
                     int *t = Ucur;
                     Ucur = Unext;
                     Unext = t;
+                    ucur_sel ^= 1;
                     __syncthreads();
+                    tick(5);
                 }
                 // any up vertices left at level 0 would be the root: never produced
                 if (case3) {  // distances changed: re-classify from the next insertion
@@ -500,6 +574,15 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
             ins = p;
             __syncthreads();  // s_work is rewritten by the next window
         }
+        if (a.root_prof && tid == 0) {
+            unsigned long long t1;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t1));
+            unsigned long long *rp4 = a.root_prof + 4 * (size_t)slot;
+            rp4[0] = prof_t0;
+            rp4[1] = t1;
+            rp4[2] = prof_jobs;
+            rp4[3] = st_touched - prof_touch0;
+        }
     }
     if (tid == 0) {
         a.ws.wepoch[wk] = epoch;
@@ -508,8 +591,17 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
         if (st_c3) atomicAdd(a.stats + kStCase3, st_c3);
         if (st_touched) atomicAdd(a.stats + kStTouched, st_touched);
         if (st_down) atomicAdd(a.stats + kStDown, st_down);
+        for (int q = 0; q < 10; ++q)
+            if (tm_ph[q]) atomicAdd(a.stats + kStTime0 + q, tm_ph[q]);
     }
-    if (st_scanned) atomicAdd(a.stats + kStScanned, st_scanned);
+    const unsigned long long sc[6] = {sc_down, sc_rem, sc_dpull, sc_dpush, sc_up2, sc_up3};
+    unsigned long long tot = 0;
+#pragma unroll
+    for (int q = 0; q < 6; ++q) {
+        tot += sc[q];
+        if (sc[q]) atomicAdd(a.stats + kStPhase0 + q, sc[q]);
+    }
+    if (tot) atomicAdd(a.stats + kStScanned, tot);
     if (st_bytes) atomicAdd(a.stats + kStBytes, st_bytes);
 }
 

@@ -87,6 +87,8 @@ SIGNATURES = {
     "dbc_synchronize": (ctypes.c_int, [_P]),
     "dbc_get_timings": (ctypes.c_int, [_P, _P]),
     "dbc_reset_timings": (ctypes.c_int, [_P]),
+    "dbc_debug_counters": (ctypes.c_int, [_P, _P, ctypes.c_int32]),
+    "dbc_debug_root_profile": (ctypes.c_int, [_P, ctypes.c_int32, _P]),
     "dbc_device_bytes": (ctypes.c_int, [_P, _P]),
     "dbc_strerror": (ctypes.c_char_p, [ctypes.c_int]),
     "dbc_last_error": (ctypes.c_char_p, [_P]),
@@ -246,6 +248,21 @@ class DynamicBC:
 
     def reset_timings(self):
         _check(self._ctx, self._lib.dbc_reset_timings(self._ctx))
+
+    def debug_counters(self):
+        names = ["case1", "case2", "case3", "touched", "down", "scanned", "alg_bytes",
+                 "static_bytes", "sc_down", "sc_removal", "sc_dpull", "sc_dpush", "sc_up2", "sc_up3",
+                 "ns_down", "ns_removal", "ns_up_setup", "ns_up_rest", "ns_x", "ns_up_end",
+                 "ns_up_prep", "ns_up_scan", "ns_up_pull", "ns_up_push"]
+        out = np.zeros(len(names), dtype=np.int64)
+        _check(self._ctx, self._lib.dbc_debug_counters(self._ctx, _np_ptr(out), out.size))
+        return dict(zip(names, out.tolist()))
+
+    def root_profile(self, enable=True, read=True):
+        out = np.zeros((self.num_local_roots(), 4), dtype=np.int64) if read else None
+        _check(self._ctx, self._lib.dbc_debug_root_profile(
+            self._ctx, int(enable), _np_ptr(out) if read else None))
+        return out
 
     def device_bytes(self):
         b = ctypes.c_int64()

@@ -1,0 +1,27 @@
+import sys, os
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np, workloads as W
+from paper_conf_ipps_mclaughlinb14_b200 import DynamicBC, FLAG_TIMING
+name = sys.argv[1] if len(sys.argv) > 1 else "rmat16"
+B = int(sys.argv[2]) if len(sys.argv) > 2 else 1000
+wl = W.make_workload(name, insertions=B)
+g = wl.graph
+dbc = DynamicBC(g.n, g.row_ptr, g.col, wl.roots, flags=FLAG_TIMING)
+dbc.static_compute(); dbc.synchronize()
+c0 = dbc.debug_counters()
+dbc.root_profile(True, read=False)
+dbc.insert_edges(wl.ins_u, wl.ins_v)
+c1 = dbc.debug_counters()
+d = {k: c1[k] - c0[k] for k in c1}
+print(d)
+work = d["case2"] + d["case3"]
+print("per working job:", {k: round(v / max(work, 1), 1) for k, v in d.items() if k.startswith("sc_") or k.startswith("ns_") or k in ("touched", "down", "scanned")})
+print("roots deg: median", np.median(g.degree()[wl.roots]), "mean", g.degree()[wl.roots].mean())
+print(dbc.timings())
+prof = dbc.root_profile(True)
+dur = (prof[:, 1] - prof[:, 0]) / 1e6
+print("root chain ms: min %.2f median %.2f p90 %.2f max %.2f; kernel span %.2f" % (dur.min(), np.median(dur), np.percentile(dur, 90), dur.max(), (prof[:,1].max()-prof[:,0].min())/1e6))
+order = np.argsort(-dur)[:8]
+for i in order:
+    print("slot", i, "root", wl.roots[i], "deg", g.degree()[wl.roots[i]], "ms %.2f" % dur[i], "jobs", prof[i,2], "touched", prof[i,3], "start %.2f" % ((prof[i,0]-prof[:,0].min())/1e6))
+print("jobs: median", np.median(prof[:,2]), "max", prof[:,2].max(), "touched/job median", np.median(prof[:,3]/np.maximum(prof[:,2],1)))
