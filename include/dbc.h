@@ -78,6 +78,9 @@ typedef enum {
                                   partial as sum over local slots of delta_s(v)
                                   (Eq. (3)) instead of the incrementally updated
                                   value: removes drift over long streams          */
+#define DBC_FLAG_NO_REORDER 0x8u /* keep the caller's vertex numbering internally
+                                  (default: BFS-order relabelling for locality;
+                                  invisible at the ABI, results identical)        */
 
 typedef struct {
     int32_t device;        /* CUDA device ordinal (default 0)                      */
@@ -163,8 +166,9 @@ dbc_status dbc_insert_edges_device(dbc_ctx *c, const int32_t *u_device,
  * DBC_ENUMERIC if an earlier update overflowed. */
 dbc_status dbc_get_bc(dbc_ctx *c, double *bc);
 
-/* Device pointer to this rank's BC partial, fp64[n] (valid until destroy);
- * for an in-place NCCL sum-all-reduce across ranks.  Not synchronising. */
+/* Device pointer to this rank's BC partial, fp64[n] in the caller's vertex
+ * order (a copy refreshed by this call, valid until the next call or destroy);
+ * for a sum all-reduce across ranks.  Asynchronous on the context stream. */
 dbc_status dbc_get_bc_partial_device(dbc_ctx *c, double **bc_device);
 
 /* Copies one root's state to host arrays of n elements (any may be NULL).

@@ -23,7 +23,10 @@ struct dbc_ctx {
     int64_t nnz = 0, nnz0 = 0, col_cap = 0;
     int64_t edge_cap = 0, inserted = 0;
     int32_t k = 0, k_loc = 0;
-    std::vector<int32_t> roots_local;
+    std::vector<int32_t> roots_local;        // internal vertex ids of the local roots
+    std::vector<int32_t> perm, iperm;        // external -> internal id, internal -> external
+    int32_t *perm_d = nullptr;               // device copy of perm
+    double *bc_ext = nullptr;                // BC partial in external order (for callers)
     cudaStream_t stream = nullptr;
     bool own_stream = false;
     int workers = 0;
@@ -195,6 +198,54 @@ static bool validate_csr(int32_t n, const int64_t *rp, const int32_t *col, std::
     return true;
 }
 
+// Locality relabelling (internal only): vertices in BFS order per component,
+// components started from a minimum-degree vertex, isolated vertices last.
+// Neighbours with nearby ids make the random d / sigma gathers of a level share
+// sectors and cache lines.  Row entry order is preserved (canonical order of
+// the sums, R5), so results are bit-identical to the unrelabelled run.
+static void bfs_order(int32_t n, const int64_t *rp, const int32_t *col, std::vector<int32_t> &perm,
+                      std::vector<int32_t> &iperm) {
+    std::vector<int32_t> byDeg;
+    byDeg.reserve(n);
+    int64_t maxdeg = 0;
+    for (int32_t v = 0; v < n; ++v) maxdeg = std::max<int64_t>(maxdeg, rp[v + 1] - rp[v]);
+    {  // counting sort of non-isolated vertices by degree
+        std::vector<int64_t> cnt((size_t)maxdeg + 2, 0);
+        for (int32_t v = 0; v < n; ++v) cnt[(size_t)(rp[v + 1] - rp[v])]++;
+        std::vector<int64_t> pos((size_t)maxdeg + 2, 0);
+        for (int64_t d = 1; d <= maxdeg; ++d) pos[d + 1] = pos[d] + cnt[d];
+        byDeg.assign((size_t)(n - cnt[0]), 0);
+        for (int32_t v = 0; v < n; ++v) {
+            const int64_t d = rp[v + 1] - rp[v];
+            if (d > 0) byDeg[(size_t)pos[d]++] = v;
+        }
+    }
+    perm.assign(n, -1);
+    iperm.clear();
+    iperm.reserve(n);
+    for (int32_t s0 : byDeg) {
+        if (perm[s0] >= 0) continue;
+        size_t head = iperm.size();
+        perm[s0] = (int32_t)iperm.size();
+        iperm.push_back(s0);
+        while (head < iperm.size()) {
+            const int32_t v = iperm[head++];
+            for (int64_t j = rp[v]; j < rp[v + 1]; ++j) {
+                const int32_t w = col[j];
+                if (perm[w] < 0) {
+                    perm[w] = (int32_t)iperm.size();
+                    iperm.push_back(w);
+                }
+            }
+        }
+    }
+    for (int32_t v = 0; v < n; ++v)
+        if (perm[v] < 0) {
+            perm[v] = (int32_t)iperm.size();
+            iperm.push_back(v);
+        }
+}
+
 static GView view_of(const dbc_ctx *c) {
     GView g;
     g.rp = c->rp[c->cur];
@@ -267,7 +318,14 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
         delete c;
         return s;
     }
-    for (int32_t slot = opt.rank; slot < k; slot += opt.world) c->roots_local.push_back(roots[slot]);
+    if (opt.flags & DBC_FLAG_NO_REORDER) {
+        c->perm.resize(n);
+        for (int32_t v = 0; v < n; ++v) c->perm[v] = v;
+        c->iperm = c->perm;
+    } else {
+        bfs_order(n, row_ptr, col, c->perm, c->iperm);
+    }
+    for (int32_t slot = opt.rank; slot < k; slot += opt.world) c->roots_local.push_back(c->perm[roots[slot]]);
     c->k_loc = (int32_t)c->roots_local.size();
 
     auto bail = [&](dbc_status s) {
@@ -337,6 +395,8 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->d, kn);
     AL(c->sd, kn);
     AL(c->bc, (size_t)n);
+    AL(c->bc_ext, (size_t)n);
+    AL(c->perm_d, (size_t)n);
     AL(c->roots_d, (size_t)c->k_loc);
     const size_t wn = (size_t)c->workers * n;
     AL(c->ws.mark, wn);
@@ -360,16 +420,24 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
 
     // upload CSR (int32 offsets), roots; zero scratch
     {
+        // relabelled CSR: row i = row of external vertex iperm[i], entries mapped, order kept
         std::vector<int32_t> rp32((size_t)n + 1);
-        for (int32_t v = 0; v <= n; ++v) rp32[v] = (int32_t)row_ptr[v];
-        std::vector<int32_t> srt(col, col + c->nnz0);
+        std::vector<int32_t> col2((size_t)c->nnz0);
+        rp32[0] = 0;
+        for (int32_t i = 0; i < n; ++i) {
+            const int32_t v = c->iperm[i];
+            int64_t o = rp32[i];
+            for (int64_t j = row_ptr[v]; j < row_ptr[v + 1]; ++j) col2[(size_t)o++] = c->perm[col[j]];
+            rp32[i + 1] = (int32_t)o;
+        }
+        std::vector<int32_t> srt(col2);
         {
             unsigned nt = std::max(1u, std::min(32u, std::thread::hardware_concurrency()));
             std::vector<std::thread> th;
             for (unsigned t = 0; t < nt; ++t)
                 th.emplace_back([&, t] {
                     for (int64_t v = t; v < n; v += nt)
-                        std::sort(srt.begin() + row_ptr[v], srt.begin() + row_ptr[v + 1]);
+                        std::sort(srt.begin() + rp32[v], srt.begin() + rp32[v + 1]);
                 });
             for (auto &x : th) x.join();
         }
@@ -379,7 +447,8 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
             return bail(DBC_ECUDA);
         }
         if (cudaMemcpy(c->rp[0], rp32.data(), sizeof(int32_t) * (n + 1), cudaMemcpyHostToDevice) != cudaSuccess ||
-            (c->nnz0 && cudaMemcpy(c->col[0], col, sizeof(int32_t) * c->nnz0, cudaMemcpyHostToDevice) != cudaSuccess) ||
+            (c->nnz0 && cudaMemcpy(c->col[0], col2.data(), sizeof(int32_t) * c->nnz0, cudaMemcpyHostToDevice) != cudaSuccess) ||
+            cudaMemcpy(c->perm_d, c->perm.data(), sizeof(int32_t) * n, cudaMemcpyHostToDevice) != cudaSuccess ||
             (c->k_loc && cudaMemcpy(c->roots_d, c->roots_local.data(), sizeof(int32_t) * c->k_loc,
                                     cudaMemcpyHostToDevice) != cudaSuccess)) {
             fail(c, DBC_ECUDA, "upload failed: %s", cudaGetErrorString(cudaGetLastError()));
@@ -563,7 +632,15 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
 extern "C" dbc_status dbc_insert_edges_device(dbc_ctx *c, const int32_t *u, const int32_t *v,
                                               int64_t count, dbc_insert_stats *stats) {
     if (!c) return DBC_EINVAL;
-    return insert_device(c, u, v, count, stats);
+    if (count < 0 || (count > 0 && (!u || !v))) return fail(c, DBC_EINVAL, "bad batch");
+    if (c->inserted + count > c->edge_cap)
+        return fail(c, DBC_ECAPACITY, "edge capacity %lld exhausted (%lld inserted, batch %lld)",
+                    (long long)c->edge_cap, (long long)c->inserted, (long long)count);
+    if (!c->have_state) return fail(c, DBC_ESTATE, "dbc_static_compute must run before insertions");
+    CK(cudaSetDevice(c->device));
+    map_ids(u, v, c->bu, c->bv, count, c->perm_d, c->n, c->stream);  // caller's ids -> internal
+    CK(cudaGetLastError());
+    return insert_device(c, c->bu, c->bv, count, stats);
 }
 
 extern "C" dbc_status dbc_insert_edges(dbc_ctx *c, const int32_t *u, const int32_t *v, int64_t count,
@@ -578,6 +655,8 @@ extern "C" dbc_status dbc_insert_edges(dbc_ctx *c, const int32_t *u, const int32
     if (count) {
         CK(cudaMemcpyAsync(c->bu, u, sizeof(int32_t) * count, cudaMemcpyHostToDevice, c->stream));
         CK(cudaMemcpyAsync(c->bv, v, sizeof(int32_t) * count, cudaMemcpyHostToDevice, c->stream));
+        map_ids(c->bu, c->bv, c->bu, c->bv, count, c->perm_d, c->n, c->stream);
+        CK(cudaGetLastError());
     }
     return insert_device(c, c->bu, c->bv, count, stats);
 }
@@ -605,7 +684,9 @@ extern "C" dbc_status dbc_get_bc_partial_device(dbc_ctx *c, double **p) {
         exact_bc(c->sd, c->roots_d, c->k_loc, c->n, c->bc, c->stream);
         CK(cudaGetLastError());
     }
-    *p = c->bc;
+    gather_ext(c->bc, c->perm_d, c->n, c->bc_ext, c->stream);  // external vertex order
+    CK(cudaGetLastError());
+    *p = c->bc_ext;
     return DBC_OK;
 }
 
@@ -626,15 +707,22 @@ extern "C" dbc_status dbc_get_root_state(dbc_ctx *c, int32_t slot, int32_t *d, d
     if (!c->have_state) return fail(c, DBC_ESTATE, "no state: call dbc_static_compute first");
     CK(cudaSetDevice(c->device));
     const size_t li = (size_t)(slot - c->rank) / c->world, n = (size_t)c->n;
-    if (d) CK(cudaMemcpyAsync(d, c->d + li * n, sizeof(int32_t) * n, cudaMemcpyDeviceToHost, c->stream));
+    if (d) {
+        std::vector<int32_t> tmp(n);
+        CK(cudaMemcpyAsync(tmp.data(), c->d + li * n, sizeof(int32_t) * n, cudaMemcpyDeviceToHost,
+                           c->stream));
+        CK(cudaStreamSynchronize(c->stream));
+        for (size_t v = 0; v < n; ++v) d[v] = tmp[(size_t)c->perm[v]];
+    }
     if (sigma || delta) {
         std::vector<double2> tmp(n);
         CK(cudaMemcpyAsync(tmp.data(), c->sd + li * n, sizeof(double2) * n, cudaMemcpyDeviceToHost,
                            c->stream));
         CK(cudaStreamSynchronize(c->stream));
-        for (size_t i = 0; i < n; ++i) {
-            if (sigma) sigma[i] = tmp[i].x;
-            if (delta) delta[i] = tmp[i].y;
+        for (size_t v = 0; v < n; ++v) {
+            const double2 t = tmp[(size_t)c->perm[v]];
+            if (sigma) sigma[v] = t.x;
+            if (delta) delta[v] = t.y;
         }
     }
     return check_err(c);

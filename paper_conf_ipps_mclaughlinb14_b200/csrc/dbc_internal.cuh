@@ -38,7 +38,9 @@ enum StatIdx : int {
     kStStaticBytes,
     kStPhase0,  // 6 counters: entries scanned by down / removal / D-pull / D-push / up@2 / up@>=3
     kStTime0 = kStPhase0 + 6,  // 10 timers (ns, thread 0): down, removal, up-setup, up-rest, -, up-end, up-prep, up-scan, up-pull, up-push
-    kStCount = kStTime0 + 10
+    kStLevDown = kStTime0 + 10,  // level steps of the down phase
+    kStLevUp,                    // level steps of the up phase
+    kStCount
 };
 
 struct GView {

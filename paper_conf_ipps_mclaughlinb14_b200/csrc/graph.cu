@@ -263,6 +263,35 @@ int append_batch(const AppendBufs &B, const int32_t *rp_old, const int32_t *col_
     return launches + 3;
 }
 
+// external -> internal vertex ids of a batch (out-of-range ids are passed
+// through unchanged so validation still rejects them)
+__global__ void k_map_ids(const int32_t *su, const int32_t *sv, int32_t *du, int32_t *dv, int64_t cnt,
+                          const int32_t *perm, int32_t n) {
+    const int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (e >= cnt) return;
+    const int a = su[e], b = sv[e];
+    du[e] = (a >= 0 && a < n) ? perm[a] : a;
+    dv[e] = (b >= 0 && b < n) ? perm[b] : b;
+}
+
+int map_ids(const int32_t *su, const int32_t *sv, int32_t *du, int32_t *dv, int64_t cnt,
+            const int32_t *perm, int32_t n, cudaStream_t s) {
+    if (cnt == 0) return 0;
+    k_map_ids<<<blocks_for(cnt, 256), 256, 0, s>>>(su, sv, du, dv, cnt, perm, n);
+    return 1;
+}
+
+// out[v] = in[perm[v]]: internal -> external order
+__global__ void k_gather_ext(const double *in, const int32_t *perm, int32_t n, double *out) {
+    const int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (v < n) out[v] = in[perm[v]];
+}
+
+int gather_ext(const double *in, const int32_t *perm, int32_t n, double *out, cudaStream_t s) {
+    k_gather_ext<<<blocks_for(n, 256), 256, 0, s>>>(in, perm, n, out);
+    return 1;
+}
+
 // BC partial rebased as the column sum of delta over local slots (DBC_FLAG_EXACT_BC)
 __global__ void k_exact_bc(const double2 *sd, const int32_t *roots, int32_t k_loc, int32_t n,
                            double *bc) {

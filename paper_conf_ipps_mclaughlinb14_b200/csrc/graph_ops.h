@@ -29,6 +29,9 @@ int validate_batch(const AppendBufs &B, const GView &g, const int32_t *rp_old, i
 int append_batch(const AppendBufs &B, const int32_t *rp_old, const int32_t *col_old,
                  const int32_t *scol_old, int32_t *rp_new, int32_t *col_new, int32_t *scol_new,
                  int32_t n, cudaStream_t s);
+int map_ids(const int32_t *su, const int32_t *sv, int32_t *du, int32_t *dv, int64_t cnt,
+            const int32_t *perm, int32_t n, cudaStream_t s);
+int gather_ext(const double *in, const int32_t *perm, int32_t n, double *out, cudaStream_t s);
 int exact_bc(const double2 *sd, const int32_t *roots, int32_t k_loc, int32_t n, double *bc,
              cudaStream_t s);
 

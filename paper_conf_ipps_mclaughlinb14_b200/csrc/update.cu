@@ -53,6 +53,7 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
     __shared__ ChunkSmem I;              // items of the current up-phase chunk
     __shared__ int s_l1[kChunk];         // chunk slots resolved against adj(root)
     __shared__ int s_nl1;
+    __shared__ int s_nbigI;              // long rows of the current level in I
     __shared__ int s_un[2][kUcap];       // up frontier ping-pong (overflow: Ua / Ub)
     __shared__ uint32_t s_work[kWarps];  // window classification bits (1 = Case 2/3)
     __shared__ int s_job[4];             // uh, ul, L0, case3 of the current job
@@ -81,7 +82,7 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
 
     unsigned long long st_bytes = 0, st_touched = 0, st_down = 0;
     unsigned long long sc_down = 0, sc_rem = 0, sc_dpull = 0, sc_dpush = 0, sc_up2 = 0, sc_up3 = 0;
-    unsigned long long st_c1 = 0, st_c2 = 0, st_c3 = 0;
+    unsigned long long st_c1 = 0, st_c2 = 0, st_c3 = 0, st_lvd = 0, st_lvu = 0;
     // per-phase wall time seen by thread 0 (diagnostic): down, removal, up-split, up-big, up-L1, up-level-end
     unsigned long long tm_ph[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
     unsigned long long tclk = 0;
@@ -103,6 +104,8 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
         s_nbig = 0;
         s_nbig2 = 0;
         s_nbig3 = 0;
+        s_nbigI = 0;
+        s_nl1 = 0;
     }
 
     for (;;) {
@@ -271,6 +274,7 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                 }
                 // D levels: level L0 + j occupies Dv[Doff[j] .. Doff[j+1]), j < nlev
                 const int LmaxD = L0 + nlev - 1;
+                st_lvd += nlev;
                 const int dtotal = le;
                 if (tid == 0) {
                     st_down += dtotal;
@@ -351,6 +355,7 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                 for (int l = Lmax; l >= 1; --l) {
                     if (l < L0 && ucnt == 0) break;  // nothing left above the insertion
                     const bool push = l >= 2;          // level-1 vertices only feed the root
+                    ++st_lvu;
                     // queue p for level l-1 unless already queued (plain flag store; a
                     // rare duplicate from a race is dropped when the list is processed)
                     auto claim_up = [&](int y, uint32_t my) {
@@ -423,88 +428,137 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                         __syncthreads();
                     }
                     tick(2);
-                    // One flattened pass per chunk of the level's items: the down
-                    // segment first, then the up frontier, then removal targets.
-                    const int total = nDl + ucnt + rcnt;
-                    for (int base = 0; base < total; base += kChunk) {
-                        const int cnt = min(kChunk, total - base);
-                        const int nDc = max(0, min(cnt, nDl - base));
-                        if (tid == 0) s_nl1 = 0;
-                        __syncthreads();
-                        // --- A: per-item prep (independent loads) ---
-                        for (int t = tid; t < cnt; t += kBlock) {
-                            const int q = base + t;
-                            int x = -1, meta = 0, beg = 0, len = 0;
+                    // Items of level l: the down segment, then the up frontier, then
+                    // removal targets.  Short rows are handled completely by their
+                    // lane (prep, pull, push, epilogue); long rows are collected in
+                    // shared memory and processed by the flattened chunk pass.
+                    auto resolve = [&](int q, int &x, int &meta, double &c0, double &c1, double &c2,
+                                       int2 &r, bool &need) {
+                        // returns false for an inactive item
+                        if (q < nDl) {
+                            const int idx = b0 + q;
+                            x = Dv[idx];
+                            const double2 s2 = ldcg_d2(sdr + x);
+                            c0 = s2.x;  // sigma (new)
+                            c1 = s2.y;  // delta (old)
+                            c2 = Dsig[idx];
+                            meta = (Dold[idx] == l) ? kMetaNotPulled : 0;
+                            r = row_of(g, x, lim);
+                            need = true;
+                            st_bytes += 8 + 16 + 8 + 4;
+                            return true;
+                        }
+                        const int qi = q - nDl;
+                        x = -1;
+                        if (qi < ucnt)
+                            x = (qi < kUcap) ? s_un[ucur_sel][qi] : Ucur[qi - kUcap];
+                        else if (Rl[qi - ucnt] == l)
+                            x = Rv[qi - ucnt];
+                        if (x < 0) return false;
+                        // first claimant processes the vertex (drops duplicates)
+                        if (atomicMax(mark + x, E | 3u) != mU) return false;
+                        meta = kMetaUp;
+                        c1 = ldcg_d(dacc + x);  // Ddelta (complete: level l+1 is done)
+                        const double2 s2 = ldcg_d2(sdr + x);
+                        c0 = s2.x;
+                        c2 = s2.y;
+                        st_bytes += 24;
+                        need = push && c1 != 0.0;
+                        r = need ? row_of(g, x, lim) : make_int2(0, 0);
+                        return true;
+                    };
+                    auto inlane = [&](int x, int meta, double c0, double c1, double c2, int2 r) {
+                        const bool wantpush = push && r.y > r.x;
+                        if (meta & kMetaUp) {
+                            if (wantpush) {
+                                row_walk(g, dr, sdr, r, [&](int dp) { return dp == l - 1; },
+                                         [&](int pp, int dp, double2 sv) {
+                                             if (dp == l - 1) up_visit(c1, c0, pp, dp, sv, ldcg_u(mark + pp));
+                                         });
+                                (l == 2 ? sc_up2 : sc_up3) += r.y - r.x;
+                                st_bytes += 8 + 8ull * (r.y - r.x);
+                            }
+                            up_finish(x, c1, c2);
+                        } else {
+                            double dn = 0.0;
+                            row_walk(g, dr, sdr, r, [&](int dy) { return dy == l + 1; },
+                                     [&](int y, int dy, double2 sv) { dn += dpull_visit(c0, y, dy, sv); });
+                            sc_dpull += r.y - r.x;
+                            st_bytes += 8ull * (r.y - r.x);
+                            if (wantpush) {
+                                row_walk(g, dr, sdr, r, [&](int dp) { return dp == l - 1; },
+                                         [&](int pp, int dp, double2 sv) {
+                                             if (dp == l - 1)
+                                                 dpush_visit(x, c0, dn, c1, c2, (meta & kMetaNotPulled) != 0,
+                                                             pp, dp, sv, ldcg_u(mark + pp));
+                                         });
+                                (l == 2 ? sc_up2 : sc_up3) += r.y - r.x;
+                                st_bytes += 8ull * (r.y - r.x);
+                            }
+                            d_finish(x, dn, c1);
+                        }
+                    };
+                    auto split_range = [&](int q0, int q1, bool small_inlane) {
+                        for (int q = q0 + tid; q < q1; q += kBlock) {
+                            int x, meta = 0;
                             double c0 = 0.0, c1 = 0.0, c2 = 0.0;
-                            if (q < nDl) {
-                                const int idx = b0 + q;
-                                x = Dv[idx];
-                                const double2 s2 = ldcg_d2(sdr + x);
-                                c0 = s2.x;  // sigma (new)
-                                c1 = s2.y;  // delta (old)
-                                c2 = Dsig[idx];
-                                meta = (Dold[idx] == l) ? kMetaNotPulled : 0;
-                                const int2 r = row_of(g, x, lim);
-                                beg = r.x;
-                                len = r.y - r.x;
-                                st_bytes += 8 + 16 + 8 + 4;
-                            } else {
-                                const int qi = q - nDl;
-                                if (qi < ucnt) {
-                                    x = (qi < kUcap) ? s_un[ucur_sel][qi] : Ucur[qi - kUcap];
-                                } else if (Rl[qi - ucnt] == l) {
-                                    x = Rv[qi - ucnt];
-                                }
-                                // first claimant processes the vertex (drops duplicates)
-                                if (x >= 0 && atomicMax(mark + x, E | 3u) != mU) x = -1;
-                                if (x >= 0) {
-                                    meta = kMetaUp;
-                                    c1 = ldcg_d(dacc + x);  // Ddelta (complete: level l+1 is done)
-                                    const double2 s2 = ldcg_d2(sdr + x);
-                                    c0 = s2.x;
-                                    c2 = s2.y;
-                                    st_bytes += 24;
-                                    if (push && c1 != 0.0) {
-                                        const int2 r = row_of(g, x, lim);
-                                        beg = r.x;
-                                        len = r.y - r.x;
-                                        st_bytes += 8;
-                                        // level 2: resolve against adj(root) when cheaper
-                                        if (l == 2 && len > kSmallDeg && s_ds >= 0 &&
-                                            s_ds * (33 - __clz(len)) < len) {
-                                            s_l1[atomicAdd(&s_nl1, 1)] = t;
-                                            len = 0;
-                                        }
-                                    }
-                                }
+                            int2 r = make_int2(0, 0);
+                            bool need = false;
+                            if (!resolve(q, x, meta, c0, c1, c2, r, need)) continue;
+                            const int len = r.y - r.x;
+                            if (small_inlane && len <= kSmallDeg) {
+                                inlane(x, meta, c0, c1, c2, r);
+                                continue;
+                            }
+                            const int t = atomicAdd(&s_nbigI, 1);
+                            if (t >= kChunk) {  // shared list full: stay in-lane
+                                inlane(x, meta, c0, c1, c2, r);
+                                continue;
+                            }
+                            int elen = len;
+                            // level 2: resolve against adj(root) when cheaper than a scan
+                            if ((meta & kMetaUp) && l == 2 && s_ds >= 0 && s_ds * (33 - __clz(len)) < len) {
+                                s_l1[atomicAdd(&s_nl1, 1)] = t;
+                                elen = 0;
                             }
                             I.v[t] = x;
                             I.meta[t] = meta;
-                            I.beg[t] = beg;
-                            I.off[t + 1] = len;
+                            I.beg[t] = r.x;
+                            I.off[t + 1] = elen;
                             I.acc[t] = 0.0;
                             I.c0[t] = c0;
                             I.c1[t] = c1;
                             I.c2[t] = c2;
                         }
-                        __syncthreads();
-                        tick(6);
-                        chunk_scan(I.off, cnt);  // off[0..cnt], ends with a barrier
-                        tick(7);
-                        // --- C1: delta pull of the down vertices (Eq. (2)) ---
-                        const int E1 = I.off[nDc], E = I.off[cnt];
+                    };
+                    // small levels (<= one item per thread): short rows in-lane;
+                    // large levels: every row through the flattened pass, in chunks
+                    const int total = nDl + ucnt + rcnt;
+                    const bool small_level = total <= kBlock;
+                    const int step = small_level ? total : kChunk;
+                    for (int cb = 0; cb < total; cb += step) {
+                    const int ce = min(total, cb + step);
+                    split_range(cb, min(ce, nDl), small_level);  // down rows first: pull precedes push
+                    __syncthreads();
+                    const int nDb = min(s_nbigI, kChunk);
+                    split_range(max(cb, nDl), ce, small_level);
+                    __syncthreads();
+                    const int nb = min(s_nbigI, kChunk);
+                    if (nb > 0) {
+                        chunk_scan(I.off, nb);  // off[0..nb], ends with a barrier
+                        // --- C1: delta pull of the long down rows (Eq. (2)) ---
+                        const int E1 = I.off[nDb], E = I.off[nb];
                         if (E1 > 0)
-                            flat_entries(I.off, cnt, E1, [&](int t, int e) { return ldg_i(g.col + I.beg[t] + e - I.off[t]); },
+                            flat_entries(I.off, nb, E1, [&](int t, int e) { return ldg_i(g.col + I.beg[t] + e - I.off[t]); },
                                          dr, I.acc, [&](int t, int y, int dy) -> double {
                                              sc_dpull++;
                                              st_bytes += 8;
                                              if (dy != l + 1) return 0.0;
                                              return dpull_visit(I.c0[t], y, dy, ldcg_d2(sdr + y));
                                          });
-                        tick(8);
-                        // --- C2: pushes towards level l-1 (down: new - old, up: sigma ratio * Ddelta) ---
+                        // --- C2: pushes towards level l-1 ---
                         if (push && E > 0)
-                            flat_entries(I.off, cnt, E, [&](int t, int e) { return ldg_i(g.col + I.beg[t] + e - I.off[t]); },
+                            flat_entries(I.off, nb, E, [&](int t, int e) { return ldg_i(g.col + I.beg[t] + e - I.off[t]); },
                                          dr, nullptr, [&](int t, int pp, int dp) -> double {
                                              (l == 2 ? sc_up2 : sc_up3)++;
                                              st_bytes += 8;
@@ -519,7 +573,6 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                                                              (meta & kMetaNotPulled) != 0, pp, dp, sv, mp);
                                              return 0.0;
                                          });
-                        tick(9);
                         // --- C3: level-2 rows resolved against adj(root) ---
                         const int nl1 = s_nl1;
                         if (nl1 > 0) {
@@ -536,23 +589,29 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                             }
                             __syncthreads();
                         }
-                        // --- D: per-item epilogue (Alg. 8 fused) ---
-                        for (int t = tid; t < cnt; t += kBlock) {
-                            const int x = I.v[t];
-                            if (x < 0) continue;
+                        // --- epilogue of the long rows (Alg. 8 fused) ---
+                        for (int t = tid; t < nb; t += kBlock) {
                             if (I.meta[t] & kMetaUp)
-                                up_finish(x, I.c1[t], I.c2[t]);
+                                up_finish(I.v[t], I.c1[t], I.c2[t]);
                             else
-                                d_finish(x, I.acc[t], I.c1[t]);
+                                d_finish(I.v[t], I.acc[t], I.c1[t]);
                         }
                         __syncthreads();
                     }
+                    if (tid == 0) {
+                        s_nbigI = 0;
+                        s_nl1 = 0;
+                    }
+                    __syncthreads();
+                    }  // chunks
                     tick(3);
                     tick(4);
                     ucnt = s_ucnt;
                     __syncthreads();
                     if (tid == 0) {
                         s_ucnt = 0;
+                        s_nbigI = 0;
+                        s_nl1 = 0;
                         s_nbig = 0;
                         s_nbig2 = 0;
                         s_nbig3 = 0;
@@ -591,6 +650,8 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
         if (st_c3) atomicAdd(a.stats + kStCase3, st_c3);
         if (st_touched) atomicAdd(a.stats + kStTouched, st_touched);
         if (st_down) atomicAdd(a.stats + kStDown, st_down);
+        if (st_lvd) atomicAdd(a.stats + kStLevDown, st_lvd);
+        if (st_lvu) atomicAdd(a.stats + kStLevUp, st_lvu);
         for (int q = 0; q < 10; ++q)
             if (tm_ph[q]) atomicAdd(a.stats + kStTime0 + q, tm_ph[q]);
     }

@@ -21,6 +21,7 @@ DBC_INF = 2**31 - 1
 FLAG_MODE_S = 0x1
 FLAG_TIMING = 0x2
 FLAG_EXACT_BC = 0x4
+FLAG_NO_REORDER = 0x8
 
 STATUS = {
     0: "DBC_OK", -1: "DBC_EINVAL", -2: "DBC_ENOMEM", -3: "DBC_ECUDA", -4: "DBC_ENCCL",
@@ -253,7 +254,7 @@ class DynamicBC:
         names = ["case1", "case2", "case3", "touched", "down", "scanned", "alg_bytes",
                  "static_bytes", "sc_down", "sc_removal", "sc_dpull", "sc_dpush", "sc_up2", "sc_up3",
                  "ns_down", "ns_removal", "ns_up_setup", "ns_up_rest", "ns_x", "ns_up_end",
-                 "ns_up_prep", "ns_up_scan", "ns_up_pull", "ns_up_push"]
+                 "ns_up_prep", "ns_up_scan", "ns_up_pull", "ns_up_push", "levels_down", "levels_up"]
         out = np.zeros(len(names), dtype=np.int64)
         _check(self._ctx, self._lib.dbc_debug_counters(self._ctx, _np_ptr(out), out.size))
         return dict(zip(names, out.tolist()))

@@ -291,3 +291,24 @@ def test_rmat16_full_size_batch_parity():
         for (d0, s0), s in zip(dyn, range(0, 256, 15)):
             d1, s1, _ = dbc.get_root_state(s)
             assert np.array_equal(d0, d1) and np.array_equal(s0, s1)
+
+
+@pytest.mark.parametrize("name", ["karate", "rmat10", "delaunay12u"])
+def test_no_reorder_flag_matches_oracle(name):
+    """Internal BFS relabelling (default) and the caller's numbering give the same results."""
+    from paper_conf_ipps_mclaughlinb14_b200 import FLAG_NO_REORDER
+
+    wl = W.make_workload(name)
+    ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
+    for u, v in zip(wl.ins_u, wl.ins_v):
+        ref.insert(u, v)
+    want = ref.compute()
+    outs = []
+    for flags in (FLAG_NO_REORDER, 0):
+        with _dbc(wl.graph, wl.roots, flags=flags) as dbc:
+            dbc.static_compute()
+            dbc.insert_edges(wl.ins_u, wl.ins_v)
+            check_all(dbc, want, wl.roots.size)
+            outs.append([dbc.get_root_state(s) for s in range(wl.roots.size)])
+    for (d0, s0, _), (d1, s1, _) in zip(*outs):
+        assert np.array_equal(d0, d1) and np.array_equal(s0, s1)

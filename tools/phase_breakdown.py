@@ -4,7 +4,7 @@ import numpy as np, workloads as W
 from paper_conf_ipps_mclaughlinb14_b200 import DynamicBC, FLAG_TIMING
 name = sys.argv[1] if len(sys.argv) > 1 else "rmat16"
 B = int(sys.argv[2]) if len(sys.argv) > 2 else 1000
-wl = W.make_workload(name, insertions=B)
+wl = W.make_workload(name, insertions=B, k=int(sys.argv[3]) if len(sys.argv) > 3 else None)
 g = wl.graph
 dbc = DynamicBC(g.n, g.row_ptr, g.col, wl.roots, flags=FLAG_TIMING)
 dbc.static_compute(); dbc.synchronize()
@@ -15,7 +15,7 @@ c1 = dbc.debug_counters()
 d = {k: c1[k] - c0[k] for k in c1}
 print(d)
 work = d["case2"] + d["case3"]
-print("per working job:", {k: round(v / max(work, 1), 1) for k, v in d.items() if k.startswith("sc_") or k.startswith("ns_") or k in ("touched", "down", "scanned")})
+print("per working job:", {k: round(v / max(work, 1), 1) for k, v in d.items() if k.startswith("sc_") or k.startswith("ns_") or k.startswith("levels") or k in ("touched", "down", "scanned")})
 print("roots deg: median", np.median(g.degree()[wl.roots]), "mean", g.degree()[wl.roots].mean())
 print(dbc.timings())
 prof = dbc.root_profile(True)
