@@ -43,8 +43,8 @@ struct dbc_ctx {
     int32_t *bu = nullptr, *bv = nullptr;  // host-API batch staging
 
     // state
-    int32_t *d = nullptr;
-    double2 *sd = nullptr;
+    int32_t *d = nullptr;    // [k_loc][n]
+    double2 *sd = nullptr;   // [k_loc][n] (sigma, delta)
     double *bc = nullptr;
     int32_t *roots_d = nullptr;
 
@@ -356,7 +356,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     c->ev_ok = true;
 
     // workers: persistent CTAs; bounded by roots and by a scratch-memory budget
-    const size_t per_worker = (size_t)n * (4 + 8 + 8 + 4 + 4 + 8 + 4 + 4 + 4 + 4 + 8) + (size_t)(n + 2) * 4 + 64;
+    const size_t per_worker = (size_t)n * (4 + 8 + 8 + 4 + 4 + 8 + 4 + 4 + 4 + 4 + 4) + (size_t)(n + 2) * 4 + 64;
     size_t free_b = 0, total_b = 0;
     cudaMemGetInfo(&free_b, &total_b);
     const size_t state_b = (size_t)c->k_loc * n * 20 + (size_t)c->col_cap * 8 + (size_t)n * 40;
@@ -410,7 +410,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->ws.U1, wn);
     AL(c->ws.Rv, wn);
     AL(c->ws.Rl, wn);
-    AL(c->ws.Bq, 2 * wn);
+    AL(c->ws.Bq, wn);
     AL(c->ws.wepoch, (size_t)c->workers);
     AL(c->next_slot, 1);
     AL(c->stats, (size_t)kStCount);
@@ -707,22 +707,17 @@ extern "C" dbc_status dbc_get_root_state(dbc_ctx *c, int32_t slot, int32_t *d, d
     if (!c->have_state) return fail(c, DBC_ESTATE, "no state: call dbc_static_compute first");
     CK(cudaSetDevice(c->device));
     const size_t li = (size_t)(slot - c->rank) / c->world, n = (size_t)c->n;
-    if (d) {
-        std::vector<int32_t> tmp(n);
-        CK(cudaMemcpyAsync(tmp.data(), c->d + li * n, sizeof(int32_t) * n, cudaMemcpyDeviceToHost,
-                           c->stream));
-        CK(cudaStreamSynchronize(c->stream));
-        for (size_t v = 0; v < n; ++v) d[v] = tmp[(size_t)c->perm[v]];
-    }
-    if (sigma || delta) {
-        std::vector<double2> tmp(n);
-        CK(cudaMemcpyAsync(tmp.data(), c->sd + li * n, sizeof(double2) * n, cudaMemcpyDeviceToHost,
-                           c->stream));
+    {
+        std::vector<int32_t> td(n);
+        std::vector<double2> ts(n);
+        CK(cudaMemcpyAsync(td.data(), c->d + li * n, sizeof(int32_t) * n, cudaMemcpyDeviceToHost, c->stream));
+        CK(cudaMemcpyAsync(ts.data(), c->sd + li * n, sizeof(double2) * n, cudaMemcpyDeviceToHost, c->stream));
         CK(cudaStreamSynchronize(c->stream));
         for (size_t v = 0; v < n; ++v) {
-            const double2 t = tmp[(size_t)c->perm[v]];
-            if (sigma) sigma[v] = t.x;
-            if (delta) delta[v] = t.y;
+            const size_t i = (size_t)c->perm[v];
+            if (d) d[v] = td[i];
+            if (sigma) sigma[v] = ts[i].x;
+            if (delta) delta[v] = ts[i].y;
         }
     }
     return check_err(c);

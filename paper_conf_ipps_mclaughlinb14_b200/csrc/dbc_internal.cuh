@@ -1,13 +1,16 @@
 // dbc_internal.cuh -- shared device-side definitions of libdbc (B200 / sm_100a).
 //
-// Layout in HBM (DESIGN.md Sec. 4):
+// Layout in HBM (DESIGN.md Sec. 6):
 //   graph   rp int32[n+1] (bit 31 of rp[v] = "row v has entries of the current
-//           batch"), col int32[cap]; for flagged rows xinfo[v] = {first tag
-//           index, count} and xtag[] = batch-local insertion index of each batch
-//           entry, in row order.  Row v = col[rp[v] .. rp[v+1]) (masked): the
-//           base part, then the current batch's entries sorted by insertion index.
-//   state   d int32[k_loc][n], sd double2[k_loc][n] = (sigma, delta) per vertex,
-//           root-major (each root's arrays contiguous), bc double[n].
+//           batch"), col int32[cap] in canonical order, scol int32[cap] (same
+//           rows sorted by id); for flagged rows xinfo[v] = {first, count} into
+//           the batch arrays xtag (insertion index) / xnbr (neighbour).  Row v at
+//           insertion i = base part + batch entries with index <= i.
+//   state   root-major (each root's arrays contiguous): d int32[k_loc][n], the
+//           filter every neighbour gather reads (kept apart from sigma/delta so
+//           the filter footprint stays small and L2-friendly), and sd
+//           double2[k_loc][n] = (sigma, delta), so the successor pair of Eq. (2)
+//           arrives in one 16-byte gather; bc double[n].
 //   scratch per persistent worker CTA, n-sized arrays (epoch-tagged, never
 //           cleared between jobs -- no O(n) work per root per insertion,
 //           SURVEY.md Sec. 7 hard part (iii)).
@@ -27,7 +30,8 @@ constexpr uint32_t kFull = 0xffffffffu;
 constexpr int32_t kInf = INT32_MAX;
 constexpr int32_t kMask = 0x7fffffff;
 constexpr uint32_t kDown = 1u;           // mark state: in the down set D (Alg. 2 t[v] = down)
-constexpr uint32_t kUp = 2u;             // mark state: found by the up phase (t[v] = up)
+constexpr uint32_t kUp = 2u;             // mark state: queued by the up phase (t[v] = up)
+constexpr uint32_t kUpDone = 3u;         // mark state: up vertex processed
 constexpr double kExact = 9007199254740992.0;  // 2^53
 
 enum ErrBits : int { kErrNumeric = 1, kErrOverflow = 2 };
@@ -36,11 +40,18 @@ enum ErrBits : int { kErrNumeric = 1, kErrOverflow = 2 };
 enum StatIdx : int {
     kStCase1 = 0, kStCase2, kStCase3, kStTouched, kStDown, kStScanned, kStBytes,
     kStStaticBytes,
-    kStPhase0,  // 6 counters: entries scanned by down / removal / D-pull / D-push / up@2 / up@>=3
-    kStTime0 = kStPhase0 + 6,  // 10 timers (ns, thread 0): down, removal, up-setup, up-rest, -, up-end, up-prep, up-scan, up-pull, up-push
+    kStPhase0,                 // 6: entries scanned by down / removal / D-pull / D-push / up@2 / up@>=3
+    kStTime0 = kStPhase0 + 6,  // 10 timers (ns, thread 0), see update.cu tick()
     kStLevDown = kStTime0 + 10,  // level steps of the down phase
     kStLevUp,                    // level steps of the up phase
     kStCount
+};
+
+// The state of one root (pointers into the root-major arrays).
+struct Root {
+    int32_t *d;    // distance, kInf = unreachable
+    double2 *sd;   // (sigma, delta)
+    __device__ __forceinline__ int dist(int y) const { return d[y]; }
 };
 
 struct GView {
@@ -53,7 +64,7 @@ struct GView {
 };
 
 // Scratch of the persistent workers (one CTA = one worker), each array
-// worker-major with stride n (DESIGN.md Sec. 4).
+// worker-major with stride n (DESIGN.md Sec. 6).
 struct Scratch {
     uint32_t *mark;            // epoch<<2 | state
     unsigned long long *lowrec;  // (epoch << 32) | old d, written by the lowering thread
@@ -62,27 +73,23 @@ struct Scratch {
     int32_t *Dold;             // old d of D[i]
     double *Dsig;              // old sigma of D[i]
     int32_t *Doff;             // level offsets of D (also static level offsets), n+2
-    int32_t *U0, *U1;          // up frontier ping-pong
+    int32_t *U0, *U1;          // up frontier overflow ping-pong
     int32_t *Rv, *Rl;          // removal-push targets and their levels (Case 3)
-    int32_t *Bq;               // big-row queues of the current level, 2n per worker
+    int32_t *Bq;               // long-row queue of the current level, n per worker
     uint32_t *wepoch;          // per-worker epoch counter
 };
 
 // ---------------------------------------------------------------------------
-// loads: the immutable graph through the read-only path; mutable state with
+// Loads: the immutable graph through the read-only path; mutable state with
 // plain (L1-cacheable) loads.  A worker CTA is the only writer of its root's
-// arrays and of its scratch during a launch, every cross-thread dependency is
-// ordered by __syncthreads() -- which makes all earlier global writes and
-// atomics of the block visible to it -- and the same-level races the
-// algorithm tolerates (lowering, claims) are resolved by atomics, so a stale
-// line can only cost a redundant atomic, never a wrong value.  L1 is
-// invalidated between launches.
+// records and of its scratch during a launch; every cross-thread dependency is
+// ordered by __syncthreads() (which makes all earlier global writes and
+// atomics of the block visible to it); the same-level races the algorithm
+// tolerates (lowering, claims) are resolved by atomics, so a stale line can
+// only cost a redundant atomic, never a wrong value.  L1 is invalidated
+// between launches.
 __device__ __forceinline__ int ldg_i(const int32_t *p) { return __ldg(p); }
-__device__ __forceinline__ int ldcg_i(const int32_t *p) { return *p; }
-__device__ __forceinline__ double ldcg_d(const double *p) { return *p; }
-__device__ __forceinline__ double2 ldcg_d2(const double2 *p) { return *p; }
-__device__ __forceinline__ uint32_t ldcg_u(const uint32_t *p) { return *p; }
-__device__ __forceinline__ unsigned long long ldcg_ull(const unsigned long long *p) { return *p; }
+
 
 // Adjacency row of v, restricted to batch entries with insertion index <= limit
 // (canonical order: base row, then inserted neighbours in insertion order).
@@ -124,203 +131,75 @@ __device__ __forceinline__ bool adjacent_visible(const GView &g, int x, int p, i
 }
 
 // ---------------------------------------------------------------------------
-// Chunked flattened level pass (up phase): up to kChunk items per chunk held in
-// shared memory; all of their row entries are spread over the CTA.
-constexpr int kChunk = 512;
-constexpr int kUcap = 1024;  // up-frontier entries kept in shared memory
-constexpr int kMetaUp = 1, kMetaNotPulled = 2;
-constexpr int kFlatU = 4;  // contiguous entries per thread per step
+// Level processing (the paper's node-based parallelism, Sec. III, P:272-274,
+// re-mapped for B200): the vertices of one BFS level are split by row length.
+//  * short rows (<= kSmallDeg entries): one lane walks the whole row in
+//    canonical order with kRowUnroll entries in flight (bit-exact pull sums);
+//  * long rows (hubs): processed by the whole CTA with their entries
+//    flattened (every thread takes a few entries per step, gathers hoisted),
+//    per-row reductions through warp-aggregated shared-memory fp64 atomics --
+//    the load-balanced "advance" of Merrill et al. [19] (cited at P:322).
 
-struct ChunkSmem {
-    int v[kChunk];
-    int meta[kChunk];
-    int beg[kChunk];
-    int off[kChunk + 1];
-    double acc[kChunk], c0[kChunk], c1[kChunk], c2[kChunk];
-};
-
-// exclusive scan in place of off[1..cnt] (lengths) -> off[0..cnt]; ends with a barrier
-__device__ __forceinline__ void chunk_scan(int *off, int cnt) {
-    __shared__ int ws[kWarps];
-    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-    constexpr int per = kChunk / kBlock;  // items per thread
-    int vals[per];
-    int run = 0;
-#pragma unroll
-    for (int q = 0; q < per; ++q) {
-        const int i = tid * per + q;
-        vals[q] = (i < cnt) ? off[i + 1] : 0;
-        run += vals[q];
-    }
-    int incl = run;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const int y = __shfl_up_sync(kFull, incl, o);
-        if (lane >= o) incl += y;
-    }
-    if (lane == 31) ws[wid] = incl;
-    __syncthreads();
-    int wbase = 0;
-    for (int w = 0; w < wid; ++w) wbase += ws[w];
-    int ex = wbase + incl - run;
-#pragma unroll
-    for (int q = 0; q < per; ++q) {
-        const int i = tid * per + q;
-        ex += vals[q];
-        if (i < cnt) off[i + 1] = ex;
-    }
-    if (tid == 0) off[0] = 0;
-    __syncthreads();
-}
-
-// Flattened entries [0, E) of the chunk's rows (off = exclusive offsets of cnt
-// rows): thread tid takes kFlatU consecutive entries per step (one binary
-// search, then linear advance), gathers column + distance up front, and calls
-// f(t, y, dy); if acc != nullptr the returned contribution is summed into
-// acc[t] (warp-aggregated shared-memory atomics).  Ends with a barrier.
-template <class Col, class F>
-__device__ __forceinline__ void flat_entries(const int *off, int cnt, int E, Col colf,
-                                             const int32_t *dr, double *acc, F f) {
-    const int tid = threadIdx.x, lane = tid & 31;
-    for (int base = 0; base < E; base += kBlock * kFlatU) {
-        const int e0 = base + tid * kFlatU;
-        int t[kFlatU], y[kFlatU], dy[kFlatU];
-        int cur = -1;
-        if (e0 < E) {
-            int lo = 0, hi = cnt - 1;  // last row with off[row] <= e0
-            while (lo < hi) {
-                const int mid = (lo + hi + 1) >> 1;
-                if (off[mid] <= e0) lo = mid; else hi = mid - 1;
-            }
-            cur = lo;
-        }
-#pragma unroll
-        for (int u = 0; u < kFlatU; ++u) {
-            const int e = e0 + u;
-            t[u] = -1;
-            if (e < E) {
-                while (off[cur + 1] <= e) ++cur;
-                t[u] = cur;
-                y[u] = colf(cur, e);
-            }
-        }
-#pragma unroll
-        for (int u = 0; u < kFlatU; ++u)
-            if (t[u] >= 0) dy[u] = ldcg_i(dr + y[u]);
-#pragma unroll
-        for (int u = 0; u < kFlatU; ++u) {
-            double c = 0.0;
-            if (t[u] >= 0) c = f(t[u], y[u], dy[u]);
-            if (acc) {
-                const int t0 = __shfl_sync(kFull, t[u], 0);
-                const bool uni = __all_sync(kFull, t[u] == t0 || t[u] < 0);
-                if (uni) {
-                    if (t0 >= 0) {
-#pragma unroll
-                        for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(kFull, c, o);
-                        if (lane == 0 && c != 0.0) atomicAdd(acc + t0, c);
-                    }
-                } else if (c != 0.0) {
-                    atomicAdd(acc + t[u], c);
-                }
-            }
-        }
-    }
-    __syncthreads();
-}
-
-// Sequential walk of one (small) row in canonical order with kRowUnroll entries
-// in flight: column, distance and -- for entries passing want(dy) -- the
-// (sigma, delta) pair are gathered up front, then f(y, dy, sd) runs in order.
+// Sequential walk of one (small) row in canonical order: columns, then the
+// neighbours' distances, then -- only for entries passing want(d) -- their
+// (sigma, delta) pair and mk[y] (if mk), kRowUnroll entries in flight; then
+// f(y, d, sd, mark) runs in order.
 constexpr int kRowUnroll = 8;
 template <class Want, class F>
-__device__ __forceinline__ void row_walk(const GView &g, const int32_t *dr, const double2 *sdr,
+__device__ __forceinline__ void row_walk(const GView &g, const Root &st, const uint32_t *mk,
                                          int2 r, Want want, F f) {
     for (int j = r.x; j < r.y; j += kRowUnroll) {
         int y[kRowUnroll], dy[kRowUnroll];
-        double2 sv[kRowUnroll];
+        double2 q[kRowUnroll];
+        uint32_t mm[kRowUnroll];
 #pragma unroll
         for (int u = 0; u < kRowUnroll; ++u) y[u] = (j + u < r.y) ? ldg_i(g.col + j + u) : -1;
 #pragma unroll
-        for (int u = 0; u < kRowUnroll; ++u) dy[u] = (y[u] >= 0) ? ldcg_i(dr + y[u]) : kInf;
+        for (int u = 0; u < kRowUnroll; ++u) dy[u] = (y[u] >= 0) ? st.dist(y[u]) : kInf;
+#pragma unroll
+        for (int u = 0; u < kRowUnroll; ++u) {
+            const bool w = y[u] >= 0 && want(dy[u]);
+            q[u] = w ? st.sd[y[u]] : make_double2(0.0, 0.0);
+            mm[u] = (mk && w) ? mk[y[u]] : 0u;
+        }
 #pragma unroll
         for (int u = 0; u < kRowUnroll; ++u)
-            sv[u] = (y[u] >= 0 && want(dy[u])) ? ldcg_d2(sdr + y[u]) : make_double2(0.0, 0.0);
-#pragma unroll
-        for (int u = 0; u < kRowUnroll; ++u)
-            if (y[u] >= 0) f(y[u], dy[u], sv[u]);
+            if (y[u] >= 0) f(y[u], dy[u], q[u], mm[u]);
     }
 }
 
-template <int G>
-__device__ __forceinline__ double group_sum(double x) {
-    if constexpr (G == 32) {
-#pragma unroll
-        for (int o = 16; o; o >>= 1) x += __shfl_xor_sync(kFull, x, o);
-    }
-    return x;  // butterfly: every lane ends with the same (commutative) value
-}
-
-template <int G>
-__device__ __forceinline__ void group_sync() {
-    if constexpr (G == 32) __syncwarp();
-}
-
-using G1 = std::integral_constant<int, 1>;
-using G32 = std::integral_constant<int, 32>;
-
-// ---------------------------------------------------------------------------
-// Level processing (the paper's node-based parallelism, Sec. III, P:272-274,
-// re-mapped for B200): the vertices of one BFS level are split by row length.
-//  * small rows (<= kSmallDeg entries): one lane walks the whole row in
-//    canonical order (bit-exact pull sums for free, 32 independent rows per
-//    warp in flight);
-//  * big rows (hubs): queued, then processed in rounds of <= kBig rows whose
-//    entries are flattened across the whole CTA (every thread takes entries
-//    e = tid, tid + kBlock, ..., kUnroll of them per step with the column and
-//    distance gathers hoisted), per-row reductions going through warp-
-//    aggregated shared-memory fp64 atomics.  This is the load-balanced
-//    "advance" Merrill et al. [19] (cited at P:322) describe, restricted to the
-//    rows that need it.
-
-constexpr int kBig = 128;     // big rows per round
+// --- long rows: rounds of up to kBig rows staged in shared memory -----------
+constexpr int kBig = 128;     // long rows per round (down phase / static)
 constexpr int kUnroll = 4;    // entries per thread in flight
-constexpr int kAdjCap = 512;  // longest root row kept in shared memory (level-2 shortcut)
 
 struct BigSmem {
-    int idx[kBig];    // item index (caller's list) of each big row
+    int idx[kBig];    // item index (caller's list) of each long row
     int v[kBig];      // vertex
     int b[kBig];      // row begin
     int off[kBig + 1];  // exclusive scan of row lengths; off[m] = total
     double acc[kBig];   // per-row reduction
-    double c0[kBig], c1[kBig];  // per-row constants of the caller
+    double c0[kBig];    // per-row constant of the caller
     int m;            // rows in this round
 };
 
-// Pass over `count` items: small rows processed inline by their lane; big rows
-// handed (as item indices) to enqueue().
-//   get(idx, &v) -> bool : item idx is active, vertex v
-//   need_row(idx, v)     : whether the row is needed at all
-//   small(idx, v, row)   : process one small row sequentially
-template <class Get, class NeedRow, class Small, class Enq>
+// Pass over `count` items: short rows processed inline by their lane, long
+// rows handed (as item indices) to enqueue().
+template <class Get, class Small, class Enq>
 __device__ __forceinline__ void split_pass(int count, const GView &g, int limit, Get get,
-                                           NeedRow need_row, Small small, Enq enqueue) {
+                                           Small small, Enq enqueue) {
     for (int idx = threadIdx.x; idx < count; idx += kBlock) {
         int v = 0;
         if (!get(idx, v)) continue;
-        int2 r = make_int2(0, 0);
-        if (need_row(idx, v)) r = row_of(g, v, limit);
-        if (r.y - r.x > kSmallDeg) {
-            enqueue(idx, v, r);
-        } else {
+        const int2 r = row_of(g, v, limit);
+        if (r.y - r.x > kSmallDeg)
+            enqueue(idx);
+        else
             small(idx, v, r);
-        }
     }
 }
 
-// Load a round of m <= kBig queued big rows into shared memory (rows, offsets).
-// fetch(t) -> item index of the t-th row of the round; getv(idx) -> vertex.
-// Caller must __syncthreads() before (queue complete) -- this ends with a barrier.
+// Load a round of m <= kBig queued long rows (rows, offsets).  Caller must
+// __syncthreads() before (queue complete); ends with a barrier.
 template <class Fetch, class GetV>
 __device__ __forceinline__ void big_load(BigSmem &S, int m, Fetch fetch, GetV getv,
                                          const GView &g, int limit) {
@@ -366,19 +245,38 @@ __device__ __forceinline__ void big_load(BigSmem &S, int m, Fetch fetch, GetV ge
     __syncthreads();
 }
 
-// Flattened pass over all entries of the loaded round.  f(t, y, dy) is called
-// for every entry (t = row slot, y = neighbour, dy = d[y] gathered up front)
-// and returns a contribution that is summed into S.acc[t].  Ends with a barrier.
-template <class F>
-__device__ __forceinline__ void big_entries(BigSmem &S, const GView &g, const int32_t *dr, F f) {
-    const int tid = threadIdx.x, lane = tid & 31;
+// warp-aggregated shared-memory accumulation of c into acc[t] (all lanes call;
+// t < 0 = no contribution)
+__device__ __forceinline__ void acc_add(double *acc, int t, double c) {
+    const int lane = threadIdx.x & 31;
+    const int t0 = __shfl_sync(kFull, t, 0);
+    const bool uni = __all_sync(kFull, t == t0 || t < 0);
+    if (uni) {
+        if (t0 >= 0) {
+#pragma unroll
+            for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(kFull, c, o);
+            if (lane == 0 && c != 0.0) atomicAdd(acc + t0, c);
+        }
+    } else if (t >= 0 && c != 0.0) {
+        atomicAdd(acc + t, c);
+    }
+}
+
+// Flattened pass over all entries of a loaded round (strided mapping).
+// f(t, y, d, sd) returns a contribution summed into S.acc[t]; sd is gathered
+// only for entries passing want(d).  Ends with a barrier.
+template <class Want, class F>
+__device__ __forceinline__ void big_entries(BigSmem &S, const GView &g, const Root &st, Want want, F f) {
+    const int tid = threadIdx.x;
     const int m = S.m, E = S.off[m];
     for (int base = 0; base < E; base += kUnroll * kBlock) {
         int t[kUnroll], y[kUnroll], dy[kUnroll];
+        double2 q[kUnroll];
 #pragma unroll
         for (int u = 0; u < kUnroll; ++u) {
             const int e = base + u * kBlock + tid;
             t[u] = -1;
+            y[u] = 0;
             if (e < E) {
                 int lo = 0, hi = m - 1;  // last t with off[t] <= e
                 while (lo < hi) {
@@ -390,39 +288,133 @@ __device__ __forceinline__ void big_entries(BigSmem &S, const GView &g, const in
             }
         }
 #pragma unroll
+        for (int u = 0; u < kUnroll; ++u) dy[u] = (t[u] >= 0) ? st.dist(y[u]) : kInf;
+#pragma unroll
         for (int u = 0; u < kUnroll; ++u)
-            if (t[u] >= 0) dy[u] = ldcg_i(dr + y[u]);
+            q[u] = (t[u] >= 0 && want(dy[u])) ? st.sd[y[u]] : make_double2(0.0, 0.0);
 #pragma unroll
         for (int u = 0; u < kUnroll; ++u) {
             double c = 0.0;
-            if (t[u] >= 0) c = f(t[u], y[u], dy[u]);
-            const int t0 = __shfl_sync(kFull, t[u], 0);
-            const bool uni = __all_sync(kFull, t[u] == t0 || t[u] < 0);
-            if (uni) {
-                if (t0 >= 0) {
+            if (t[u] >= 0) c = f(t[u], y[u], dy[u], q[u]);
+            acc_add(S.acc, t[u], c);
+        }
+    }
+    __syncthreads();
+}
+
+// --- up phase: chunked flattened level pass ----------------------------------
+constexpr int kChunk = 512;   // items per chunk (shared memory)
+constexpr int kUcap = 1024;   // up-frontier entries kept in shared memory
+constexpr int kMetaUp = 1, kMetaNotPulled = 2;
+constexpr int kFlatU = 4;     // contiguous entries per thread per step
+constexpr int kAdjCap = 512;  // longest root row kept in shared memory (level-2 shortcut)
+
+struct ChunkSmem {
+    int v[kChunk];
+    int meta[kChunk];
+    int beg[kChunk];
+    int off[kChunk + 1];
+    double acc[kChunk], c0[kChunk], c1[kChunk], c2[kChunk];
+};
+
+// exclusive scan in place of off[1..cnt] (lengths) -> off[0..cnt]; ends with a barrier
+__device__ __forceinline__ void chunk_scan(int *off, int cnt) {
+    __shared__ int ws[kWarps];
+    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+    constexpr int per = kChunk / kBlock;  // items per thread
+    int vals[per];
+    int run = 0;
 #pragma unroll
-                    for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(kFull, c, o);
-                    if (lane == 0 && c != 0.0) atomicAdd(&S.acc[t0], c);
-                }
-            } else if (c != 0.0) {
-                atomicAdd(&S.acc[t[u]], c);
+    for (int q = 0; q < per; ++q) {
+        const int i = tid * per + q;
+        vals[q] = (i < cnt) ? off[i + 1] : 0;
+        run += vals[q];
+    }
+    int incl = run;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(kFull, incl, o);
+        if (lane >= o) incl += y;
+    }
+    if (lane == 31) ws[wid] = incl;
+    __syncthreads();
+    int wbase = 0;
+    for (int w = 0; w < wid; ++w) wbase += ws[w];
+    int ex = wbase + incl - run;
+#pragma unroll
+    for (int q = 0; q < per; ++q) {
+        const int i = tid * per + q;
+        ex += vals[q];
+        if (i < cnt) off[i + 1] = ex;
+    }
+    if (tid == 0) off[0] = 0;
+    __syncthreads();
+}
+
+// Flattened entries [0, E) of the chunk's rows (off = exclusive offsets of cnt
+// rows): thread tid takes kFlatU consecutive entries per step (one binary
+// search, then linear advance), gathers columns and record halves up front and
+// calls f(t, y, d, sd, mark) (sd, mark gathered for want(d)); if acc != nullptr
+// the returned contribution is
+// summed into acc[t].  Ends with a barrier.
+template <class Want, class Col, class F>
+__device__ __forceinline__ void flat_entries(const int *off, int cnt, int E, Col colf, const Root &st,
+                                             const uint32_t *mk, Want want, double *acc, F f) {
+    const int tid = threadIdx.x;
+    for (int base = 0; base < E; base += kBlock * kFlatU) {
+        const int e0 = base + tid * kFlatU;
+        int t[kFlatU], y[kFlatU], dy[kFlatU];
+        double2 q[kFlatU];
+        uint32_t mm[kFlatU];
+        int cur = -1;
+        if (e0 < E) {
+            int lo = 0, hi = cnt - 1;  // last row with off[row] <= e0
+            while (lo < hi) {
+                const int mid = (lo + hi + 1) >> 1;
+                if (off[mid] <= e0) lo = mid; else hi = mid - 1;
             }
+            cur = lo;
+        }
+#pragma unroll
+        for (int u = 0; u < kFlatU; ++u) {
+            const int e = e0 + u;
+            t[u] = -1;
+            y[u] = 0;
+            if (e < E) {
+                while (off[cur + 1] <= e) ++cur;
+                t[u] = cur;
+                y[u] = colf(cur, e);
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < kFlatU; ++u) dy[u] = (t[u] >= 0) ? st.dist(y[u]) : kInf;
+#pragma unroll
+        for (int u = 0; u < kFlatU; ++u) {
+            const bool w = t[u] >= 0 && want(dy[u]);
+            q[u] = w ? st.sd[y[u]] : make_double2(0.0, 0.0);
+            mm[u] = (mk && w) ? mk[y[u]] : 0u;
+        }
+#pragma unroll
+        for (int u = 0; u < kFlatU; ++u) {
+            double c = 0.0;
+            if (t[u] >= 0) c = f(t[u], y[u], dy[u], q[u], mm[u]);
+            if (acc) acc_add(acc, t[u], c);
         }
     }
     __syncthreads();
 }
 
 // ---------------------------------------------------------------------------
-// kernel entry points (defined in graph.cu / static_brandes.cu / update.cu)
+// kernel entry points (defined in static_brandes.cu / update.cu)
 struct UpdateArgs {
     GView g;
     int32_t n;
     int32_t k_loc;
-    const int32_t *roots;  // local roots, [k_loc]
-    int32_t *d;
-    double2 *sd;
+    const int32_t *roots;  // local roots (internal ids), [k_loc]
+    int32_t *d;            // [k_loc][n]
+    double2 *sd;           // [k_loc][n]
     double *bc;
-    const int32_t *ins_u, *ins_v;  // batch, device
+    const int32_t *ins_u, *ins_v;  // batch, device (internal ids)
     int32_t ins_begin, ins_end;    // batch-local insertion range of this launch
     Scratch ws;
     int32_t *next_slot;            // work counter (zeroed before launch)

@@ -3,7 +3,7 @@
 // the dynamic update maintains, and is the GPU recompute baseline of Table III
 // (the paper used Jia et al. [13] in that role).
 //
-// B200 design (DESIGN.md Sec. 5 K1): persistent grid, one worker CTA per root at
+// B200 design (DESIGN.md Sec. 6 K1): persistent grid, one worker CTA per root at
 // a time (roots fetched with an atomic counter -- the coarse-grained root
 // parallelism of Fig. 3), level-synchronous BFS inside the CTA with
 // the frontier kept as a level-ordered queue (Alg. 5's Q/QQ).  The
@@ -26,10 +26,10 @@ __global__ void __launch_bounds__(kBlock, 2) static_kernel(StaticArgs a) {
     const size_t n = (size_t)a.n;
     int32_t *order = a.ws.Dv + (size_t)w * n;
     int32_t *loff = a.ws.Doff + (size_t)w * (n + 2);
-    int32_t *Bq = a.ws.Bq + (size_t)w * 2 * n;
+    int32_t *Bq = a.ws.Bq + (size_t)w * n;
     const GView &g = a.g;
     unsigned long long bytes = 0;
-    auto enq = [&](int idx, int, int2) { Bq[atomicAdd(&s_nbig, 1)] = idx; };
+    auto enq = [&](int idx) { Bq[atomicAdd(&s_nbig, 1)] = idx; };
     if (tid == 0) s_nbig = 0;
 
     for (;;) {
@@ -39,22 +39,18 @@ __global__ void __launch_bounds__(kBlock, 2) static_kernel(StaticArgs a) {
         __syncthreads();
         if (slot >= a.k_loc) break;
         const int s = a.roots[slot];
-        int32_t *dr = a.d + (size_t)slot * n;
-        double2 *sdr = a.sd + (size_t)slot * n;
+        const Root st{a.d + (size_t)slot * n, a.sd + (size_t)slot * n};
 
-        // Stage 1 (Alg. 1 lines 3-9): d = INF, sigma = delta = 0 (vectorised stores).
-        {
-            int4 *d4 = reinterpret_cast<int4 *>(dr);
-            const size_t n4 = ((size_t)slot * n) % 4 == 0 ? n / 4 : 0;
-            for (size_t v = tid; v < n4; v += kBlock) d4[v] = make_int4(kInf, kInf, kInf, kInf);
-            for (size_t v = n4 * 4 + tid; v < n; v += kBlock) dr[v] = kInf;
-            for (size_t v = tid; v < n; v += kBlock) sdr[v] = make_double2(0.0, 0.0);
+        // Stage 1 (Alg. 1 lines 3-9): d = INF, sigma = delta = 0 (vector stores)
+        for (size_t v = tid; v < n; v += kBlock) {
+            st.d[v] = kInf;
+            st.sd[v] = make_double2(0.0, 0.0);
         }
-        if (tid == 0) bytes += 20ull * n;
+        if (tid == 0) bytes += 20ull * n;  // d, sigma, delta initialised
         __syncthreads();
         if (tid == 0) {
-            dr[s] = 0;
-            sdr[s] = make_double2(1.0, 0.0);
+            st.d[s] = 0;
+            st.sd[s].x = 1.0;
             order[0] = s;
             loff[0] = 0;
             loff[1] = 1;
@@ -65,12 +61,12 @@ __global__ void __launch_bounds__(kBlock, 2) static_kernel(StaticArgs a) {
         // Stage 2: level-synchronous BFS; level L's sigma pull fused with the
         // discovery of level L+1 (one scan of each row).
         int L = 0, lb = 0, le = 1, nl = 1;
-        auto fwd_visit = [&](int x, int dx, double2 sv) -> double {
+        auto fwd_visit = [&](int x, int dx, double sx) -> double {
             if (dx == L - 1) {
-                bytes += 8;
-                return sv.x;
+                bytes += 8;  // sigma of a predecessor
+                return sx;
             }
-            if (dx == kInf && atomicCAS(dr + x, kInf, L + 1) == kInf) {
+            if (dx == kInf && atomicCAS(st.d + x, kInf, L + 1) == kInf) {
                 order[atomicAdd(&s_tail, 1)] = x;
                 bytes += 4;
             }
@@ -79,7 +75,7 @@ __global__ void __launch_bounds__(kBlock, 2) static_kernel(StaticArgs a) {
         auto fwd_finish = [&](int v, double sum) {
             bytes += 8;
             if (L > 0) {
-                sdr[v].x = sum;
+                st.sd[v].x = sum;
                 bytes += 8;
                 if (!(sum <= 1.7976931348623157e308)) atomicOr(a.err, kErrNumeric);
             }
@@ -87,12 +83,11 @@ __global__ void __launch_bounds__(kBlock, 2) static_kernel(StaticArgs a) {
         while (lb < le) {
             split_pass(
                 le - lb, g, INT32_MAX, [&](int i, int &v) { v = order[lb + i]; return true; },
-                [&](int, int) { return true; },
                 [&](int, int v, int2 r) {
                     double sum = 0.0;  // canonical order
-                    row_walk(g, dr, sdr, r, [&](int dx) { return dx == L - 1; },
-                             [&](int x, int dx, double2 sv) { sum += fwd_visit(x, dx, sv); });
-                    bytes += 8ull * (r.y - r.x);
+                    row_walk(g, st, nullptr, r, [&](int dx) { return dx == L - 1; },
+                             [&](int x, int dx, double2 q, uint32_t) { sum += fwd_visit(x, dx, q.x); });
+                    bytes += 8 + 8ull * (r.y - r.x);  // row bounds, col + d per entry
                     fwd_finish(v, sum);
                 },
                 enq);
@@ -102,10 +97,9 @@ __global__ void __launch_bounds__(kBlock, 2) static_kernel(StaticArgs a) {
                 const int m = min(kBig, nbig - r0);
                 big_load(S, m, [&](int t) { return Bq[r0 + t]; }, [&](int i) { return order[lb + i]; },
                          g, INT32_MAX);
-                big_entries(S, g, dr, [&](int, int x, int dx) {
+                big_entries(S, g, st, [&](int dx) { return dx == L - 1; }, [&](int, int x, int dx, double2 q) {
                     bytes += 8;
-                    const double2 sv = (dx == L - 1) ? ldcg_d2(sdr + x) : make_double2(0.0, 0.0);
-                    return fwd_visit(x, dx, sv);
+                    return fwd_visit(x, dx, q.x);
                 });
                 if (tid < m) {
                     double sum = S.acc[tid];
@@ -115,7 +109,7 @@ __global__ void __launch_bounds__(kBlock, 2) static_kernel(StaticArgs a) {
                         sum = 0.0;
                         for (int j = r.x; j < r.y; ++j) {
                             const int x = ldg_i(g.col + j);
-                            if (ldcg_i(dr + x) == L - 1) sum += ldcg_d2(sdr + x).x;
+                            if (st.dist(x) == L - 1) sum += st.sd[x].x;
                         }
                     }
                     fwd_finish(v, sum);
@@ -140,25 +134,24 @@ __global__ void __launch_bounds__(kBlock, 2) static_kernel(StaticArgs a) {
         // BC partial += delta (Eq. (3)), root excluded (delta_s(s) = 0).
         for (int lev = nl - 2; lev >= 1; --lev) {
             const int b0 = loff[lev], b1 = loff[lev + 1];
-            auto bwd_visit = [&](double sv, int y, int dy, double2 t) -> double {
+            auto bwd_visit = [&](double sv, int dy, double sy, double dly) -> double {
                 if (dy != lev + 1) return 0.0;
-                bytes += 16;
-                return __dmul_rn(__ddiv_rn(sv, t.x), __dadd_rn(1.0, t.y));
+                bytes += 16;  // sigma, delta of a successor
+                return __dmul_rn(__ddiv_rn(sv, sy), __dadd_rn(1.0, dly));
             };
             auto bwd_finish = [&](int v, double acc) {
-                sdr[v].y = acc;
+                st.sd[v].y = acc;
                 atomicAdd(a.bc + v, acc);
                 bytes += 8 + 8 + 16;
             };
             split_pass(
                 b1 - b0, g, INT32_MAX, [&](int i, int &v) { v = order[b0 + i]; return true; },
-                [&](int, int) { return true; },
                 [&](int, int v, int2 r) {
-                    const double sv = ldcg_d2(sdr + v).x;
+                    const double sv = st.sd[v].x;
                     double acc = 0.0;
-                    row_walk(g, dr, sdr, r, [&](int dy) { return dy == lev + 1; },
-                             [&](int y, int dy, double2 t) { acc += bwd_visit(sv, y, dy, t); });
-                    bytes += 8ull * (r.y - r.x);
+                    row_walk(g, st, nullptr, r, [&](int dy) { return dy == lev + 1; },
+                             [&](int, int dy, double2 q, uint32_t) { acc += bwd_visit(sv, dy, q.x, q.y); });
+                    bytes += 8 + 8 + 8ull * (r.y - r.x);
                     bwd_finish(v, acc);
                 },
                 enq);
@@ -168,12 +161,11 @@ __global__ void __launch_bounds__(kBlock, 2) static_kernel(StaticArgs a) {
                 const int m = min(kBig, nbig - r0);
                 big_load(S, m, [&](int t) { return Bq[r0 + t]; }, [&](int i) { return order[b0 + i]; },
                          g, INT32_MAX);
-                if (tid < m) S.c0[tid] = ldcg_d2(sdr + S.v[tid]).x;
+                if (tid < m) S.c0[tid] = st.sd[S.v[tid]].x;
                 __syncthreads();
-                big_entries(S, g, dr, [&](int t, int y, int dy) {
+                big_entries(S, g, st, [&](int dy) { return dy == lev + 1; }, [&](int t, int, int dy, double2 q) {
                     bytes += 8;
-                    const double2 sv = (dy == lev + 1) ? ldcg_d2(sdr + y) : make_double2(0.0, 0.0);
-                    return bwd_visit(S.c0[t], y, dy, sv);
+                    return bwd_visit(S.c0[t], dy, q.x, q.y);
                 });
                 if (tid < m) bwd_finish(S.v[tid], S.acc[tid]);
                 __syncthreads();

@@ -37,29 +37,32 @@
 
 namespace dbc {
 
-constexpr int kSrcR = 0x40000000;  // back-queue tag: item is a removal-push target
+// per-phase timers (diagnostic; %globaltimer reads sit on thread 0's critical
+// path, so they are compiled in only with -DDBC_PHASE_TIMERS)
+#ifdef DBC_PHASE_TIMERS
+constexpr bool kPhaseTimers = true;
+#else
+constexpr bool kPhaseTimers = false;
+#endif
 
 __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
     __shared__ int s_slot;
-    __shared__ int s_dcnt;   // |D| (absolute positions in Dv)
-    __shared__ int s_ucnt;   // next up frontier size
-    __shared__ int s_rcnt;   // |R|
-    __shared__ int s_rmax;   // deepest removal-push target level
-    __shared__ int s_nbig, s_nbig2;      // big-row queue (front: D rows, back: U/R rows)
-    __shared__ int s_nbig3;              // level-2 up rows resolved against adj(root)
-    __shared__ int s_ds;                 // |adj(root)| as of the insertion (-1: too long)
-    __shared__ int s_adjs[kAdjCap];      // adj(root) = the level-1 vertices
-    __shared__ int s_adjdeg[kAdjCap];    // their degrees
-    __shared__ ChunkSmem I;              // items of the current up-phase chunk
-    __shared__ int s_l1[kChunk];         // chunk slots resolved against adj(root)
-    __shared__ int s_nl1;
-    __shared__ int s_nbigI;              // long rows of the current level in I
-    __shared__ int s_un[2][kUcap];       // up frontier ping-pong (overflow: Ua / Ub)
+    __shared__ int s_dcnt;     // |D| (absolute positions in Dv)
+    __shared__ int s_ucnt;     // next up frontier size
+    __shared__ int s_rcnt;     // |R|
+    __shared__ int s_rmax;     // deepest removal-push target level
+    __shared__ int s_nbig;     // long-row queue (down phase / removal)
+    __shared__ int s_nbigI;    // long rows of the current up level (in I)
+    __shared__ int s_nl1;      // of those, resolved against adj(root)
+    __shared__ int s_ds;       // |adj(root)| as of the insertion (-1: too long)
     __shared__ uint32_t s_work[kWarps];  // window classification bits (1 = Case 2/3)
     __shared__ int s_job[4];             // uh, ul, L0, case3 of the current job
     __shared__ BigSmem S;
-    __shared__ double s_c2[kBig];
-    __shared__ int s_f0[kBig];
+    __shared__ ChunkSmem I;              // long rows of the current up level
+    __shared__ int s_l1[kChunk];
+    __shared__ int s_adjs[kAdjCap];      // adj(root) = the level-1 vertices
+    __shared__ int s_adjdeg[kAdjCap];    // their degrees
+    __shared__ int s_un[2][kUcap];       // up frontier ping-pong (overflow: U0 / U1)
 
     const int tid = threadIdx.x;
     const int wk = blockIdx.x;
@@ -76,34 +79,28 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
     int32_t *Ub = a.ws.U1 + (size_t)wk * n;
     int32_t *Rv = a.ws.Rv + (size_t)wk * n;
     int32_t *Rl = a.ws.Rl + (size_t)wk * n;
-    int32_t *Bq = a.ws.Bq + (size_t)wk * 2 * n;
+    int32_t *Bq = a.ws.Bq + (size_t)wk * n;
     uint32_t epoch = a.ws.wepoch[wk];
     const GView &g = a.g;
 
     unsigned long long st_bytes = 0, st_touched = 0, st_down = 0;
-    unsigned long long sc_down = 0, sc_rem = 0, sc_dpull = 0, sc_dpush = 0, sc_up2 = 0, sc_up3 = 0;
     unsigned long long st_c1 = 0, st_c2 = 0, st_c3 = 0, st_lvd = 0, st_lvu = 0;
-    // per-phase wall time seen by thread 0 (diagnostic): down, removal, up-split, up-big, up-L1, up-level-end
+    unsigned long long sc_down = 0, sc_rem = 0, sc_dpull = 0, sc_dpush = 0, sc_up2 = 0, sc_up3 = 0;
+    // per-phase wall time seen by thread 0 (diagnostic)
     unsigned long long tm_ph[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
     unsigned long long tclk = 0;
     auto tick = [&](int ph) {
-        if (tid == 0) {
+        if (kPhaseTimers && tid == 0) {
             unsigned long long t;
             asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
             if (ph >= 0) tm_ph[ph] += t - tclk;
             tclk = t;
         }
     };
-
-    auto enq_front = [&](int idx, int, int2) { Bq[atomicAdd(&s_nbig, 1)] = idx; };
-    auto enq_back = [&](int idx) { Bq[n - 1 - atomicAdd(&s_nbig2, 1)] = idx; };
-    auto enq_l1 = [&](int idx) { Bq[n + atomicAdd(&s_nbig3, 1)] = idx; };
-    auto fetch_front = [&](int r0) { return [=](int t) { return Bq[r0 + t]; }; };
+    auto enq_front = [&](int idx) { Bq[atomicAdd(&s_nbig, 1)] = idx; };
 
     if (tid == 0) {
         s_nbig = 0;
-        s_nbig2 = 0;
-        s_nbig3 = 0;
         s_nbigI = 0;
         s_nl1 = 0;
     }
@@ -114,8 +111,7 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
         const int slot = s_slot;
         __syncthreads();
         if (slot >= a.k_loc) break;
-        int32_t *dr = a.d + (size_t)slot * n;
-        double2 *sdr = a.sd + (size_t)slot * n;
+        const Root st{a.d + (size_t)slot * n, a.sd + (size_t)slot * n};
         const int sroot = a.roots[slot];
         unsigned long long prof_t0 = 0, prof_jobs = 0, prof_touch0 = st_touched;
         if (a.root_prof && tid == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(prof_t0));
@@ -132,7 +128,7 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                 bool work = false;
                 if (j < wend) {
                     const int u = __ldg(a.ins_u + j), v = __ldg(a.ins_v + j);
-                    work = ldcg_i(dr + u) != ldcg_i(dr + v);
+                    work = st.dist(u) != st.dist(v);
                 }
                 const unsigned bal = __ballot_sync(kFull, work);
                 if ((tid & 31) == 0) s_work[tid >> 5] = bal;
@@ -155,7 +151,7 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                 const uint32_t mD = E | kDown, mU = E | kUp;
                 if (tid == 0) {
                     const int u = __ldg(a.ins_u + p), v = __ldg(a.ins_v + p);
-                    const int du = ldcg_i(dr + u), dv = ldcg_i(dr + v);
+                    const int du = st.dist(u), dv = st.dist(v);
                     const bool u_is_high = du < dv;
                     const int uh = u_is_high ? u : v, ul = u_is_high ? v : u;
                     const int dh = u_is_high ? du : dv, dlo = u_is_high ? dv : du;
@@ -168,7 +164,7 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                     st_bytes += 8;
                     if (c3) {
                         lowrec[ul] = ((unsigned long long)epoch << 32) | (uint32_t)dlo;
-                        dr[ul] = L0;
+                        st.d[ul] = L0;
                     }
                     mark[ul] = mD;
                     Dv[0] = ul;
@@ -193,22 +189,22 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                 int L = L0, lb = 0, le = 1, nlev = 1;
                 // per-D-entry epilogue: record old d / sigma, store the new sigma
                 auto down_finish = [&](int idx, int w, double sum) {
-                    const unsigned long long lr = ldcg_ull(lowrec + w);
+                    const unsigned long long lr = lowrec[w];
                     const int od = ((uint32_t)(lr >> 32) == epoch) ? (int)(uint32_t)lr : L;
                     Dold[idx] = od;
-                    Dsig[idx] = ldcg_d2(sdr + w).x;
-                    sdr[w].x = sum;
+                    Dsig[idx] = st.sd[w].x;
+                    st.sd[w].x = sum;
                     if (!(sum <= 1.7976931348623157e308)) atomicOr(a.err, kErrNumeric);
                     st_bytes += 8 + 8 + 20;
                 };
                 // one neighbour y of a level-L vertex; returns sigma[y] if y is a predecessor
-                auto down_visit = [&](int y, int dy, double2 sv) -> double {
+                auto down_visit = [&](int y, int dy, double sy) -> double {
                     if (dy == L - 1) {
                         st_bytes += 8;
-                        return sv.x;
+                        return sy;
                     }
                     if (dy > L + 1) {  // Case 3 pull-up
-                        const int old = atomicMin(dr + y, L + 1);
+                        const int old = atomicMin(st.d + y, L + 1);
                         if (old > L + 1) {
                             lowrec[y] = ((unsigned long long)epoch << 32) | (uint32_t)old;
                             st_bytes += 4;
@@ -222,11 +218,10 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                 while (true) {
                     split_pass(
                         le - lb, g, lim, [&](int i, int &w) { w = Dv[lb + i]; return true; },
-                        [&](int, int) { return true; },
                         [&](int i, int w, int2 r) {
                             double sum = 0.0;  // canonical order: bit-exact
-                            row_walk(g, dr, sdr, r, [&](int dy) { return dy == L - 1; },
-                                     [&](int y, int dy, double2 sv) { sum += down_visit(y, dy, sv); });
+                            row_walk(g, st, nullptr, r, [&](int dy) { return dy == L - 1; },
+                                     [&](int y, int dy, double2 q, uint32_t) { sum += down_visit(y, dy, q.x); });
                             st_bytes += 8 + 8ull * (r.y - r.x);
                             sc_down += r.y - r.x;
                             down_finish(lb + i, w, sum);
@@ -236,13 +231,14 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                     const int nbig = s_nbig;
                     for (int r0 = 0; r0 < nbig; r0 += kBig) {
                         const int m = min(kBig, nbig - r0);
-                        big_load(S, m, fetch_front(r0), [&](int i) { return Dv[lb + i]; }, g, lim);
-                        big_entries(S, g, dr, [&](int, int y, int dy) {
-                            st_bytes += 8;
-                            sc_down++;
-                            const double2 sv = (dy == L - 1) ? ldcg_d2(sdr + y) : make_double2(0.0, 0.0);
-                            return down_visit(y, dy, sv);
-                        });
+                        big_load(S, m, [&](int t) { return Bq[r0 + t]; }, [&](int i) { return Dv[lb + i]; },
+                                 g, lim);
+                        big_entries(S, g, st, [&](int dy) { return dy == L - 1; },
+                                    [&](int, int y, int dy, double2 q) {
+                                        st_bytes += 8;
+                                        sc_down++;
+                                        return down_visit(y, dy, q.x);
+                                    });
                         if (tid < m) {
                             double sum = S.acc[tid];
                             const int w = S.v[tid];
@@ -251,7 +247,7 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                                 sum = 0.0;
                                 for (int j = r.x; j < r.y; ++j) {
                                     const int y = ldg_i(g.col + j);
-                                    if (ldcg_i(dr + y) == L - 1) sum += ldcg_d2(sdr + y).x;
+                                    if (st.dist(y) == L - 1) sum += st.sd[y].x;
                                 }
                             }
                             st_bytes += 8;
@@ -274,23 +270,21 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                 }
                 // D levels: level L0 + j occupies Dv[Doff[j] .. Doff[j+1]), j < nlev
                 const int LmaxD = L0 + nlev - 1;
-                st_lvd += nlev;
                 const int dtotal = le;
+                st_lvd += nlev;
                 if (tid == 0) {
                     st_down += dtotal;
                     st_touched += dtotal;
                 }
-                __syncthreads();
 
                 tick(0);
                 // ================= (0) Case-3 removal pushes =================
                 if (case3) {
                     // a pulled-up w (finite old level od) loses its old predecessors x
                     auto rem_visit = [&](int w, int od, double osig, double coef, int x, int dx,
-                                         double2 sv) {
+                                         double sx) {
                         if (dx != od - 1 || (x == uh && w == ul)) return;
-                        if (ldcg_u(mark + x) == mD) return;
-                        const double sx = sv.x;
+                        if (mark[x] == mD) return;
                         atomicAdd(dacc + x, -__dmul_rn(__ddiv_rn(sx, osig), coef));
                         st_bytes += 24;
                         if (atomicMax(mark + x, mU) < E) {
@@ -305,15 +299,16 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                         [&](int i, int &w) {
                             const int od = Dold[i];
                             w = Dv[i];
-                            return od != kInf && od != ldcg_i(dr + w);
+                            return od != kInf && od != st.dist(w);
                         },
-                        [&](int, int) { return true; },
                         [&](int i, int w, int2 r) {
                             const int od = Dold[i];
                             const double osig = Dsig[i];
-                            const double coef = 1.0 + ldcg_d2(sdr + w).y;  // delta still old
-                            row_walk(g, dr, sdr, r, [&](int dx) { return dx == od - 1; },
-                                     [&](int x, int dx, double2 sv) { rem_visit(w, od, osig, coef, x, dx, sv); });
+                            const double coef = 1.0 + st.sd[w].y;  // delta still old
+                            row_walk(g, st, nullptr, r, [&](int dx) { return dx == od - 1; },
+                                     [&](int x, int dx, double2 q, uint32_t) {
+                                         rem_visit(w, od, osig, coef, x, dx, q.x);
+                                     });
                             st_bytes += 16 + 8ull * (r.y - r.x);
                             sc_rem += r.y - r.x;
                         },
@@ -322,20 +317,20 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                     const int nbig = s_nbig;
                     for (int r0 = 0; r0 < nbig; r0 += kBig) {
                         const int m = min(kBig, nbig - r0);
-                        big_load(S, m, fetch_front(r0), [&](int i) { return Dv[i]; }, g, lim);
+                        big_load(S, m, [&](int t) { return Bq[r0 + t]; }, [&](int i) { return Dv[i]; },
+                                 g, lim);
                         if (tid < m) {
                             const int i = S.idx[tid];
-                            s_f0[tid] = Dold[i];
                             S.c0[tid] = Dsig[i];
-                            S.c1[tid] = 1.0 + ldcg_d2(sdr + S.v[tid]).y;
+                            s_l1[tid] = Dold[i];  // reused: old level of each row
                             st_bytes += 16;
                         }
                         __syncthreads();
-                        big_entries(S, g, dr, [&](int t, int x, int dx) {
+                        big_entries(S, g, st, [](int) { return true; }, [&](int t, int x, int dx, double2 q) {
                             st_bytes += 8;
                             sc_rem++;
-                            const double2 sv = (dx == s_f0[t] - 1) ? ldcg_d2(sdr + x) : make_double2(0.0, 0.0);
-                            rem_visit(S.v[t], s_f0[t], S.c0[t], S.c1[t], x, dx, sv);
+                            const int w = S.v[t];
+                            rem_visit(w, s_l1[t], S.c0[t], 1.0 + st.sd[w].y, x, dx, q.x);
                             return 0.0;
                         });
                     }
@@ -368,30 +363,26 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                             Unext[pos - kUcap] = y;
                     };
                     // up vertex x (not in D): push sigma[p]/sigma[x] * Ddelta[x] upwards
-                    auto up_visit = [&](double gx, double sx, int pp, int dp, double2 sv, uint32_t mp) {
-                        if (dp != l - 1) return;
-                        const double sp = sv.x;
+                    auto up_visit = [&](double gx, double sx, int pp, double sp, uint32_t mp) {
                         atomicAdd(dacc + pp, __dmul_rn(__ddiv_rn(sp, sx), gx));
                         st_bytes += 24;
                         claim_up(pp, mp);
                     };
                     auto up_finish = [&](int x, double gx, double odel) {
                         dacc[x] = 0.0;
-                        sdr[x].y = odel + gx;
+                        st.sd[x].y = odel + gx;
                         atomicAdd(a.bc + x, gx);
                         st_bytes += 8 + 8 + 16 + 16;
                     };
                     // down vertex x: pull delta (Eq. (2)), then push new-minus-old contributions
-                    auto dpull_visit = [&](double sx, int y, int dy, double2 t) -> double {
+                    auto dpull_visit = [&](double sx, int dy, double sy, double dly) -> double {
                         if (dy != l + 1) return 0.0;
                         st_bytes += 16;
-                        return __dmul_rn(__ddiv_rn(sx, t.x), __dadd_rn(1.0, t.y));
+                        return __dmul_rn(__ddiv_rn(sx, sy), __dadd_rn(1.0, dly));
                     };
                     auto dpush_visit = [&](int x, double sx, double dn, double odel, double osig,
-                                           bool not_pulled, int pp, int dp, double2 sv, uint32_t mp) {
-                        if (dp != l - 1) return;
+                                           bool not_pulled, int pp, double sp, uint32_t mp) {
                         if (mp == mD) return;
-                        const double sp = sv.x;
                         double dlt = __dmul_rn(__ddiv_rn(sp, sx), 1.0 + dn);
                         if (not_pulled && !(pp == uh && x == ul))
                             dlt = __dsub_rn(dlt, __dmul_rn(__ddiv_rn(sp, osig), 1.0 + odel));
@@ -400,7 +391,7 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                         claim_up(pp, mp);
                     };
                     auto d_finish = [&](int x, double dn, double odel) {
-                        sdr[x].y = dn;
+                        st.sd[x].y = dn;
                         atomicAdd(a.bc + x, dn - odel);
                         st_bytes += 8 + 16 + 16;
                     };
@@ -429,22 +420,19 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                     }
                     tick(2);
                     // Items of level l: the down segment, then the up frontier, then
-                    // removal targets.  Short rows are handled completely by their
-                    // lane (prep, pull, push, epilogue); long rows are collected in
-                    // shared memory and processed by the flattened chunk pass.
+                    // removal targets.  resolve() issues everything an item needs as
+                    // one round of independent loads.
                     auto resolve = [&](int q, int &x, int &meta, double &c0, double &c1, double &c2,
-                                       int2 &r, bool &need) {
-                        // returns false for an inactive item
+                                       int2 &r) -> bool {
                         if (q < nDl) {
                             const int idx = b0 + q;
                             x = Dv[idx];
-                            const double2 s2 = ldcg_d2(sdr + x);
-                            c0 = s2.x;  // sigma (new)
-                            c1 = s2.y;  // delta (old)
+                            const double2 s2 = st.sd[x];
+                            c0 = s2.x;                // sigma (new)
+                            c1 = s2.y;                // delta (old)
                             c2 = Dsig[idx];
                             meta = (Dold[idx] == l) ? kMetaNotPulled : 0;
                             r = row_of(g, x, lim);
-                            need = true;
                             st_bytes += 8 + 16 + 8 + 4;
                             return true;
                         }
@@ -455,25 +443,28 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                         else if (Rl[qi - ucnt] == l)
                             x = Rv[qi - ucnt];
                         if (x < 0) return false;
-                        // first claimant processes the vertex (drops duplicates)
-                        if (atomicMax(mark + x, E | 3u) != mU) return false;
+                        // the dedup claim and the loads are issued together
+                        const uint32_t prev = atomicMax(mark + x, E | kUpDone);
+                        const double gx = dacc[x];  // Ddelta (complete: level l+1 is done)
+                        const double2 s2 = st.sd[x];
+                        const double sx = s2.x, odl = s2.y;
+                        const int2 rr = push ? row_of(g, x, lim) : make_int2(0, 0);
+                        if (prev != mU) return false;  // a duplicate: the first claimant processes
                         meta = kMetaUp;
-                        c1 = ldcg_d(dacc + x);  // Ddelta (complete: level l+1 is done)
-                        const double2 s2 = ldcg_d2(sdr + x);
-                        c0 = s2.x;
-                        c2 = s2.y;
+                        c0 = sx;
+                        c1 = gx;
+                        c2 = odl;
                         st_bytes += 24;
-                        need = push && c1 != 0.0;
-                        r = need ? row_of(g, x, lim) : make_int2(0, 0);
+                        r = (push && gx != 0.0) ? rr : make_int2(0, 0);
                         return true;
                     };
                     auto inlane = [&](int x, int meta, double c0, double c1, double c2, int2 r) {
                         const bool wantpush = push && r.y > r.x;
                         if (meta & kMetaUp) {
                             if (wantpush) {
-                                row_walk(g, dr, sdr, r, [&](int dp) { return dp == l - 1; },
-                                         [&](int pp, int dp, double2 sv) {
-                                             if (dp == l - 1) up_visit(c1, c0, pp, dp, sv, ldcg_u(mark + pp));
+                                row_walk(g, st, mark, r, [&](int dp) { return dp == l - 1; },
+                                         [&](int pp, int dp, double2 q, uint32_t mp) {
+                                             if (dp == l - 1) up_visit(c1, c0, pp, q.x, mp);
                                          });
                                 (l == 2 ? sc_up2 : sc_up3) += r.y - r.x;
                                 st_bytes += 8 + 8ull * (r.y - r.x);
@@ -481,18 +472,18 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                             up_finish(x, c1, c2);
                         } else {
                             double dn = 0.0;
-                            row_walk(g, dr, sdr, r, [&](int dy) { return dy == l + 1; },
-                                     [&](int y, int dy, double2 sv) { dn += dpull_visit(c0, y, dy, sv); });
+                            row_walk(g, st, nullptr, r, [&](int dy) { return dy == l + 1; },
+                                     [&](int, int dy, double2 q, uint32_t) { dn += dpull_visit(c0, dy, q.x, q.y); });
                             sc_dpull += r.y - r.x;
                             st_bytes += 8ull * (r.y - r.x);
                             if (wantpush) {
-                                row_walk(g, dr, sdr, r, [&](int dp) { return dp == l - 1; },
-                                         [&](int pp, int dp, double2 sv) {
+                                row_walk(g, st, mark, r, [&](int dp) { return dp == l - 1; },
+                                         [&](int pp, int dp, double2 q, uint32_t mp) {
                                              if (dp == l - 1)
-                                                 dpush_visit(x, c0, dn, c1, c2, (meta & kMetaNotPulled) != 0,
-                                                             pp, dp, sv, ldcg_u(mark + pp));
+                                                 dpush_visit(x, c0, dn, c1, c2, (meta & kMetaNotPulled) != 0, pp,
+                                                             q.x, mp);
                                          });
-                                (l == 2 ? sc_up2 : sc_up3) += r.y - r.x;
+                                sc_dpush += r.y - r.x;
                                 st_bytes += 8ull * (r.y - r.x);
                             }
                             d_finish(x, dn, c1);
@@ -503,8 +494,7 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                             int x, meta = 0;
                             double c0 = 0.0, c1 = 0.0, c2 = 0.0;
                             int2 r = make_int2(0, 0);
-                            bool need = false;
-                            if (!resolve(q, x, meta, c0, c1, c2, r, need)) continue;
+                            if (!resolve(q, x, meta, c0, c1, c2, r)) continue;
                             const int len = r.y - r.x;
                             if (small_inlane && len <= kSmallDeg) {
                                 inlane(x, meta, c0, c1, c2, r);
@@ -537,84 +527,83 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
                     const bool small_level = total <= kBlock;
                     const int step = small_level ? total : kChunk;
                     for (int cb = 0; cb < total; cb += step) {
-                    const int ce = min(total, cb + step);
-                    split_range(cb, min(ce, nDl), small_level);  // down rows first: pull precedes push
-                    __syncthreads();
-                    const int nDb = min(s_nbigI, kChunk);
-                    split_range(max(cb, nDl), ce, small_level);
-                    __syncthreads();
-                    const int nb = min(s_nbigI, kChunk);
-                    if (nb > 0) {
-                        chunk_scan(I.off, nb);  // off[0..nb], ends with a barrier
-                        // --- C1: delta pull of the long down rows (Eq. (2)) ---
-                        const int E1 = I.off[nDb], E = I.off[nb];
-                        if (E1 > 0)
-                            flat_entries(I.off, nb, E1, [&](int t, int e) { return ldg_i(g.col + I.beg[t] + e - I.off[t]); },
-                                         dr, I.acc, [&](int t, int y, int dy) -> double {
-                                             sc_dpull++;
-                                             st_bytes += 8;
-                                             if (dy != l + 1) return 0.0;
-                                             return dpull_visit(I.c0[t], y, dy, ldcg_d2(sdr + y));
-                                         });
-                        // --- C2: pushes towards level l-1 ---
-                        if (push && E > 0)
-                            flat_entries(I.off, nb, E, [&](int t, int e) { return ldg_i(g.col + I.beg[t] + e - I.off[t]); },
-                                         dr, nullptr, [&](int t, int pp, int dp) -> double {
-                                             (l == 2 ? sc_up2 : sc_up3)++;
-                                             st_bytes += 8;
-                                             if (dp != l - 1) return 0.0;
-                                             const double2 sv = ldcg_d2(sdr + pp);
-                                             const uint32_t mp = ldcg_u(mark + pp);
-                                             const int meta = I.meta[t];
-                                             if (meta & kMetaUp)
-                                                 up_visit(I.c1[t], I.c0[t], pp, dp, sv, mp);
-                                             else
-                                                 dpush_visit(I.v[t], I.c0[t], I.acc[t], I.c1[t], I.c2[t],
-                                                             (meta & kMetaNotPulled) != 0, pp, dp, sv, mp);
-                                             return 0.0;
-                                         });
-                        // --- C3: level-2 rows resolved against adj(root) ---
-                        const int nl1 = s_nl1;
-                        if (nl1 > 0) {
-                            const int ds = s_ds, npairs = nl1 * ds;
-                            for (int qq = tid; qq < npairs; qq += kBlock) {
-                                const int li = qq / ds, j = qq - li * ds;
-                                const int t = s_l1[li];
-                                const int x = I.v[t], pp = s_adjs[j];
-                                const int degx = (ldg_i(g.rp + x + 1) & kMask) - (ldg_i(g.rp + x) & kMask);
-                                const bool adj = (s_adjdeg[j] < degx) ? adjacent_visible(g, pp, x, lim)
-                                                                      : adjacent_visible(g, x, pp, lim);
-                                st_bytes += 32;
-                                if (adj) up_visit(I.c1[t], I.c0[t], pp, 1, ldcg_d2(sdr + pp), ldcg_u(mark + pp));
+                        const int ce = min(total, cb + step);
+                        split_range(cb, min(ce, nDl), small_level);  // down rows first: pull precedes push
+                        __syncthreads();
+                        const int nDb = min(s_nbigI, kChunk);
+                        split_range(max(cb, nDl), ce, small_level);
+                        __syncthreads();
+                        tick(6);
+                        const int nb = min(s_nbigI, kChunk);
+                        if (nb > 0) {
+                            chunk_scan(I.off, nb);  // off[0..nb], ends with a barrier
+                            tick(7);
+                            auto colf = [&](int t, int e) { return ldg_i(g.col + I.beg[t] + e - I.off[t]); };
+                            // --- C1: delta pull of the long down rows (Eq. (2)) ---
+                            const int E1 = I.off[nDb], E2 = I.off[nb];
+                            if (E1 > 0)
+                                flat_entries(I.off, nb, E1, colf, st, nullptr, [&](int dy) { return dy == l + 1; },
+                                             I.acc, [&](int t, int, int dy, double2 q, uint32_t) {
+                                                 sc_dpull++;
+                                                 st_bytes += 8;
+                                                 return dpull_visit(I.c0[t], dy, q.x, q.y);
+                                             });
+                            tick(8);
+                            // --- C2: pushes towards level l-1 ---
+                            if (push && E2 > 0)
+                                flat_entries(
+                                    I.off, nb, E2, colf, st, mark, [&](int dp) { return dp == l - 1; }, nullptr,
+                                    [&](int t, int pp, int dp, double2 q, uint32_t mp) -> double {
+                                        const double sp = q.x;
+                                        (l == 2 ? sc_up2 : sc_up3)++;
+                                        st_bytes += 8;
+                                        if (dp != l - 1) return 0.0;
+                                        const int meta = I.meta[t];
+                                        if (meta & kMetaUp)
+                                            up_visit(I.c1[t], I.c0[t], pp, sp, mp);
+                                        else
+                                            dpush_visit(I.v[t], I.c0[t], I.acc[t], I.c1[t], I.c2[t],
+                                                        (meta & kMetaNotPulled) != 0, pp, sp, mp);
+                                        return 0.0;
+                                    });
+                            tick(9);
+                            // --- C3: level-2 rows resolved against adj(root) ---
+                            const int nl1 = s_nl1;
+                            if (nl1 > 0) {
+                                const int ds = s_ds, npairs = nl1 * ds;
+                                for (int qq = tid; qq < npairs; qq += kBlock) {
+                                    const int li = qq / ds, j = qq - li * ds;
+                                    const int t = s_l1[li];
+                                    const int x = I.v[t], pp = s_adjs[j];
+                                    const int degx = (ldg_i(g.rp + x + 1) & kMask) - (ldg_i(g.rp + x) & kMask);
+                                    const bool adj = (s_adjdeg[j] < degx) ? adjacent_visible(g, pp, x, lim)
+                                                                          : adjacent_visible(g, x, pp, lim);
+                                    st_bytes += 32;
+                                    if (adj) up_visit(I.c1[t], I.c0[t], pp, st.sd[pp].x, mark[pp]);
+                                }
+                                __syncthreads();
+                            }
+                            tick(4);
+                            // --- epilogue of the long rows (Alg. 8 fused) ---
+                            for (int t = tid; t < nb; t += kBlock) {
+                                if (I.meta[t] & kMetaUp)
+                                    up_finish(I.v[t], I.c1[t], I.c2[t]);
+                                else
+                                    d_finish(I.v[t], I.acc[t], I.c1[t]);
                             }
                             __syncthreads();
                         }
-                        // --- epilogue of the long rows (Alg. 8 fused) ---
-                        for (int t = tid; t < nb; t += kBlock) {
-                            if (I.meta[t] & kMetaUp)
-                                up_finish(I.v[t], I.c1[t], I.c2[t]);
-                            else
-                                d_finish(I.v[t], I.acc[t], I.c1[t]);
+                        if (tid == 0) {
+                            s_nbigI = 0;
+                            s_nl1 = 0;
                         }
                         __syncthreads();
-                    }
-                    if (tid == 0) {
-                        s_nbigI = 0;
-                        s_nl1 = 0;
-                    }
-                    __syncthreads();
                     }  // chunks
                     tick(3);
-                    tick(4);
                     ucnt = s_ucnt;
                     __syncthreads();
                     if (tid == 0) {
                         s_ucnt = 0;
-                        s_nbigI = 0;
-                        s_nl1 = 0;
-                        s_nbig = 0;
-                        s_nbig2 = 0;
-                        s_nbig3 = 0;
                         st_touched += ucnt;
                     }
                     int *t = Ucur;

@@ -15,7 +15,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libdbc.so")
+LIB_PATH = os.environ.get("DBC_LIB_PATH") or os.path.join(_HERE, "libdbc.so")
 
 DBC_INF = 2**31 - 1
 FLAG_MODE_S = 0x1
@@ -108,6 +108,8 @@ def load_library():
             raise ImportError(f"{LIB_PATH} not built: run `python -c 'import __graft_entry__ as g; g.build()'`")
         lib = ctypes.CDLL(LIB_PATH)
         for name, (res, args) in SIGNATURES.items():
+            if name.startswith("dbc_debug_") and not hasattr(lib, name):
+                continue  # diagnostics are optional (older builds)
             f = getattr(lib, name)
             f.restype = res
             f.argtypes = args
@@ -253,8 +255,8 @@ class DynamicBC:
     def debug_counters(self):
         names = ["case1", "case2", "case3", "touched", "down", "scanned", "alg_bytes",
                  "static_bytes", "sc_down", "sc_removal", "sc_dpull", "sc_dpush", "sc_up2", "sc_up3",
-                 "ns_down", "ns_removal", "ns_up_setup", "ns_up_rest", "ns_x", "ns_up_end",
-                 "ns_up_prep", "ns_up_scan", "ns_up_pull", "ns_up_push", "levels_down", "levels_up"]
+                 "ns_down", "ns_removal", "ns_up_setup", "ns_up_epi", "ns_up_l1pairs", "ns_up_end",
+                 "ns_up_split", "ns_up_scan", "ns_up_pull", "ns_up_push", "levels_down", "levels_up"]
         out = np.zeros(len(names), dtype=np.int64)
         _check(self._ctx, self._lib.dbc_debug_counters(self._ctx, _np_ptr(out), out.size))
         return dict(zip(names, out.tolist()))

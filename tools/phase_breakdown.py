@@ -25,3 +25,5 @@ order = np.argsort(-dur)[:8]
 for i in order:
     print("slot", i, "root", wl.roots[i], "deg", g.degree()[wl.roots[i]], "ms %.2f" % dur[i], "jobs", prof[i,2], "touched", prof[i,3], "start %.2f" % ((prof[i,0]-prof[:,0].min())/1e6))
 print("jobs: median", np.median(prof[:,2]), "max", prof[:,2].max(), "touched/job median", np.median(prof[:,3]/np.maximum(prof[:,2],1)))
+st = (prof[:, 0] - prof[:, 0].min()) / 1e6
+print("root start ms: min %.2f median %.2f max %.2f; #late(>1ms) %d" % (st.min(), np.median(st), st.max(), (st > 1).sum()))
