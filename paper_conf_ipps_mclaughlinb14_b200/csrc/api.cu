@@ -5,6 +5,7 @@
 #include <algorithm>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <thread>
@@ -30,6 +31,7 @@ struct dbc_ctx {
     cudaStream_t stream = nullptr;
     bool own_stream = false;
     int workers = 0;
+    int block = 256;   // threads per worker CTA (256 or 128)
     int nsm = 148;
     bool have_state = false;
     uint64_t epoch_used = 0;
@@ -361,7 +363,13 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     cudaMemGetInfo(&free_b, &total_b);
     const size_t state_b = (size_t)c->k_loc * n * 20 + (size_t)c->col_cap * 8 + (size_t)n * 40;
     size_t budget = free_b > state_b ? (free_b - state_b) / 2 : 0;
-    int want = opt.workers ? opt.workers : 2 * c->nsm;
+    // more roots than two 256-thread CTAs per SM can hold and no hub rows:
+    // 128-thread CTAs, four per SM, so that every root chain is resident at once
+    int64_t maxdeg = 0;
+    for (int32_t v = 0; v < n; ++v) maxdeg = std::max<int64_t>(maxdeg, row_ptr[v + 1] - row_ptr[v]);
+    c->block = (c->k_loc > 2 * c->nsm && maxdeg <= 256) ? 128 : 256;  // hubs need the wide CTA
+    if (const char *eb = getenv("DBC_BLOCK")) c->block = (atoi(eb) == 128) ? 128 : 256;
+    int want = opt.workers ? opt.workers : (c->block == 128 ? 4 : 2) * c->nsm;
     want = std::min(want, c->k_loc);
     int fit = (int)std::min<size_t>(budget / per_worker, 1 << 20);
     c->workers = std::max(0, std::min(want, fit));
@@ -506,7 +514,10 @@ extern "C" dbc_status dbc_static_compute(dbc_ctx *c) {
         a.next_slot = c->next_slot;
         a.stats = c->stats;
         a.err = c->err;
-        launch_static(a, c->workers, c->stream);
+        if (c->block == 128)
+            launch_static_128(a, c->workers, c->stream);
+        else
+            launch_static_256(a, c->workers, c->stream);
         CK(cudaGetLastError());
     }
     if (tm) {
@@ -592,14 +603,20 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
                 CK(cudaMemsetAsync(c->next_slot, 0, sizeof(int32_t), c->stream));
                 a.ins_begin = (int32_t)i;
                 a.ins_end = (int32_t)i + 1;
-                launch_update(a, c->workers, c->stream);
+                if (c->block == 128)
+                    launch_update_128(a, c->workers, c->stream);
+                else
+                    launch_update_256(a, c->workers, c->stream);
                 ++ulaunch;
             }
         } else {
             CK(cudaMemsetAsync(c->next_slot, 0, sizeof(int32_t), c->stream));
             a.ins_begin = 0;
             a.ins_end = (int32_t)cnt;
-            launch_update(a, c->workers, c->stream);
+            if (c->block == 128)
+                launch_update_128(a, c->workers, c->stream);
+            else
+                launch_update_256(a, c->workers, c->stream);
             ++ulaunch;
         }
         CK(cudaGetLastError());

@@ -23,7 +23,13 @@
 
 namespace dbc {
 
-constexpr int kBlock = 256;              // threads per worker CTA
+// threads per worker CTA; the kernels are compiled once per value (Makefile):
+// 256 (2 CTAs/SM) for few roots with hub-heavy rows, 128 (4 CTAs/SM) when
+// there are more roots than 2 x #SMs (all root chains resident at once).
+#ifndef DBC_BLOCK
+#define DBC_BLOCK 256
+#endif
+constexpr int kBlock = DBC_BLOCK;
 constexpr int kWarps = kBlock / 32;
 constexpr int kSmallDeg = 32;            // rows <= this are walked by one lane
 constexpr uint32_t kFull = 0xffffffffu;
@@ -437,7 +443,9 @@ struct StaticArgs {
     int32_t *err;
 };
 
-void launch_update(const UpdateArgs &a, int workers, cudaStream_t s);
-void launch_static(const StaticArgs &a, int workers, cudaStream_t s);
+void launch_update_256(const UpdateArgs &a, int workers, cudaStream_t s);
+void launch_update_128(const UpdateArgs &a, int workers, cudaStream_t s);
+void launch_static_256(const StaticArgs &a, int workers, cudaStream_t s);
+void launch_static_128(const StaticArgs &a, int workers, cudaStream_t s);
 
 }  // namespace dbc

@@ -16,7 +16,8 @@
 
 namespace dbc {
 
-__global__ void __launch_bounds__(kBlock, 2) static_kernel(StaticArgs a) {
+namespace {
+__global__ void __launch_bounds__(kBlock, 512 / kBlock) static_kernel(StaticArgs a) {
     __shared__ int s_slot;
     __shared__ int s_tail;
     __shared__ int s_nbig;
@@ -178,7 +179,11 @@ __global__ void __launch_bounds__(kBlock, 2) static_kernel(StaticArgs a) {
     if (bytes) atomicAdd(a.stats + kStStaticBytes, bytes);
 }
 
-void launch_static(const StaticArgs &a, int workers, cudaStream_t s) {
+}  // namespace
+
+#define DBC_CAT2(a, b) a##b
+#define DBC_CAT(a, b) DBC_CAT2(a, b)
+void DBC_CAT(launch_static_, DBC_BLOCK)(const StaticArgs &a, int workers, cudaStream_t s) {
     static_kernel<<<workers, kBlock, 0, s>>>(a);
 }
 

@@ -45,7 +45,8 @@ constexpr bool kPhaseTimers = true;
 constexpr bool kPhaseTimers = false;
 #endif
 
-__global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
+namespace {
+__global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs a) {
     __shared__ int s_slot;
     __shared__ int s_dcnt;     // |D| (absolute positions in Dv)
     __shared__ int s_ucnt;     // next up frontier size
@@ -655,7 +656,11 @@ __global__ void __launch_bounds__(kBlock, 2) update_kernel(UpdateArgs a) {
     if (st_bytes) atomicAdd(a.stats + kStBytes, st_bytes);
 }
 
-void launch_update(const UpdateArgs &a, int workers, cudaStream_t s) {
+}  // namespace
+
+#define DBC_CAT2(a, b) a##b
+#define DBC_CAT(a, b) DBC_CAT2(a, b)
+void DBC_CAT(launch_update_, DBC_BLOCK)(const UpdateArgs &a, int workers, cudaStream_t s) {
     update_kernel<<<workers, kBlock, 0, s>>>(a);
 }
 

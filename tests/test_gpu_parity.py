@@ -312,3 +312,18 @@ def test_no_reorder_flag_matches_oracle(name):
             outs.append([dbc.get_root_state(s) for s in range(wl.roots.size)])
     for (d0, s0, _), (d1, s1, _) in zip(*outs):
         assert np.array_equal(d0, d1) and np.array_equal(s0, s1)
+
+
+@pytest.mark.parametrize("name", ["karate", "rmat10", "delaunay12u"])
+def test_block128_kernels_match_oracle(name, monkeypatch):
+    """The 128-thread kernel build (chosen when there are more roots than 2 x SMs)."""
+    monkeypatch.setenv("DBC_BLOCK", "128")
+    wl = W.make_workload(name)
+    ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
+    with _dbc(wl.graph, wl.roots) as dbc:
+        dbc.static_compute()
+        check_all(dbc, ref.compute(), wl.roots.size)
+        dbc.insert_edges(wl.ins_u, wl.ins_v)
+        for u, v in zip(wl.ins_u, wl.ins_v):
+            ref.insert(u, v)
+        check_all(dbc, ref.compute(), wl.roots.size)
