@@ -119,6 +119,8 @@ typedef struct {
     int64_t kernel_launches_total;
     int64_t insertions_total;
     int64_t alg_bytes_total;   /* update kernels' algorithmic bytes            */
+    int32_t heavy_roots;       /* roots run on the wide heavy lane in the last insert call */
+    int32_t reserved2;
 } dbc_timings;
 
 /* Fills *opt with defaults (device 0, rank 0, world 1, automatic sizes). */
@@ -198,9 +200,10 @@ dbc_status dbc_reset_timings(dbc_ctx *c);
 dbc_status dbc_debug_counters(dbc_ctx *c, int64_t *out, int32_t count);
 
 /* Diagnostic per-root profile of the update kernel: enable != 0 turns recording
- * on for later insert calls; out (nullable, int64[4 * k_local]) receives, per
+ * on for later insert calls; out (nullable, int64[6 * k_local]) receives, per
  * local root slot of the last update launch, {start ns, end ns, working
- * (Case 2/3) insertions, touched vertices}.  Synchronises when out != NULL. */
+ * (Case 2/3) insertions, touched vertices, adjacency entries scanned, level
+ * steps}.  Synchronises when out != NULL. */
 dbc_status dbc_debug_root_profile(dbc_ctx *c, int32_t enable, int64_t *out);
 
 /* Device memory held by the context, in bytes. */

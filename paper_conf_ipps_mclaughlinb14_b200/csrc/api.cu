@@ -32,6 +32,14 @@ struct dbc_ctx {
     bool own_stream = false;
     int workers = 0;
     int block = 256;   // threads per worker CTA (256 or 128)
+    // heavy lanes: the slowest root chains of the previous batch run on
+    // 2x-wide CTAs (hblock threads) on a high-priority stream
+    int hblock = 512, heavy_cap = 0;
+    cudaStream_t hstream = nullptr;
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+    int32_t *slots_d = nullptr;
+    std::vector<double> root_ms;   // chain time per local slot, last Mode-A launch
+    bool prof_pending = false;
     int nsm = 148;
     bool have_state = false;
     uint64_t epoch_used = 0;
@@ -147,6 +155,9 @@ void dbc_destroy(dbc_ctx *c) {
     for (void *p : c->allocs) cudaFree(p);
     if (c->ev_ok)
         for (auto &e : c->ev) cudaEventDestroy(e);
+    if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+    if (c->ev_join) cudaEventDestroy(c->ev_join);
+    if (c->hstream) cudaStreamDestroy(c->hstream);
     if (c->own_stream && c->stream) cudaStreamDestroy(c->stream);
     delete c;
 }
@@ -262,7 +273,7 @@ static GView view_of(const dbc_ctx *c) {
 static Scratch worker_scratch(const dbc_ctx *c) { return c->ws; }
 
 static dbc_status reset_epochs(dbc_ctx *c) {
-    const size_t nw = (size_t)c->workers, n = (size_t)c->n;
+    const size_t nw = (size_t)c->workers + c->heavy_cap, n = (size_t)c->n;
     if (!nw) return DBC_OK;
     CK(cudaMemsetAsync(c->ws.mark, 0, sizeof(uint32_t) * nw * n, c->stream));
     CK(cudaMemsetAsync(c->ws.lowrec, 0, sizeof(unsigned long long) * nw * n, c->stream));
@@ -356,6 +367,16 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
             return bail(DBC_ECUDA);
         }
     c->ev_ok = true;
+    {
+        int lo = 0, hi = 0;
+        cudaDeviceGetStreamPriorityRange(&lo, &hi);
+        if (cudaStreamCreateWithPriority(&c->hstream, cudaStreamNonBlocking, hi) != cudaSuccess ||
+            cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
+            cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming) != cudaSuccess) {
+            fail(c, DBC_ECUDA, "heavy-lane stream creation failed");
+            return bail(DBC_ECUDA);
+        }
+    }
 
     // workers: persistent CTAs; bounded by roots and by a scratch-memory budget
     const size_t per_worker = (size_t)n * (4 + 8 + 8 + 4 + 4 + 8 + 4 + 4 + 4 + 4 + 4) + (size_t)(n + 2) * 4 + 64;
@@ -368,11 +389,15 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     int64_t maxdeg = 0;
     for (int32_t v = 0; v < n; ++v) maxdeg = std::max<int64_t>(maxdeg, row_ptr[v + 1] - row_ptr[v]);
     c->block = (c->k_loc > 2 * c->nsm && maxdeg <= 256) ? 128 : 256;  // hubs need the wide CTA
-    if (const char *eb = getenv("DBC_BLOCK")) c->block = (atoi(eb) == 128) ? 128 : 256;
-    int want = opt.workers ? opt.workers : (c->block == 128 ? 4 : 2) * c->nsm;
+    if (const char *eb = getenv("DBC_BLOCK")) c->block = atoi(eb) == 128 ? 128 : (atoi(eb) == 512 ? 512 : 256);
+    int want = opt.workers ? opt.workers : (c->block == 128 ? 4 : (c->block == 512 ? 1 : 2)) * c->nsm;
     want = std::min(want, c->k_loc);
     int fit = (int)std::min<size_t>(budget / per_worker, 1 << 20);
     c->workers = std::max(0, std::min(want, fit));
+    c->hblock = c->block == 128 ? 256 : 512;
+    // only hub-heavy graphs (256-thread build) have step-bound slow roots
+    c->heavy_cap = (c->block != 256 || opt.workers) ? 0 : std::max(0, std::min(c->nsm / 4, (int)(fit - c->workers)));
+    if (getenv("DBC_NO_HEAVY")) c->heavy_cap = 0;
     if (c->k_loc > 0 && c->workers == 0) {
         fail(c, DBC_ENOMEM, "not enough device memory for one worker (%zu bytes)", per_worker);
         return bail(DBC_ENOMEM);
@@ -406,24 +431,26 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->bc_ext, (size_t)n);
     AL(c->perm_d, (size_t)n);
     AL(c->roots_d, (size_t)c->k_loc);
-    const size_t wn = (size_t)c->workers * n;
+    const size_t nwk = (size_t)c->workers + c->heavy_cap;  // scratch for both lanes
+    const size_t wn = nwk * n;
     AL(c->ws.mark, wn);
     AL(c->ws.lowrec, wn);
     AL(c->ws.dacc, wn);
     AL(c->ws.Dv, wn);
     AL(c->ws.Dold, wn);
     AL(c->ws.Dsig, wn);
-    AL(c->ws.Doff, (size_t)c->workers * (n + 2));
+    AL(c->ws.Doff, nwk * (n + 2));
     AL(c->ws.U0, wn);
     AL(c->ws.U1, wn);
     AL(c->ws.Rv, wn);
     AL(c->ws.Rl, wn);
     AL(c->ws.Bq, wn);
-    AL(c->ws.wepoch, (size_t)c->workers);
-    AL(c->next_slot, 1);
+    AL(c->ws.wepoch, nwk);
+    AL(c->next_slot, 2);
+    AL(c->slots_d, (size_t)std::max(c->k_loc, 1));
     AL(c->stats, (size_t)kStCount);
     AL(c->err, 1);
-    AL(c->root_prof, (size_t)4 * std::max(c->k_loc, 1));
+    AL(c->root_prof, (size_t)6 * std::max(c->k_loc, 1));
 #undef AL
 
     // upload CSR (int32 offsets), roots; zero scratch
@@ -554,6 +581,14 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     CK(cudaMemcpyAsync(&bad, c->ab.bad, sizeof(int32_t), cudaMemcpyDeviceToHost, c->stream));
     CK(cudaStreamSynchronize(c->stream));  // all earlier work is complete here
     TRY(fold_timings(c));
+    if (c->prof_pending) {  // chain time per root of the previous batch (heavy-lane choice)
+        std::vector<unsigned long long> pr((size_t)6 * c->k_loc);
+        CK(cudaMemcpy(pr.data(), c->root_prof, sizeof(unsigned long long) * pr.size(),
+                      cudaMemcpyDeviceToHost));
+        c->root_ms.assign(c->k_loc, 0.0);
+        for (int i = 0; i < c->k_loc; ++i) c->root_ms[i] = (double)(pr[6 * i + 1] - pr[6 * i]) * 1e-6;
+        c->prof_pending = false;
+    }
     if (bad) {
         const char *why = (bad & 1) ? "self loop or vertex out of range"
                           : (bad & 2) ? "edge already present"
@@ -595,29 +630,79 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     a.stats = c->stats;
     a.err = c->err;
     a.root_prof = c->prof_on ? c->root_prof : nullptr;
+    a.slot_list = nullptr;
+    a.slot_count = 0;
+    a.worker_base = 0;
     if (tm) CK(cudaEventRecord(c->ev[2], c->stream));
     int ulaunch = 0;
     if (c->workers) {
-        if (c->flags & DBC_FLAG_MODE_S) {
+        if (!(c->flags & DBC_FLAG_MODE_S)) {
+            // Mode A with heavy lanes: order slots by last chain time (longest
+            // first), the slowest ones go to the wide CTAs
+            a.root_prof = c->root_prof;
+            const int k = c->k_loc;
+            std::vector<int32_t> order(k);
+            for (int i = 0; i < k; ++i) order[i] = i;
+            int nh = 0;
+            if ((int)c->root_ms.size() == k && k > 1) {
+                std::stable_sort(order.begin(), order.end(),
+                                 [&](int x, int y) { return c->root_ms[x] > c->root_ms[y]; });
+                std::vector<double> srt(c->root_ms);
+                std::nth_element(srt.begin(), srt.begin() + k / 2, srt.end());
+                const double med = srt[k / 2];
+                while (nh < c->heavy_cap && nh < k - 1 && c->root_ms[order[nh]] > 1.3 * med) ++nh;
+            }
+            // slot list: normal slots (longest first), then the heavy ones
+            std::vector<int32_t> list;
+            list.reserve(k);
+            for (int i = nh; i < k; ++i) list.push_back(order[i]);
+            for (int i = 0; i < nh; ++i) list.push_back(order[i]);
+            CK(cudaMemcpyAsync(c->slots_d, list.data(), sizeof(int32_t) * k, cudaMemcpyHostToDevice,
+                               c->stream));
+            CK(cudaMemsetAsync(c->next_slot, 0, 2 * sizeof(int32_t), c->stream));
+            a.ins_begin = 0;
+            a.ins_end = (int32_t)cnt;
+            if (nh > 0) {  // heavy lane first, on the high-priority stream
+                CK(cudaEventRecord(c->ev_fork, c->stream));
+                CK(cudaStreamWaitEvent(c->hstream, c->ev_fork, 0));
+                UpdateArgs h = a;
+                h.slot_list = c->slots_d + (k - nh);
+                h.slot_count = nh;
+                h.worker_base = c->workers;
+                h.next_slot = c->next_slot + 1;
+                if (c->hblock == 512)
+                    launch_update_512(h, nh, c->hstream);
+                else
+                    launch_update_256(h, nh, c->hstream);
+                CK(cudaEventRecord(c->ev_join, c->hstream));
+                ++ulaunch;
+            }
+            a.slot_list = c->slots_d;
+            a.slot_count = k - nh;
+            const int wl = std::min(c->workers, k - nh);
+            if (c->block == 128)
+                launch_update_128(a, wl, c->stream);
+            else if (c->block == 512)
+                launch_update_512(a, wl, c->stream);
+            else
+                launch_update_256(a, wl, c->stream);
+            ++ulaunch;
+            if (nh > 0) CK(cudaStreamWaitEvent(c->stream, c->ev_join, 0));
+            c->prof_pending = true;
+            c->tm.heavy_roots = nh;
+        } else {
             for (int64_t i = 0; i < cnt; ++i) {
                 CK(cudaMemsetAsync(c->next_slot, 0, sizeof(int32_t), c->stream));
                 a.ins_begin = (int32_t)i;
                 a.ins_end = (int32_t)i + 1;
                 if (c->block == 128)
                     launch_update_128(a, c->workers, c->stream);
+                else if (c->block == 512)
+                    launch_update_512(a, c->workers, c->stream);
                 else
                     launch_update_256(a, c->workers, c->stream);
                 ++ulaunch;
             }
-        } else {
-            CK(cudaMemsetAsync(c->next_slot, 0, sizeof(int32_t), c->stream));
-            a.ins_begin = 0;
-            a.ins_end = (int32_t)cnt;
-            if (c->block == 128)
-                launch_update_128(a, c->workers, c->stream);
-            else
-                launch_update_256(a, c->workers, c->stream);
-            ++ulaunch;
         }
         CK(cudaGetLastError());
     }
@@ -779,7 +864,7 @@ extern "C" dbc_status dbc_debug_root_profile(dbc_ctx *c, int32_t enable, int64_t
     CK(cudaSetDevice(c->device));
     c->prof_on = enable != 0;
     if (out) {
-        CK(cudaMemcpyAsync(out, c->root_prof, sizeof(int64_t) * 4 * c->k_loc, cudaMemcpyDeviceToHost,
+        CK(cudaMemcpyAsync(out, c->root_prof, sizeof(int64_t) * 6 * c->k_loc, cudaMemcpyDeviceToHost,
                            c->stream));
         CK(cudaStreamSynchronize(c->stream));
     }

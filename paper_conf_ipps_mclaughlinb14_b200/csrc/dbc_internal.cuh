@@ -426,7 +426,10 @@ struct UpdateArgs {
     int32_t *next_slot;            // work counter (zeroed before launch)
     unsigned long long *stats;     // kStCount counters
     int32_t *err;
-    unsigned long long *root_prof; // nullable: per local slot {t_begin, t_end, jobs, touched}
+    unsigned long long *root_prof; // nullable: per local slot {t_begin, t_end, jobs, ...}
+    const int32_t *slot_list;      // nullable: the slots this launch processes (else 0..k_loc-1)
+    int32_t slot_count;            // entries of slot_list
+    int32_t worker_base;           // scratch index of CTA 0
 };
 
 struct StaticArgs {
@@ -445,6 +448,7 @@ struct StaticArgs {
 
 void launch_update_256(const UpdateArgs &a, int workers, cudaStream_t s);
 void launch_update_128(const UpdateArgs &a, int workers, cudaStream_t s);
+void launch_update_512(const UpdateArgs &a, int workers, cudaStream_t s);
 void launch_static_256(const StaticArgs &a, int workers, cudaStream_t s);
 void launch_static_128(const StaticArgs &a, int workers, cudaStream_t s);
 

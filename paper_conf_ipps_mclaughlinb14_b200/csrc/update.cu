@@ -63,10 +63,11 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
     __shared__ int s_l1[kChunk];
     __shared__ int s_adjs[kAdjCap];      // adj(root) = the level-1 vertices
     __shared__ int s_adjdeg[kAdjCap];    // their degrees
+    __shared__ double s_l1acc[kAdjCap];  // per level-1 vertex: sum of Ddelta[x] / sigma[x]
     __shared__ int s_un[2][kUcap];       // up frontier ping-pong (overflow: U0 / U1)
 
     const int tid = threadIdx.x;
-    const int wk = blockIdx.x;
+    const int wk = a.worker_base + blockIdx.x;  // scratch of this worker
     const size_t n = (size_t)a.n;
 
     uint32_t *mark = a.ws.mark + (size_t)wk * n;
@@ -107,14 +108,20 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
     }
 
     for (;;) {
-        if (tid == 0) s_slot = atomicAdd(a.next_slot, 1);
+        if (tid == 0) {
+            const int q = atomicAdd(a.next_slot, 1);
+            const int cnt = a.slot_list ? a.slot_count : a.k_loc;
+            s_slot = q < cnt ? (a.slot_list ? a.slot_list[q] : q) : -1;
+        }
         __syncthreads();
         const int slot = s_slot;
         __syncthreads();
-        if (slot >= a.k_loc) break;
+        if (slot < 0) break;
         const Root st{a.d + (size_t)slot * n, a.sd + (size_t)slot * n};
         const int sroot = a.roots[slot];
         unsigned long long prof_t0 = 0, prof_jobs = 0, prof_touch0 = st_touched;
+        const unsigned long long prof_sc0 = sc_down + sc_rem + sc_dpull + sc_dpush + sc_up2 + sc_up3;
+        const unsigned long long prof_lv0 = st_lvd + st_lvu;
         if (a.root_prof && tid == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(prof_t0));
 
         // Insertions are walked in order.  Classification (K2) of a window of
@@ -352,11 +359,12 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                     if (l < L0 && ucnt == 0) break;  // nothing left above the insertion
                     const bool push = l >= 2;          // level-1 vertices only feed the root
                     ++st_lvu;
-                    // queue p for level l-1 unless already queued (plain flag store; a
-                    // rare duplicate from a race is dropped when the list is processed)
+                    // queue p for level l-1 unless already queued: the prefetched mark
+                    // filters the common case, the returning atomic elects one
+                    // appender among concurrent pushers (no duplicates)
                     auto claim_up = [&](int y, uint32_t my) {
                         if (my >= E) return;
-                        mark[y] = mU;
+                        if (atomicMax(mark + y, mU) >= E) return;
                         const int pos = atomicAdd(&s_ucnt, 1);
                         if (pos < kUcap)
                             s_un[ucur_sel ^ 1][pos] = y;
@@ -572,6 +580,11 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                             const int nl1 = s_nl1;
                             if (nl1 > 0) {
                                 const int ds = s_ds, npairs = nl1 * ds;
+                                for (int j = tid; j < ds; j += kBlock) s_l1acc[j] = 0.0;
+                                __syncthreads();
+                                // Ddelta[p] += sigma[p] * sum_x Ddelta[x] / sigma[x] over the
+                                // level-2 rows x adjacent to level-1 vertex p (per-p sums in
+                                // shared memory, one global update per p)
                                 for (int qq = tid; qq < npairs; qq += kBlock) {
                                     const int li = qq / ds, j = qq - li * ds;
                                     const int t = s_l1[li];
@@ -580,7 +593,17 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                                     const bool adj = (s_adjdeg[j] < degx) ? adjacent_visible(g, pp, x, lim)
                                                                           : adjacent_visible(g, x, pp, lim);
                                     st_bytes += 32;
-                                    if (adj) up_visit(I.c1[t], I.c0[t], pp, st.sd[pp].x, mark[pp]);
+                                    if (adj) atomicAdd(&s_l1acc[j], __ddiv_rn(I.c1[t], I.c0[t]));
+                                }
+                                __syncthreads();
+                                for (int j = tid; j < ds; j += kBlock) {
+                                    const double w = s_l1acc[j];
+                                    if (w != 0.0) {
+                                        const int pp = s_adjs[j];
+                                        atomicAdd(dacc + pp, __dmul_rn(st.sd[pp].x, w));
+                                        st_bytes += 24;
+                                        claim_up(pp, mark[pp]);
+                                    }
                                 }
                                 __syncthreads();
                             }
@@ -626,11 +649,13 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
         if (a.root_prof && tid == 0) {
             unsigned long long t1;
             asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t1));
-            unsigned long long *rp4 = a.root_prof + 4 * (size_t)slot;
+            unsigned long long *rp4 = a.root_prof + 6 * (size_t)slot;
             rp4[0] = prof_t0;
             rp4[1] = t1;
             rp4[2] = prof_jobs;
             rp4[3] = st_touched - prof_touch0;
+            rp4[4] = sc_down + sc_rem + sc_dpull + sc_dpush + sc_up2 + sc_up3 - prof_sc0;
+            rp4[5] = st_lvd + st_lvu - prof_lv0;
         }
     }
     if (tid == 0) {

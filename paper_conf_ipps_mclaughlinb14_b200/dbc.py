@@ -67,6 +67,7 @@ class Timings(ctypes.Structure):
         ("append_ms_total", ctypes.c_double), ("update_ms_total", ctypes.c_double),
         ("update_launches_total", ctypes.c_int64), ("kernel_launches_total", ctypes.c_int64),
         ("insertions_total", ctypes.c_int64), ("alg_bytes_total", ctypes.c_int64),
+        ("heavy_roots", ctypes.c_int32), ("reserved2", ctypes.c_int32),
     ]
 
     def as_dict(self):
@@ -262,7 +263,7 @@ class DynamicBC:
         return dict(zip(names, out.tolist()))
 
     def root_profile(self, enable=True, read=True):
-        out = np.zeros((self.num_local_roots(), 4), dtype=np.int64) if read else None
+        out = np.zeros((self.num_local_roots(), 6), dtype=np.int64) if read else None
         _check(self._ctx, self._lib.dbc_debug_root_profile(
             self._ctx, int(enable), _np_ptr(out) if read else None))
         return out

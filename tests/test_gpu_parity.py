@@ -327,3 +327,21 @@ def test_block128_kernels_match_oracle(name, monkeypatch):
         for u, v in zip(wl.ins_u, wl.ins_v):
             ref.insert(u, v)
         check_all(dbc, ref.compute(), wl.roots.size)
+
+
+def test_heavy_lane_batches_match_oracle():
+    """Several Mode-A batches so the adaptive heavy lane (2x-wide CTAs for the
+    slowest roots of the previous batch) is exercised; d/sigma bit-exact."""
+    wl = W.make_workload("rmat10", insertions=120)
+    ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
+    with _dbc(wl.graph, wl.roots) as dbc:
+        dbc.static_compute()
+        heavy = 0
+        for b in range(4):
+            sl = slice(30 * b, 30 * (b + 1))
+            dbc.insert_edges(wl.ins_u[sl], wl.ins_v[sl])
+            for u, v in zip(wl.ins_u[sl], wl.ins_v[sl]):
+                ref.insert(u, v)
+            heavy = max(heavy, dbc.timings()["heavy_roots"])
+        check_all(dbc, ref.compute(), wl.roots.size)
+        assert heavy > 0  # the heavy lane was used

@@ -4,7 +4,9 @@ import numpy as np, workloads as W
 from paper_conf_ipps_mclaughlinb14_b200 import DynamicBC, FLAG_TIMING
 name = sys.argv[1] if len(sys.argv) > 1 else "rmat16"
 B = int(sys.argv[2]) if len(sys.argv) > 2 else 1000
-wl = W.make_workload(name, insertions=B, k=int(sys.argv[3]) if len(sys.argv) > 3 else None)
+wl = W.make_workload(name, insertions=B, k=int(sys.argv[3]) if len(sys.argv) > 3 and int(sys.argv[3]) > 0 else None)
+if len(sys.argv) > 4:  # explicit root list, e.g. 650960,3614
+    wl.roots = np.array([int(x) for x in sys.argv[4].split(",")], dtype=np.int32)
 g = wl.graph
 dbc = DynamicBC(g.n, g.row_ptr, g.col, wl.roots, flags=FLAG_TIMING)
 dbc.static_compute(); dbc.synchronize()
@@ -23,7 +25,10 @@ dur = (prof[:, 1] - prof[:, 0]) / 1e6
 print("root chain ms: min %.2f median %.2f p90 %.2f max %.2f; kernel span %.2f" % (dur.min(), np.median(dur), np.percentile(dur, 90), dur.max(), (prof[:,1].max()-prof[:,0].min())/1e6))
 order = np.argsort(-dur)[:8]
 for i in order:
-    print("slot", i, "root", wl.roots[i], "deg", g.degree()[wl.roots[i]], "ms %.2f" % dur[i], "jobs", prof[i,2], "touched", prof[i,3], "start %.2f" % ((prof[i,0]-prof[:,0].min())/1e6))
+    print("slot", i, "root", wl.roots[i], "deg", g.degree()[wl.roots[i]], "ms %.2f" % dur[i], "jobs", prof[i,2], "touched/job", prof[i,3]//max(prof[i,2],1), "scanned/job", prof[i,4]//max(prof[i,2],1), "levels/job %.1f" % (prof[i,5]/max(prof[i,2],1)), "us/job %.1f" % (dur[i]*1e3/max(prof[i,2],1)), "start %.2f" % ((prof[i,0]-prof[:,0].min())/1e6))
+med = np.argsort(dur)[len(dur)//2]
+i = med
+print("median root: slot", i, "deg", g.degree()[wl.roots[i]], "ms %.2f" % dur[i], "jobs", prof[i,2], "touched/job", prof[i,3]//max(prof[i,2],1), "scanned/job", prof[i,4]//max(prof[i,2],1), "levels/job %.1f" % (prof[i,5]/max(prof[i,2],1)), "us/job %.1f" % (dur[i]*1e3/max(prof[i,2],1)))
 print("jobs: median", np.median(prof[:,2]), "max", prof[:,2].max(), "touched/job median", np.median(prof[:,3]/np.maximum(prof[:,2],1)))
 st = (prof[:, 0] - prof[:, 0].min()) / 1e6
 print("root start ms: min %.2f median %.2f max %.2f; #late(>1ms) %d" % (st.min(), np.median(st), st.max(), (st > 1).sum()))
