@@ -55,6 +55,8 @@ struct dbc_ctx {
     // state
     int32_t *d = nullptr;    // [k_loc][n]
     double2 *sd = nullptr;   // [k_loc][n] (sigma, delta)
+    uint32_t *l2mask = nullptr;  // [k_loc][n] level-2 predecessor masks
+    int32_t *mask_ds = nullptr;  // [k_loc]
     double *bc = nullptr;
     int32_t *roots_d = nullptr;
 
@@ -382,7 +384,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     const size_t per_worker = (size_t)n * (4 + 8 + 8 + 4 + 4 + 8 + 4 + 4 + 4 + 4 + 4) + (size_t)(n + 2) * 4 + 64;
     size_t free_b = 0, total_b = 0;
     cudaMemGetInfo(&free_b, &total_b);
-    const size_t state_b = (size_t)c->k_loc * n * 20 + (size_t)c->col_cap * 8 + (size_t)n * 40;
+    const size_t state_b = (size_t)c->k_loc * n * 24 + (size_t)c->col_cap * 8 + (size_t)n * 40;
     size_t budget = free_b > state_b ? (free_b - state_b) / 2 : 0;
     // more roots than two 256-thread CTAs per SM can hold and no hub rows:
     // 128-thread CTAs, four per SM, so that every root chain is resident at once
@@ -427,6 +429,8 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     const size_t kn = (size_t)c->k_loc * n;
     AL(c->d, kn);
     AL(c->sd, kn);
+    AL(c->l2mask, kn);
+    AL(c->mask_ds, (size_t)std::max(c->k_loc, 1));
     AL(c->bc, (size_t)n);
     AL(c->bc_ext, (size_t)n);
     AL(c->perm_d, (size_t)n);
@@ -536,6 +540,8 @@ extern "C" dbc_status dbc_static_compute(dbc_ctx *c) {
         a.roots = c->roots_d;
         a.d = c->d;
         a.sd = c->sd;
+        a.l2mask = c->l2mask;
+        a.mask_ds = c->mask_ds;
         a.bc = c->bc;
         a.ws = worker_scratch(c);
         a.next_slot = c->next_slot;
@@ -622,6 +628,8 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     a.roots = c->roots_d;
     a.d = c->d;
     a.sd = c->sd;
+    a.l2mask = c->l2mask;
+    a.mask_ds = c->mask_ds;
     a.bc = c->bc;
     a.ins_u = u;
     a.ins_v = v;

@@ -185,6 +185,7 @@ struct BigSmem {
     int off[kBig + 1];  // exclusive scan of row lengths; off[m] = total
     double acc[kBig];   // per-row reduction
     double c0[kBig];    // per-row constant of the caller
+    unsigned mk[kBig];  // per-row level-2 predecessor mask being built
     int m;            // rows in this round
 };
 
@@ -311,9 +312,9 @@ __device__ __forceinline__ void big_entries(BigSmem &S, const GView &g, const Ro
 // --- up phase: chunked flattened level pass ----------------------------------
 constexpr int kChunk = 512;   // items per chunk (shared memory)
 constexpr int kUcap = 1024;   // up-frontier entries kept in shared memory
-constexpr int kMetaUp = 1, kMetaNotPulled = 2;
+constexpr int kMetaUp = 1, kMetaNotPulled = 2, kMetaMask = 4;
 constexpr int kFlatU = 4;     // contiguous entries per thread per step
-constexpr int kAdjCap = 512;  // longest root row kept in shared memory (level-2 shortcut)
+constexpr int kAdjCap = 256;  // longest root row kept in shared memory (level-2 shortcut)
 
 struct ChunkSmem {
     int v[kChunk];
@@ -321,6 +322,7 @@ struct ChunkSmem {
     int beg[kChunk];
     int off[kChunk + 1];
     double acc[kChunk], c0[kChunk], c1[kChunk], c2[kChunk];
+    unsigned mk[kChunk];  // level-2 predecessor mask of masked up items
 };
 
 // exclusive scan in place of off[1..cnt] (lengths) -> off[0..cnt]; ends with a barrier
@@ -411,6 +413,37 @@ __device__ __forceinline__ void flat_entries(const int *off, int cnt, int E, Col
 }
 
 // ---------------------------------------------------------------------------
+// Level-2 predecessor masks (roots with at most kMaskDeg neighbours): bit j of
+// mask[x] is set iff x (a level-2 vertex) is adjacent to the j-th neighbour of
+// the root in the root's canonical row.  The level-1 predecessors of a level-2
+// vertex -- the pushes of the up phase into level 1 -- then come from one
+// gather instead of a scan of x's row.  Valid for vertices with d == 2 only.
+constexpr int kMaskDeg = 32;
+
+// (Re)build all masks of one root from its row rs (as of `limit`): clear the
+// masks of every level-2 vertex, then OR in one bit per level-1 neighbour.
+// Whole CTA; ends with a barrier.
+__device__ __forceinline__ void build_l2masks(const GView &g, const Root &st, uint32_t *mask,
+                                              int2 rs, int limit) {
+    const int ds = rs.y - rs.x;
+    for (int pass = 0; pass < 2; ++pass) {
+        for (int j = 0; j < ds; ++j) {
+            const int p = ldg_i(g.col + rs.x + j);
+            const int2 rp = row_of(g, p, limit);
+            for (int e = rp.x + (int)threadIdx.x; e < rp.y; e += kBlock) {
+                const int x = ldg_i(g.col + e);
+                if (st.dist(x) != 2) continue;
+                if (pass == 0)
+                    mask[x] = 0u;
+                else
+                    atomicOr(mask + x, 1u << j);
+            }
+        }
+        __syncthreads();
+    }
+}
+
+// ---------------------------------------------------------------------------
 // kernel entry points (defined in static_brandes.cu / update.cu)
 struct UpdateArgs {
     GView g;
@@ -426,6 +459,8 @@ struct UpdateArgs {
     int32_t *next_slot;            // work counter (zeroed before launch)
     unsigned long long *stats;     // kStCount counters
     int32_t *err;
+    uint32_t *l2mask;              // [k_loc][n] level-2 predecessor masks (see below)
+    int32_t *mask_ds;              // [k_loc] root degree the masks were built for (-1: none)
     unsigned long long *root_prof; // nullable: per local slot {t_begin, t_end, jobs, ...}
     const int32_t *slot_list;      // nullable: the slots this launch processes (else 0..k_loc-1)
     int32_t slot_count;            // entries of slot_list
@@ -444,6 +479,8 @@ struct StaticArgs {
     int32_t *next_slot;
     unsigned long long *stats;
     int32_t *err;
+    uint32_t *l2mask;
+    int32_t *mask_ds;
 };
 
 void launch_update_256(const UpdateArgs &a, int workers, cudaStream_t s);

@@ -131,6 +131,14 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) static_kernel(StaticArgs
         }
         // levels 0 .. nl-2 are non-empty; loff[j] .. loff[j+1] is level j.
 
+        // level-2 predecessor masks for the update kernel (roots of degree <= 32)
+        {
+            const int2 rs = row_of(g, s, INT32_MAX);
+            const bool ok = rs.y - rs.x <= kMaskDeg;
+            if (ok) build_l2masks(g, st, a.l2mask + (size_t)slot * n, rs, INT32_MAX);
+            if (tid == 0) a.mask_ds[slot] = ok ? rs.y - rs.x : -1;
+        }
+
         // Stage 3: dependency accumulation in reverse level order (Eq. (2)),
         // BC partial += delta (Eq. (3)), root excluded (delta_s(s) = 0).
         for (int lev = nl - 2; lev >= 1; --lev) {

@@ -57,7 +57,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
     __shared__ int s_nl1;      // of those, resolved against adj(root)
     __shared__ int s_ds;       // |adj(root)| as of the insertion (-1: too long)
     __shared__ uint32_t s_work[kWarps];  // window classification bits (1 = Case 2/3)
-    __shared__ int s_job[4];             // uh, ul, L0, case3 of the current job
+    __shared__ int s_job[6];             // uh, ul, L0, case3, mask state, root degree of the job
     __shared__ BigSmem S;
     __shared__ ChunkSmem I;              // long rows of the current up level
     __shared__ int s_l1[kChunk];
@@ -119,6 +119,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
         if (slot < 0) break;
         const Root st{a.d + (size_t)slot * n, a.sd + (size_t)slot * n};
         const int sroot = a.roots[slot];
+        uint32_t *mask = a.l2mask + (size_t)slot * n;
         unsigned long long prof_t0 = 0, prof_jobs = 0, prof_touch0 = st_touched;
         const unsigned long long prof_sc0 = sc_down + sc_rem + sc_dpull + sc_dpush + sc_up2 + sc_up3;
         const unsigned long long prof_lv0 = st_lvd + st_lvu;
@@ -157,6 +158,18 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                 ++prof_jobs;
                 const uint32_t E = epoch << 2;
                 const uint32_t mD = E | kDown, mU = E | kUp;
+                if (tid < 32) {  // warp 0: the root's row as of this insertion (level-2 masks)
+                    const int2 rs = row_of(g, sroot, p);
+                    const int dsr = rs.y - rs.x;
+                    if (dsr <= kMaskDeg && tid < dsr) s_adjs[tid] = ldg_i(g.col + rs.x + tid);
+                    if (tid == 0) {
+                        const int built = a.mask_ds[slot];
+                        // 1: masks valid; 2: the root gained a neighbour -> rebuild after the down phase
+                        s_job[4] = (dsr > kMaskDeg) ? 0 : (built == dsr ? 1 : 2);
+                        s_job[5] = dsr;
+                        if (dsr > kMaskDeg && built >= 0) a.mask_ds[slot] = -1;
+                    }
+                }
                 if (tid == 0) {
                     const int u = __ldg(a.ins_u + p), v = __ldg(a.ins_v + p);
                     const int du = st.dist(u), dv = st.dist(v);
@@ -190,13 +203,23 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                 __syncthreads();
                 const int uh = s_job[0], ul = s_job[1], L0 = s_job[2];
                 const bool case3 = s_job[3] != 0;
+                const int mstate = s_job[4], dsr = s_job[5];
+                const bool mvalid = mstate == 1;  // masks usable during this job's down phase
+                // bit of a level-1 vertex in the masks (its position in the root's row)
+                auto l1bit = [&](int y) -> uint32_t {
+                    for (int j = 0; j < dsr; ++j)
+                        if (s_adjs[j] == y) return 1u << j;
+                    return 0u;
+                };
                 const int lim = p;  // graph as of this insertion (edge p included)
 
                 tick(-1);
                 // ================= down phase (K3) =================
                 int L = L0, lb = 0, le = 1, nlev = 1;
                 // per-D-entry epilogue: record old d / sigma, store the new sigma
-                auto down_finish = [&](int idx, int w, double sum) {
+                // (and, at level 2, the vertex's level-1 predecessor mask)
+                auto down_finish = [&](int idx, int w, double sum, uint32_t m) {
+                    if (mvalid && L == 2) mask[w] = m;
                     const unsigned long long lr = lowrec[w];
                     const int od = ((uint32_t)(lr >> 32) == epoch) ? (int)(uint32_t)lr : L;
                     Dold[idx] = od;
@@ -228,11 +251,15 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                         le - lb, g, lim, [&](int i, int &w) { w = Dv[lb + i]; return true; },
                         [&](int i, int w, int2 r) {
                             double sum = 0.0;  // canonical order: bit-exact
+                            uint32_t m = 0u;
                             row_walk(g, st, nullptr, r, [&](int dy) { return dy == L - 1; },
-                                     [&](int y, int dy, double2 q, uint32_t) { sum += down_visit(y, dy, q.x); });
+                                     [&](int y, int dy, double2 q, uint32_t) {
+                                         if (mvalid && L == 2 && dy == 1) m |= l1bit(y);
+                                         sum += down_visit(y, dy, q.x);
+                                     });
                             st_bytes += 8 + 8ull * (r.y - r.x);
                             sc_down += r.y - r.x;
-                            down_finish(lb + i, w, sum);
+                            down_finish(lb + i, w, sum, m);
                         },
                         enq_front);
                     __syncthreads();
@@ -241,10 +268,13 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                         const int m = min(kBig, nbig - r0);
                         big_load(S, m, [&](int t) { return Bq[r0 + t]; }, [&](int i) { return Dv[lb + i]; },
                                  g, lim);
+                        if (tid < m) S.mk[tid] = 0u;
+                        __syncthreads();
                         big_entries(S, g, st, [&](int dy) { return dy == L - 1; },
-                                    [&](int, int y, int dy, double2 q) {
+                                    [&](int t, int y, int dy, double2 q) {
                                         st_bytes += 8;
                                         sc_down++;
+                                        if (mvalid && L == 2 && dy == 1) atomicOr(&S.mk[t], l1bit(y));
                                         return down_visit(y, dy, q.x);
                                     });
                         if (tid < m) {
@@ -259,7 +289,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                                 }
                             }
                             st_bytes += 8;
-                            down_finish(lb + S.idx[tid], w, sum);
+                            down_finish(lb + S.idx[tid], w, sum, S.mk[tid]);
                         }
                         __syncthreads();
                     }
@@ -284,6 +314,13 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                     st_down += dtotal;
                     st_touched += dtotal;
                 }
+
+                // the root gained a neighbour (Case 3 with u_high = root): rebuild its masks
+                if (mstate == 2) {
+                    build_l2masks(g, st, mask, row_of(g, sroot, lim), lim);
+                    if (tid == 0) a.mask_ds[slot] = dsr;
+                }
+                const bool mok = mstate != 0;  // masks valid for the up phase
 
                 tick(0);
                 // ================= (0) Case-3 removal pushes =================
@@ -432,7 +469,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                     // removal targets.  resolve() issues everything an item needs as
                     // one round of independent loads.
                     auto resolve = [&](int q, int &x, int &meta, double &c0, double &c1, double &c2,
-                                       int2 &r) -> bool {
+                                       int2 &r, uint32_t &mk) -> bool {
                         if (q < nDl) {
                             const int idx = b0 + q;
                             x = Dv[idx];
@@ -457,19 +494,28 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                         const double gx = dacc[x];  // Ddelta (complete: level l+1 is done)
                         const double2 s2 = st.sd[x];
                         const double sx = s2.x, odl = s2.y;
-                        const int2 rr = push ? row_of(g, x, lim) : make_int2(0, 0);
+                        const bool usemask = l == 2 && mok;  // level-1 predecessors from the mask
+                        const int2 rr = (push && !usemask) ? row_of(g, x, lim) : make_int2(0, 0);
+                        mk = usemask ? mask[x] : 0u;
                         if (prev != mU) return false;  // a duplicate: the first claimant processes
-                        meta = kMetaUp;
+                        meta = kMetaUp | (usemask ? kMetaMask : 0);
                         c0 = sx;
                         c1 = gx;
                         c2 = odl;
-                        st_bytes += 24;
+                        st_bytes += 24 + (usemask ? 4 : 0);
                         r = (push && gx != 0.0) ? rr : make_int2(0, 0);
+                        if (gx == 0.0) mk = 0u;
                         return true;
                     };
-                    auto inlane = [&](int x, int meta, double c0, double c1, double c2, int2 r) {
+                    auto inlane = [&](int x, int meta, double c0, double c1, double c2, int2 r, uint32_t mk) {
                         const bool wantpush = push && r.y > r.x;
-                        if (meta & kMetaUp) {
+                        if (meta & kMetaMask) {  // level 2: predecessors = set bits (root's row order)
+                            for (uint32_t b = mk; b; b &= b - 1) {
+                                const int pp = s_adjs[__ffs(b) - 1];
+                                up_visit(c1, c0, pp, st.sd[pp].x, mark[pp]);
+                            }
+                            up_finish(x, c1, c2);
+                        } else if (meta & kMetaUp) {
                             if (wantpush) {
                                 row_walk(g, st, mark, r, [&](int dp) { return dp == l - 1; },
                                          [&](int pp, int dp, double2 q, uint32_t mp) {
@@ -503,23 +549,29 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                             int x, meta = 0;
                             double c0 = 0.0, c1 = 0.0, c2 = 0.0;
                             int2 r = make_int2(0, 0);
-                            if (!resolve(q, x, meta, c0, c1, c2, r)) continue;
+                            uint32_t mk = 0u;
+                            if (!resolve(q, x, meta, c0, c1, c2, r, mk)) continue;
                             const int len = r.y - r.x;
                             if (small_inlane && len <= kSmallDeg) {
-                                inlane(x, meta, c0, c1, c2, r);
+                                inlane(x, meta, c0, c1, c2, r, mk);
                                 continue;
                             }
                             const int t = atomicAdd(&s_nbigI, 1);
                             if (t >= kChunk) {  // shared list full: stay in-lane
-                                inlane(x, meta, c0, c1, c2, r);
+                                inlane(x, meta, c0, c1, c2, r, mk);
                                 continue;
                             }
                             int elen = len;
-                            // level 2: resolve against adj(root) when cheaper than a scan
-                            if ((meta & kMetaUp) && l == 2 && s_ds >= 0 && s_ds * (33 - __clz(len)) < len) {
+                            if (meta & kMetaMask) {  // level 2 via the mask
+                                if (mk) s_l1[atomicAdd(&s_nl1, 1)] = t;
+                                elen = 0;
+                            } else if ((meta & kMetaUp) && l == 2 && s_ds >= 0 &&
+                                       s_ds * (33 - __clz(len)) < len) {
+                                // level 2 without masks: resolve against adj(root) by search
                                 s_l1[atomicAdd(&s_nl1, 1)] = t;
                                 elen = 0;
                             }
+                            I.mk[t] = mk;
                             I.v[t] = x;
                             I.meta[t] = meta;
                             I.beg[t] = r.x;
@@ -589,10 +641,15 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                                     const int li = qq / ds, j = qq - li * ds;
                                     const int t = s_l1[li];
                                     const int x = I.v[t], pp = s_adjs[j];
-                                    const int degx = (ldg_i(g.rp + x + 1) & kMask) - (ldg_i(g.rp + x) & kMask);
-                                    const bool adj = (s_adjdeg[j] < degx) ? adjacent_visible(g, pp, x, lim)
-                                                                          : adjacent_visible(g, x, pp, lim);
-                                    st_bytes += 32;
+                                    bool adj;
+                                    if (I.meta[t] & kMetaMask) {
+                                        adj = (I.mk[t] >> j) & 1u;
+                                    } else {
+                                        const int degx = (ldg_i(g.rp + x + 1) & kMask) - (ldg_i(g.rp + x) & kMask);
+                                        adj = (s_adjdeg[j] < degx) ? adjacent_visible(g, pp, x, lim)
+                                                                   : adjacent_visible(g, x, pp, lim);
+                                        st_bytes += 32;
+                                    }
                                     if (adj) atomicAdd(&s_l1acc[j], __ddiv_rn(I.c1[t], I.c0[t]));
                                 }
                                 __syncthreads();
