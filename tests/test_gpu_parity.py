@@ -345,3 +345,53 @@ def test_heavy_lane_batches_match_oracle():
             heavy = max(heavy, dbc.timings()["heavy_roots"])
         check_all(dbc, ref.compute(), wl.roots.size)
         assert heavy > 0  # the heavy lane was used
+
+
+def _sampled_full_size(name, insertions, sample):
+    """Full-size config in the bench launch configuration (Mode A, one batch):
+    sampled roots' d/sigma bit-exact and delta within tolerance vs the oracle on
+    the final graph; incremental BC vs the GPU's own column sum of delta
+    (Eq. (3), DBC_FLAG_EXACT_BC rebase) within 1e-9; GPU dynamic == GPU static."""
+    from paper_conf_ipps_mclaughlinb14_b200 import DynamicBC, FLAG_EXACT_BC
+
+    wl = W.make_workload(name, insertions=insertions)
+    g = wl.graph
+    with DynamicBC(g.n, g.row_ptr, g.col, wl.roots) as dbc:
+        dbc.static_compute()
+        half = insertions // 2
+        dbc.insert_edges(wl.ins_u[:half], wl.ins_v[:half])  # two batches: heavy lanes engage
+        dbc.insert_edges(wl.ins_u[half:], wl.ins_v[half:])
+        bc_inc = dbc.get_bc()
+        ref = oracle.NaiveDynamicBC(g, wl.roots)
+        for u, v in zip(wl.ins_u, wl.ins_v):
+            ref.insert(u, v)
+        rp, col = ref.csr()
+        slots = np.linspace(0, wl.roots.size - 1, sample).astype(np.int32)
+        _, d_ref, s_ref, dl_ref = oracle.brandes(g.n, rp, col, wl.roots[slots])
+        dyn = {}
+        for i, slot in enumerate(slots):
+            d, s, dl = dbc.get_root_state(int(slot))
+            assert np.array_equal(d, d_ref[i]), f"d slot {slot}"
+            assert np.array_equal(s, s_ref[i]), f"sigma slot {slot}"
+            err = np.abs(dl - dl_ref[i]) / np.maximum(np.abs(dl_ref[i]), 1.0)
+            assert err.max() <= DELTA_TOL
+            dyn[int(slot)] = (d, s)
+        dbc.static_compute()  # GPU recompute on the final graph
+        for slot, (d0, s0) in dyn.items():
+            d1, s1, _ = dbc.get_root_state(slot)
+            assert np.array_equal(d0, d1) and np.array_equal(s0, s1)
+    # Eq. (3) column sum on a fresh context that replays the same batches
+    with DynamicBC(g.n, g.row_ptr, g.col, wl.roots, flags=FLAG_EXACT_BC) as dbc:
+        dbc.static_compute()
+        dbc.insert_edges(wl.ins_u[:half], wl.ins_v[:half])
+        dbc.insert_edges(wl.ins_u[half:], wl.ins_v[half:])
+        bc_exact = dbc.get_bc()
+    assert_bc(bc_inc, bc_exact)
+
+
+def test_delaunay18_full_size_sampled():
+    _sampled_full_size("delaunay18", 1000, 4)
+
+
+def test_kron20_full_size_sampled():
+    _sampled_full_size("kron20", 600, 3)
