@@ -252,11 +252,42 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                         [&](int i, int w, int2 r) {
                             double sum = 0.0;  // canonical order: bit-exact
                             uint32_t m = 0u;
-                            row_walk(g, st, nullptr, r, [&](int dy) { return dy == L - 1; },
-                                     [&](int y, int dy, double2 q, uint32_t) {
-                                         if (mvalid && L == 2 && dy == 1) m |= l1bit(y);
-                                         sum += down_visit(y, dy, q.x);
-                                     });
+                            for (int j = r.x; j < r.y; j += kRowUnroll) {
+                                int y[kRowUnroll], dy[kRowUnroll], om[kRowUnroll];
+                                uint32_t oc[kRowUnroll];
+                                double sy[kRowUnroll];
+#pragma unroll
+                                for (int u = 0; u < kRowUnroll; ++u) y[u] = (j + u < r.y) ? ldg_i(g.col + j + u) : -1;
+#pragma unroll
+                                for (int u = 0; u < kRowUnroll; ++u) dy[u] = (y[u] >= 0) ? st.d[y[u]] : kInf;
+#pragma unroll
+                                for (int u = 0; u < kRowUnroll; ++u)
+                                    sy[u] = (y[u] >= 0 && dy[u] == L - 1) ? st.sd[y[u]].x : 0.0;
+                                // issue every lowering and claim of the block, then consume
+#pragma unroll
+                                for (int u = 0; u < kRowUnroll; ++u)
+                                    om[u] = (y[u] >= 0 && dy[u] > L + 1) ? atomicMin(st.d + y[u], L + 1) : 0;
+#pragma unroll
+                                for (int u = 0; u < kRowUnroll; ++u)
+                                    oc[u] = mD;
+#pragma unroll
+                                for (int u = 0; u < kRowUnroll; ++u)
+                                    if (y[u] >= 0 && dy[u] >= L + 1) oc[u] = atomicMax(mark + y[u], mD);
+#pragma unroll
+                                for (int u = 0; u < kRowUnroll; ++u) {
+                                    if (y[u] < 0) continue;
+                                    if (dy[u] == L - 1) {  // predecessor: canonical-order sum
+                                        sum += sy[u];
+                                        st_bytes += 8;
+                                        if (mvalid && L == 2) m |= l1bit(y[u]);
+                                    }
+                                    if (dy[u] > L + 1 && om[u] > L + 1) {  // first lowerer (Case 3)
+                                        lowrec[y[u]] = ((unsigned long long)epoch << 32) | (uint32_t)om[u];
+                                        st_bytes += 4;
+                                    }
+                                    if (dy[u] >= L + 1 && oc[u] < mD) Dv[atomicAdd(&s_dcnt, 1)] = y[u];
+                                }
+                            }
                             st_bytes += 8 + 8ull * (r.y - r.x);
                             sc_down += r.y - r.x;
                             down_finish(lb + i, w, sum, m);
@@ -517,10 +548,40 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                             up_finish(x, c1, c2);
                         } else if (meta & kMetaUp) {
                             if (wantpush) {
-                                row_walk(g, st, mark, r, [&](int dp) { return dp == l - 1; },
-                                         [&](int pp, int dp, double2 q, uint32_t mp) {
-                                             if (dp == l - 1) up_visit(c1, c0, pp, q.x, mp);
-                                         });
+                                for (int j = r.x; j < r.y; j += kRowUnroll) {
+                                    int y[kRowUnroll], dy[kRowUnroll];
+                                    uint32_t mp[kRowUnroll], oc[kRowUnroll];
+                                    double sp[kRowUnroll];
+#pragma unroll
+                                    for (int u = 0; u < kRowUnroll; ++u)
+                                        y[u] = (j + u < r.y) ? ldg_i(g.col + j + u) : -1;
+#pragma unroll
+                                    for (int u = 0; u < kRowUnroll; ++u) dy[u] = (y[u] >= 0) ? st.d[y[u]] : kInf;
+#pragma unroll
+                                    for (int u = 0; u < kRowUnroll; ++u) {
+                                        const bool pr = y[u] >= 0 && dy[u] == l - 1;
+                                        sp[u] = pr ? st.sd[y[u]].x : 0.0;
+                                        mp[u] = pr ? mark[y[u]] : 0xffffffffu;
+                                    }
+#pragma unroll
+                                    for (int u = 0; u < kRowUnroll; ++u)
+                                        if (y[u] >= 0 && dy[u] == l - 1) {
+                                            atomicAdd(dacc + y[u], __dmul_rn(__ddiv_rn(sp[u], c0), c1));
+                                            st_bytes += 24;
+                                        }
+#pragma unroll
+                                    for (int u = 0; u < kRowUnroll; ++u)
+                                        oc[u] = (mp[u] < E) ? atomicMax(mark + y[u], mU) : 0xffffffffu;
+#pragma unroll
+                                    for (int u = 0; u < kRowUnroll; ++u)
+                                        if (oc[u] < E) {
+                                            const int pos = atomicAdd(&s_ucnt, 1);
+                                            if (pos < kUcap)
+                                                s_un[ucur_sel ^ 1][pos] = y[u];
+                                            else
+                                                Unext[pos - kUcap] = y[u];
+                                        }
+                                }
                                 (l == 2 ? sc_up2 : sc_up3) += r.y - r.x;
                                 st_bytes += 8 + 8ull * (r.y - r.x);
                             }
