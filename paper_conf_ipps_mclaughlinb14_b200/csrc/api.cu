@@ -70,7 +70,8 @@ struct dbc_ctx {
     std::vector<void *> allocs;
     int64_t bytes = 0;
 
-    cudaEvent_t ev[6] = {};
+    cudaEvent_t ev[10] = {};  // [0..3]/[6..9]: insert-call sets A/B, [4..5]: static
+    int evset = 0;            // set of the most recent insert call (0 -> ev[0..3], 1 -> ev[6..9])
     bool ev_ok = false;
     dbc_timings tm{};
     bool tm_pending = false, tm_static = false;
@@ -511,8 +512,9 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
 // has completed whenever this is called after a stream synchronisation)
 static dbc_status fold_timings(dbc_ctx *c) {
     if (c->tm_pending) {
-        CK(cudaEventElapsedTime(&c->tm.append_ms, c->ev[0], c->ev[1]));
-        CK(cudaEventElapsedTime(&c->tm.update_ms, c->ev[2], c->ev[3]));
+        cudaEvent_t *e = c->ev + (c->evset ? 6 : 0);  // the previous call's set
+        CK(cudaEventElapsedTime(&c->tm.append_ms, e[0], e[1]));
+        CK(cudaEventElapsedTime(&c->tm.update_ms, e[2], e[3]));
         c->tm.append_ms_total += c->tm.append_ms;
         c->tm.update_ms_total += c->tm.update_ms;
         c->tm_pending = false;
@@ -579,7 +581,9 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     CK(cudaSetDevice(c->device));
     const bool tm = c->flags & DBC_FLAG_TIMING;
     int launches = 0;
-    if (tm) CK(cudaEventRecord(c->ev[0], c->stream));
+    // alternate event sets so the previous call's events survive until folded
+    cudaEvent_t *ev = c->ev + (c->evset ? 0 : 6);
+    if (tm) CK(cudaEventRecord(ev[0], c->stream));
     GView g = view_of(c);
     launches += validate_batch(c->ab, g, c->rp[c->cur], c->n, u, v, cnt, c->stream);
     CK(cudaGetLastError());
@@ -614,7 +618,7 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     c->cur = nb;
     c->nnz += 2 * cnt;
     c->inserted += cnt;
-    if (tm) CK(cudaEventRecord(c->ev[1], c->stream));
+    if (tm) CK(cudaEventRecord(ev[1], c->stream));
 
     // epoch budget: each job of a worker consumes one epoch (30 bits available)
     const uint64_t jobs = (uint64_t)c->k_loc * (uint64_t)cnt;
@@ -641,7 +645,7 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     a.slot_list = nullptr;
     a.slot_count = 0;
     a.worker_base = 0;
-    if (tm) CK(cudaEventRecord(c->ev[2], c->stream));
+    if (tm) CK(cudaEventRecord(ev[2], c->stream));
     int ulaunch = 0;
     if (c->workers) {
         if (!(c->flags & DBC_FLAG_MODE_S)) {
@@ -715,7 +719,8 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
         CK(cudaGetLastError());
     }
     if (tm) {
-        CK(cudaEventRecord(c->ev[3], c->stream));
+        CK(cudaEventRecord(ev[3], c->stream));
+        c->evset ^= 1;
         c->tm_pending = true;
     }
     launches += ulaunch;

@@ -49,7 +49,7 @@ namespace {
 __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs a) {
     __shared__ int s_slot;
     __shared__ int s_dcnt;     // |D| (absolute positions in Dv)
-    __shared__ int s_ucnt;     // next up frontier size
+    __shared__ int s_ucnt2[2]; // up frontier sizes (list ucur_sel is read, ucur_sel^1 filled)
     __shared__ int s_rcnt;     // |R|
     __shared__ int s_rmax;     // deepest removal-push target level
     __shared__ int s_nbig;     // long-row queue (down phase / removal)
@@ -192,7 +192,8 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                     Doff[0] = 0;
                     Doff[1] = 1;
                     s_dcnt = 1;
-                    s_ucnt = 0;
+                    s_ucnt2[0] = 0;
+                    s_ucnt2[1] = 0;
                     s_rcnt = 0;
                     s_rmax = 0;
                     s_job[0] = uh;
@@ -433,7 +434,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                     auto claim_up = [&](int y, uint32_t my) {
                         if (my >= E) return;
                         if (atomicMax(mark + y, mU) >= E) return;
-                        const int pos = atomicAdd(&s_ucnt, 1);
+                        const int pos = atomicAdd(&s_ucnt2[ucur_sel ^ 1], 1);
                         if (pos < kUcap)
                             s_un[ucur_sel ^ 1][pos] = y;
                         else
@@ -575,7 +576,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
 #pragma unroll
                                     for (int u = 0; u < kRowUnroll; ++u)
                                         if (oc[u] < E) {
-                                            const int pos = atomicAdd(&s_ucnt, 1);
+                                            const int pos = atomicAdd(&s_ucnt2[ucur_sel ^ 1], 1);
                                             if (pos < kUcap)
                                                 s_un[ucur_sel ^ 1][pos] = y[u];
                                             else
@@ -648,13 +649,21 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                     const int total = nDl + ucnt + rcnt;
                     const bool small_level = total <= kBlock;
                     const int step = small_level ? total : kChunk;
+                    bool first_barrier = true;
                     for (int cb = 0; cb < total; cb += step) {
                         const int ce = min(total, cb + step);
-                        split_range(cb, min(ce, nDl), small_level);  // down rows first: pull precedes push
-                        __syncthreads();
-                        const int nDb = min(s_nbigI, kChunk);
+                        int nDb = 0;
+                        if (cb < nDl) {  // down rows first: their pull precedes their push
+                            split_range(cb, min(ce, nDl), small_level);
+                            __syncthreads();
+                            nDb = min(s_nbigI, kChunk);
+                        }
                         split_range(max(cb, nDl), ce, small_level);
                         __syncthreads();
+                        if (first_barrier) {  // the current list's count was read last level
+                            first_barrier = false;
+                            if (tid == 0) s_ucnt2[ucur_sel] = 0;
+                        }
                         tick(6);
                         const int nb = min(s_nbigI, kChunk);
                         if (nb > 0) {
@@ -742,17 +751,13 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                         __syncthreads();
                     }  // chunks
                     tick(3);
-                    ucnt = s_ucnt;
-                    __syncthreads();
-                    if (tid == 0) {
-                        s_ucnt = 0;
-                        st_touched += ucnt;
-                    }
+                    // the chunk loop ended with a barrier: every append of this level is in
+                    ucnt = s_ucnt2[ucur_sel ^ 1];
+                    if (tid == 0) st_touched += ucnt;
                     int *t = Ucur;
                     Ucur = Unext;
                     Unext = t;
                     ucur_sel ^= 1;
-                    __syncthreads();
                     tick(5);
                 }
                 // any up vertices left at level 0 would be the root: never produced

@@ -12,7 +12,12 @@ dbc = DynamicBC(g.n, g.row_ptr, g.col, wl.roots, flags=FLAG_TIMING)
 dbc.static_compute(); dbc.synchronize()
 c0 = dbc.debug_counters()
 dbc.root_profile(True, read=False)
-dbc.insert_edges(wl.ins_u, wl.ins_v)
+nb = int(os.environ.get("PB_BATCHES", "1"))
+bs = len(wl.ins_u) // nb
+for b in range(nb):
+    if b == nb - 1:
+        c0 = dbc.debug_counters()
+    dbc.insert_edges(wl.ins_u[b * bs:(b + 1) * bs], wl.ins_v[b * bs:(b + 1) * bs])
 c1 = dbc.debug_counters()
 d = {k: c1[k] - c0[k] for k in c1}
 print(d)
