@@ -279,13 +279,15 @@ def local_slots(k: int, rank: int, world: int):
     return list(range(rank, k, world))
 
 
-def allreduce_bc(dbc: DynamicBC, group=None):
-    """Sum the per-rank BC partials in place over torch.distributed (NCCL on GPUs)
-    and return the global BC on the host.  The only cross-GPU exchange (A5)."""
+def allreduce_bc(dbc: DynamicBC, group=None, force=False):
+    """Sum the per-rank BC partials over torch.distributed (NCCL on GPUs) and
+    return the global BC on the host -- the only cross-GPU exchange of the
+    method.  force=True runs the collective even for a
+    single rank (tests)."""
     import torch
     import torch.distributed as dist
 
-    if dbc.world == 1 or not dist.is_initialized():
+    if not dist.is_initialized() or (dbc.world == 1 and not force):
         return dbc.get_bc()
     ptr = dbc.bc_partial_device_ptr()
     dbc.synchronize()
