@@ -60,6 +60,8 @@ def parse():
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-budget-s", type=float, default=12.0)
+    p.add_argument("--shard", default="", help="R/N: run rank R's root shard of an N-GPU job on this "
+                   "single GPU (per-GPU view of configs that need N GPUs, e.g. kron22 on 8)")
     return p.parse_args()
 
 
@@ -218,6 +220,11 @@ def run_ours(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    shard_rank, shard_world = rank, world
+    if args.shard:
+        if world > 1:
+            raise SystemExit("--shard emulates one rank on one GPU; do not combine with torchrun")
+        shard_rank, shard_world = (int(x) for x in args.shard.split("/"))
     if world > 1:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
         torch.cuda.set_device(local)
@@ -240,7 +247,7 @@ def run_ours(args):
     flags = FLAG_TIMING | (FLAG_MODE_S if args.mode == "S" else 0)
     stream = torch.cuda.Stream(device=dev)  # the library and the timing events share it
     torch.cuda.set_stream(stream)
-    dbc = DynamicBC(g.n, g.row_ptr, g.col, wl.roots, device=dev, rank=rank, world=world,
+    dbc = DynamicBC(g.n, g.row_ptr, g.col, wl.roots, device=dev, rank=shard_rank, world=shard_world,
                     workers=args.workers, edge_capacity=B * nb, flags=flags,
                     stream=stream.cuda_stream)
 
@@ -346,7 +353,7 @@ def run_ours(args):
             cpu = {"value": None, "unit": "insertions/s", "cores": 1, "kind": "oracle",
                    "sample": f"unavailable: {ex}"}
 
-    state_mb = 20.0 * k * g.n / world / 1e6
+    state_mb = 24.0 * k * g.n / shard_world / 1e6
     line = {
         "metric": "edge insertions/sec (device-timed)",
         "value": value,
@@ -367,6 +374,8 @@ def run_ours(args):
             "protocol": "remove-then-reinsert (P:440)" if cfg["mode"] == "reinsert" else "uniform non-edges",
             "l2": f"inputs larger than L2: per-GPU d/sigma/delta state {state_mb:.0f} MB vs 126 MB L2",
             "static_recompute_ms": static_ms,
+            "shard": (f"rank {shard_rank} of {shard_world} (roots slot % {shard_world} == {shard_rank}) "
+                      f"on one GPU" if args.shard else None),
             "speedup_vs_static": (static_ms / 1e3) / per_ins_s,
             "us_per_insertion": per_ins_s * 1e6,
             "case_mix": case_mix,
