@@ -39,6 +39,8 @@ struct dbc_ctx {
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     int32_t *slots_d = nullptr;
     std::vector<double> root_ms;   // chain time per local slot, last Mode-A launch
+    HelpBoard help{};              // cooperative help board (Mode A)
+    bool help_on = true;
     bool prof_pending = false;
     int nsm = 148;
     bool have_state = false;
@@ -382,7 +384,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     }
 
     // workers: persistent CTAs; bounded by roots and by a scratch-memory budget
-    const size_t per_worker = (size_t)n * (4 + 8 + 8 + 4 + 4 + 8 + 4 + 4 + 4 + 4 + 4) + (size_t)(n + 2) * 4 + 64;
+    const size_t per_worker = (size_t)n * (4 + 8 + 8 + 4 + 4 + 8 + 4 + 4 + 4 + 4 + 4 + 4) + sizeof(ChunkSmem) + (size_t)(n + 2) * 4 + 64;
     size_t free_b = 0, total_b = 0;
     cudaMemGetInfo(&free_b, &total_b);
     const size_t state_b = (size_t)c->k_loc * n * 24 + (size_t)c->col_cap * 8 + (size_t)n * 40;
@@ -451,6 +453,15 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->ws.Rl, wn);
     AL(c->ws.Bq, wn);
     AL(c->ws.wepoch, nwk);
+    AL(c->help.word, nwk);
+    AL(c->help.done, nwk);
+    AL(c->help.ctx, nwk);
+    AL(c->help.mir, nwk);
+    AL(c->help.gapp, nwk);
+    AL(c->help.gU, wn);
+    AL(c->help.roots_left, 1);
+    c->help.nworkers = (int)nwk;
+    if (const char *e = getenv("DBC_NO_HELP")) c->help_on = atoi(e) == 0;
     AL(c->next_slot, 2);
     AL(c->slots_d, (size_t)std::max(c->k_loc, 1));
     AL(c->stats, (size_t)kStCount);
@@ -645,6 +656,7 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     a.slot_list = nullptr;
     a.slot_count = 0;
     a.worker_base = 0;
+    a.help = HelpBoard{};  // Mode S: no cooperative help
     if (tm) CK(cudaEventRecord(ev[2], c->stream));
     int ulaunch = 0;
     if (c->workers) {
@@ -674,6 +686,13 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
             CK(cudaMemsetAsync(c->next_slot, 0, 2 * sizeof(int32_t), c->stream));
             a.ins_begin = 0;
             a.ins_end = (int32_t)cnt;
+            if (c->help_on) {  // fresh board: all requests closed, every root chain pending
+                a.help = c->help;
+                CK(cudaMemsetAsync(c->help.word, 0, sizeof(unsigned long long) * c->help.nworkers, c->stream));
+                const int left = k;
+                CK(cudaMemcpyAsync(c->help.roots_left, &left, sizeof(int), cudaMemcpyHostToDevice, c->stream));
+                CK(cudaStreamSynchronize(c->stream));  // `left` is a host stack value
+            }
             if (nh > 0) {  // heavy lane first, on the high-priority stream
                 CK(cudaEventRecord(c->ev_fork, c->stream));
                 CK(cudaStreamWaitEvent(c->hstream, c->ev_fork, 0));

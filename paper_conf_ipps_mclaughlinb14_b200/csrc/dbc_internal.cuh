@@ -50,6 +50,9 @@ enum StatIdx : int {
     kStTime0 = kStPhase0 + 6,  // 10 timers (ns, thread 0), see update.cu tick()
     kStLevDown = kStTime0 + 10,  // level steps of the down phase
     kStLevUp,                    // level steps of the up phase
+    kStHelpReq,                  // C2 passes published for cooperative help
+    kStHelpBlk,                  // blocks of them processed by helpers
+    kStHelpBlkAll,               // all blocks of published passes
     kStCount
 };
 
@@ -365,11 +368,11 @@ __device__ __forceinline__ void chunk_scan(int *off, int cnt) {
 // calls f(t, y, d, sd, mark) (sd, mark gathered for want(d)); if acc != nullptr
 // the returned contribution is
 // summed into acc[t].  Ends with a barrier.
-template <class Want, class Col, class F>
+template <bool kCG = false, class Want, class Col, class F>
 __device__ __forceinline__ void flat_entries(const int *off, int cnt, int E, Col colf, const Root &st,
-                                             const uint32_t *mk, Want want, double *acc, F f) {
+                                             const uint32_t *mk, Want want, double *acc, F f, int Ebeg = 0) {
     const int tid = threadIdx.x;
-    for (int base = 0; base < E; base += kBlock * kFlatU) {
+    for (int base = Ebeg; base < E; base += kBlock * kFlatU) {
         const int e0 = base + tid * kFlatU;
         int t[kFlatU], y[kFlatU], dy[kFlatU];
         double2 q[kFlatU];
@@ -395,12 +398,13 @@ __device__ __forceinline__ void flat_entries(const int *off, int cnt, int E, Col
             }
         }
 #pragma unroll
-        for (int u = 0; u < kFlatU; ++u) dy[u] = (t[u] >= 0) ? st.dist(y[u]) : kInf;
+        for (int u = 0; u < kFlatU; ++u)
+            dy[u] = (t[u] >= 0) ? (kCG ? __ldcg(st.d + y[u]) : st.dist(y[u])) : kInf;
 #pragma unroll
         for (int u = 0; u < kFlatU; ++u) {
             const bool w = t[u] >= 0 && want(dy[u]);
-            q[u] = w ? st.sd[y[u]] : make_double2(0.0, 0.0);
-            mm[u] = (mk && w) ? mk[y[u]] : 0u;
+            q[u] = w ? (kCG ? __ldcg(st.sd + y[u]) : st.sd[y[u]]) : make_double2(0.0, 0.0);
+            mm[u] = (mk && w) ? (kCG ? __ldcg(mk + y[u]) : mk[y[u]]) : 0u;
         }
 #pragma unroll
         for (int u = 0; u < kFlatU; ++u) {
@@ -444,6 +448,38 @@ __device__ __forceinline__ void build_l2masks(const GView &g, const Root &st, ui
 }
 
 // ---------------------------------------------------------------------------
+// Cooperative help: a worker whose up-level push pass (C2)
+// has many entries publishes it on a help board; workers that have run out of
+// roots join it block by block.  Per owner: a packed word
+//   bit 63 open | bits 40..59 blocks | bits 16..35 next block | bits 0..15 seq
+// (helpers grab a block with one atomicAdd of 1 << 16), a done counter, the
+// job context, a global mirror of the chunk and a global append list.
+constexpr int kHelpEntries = 4096;     // entries per help block
+constexpr int kHelpMinBlocks = 3;      // publish only passes of >= 3 blocks
+struct HelpCtx {
+    int root_slot, l, uh, ul, cnt, nblocks, E2;
+    uint32_t E;  // epoch << 2 of the job
+};
+struct HelpBoard {
+    unsigned long long *word;  // [workers]
+    int *done;                 // [workers]
+    HelpCtx *ctx;              // [workers]
+    ChunkSmem *mir;            // [workers]
+    int *gapp;                 // [workers] global append counters
+    int32_t *gU;               // [workers][n] global append lists
+    int *roots_left;           // [1] root chains not yet finished (both lanes)
+    int nworkers;
+};
+__device__ __forceinline__ unsigned long long help_pack(int open, int nblocks, int next, int seq) {
+    return ((unsigned long long)(open ? 1 : 0) << 63) | ((unsigned long long)(nblocks & 0xFFFFF) << 40) |
+           ((unsigned long long)(next & 0xFFFFF) << 16) | (unsigned long long)(seq & 0xFFFF);
+}
+__device__ __forceinline__ bool help_open(unsigned long long w) { return (w >> 63) != 0; }
+__device__ __forceinline__ int help_nblocks(unsigned long long w) { return (int)((w >> 40) & 0xFFFFF); }
+__device__ __forceinline__ int help_next(unsigned long long w) { return (int)((w >> 16) & 0xFFFFF); }
+__device__ __forceinline__ int help_seq(unsigned long long w) { return (int)(w & 0xFFFF); }
+
+// ---------------------------------------------------------------------------
 // kernel entry points (defined in static_brandes.cu / update.cu)
 struct UpdateArgs {
     GView g;
@@ -465,6 +501,7 @@ struct UpdateArgs {
     const int32_t *slot_list;      // nullable: the slots this launch processes (else 0..k_loc-1)
     int32_t slot_count;            // entries of slot_list
     int32_t worker_base;           // scratch index of CTA 0
+    HelpBoard help;                // help.word == nullptr: no cooperative help
 };
 
 struct StaticArgs {

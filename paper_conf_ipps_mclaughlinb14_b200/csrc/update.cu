@@ -46,6 +46,48 @@ constexpr bool kPhaseTimers = false;
 #endif
 
 namespace {
+// One push of a helped C2 pass (owner or helper): the same arithmetic as the
+// owner's up_visit / dpush_visit, with claims appended to the global list.
+__device__ __forceinline__ void help_push_entry(const ChunkSmem &M, int t, int pp, int dp, double sp,
+                                                uint32_t mp, const HelpCtx &cx, uint32_t *mark,
+                                                double *dacc, int32_t *gU, int *gapp,
+                                                unsigned long long &bytes) {
+    if (dp != cx.l - 1) return;
+    const uint32_t E = cx.E, mD = E | kDown, mU = E | kUp;
+    const int meta = M.meta[t];
+    double dlt;
+    if (meta & kMetaUp) {
+        dlt = __dmul_rn(__ddiv_rn(sp, M.c0[t]), M.c1[t]);
+    } else {
+        if (mp == mD) return;
+        dlt = __dmul_rn(__ddiv_rn(sp, M.c0[t]), 1.0 + M.acc[t]);
+        if ((meta & kMetaNotPulled) && !(pp == cx.uh && M.v[t] == cx.ul))
+            dlt = __dsub_rn(dlt, __dmul_rn(__ddiv_rn(sp, M.c2[t]), 1.0 + M.c1[t]));
+    }
+    atomicAdd(dacc + pp, dlt);
+    bytes += 24;
+    if (mp >= E) return;
+    if (atomicMax(mark + pp, mU) >= E) return;
+    gU[atomicAdd(gapp, 1)] = pp;
+}
+
+// Entries [e0, e1) of a published chunk M (in this CTA's shared memory).
+// kCG: the owner's state is read through L2 (helpers run on other SMs).
+template <bool kCG>
+__device__ __forceinline__ void help_run_block(const ChunkSmem &M, int e0, int e1, const GView &g,
+                                               const Root &st, uint32_t *mark, double *dacc, int32_t *gU,
+                                               int *gapp, const HelpCtx &cx, unsigned long long &bytes) {
+    auto colf = [&](int t, int e) { return ldg_i(g.col + M.beg[t] + e - M.off[t]); };
+    flat_entries<kCG>(
+        M.off, cx.cnt, e1, colf, st, mark, [&](int dp) { return dp == cx.l - 1; }, nullptr,
+        [&](int t, int pp, int dp, double2 q, uint32_t mp) -> double {
+            bytes += 8;
+            help_push_entry(M, t, pp, dp, q.x, mp, cx, mark, dacc, gU, gapp, bytes);
+            return 0.0;
+        },
+        e0);
+}
+
 __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs a) {
     __shared__ int s_slot;
     __shared__ int s_dcnt;     // |D| (absolute positions in Dv)
@@ -65,6 +107,8 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
     __shared__ int s_adjdeg[kAdjCap];    // their degrees
     __shared__ double s_l1acc[kAdjCap];  // per level-1 vertex: sum of Ddelta[x] / sigma[x]
     __shared__ int s_un[2][kUcap];       // up frontier ping-pong (overflow: U0 / U1)
+    __shared__ int s_hb, s_hpick, s_hseq; // cooperative help: grabbed block, owner, request
+    __shared__ HelpCtx s_hctx;
 
     const int tid = threadIdx.x;
     const int wk = a.worker_base + blockIdx.x;  // scratch of this worker
@@ -84,6 +128,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
     int32_t *Bq = a.ws.Bq + (size_t)wk * n;
     uint32_t epoch = a.ws.wepoch[wk];
     const GView &g = a.g;
+    int hseq = 0;  // this worker's help-request sequence
 
     unsigned long long st_bytes = 0, st_touched = 0, st_down = 0;
     unsigned long long st_c1 = 0, st_c2 = 0, st_c3 = 0, st_lvd = 0, st_lvu = 0;
@@ -523,7 +568,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                         if (x < 0) return false;
                         // the dedup claim and the loads are issued together
                         const uint32_t prev = atomicMax(mark + x, E | kUpDone);
-                        const double gx = dacc[x];  // Ddelta (complete: level l+1 is done)
+                        const double gx = __ldcg(dacc + x);  // Ddelta (complete; helpers add via L2)
                         const double2 s2 = st.sd[x];
                         const double sx = s2.x, odl = s2.y;
                         const bool usemask = l == 2 && mok;  // level-1 predecessors from the mask
@@ -681,7 +726,77 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                                              });
                             tick(8);
                             // --- C2: pushes towards level l-1 ---
-                            if (push && E2 > 0)
+                            const int nblk = (E2 + kHelpEntries - 1) / kHelpEntries;
+                            if (push && E2 > 0 && a.help.word && nblk >= kHelpMinBlocks) {
+                                // publish the chunk; idle workers help block by block
+                                ChunkSmem *mir = a.help.mir + wk;
+                                for (int t = tid; t < nb; t += kBlock) {
+                                    mir->v[t] = I.v[t];
+                                    mir->meta[t] = I.meta[t];
+                                    mir->beg[t] = I.beg[t];
+                                    mir->off[t + 1] = I.off[t + 1];
+                                    mir->acc[t] = I.acc[t];
+                                    mir->c0[t] = I.c0[t];
+                                    mir->c1[t] = I.c1[t];
+                                    mir->c2[t] = I.c2[t];
+                                }
+                                HelpCtx cx;
+                                cx.root_slot = slot;
+                                cx.l = l;
+                                cx.uh = uh;
+                                cx.ul = ul;
+                                cx.cnt = nb;
+                                cx.nblocks = nblk;
+                                cx.E2 = E2;
+                                cx.E = E;
+                                if (tid == 0) {
+                                    mir->off[0] = 0;
+                                    a.help.ctx[wk] = cx;
+                                    a.help.done[wk] = 0;
+                                    a.help.gapp[wk] = 0;
+                                }
+                                __threadfence();
+                                __syncthreads();
+                                if (tid == 0) {
+                                    atomicAdd(a.stats + kStHelpReq, 1ull);
+                                    atomicAdd(a.stats + kStHelpBlkAll, (unsigned long long)nblk);
+                                    hseq = (hseq + 1) & 0xFFFF;
+                                    atomicExch(a.help.word + wk, help_pack(1, nblk, 0, hseq));
+                                }
+                                int32_t *gU = a.help.gU + (size_t)wk * n;
+                                int *gapp = a.help.gapp + wk;
+                                for (;;) {  // the owner takes blocks too
+                                    if (tid == 0) {
+                                        const unsigned long long w = atomicAdd(a.help.word + wk, 1ull << 16);
+                                        s_hb = help_next(w) < nblk ? help_next(w) : -1;
+                                    }
+                                    __syncthreads();
+                                    const int b = s_hb;
+                                    __syncthreads();
+                                    if (b < 0) break;
+                                    help_run_block<false>(I, b * kHelpEntries, min(E2, (b + 1) * kHelpEntries), g,
+                                                          st, mark, dacc, gU, gapp, cx, st_bytes);
+                                    __threadfence();
+                                    __syncthreads();
+                                    if (tid == 0) atomicAdd(a.help.done + wk, 1);
+                                }
+                                if (tid == 0) {  // wait for the helpers' blocks, then close
+                                    while (atomicAdd(a.help.done + wk, 0) < nblk) __nanosleep(256);
+                                    atomicExch(a.help.word + wk, help_pack(0, 0, 0, hseq));
+                                    __threadfence();
+                                }
+                                __syncthreads();
+                                const int gc = __ldcg(gapp);  // merge the global appends
+                                for (int i = tid; i < gc; i += kBlock) {
+                                    const int y = __ldcg(gU + i);
+                                    const int pos = atomicAdd(&s_ucnt2[ucur_sel ^ 1], 1);
+                                    if (pos < kUcap)
+                                        s_un[ucur_sel ^ 1][pos] = y;
+                                    else
+                                        Unext[pos - kUcap] = y;
+                                }
+                                __syncthreads();
+                            } else if (push && E2 > 0)
                                 flat_entries(
                                     I.off, nb, E2, colf, st, mark, [&](int dp) { return dp == l - 1; }, nullptr,
                                     [&](int t, int pp, int dp, double2 q, uint32_t mp) -> double {
@@ -769,6 +884,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
             ins = p;
             __syncthreads();  // s_work is rewritten by the next window
         }
+        if (a.help.word && tid == 0) atomicSub(a.help.roots_left, 1);
         if (a.root_prof && tid == 0) {
             unsigned long long t1;
             asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t1));
@@ -779,6 +895,91 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
             rp4[3] = st_touched - prof_touch0;
             rp4[4] = sc_down + sc_rem + sc_dpull + sc_dpush + sc_up2 + sc_up3 - prof_sc0;
             rp4[5] = st_lvd + st_lvu - prof_lv0;
+        }
+    }
+    // ---- out of roots: help the C2 passes of workers still running ----
+    if (a.help.word) {
+        int cur_owner = -1, cur_seq = -1;
+        for (;;) {
+            // the whole CTA scans the board (one word per thread), first open one wins
+            if (tid == 0) s_hpick = INT32_MAX;
+            __syncthreads();
+            {
+                const int nw = a.help.nworkers;
+                for (int i = tid; i < nw; i += kBlock) {
+                    const int o = (wk + 1 + i) % nw;
+                    const unsigned long long w = __ldcg(a.help.word + o);
+                    if (help_open(w) && help_next(w) < help_nblocks(w)) atomicMin(&s_hpick, i);
+                }
+            }
+            __syncthreads();
+            if (tid == 0) {
+                int pick = -1, b = -1, sq = -1;
+                if (atomicAdd(a.help.roots_left, 0) <= 0) {
+                    pick = -2;
+                } else {
+                    if (s_hpick != INT32_MAX) pick = (wk + 1 + s_hpick) % a.help.nworkers;
+                    if (pick >= 0) {
+                        const unsigned long long w = atomicAdd(a.help.word + pick, 1ull << 16);
+                        if (help_open(w) && help_next(w) < help_nblocks(w)) {
+                            b = help_next(w);
+                            sq = help_seq(w);
+                        }
+                    }
+                }
+                s_hpick = pick;
+                s_hb = b;
+                s_hseq = sq;
+            }
+            __syncthreads();
+            const int pick = s_hpick, b = s_hb, sq = s_hseq;
+            __syncthreads();
+            if (pick == -2) break;
+            if (b < 0) {
+                __nanosleep(1000);
+                continue;
+            }
+            if (pick != cur_owner || sq != cur_seq) {  // a new request: load its chunk
+                if (tid == 0) {
+                    const HelpCtx *src = a.help.ctx + pick;
+                    s_hctx.root_slot = __ldcg(&src->root_slot);
+                    s_hctx.l = __ldcg(&src->l);
+                    s_hctx.uh = __ldcg(&src->uh);
+                    s_hctx.ul = __ldcg(&src->ul);
+                    s_hctx.cnt = __ldcg(&src->cnt);
+                    s_hctx.nblocks = __ldcg(&src->nblocks);
+                    s_hctx.E2 = __ldcg(&src->E2);
+                    s_hctx.E = __ldcg(&src->E);
+                }
+                __syncthreads();
+                const ChunkSmem *mir = a.help.mir + pick;
+                const int cnt = s_hctx.cnt;
+                for (int t = tid; t < cnt; t += kBlock) {
+                    I.v[t] = __ldcg(&mir->v[t]);
+                    I.meta[t] = __ldcg(&mir->meta[t]);
+                    I.beg[t] = __ldcg(&mir->beg[t]);
+                    I.off[t + 1] = __ldcg(&mir->off[t + 1]);
+                    I.acc[t] = __ldcg(&mir->acc[t]);
+                    I.c0[t] = __ldcg(&mir->c0[t]);
+                    I.c1[t] = __ldcg(&mir->c1[t]);
+                    I.c2[t] = __ldcg(&mir->c2[t]);
+                }
+                if (tid == 0) I.off[0] = 0;
+                __syncthreads();
+                cur_owner = pick;
+                cur_seq = sq;
+            }
+            const HelpCtx cx = s_hctx;
+            const Root ost{a.d + (size_t)cx.root_slot * n, a.sd + (size_t)cx.root_slot * n};
+            help_run_block<true>(I, b * kHelpEntries, min(cx.E2, (b + 1) * kHelpEntries), g, ost,
+                                 a.ws.mark + (size_t)pick * n, a.ws.dacc + (size_t)pick * n,
+                                 a.help.gU + (size_t)pick * n, a.help.gapp + pick, cx, st_bytes);
+            __threadfence();
+            __syncthreads();
+            if (tid == 0) {
+                atomicAdd(a.help.done + pick, 1);
+                atomicAdd(a.stats + kStHelpBlk, 1ull);
+            }
         }
     }
     if (tid == 0) {

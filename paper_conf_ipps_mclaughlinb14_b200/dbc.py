@@ -257,7 +257,8 @@ class DynamicBC:
         names = ["case1", "case2", "case3", "touched", "down", "scanned", "alg_bytes",
                  "static_bytes", "sc_down", "sc_removal", "sc_dpull", "sc_dpush", "sc_up2", "sc_up3",
                  "ns_down", "ns_removal", "ns_up_setup", "ns_up_epi", "ns_up_l1pairs", "ns_up_end",
-                 "ns_up_split", "ns_up_scan", "ns_up_pull", "ns_up_push", "levels_down", "levels_up"]
+                 "ns_up_split", "ns_up_scan", "ns_up_pull", "ns_up_push", "levels_down", "levels_up",
+                 "help_requests", "help_blocks_by_helpers", "help_blocks_all"]
         out = np.zeros(len(names), dtype=np.int64)
         _check(self._ctx, self._lib.dbc_debug_counters(self._ctx, _np_ptr(out), out.size))
         return dict(zip(names, out.tolist()))

@@ -270,8 +270,12 @@ def test_rmat16_full_size_batch_parity():
     g = wl.graph
     with _dbc(g, wl.roots) as dbc:
         dbc.static_compute()
+        c0 = dbc.debug_counters()
         st = dbc.insert_edges(wl.ins_u, wl.ins_v, stats=True)
         assert st["case1"] + st["case2"] + st["case3"] == 256 * 1000
+        c1 = dbc.debug_counters()
+        # the cooperative help path (idle CTAs take blocks of a heavy C2 push) ran
+        assert c1["help_blocks_by_helpers"] > c0["help_blocks_by_helpers"]
         bc = dbc.get_bc()
         ref = oracle.NaiveDynamicBC(g, wl.roots)
         for u, v in zip(wl.ins_u, wl.ins_v):
@@ -395,3 +399,20 @@ def test_delaunay18_full_size_sampled():
 
 def test_kron20_full_size_sampled():
     _sampled_full_size("kron20", 600, 3)
+
+
+def test_help_off_matches_help_on(monkeypatch):
+    """DBC_NO_HELP=1 (every C2 push done by its owner CTA) and the default
+    cooperative path give bitwise-equal d/sigma and BC within tolerance."""
+    wl = W.make_workload("rmat16", insertions=400)
+    g = wl.graph
+    outs = []
+    for off in ("1", "0"):
+        monkeypatch.setenv("DBC_NO_HELP", off)
+        with _dbc(g, wl.roots) as dbc:
+            dbc.static_compute()
+            dbc.insert_edges(wl.ins_u, wl.ins_v)
+            outs.append((dbc.get_bc(), [dbc.get_root_state(s)[:2] for s in range(0, 256, 9)]))
+    assert_bc(outs[1][0], outs[0][0])
+    for (d0, s0), (d1, s1) in zip(outs[0][1], outs[1][1]):
+        assert np.array_equal(d0, d1) and np.array_equal(s0, s1)
