@@ -81,6 +81,11 @@ typedef enum {
 #define DBC_FLAG_NO_REORDER 0x8u /* keep the caller's vertex numbering internally
                                   (default: BFS-order relabelling for locality;
                                   invisible at the ABI, results identical)        */
+#define DBC_FLAG_NO_MERGE 0x10u /* Mode A: one job per insertion.  Default: a run of
+                                  Case-2 insertions of a root (no distance change,
+                                  P:150-155) between Case-3 ones is repaired as one
+                                  job seeded with every u_low -- the same d/sigma
+                                  (bit-exact) and BC (within rounding)            */
 
 typedef struct {
     int32_t device;        /* CUDA device ordinal (default 0)                      */

@@ -8,6 +8,7 @@ from .dbc import (  # noqa: F401
     DBC_INF,
     FLAG_EXACT_BC,
     FLAG_MODE_S,
+    FLAG_NO_MERGE,
     FLAG_NO_REORDER,
     FLAG_TIMING,
     DBCError,
@@ -19,6 +20,6 @@ from .dbc import (  # noqa: F401
 )
 
 __all__ = [
-    "DynamicBC", "DBCError", "DBC_INF", "FLAG_MODE_S", "FLAG_TIMING", "FLAG_EXACT_BC", "FLAG_NO_REORDER",
+    "DynamicBC", "DBCError", "DBC_INF", "FLAG_MODE_S", "FLAG_TIMING", "FLAG_EXACT_BC", "FLAG_NO_REORDER", "FLAG_NO_MERGE",
     "LIB_PATH", "load_library", "local_slots", "allreduce_bc",
 ]

@@ -657,6 +657,7 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     a.slot_count = 0;
     a.worker_base = 0;
     a.help = HelpBoard{};  // Mode S: no cooperative help
+    a.merge = (c->flags & DBC_FLAG_NO_MERGE) ? 0 : 1;
     if (tm) CK(cudaEventRecord(ev[2], c->stream));
     int ulaunch = 0;
     if (c->workers) {

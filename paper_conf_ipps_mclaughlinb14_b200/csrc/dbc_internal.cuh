@@ -53,6 +53,8 @@ enum StatIdx : int {
     kStHelpReq,                  // C2 passes published for cooperative help
     kStHelpBlk,                  // blocks of them processed by helpers
     kStHelpBlkAll,               // all blocks of published passes
+    kStGroups,                   // Case-2 group jobs (>= 2 insertions repaired together)
+    kStGroupIns,                 // insertions in those group jobs
     kStCount
 };
 
@@ -137,6 +139,21 @@ __device__ __forceinline__ bool adjacent_visible(const GView &g, int x, int p, i
             if (ldg_i(g.xnbr + xi.x + k) == p) return ldg_i(g.xtag + xi.x + k) <= limit;
     }
     return true;
+}
+
+// Is (x, p) an edge inserted by insertion g0 .. lim of the current batch?  x
+// must have batch entries (rp[x] flagged).  A job's pushes subtract the old
+// contribution sigma[p]/sigma_old(x)*(1+delta_old(x)) only over edges that
+// existed before the job -- for a single insertion this is Alg. 2's guard
+// "v != u_high or w != u_low", for a Case-2 group every edge of it.
+__device__ __forceinline__ bool new_edge(const GView &g, int x, int p, int g0, int lim) {
+    const int2 xi = __ldg(g.xinfo + x);
+    for (int k = 0; k < xi.y; ++k)
+        if (ldg_i(g.xnbr + xi.x + k) == p) {
+            const int t = ldg_i(g.xtag + xi.x + k);
+            return t >= g0 && t <= lim;
+        }
+    return false;
 }
 
 // ---------------------------------------------------------------------------
@@ -314,8 +331,9 @@ __device__ __forceinline__ void big_entries(BigSmem &S, const GView &g, const Ro
 
 // --- up phase: chunked flattened level pass ----------------------------------
 constexpr int kChunk = 512;   // items per chunk (shared memory)
-constexpr int kUcap = 1024;   // up-frontier entries kept in shared memory
+constexpr int kUcap = kBlock >= 512 ? 768 : 1024;   // up-frontier entries kept in shared memory
 constexpr int kMetaUp = 1, kMetaNotPulled = 2, kMetaMask = 4;
+constexpr int kMetaNew = 8;  // down row with batch entries: its pushes check new_edge()
 constexpr int kFlatU = 4;     // contiguous entries per thread per step
 constexpr int kAdjCap = 256;  // longest root row kept in shared memory (level-2 shortcut)
 
@@ -457,7 +475,7 @@ __device__ __forceinline__ void build_l2masks(const GView &g, const Root &st, ui
 constexpr int kHelpEntries = 4096;     // entries per help block
 constexpr int kHelpMinBlocks = 3;      // publish only passes of >= 3 blocks
 struct HelpCtx {
-    int root_slot, l, uh, ul, cnt, nblocks, E2;
+    int root_slot, l, g0, lim, cnt, nblocks, E2;  // g0..lim: the job's insertions
     uint32_t E;  // epoch << 2 of the job
 };
 struct HelpBoard {
@@ -502,6 +520,7 @@ struct UpdateArgs {
     int32_t slot_count;            // entries of slot_list
     int32_t worker_base;           // scratch index of CTA 0
     HelpBoard help;                // help.word == nullptr: no cooperative help
+    int32_t merge;                 // 1: repair runs of Case-2 insertions as one job
 };
 
 struct StaticArgs {

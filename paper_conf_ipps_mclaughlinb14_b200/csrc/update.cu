@@ -48,8 +48,8 @@ constexpr bool kPhaseTimers = false;
 namespace {
 // One push of a helped C2 pass (owner or helper): the same arithmetic as the
 // owner's up_visit / dpush_visit, with claims appended to the global list.
-__device__ __forceinline__ void help_push_entry(const ChunkSmem &M, int t, int pp, int dp, double sp,
-                                                uint32_t mp, const HelpCtx &cx, uint32_t *mark,
+__device__ __forceinline__ void help_push_entry(const GView &g, const ChunkSmem &M, int t, int pp, int dp,
+                                                double sp, uint32_t mp, const HelpCtx &cx, uint32_t *mark,
                                                 double *dacc, int32_t *gU, int *gapp,
                                                 unsigned long long &bytes) {
     if (dp != cx.l - 1) return;
@@ -61,7 +61,7 @@ __device__ __forceinline__ void help_push_entry(const ChunkSmem &M, int t, int p
     } else {
         if (mp == mD) return;
         dlt = __dmul_rn(__ddiv_rn(sp, M.c0[t]), 1.0 + M.acc[t]);
-        if ((meta & kMetaNotPulled) && !(pp == cx.uh && M.v[t] == cx.ul))
+        if ((meta & kMetaNotPulled) && !((meta & kMetaNew) && new_edge(g, M.v[t], pp, cx.g0, cx.lim)))
             dlt = __dsub_rn(dlt, __dmul_rn(__ddiv_rn(sp, M.c2[t]), 1.0 + M.c1[t]));
     }
     atomicAdd(dacc + pp, dlt);
@@ -82,7 +82,7 @@ __device__ __forceinline__ void help_run_block(const ChunkSmem &M, int e0, int e
         M.off, cx.cnt, e1, colf, st, mark, [&](int dp) { return dp == cx.l - 1; }, nullptr,
         [&](int t, int pp, int dp, double2 q, uint32_t mp) -> double {
             bytes += 8;
-            help_push_entry(M, t, pp, dp, q.x, mp, cx, mark, dacc, gU, gapp, bytes);
+            help_push_entry(g, M, t, pp, dp, q.x, mp, cx, mark, dacc, gU, gapp, bytes);
             return 0.0;
         },
         e0);
@@ -99,7 +99,10 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
     __shared__ int s_nl1;      // of those, resolved against adj(root)
     __shared__ int s_ds;       // |adj(root)| as of the insertion (-1: too long)
     __shared__ uint32_t s_work[kWarps];  // window classification bits (1 = Case 2/3)
-    __shared__ int s_job[6];             // uh, ul, L0, case3, mask state, root degree of the job
+    __shared__ uint32_t s_c3[kWarps];    // window classification bits (1 = Case 3)
+    __shared__ int s_wul[kBlock];        // window: u_low of each insertion
+    __shared__ int s_wlev[kBlock];       // window: d[u_low] + 0 (Case 2: its level)
+    __shared__ int s_job[8];             // uh, ul, L0, case3, mask state, root degree, lim, last seed level
     __shared__ BigSmem S;
     __shared__ ChunkSmem I;              // long rows of the current up level
     __shared__ int s_l1[kChunk];
@@ -179,13 +182,21 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
             const int wend = min(ins + kBlock, a.ins_end);
             {
                 const int j = ins + tid;
-                bool work = false;
+                bool work = false, c3 = false;
                 if (j < wend) {
                     const int u = __ldg(a.ins_u + j), v = __ldg(a.ins_v + j);
-                    work = st.dist(u) != st.dist(v);
+                    const int du = st.dist(u), dv = st.dist(v);
+                    work = du != dv;
+                    c3 = work && (min(du, dv) + 1 != max(du, dv));
+                    s_wul[tid] = du < dv ? v : u;
+                    s_wlev[tid] = max(du, dv);
                 }
                 const unsigned bal = __ballot_sync(kFull, work);
-                if ((tid & 31) == 0) s_work[tid >> 5] = bal;
+                const unsigned bal3 = __ballot_sync(kFull, c3);
+                if ((tid & 31) == 0) {
+                    s_work[tid >> 5] = bal;
+                    s_c3[tid >> 5] = bal3;
+                }
             }
             __syncthreads();
             int p = ins;
@@ -203,8 +214,36 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                 ++prof_jobs;
                 const uint32_t E = epoch << 2;
                 const uint32_t mD = E | kDown, mU = E | kUp;
-                if (tid < 32) {  // warp 0: the root's row as of this insertion (level-2 masks)
-                    const int2 rs = row_of(g, sroot, p);
+                // A Case-2 insertion changes no distance, so a run of them (Case-1
+                // insertions in between are no-ops; it ends before the next Case 3)
+                // is repaired as ONE job whose D is seeded with every u_low: d and
+                // sigma after it are those of the graph with all the run's edges --
+                // exactly what the insertions one by one give (R18).
+                int glast = off;  // window offset of the job's last insertion
+                if (a.merge && !((s_c3[off >> 5] >> (off & 31)) & 1u)) {
+                    const int nwin = wend - ins;
+                    int c3pos = nwin;  // first Case 3 after off
+                    for (int w = (off >> 5); w < kWarps && w * 32 < nwin; ++w) {
+                        uint32_t b = s_c3[w];
+                        if (w == (off >> 5)) b &= ~((2u << (off & 31)) - 1u);
+                        if (b) {
+                            c3pos = min(nwin, w * 32 + __ffs(b) - 1);
+                            break;
+                        }
+                    }
+                    for (int w = (c3pos - 1) >> 5; w >= (off >> 5); --w) {  // last Case 2 before it
+                        uint32_t b = s_work[w] & ~s_c3[w];
+                        const int hi = c3pos - 32 * w;  // positions < c3pos
+                        if (hi < 32) b &= (1u << hi) - 1u;
+                        if (b) {
+                            glast = w * 32 + 31 - __clz(b);
+                            break;
+                        }
+                    }
+                }
+                const int lim = ins + glast;  // graph as of the job's last insertion
+                if (tid < 32) {  // warp 0: the root's row as of this job (level-2 masks)
+                    const int2 rs = row_of(g, sroot, lim);
                     const int dsr = rs.y - rs.x;
                     if (dsr <= kMaskDeg && tid < dsr) s_adjs[tid] = ldg_i(g.col + rs.x + tid);
                     if (tid == 0) {
@@ -214,6 +253,19 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                         s_job[5] = dsr;
                         if (dsr > kMaskDeg && built >= 0) a.mask_ds[slot] = -1;
                     }
+                }
+                const bool group = glast != off;
+                if (group) {  // seed levels: min and max d[u_low] over the run's Case-2 insertions
+                    if (tid == 0) {
+                        s_job[2] = INT32_MAX;
+                        s_job[7] = 0;
+                    }
+                    __syncthreads();
+                    for (int q = off + tid; q <= glast; q += kBlock)
+                        if (((s_work[q >> 5] & ~s_c3[q >> 5]) >> (q & 31)) & 1u) {
+                            atomicMin(&s_job[2], s_wlev[q]);
+                            atomicMax(&s_job[7], s_wlev[q]);
+                        }
                 }
                 if (tid == 0) {
                     const int u = __ldg(a.ins_u + p), v = __ldg(a.ins_v + p);
@@ -225,31 +277,64 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                     const bool c3 = dlo > L0;
                     if (c3)
                         st_c3++;
-                    else
-                        st_c2++;
                     st_bytes += 8;
                     if (c3) {
                         lowrec[ul] = ((unsigned long long)epoch << 32) | (uint32_t)dlo;
                         st.d[ul] = L0;
                     }
-                    mark[ul] = mD;
-                    Dv[0] = ul;
                     Doff[0] = 0;
-                    Doff[1] = 1;
-                    s_dcnt = 1;
+                    if (!group) {
+                        st_c2 += !c3;
+                        mark[ul] = mD;
+                        Dv[0] = ul;
+                        Doff[1] = 1;
+                        s_dcnt = 1;
+                        s_job[2] = L0;
+                        s_job[7] = L0;
+                    } else {
+                        s_dcnt = 0;
+                    }
                     s_ucnt2[0] = 0;
                     s_ucnt2[1] = 0;
                     s_rcnt = 0;
                     s_rmax = 0;
                     s_job[0] = uh;
                     s_job[1] = ul;
-                    s_job[2] = L0;
                     s_job[3] = c3;
                 }
                 __syncthreads();
                 const int uh = s_job[0], ul = s_job[1], L0 = s_job[2];
+                const int Lseed = s_job[7];  // deepest seed level
+                const int g0 = p;            // the job's insertions: g0 .. lim
                 const bool case3 = s_job[3] != 0;
                 const int mstate = s_job[4], dsr = s_job[5];
+                // group: enqueue the not yet claimed u_low of level Lq (Case 2 of the run)
+                auto inject = [&](int Lq) {
+                    for (int q = off + tid; q <= glast; q += kBlock)
+                        if (((s_work[q >> 5] & ~s_c3[q >> 5]) >> (q & 31)) & 1u && s_wlev[q] == Lq) {
+                            const int w = s_wul[q];
+                            if (atomicMax(mark + w, mD) < mD) Dv[atomicAdd(&s_dcnt, 1)] = w;
+                        }
+                };
+                if (group) {
+                    inject(L0);
+                    __syncthreads();
+                    if (tid == 0) {
+                        Doff[1] = s_dcnt;
+                        int c2 = 0;
+                        for (int w = (off >> 5); w <= (glast >> 5); ++w) {
+                            uint32_t b = s_work[w] & ~s_c3[w];
+                            if (w == (off >> 5)) b &= ~((1u << (off & 31)) - 1u);
+                            if (w == (glast >> 5) && (glast & 31) != 31) b &= (2u << (glast & 31)) - 1u;
+                            c2 += __popc(b);
+                        }
+                        st_c2 += c2;
+                        st_c1 += (glast - off + 1) - c2;  // Case-1 insertions inside the run
+                        atomicAdd(a.stats + kStGroups, 1ull);
+                        atomicAdd(a.stats + kStGroupIns, (unsigned long long)c2);
+                    }
+                    __syncthreads();
+                }
                 const bool mvalid = mstate == 1;  // masks usable during this job's down phase
                 // bit of a level-1 vertex in the masks (its position in the root's row)
                 auto l1bit = [&](int y) -> uint32_t {
@@ -257,11 +342,10 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                         if (s_adjs[j] == y) return 1u << j;
                     return 0u;
                 };
-                const int lim = p;  // graph as of this insertion (edge p included)
 
                 tick(-1);
                 // ================= down phase (K3) =================
-                int L = L0, lb = 0, le = 1, nlev = 1;
+                int L = L0, lb = 0, le = group ? Doff[1] : 1, nlev = 1;
                 // per-D-entry epilogue: record old d / sigma, store the new sigma
                 // (and, at level 2, the vertex's level-1 predecessor mask)
                 auto down_finish = [&](int idx, int w, double sum, uint32_t m) {
@@ -370,14 +454,18 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                         }
                         __syncthreads();
                     }
+                    if (L < Lseed) {  // seeds of the next level (claimed children stay once)
+                        inject(L + 1);
+                        __syncthreads();
+                    }
                     const int ne = s_dcnt;
                     __syncthreads();  // everyone has read nbig / ne
                     if (tid == 0) {
                         s_nbig = 0;
-                        if (ne != le) Doff[nlev + 1] = ne;
+                        if (ne != le || L < Lseed) Doff[nlev + 1] = ne;
                     }
                     __syncthreads();  // reset visible before the next level enqueues
-                    if (ne == le) break;
+                    if (ne == le && L >= Lseed) break;
                     lb = le;
                     le = ne;
                     ++nlev;
@@ -504,10 +592,10 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                         return __dmul_rn(__ddiv_rn(sx, sy), __dadd_rn(1.0, dly));
                     };
                     auto dpush_visit = [&](int x, double sx, double dn, double odel, double osig,
-                                           bool not_pulled, int pp, double sp, uint32_t mp) {
+                                           int meta, int pp, double sp, uint32_t mp) {
                         if (mp == mD) return;
                         double dlt = __dmul_rn(__ddiv_rn(sp, sx), 1.0 + dn);
-                        if (not_pulled && !(pp == uh && x == ul))
+                        if ((meta & kMetaNotPulled) && !((meta & kMetaNew) && new_edge(g, x, pp, g0, lim)))
                             dlt = __dsub_rn(dlt, __dmul_rn(__ddiv_rn(sp, osig), 1.0 + odel));
                         atomicAdd(dacc + pp, dlt);
                         st_bytes += 24;
@@ -554,7 +642,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                             c0 = s2.x;                // sigma (new)
                             c1 = s2.y;                // delta (old)
                             c2 = Dsig[idx];
-                            meta = (Dold[idx] == l) ? kMetaNotPulled : 0;
+                            meta = ((Dold[idx] == l) ? kMetaNotPulled : 0) | ((ldg_i(g.rp + x) < 0) ? kMetaNew : 0);
                             r = row_of(g, x, lim);
                             st_bytes += 8 + 16 + 8 + 4;
                             return true;
@@ -642,8 +730,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                                 row_walk(g, st, mark, r, [&](int dp) { return dp == l - 1; },
                                          [&](int pp, int dp, double2 q, uint32_t mp) {
                                              if (dp == l - 1)
-                                                 dpush_visit(x, c0, dn, c1, c2, (meta & kMetaNotPulled) != 0, pp,
-                                                             q.x, mp);
+                                                 dpush_visit(x, c0, dn, c1, c2, meta, pp, q.x, mp);
                                          });
                                 sc_dpush += r.y - r.x;
                                 st_bytes += 8ull * (r.y - r.x);
@@ -743,8 +830,8 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                                 HelpCtx cx;
                                 cx.root_slot = slot;
                                 cx.l = l;
-                                cx.uh = uh;
-                                cx.ul = ul;
+                                cx.g0 = g0;
+                                cx.lim = lim;
                                 cx.cnt = nb;
                                 cx.nblocks = nblk;
                                 cx.E2 = E2;
@@ -808,8 +895,8 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                                         if (meta & kMetaUp)
                                             up_visit(I.c1[t], I.c0[t], pp, sp, mp);
                                         else
-                                            dpush_visit(I.v[t], I.c0[t], I.acc[t], I.c1[t], I.c2[t],
-                                                        (meta & kMetaNotPulled) != 0, pp, sp, mp);
+                                            dpush_visit(I.v[t], I.c0[t], I.acc[t], I.c1[t], I.c2[t], meta, pp, sp,
+                                                        mp);
                                         return 0.0;
                                     });
                             tick(9);
@@ -880,6 +967,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                     ++p;
                     break;
                 }
+                p = lim;  // a group job: continue after its last insertion
             }
             ins = p;
             __syncthreads();  // s_work is rewritten by the next window
@@ -944,8 +1032,8 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                     const HelpCtx *src = a.help.ctx + pick;
                     s_hctx.root_slot = __ldcg(&src->root_slot);
                     s_hctx.l = __ldcg(&src->l);
-                    s_hctx.uh = __ldcg(&src->uh);
-                    s_hctx.ul = __ldcg(&src->ul);
+                    s_hctx.g0 = __ldcg(&src->g0);
+                    s_hctx.lim = __ldcg(&src->lim);
                     s_hctx.cnt = __ldcg(&src->cnt);
                     s_hctx.nblocks = __ldcg(&src->nblocks);
                     s_hctx.E2 = __ldcg(&src->E2);

@@ -22,6 +22,7 @@ FLAG_MODE_S = 0x1
 FLAG_TIMING = 0x2
 FLAG_EXACT_BC = 0x4
 FLAG_NO_REORDER = 0x8
+FLAG_NO_MERGE = 0x10
 
 STATUS = {
     0: "DBC_OK", -1: "DBC_EINVAL", -2: "DBC_ENOMEM", -3: "DBC_ECUDA", -4: "DBC_ENCCL",
@@ -258,7 +259,8 @@ class DynamicBC:
                  "static_bytes", "sc_down", "sc_removal", "sc_dpull", "sc_dpush", "sc_up2", "sc_up3",
                  "ns_down", "ns_removal", "ns_up_setup", "ns_up_epi", "ns_up_l1pairs", "ns_up_end",
                  "ns_up_split", "ns_up_scan", "ns_up_pull", "ns_up_push", "levels_down", "levels_up",
-                 "help_requests", "help_blocks_by_helpers", "help_blocks_all"]
+                 "help_requests", "help_blocks_by_helpers", "help_blocks_all",
+                 "case2_groups", "case2_group_insertions"]
         out = np.zeros(len(names), dtype=np.int64)
         _check(self._ctx, self._lib.dbc_debug_counters(self._ctx, _np_ptr(out), out.size))
         return dict(zip(names, out.tolist()))

@@ -416,3 +416,30 @@ def test_help_off_matches_help_on(monkeypatch):
     assert_bc(outs[1][0], outs[0][0])
     for (d0, s0), (d1, s1) in zip(outs[0][1], outs[1][1]):
         assert np.array_equal(d0, d1) and np.array_equal(s0, s1)
+
+
+@pytest.mark.parametrize("name", ["karate", "rmat10", "delaunay12u", "smallworld"])
+def test_case2_groups_match_oracle_and_no_merge(name):
+    """Runs of Case-2 insertions repaired as one multi-seed job (default) give the
+    oracle's d/sigma bit-exact and BC within tolerance, and the same d/sigma as
+    DBC_FLAG_NO_MERGE (one job per insertion); group jobs actually formed."""
+    from paper_conf_ipps_mclaughlinb14_b200 import FLAG_NO_MERGE
+
+    wl = W.make_workload(name)
+    ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
+    for u, v in zip(wl.ins_u, wl.ins_v):
+        ref.insert(u, v)
+    want = ref.compute()
+    outs = []
+    for flags in (FLAG_NO_MERGE, 0):
+        with _dbc(wl.graph, wl.roots, flags=flags) as dbc:
+            dbc.static_compute()
+            c0 = dbc.debug_counters()
+            dbc.insert_edges(wl.ins_u, wl.ins_v)
+            c1 = dbc.debug_counters()
+            check_all(dbc, want, wl.roots.size)
+            outs.append([dbc.get_root_state(s)[:2] for s in range(wl.roots.size)])
+            groups = c1["case2_groups"] - c0["case2_groups"]
+            assert (groups == 0) if flags else (groups > 0 or name == "karate")
+    for (d0, s0), (d1, s1) in zip(*outs):
+        assert np.array_equal(d0, d1) and np.array_equal(s0, s1)
