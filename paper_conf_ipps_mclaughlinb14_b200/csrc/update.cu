@@ -101,8 +101,8 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
     __shared__ uint32_t s_work[kWarps];  // window classification bits (1 = Case 2/3)
     __shared__ uint32_t s_c3[kWarps];    // window classification bits (1 = Case 3)
     __shared__ int s_wul[kBlock];        // window: u_low of each insertion
-    __shared__ int s_wlev[kBlock];       // window: d[u_low] + 0 (Case 2: its level)
-    __shared__ int s_job[8];             // uh, ul, L0, case3, mask state, root degree, lim, last seed level
+    __shared__ int s_wlev[kBlock];       // window: seed level d[u_high] + 1 (INT32_MAX: Case 1)
+    __shared__ int s_job[8];             // [2] lowest seed level, [3] any lowering, [4] mask state, [5] root degree, [7] deepest seed level
     __shared__ BigSmem S;
     __shared__ ChunkSmem I;              // long rows of the current up level
     __shared__ int s_l1[kChunk];
@@ -173,23 +173,31 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
         const unsigned long long prof_lv0 = st_lvd + st_lvu;
         if (a.root_prof && tid == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(prof_t0));
 
-        // Insertions are walked in order.  Classification (K2) of a window of
-        // kBlock insertions runs in parallel against the current d; a Case-2
-        // job leaves d unchanged so the window stays valid, a Case-3 job
-        // lowers distances, so the window is re-classified after it.
+        // Insertions are taken in windows (kBlock of them, or 1 with
+        // DBC_FLAG_NO_MERGE).  A window is ONE job (R18): every
+        // insertion e = (a, b) with d[a] < d[b] at the window start is a seed
+        // of level d[a] + 1, injected when the down phase reaches that level if
+        // a still has that distance (else a was lowered, is in D, and its own
+        // row walk covers e); b is then lowered (Case 3) or just
+        // claimed (Case 2).  The result is the state of the graph
+        // with all of the window's edges -- what the insertions one by one give.
+        const int win = a.merge ? kBlock : 1;
         int ins = a.ins_begin;
         while (ins < a.ins_end) {
-            const int wend = min(ins + kBlock, a.ins_end);
-            {
+            const int wend = min(ins + win, a.ins_end);
+            const int nwin = wend - ins;
+            {  // classification (K2) against the window-start distances
                 const int j = ins + tid;
                 bool work = false, c3 = false;
+                int lev = INT32_MAX;
                 if (j < wend) {
                     const int u = __ldg(a.ins_u + j), v = __ldg(a.ins_v + j);
                     const int du = st.dist(u), dv = st.dist(v);
                     work = du != dv;
                     c3 = work && (min(du, dv) + 1 != max(du, dv));
                     s_wul[tid] = du < dv ? v : u;
-                    s_wlev[tid] = max(du, dv);
+                    lev = work ? min(du, dv) + 1 : INT32_MAX;
+                    s_wlev[tid] = lev;
                 }
                 const unsigned bal = __ballot_sync(kFull, work);
                 const unsigned bal3 = __ballot_sync(kFull, c3);
@@ -197,51 +205,46 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                     s_work[tid >> 5] = bal;
                     s_c3[tid >> 5] = bal3;
                 }
+                if (tid == 0) {
+                    s_job[2] = INT32_MAX;  // lowest seed level
+                    s_job[7] = 0;          // deepest seed level
+                    s_job[3] = 0;          // any distance lowered in this job
+                }
+                __syncthreads();
+                if (work) {
+                    atomicMin(&s_job[2], lev);
+                    atomicMax(&s_job[7], lev);
+                }
             }
             __syncthreads();
-            int p = ins;
-            for (; p < wend; ++p) {
-                const int off = p - ins;
-                if (!((s_work[off >> 5] >> (off & 31)) & 1u)) {  // Case 1: no work
-                    if (tid == 0) {
-                        st_c1++;
-                        st_bytes += 8;
+            {
+                int nw = 0, n3 = 0;
+                for (int w = 0; w * 32 < nwin; ++w) {
+                    nw += __popc(s_work[w]);
+                    n3 += __popc(s_c3[w]);
+                }
+                if (tid == 0) {
+                    st_c1 += nwin - nw;
+                    st_c2 += nw - n3;
+                    st_c3 += n3;
+                    st_bytes += 8ull * nwin;
+                    if (nw > 1) {
+                        atomicAdd(a.stats + kStGroups, 1ull);
+                        atomicAdd(a.stats + kStGroupIns, (unsigned long long)nw);
                     }
+                }
+                if (nw == 0) {  // Case 1 throughout: nothing changes
+                    ins = wend;
+                    __syncthreads();  // s_work is rewritten by the next window
                     continue;
                 }
-                // ---------------- classify + seed (tid 0, broadcast) ----------------
+            }
+            {
                 ++epoch;
                 ++prof_jobs;
                 const uint32_t E = epoch << 2;
                 const uint32_t mD = E | kDown, mU = E | kUp;
-                // A Case-2 insertion changes no distance, so a run of them (Case-1
-                // insertions in between are no-ops; it ends before the next Case 3)
-                // is repaired as ONE job whose D is seeded with every u_low: d and
-                // sigma after it are those of the graph with all the run's edges --
-                // exactly what the insertions one by one give (R18).
-                int glast = off;  // window offset of the job's last insertion
-                if (a.merge && !((s_c3[off >> 5] >> (off & 31)) & 1u)) {
-                    const int nwin = wend - ins;
-                    int c3pos = nwin;  // first Case 3 after off
-                    for (int w = (off >> 5); w < kWarps && w * 32 < nwin; ++w) {
-                        uint32_t b = s_c3[w];
-                        if (w == (off >> 5)) b &= ~((2u << (off & 31)) - 1u);
-                        if (b) {
-                            c3pos = min(nwin, w * 32 + __ffs(b) - 1);
-                            break;
-                        }
-                    }
-                    for (int w = (c3pos - 1) >> 5; w >= (off >> 5); --w) {  // last Case 2 before it
-                        uint32_t b = s_work[w] & ~s_c3[w];
-                        const int hi = c3pos - 32 * w;  // positions < c3pos
-                        if (hi < 32) b &= (1u << hi) - 1u;
-                        if (b) {
-                            glast = w * 32 + 31 - __clz(b);
-                            break;
-                        }
-                    }
-                }
-                const int lim = ins + glast;  // graph as of the job's last insertion
+                const int g0 = ins, lim = wend - 1;  // the job's insertions; graph as of lim
                 if (tid < 32) {  // warp 0: the root's row as of this job (level-2 masks)
                     const int2 rs = row_of(g, sroot, lim);
                     const int dsr = rs.y - rs.x;
@@ -254,87 +257,42 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                         if (dsr > kMaskDeg && built >= 0) a.mask_ds[slot] = -1;
                     }
                 }
-                const bool group = glast != off;
-                if (group) {  // seed levels: min and max d[u_low] over the run's Case-2 insertions
-                    if (tid == 0) {
-                        s_job[2] = INT32_MAX;
-                        s_job[7] = 0;
-                    }
-                    __syncthreads();
-                    for (int q = off + tid; q <= glast; q += kBlock)
-                        if (((s_work[q >> 5] & ~s_c3[q >> 5]) >> (q & 31)) & 1u) {
-                            atomicMin(&s_job[2], s_wlev[q]);
-                            atomicMax(&s_job[7], s_wlev[q]);
-                        }
-                }
                 if (tid == 0) {
-                    const int u = __ldg(a.ins_u + p), v = __ldg(a.ins_v + p);
-                    const int du = st.dist(u), dv = st.dist(v);
-                    const bool u_is_high = du < dv;
-                    const int uh = u_is_high ? u : v, ul = u_is_high ? v : u;
-                    const int dh = u_is_high ? du : dv, dlo = u_is_high ? dv : du;
-                    const int L0 = dh + 1;
-                    const bool c3 = dlo > L0;
-                    if (c3)
-                        st_c3++;
-                    st_bytes += 8;
-                    if (c3) {
-                        lowrec[ul] = ((unsigned long long)epoch << 32) | (uint32_t)dlo;
-                        st.d[ul] = L0;
-                    }
                     Doff[0] = 0;
-                    if (!group) {
-                        st_c2 += !c3;
-                        mark[ul] = mD;
-                        Dv[0] = ul;
-                        Doff[1] = 1;
-                        s_dcnt = 1;
-                        s_job[2] = L0;
-                        s_job[7] = L0;
-                    } else {
-                        s_dcnt = 0;
-                    }
+                    s_dcnt = 0;
                     s_ucnt2[0] = 0;
                     s_ucnt2[1] = 0;
                     s_rcnt = 0;
                     s_rmax = 0;
-                    s_job[0] = uh;
-                    s_job[1] = ul;
-                    s_job[3] = c3;
                 }
                 __syncthreads();
-                const int uh = s_job[0], ul = s_job[1], L0 = s_job[2];
-                const int Lseed = s_job[7];  // deepest seed level
-                const int g0 = p;            // the job's insertions: g0 .. lim
-                const bool case3 = s_job[3] != 0;
+                const int L0 = s_job[2];
+                const int Lseed = s_job[7];
                 const int mstate = s_job[4], dsr = s_job[5];
-                // group: enqueue the not yet claimed u_low of level Lq (Case 2 of the run)
+                // enqueue the seeds of level Lq (between levels: no concurrent lowering)
                 auto inject = [&](int Lq) {
-                    for (int q = off + tid; q <= glast; q += kBlock)
-                        if (((s_work[q >> 5] & ~s_c3[q >> 5]) >> (q & 31)) & 1u && s_wlev[q] == Lq) {
-                            const int w = s_wul[q];
-                            if (atomicMax(mark + w, mD) < mD) Dv[atomicAdd(&s_dcnt, 1)] = w;
+                    for (int q = tid; q < nwin; q += kBlock) {
+                        if (s_wlev[q] != Lq) continue;
+                        const int b = s_wul[q];
+                        const int u = __ldg(a.ins_u + ins + q), v = __ldg(a.ins_v + ins + q);
+                        const int hi = (u == b) ? v : u;
+                        if (st.d[hi] != Lq - 1) continue;  // lowered: in D, its row walk covers e
+                        const int db = st.d[b];
+                        if (db < Lq) continue;
+                        if (db > Lq) {  // Case 3: pull b up to level Lq
+                            const int old = atomicMin(st.d + b, Lq);
+                            if (old > Lq) {
+                                lowrec[b] = ((unsigned long long)epoch << 32) | (uint32_t)old;
+                                s_job[3] = 1;
+                            }
                         }
-                };
-                if (group) {
-                    inject(L0);
-                    __syncthreads();
-                    if (tid == 0) {
-                        Doff[1] = s_dcnt;
-                        int c2 = 0;
-                        for (int w = (off >> 5); w <= (glast >> 5); ++w) {
-                            uint32_t b = s_work[w] & ~s_c3[w];
-                            if (w == (off >> 5)) b &= ~((1u << (off & 31)) - 1u);
-                            if (w == (glast >> 5) && (glast & 31) != 31) b &= (2u << (glast & 31)) - 1u;
-                            c2 += __popc(b);
-                        }
-                        st_c2 += c2;
-                        st_c1 += (glast - off + 1) - c2;  // Case-1 insertions inside the run
-                        atomicAdd(a.stats + kStGroups, 1ull);
-                        atomicAdd(a.stats + kStGroupIns, (unsigned long long)c2);
+                        if (atomicMax(mark + b, mD) < mD) Dv[atomicAdd(&s_dcnt, 1)] = b;
                     }
-                    __syncthreads();
-                }
+                };
+                inject(L0);
+                __syncthreads();
+                const int le0 = s_dcnt;
+                if (tid == 0) Doff[1] = le0;
                 const bool mvalid = mstate == 1;  // masks usable during this job's down phase
                 // bit of a level-1 vertex in the masks (its position in the root's row)
                 auto l1bit = [&](int y) -> uint32_t {
@@ -345,7 +303,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
 
                 tick(-1);
                 // ================= down phase (K3) =================
-                int L = L0, lb = 0, le = group ? Doff[1] : 1, nlev = 1;
+                int L = L0, lb = 0, le = le0, nlev = 1;
                 // per-D-entry epilogue: record old d / sigma, store the new sigma
                 // (and, at level 2, the vertex's level-1 predecessor mask)
                 auto down_finish = [&](int idx, int w, double sum, uint32_t m) {
@@ -368,6 +326,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                         const int old = atomicMin(st.d + y, L + 1);
                         if (old > L + 1) {
                             lowrec[y] = ((unsigned long long)epoch << 32) | (uint32_t)old;
+                            s_job[3] = 1;
                             st_bytes += 4;
                         }
                         dy = L + 1;
@@ -413,6 +372,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                                     }
                                     if (dy[u] > L + 1 && om[u] > L + 1) {  // first lowerer (Case 3)
                                         lowrec[y[u]] = ((unsigned long long)epoch << 32) | (uint32_t)om[u];
+                                        s_job[3] = 1;
                                         st_bytes += 4;
                                     }
                                     if (dy[u] >= L + 1 && oc[u] < mD) Dv[atomicAdd(&s_dcnt, 1)] = y[u];
@@ -486,6 +446,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                     if (tid == 0) a.mask_ds[slot] = dsr;
                 }
                 const bool mok = mstate != 0;  // masks valid for the up phase
+                const bool case3 = s_job[3] != 0;  // some distance was lowered (read after the level barriers)
 
                 tick(0);
                 // ================= (0) Case-3 removal pushes =================
@@ -493,8 +454,9 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                     // a pulled-up w (finite old level od) loses its old predecessors x
                     auto rem_visit = [&](int w, int od, double osig, double coef, int x, int dx,
                                          double sx) {
-                        if (dx != od - 1 || (x == uh && w == ul)) return;
+                        if (dx != od - 1) return;
                         if (mark[x] == mD) return;
+                        if (ldg_i(g.rp + w) < 0 && new_edge(g, w, x, g0, lim)) return;  // not an old predecessor
                         atomicAdd(dacc + x, -__dmul_rn(__ddiv_rn(sx, osig), coef));
                         st_bytes += 24;
                         if (atomicMax(mark + x, mU) < E) {
@@ -963,13 +925,8 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                     tick(5);
                 }
                 // any up vertices left at level 0 would be the root: never produced
-                if (case3) {  // distances changed: re-classify from the next insertion
-                    ++p;
-                    break;
-                }
-                p = lim;  // a group job: continue after its last insertion
             }
-            ins = p;
+            ins = wend;
             __syncthreads();  // s_work is rewritten by the next window
         }
         if (a.help.word && tid == 0) atomicSub(a.help.roots_left, 1);
