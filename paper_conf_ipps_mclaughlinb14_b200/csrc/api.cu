@@ -453,6 +453,10 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->ws.Rl, wn);
     AL(c->ws.Bq, wn);
     AL(c->ws.wepoch, nwk);
+    c->ws.wcap = kWindow;
+    if (const char *e = getenv("DBC_WINDOW")) c->ws.wcap = std::max(1, atoi(e));
+    AL(c->ws.Wul, nwk * (size_t)c->ws.wcap);
+    AL(c->ws.Wlev, nwk * (size_t)c->ws.wcap);
     AL(c->help.word, nwk);
     AL(c->help.done, nwk);
     AL(c->help.ctx, nwk);

@@ -87,6 +87,8 @@ struct Scratch {
     int32_t *U0, *U1;          // up frontier overflow ping-pong
     int32_t *Rv, *Rl;          // removal-push targets and their levels (Case 3)
     int32_t *Bq;               // long-row queue of the current level, n per worker
+    int32_t *Wul, *Wlev;       // window of insertions: u_low and seed level, wcap per worker
+    int32_t wcap;              // window capacity (insertions per job)
     uint32_t *wepoch;          // per-worker epoch counter
 };
 
@@ -206,6 +208,7 @@ struct BigSmem {
     double acc[kBig];   // per-row reduction
     double c0[kBig];    // per-row constant of the caller
     unsigned mk[kBig];  // per-row level-2 predecessor mask being built
+    int ext[kBig];      // per-row: a predecessor outside D was seen (update down phase)
     int m;            // rows in this round
 };
 
@@ -331,10 +334,12 @@ __device__ __forceinline__ void big_entries(BigSmem &S, const GView &g, const Ro
 
 // --- up phase: chunked flattened level pass ----------------------------------
 constexpr int kChunk = 512;   // items per chunk (shared memory)
-constexpr int kUcap = kBlock >= 512 ? 768 : 1024;   // up-frontier entries kept in shared memory
+constexpr int kUcap = 1024;   // up-frontier entries kept in shared memory
 constexpr int kMetaUp = 1, kMetaNotPulled = 2, kMetaMask = 4;
 constexpr int kMetaNew = 8;  // down row with batch entries: its pushes check new_edge()
+constexpr int kMetaExt = 16; // down row with a predecessor outside D: it has pushes to make
 constexpr int kFlatU = 4;     // contiguous entries per thread per step
+constexpr int kWindow = 4096;  // default insertions per Mode-A job (DBC_WINDOW overrides)
 constexpr int kAdjCap = 256;  // longest root row kept in shared memory (level-2 shortcut)
 
 struct ChunkSmem {
@@ -520,7 +525,7 @@ struct UpdateArgs {
     int32_t slot_count;            // entries of slot_list
     int32_t worker_base;           // scratch index of CTA 0
     HelpBoard help;                // help.word == nullptr: no cooperative help
-    int32_t merge;                 // 1: repair runs of Case-2 insertions as one job
+    int32_t merge;                 // 1: a window of ws.wcap insertions per job; 0: one per insertion
 };
 
 struct StaticArgs {

@@ -46,6 +46,11 @@ constexpr bool kPhaseTimers = false;
 #endif
 
 namespace {
+// Dold[i] = old level of D[i] (low 31 bits) | kExtPred if D[i] has a predecessor
+// outside D (only such rows push in the up phase)
+constexpr int32_t kOldMask = 0x7fffffff;
+constexpr int32_t kExtPred = INT32_MIN;
+
 // One push of a helped C2 pass (owner or helper): the same arithmetic as the
 // owner's up_visit / dpush_visit, with claims appended to the global list.
 __device__ __forceinline__ void help_push_entry(const GView &g, const ChunkSmem &M, int t, int pp, int dp,
@@ -96,12 +101,10 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
     __shared__ int s_rmax;     // deepest removal-push target level
     __shared__ int s_nbig;     // long-row queue (down phase / removal)
     __shared__ int s_nbigI;    // long rows of the current up level (in I)
+    __shared__ int s_noext;    // the chunk holds down rows without pushes
     __shared__ int s_nl1;      // of those, resolved against adj(root)
     __shared__ int s_ds;       // |adj(root)| as of the insertion (-1: too long)
-    __shared__ uint32_t s_work[kWarps];  // window classification bits (1 = Case 2/3)
-    __shared__ uint32_t s_c3[kWarps];    // window classification bits (1 = Case 3)
-    __shared__ int s_wul[kBlock];        // window: u_low of each insertion
-    __shared__ int s_wlev[kBlock];       // window: seed level d[u_high] + 1 (INT32_MAX: Case 1)
+    __shared__ int s_wcnt[2];            // window: insertions with work, of which Case 3
     __shared__ int s_job[8];             // [2] lowest seed level, [3] any lowering, [4] mask state, [5] root degree, [7] deepest seed level
     __shared__ BigSmem S;
     __shared__ ChunkSmem I;              // long rows of the current up level
@@ -129,6 +132,8 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
     int32_t *Rv = a.ws.Rv + (size_t)wk * n;
     int32_t *Rl = a.ws.Rl + (size_t)wk * n;
     int32_t *Bq = a.ws.Bq + (size_t)wk * n;
+    int32_t *Wul = a.ws.Wul + (size_t)wk * a.ws.wcap;    // window: u_low of each insertion
+    int32_t *Wlev = a.ws.Wlev + (size_t)wk * a.ws.wcap;  // window: seed level d[u_high] + 1 (INT32_MAX: Case 1)
     uint32_t epoch = a.ws.wepoch[wk];
     const GView &g = a.g;
     int hseq = 0;  // this worker's help-request sequence
@@ -153,6 +158,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
         s_nbig = 0;
         s_nbigI = 0;
         s_nl1 = 0;
+        s_noext = 0;
     }
 
     for (;;) {
@@ -173,7 +179,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
         const unsigned long long prof_lv0 = st_lvd + st_lvu;
         if (a.root_prof && tid == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(prof_t0));
 
-        // Insertions are taken in windows (kBlock of them, or 1 with
+        // Insertions are taken in windows (ws.wcap of them, or 1 with
         // DBC_FLAG_NO_MERGE).  A window is ONE job (R18): every
         // insertion e = (a, b) with d[a] < d[b] at the window start is a seed
         // of level d[a] + 1, injected when the down phase reaches that level if
@@ -181,48 +187,53 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
         // row walk covers e); b is then lowered (Case 3) or just
         // claimed (Case 2).  The result is the state of the graph
         // with all of the window's edges -- what the insertions one by one give.
-        const int win = a.merge ? kBlock : 1;
+        const int win = a.merge ? a.ws.wcap : 1;
         int ins = a.ins_begin;
         while (ins < a.ins_end) {
             const int wend = min(ins + win, a.ins_end);
             const int nwin = wend - ins;
+            if (tid == 0) {
+                s_job[2] = INT32_MAX;  // lowest seed level
+                s_job[7] = 0;          // deepest seed level
+                s_job[3] = 0;          // any distance lowered in this job
+                s_wcnt[0] = 0;
+                s_wcnt[1] = 0;
+            }
+            __syncthreads();
             {  // classification (K2) against the window-start distances
-                const int j = ins + tid;
-                bool work = false, c3 = false;
-                int lev = INT32_MAX;
-                if (j < wend) {
-                    const int u = __ldg(a.ins_u + j), v = __ldg(a.ins_v + j);
+                int lmin = INT32_MAX, lmax = 0, cw = 0, c3n = 0;
+                for (int q = tid; q < nwin; q += kBlock) {
+                    const int u = __ldg(a.ins_u + ins + q), v = __ldg(a.ins_v + ins + q);
                     const int du = st.dist(u), dv = st.dist(v);
-                    work = du != dv;
-                    c3 = work && (min(du, dv) + 1 != max(du, dv));
-                    s_wul[tid] = du < dv ? v : u;
-                    lev = work ? min(du, dv) + 1 : INT32_MAX;
-                    s_wlev[tid] = lev;
+                    const bool work = du != dv;
+                    const int lev = work ? min(du, dv) + 1 : INT32_MAX;
+                    Wul[q] = du < dv ? v : u;
+                    Wlev[q] = lev;
+                    if (work) {
+                        ++cw;
+                        c3n += min(du, dv) + 1 != max(du, dv);
+                        lmin = min(lmin, lev);
+                        lmax = max(lmax, lev);
+                    }
                 }
-                const unsigned bal = __ballot_sync(kFull, work);
-                const unsigned bal3 = __ballot_sync(kFull, c3);
-                if ((tid & 31) == 0) {
-                    s_work[tid >> 5] = bal;
-                    s_c3[tid >> 5] = bal3;
+                // warp-aggregated, then one shared atomic per warp
+#pragma unroll
+                for (int o = 16; o; o >>= 1) {
+                    cw += __shfl_xor_sync(kFull, cw, o);
+                    c3n += __shfl_xor_sync(kFull, c3n, o);
+                    lmin = min(lmin, __shfl_xor_sync(kFull, lmin, o));
+                    lmax = max(lmax, __shfl_xor_sync(kFull, lmax, o));
                 }
-                if (tid == 0) {
-                    s_job[2] = INT32_MAX;  // lowest seed level
-                    s_job[7] = 0;          // deepest seed level
-                    s_job[3] = 0;          // any distance lowered in this job
-                }
-                __syncthreads();
-                if (work) {
-                    atomicMin(&s_job[2], lev);
-                    atomicMax(&s_job[7], lev);
+                if ((tid & 31) == 0 && cw) {
+                    atomicAdd(&s_wcnt[0], cw);
+                    atomicAdd(&s_wcnt[1], c3n);
+                    atomicMin(&s_job[2], lmin);
+                    atomicMax(&s_job[7], lmax);
                 }
             }
             __syncthreads();
             {
-                int nw = 0, n3 = 0;
-                for (int w = 0; w * 32 < nwin; ++w) {
-                    nw += __popc(s_work[w]);
-                    n3 += __popc(s_c3[w]);
-                }
+                const int nw = s_wcnt[0], n3 = s_wcnt[1];
                 if (tid == 0) {
                     st_c1 += nwin - nw;
                     st_c2 += nw - n3;
@@ -235,7 +246,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                 }
                 if (nw == 0) {  // Case 1 throughout: nothing changes
                     ins = wend;
-                    __syncthreads();  // s_work is rewritten by the next window
+                    __syncthreads();  // the counters are reset by the next window
                     continue;
                 }
             }
@@ -272,8 +283,8 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                 // enqueue the seeds of level Lq (between levels: no concurrent lowering)
                 auto inject = [&](int Lq) {
                     for (int q = tid; q < nwin; q += kBlock) {
-                        if (s_wlev[q] != Lq) continue;
-                        const int b = s_wul[q];
+                        if (Wlev[q] != Lq) continue;
+                        const int b = Wul[q];
                         const int u = __ldg(a.ins_u + ins + q), v = __ldg(a.ins_v + ins + q);
                         const int hi = (u == b) ? v : u;
                         if (st.d[hi] != Lq - 1) continue;  // lowered: in D, its row walk covers e
@@ -306,11 +317,11 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                 int L = L0, lb = 0, le = le0, nlev = 1;
                 // per-D-entry epilogue: record old d / sigma, store the new sigma
                 // (and, at level 2, the vertex's level-1 predecessor mask)
-                auto down_finish = [&](int idx, int w, double sum, uint32_t m) {
+                auto down_finish = [&](int idx, int w, double sum, uint32_t m, bool ext) {
                     if (mvalid && L == 2) mask[w] = m;
                     const unsigned long long lr = lowrec[w];
                     const int od = ((uint32_t)(lr >> 32) == epoch) ? (int)(uint32_t)lr : L;
-                    Dold[idx] = od;
+                    Dold[idx] = od | (ext ? kExtPred : 0);
                     Dsig[idx] = st.sd[w].x;
                     st.sd[w].x = sum;
                     if (!(sum <= 1.7976931348623157e308)) atomicOr(a.err, kErrNumeric);
@@ -341,17 +352,21 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                         [&](int i, int w, int2 r) {
                             double sum = 0.0;  // canonical order: bit-exact
                             uint32_t m = 0u;
+                            bool ext = false;
                             for (int j = r.x; j < r.y; j += kRowUnroll) {
                                 int y[kRowUnroll], dy[kRowUnroll], om[kRowUnroll];
-                                uint32_t oc[kRowUnroll];
+                                uint32_t oc[kRowUnroll], pm[kRowUnroll];
                                 double sy[kRowUnroll];
 #pragma unroll
                                 for (int u = 0; u < kRowUnroll; ++u) y[u] = (j + u < r.y) ? ldg_i(g.col + j + u) : -1;
 #pragma unroll
                                 for (int u = 0; u < kRowUnroll; ++u) dy[u] = (y[u] >= 0) ? st.d[y[u]] : kInf;
 #pragma unroll
-                                for (int u = 0; u < kRowUnroll; ++u)
-                                    sy[u] = (y[u] >= 0 && dy[u] == L - 1) ? st.sd[y[u]].x : 0.0;
+                                for (int u = 0; u < kRowUnroll; ++u) {
+                                    const bool pr = y[u] >= 0 && dy[u] == L - 1;
+                                    sy[u] = pr ? st.sd[y[u]].x : 0.0;
+                                    pm[u] = pr ? mark[y[u]] : mD;
+                                }
                                 // issue every lowering and claim of the block, then consume
 #pragma unroll
                                 for (int u = 0; u < kRowUnroll; ++u)
@@ -367,6 +382,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                                     if (y[u] < 0) continue;
                                     if (dy[u] == L - 1) {  // predecessor: canonical-order sum
                                         sum += sy[u];
+                                        ext |= pm[u] != mD;
                                         st_bytes += 8;
                                         if (mvalid && L == 2) m |= l1bit(y[u]);
                                     }
@@ -380,7 +396,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                             }
                             st_bytes += 8 + 8ull * (r.y - r.x);
                             sc_down += r.y - r.x;
-                            down_finish(lb + i, w, sum, m);
+                            down_finish(lb + i, w, sum, m, ext);
                         },
                         enq_front);
                     __syncthreads();
@@ -389,13 +405,17 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                         const int m = min(kBig, nbig - r0);
                         big_load(S, m, [&](int t) { return Bq[r0 + t]; }, [&](int i) { return Dv[lb + i]; },
                                  g, lim);
-                        if (tid < m) S.mk[tid] = 0u;
+                        if (tid < m) {
+                            S.mk[tid] = 0u;
+                            S.ext[tid] = 0;
+                        }
                         __syncthreads();
                         big_entries(S, g, st, [&](int dy) { return dy == L - 1; },
                                     [&](int t, int y, int dy, double2 q) {
                                         st_bytes += 8;
                                         sc_down++;
                                         if (mvalid && L == 2 && dy == 1) atomicOr(&S.mk[t], l1bit(y));
+                                        if (dy == L - 1 && mark[y] != mD) S.ext[t] = 1;
                                         return down_visit(y, dy, q.x);
                                     });
                         if (tid < m) {
@@ -410,7 +430,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                                 }
                             }
                             st_bytes += 8;
-                            down_finish(lb + S.idx[tid], w, sum, S.mk[tid]);
+                            down_finish(lb + S.idx[tid], w, sum, S.mk[tid], S.ext[tid] != 0);
                         }
                         __syncthreads();
                     }
@@ -469,12 +489,12 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                     split_pass(
                         dtotal, g, lim,
                         [&](int i, int &w) {
-                            const int od = Dold[i];
+                            const int od = Dold[i] & kOldMask;
                             w = Dv[i];
                             return od != kInf && od != st.dist(w);
                         },
                         [&](int i, int w, int2 r) {
-                            const int od = Dold[i];
+                            const int od = Dold[i] & kOldMask;
                             const double osig = Dsig[i];
                             const double coef = 1.0 + st.sd[w].y;  // delta still old
                             row_walk(g, st, nullptr, r, [&](int dx) { return dx == od - 1; },
@@ -494,7 +514,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                         if (tid < m) {
                             const int i = S.idx[tid];
                             S.c0[tid] = Dsig[i];
-                            s_l1[tid] = Dold[i];  // reused: old level of each row
+                            s_l1[tid] = Dold[i] & kOldMask;  // reused: old level of each row
                             st_bytes += 16;
                         }
                         __syncthreads();
@@ -604,7 +624,9 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                             c0 = s2.x;                // sigma (new)
                             c1 = s2.y;                // delta (old)
                             c2 = Dsig[idx];
-                            meta = ((Dold[idx] == l) ? kMetaNotPulled : 0) | ((ldg_i(g.rp + x) < 0) ? kMetaNew : 0);
+                            const int od = Dold[idx];
+                            meta = (((od & kOldMask) == l) ? kMetaNotPulled : 0) | ((od < 0) ? kMetaExt : 0) |
+                                   ((ldg_i(g.rp + x) < 0) ? kMetaNew : 0);
                             r = row_of(g, x, lim);
                             st_bytes += 8 + 16 + 8 + 4;
                             return true;
@@ -688,7 +710,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                                      [&](int, int dy, double2 q, uint32_t) { dn += dpull_visit(c0, dy, q.x, q.y); });
                             sc_dpull += r.y - r.x;
                             st_bytes += 8ull * (r.y - r.x);
-                            if (wantpush) {
+                            if (wantpush && (meta & kMetaExt)) {  // some predecessor outside D
                                 row_walk(g, st, mark, r, [&](int dp) { return dp == l - 1; },
                                          [&](int pp, int dp, double2 q, uint32_t mp) {
                                              if (dp == l - 1)
@@ -727,6 +749,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                                 s_l1[atomicAdd(&s_nl1, 1)] = t;
                                 elen = 0;
                             }
+                            if (!(meta & (kMetaUp | kMetaExt))) s_noext = 1;  // a down row without pushes
                             I.mk[t] = mk;
                             I.v[t] = x;
                             I.meta[t] = meta;
@@ -765,7 +788,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                             tick(7);
                             auto colf = [&](int t, int e) { return ldg_i(g.col + I.beg[t] + e - I.off[t]); };
                             // --- C1: delta pull of the long down rows (Eq. (2)) ---
-                            const int E1 = I.off[nDb], E2 = I.off[nb];
+                            const int E1 = I.off[nDb];
                             if (E1 > 0)
                                 flat_entries(I.off, nb, E1, colf, st, nullptr, [&](int dy) { return dy == l + 1; },
                                              I.acc, [&](int t, int, int dy, double2 q, uint32_t) {
@@ -774,7 +797,26 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                                                  return dpull_visit(I.c0[t], dy, q.x, q.y);
                                              });
                             tick(8);
-                            // --- C2: pushes towards level l-1 ---
+                            // --- C2: pushes towards level l-1 (down rows only if they have a
+                            // predecessor outside D: drop the others from the offsets) ---
+                            if (push && s_noext) {
+                                constexpr int per = (kChunk + kBlock - 1) / kBlock;
+                                int ln[per];
+#pragma unroll
+                                for (int k = 0; k < per; ++k) {
+                                    const int t = tid + k * kBlock;
+                                    ln[k] = (t < nb && (I.meta[t] & (kMetaUp | kMetaExt))) ? I.off[t + 1] - I.off[t] : 0;
+                                }
+                                __syncthreads();
+#pragma unroll
+                                for (int k = 0; k < per; ++k) {
+                                    const int t = tid + k * kBlock;
+                                    if (t < nb) I.off[t + 1] = ln[k];
+                                }
+                                __syncthreads();
+                                chunk_scan(I.off, nb);
+                            }
+                            const int E2 = I.off[nb];
                             const int nblk = (E2 + kHelpEntries - 1) / kHelpEntries;
                             if (push && E2 > 0 && a.help.word && nblk >= kHelpMinBlocks) {
                                 // publish the chunk; idle workers help block by block
@@ -911,6 +953,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                         if (tid == 0) {
                             s_nbigI = 0;
                             s_nl1 = 0;
+                            s_noext = 0;
                         }
                         __syncthreads();
                     }  // chunks
@@ -927,7 +970,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                 // any up vertices left at level 0 would be the root: never produced
             }
             ins = wend;
-            __syncthreads();  // s_work is rewritten by the next window
+            __syncthreads();  // the counters are reset by the next window
         }
         if (a.help.word && tid == 0) atomicSub(a.help.roots_left, 1);
         if (a.root_prof && tid == 0) {
