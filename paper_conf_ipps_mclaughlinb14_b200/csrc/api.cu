@@ -31,7 +31,9 @@ struct dbc_ctx {
     cudaStream_t stream = nullptr;
     bool own_stream = false;
     int workers = 0;
-    int block = 256;   // threads per worker CTA (256 or 128)
+    int block = 512;   // threads per update worker CTA (512, 256 or 128)
+    int sblock = 256, sworkers = 0;  // static kernel: its own CTA width and grid
+    size_t nscratch = 0;             // worker scratch sets allocated
     // heavy lanes: the slowest root chains of the previous batch run on
     // 2x-wide CTAs (hblock threads) on a high-priority stream
     int hblock = 512, heavy_cap = 0;
@@ -278,7 +280,7 @@ static GView view_of(const dbc_ctx *c) {
 static Scratch worker_scratch(const dbc_ctx *c) { return c->ws; }
 
 static dbc_status reset_epochs(dbc_ctx *c) {
-    const size_t nw = (size_t)c->workers + c->heavy_cap, n = (size_t)c->n;
+    const size_t nw = c->nscratch, n = (size_t)c->n;
     if (!nw) return DBC_OK;
     CK(cudaMemsetAsync(c->ws.mark, 0, sizeof(uint32_t) * nw * n, c->stream));
     CK(cudaMemsetAsync(c->ws.lowrec, 0, sizeof(unsigned long long) * nw * n, c->stream));
@@ -389,16 +391,21 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     cudaMemGetInfo(&free_b, &total_b);
     const size_t state_b = (size_t)c->k_loc * n * 24 + (size_t)c->col_cap * 8 + (size_t)n * 40;
     size_t budget = free_b > state_b ? (free_b - state_b) / 2 : 0;
-    // more roots than two 256-thread CTAs per SM can hold and no hub rows:
-    // 128-thread CTAs, four per SM, so that every root chain is resident at once
+    // Update: a job is a window of up to 4096 insertions whose levels are wide,
+    // so one 512-thread CTA per SM beats more, narrower CTAs.
+    // Static: more roots than two 256-thread CTAs per SM can hold and no hub
+    // rows -> 128-thread CTAs, four per SM, every root resident at once.
     int64_t maxdeg = 0;
     for (int32_t v = 0; v < n; ++v) maxdeg = std::max<int64_t>(maxdeg, row_ptr[v + 1] - row_ptr[v]);
-    c->block = (c->k_loc > 2 * c->nsm && maxdeg <= 256) ? 128 : 256;  // hubs need the wide CTA
-    if (const char *eb = getenv("DBC_BLOCK")) c->block = atoi(eb) == 128 ? 128 : (atoi(eb) == 512 ? 512 : 256);
+    c->sblock = (c->k_loc > 2 * c->nsm && maxdeg <= 256) ? 128 : 256;  // hubs need the wide CTA
+    c->block = 512;
+    if (const char *eb = getenv("DBC_BLOCK")) c->block = atoi(eb) == 128 ? 128 : (atoi(eb) == 256 ? 256 : 512);
     int want = opt.workers ? opt.workers : (c->block == 128 ? 4 : (c->block == 512 ? 1 : 2)) * c->nsm;
     want = std::min(want, c->k_loc);
     int fit = (int)std::min<size_t>(budget / per_worker, 1 << 20);
     c->workers = std::max(0, std::min(want, fit));
+    c->sworkers = std::max(0, std::min({opt.workers ? opt.workers : (c->sblock == 128 ? 4 : 2) * c->nsm,
+                                        c->k_loc, fit}));
     c->hblock = c->block == 128 ? 256 : 512;
     // only hub-heavy graphs (256-thread build) have step-bound slow roots
     c->heavy_cap = (c->block != 256 || opt.workers) ? 0 : std::max(0, std::min(c->nsm / 4, (int)(fit - c->workers)));
@@ -438,7 +445,8 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->bc_ext, (size_t)n);
     AL(c->perm_d, (size_t)n);
     AL(c->roots_d, (size_t)c->k_loc);
-    const size_t nwk = (size_t)c->workers + c->heavy_cap;  // scratch for both lanes
+    const size_t nwk = std::max((size_t)c->workers + c->heavy_cap, (size_t)c->sworkers);  // both lanes; static
+    c->nscratch = nwk;
     const size_t wn = nwk * n;
     AL(c->ws.mark, wn);
     AL(c->ws.lowrec, wn);
@@ -564,10 +572,10 @@ extern "C" dbc_status dbc_static_compute(dbc_ctx *c) {
         a.next_slot = c->next_slot;
         a.stats = c->stats;
         a.err = c->err;
-        if (c->block == 128)
-            launch_static_128(a, c->workers, c->stream);
+        if (c->sblock == 128)
+            launch_static_128(a, c->sworkers, c->stream);
         else
-            launch_static_256(a, c->workers, c->stream);
+            launch_static_256(a, c->sworkers, c->stream);
         CK(cudaGetLastError());
     }
     if (tm) {

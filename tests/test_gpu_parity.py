@@ -333,9 +333,11 @@ def test_block128_kernels_match_oracle(name, monkeypatch):
         check_all(dbc, ref.compute(), wl.roots.size)
 
 
-def test_heavy_lane_batches_match_oracle():
+def test_heavy_lane_batches_match_oracle(monkeypatch):
     """Several Mode-A batches so the adaptive heavy lane (2x-wide CTAs for the
-    slowest roots of the previous batch) is exercised; d/sigma bit-exact."""
+    slowest roots of the previous batch; 256-thread build) is exercised; d/sigma bit-exact."""
+    monkeypatch.setenv("DBC_BLOCK", "256")
+    monkeypatch.setenv("DBC_WINDOW", "8")  # several jobs per root and batch
     wl = W.make_workload("rmat10", insertions=120)
     ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
     with _dbc(wl.graph, wl.roots) as dbc:
@@ -443,3 +445,19 @@ def test_case2_groups_match_oracle_and_no_merge(name):
             assert (groups == 0) if flags else (groups > 0 or name == "karate")
     for (d0, s0), (d1, s1) in zip(*outs):
         assert np.array_equal(d0, d1) and np.array_equal(s0, s1)
+
+
+@pytest.mark.parametrize("window", ["2", "7", "64"])
+@pytest.mark.parametrize("name", ["rmat10", "delaunay12u"])
+def test_window_sizes_match_oracle(name, window, monkeypatch):
+    """Jobs of `window` insertions (seed injection across several windows per
+    batch, Case 3 inside windows): oracle d/sigma bit-exact, BC within tolerance."""
+    monkeypatch.setenv("DBC_WINDOW", window)
+    wl = W.make_workload(name)
+    ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
+    for u, v in zip(wl.ins_u, wl.ins_v):
+        ref.insert(u, v)
+    with _dbc(wl.graph, wl.roots) as dbc:
+        dbc.static_compute()
+        dbc.insert_edges(wl.ins_u, wl.ins_v)
+        check_all(dbc, ref.compute(), wl.roots.size)
