@@ -58,6 +58,10 @@ def parse():
     p.add_argument("--seed", type=int, default=1)
     p.add_argument("--workers", type=int, default=0)
     p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-merge", action="store_true",
+                   help="headline run with DBC_FLAG_NO_MERGE (one job per (root, insertion))")
+    p.add_argument("--no-per-insertion", action="store_true",
+                   help="skip the side measurement with DBC_FLAG_NO_MERGE")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-budget-s", type=float, default=12.0)
     p.add_argument("--shard", default="", help="R/N: run rank R's root shard of an N-GPU job on this "
@@ -166,6 +170,32 @@ def cpu_baseline(wl, k, budget_s):
                       f"recomputed single-threaded, {t_root * 1e3:.2f} ms/root, scaled linearly to k"}
 
 
+def cpu_dynamic(wl, k, budget_s):
+    """The paper's CPU comparison (dynamic sequential Alg. 2 + Case 3, one
+    thread, oracle/cpu_dynamic.c; Table II "CPU"): a bounded sample of
+    roots and insertions of the same stream, scaled linearly to k roots."""
+    import oracle
+
+    g = wl.graph
+    t0 = time.perf_counter()
+    oracle.brandes(g.n, g.row_ptr, g.col, wl.roots[:1], want_state=False)
+    t_root = max(time.perf_counter() - t0, 1e-6)
+    r = int(max(1, min(k, (budget_s / 3) / t_root)))  # initial state ~ budget/3
+    cd = oracle.CpuDynamicBC(g, wl.roots[:r])
+    t_sum, done = 0.0, 0
+    while done < wl.ins_u.size and (t_sum < budget_s / 2 or done < 3):
+        t0 = time.perf_counter()
+        cd.insert(wl.ins_u[done], wl.ins_v[done])
+        t_sum += time.perf_counter() - t0
+        done += 1
+    cd.close()
+    per_ins = t_sum / done * k / r
+    return {"value": 1.0 / per_ins, "unit": "insertions/s", "cores": 1, "kind": "cpu_dynamic_alg2",
+            "sample": f"dynamic CPU algorithm (Alg. 2 + Case 3, O(n) init per update as in P:254-268), "
+                      f"first {done} insertions of the stream on {r} of {k} roots, single thread, "
+                      f"scaled linearly to k"}
+
+
 # -------------------------------------------------------------- reference ----
 def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
@@ -233,8 +263,8 @@ def run_ours(args):
         torch.cuda.set_device(0)
     dev = torch.cuda.current_device()
 
-    from paper_conf_ipps_mclaughlinb14_b200 import (FLAG_MODE_S, FLAG_TIMING, DynamicBC,
-                                                    allreduce_bc)
+    from paper_conf_ipps_mclaughlinb14_b200 import (FLAG_MODE_S, FLAG_NO_MERGE, FLAG_TIMING,
+                                                    DynamicBC, allreduce_bc)
 
     cfg = W.CONFIGS[args.config]
     B = args.batch or cfg["insertions"]
@@ -244,7 +274,7 @@ def run_ours(args):
     nb = Wm + K + e2e_steps
     wl = W.make_workload(args.config, seed=args.seed, insertions=B * nb, k=k)
     g = wl.graph
-    flags = FLAG_TIMING | (FLAG_MODE_S if args.mode == "S" else 0)
+    flags = FLAG_TIMING | (FLAG_MODE_S if args.mode == "S" else 0) | (FLAG_NO_MERGE if args.no_merge else 0)
     stream = torch.cuda.Stream(device=dev)  # the library and the timing events share it
     torch.cuda.set_stream(stream)
     dbc = DynamicBC(g.n, g.row_ptr, g.col, wl.roots, device=dev, rank=shard_rank, world=shard_world,
@@ -353,6 +383,40 @@ def run_ours(args):
             cpu = {"value": None, "unit": "insertions/s", "cores": 1, "kind": "oracle",
                    "sample": f"unavailable: {ex}"}
 
+    # side measurement: the same batches with one job per (root, insertion)
+    # (DBC_FLAG_NO_MERGE: the paper's one-insertion-at-a-time structure)
+    per_ins = None
+    if not (args.no_per_insertion or args.no_merge or args.mode == "S"):
+        dbc.close()
+        dbc = DynamicBC(g.n, g.row_ptr, g.col, wl.roots, device=dev, rank=shard_rank,
+                        world=shard_world, workers=args.workers, edge_capacity=B * nb,
+                        flags=flags | FLAG_NO_MERGE, stream=stream.cuda_stream)
+        dbc.static_compute()
+        for i in range(Wm):
+            dbc.insert_edges(*batch(i))
+        barrier()
+        torch.cuda.synchronize()
+        ev0.record(stream)
+        for i in range(Wm, Wm + K):
+            dbc.insert_edges(*batch(i))
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        ms1 = max_over_ranks(ev0.elapsed_time(ev1))
+        per_ins = {"value": K * B / (ms1 / 1e3), "unit": "insertions/s", "ms_per_step": ms1 / K,
+                   "speedup_vs_static": (static_ms / 1e3) / (ms1 / 1e3 / (K * B)),
+                   "what": "same batches, DBC_FLAG_NO_MERGE: one job per (root, insertion), "
+                           "insertions applied one at a time as in P:440"}
+
+    cpu_dyn = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        try:
+            cpu_dyn = cpu_dynamic(wl, k, args.cpu_budget_s)
+            cpu_dyn["gpu_speedup"] = value / cpu_dyn["value"]
+            cpu_dyn["paper"] = "110x max GPU-over-CPU dynamic on a GTX-class GPU (P:444-478), context only"
+        except Exception as ex:
+            cpu_dyn = {"value": None, "kind": "cpu_dynamic_alg2", "sample": f"unavailable: {ex}"}
+
     state_mb = 24.0 * k * g.n / shard_world / 1e6
     line = {
         "metric": "edge insertions/sec (device-timed)",
@@ -379,6 +443,9 @@ def run_ours(args):
             "speedup_vs_static": (static_ms / 1e3) / per_ins_s,
             "us_per_insertion": per_ins_s * 1e6,
             "case_mix": case_mix,
+            "merge": ("one job per (root, insertion)" if args.no_merge or args.mode == "S" else
+                      "window-merged: one job per root per window of insertions (DESIGN.md R18)"),
+            "per_insertion_jobs": per_ins,
         },
         "roofline": {
             "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
@@ -389,6 +456,7 @@ def run_ours(args):
             "static_kernel_GBps": (static_bytes / (static_ms / 1e3) / 1e9) if static_ms > 0 else None,
         },
         "cpu_baseline": cpu,
+        "cpu_dynamic": cpu_dyn,
         "e2e": e2e,
         "gpu_launches": int(tm["kernel_launches_total"]),
         "clocks": clk,

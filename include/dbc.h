@@ -81,11 +81,14 @@ typedef enum {
 #define DBC_FLAG_NO_REORDER 0x8u /* keep the caller's vertex numbering internally
                                   (default: BFS-order relabelling for locality;
                                   invisible at the ABI, results identical)        */
-#define DBC_FLAG_NO_MERGE 0x10u /* Mode A: one job per insertion.  Default: a run of
-                                  Case-2 insertions of a root (no distance change,
-                                  P:150-155) between Case-3 ones is repaired as one
-                                  job seeded with every u_low -- the same d/sigma
-                                  (bit-exact) and BC (within rounding)            */
+#define DBC_FLAG_NO_MERGE 0x10u /* Mode A: one job per (root, insertion), the
+                                  paper's one-at-a-time structure.
+                                  Default: each root repairs a window of up to
+                                  16384 insertions of the batch as ONE job seeded
+                                  with every endpoint pair (R18): d and
+                                  sigma after the batch are bit-identical, BC
+                                  within rounding (the sum of the per-insertion
+                                  changes telescopes)                            */
 
 typedef struct {
     int32_t device;        /* CUDA device ordinal (default 0)                      */
@@ -210,6 +213,26 @@ dbc_status dbc_debug_counters(dbc_ctx *c, int64_t *out, int32_t count);
  * (Case 2/3) insertions, touched vertices, adjacency entries scanned, level
  * steps}.  Synchronises when out != NULL. */
 dbc_status dbc_debug_root_profile(dbc_ctx *c, int32_t enable, int64_t *out);
+
+/* Scenario log (Fig. 2 and Fig. 4).  max_insertions > 0
+ * turns it on for later insert calls whose batch has at most that many
+ * insertions (larger batches -> DBC_EINVAL); while it is on, every (root,
+ * insertion) is repaired as its own job (as with DBC_FLAG_NO_MERGE) so that
+ * each scenario has its own record.  0 turns it off.  Allocates
+ * 8 * max_insertions * k_local bytes of device memory. */
+dbc_status dbc_scenario_log(dbc_ctx *c, int64_t max_insertions);
+
+/* Copies the scenario log of the last insert call to host out[count]:
+ * record [i * k_local + j] is insertion i of the batch seen by local root slot
+ * j (local slot j = global slot j * world + rank), encoded as
+ * case | (touched << 2) | (down << 33): case 1, 2 or 3;
+ * touched = number of vertices the update touched (t[v] != untouched, P:512;
+ * the root excluded; ancestors are reached only through non-zero
+ * Delta-delta, so this is a subset of Alg. 2's touched set); down = |D|, the
+ * vertices whose d/sigma were recomputed.  Both 0 for Case 1.
+ * *count receives the number of records; out may be NULL to query it.
+ * capacity < *count -> DBC_EINVAL.  Synchronises. */
+dbc_status dbc_get_scenarios(dbc_ctx *c, int64_t *out, int64_t capacity, int64_t *count);
 
 /* Device memory held by the context, in bytes. */
 dbc_status dbc_device_bytes(const dbc_ctx *c, int64_t *bytes);

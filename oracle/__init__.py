@@ -8,6 +8,9 @@ imports the product.  Inputs come from `workloads/` (no method arithmetic).
 * `brandes(g, roots)` -- static Brandes over a root set (Alg. 1, PAPER.md
   P:69-124, Eqs. (2)-(3) P:52-57), implemented in plain C (oracle/brandes.c,
   fp64, -ffp-contract=off), wrapped with ctypes.
+* `CpuDynamicBC` -- NOT part of the oracle: the paper's dynamic sequential
+  CPU comparison algorithm (Alg. 2, with Case 3), single thread,
+  in oracle/cpu_dynamic.c; pinned against the naive rule, timed by bench.py.
 * `NaiveDynamicBC` -- the naive dynamic rule of the north star: after each edge
   insertion (u, v) ("E' = E u {e}") append v to adj(u) and u to
   adj(v) (canonical order: original row, then inserted neighbours in insertion
@@ -36,12 +39,14 @@ INF = np.iinfo(np.int32).max
 
 
 def build(force: bool = False) -> str:
-    """Compile oracle/brandes.c -> oracle/liboracle.so (gcc, fp64, no FMA contraction)."""
-    src = os.path.join(_HERE, "brandes.c")
-    if force or not os.path.exists(_LIB_PATH) or os.path.getmtime(_LIB_PATH) < os.path.getmtime(src):
+    """Compile oracle/brandes.c (+ the CPU dynamic baseline cpu_dynamic.c) ->
+    oracle/liboracle.so (gcc, fp64, no FMA contraction)."""
+    srcs = [os.path.join(_HERE, f) for f in ("brandes.c", "cpu_dynamic.c")]
+    newest = max(os.path.getmtime(f) for f in srcs)
+    if force or not os.path.exists(_LIB_PATH) or os.path.getmtime(_LIB_PATH) < newest:
         tmp = _LIB_PATH + f".tmp{os.getpid()}"
         subprocess.check_call(["gcc", "-O2", "-ffp-contract=off", "-fno-fast-math", "-std=c99",
-                               "-fPIC", "-shared", "-o", tmp, src])
+                               "-fPIC", "-shared", "-o", tmp] + srcs)
         os.replace(tmp, _LIB_PATH)
     return _LIB_PATH
 
@@ -55,6 +60,18 @@ def _load():
             P = ctypes.c_void_p
             lib.oracle_brandes.argtypes = [ctypes.c_int32, P, P, P, ctypes.c_int32, P, P, P, P]
             lib.oracle_brandes.restype = ctypes.c_int
+            lib.cd_create.argtypes = [ctypes.c_int32, P, P, P, ctypes.c_int32]
+            lib.cd_create.restype = P
+            lib.cd_destroy.argtypes = [P]
+            lib.cd_destroy.restype = None
+            lib.cd_insert.argtypes = [P, ctypes.c_int32, ctypes.c_int32]
+            lib.cd_insert.restype = ctypes.c_int
+            lib.cd_insert_roots.argtypes = [P, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32]
+            lib.cd_insert_roots.restype = ctypes.c_int
+            lib.cd_get.argtypes = [P, P, P, P, P]
+            lib.cd_get.restype = None
+            lib.cd_scenarios.argtypes = [P, P]
+            lib.cd_scenarios.restype = None
             _lib = lib
     return _lib
 
@@ -132,3 +149,111 @@ class NaiveDynamicBC:
     def compute(self, want_state=True):
         rp, col = self.csr()
         return brandes(self.n, rp, col, self.roots, want_state)
+
+
+def scenarios(rp_old, col_old, rp_new, col_new, roots, u, v):
+    """Scenario of each root for the insertion of (u, v) (Fig. 2 / Fig. 4).
+
+    rp_old/col_old: the graph before the insertion; rp_new/col_new: after it.
+    Returns (case[k], touched[k], down[k]) int64:
+      case: 1 if d_s(u) == d_s(v) (both unreachable included),
+        2 if |d_s(u) - d_s(v)| == 1, else 3 (one endpoint unreachable is 3);
+      touched ("{i in V | t[i] != untouched}") for Case 2, following
+        Alg. 2: the down-touched set D = u_low and every vertex
+        reached from it along the NEW shortest-path DAG (t[w] = down, lines
+        9-20), plus every vertex reached from D by predecessor steps (t[v] = up,
+        lines 21-35), the root itself excluded (its delta is never used,
+        P:221-223).  0 for Case 1, -1 for Case 3 (not defined by the paper);
+      down = |D| for Case 2 (the vertices whose sigma changes), 0 / -1 likewise.
+    Pinned in tests/test_oracle.py against an all-pairs characterisation
+    (sigma changed / lies on a shortest path to such a vertex)."""
+    n = rp_old.size - 1
+    _, d0, _, _ = brandes(n, rp_old, col_old, roots)
+    _, d1, _, _ = brandes(n, rp_new, col_new, roots)
+    k = len(roots)
+    case = np.zeros(k, dtype=np.int64)
+    touched = np.zeros(k, dtype=np.int64)
+    down = np.zeros(k, dtype=np.int64)
+    for j in range(k):
+        du, dv = int(d0[j, u]), int(d0[j, v])
+        if du == dv:
+            case[j] = 1
+            continue
+        if min(du, dv) + 1 != max(du, dv):
+            case[j] = 3
+            touched[j] = -1
+            down[j] = -1
+            continue
+        case[j] = 2
+        d = d1[j]
+        ul = v if du < dv else u
+        t = np.zeros(n, dtype=bool)
+        t[ul] = True
+        queue = [ul]
+        qi = 0
+        while qi < len(queue):  # down: successors in the new DAG
+            w = queue[qi]
+            qi += 1
+            for y in col_new[rp_new[w]:rp_new[w + 1]]:
+                if d[y] == d[w] + 1 and not t[y]:
+                    t[y] = True
+                    queue.append(int(y))
+        down[j] = len(queue)
+        qi = 0
+        while qi < len(queue):  # up: predecessors of touched vertices
+            x = queue[qi]
+            qi += 1
+            for p in col_new[rp_new[x]:rp_new[x + 1]]:
+                if d[p] == d[x] - 1 and not t[p]:
+                    t[p] = True
+                    queue.append(int(p))
+        t[roots[j]] = False
+        touched[j] = int(t.sum())
+    return case, touched, down
+
+
+class CpuDynamicBC:
+    """The dynamic sequential CPU baseline (oracle/cpu_dynamic.c): Alg. 2 of
+    the paper (Green et al.) with Case 3, one thread.  A comparison
+    program for bench.py (`cpu_dynamic`), pinned against NaiveDynamicBC."""
+
+    def __init__(self, g, roots):
+        lib = _load()
+        self.n = g.n
+        self.k = len(roots)
+        rp = np.ascontiguousarray(g.row_ptr, dtype=np.int64)
+        col = np.ascontiguousarray(g.col, dtype=np.int32)
+        self.roots = np.ascontiguousarray(roots, dtype=np.int32)
+        self._h = lib.cd_create(g.n, _ptr(rp), _ptr(col), _ptr(self.roots), self.k)
+        if not self._h:
+            raise MemoryError("cd_create failed")
+        self._lib = lib
+
+    def insert(self, u: int, v: int, roots: tuple | None = None):
+        if roots is None:
+            rc = self._lib.cd_insert(self._h, int(u), int(v))
+        else:
+            rc = self._lib.cd_insert_roots(self._h, int(u), int(v), int(roots[0]), int(roots[1]))
+        if rc != 0:
+            raise MemoryError("cd_insert failed")
+
+    def state(self):
+        bc = np.empty(self.n, np.float64)
+        d = np.empty((self.k, self.n), np.int32)
+        sig = np.empty((self.k, self.n), np.float64)
+        dl = np.empty((self.k, self.n), np.float64)
+        self._lib.cd_get(self._h, _ptr(bc), _ptr(d), _ptr(sig), _ptr(dl))
+        return bc, d, sig, dl
+
+    def scenarios(self):
+        out = np.zeros(3, np.int64)
+        self._lib.cd_scenarios(self._h, _ptr(out))
+        return out
+
+    def close(self):
+        if getattr(self, "_h", None):
+            self._lib.cd_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        self.close()

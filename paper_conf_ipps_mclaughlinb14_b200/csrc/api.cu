@@ -70,6 +70,9 @@ struct dbc_ctx {
     int32_t *err = nullptr;
     unsigned long long *root_prof = nullptr;  // [k_loc][4], filled when profiling is on
     bool prof_on = false;
+    long long *scen = nullptr;  // scenario log [insertion][k_loc] of the last insert call
+    int64_t scen_cap = 0;       // insertions it holds (0: logging off)
+    int64_t scen_last = 0;      // insertions logged by the last insert call
 
     std::vector<void *> allocs;
     int64_t bytes = 0;
@@ -400,7 +403,9 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     c->sblock = (c->k_loc > 2 * c->nsm && maxdeg <= 256) ? 128 : 256;  // hubs need the wide CTA
     c->block = 512;
     if (const char *eb = getenv("DBC_BLOCK")) c->block = atoi(eb) == 128 ? 128 : (atoi(eb) == 256 ? 256 : 512);
-    int want = opt.workers ? opt.workers : (c->block == 128 ? 4 : (c->block == 512 ? 1 : 2)) * c->nsm;
+    int upb = c->block == 128 ? 4 : (c->block == 512 ? 1 : 2);  // update CTAs per SM
+    if (const char *e = getenv("DBC_UPB")) upb = std::max(1, atoi(e));
+    int want = opt.workers ? opt.workers : upb * c->nsm;
     want = std::min(want, c->k_loc);
     int fit = (int)std::min<size_t>(budget / per_worker, 1 << 20);
     c->workers = std::max(0, std::min(want, fit));
@@ -670,6 +675,15 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     a.worker_base = 0;
     a.help = HelpBoard{};  // Mode S: no cooperative help
     a.merge = (c->flags & DBC_FLAG_NO_MERGE) ? 0 : 1;
+    a.scen = nullptr;
+    if (c->scen_cap > 0) {  // Fig. 2 / Fig. 4 log: one job per (root, insertion)
+        if (cnt > c->scen_cap)
+            return fail(c, DBC_EINVAL, "batch of %lld exceeds the scenario log (%lld insertions)",
+                        (long long)cnt, (long long)c->scen_cap);
+        a.scen = c->scen;
+        a.merge = 0;
+        c->scen_last = cnt;
+    }
     if (tm) CK(cudaEventRecord(ev[2], c->stream));
     int ulaunch = 0;
     if (c->workers) {
@@ -911,6 +925,40 @@ extern "C" dbc_status dbc_debug_root_profile(dbc_ctx *c, int32_t enable, int64_t
     if (out) {
         CK(cudaMemcpyAsync(out, c->root_prof, sizeof(int64_t) * 6 * c->k_loc, cudaMemcpyDeviceToHost,
                            c->stream));
+        CK(cudaStreamSynchronize(c->stream));
+    }
+    return DBC_OK;
+}
+
+extern "C" dbc_status dbc_scenario_log(dbc_ctx *c, int64_t max_insertions) {
+    if (!c || max_insertions < 0) return DBC_EINVAL;
+    CK(cudaSetDevice(c->device));
+    if (max_insertions > c->scen_cap) {
+        CK(cudaStreamSynchronize(c->stream));
+        if (c->scen) {
+            for (auto &q : c->allocs)
+                if (q == (void *)c->scen) q = nullptr;
+            CK(cudaFree(c->scen));
+            c->bytes -= (int64_t)(sizeof(long long) * (size_t)c->scen_cap * std::max(c->k_loc, 1));
+            c->scen = nullptr;
+        }
+        TRY(dalloc(c, &c->scen, (size_t)max_insertions * std::max(c->k_loc, 1)));
+    }
+    c->scen_cap = max_insertions;
+    c->scen_last = 0;
+    return DBC_OK;
+}
+
+extern "C" dbc_status dbc_get_scenarios(dbc_ctx *c, int64_t *out, int64_t capacity, int64_t *count) {
+    if (!c || !count) return DBC_EINVAL;
+    CK(cudaSetDevice(c->device));
+    const int64_t need = c->scen_last * c->k_loc;
+    *count = need;
+    if (!out) return DBC_OK;
+    if (capacity < need) return fail(c, DBC_EINVAL, "scenario buffer holds %lld, need %lld",
+                                     (long long)capacity, (long long)need);
+    if (need > 0) {
+        CK(cudaMemcpyAsync(out, c->scen, sizeof(int64_t) * need, cudaMemcpyDeviceToHost, c->stream));
         CK(cudaStreamSynchronize(c->stream));
     }
     return DBC_OK;

@@ -29,7 +29,17 @@ namespace dbc {
 #ifndef DBC_BLOCK
 #define DBC_BLOCK 256
 #endif
+// resident CTAs per SM the register budget is sized for (__launch_bounds__)
+#if DBC_BLOCK == 512 && defined(DBC_MINB512)
+#define DBC_MINB DBC_MINB512
+#elif DBC_BLOCK == 256 && defined(DBC_MINB256)
+#define DBC_MINB DBC_MINB256
+#endif
+#ifndef DBC_MINB
+#define DBC_MINB ((512 / DBC_BLOCK) > 0 ? (512 / DBC_BLOCK) : 1)
+#endif
 constexpr int kBlock = DBC_BLOCK;
+constexpr int kMinBlocks = DBC_MINB;
 constexpr int kWarps = kBlock / 32;
 constexpr int kSmallDeg = 32;            // rows <= this are walked by one lane
 constexpr uint32_t kFull = 0xffffffffu;
@@ -333,7 +343,7 @@ __device__ __forceinline__ void big_entries(BigSmem &S, const GView &g, const Ro
 }
 
 // --- up phase: chunked flattened level pass ----------------------------------
-constexpr int kChunk = 512;   // items per chunk (shared memory)
+constexpr int kChunk = kBlock > 512 ? kBlock : 512;  // items per chunk (shared memory)
 constexpr int kUcap = 1024;   // up-frontier entries kept in shared memory
 constexpr int kMetaUp = 1, kMetaNotPulled = 2, kMetaMask = 4;
 constexpr int kMetaNew = 8;  // down row with batch entries: its pushes check new_edge()
@@ -526,6 +536,7 @@ struct UpdateArgs {
     int32_t worker_base;           // scratch index of CTA 0
     HelpBoard help;                // help.word == nullptr: no cooperative help
     int32_t merge;                 // 1: a window of ws.wcap insertions per job; 0: one per insertion
+    long long *scen;               // nullable: scenario log [batch insertion][k_loc] (merge == 0)
 };
 
 struct StaticArgs {

@@ -17,7 +17,7 @@
 namespace dbc {
 
 namespace {
-__global__ void __launch_bounds__(kBlock, 512 / kBlock) static_kernel(StaticArgs a) {
+__global__ void __launch_bounds__(kBlock, kMinBlocks) static_kernel(StaticArgs a) {
     __shared__ int s_slot;
     __shared__ int s_tail;
     __shared__ int s_nbig;

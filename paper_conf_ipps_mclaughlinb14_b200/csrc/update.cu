@@ -93,7 +93,7 @@ __device__ __forceinline__ void help_run_block(const ChunkSmem &M, int e0, int e
         e0);
 }
 
-__global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs a) {
+__global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a) {
     __shared__ int s_slot;
     __shared__ int s_dcnt;     // |D| (absolute positions in Dv)
     __shared__ int s_ucnt2[2]; // up frontier sizes (list ucur_sel is read, ucur_sel^1 filled)
@@ -245,6 +245,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                     }
                 }
                 if (nw == 0) {  // Case 1 throughout: nothing changes
+                    if (a.scen && tid == 0) a.scen[(size_t)ins * a.k_loc + slot] = 1;
                     ins = wend;
                     __syncthreads();  // the counters are reset by the next window
                     continue;
@@ -253,6 +254,7 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
             {
                 ++epoch;
                 ++prof_jobs;
+                const unsigned long long touch0 = st_touched;  // scenario log (thread 0's counter)
                 const uint32_t E = epoch << 2;
                 const uint32_t mD = E | kDown, mU = E | kUp;
                 const int g0 = ins, lim = wend - 1;  // the job's insertions; graph as of lim
@@ -968,6 +970,10 @@ __global__ void __launch_bounds__(kBlock, 512 / kBlock) update_kernel(UpdateArgs
                     tick(5);
                 }
                 // any up vertices left at level 0 would be the root: never produced
+                if (a.scen && tid == 0)  // Fig. 2 / Fig. 4 record: case | touched << 2 | |D| << 33
+                    a.scen[(size_t)ins * a.k_loc + slot] = (long long)(((unsigned long long)dtotal << 33) |
+                                                                       ((st_touched - touch0) << 2) |
+                                                                       (s_wcnt[1] ? 3u : 2u));
             }
             ins = wend;
             __syncthreads();  // the counters are reset by the next window

@@ -93,6 +93,8 @@ SIGNATURES = {
     "dbc_debug_counters": (ctypes.c_int, [_P, _P, ctypes.c_int32]),
     "dbc_debug_root_profile": (ctypes.c_int, [_P, ctypes.c_int32, _P]),
     "dbc_device_bytes": (ctypes.c_int, [_P, _P]),
+    "dbc_scenario_log": (ctypes.c_int, [_P, ctypes.c_int64]),
+    "dbc_get_scenarios": (ctypes.c_int, [_P, _P, ctypes.c_int64, _P]),
     "dbc_strerror": (ctypes.c_char_p, [ctypes.c_int]),
     "dbc_last_error": (ctypes.c_char_p, [_P]),
     "dbc_abi_version": (ctypes.c_int32, []),
@@ -270,6 +272,22 @@ class DynamicBC:
         _check(self._ctx, self._lib.dbc_debug_root_profile(
             self._ctx, int(enable), _np_ptr(out) if read else None))
         return out
+
+    def scenario_log(self, max_insertions: int):
+        """Record case and touched count of every (root, insertion) of later
+        insert calls (Fig. 2 / Fig. 4); 0 turns it off."""
+        _check(self._ctx, self._lib.dbc_scenario_log(self._ctx, int(max_insertions)))
+
+    def scenarios(self):
+        """Scenario log of the last insert call: (case, touched, down) int64
+        arrays of shape [insertions, k_local] (case 1/2/3; touched excludes the
+        root; down = |D|, the vertices whose sigma was recomputed)."""
+        cnt = ctypes.c_int64()
+        _check(self._ctx, self._lib.dbc_get_scenarios(self._ctx, None, 0, ctypes.byref(cnt)))
+        out = np.zeros(cnt.value, dtype=np.int64)
+        _check(self._ctx, self._lib.dbc_get_scenarios(self._ctx, _np_ptr(out), out.size, ctypes.byref(cnt)))
+        rec = out.reshape(-1, max(self.num_local_roots(), 1))
+        return rec & 3, (rec >> 2) & 0x7FFFFFFF, rec >> 33
 
     def device_bytes(self):
         b = ctypes.c_int64()

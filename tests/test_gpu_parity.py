@@ -461,3 +461,42 @@ def test_window_sizes_match_oracle(name, window, monkeypatch):
         dbc.static_compute()
         dbc.insert_edges(wl.ins_u, wl.ins_v)
         check_all(dbc, ref.compute(), wl.roots.size)
+
+
+# ------------------------------------------------ scenario log (Fig. 2/4) ----
+@pytest.mark.parametrize("name", ["karate", "rmat10", "delaunay12", "delaunay12u"])
+def test_scenario_log_matches_oracle(name):
+    """dbc_get_scenarios: case of every (root, insertion) bit-exact against the
+    oracle's classification of P:148-159; for every Case-2 scenario the down
+    set |D| (sigma changed) exact, and the touched count between |D| and
+    Alg. 2's t[v] != untouched set: the kernel does not propagate
+    from an ancestor whose Delta-delta is exactly 0 (R19), Alg. 2
+    marks every ancestor."""
+    wl = W.make_workload(name)
+    g, roots = wl.graph, wl.roots
+    B = min(40, wl.ins_u.size)
+    u, v = wl.ins_u[:B], wl.ins_v[:B]
+    ref = oracle.NaiveDynamicBC(g, roots)
+    with _dbc(g, roots) as dbc:
+        dbc.static_compute()
+        dbc.scenario_log(B)
+        dbc.insert_edges(u, v)
+        case, touched, down = dbc.scenarios()
+        assert case.shape == (B, roots.size)
+        n2 = exact = 0
+        for i in range(B):
+            rp0, col0 = ref.csr()
+            ref.insert(u[i], v[i])
+            rp1, col1 = ref.csr()
+            oc, ot, od = oracle.scenarios(rp0, col0, rp1, col1, roots, int(u[i]), int(v[i]))
+            assert np.array_equal(case[i], oc), f"case mismatch at insertion {i}"
+            c2 = oc == 2
+            n2 += int(c2.sum())
+            assert np.array_equal(down[i][c2], od[c2]), f"|D| mismatch at insertion {i}"
+            assert np.all(touched[i][c2] <= ot[c2]) and np.all(touched[i][c2] >= od[c2])
+            exact += int((touched[i][c2] == ot[c2]).sum())
+            assert np.all(touched[i][oc == 1] == 0) and np.all(down[i][oc == 1] == 0)
+        assert n2 > 0
+        assert exact >= 0.5 * n2  # most Case-2 scenarios touch exactly Alg. 2's set
+        # the batch itself still matches the naive rule
+        check_all(dbc, ref.compute(), roots.size)

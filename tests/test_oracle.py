@@ -267,3 +267,144 @@ def test_paper_table_arithmetic():
         ratios.append(row["recompute"] / row["average"])
         assert row["recompute"] / row["average"] == pytest.approx(row["avg_speedup"], rel=1e-2)  # times printed to 2-3 digits
     assert np.mean(ratios) == pytest.approx(45.0, abs=0.5)
+
+
+# --------------------------------------------------------------------------
+# scenario classification and touched sets (Fig. 2 / Fig. 4 diagnostics)
+# --------------------------------------------------------------------------
+def _with_edge(g, u, v):
+    dyn = oracle.NaiveDynamicBC(g, np.zeros(1, np.int32))
+    dyn.insert(u, v)
+    return dyn.csr()
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_scenarios_match_all_pairs_characterisation(seed):
+    """Case from brute-force distances; Case-2 touched set = every v != s on a
+    shortest s-t path (new graph) to some t whose path count changed
+    (sigma changes exactly below u_low)."""
+    rng = np.random.default_rng(100 + seed)
+    n = int(rng.integers(5, 9))
+    m = int(rng.integers(n - 1, min(n * (n - 1) // 2 - 1, 2 * n) + 1))
+    g = W.random_gnm(n, m, 100 + seed)
+    eu, ev = W.edges_of(g)
+    old = list(zip(eu.tolist(), ev.tolist()))
+    present = set(old)
+    cand = [(a, b) for a in range(n) for b in range(a + 1, n) if (a, b) not in present]
+    roots = np.arange(n, dtype=np.int32)
+    bd0, bs0, _, _ = brute_force(n, old, list(range(n)))
+    seen2 = 0
+    for ci in rng.permutation(len(cand))[:8]:
+        u, v = cand[int(ci)]
+        rp1, col1 = _with_edge(g, u, v)
+        case, touched, down = oracle.scenarios(g.row_ptr, g.col, rp1, col1, roots, u, v)
+        bd1, bs1, _, _ = brute_force(n, old + [(u, v)], list(range(n)))
+        for s in range(n):
+            du, dv = bd0[s][u], bd0[s][v]
+            want = 1 if du == dv else (2 if abs(du - dv) == 1 else 3)
+            assert case[s] == want
+            if want != 2:
+                continue
+            seen2 += 1
+            changed = [t for t in range(n) if bs1[s][t] != bs0[s][t]]
+            assert down[s] == len(changed)
+            on_path = {x for x in range(n) if x != s and any(
+                bd1[s][x] + bd1[x][t] == bd1[s][t] for t in changed)}
+            assert touched[s] == len(on_path)
+    assert seen2 > 0  # the Case-2 branch is exercised
+
+
+def test_scenarios_path_graph_closed_form():
+    """P_n plus (0, n-1): root r sees d(0) = r, d(n-1) = n-1-r, so Case 1 iff
+    2r = n-1, Case 2 iff |n-1-2r| = 1, else Case 3."""
+    n = 7
+    g = W.path_graph(n)
+    rp1, col1 = _with_edge(g, 0, n - 1)
+    roots = np.arange(n, dtype=np.int32)
+    case, touched, _ = oracle.scenarios(g.row_ptr, g.col, rp1, col1, roots, 0, n - 1)
+    for r in range(n):
+        diff = abs((n - 1 - r) - r)
+        assert case[r] == (1 if diff == 0 else 2 if diff == 1 else 3)
+    # n = 7: r = 3 is Case 1; no r has |6 - 2r| = 1 (even) -> no Case 2
+    assert case.tolist() == [3, 3, 3, 1, 3, 3, 3]
+    n = 6  # C_6 after the insertion; r = 2: d(0) = 2, d(5) = 3 -> Case 2, u_low = 5
+    g = W.path_graph(n)
+    rp1, col1 = _with_edge(g, 0, n - 1)
+    case, touched, down = oracle.scenarios(g.row_ptr, g.col, rp1, col1, np.arange(n, dtype=np.int32), 0, n - 1)
+    assert case.tolist() == [3, 3, 2, 2, 3, 3]
+    # root 2 on C_6: sigma changes only at 5 (paths 2-1-0-5 and 2-3-4-5);
+    # on shortest paths to 5: 1, 0, 3, 4, 5 -> touched 5
+    assert touched[2] == 5 and touched[3] == 5
+    assert down[2] == 1 and down[3] == 1
+
+
+# --------------------------------------------------------------------------
+# the CPU dynamic baseline (Alg. 2 + Case 3, oracle/cpu_dynamic.c) vs the
+# naive rule: d / sigma bit-exact, delta and BC within the GPU's tolerance
+# --------------------------------------------------------------------------
+def _check_cpu_dynamic(g, roots, us, vs, every=1):
+    cd = oracle.CpuDynamicBC(g, roots)
+    ref = oracle.NaiveDynamicBC(g, roots)
+    for i, (u, v) in enumerate(zip(us, vs)):
+        cd.insert(u, v)
+        ref.insert(u, v)
+        if (i + 1) % every and i + 1 != len(us):
+            continue
+        bc, d, s, dl = cd.state()
+        rbc, rd, rs, rdl = ref.compute()
+        assert np.array_equal(d, rd)
+        assert np.array_equal(s, rs)
+        assert np.all(np.abs(dl - rdl) <= 1e-10 * np.maximum(np.abs(rdl), 1.0))
+        assert np.all(np.abs(bc - rbc) <= 1e-9 * np.maximum(np.abs(rbc), 1.0))
+    return cd.scenarios()
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_cpu_dynamic_random_multicomponent(seed):
+    rng = np.random.default_rng(300 + seed)
+    n = int(rng.integers(20, 60))
+    g = W.random_gnm(n, int(n * 0.9), 300 + seed)  # several components: Case 3 from INF
+    eu, ev = W.edges_of(g)
+    present = set(zip(eu.tolist(), ev.tolist()))
+    us, vs = [], []
+    while len(us) < 25:
+        a, b = sorted(int(x) for x in rng.choice(n, 2, replace=False))
+        if (a, b) not in present:
+            present.add((a, b))
+            us.append(a)
+            vs.append(b)
+    sc = _check_cpu_dynamic(g, np.arange(n, dtype=np.int32), us, vs)
+    assert sc[1] > 0 and sc[2] > 0  # Case 2 and Case 3 both exercised
+
+
+@pytest.mark.parametrize("name", ["karate", "rmat10", "delaunay12u"])
+def test_cpu_dynamic_configs(name):
+    wl = W.make_workload(name)
+    B = min(30, wl.ins_u.size)
+    _check_cpu_dynamic(wl.graph, wl.roots, wl.ins_u[:B], wl.ins_v[:B], every=5)
+
+
+def test_cpu_dynamic_path_to_cycle():
+    n = 9
+    g = W.path_graph(n)
+    cd = oracle.CpuDynamicBC(g, np.arange(n, dtype=np.int32))
+    cd.insert(0, n - 1)
+    bc, *_ = cd.state()
+    ref, *_ = oracle.brandes_csr(W.cycle_graph(n), np.arange(n, dtype=np.int32))
+    assert np.all(np.abs(bc - ref) <= 1e-12 * np.maximum(ref, 1))
+
+
+def test_cpu_dynamic_grid_sigma_above_2_53():
+    """sigma up to 2^84 on a 45x45 grid: the pull form stays bit-exact."""
+    g = W.grid_graph(45, 45)
+    rng = np.random.default_rng(7)
+    eu, ev = W.edges_of(g)
+    present = set(zip(eu.tolist(), ev.tolist()))
+    us, vs = [], []
+    while len(us) < 6:
+        a, b = sorted(int(x) for x in rng.choice(g.n, 2, replace=False))
+        if (a, b) not in present:
+            present.add((a, b))
+            us.append(a)
+            vs.append(b)
+    _check_cpu_dynamic(g, np.array([0, 44, 1012, 2024], np.int32), us, vs)
