@@ -90,6 +90,13 @@ typedef enum {
                                   within rounding (the sum of the per-insertion
                                   changes telescopes)                            */
 
+#define DBC_FLAG_EDGE_PARALLEL 0x20u /* edge-based parallel update (Alg. 4 / Alg. 6,
+                                  P:278-356): one launch per insertion, every
+                                  level a pass of one CTA per root over all
+                                  edges -- the comparison kernel of Table II
+                                  (P:458-478).  Same results as the default
+                                  node-based kernel; slower by design        */
+
 typedef struct {
     int32_t device;        /* CUDA device ordinal (default 0)                      */
     int32_t rank;          /* this process's rank in [0, world) (default 0)        */

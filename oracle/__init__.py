@@ -14,7 +14,9 @@ imports the product.  Inputs come from `workloads/` (no method arithmetic).
 * `NaiveDynamicBC` -- the naive dynamic rule of the north star: after each edge
   insertion (u, v) ("E' = E u {e}") append v to adj(u) and u to
   adj(v) (canonical order: original row, then inserted neighbours in insertion
-  order) and recompute everything from scratch.
+  order) and recompute everything from scratch; after a deletion (the
+  decremental counterpart) remove the two entries, the rows keeping the order
+  of their remaining entries, and recompute.
 
 Pins (tests/test_oracle.py): brute-force path enumeration on n <= 9, closed
 forms (path, star, cycle, complete graph, grid binomials), networkx on karate
@@ -115,11 +117,31 @@ class NaiveDynamicBC:
         self.ins = []  # (u, v) in insertion order
 
     def insert(self, u: int, v: int):
+        if getattr(self, "adj", None) is not None:
+            self.adj[int(u)].append(int(v))
+            self.adj[int(v)].append(int(u))
+            return
         self.ins.append((int(u), int(v)))
 
+    def delete(self, u: int, v: int):
+        """Edge deletion (decremental update): E' = E minus
+        {(u, v)}; each row keeps the order of its remaining entries."""
+        if getattr(self, "adj", None) is None:  # switch to explicit neighbour lists
+            rp, col = self.csr()
+            self.adj = [col[rp[x]:rp[x + 1]].tolist() for x in range(self.n)]
+        self.adj[int(u)].remove(int(v))
+        self.adj[int(v)].remove(int(u))
+
     def csr(self):
-        """Canonical adjacency: base row, then inserted neighbours in insertion order."""
+        """Canonical adjacency: base row, then inserted neighbours in insertion order
+        (after a deletion: explicit per-vertex lists, removal keeps the order)."""
         n = self.n
+        if getattr(self, "adj", None) is not None:
+            deg = np.array([len(a) for a in self.adj], dtype=np.int64)
+            rp = np.zeros(n + 1, dtype=np.int64)
+            rp[1:] = np.cumsum(deg)
+            col = np.fromiter((y for a in self.adj for y in a), dtype=np.int32, count=int(rp[-1]))
+            return rp, col
         if not self.ins:
             return self.base_rp.copy(), self.base_col.copy()
         e = np.array(self.ins, dtype=np.int64)

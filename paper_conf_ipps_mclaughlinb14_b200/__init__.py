@@ -6,6 +6,7 @@ include/dbc.h); this package is the thin Python binding.  See DESIGN.md.
 
 from .dbc import (  # noqa: F401
     DBC_INF,
+    FLAG_EDGE_PARALLEL,
     FLAG_EXACT_BC,
     FLAG_MODE_S,
     FLAG_NO_MERGE,
@@ -21,5 +22,6 @@ from .dbc import (  # noqa: F401
 
 __all__ = [
     "DynamicBC", "DBCError", "DBC_INF", "FLAG_MODE_S", "FLAG_TIMING", "FLAG_EXACT_BC", "FLAG_NO_REORDER", "FLAG_NO_MERGE",
+    "FLAG_EDGE_PARALLEL",
     "LIB_PATH", "load_library", "local_slots", "allreduce_bc",
 ]

@@ -32,6 +32,7 @@ struct dbc_ctx {
     bool own_stream = false;
     int workers = 0;
     int block = 512;   // threads per update worker CTA (512, 256 or 128)
+    bool ub2 = false;  // 512-thread CTAs built for two per SM (update_512x2)
     int sblock = 256, sworkers = 0;  // static kernel: its own CTA width and grid
     size_t nscratch = 0;             // worker scratch sets allocated
     // heavy lanes: the slowest root chains of the previous batch run on
@@ -70,6 +71,9 @@ struct dbc_ctx {
     int32_t *err = nullptr;
     unsigned long long *root_prof = nullptr;  // [k_loc][4], filled when profiling is on
     bool prof_on = false;
+    int32_t *esrc = nullptr, *etag = nullptr;  // edge-parallel mode: entry source / insertion index
+    double *eodel = nullptr;                   // edge-parallel mode: old delta per worker and vertex
+    int eworkers = 0;
     long long *scen = nullptr;  // scenario log [insertion][k_loc] of the last insert call
     int64_t scen_cap = 0;       // insertions it holds (0: logging off)
     int64_t scen_last = 0;      // insertions logged by the last insert call
@@ -403,8 +407,12 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     c->sblock = (c->k_loc > 2 * c->nsm && maxdeg <= 256) ? 128 : 256;  // hubs need the wide CTA
     c->block = 512;
     if (const char *eb = getenv("DBC_BLOCK")) c->block = atoi(eb) == 128 ? 128 : (atoi(eb) == 256 ? 256 : 512);
-    int upb = c->block == 128 ? 4 : (c->block == 512 ? 1 : 2);  // update CTAs per SM
-    if (const char *e = getenv("DBC_UPB")) upb = std::max(1, atoi(e));
+    // Many roots per SM (>= 3 x #SMs): two register-capped 512-thread CTAs per
+    // SM keep more root chains in flight (Delaunay 2^18 / 512 roots: +29%,
+    // Kronecker 20 / 1024 roots: +3%); fewer roots: one 128-register CTA.
+    c->ub2 = c->block == 512 && c->k_loc >= 3 * c->nsm;
+    if (const char *e = getenv("DBC_UB2")) c->ub2 = c->block == 512 && atoi(e) != 0;
+    int upb = c->block == 128 ? 4 : (c->block == 512 ? (c->ub2 ? 2 : 1) : 2);  // update CTAs per SM
     int want = opt.workers ? opt.workers : upb * c->nsm;
     want = std::min(want, c->k_loc);
     int fit = (int)std::min<size_t>(budget / per_worker, 1 << 20);
@@ -484,6 +492,12 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->stats, (size_t)kStCount);
     AL(c->err, 1);
     AL(c->root_prof, (size_t)6 * std::max(c->k_loc, 1));
+    if (c->flags & DBC_FLAG_EDGE_PARALLEL) {  // Table II comparison kernel: one 512-thread CTA per SM
+        c->eworkers = std::max(0, std::min<int>({c->nsm, c->k_loc, (int)nwk}));
+        AL(c->esrc, (size_t)c->col_cap);
+        AL(c->etag, (size_t)c->col_cap);
+        AL(c->eodel, (size_t)std::max(c->eworkers, 1) * n);
+    }
 #undef AL
 
     // upload CSR (int32 offsets), roots; zero scratch
@@ -686,7 +700,34 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     }
     if (tm) CK(cudaEventRecord(ev[2], c->stream));
     int ulaunch = 0;
-    if (c->workers) {
+    if (c->eworkers) {  // edge-based parallel update (Alg. 4 / Alg. 6), one launch per insertion
+        launches += launch_edge_coo(a.g, c->n, c->esrc, c->etag, c->stream);
+        EdgeArgs e;
+        e.g = a.g;
+        e.n = c->n;
+        e.k_loc = c->k_loc;
+        e.roots = c->roots_d;
+        e.d = c->d;
+        e.sd = c->sd;
+        e.bc = c->bc;
+        e.ins_u = u;
+        e.ins_v = v;
+        e.ws = a.ws;
+        e.odel = c->eodel;
+        e.src = c->esrc;
+        e.tag = c->etag;
+        e.nnz = (int32_t)c->nnz;
+        e.stats = c->stats;
+        e.err = c->err;
+        e.next_slot = c->next_slot;
+        for (int64_t i = 0; i < cnt; ++i) {
+            CK(cudaMemsetAsync(c->next_slot, 0, sizeof(int32_t), c->stream));
+            e.ins = (int32_t)i;
+            launch_edge_update(e, c->eworkers, c->stream);
+            ++ulaunch;
+        }
+        CK(cudaGetLastError());
+    } else if (c->workers) {
         if (!(c->flags & DBC_FLAG_MODE_S)) {
             // Mode A with heavy lanes: order slots by last chain time (longest
             // first), the slowest ones go to the wide CTAs
@@ -741,7 +782,7 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
             if (c->block == 128)
                 launch_update_128(a, wl, c->stream);
             else if (c->block == 512)
-                launch_update_512(a, wl, c->stream);
+                (c->ub2 ? launch_update_512x2 : launch_update_512)(a, wl, c->stream);
             else
                 launch_update_256(a, wl, c->stream);
             ++ulaunch;
@@ -756,7 +797,7 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
                 if (c->block == 128)
                     launch_update_128(a, c->workers, c->stream);
                 else if (c->block == 512)
-                    launch_update_512(a, c->workers, c->stream);
+                    (c->ub2 ? launch_update_512x2 : launch_update_512)(a, c->workers, c->stream);
                 else
                     launch_update_256(a, c->workers, c->stream);
                 ++ulaunch;

@@ -555,7 +555,30 @@ struct StaticArgs {
     int32_t *mask_ds;
 };
 
+// Edge-based parallel update (edge_parallel.cu, DBC_FLAG_EDGE_PARALLEL).
+struct EdgeArgs {
+    GView g;
+    int32_t n;
+    int32_t k_loc;
+    const int32_t *roots;
+    int32_t *d;
+    double2 *sd;
+    double *bc;
+    const int32_t *ins_u, *ins_v;
+    int32_t ins;                // the insertion of this launch (batch-local)
+    Scratch ws;
+    double *odel;               // [workers][n] old delta by vertex
+    const int32_t *src, *tag;   // [nnz] entry source / insertion index (-1: base)
+    int32_t nnz;
+    int32_t *next_slot;
+    unsigned long long *stats;
+    int32_t *err;
+};
+int launch_edge_coo(const GView &g, int32_t n, int32_t *src, int32_t *tag, cudaStream_t s);
+void launch_edge_update(const EdgeArgs &a, int workers, cudaStream_t s);
+
 void launch_update_256(const UpdateArgs &a, int workers, cudaStream_t s);
+void launch_update_512x2(const UpdateArgs &a, int workers, cudaStream_t s);  // 64 regs, 2 CTAs/SM
 void launch_update_128(const UpdateArgs &a, int workers, cudaStream_t s);
 void launch_update_512(const UpdateArgs &a, int workers, cudaStream_t s);
 void launch_static_256(const StaticArgs &a, int workers, cudaStream_t s);

@@ -1103,7 +1103,10 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
 
 #define DBC_CAT2(a, b) a##b
 #define DBC_CAT(a, b) DBC_CAT2(a, b)
-void DBC_CAT(launch_update_, DBC_BLOCK)(const UpdateArgs &a, int workers, cudaStream_t s) {
+#ifndef DBC_LAUNCH_SUFFIX
+#define DBC_LAUNCH_SUFFIX DBC_BLOCK
+#endif
+void DBC_CAT(launch_update_, DBC_LAUNCH_SUFFIX)(const UpdateArgs &a, int workers, cudaStream_t s) {
     update_kernel<<<workers, kBlock, 0, s>>>(a);
 }
 

@@ -23,6 +23,7 @@ FLAG_TIMING = 0x2
 FLAG_EXACT_BC = 0x4
 FLAG_NO_REORDER = 0x8
 FLAG_NO_MERGE = 0x10
+FLAG_EDGE_PARALLEL = 0x20
 
 STATUS = {
     0: "DBC_OK", -1: "DBC_EINVAL", -2: "DBC_ENOMEM", -3: "DBC_ECUDA", -4: "DBC_ENCCL",

@@ -500,3 +500,69 @@ def test_scenario_log_matches_oracle(name):
         assert exact >= 0.5 * n2  # most Case-2 scenarios touch exactly Alg. 2's set
         # the batch itself still matches the naive rule
         check_all(dbc, ref.compute(), roots.size)
+
+
+# ------------------------------------------- edge-parallel variant (Table II) ----
+EDGE = 0x20  # DBC_FLAG_EDGE_PARALLEL
+
+
+@pytest.mark.parametrize("name", ["karate", "rmat10", "delaunay12", "delaunay12u", "smallworld_small"])
+def test_edge_parallel_matches_oracle(name):
+    """Alg. 4 / Alg. 6 edge-based kernel: same d/sigma (bit-exact) and BC as the
+    oracle, batch by batch."""
+    if name == "smallworld_small":
+        g = W.watts_strogatz(2000, 6, 0.1, seed=4)
+        roots = np.arange(0, 2000, 37, dtype=np.int32)
+        eu, ev = W.edges_of(g)
+        rng = np.random.default_rng(9)
+        pick = rng.choice(eu.size, 40, replace=False)
+        # reinsert: drop the picked edges from the graph first (P:440)
+        keep = np.ones(eu.size, bool)
+        keep[pick] = False
+        g = W.csr_from_edges(g.n, eu[keep], ev[keep])
+        us, vs = eu[pick], ev[pick]
+    else:
+        wl = W.make_workload(name)
+        g, roots, us, vs = wl.graph, wl.roots, wl.ins_u, wl.ins_v
+    ref = oracle.NaiveDynamicBC(g, roots)
+    with _dbc(g, roots, flags=EDGE) as dbc:
+        dbc.static_compute()
+        half = us.size // 2
+        for sl in (slice(0, half), slice(half, None)):
+            st = dbc.insert_edges(us[sl], vs[sl], stats=True)
+            for u, v in zip(us[sl], vs[sl]):
+                ref.insert(u, v)
+            assert st["case1"] + st["case2"] + st["case3"] == roots.size * us[sl].size
+            check_all(dbc, ref.compute(), roots.size)
+
+
+def test_edge_parallel_multicomponent_and_big_sigma():
+    """Case 3 from an unreachable endpoint, and sigma > 2^53 (the canonical re-sum)."""
+    g = W.random_gnm(300, 280, 5)
+    eu, ev = W.edges_of(g)
+    present = set(zip(eu.tolist(), ev.tolist()))
+    rng = np.random.default_rng(11)
+    pairs = []
+    while len(pairs) < 12:
+        a, b = sorted(int(x) for x in rng.choice(300, 2, replace=False))
+        if (a, b) not in present:
+            present.add((a, b))
+            pairs.append((a, b))
+    run_stream_single(g, np.arange(0, 300, 7), [p[0] for p in pairs], [p[1] for p in pairs],
+                      check_every=3, flags=EDGE)
+    g = W.grid_graph(60, 60)
+    cand = [(i * 60 + j, (i + 1) * 60 + j + 1) for i in range(0, 59, 7) for j in range(0, 59, 11)]
+    run_stream_single(g, np.array([0, 59, 3599, 1830], np.int32), [p[0] for p in cand[:8]],
+                      [p[1] for p in cand[:8]], check_every=4, flags=EDGE)
+
+
+def test_edge_parallel_equals_node_parallel_bitwise():
+    wl = W.make_workload("delaunay12")
+    outs = []
+    for flags in (0, EDGE):
+        with _dbc(wl.graph, wl.roots, flags=flags) as dbc:
+            dbc.static_compute()
+            dbc.insert_edges(wl.ins_u, wl.ins_v)
+            outs.append([dbc.get_root_state(s)[:2] for s in range(wl.roots.size)])
+    for (d0, s0), (d1, s1) in zip(outs[0], outs[1]):
+        assert np.array_equal(d0, d1) and np.array_equal(s0, s1)

@@ -408,3 +408,65 @@ def test_cpu_dynamic_grid_sigma_above_2_53():
             us.append(a)
             vs.append(b)
     _check_cpu_dynamic(g, np.array([0, 44, 1012, 2024], np.int32), us, vs)
+
+
+# --------------------------------------------------------------------------
+# the naive rule for edge deletion
+# --------------------------------------------------------------------------
+@pytest.mark.parametrize("n", [5, 8, 11])
+def test_delete_cycle_edge_gives_path(n):
+    """C_n minus (0, n-1) = P_n: BC(i) = 2 i (n-1-i)."""
+    g = W.cycle_graph(n)
+    dyn = oracle.NaiveDynamicBC(g, np.arange(n, dtype=np.int32))
+    dyn.delete(0, n - 1)
+    bc, *_ = dyn.compute()
+    assert bc.tolist() == [2.0 * i * (n - 1 - i) for i in range(n)]
+
+
+def test_delete_complete_to_star():
+    """K_7 minus every edge between leaves = S_7: BC(0) = 6*5, leaves 0."""
+    n = 7
+    g = W.complete_graph(n)
+    dyn = oracle.NaiveDynamicBC(g, np.arange(n, dtype=np.int32))
+    for a in range(1, n):
+        for b in range(a + 1, n):
+            dyn.delete(a, b)
+    bc, *_ = dyn.compute()
+    assert bc[0] == (n - 1) * (n - 2) and np.all(bc[1:] == 0)
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_delete_bruteforce_tiny(seed):
+    """Random deletions (and re-insertions) on tiny graphs vs path enumeration."""
+    rng = np.random.default_rng(500 + seed)
+    n = int(rng.integers(5, 9))
+    m = int(rng.integers(n, min(n * (n - 1) // 2, 2 * n) + 1))
+    g = W.random_gnm(n, m, 500 + seed)
+    eu, ev = W.edges_of(g)
+    edges = list(zip(eu.tolist(), ev.tolist()))
+    roots = np.arange(n, dtype=np.int32)
+    dyn = oracle.NaiveDynamicBC(g, roots)
+    for step in range(4):
+        a, b = edges.pop(int(rng.integers(len(edges))))
+        dyn.delete(a, b)
+        if step == 2:  # re-insert one: appended at the row ends
+            dyn.insert(a, b)
+            edges.append((a, b))
+        bc, d, sig, dl = dyn.compute()
+        bd, bs, bdl, bbc = brute_force(n, edges, roots.tolist())
+        for i in range(n):
+            assert d[i].tolist() == bd[i]
+            assert sig[i].tolist() == [float(x) for x in bs[i]]
+        for v in range(n):
+            assert bc[v] == pytest.approx(float(bbc[v]), rel=1e-12, abs=1e-12)
+
+
+def test_delete_keeps_row_order():
+    g = W.csr_from_edges(4, [0, 0, 0], [1, 2, 3])
+    dyn = oracle.NaiveDynamicBC(g, np.array([0], np.int32))
+    dyn.insert(1, 2)
+    dyn.delete(0, 2)
+    rp, col = dyn.csr()
+    assert col[rp[0]:rp[1]].tolist() == [1, 3]
+    assert col[rp[1]:rp[2]].tolist() == [0, 2]
+    assert col[rp[2]:rp[3]].tolist() == [1]

@@ -20,7 +20,8 @@ import numpy as np
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import workloads as W  # noqa: E402
-from paper_conf_ipps_mclaughlinb14_b200 import FLAG_NO_MERGE, FLAG_TIMING, DynamicBC  # noqa: E402
+from paper_conf_ipps_mclaughlinb14_b200 import (FLAG_EDGE_PARALLEL, FLAG_NO_MERGE, FLAG_TIMING,  # noqa: E402
+                                                DynamicBC)
 
 name = sys.argv[1] if len(sys.argv) > 1 else "rmat16"
 B = int(sys.argv[2]) if len(sys.argv) > 2 else 100
@@ -71,4 +72,21 @@ out["table3"] = {"static_ms": static_ms, "fastest_ms": float(per.min()), "averag
                  "what": "device time of the update kernel of single-edge dbc_insert_edges calls (graph update neglected as in P:440), "
                          "DBC_FLAG_NO_MERGE, vs one dbc_static_compute over the same roots"}
 out["table3_paper"] = "45x mean speedup over static GPU recompute; slowest 2x-43x (P:512-514)"
+
+# Table II: node-based vs edge-based parallelism, same single-edge calls
+BE = min(B, int(os.environ.get("EDGE_INSERTIONS", "20")))
+with DynamicBC(g.n, g.row_ptr, g.col, wl.roots, flags=FLAG_TIMING | FLAG_EDGE_PARALLEL) as dbc:
+    dbc.static_compute()
+    dbc.synchronize()
+    pe = []
+    for i in range(BE + 3):
+        dbc.insert_edges(wl.ins_u[i:i + 1], wl.ins_v[i:i + 1])
+        if i >= 3:
+            pe.append(dbc.timings()["update_ms"])
+pe = np.array(pe)
+out["table2"] = {"insertions": BE, "node_avg_ms": float(per[:BE].mean()), "edge_avg_ms": float(pe.mean()),
+                 "node_over_edge": float(pe.mean() / per[:BE].mean()),
+                 "what": "same first insertions, single-edge calls: node-based kernel (DBC_FLAG_NO_MERGE) vs "
+                         "edge-based kernel (DBC_FLAG_EDGE_PARALLEL, Alg. 4/6)"}
+out["table2_paper"] = "node-based 4.0x (small) to 37.2x (coPapersCiteseer) faster than edge-based (P:458-478)"
 print(json.dumps(out))
