@@ -178,6 +178,29 @@ dbc_status dbc_insert_edges_device(dbc_ctx *c, const int32_t *u_device,
                                    const int32_t *v_device, int64_t count,
                                    dbc_insert_stats *stats);
 
+/* Deletes count >= 0 undirected edges (u[i], v[i]) given in HOST memory, with
+ * the semantics of count sequential single-edge deletions (the decremental
+ * counterpart of P:440; P:144 names deletion as the adjacent workload).  The
+ * whole batch is validated first (range, self loop, duplicate pair within the
+ * batch, edge not present -> DBC_EEDGE; nothing changes on error).  Each edge
+ * leaves a tombstone in both adjacency rows (the rows keep the order of their
+ * remaining entries -- the canonical order of DESIGN.md R5); a later
+ * insertion of the same edge appends it again.  Per root the update follows
+ * DESIGN.md R20: Case 1 if d(u) == d(v); if u_low keeps another predecessor
+ * only sigma below it changes; else the affected vertices move down (or
+ * become unreachable: d = DBC_INF, sigma = delta = 0).  Requires a prior
+ * dbc_static_compute (DBC_ESTATE); not available with
+ * DBC_FLAG_EDGE_PARALLEL (DBC_EINVAL).  stats: nullable, as for insertions
+ * (case_count[2] counts deletions that moved a vertex). */
+dbc_status dbc_delete_edges(dbc_ctx *c, const int32_t *u, const int32_t *v,
+                            int64_t count, dbc_insert_stats *stats);
+
+/* Same as dbc_delete_edges with u, v in DEVICE memory (copied to the host
+ * for the batch checks). */
+dbc_status dbc_delete_edges_device(dbc_ctx *c, const int32_t *u_device,
+                                   const int32_t *v_device, int64_t count,
+                                   dbc_insert_stats *stats);
+
 /* Copies this rank's BC partial (sum over LOCAL roots, Eq. (3)) to host
  * bc[n].  With world == 1 this is the global BC.  Synchronises.  Returns
  * DBC_ENUMERIC if an earlier update overflowed. */

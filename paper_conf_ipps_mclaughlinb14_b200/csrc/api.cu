@@ -22,6 +22,7 @@ struct dbc_ctx {
     uint32_t flags = 0;
     int32_t n = 0;
     int64_t nnz = 0, nnz0 = 0, col_cap = 0;
+    int64_t deleted = 0;  // edges deleted (tombstones in the rows)
     int64_t edge_cap = 0, inserted = 0;
     int32_t k = 0, k_loc = 0;
     std::vector<int32_t> roots_local;        // internal vertex ids of the local roots
@@ -690,6 +691,7 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     a.help = HelpBoard{};  // Mode S: no cooperative help
     a.merge = (c->flags & DBC_FLAG_NO_MERGE) ? 0 : 1;
     a.scen = nullptr;
+    a.del = 0;
     if (c->scen_cap > 0) {  // Fig. 2 / Fig. 4 log: one job per (root, insertion)
         if (cnt > c->scen_cap)
             return fail(c, DBC_EINVAL, "batch of %lld exceeds the scenario log (%lld insertions)",
@@ -861,6 +863,153 @@ extern "C" dbc_status dbc_insert_edges(dbc_ctx *c, const int32_t *u, const int32
         CK(cudaGetLastError());
     }
     return insert_device(c, c->bu, c->bv, count, stats);
+}
+
+// Edge deletions (decremental update, R20): validated as a whole
+// (host: range, self loop, duplicate pair; device: presence), then applied one
+// at a time -- tombstone the edge in both rows, then one update launch over
+// all local roots for that deletion (sequential semantics, as P:440 applies
+// insertions).  u, v: caller ids on the HOST.
+static dbc_status delete_host_ids(dbc_ctx *c, const int32_t *u, const int32_t *v, int64_t cnt,
+                                  dbc_insert_stats *stats) {
+    if (!c->have_state) return fail(c, DBC_ESTATE, "dbc_static_compute must run before deletions");
+    if (c->flags & DBC_FLAG_EDGE_PARALLEL)
+        return fail(c, DBC_EINVAL, "deletions are not supported with DBC_FLAG_EDGE_PARALLEL");
+    if (cnt > c->edge_cap) return fail(c, DBC_EINVAL, "deletion batch larger than the staging buffer");
+    {
+        std::vector<int64_t> keys((size_t)cnt);
+        for (int64_t i = 0; i < cnt; ++i) {
+            const int32_t a = u[i], b = v[i];
+            if (a < 0 || a >= c->n || b < 0 || b >= c->n || a == b)
+                return fail(c, DBC_EEDGE, "deletion batch rejected: self loop or vertex out of range");
+            keys[(size_t)i] = ((int64_t)std::min(a, b) << 32) | (uint32_t)std::max(a, b);
+        }
+        std::sort(keys.begin(), keys.end());
+        if (std::adjacent_find(keys.begin(), keys.end()) != keys.end())
+            return fail(c, DBC_EEDGE, "deletion batch rejected: duplicate edge within the batch");
+    }
+    CK(cudaSetDevice(c->device));
+    const bool tm = c->flags & DBC_FLAG_TIMING;
+    cudaEvent_t *ev = c->ev + (c->evset ? 0 : 6);
+    if (tm) CK(cudaEventRecord(ev[0], c->stream));
+    int launches = 0;
+    if (cnt) {
+        CK(cudaMemcpyAsync(c->bu, u, sizeof(int32_t) * cnt, cudaMemcpyHostToDevice, c->stream));
+        CK(cudaMemcpyAsync(c->bv, v, sizeof(int32_t) * cnt, cudaMemcpyHostToDevice, c->stream));
+        launches += map_ids(c->bu, c->bv, c->bu, c->bv, cnt, c->perm_d, c->n, c->stream);
+    }
+    launches += validate_deletions(view_of(c), c->n, c->bu, c->bv, cnt, c->ab.bad, c->stream);
+    CK(cudaGetLastError());
+    int32_t bad = 0;
+    CK(cudaMemcpyAsync(&bad, c->ab.bad, sizeof(int32_t), cudaMemcpyDeviceToHost, c->stream));
+    CK(cudaStreamSynchronize(c->stream));
+    TRY(fold_timings(c));
+    c->prof_pending = false;  // a deletion launch is no guide to the next batch's heavy roots
+    if (bad) return fail(c, DBC_EEDGE, "deletion batch rejected: edge not present");
+    unsigned long long h0[kStCount] = {};
+    if (stats) TRY(read_stats(c, h0));
+    if (cnt == 0) {
+        if (stats) std::memset(stats, 0, sizeof(*stats));
+        return DBC_OK;
+    }
+    const uint64_t jobs = 2ull * (uint64_t)c->k_loc * (uint64_t)cnt;  // two epochs per job
+    if (c->epoch_used + jobs + 1 >= (1ull << 30)) TRY(reset_epochs(c));
+    c->epoch_used += jobs;
+    if (tm) CK(cudaEventRecord(ev[1], c->stream));
+    UpdateArgs a;
+    a.g = view_of(c);
+    a.n = c->n;
+    a.k_loc = c->k_loc;
+    a.roots = c->roots_d;
+    a.d = c->d;
+    a.sd = c->sd;
+    a.l2mask = c->l2mask;
+    a.mask_ds = c->mask_ds;
+    a.bc = c->bc;
+    a.ins_u = c->bu;
+    a.ins_v = c->bv;
+    a.ws = worker_scratch(c);
+    a.next_slot = c->next_slot;
+    a.stats = c->stats;
+    a.err = c->err;
+    a.root_prof = nullptr;
+    a.slot_list = nullptr;
+    a.slot_count = 0;
+    a.worker_base = 0;
+    a.help = HelpBoard{};
+    a.merge = 0;
+    a.del = 1;
+    a.scen = nullptr;
+    if (c->scen_cap > 0) {
+        if (cnt > c->scen_cap)
+            return fail(c, DBC_EINVAL, "batch of %lld exceeds the scenario log (%lld insertions)",
+                        (long long)cnt, (long long)c->scen_cap);
+        a.scen = c->scen;
+        c->scen_last = cnt;
+    }
+    if (tm) CK(cudaEventRecord(ev[2], c->stream));
+    int ulaunch = 0;
+    for (int64_t i = 0; i < cnt; ++i) {
+        launches += tombstone_edge(c->rp[c->cur], c->col[c->cur], c->scol[c->cur], c->bu, c->bv, i,
+                                   c->stream);
+        if (c->workers) {
+            CK(cudaMemsetAsync(c->next_slot, 0, sizeof(int32_t), c->stream));
+            a.ins_begin = (int32_t)i;
+            a.ins_end = (int32_t)i + 1;
+            if (c->block == 128)
+                launch_update_128(a, c->workers, c->stream);
+            else if (c->block == 512)
+                (c->ub2 ? launch_update_512x2 : launch_update_512)(a, c->workers, c->stream);
+            else
+                launch_update_256(a, c->workers, c->stream);
+            ++ulaunch;
+        }
+    }
+    CK(cudaGetLastError());
+    if (tm) {
+        CK(cudaEventRecord(ev[3], c->stream));
+        c->evset ^= 1;
+        c->tm_pending = true;
+    }
+    launches += ulaunch;
+    c->deleted += cnt;
+    c->tm.update_launches = ulaunch;
+    c->tm.kernel_launches = launches;
+    c->tm.update_launches_total += ulaunch;
+    c->tm.kernel_launches_total += launches;
+    if (stats) {
+        unsigned long long h[kStCount];
+        TRY(read_stats(c, h));
+        stats->insertions = cnt;
+        stats->case_count[0] = (int64_t)(h[kStCase1] - h0[kStCase1]);
+        stats->case_count[1] = (int64_t)(h[kStCase2] - h0[kStCase2]);
+        stats->case_count[2] = (int64_t)(h[kStCase3] - h0[kStCase3]);
+        stats->touched = (int64_t)(h[kStTouched] - h0[kStTouched]);
+        stats->down_vertices = (int64_t)(h[kStDown] - h0[kStDown]);
+        stats->edges_scanned = (int64_t)(h[kStScanned] - h0[kStScanned]);
+        stats->alg_bytes = (int64_t)(h[kStBytes] - h0[kStBytes]);
+    }
+    return DBC_OK;
+}
+
+extern "C" dbc_status dbc_delete_edges(dbc_ctx *c, const int32_t *u, const int32_t *v, int64_t count,
+                                       dbc_insert_stats *stats) {
+    if (!c) return DBC_EINVAL;
+    if (count < 0 || (count > 0 && (!u || !v))) return fail(c, DBC_EINVAL, "bad batch");
+    return delete_host_ids(c, u, v, count, stats);
+}
+
+extern "C" dbc_status dbc_delete_edges_device(dbc_ctx *c, const int32_t *u, const int32_t *v,
+                                              int64_t count, dbc_insert_stats *stats) {
+    if (!c) return DBC_EINVAL;
+    if (count < 0 || (count > 0 && (!u || !v))) return fail(c, DBC_EINVAL, "bad batch");
+    CK(cudaSetDevice(c->device));
+    std::vector<int32_t> hu((size_t)count), hv((size_t)count);  // the host-side batch checks
+    if (count) {
+        CK(cudaMemcpy(hu.data(), u, sizeof(int32_t) * count, cudaMemcpyDeviceToHost));
+        CK(cudaMemcpy(hv.data(), v, sizeof(int32_t) * count, cudaMemcpyDeviceToHost));
+    }
+    return delete_host_ids(c, hu.data(), hv.data(), count, stats);
 }
 
 static dbc_status check_err(dbc_ctx *c) {

@@ -537,6 +537,7 @@ struct UpdateArgs {
     HelpBoard help;                // help.word == nullptr: no cooperative help
     int32_t merge;                 // 1: a window of ws.wcap insertions per job; 0: one per insertion
     long long *scen;               // nullable: scenario log [batch insertion][k_loc] (merge == 0)
+    int32_t del;                   // 1: ins_u/ins_v[ins_begin] is an edge DELETION (already tombstoned)
 };
 
 struct StaticArgs {

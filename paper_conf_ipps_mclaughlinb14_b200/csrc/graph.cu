@@ -23,8 +23,9 @@ static inline unsigned blocks_for(int64_t items, int threads) {
 }
 
 // one warp per batch edge: range / self loop / presence in the current graph
+// (insertions: present -> bit 2; deletions (absent_bit = 4): absent -> bit 4)
 __global__ void k_validate_edges(GView g, int32_t n, const int32_t *u, const int32_t *v,
-                                 int64_t cnt, int32_t *bad) {
+                                 int64_t cnt, int32_t *bad, int32_t absent_bit = 0) {
     const int lane = threadIdx.x & 31;
     const int64_t e = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     if (e >= cnt) return;
@@ -39,7 +40,53 @@ __global__ void k_validate_edges(GView g, int32_t n, const int32_t *u, const int
     const int target = use_a ? b : a;
     bool found = false;
     for (int j = r.x + lane; j < r.y; j += 32) found |= (ldg_i(g.col + j) == target);
-    if (__any_sync(kFull, found) && lane == 0) atomicOr(bad, 2);
+    const bool any = __any_sync(kFull, found);
+    if (lane == 0) {
+        if (!absent_bit && any) atomicOr(bad, 2);
+        if (absent_bit && !any) atomicOr(bad, absent_bit);
+    }
+}
+
+// Deletion of edge i of the batch (u[i], v[i]): one warp per endpoint row.  The
+// canonical row keeps its order with the entry replaced by a tombstone -- the
+// row's own vertex, inert in every kernel (a self entry never satisfies a
+// predecessor / successor / lowering test) -- and the sorted row drops the
+// entry (shifted left, INT32_MAX appended: still sorted, never matched).
+__global__ void k_tombstone(const int32_t *rp, int32_t *col, int32_t *scol, const int32_t *u,
+                            const int32_t *v, int64_t i) {
+    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int a = w == 0 ? u[i] : v[i], b = w == 0 ? v[i] : u[i];
+    const int rb = rp[a] & kMask, re = rp[a + 1] & kMask;
+    for (int j = rb + lane; j < re; j += 32)
+        if (col[j] == b) col[j] = a;
+    int p = -1;
+    for (int j = rb + lane; j < re; j += 32)
+        if (scol[j] == b) p = j;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) p = max(p, __shfl_xor_sync(kFull, p, o));
+    if (p < 0) return;
+    for (int base = p; base < re - 1; base += 32) {
+        const int j = base + lane;
+        const int val = (j < re - 1) ? scol[j + 1] : 0;
+        __syncwarp();
+        if (j < re - 1) scol[j] = val;
+        __syncwarp();
+    }
+    if (lane == 0) scol[re - 1] = INT32_MAX;
+}
+
+int validate_deletions(const GView &g, int32_t n, const int32_t *u, const int32_t *v, int64_t cnt,
+                       int32_t *bad, cudaStream_t s) {
+    cudaMemsetAsync(bad, 0, sizeof(int32_t), s);
+    if (!cnt) return 0;
+    k_validate_edges<<<blocks_for(cnt * 32, 256), 256, 0, s>>>(g, n, u, v, cnt, bad, 4);
+    return 1;
+}
+
+int tombstone_edge(const int32_t *rp, int32_t *col, int32_t *scol, const int32_t *u, const int32_t *v,
+                   int64_t i, cudaStream_t s) {
+    k_tombstone<<<1, 64, 0, s>>>(rp, col, scol, u, v, i);
+    return 1;
 }
 
 // count directed batch entries per vertex; remember each entry's arrival slot

@@ -115,6 +115,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
     __shared__ int s_un[2][kUcap];       // up frontier ping-pong (overflow: U0 / U1)
     __shared__ int s_hb, s_hpick, s_hseq; // cooperative help: grabbed block, owner, request
     __shared__ HelpCtx s_hctx;
+    __shared__ int s_del[6];     // deletion job: [0] u_high, [1] u_low, [2] |A|, [3] seeds, [4] candidates, [5] u_low keeps a predecessor
+    __shared__ double s_delsd[2];  // deletion job: old sigma / delta of u_low
 
     const int tid = threadIdx.x;
     const int wk = a.worker_base + blockIdx.x;  // scratch of this worker
@@ -252,12 +254,15 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                 }
             }
             {
+                if (a.del) ++epoch;  // deletion: one epoch for the affected-set search, one for the job
                 ++epoch;
                 ++prof_jobs;
                 const unsigned long long touch0 = st_touched;  // scenario log (thread 0's counter)
                 const uint32_t E = epoch << 2;
                 const uint32_t mD = E | kDown, mU = E | kUp;
-                const int g0 = ins, lim = wend - 1;  // the job's insertions; graph as of lim
+                // the job's insertions and the graph as of lim; a deletion sees
+                // every entry (tombstoned edge excluded) and has no new edge
+                const int g0 = a.del ? INT32_MAX : ins, lim = a.del ? INT32_MAX - 1 : wend - 1;
                 if (tid < 32) {  // warp 0: the root's row as of this job (level-2 masks)
                     const int2 rs = row_of(g, sroot, lim);
                     const int dsr = rs.y - rs.x;
@@ -279,11 +284,157 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                     s_rmax = 0;
                 }
                 __syncthreads();
+                if (a.del) {
+                    // ---- edge deletion (decremental update, R20) ----
+                    // The edge (u_high, u_low) is already a tombstone in both rows.
+                    if (tid == 0) {
+                        const int u = __ldg(a.ins_u + ins), v = __ldg(a.ins_v + ins);
+                        const int uh = st.d[u] < st.d[v] ? u : v, ul = uh == u ? v : u;
+                        s_del[0] = uh;
+                        s_del[1] = ul;
+                        s_del[2] = 0;
+                        s_del[3] = 0;
+                        s_del[4] = 0;
+                        s_del[5] = 0;
+                        const double2 q = st.sd[ul];
+                        s_delsd[0] = q.x;
+                        s_delsd[1] = q.y;
+                    }
+                    __syncthreads();
+                    const int ul = s_del[1];
+                    const int Lul = st.d[ul];
+                    if (tid < 32) {  // does u_low keep a predecessor?
+                        const int2 r = row_of(g, ul, lim);
+                        bool keep = false;
+                        for (int j = r.x + tid; j < r.y && !keep; j += 32) keep = st.d[ldg_i(g.col + j)] == Lul - 1;
+                        if (__any_sync(kFull, keep) && tid == 0) s_del[5] = 1;
+                    }
+                    __syncthreads();
+                    if (s_del[5]) {  // distances unchanged: sigma shrinks below u_low (seed u_low)
+                        if (tid == 0) {
+                            Rv[0] = ul;
+                            Rl[0] = Lul;
+                            s_del[3] = 1;
+                            s_job[2] = Lul;
+                            s_job[7] = Lul;
+                        }
+                    } else {
+                        // A = the vertices whose distance grows: u_low, then level by level
+                        // every old successor all of whose predecessors are in A.  A is
+                        // raised to INF (old d kept in lowrec, tagged with the job epoch);
+                        // successors that keep a predecessor lose paths: seeds at their level.
+                        const uint32_t mA = ((epoch - 1) << 2) | kDown;  // search epoch
+                        if (tid == 0) {
+                            lowrec[ul] = ((unsigned long long)epoch << 32) | (uint32_t)Lul;
+                            st.d[ul] = kInf;
+                            Ua[0] = ul;
+                            s_del[2] = 1;
+                            s_job[3] = 1;
+                            s_wcnt[1] = 1;  // a distance changes: reported as Case 3
+                            --st_c2;
+                            ++st_c3;
+                        }
+                        __syncthreads();
+                        int fb = 0, fe = 1, la = Lul;
+                        while (fb < fe) {
+                            for (int i = fb + tid; i < fe; i += kBlock) {
+                                const int x = Ua[i];
+                                const int2 r = row_of(g, x, lim);
+                                for (int j = r.x; j < r.y; ++j) {
+                                    const int y = ldg_i(g.col + j);
+                                    if (st.d[y] == la + 1 && atomicMax(mark + y, mA) < mA)
+                                        Bq[atomicAdd(&s_del[4], 1)] = y;
+                                }
+                            }
+                            __syncthreads();
+                            const int nc = s_del[4];
+                            for (int i = tid; i < nc; i += kBlock) {
+                                const int y = Bq[i];
+                                const int2 r = row_of(g, y, lim);
+                                bool keep = false;
+                                for (int j = r.x; j < r.y && !keep; ++j) keep = st.d[ldg_i(g.col + j)] == la;
+                                if (keep) {  // y keeps its level, its sigma changes
+                                    const int q = atomicAdd(&s_del[3], 1);
+                                    Rv[q] = y;
+                                    Rl[q] = la + 1;
+                                } else {
+                                    lowrec[y] = ((unsigned long long)epoch << 32) | (uint32_t)(la + 1);
+                                    Ua[atomicAdd(&s_del[2], 1)] = y;
+                                }
+                            }
+                            __syncthreads();
+                            for (int i = tid; i < nc; i += kBlock) {  // raise the new A level (after every check)
+                                const int y = Bq[i];
+                                if ((uint32_t)(lowrec[y] >> 32) == epoch) st.d[y] = kInf;
+                            }
+                            if (tid == 0) s_del[4] = 0;
+                            __syncthreads();
+                            fb = fe;
+                            fe = s_del[2];
+                            ++la;
+                        }
+                        // seeds of A: one more than the nearest vertex outside A
+                        const int na = s_del[2];
+                        for (int i = tid; i < na; i += kBlock) {
+                            const int x = Ua[i];
+                            const int2 r = row_of(g, x, lim);
+                            int t = kInf;
+                            for (int j = r.x; j < r.y; ++j) {
+                                const int dy = st.d[ldg_i(g.col + j)];
+                                if (dy != kInf) t = min(t, dy + 1);
+                            }
+                            if (t != kInf) {
+                                const int q = atomicAdd(&s_del[3], 1);
+                                Rv[q] = x;
+                                Rl[q] = t;
+                            }
+                        }
+                        __syncthreads();
+                        const int ns = s_del[3];
+                        int lmin = INT32_MAX, lmax = 0;
+                        for (int i = tid; i < ns; i += kBlock) {
+                            lmin = min(lmin, Rl[i]);
+                            lmax = max(lmax, Rl[i]);
+                        }
+#pragma unroll
+                        for (int o = 16; o; o >>= 1) {
+                            lmin = min(lmin, __shfl_xor_sync(kFull, lmin, o));
+                            lmax = max(lmax, __shfl_xor_sync(kFull, lmax, o));
+                        }
+                        if (tid == 0) {
+                            s_job[2] = INT32_MAX;
+                            s_job[7] = 0;
+                        }
+                        __syncthreads();
+                        if ((tid & 31) == 0) {
+                            atomicMin(&s_job[2], lmin);
+                            atomicMax(&s_job[7], lmax);
+                        }
+                        __syncthreads();
+                        if (tid == 0 && ns == 0) {  // everything below u_low is cut off
+                            s_job[2] = 1;
+                            s_job[7] = 1;
+                        }
+                    }
+                    __syncthreads();
+                }
                 const int L0 = s_job[2];
                 const int Lseed = s_job[7];
                 const int mstate = s_job[4], dsr = s_job[5];
                 // enqueue the seeds of level Lq (between levels: no concurrent lowering)
                 auto inject = [&](int Lq) {
+                    if (a.del) {  // deletion seeds (u_low, or A / lost-path vertices)
+                        const int ns = s_del[3];
+                        for (int q = tid; q < ns; q += kBlock) {
+                            if (Rl[q] != Lq) continue;
+                            const int b = Rv[q];
+                            const int db = st.d[b];
+                            if (db < Lq) continue;  // reached earlier by the search
+                            if (db > Lq) atomicMin(st.d + b, Lq);  // raised vertex: old d already recorded
+                            if (atomicMax(mark + b, mD) < mD) Dv[atomicAdd(&s_dcnt, 1)] = b;
+                        }
+                        return;
+                    }
                     for (int q = tid; q < nwin; q += kBlock) {
                         if (Wlev[q] != Lq) continue;
                         const int b = Wul[q];
@@ -337,7 +488,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                     }
                     if (dy > L + 1) {  // Case 3 pull-up
                         const int old = atomicMin(st.d + y, L + 1);
-                        if (old > L + 1) {
+                        if (old > L + 1 && !(a.del && (uint32_t)(lowrec[y] >> 32) == epoch)) {
                             lowrec[y] = ((unsigned long long)epoch << 32) | (uint32_t)old;
                             s_job[3] = 1;
                             st_bytes += 4;
@@ -388,7 +539,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                         st_bytes += 8;
                                         if (mvalid && L == 2) m |= l1bit(y[u]);
                                     }
-                                    if (dy[u] > L + 1 && om[u] > L + 1) {  // first lowerer (Case 3)
+                                    if (dy[u] > L + 1 && om[u] > L + 1 &&  // first lowerer (Case 3)
+                                        !(a.del && (uint32_t)(lowrec[y[u]] >> 32) == epoch)) {
                                         lowrec[y[u]] = ((unsigned long long)epoch << 32) | (uint32_t)om[u];
                                         s_job[3] = 1;
                                         st_bytes += 4;
@@ -470,6 +622,35 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                 const bool mok = mstate != 0;  // masks valid for the up phase
                 const bool case3 = s_job[3] != 0;  // some distance was lowered (read after the level barriers)
 
+                if (a.del) {
+                    // deletion: A vertices the search never reached are cut off from
+                    // the root (d = INF, sigma = delta = 0, P:150-159 reading R4); the
+                    // deleted edge carried u_low's old contribution to u_high
+                    const int na = s_del[2];
+                    for (int i = tid; i < na; i += kBlock) {
+                        const int x = Ua[i];
+                        if (st.d[x] != kInf) continue;
+                        const double od = st.sd[x].y;
+                        if (od != 0.0) atomicAdd(a.bc + x, -od);
+                        st.sd[x] = make_double2(0.0, 0.0);
+                        st_bytes += 32;
+                    }
+                    if (tid == 0) {
+                        const int uh = s_del[0];
+                        const int dh = st.d[uh];
+                        if (dh >= 1) {  // the root's delta is never used
+                            atomicAdd(dacc + uh, -__dmul_rn(__ddiv_rn(st.sd[uh].x, s_delsd[0]), 1.0 + s_delsd[1]));
+                            if (atomicMax(mark + uh, mU) < E) {
+                                const int pos = atomicAdd(&s_rcnt, 1);
+                                Rv[pos] = uh;
+                                Rl[pos] = dh;
+                                atomicMax(&s_rmax, dh);
+                            }
+                        }
+                    }
+                    __syncthreads();
+                }
+
                 tick(0);
                 // ================= (0) Case-3 removal pushes =================
                 if (case3) {
@@ -533,6 +714,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                     __syncthreads();
                 }
                 const int rcnt = s_rcnt;
+                // a deletion's removal targets can sit one level above the seeds (u_high)
+                const int Lstop = a.del ? min(L0, st.d[s_del[0]]) : L0;
                 const int Lmax = max(LmaxD, s_rmax);
                 if (tid == 0) st_touched += rcnt;
 
@@ -542,7 +725,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                 int ucur_sel = 0;
                 int ucnt = 0;
                 for (int l = Lmax; l >= 1; --l) {
-                    if (l < L0 && ucnt == 0) break;  // nothing left above the insertion
+                    if (l < Lstop && ucnt == 0) break;  // nothing left above the insertion
                     const bool push = l >= 2;          // level-1 vertices only feed the root
                     ++st_lvu;
                     // queue p for level l-1 unless already queued: the prefetched mark

@@ -84,6 +84,8 @@ SIGNATURES = {
     "dbc_static_compute": (ctypes.c_int, [_P]),
     "dbc_insert_edges": (ctypes.c_int, [_P, _P, _P, ctypes.c_int64, _P]),
     "dbc_insert_edges_device": (ctypes.c_int, [_P, _P, _P, ctypes.c_int64, _P]),
+    "dbc_delete_edges": (ctypes.c_int, [_P, _P, _P, ctypes.c_int64, _P]),
+    "dbc_delete_edges_device": (ctypes.c_int, [_P, _P, _P, ctypes.c_int64, _P]),
     "dbc_get_bc": (ctypes.c_int, [_P, _P]),
     "dbc_get_bc_partial_device": (ctypes.c_int, [_P, _P]),
     "dbc_get_root_state": (ctypes.c_int, [_P, ctypes.c_int32, _P, _P, _P]),
@@ -201,8 +203,7 @@ class DynamicBC:
     def static_compute(self):
         _check(self._ctx, self._lib.dbc_static_compute(self._ctx))
 
-    def insert_edges(self, u, v, stats=False):
-        """Host arrays -> dbc_insert_edges; CUDA tensors -> dbc_insert_edges_device."""
+    def _edges_call(self, host_fn, dev_fn, u, v, stats):
         st = InsertStats() if stats else None
         stp = ctypes.byref(st) if st is not None else None
         if hasattr(u, "is_cuda") and u.is_cuda:
@@ -210,15 +211,22 @@ class DynamicBC:
 
             assert u.dtype == torch.int32 and v.dtype == torch.int32 and u.numel() == v.numel()
             assert u.is_contiguous() and v.is_contiguous()
-            rc = self._lib.dbc_insert_edges_device(self._ctx, ctypes.c_void_p(u.data_ptr()),
-                                                   ctypes.c_void_p(v.data_ptr()), u.numel(), stp)
+            rc = dev_fn(self._ctx, ctypes.c_void_p(u.data_ptr()), ctypes.c_void_p(v.data_ptr()), u.numel(), stp)
         else:
             uu, vv = _host(u, np.int32).ravel(), _host(v, np.int32).ravel()
             if uu.size != vv.size:
                 raise ValueError("u and v differ in length")
-            rc = self._lib.dbc_insert_edges(self._ctx, _np_ptr(uu), _np_ptr(vv), uu.size, stp)
+            rc = host_fn(self._ctx, _np_ptr(uu), _np_ptr(vv), uu.size, stp)
         _check(self._ctx, rc)
         return st.as_dict() if st is not None else None
+
+    def insert_edges(self, u, v, stats=False):
+        """Host arrays -> dbc_insert_edges; CUDA tensors -> dbc_insert_edges_device."""
+        return self._edges_call(self._lib.dbc_insert_edges, self._lib.dbc_insert_edges_device, u, v, stats)
+
+    def delete_edges(self, u, v, stats=False):
+        """Host arrays -> dbc_delete_edges; CUDA tensors -> dbc_delete_edges_device."""
+        return self._edges_call(self._lib.dbc_delete_edges, self._lib.dbc_delete_edges_device, u, v, stats)
 
     def get_bc(self, out=None):
         out = np.empty(self.n, dtype=np.float64) if out is None else out

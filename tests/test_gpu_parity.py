@@ -566,3 +566,112 @@ def test_edge_parallel_equals_node_parallel_bitwise():
             outs.append([dbc.get_root_state(s)[:2] for s in range(wl.roots.size)])
     for (d0, s0), (d1, s1) in zip(outs[0], outs[1]):
         assert np.array_equal(d0, d1) and np.array_equal(s0, s1)
+
+
+# ------------------------------------------------ edge deletion (Sec. 8(f) #4) ----
+def _existing_edges(g, count, seed, roots=None, incident_to_roots=0):
+    eu, ev = W.edges_of(g)
+    rng = np.random.default_rng(seed)
+    pick = list(rng.permutation(eu.size)[:count])
+    out = [(int(eu[i]), int(ev[i])) for i in pick]
+    if incident_to_roots and roots is not None:  # also edges at the roots (level-1 changes)
+        rs = set(int(r) for r in roots)
+        inc = [(int(a), int(b)) for a, b in zip(eu, ev) if int(a) in rs or int(b) in rs]
+        for i in rng.permutation(len(inc))[:incident_to_roots]:
+            if inc[i] not in out:
+                out.append(inc[i])
+    return out
+
+
+def run_delete_stream(g, roots, pairs, batch=1, check_every=1, flags=0):
+    roots = np.asarray(roots, np.int32)
+    ref = oracle.NaiveDynamicBC(g, roots)
+    with _dbc(g, roots, flags=flags) as dbc:
+        dbc.static_compute()
+        for b0 in range(0, len(pairs), batch):
+            chunk = pairs[b0:b0 + batch]
+            st = dbc.delete_edges([p[0] for p in chunk], [p[1] for p in chunk], stats=True)
+            assert st["case1"] + st["case2"] + st["case3"] == roots.size * len(chunk)
+            for a, b in chunk:
+                ref.delete(a, b)
+            if (b0 // batch + 1) % check_every == 0 or b0 + batch >= len(pairs):
+                check_all(dbc, ref.compute(), roots.size)
+        return dbc
+
+
+@pytest.mark.parametrize("n", [5, 8, 9])
+def test_delete_cycle_to_path_and_split(n):
+    g = W.cycle_graph(n)
+    # C_n -> P_n (distances grow), then cut the path in two (unreachable halves)
+    run_delete_stream(g, np.arange(n), [(0, n - 1), (2, 3)])
+
+
+def test_delete_complete_to_star():
+    n = 7
+    pairs = [(a, b) for a in range(1, n) for b in range(a + 1, n)]
+    run_delete_stream(W.complete_graph(n), np.arange(n), pairs)
+    run_delete_stream(W.complete_graph(n), np.arange(n), pairs, batch=len(pairs))
+
+
+@pytest.mark.parametrize("name", ["karate", "rmat10", "delaunay12"])
+def test_delete_single_and_batch_match_oracle(name):
+    wl = W.make_workload(name)
+    pairs = _existing_edges(wl.graph, 30, 1, wl.roots, incident_to_roots=6)
+    run_delete_stream(wl.graph, wl.roots, pairs, batch=1, check_every=3)
+    run_delete_stream(wl.graph, wl.roots, pairs, batch=12)
+
+
+def test_delete_multicomponent_and_isolating():
+    g = W.random_gnm(200, 230, 8)
+    roots = np.arange(0, 200, 9)
+    pairs = _existing_edges(g, 60, 2)  # tree-like graph: many deletions disconnect
+    run_delete_stream(g, roots, pairs, batch=1, check_every=5)
+
+
+def test_delete_grid_sigma_above_2_53():
+    g = W.grid_graph(45, 45)
+    roots = np.array([0, 44, 1012, 2024], np.int32)
+    run_delete_stream(g, roots, _existing_edges(g, 10, 3), batch=1, check_every=5)
+
+
+def test_delete_insert_mixed_stream():
+    """Insert a batch, delete some of those and some original edges, re-insert."""
+    wl = W.make_workload("rmat10")
+    g, roots = wl.graph, wl.roots
+    ref = oracle.NaiveDynamicBC(g, roots)
+    orig = _existing_edges(g, 10, 5)
+    with _dbc(g, roots) as dbc:
+        dbc.static_compute()
+        ins = list(zip(wl.ins_u[:20].tolist(), wl.ins_v[:20].tolist()))
+        dbc.insert_edges([p[0] for p in ins], [p[1] for p in ins])
+        for a, b in ins:
+            ref.insert(a, b)
+        dele = ins[3:9] + orig
+        dbc.delete_edges([p[0] for p in dele], [p[1] for p in dele])
+        for a, b in dele:
+            ref.delete(a, b)
+        check_all(dbc, ref.compute(), roots.size)
+        back = dele[:4] + dele[-3:]
+        dbc.insert_edges([p[0] for p in back], [p[1] for p in back])
+        for a, b in back:
+            ref.insert(a, b)
+        check_all(dbc, ref.compute(), roots.size)
+        dbc.static_compute()  # GPU recompute on the final graph == the oracle too
+        check_all(dbc, ref.compute(), roots.size)
+
+
+def test_delete_rejects_bad_batches_atomically():
+    from paper_conf_ipps_mclaughlinb14_b200 import DBCError
+
+    wl = W.make_workload("karate")
+    g, roots = wl.graph, wl.roots
+    ref = oracle.brandes_csr(g, roots)
+    eu, ev = W.edges_of(g)
+    with _dbc(g, roots) as dbc:
+        dbc.static_compute()
+        for bad in ([(int(eu[0]), int(ev[0])), (5, 9)],          # (5, 9) absent in karate
+                    [(int(eu[0]), int(ev[0])), (int(ev[0]), int(eu[0]))],  # duplicate pair
+                    [(3, 3)], [(0, 34)]):
+            with pytest.raises(DBCError):
+                dbc.delete_edges([p[0] for p in bad], [p[1] for p in bad])
+        check_all(dbc, ref, roots.size)  # nothing changed
