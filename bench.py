@@ -60,6 +60,7 @@ def parse():
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-merge", action="store_true",
                    help="headline run with DBC_FLAG_NO_MERGE (one job per (root, insertion))")
+    p.add_argument("--no-deletions", action="store_true", help="skip the edge-deletion side measurement")
     p.add_argument("--no-per-insertion", action="store_true",
                    help="skip the side measurement with DBC_FLAG_NO_MERGE")
     p.add_argument("--no-cpu-baseline", action="store_true")
@@ -383,6 +384,23 @@ def run_ours(args):
             cpu = {"value": None, "unit": "insertions/s", "cores": 1, "kind": "oracle",
                    "sample": f"unavailable: {ex}"}
 
+    # side measurement: deletions (decremental update, R20) -- the
+    # edges of the timed batches deleted again, B per step, one job per deletion
+    dels = None
+    if not args.no_deletions:
+        barrier()
+        torch.cuda.synchronize()
+        ev0.record(stream)
+        for i in range(Wm + K - 1, Wm - 1, -1):
+            dbc.delete_edges(wl.ins_u[i * B:(i + 1) * B], wl.ins_v[i * B:(i + 1) * B])
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        msd = max_over_ranks(ev0.elapsed_time(ev1))
+        dels = {"value": K * B / (msd / 1e3), "unit": "deletions/s", "ms_per_step": msd / K,
+                "what": "the K timed batches deleted again (B per step, newest first), one job per "
+                        "(root, deletion); host-side batch checks inside the timed region"}
+
     # side measurement: the same batches with one job per (root, insertion)
     # (DBC_FLAG_NO_MERGE: the paper's one-insertion-at-a-time structure)
     per_ins = None
@@ -446,6 +464,7 @@ def run_ours(args):
             "merge": ("one job per (root, insertion)" if args.no_merge or args.mode == "S" else
                       "window-merged: one job per root per window of insertions (DESIGN.md R18)"),
             "per_insertion_jobs": per_ins,
+            "deletions": dels,
         },
         "roofline": {
             "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",

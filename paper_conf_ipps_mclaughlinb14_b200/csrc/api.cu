@@ -34,6 +34,7 @@ struct dbc_ctx {
     int workers = 0;
     int block = 512;   // threads per update worker CTA (512, 256 or 128)
     bool ub2 = false;  // 512-thread CTAs built for two per SM (update_512x2)
+    bool lowdeg = false;  // max degree <= 32 (mesh-like graphs)
     int sblock = 256, sworkers = 0;  // static kernel: its own CTA width and grid
     size_t nscratch = 0;             // worker scratch sets allocated
     // heavy lanes: the slowest root chains of the previous batch run on
@@ -406,23 +407,31 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     int64_t maxdeg = 0;
     for (int32_t v = 0; v < n; ++v) maxdeg = std::max<int64_t>(maxdeg, row_ptr[v + 1] - row_ptr[v]);
     c->sblock = (c->k_loc > 2 * c->nsm && maxdeg <= 256) ? 128 : 256;  // hubs need the wide CTA
+    c->lowdeg = maxdeg <= 32;  // every row walked by one lane: no chunked up levels
     c->block = 512;
-    if (const char *eb = getenv("DBC_BLOCK")) c->block = atoi(eb) == 128 ? 128 : (atoi(eb) == 256 ? 256 : 512);
+    if (const char *eb = getenv("DBC_BLOCK"))
+        c->block = atoi(eb) == 128 ? 128 : (atoi(eb) == 256 ? 256 : (atoi(eb) == 1024 ? 1024 : 512));
     // Many roots per SM (>= 3 x #SMs): two register-capped 512-thread CTAs per
     // SM keep more root chains in flight (Delaunay 2^18 / 512 roots: +29%,
     // Kronecker 20 / 1024 roots: +3%); fewer roots: one 128-register CTA.
     c->ub2 = c->block == 512 && c->k_loc >= 3 * c->nsm;
     if (const char *e = getenv("DBC_UB2")) c->ub2 = c->block == 512 && atoi(e) != 0;
-    int upb = c->block == 128 ? 4 : (c->block == 512 ? (c->ub2 ? 2 : 1) : 2);  // update CTAs per SM
+    int upb = c->block == 128 ? 4 : (c->block >= 512 ? (c->ub2 ? 2 : 1) : 2);  // update CTAs per SM
     int want = opt.workers ? opt.workers : upb * c->nsm;
     want = std::min(want, c->k_loc);
     int fit = (int)std::min<size_t>(budget / per_worker, 1 << 20);
     c->workers = std::max(0, std::min(want, fit));
     c->sworkers = std::max(0, std::min({opt.workers ? opt.workers : (c->sblock == 128 ? 4 : 2) * c->nsm,
                                         c->k_loc, fit}));
-    c->hblock = c->block == 128 ? 256 : 512;
+    c->hblock = c->block == 128 ? 256 : (c->block == 256 ? 512 : 1024);
     // only hub-heavy graphs (256-thread build) have step-bound slow roots
-    c->heavy_cap = (c->block != 256 || opt.workers) ? 0 : std::max(0, std::min(c->nsm / 4, (int)(fit - c->workers)));
+    // heavy lanes: the slowest root chains of the previous batch on 2x-wide CTAs
+    // (hub-heavy graphs with fewer roots than worker slots: the batch time is the
+    // slowest chain); 512-thread builds use 1024-thread heavy CTAs
+    c->heavy_cap = (c->block == 128 || c->block == 1024 || c->ub2 || opt.workers) ? 0
+                   : std::max(0, std::min(c->block == 512 ? c->nsm / 8 : c->nsm / 4, (int)(fit - c->workers)));
+    if (const char *e = getenv("DBC_HEAVY_CAP"))
+        if (c->block != 1024) c->heavy_cap = std::max(0, std::min(atoi(e), (int)(fit - c->workers)));
     if (getenv("DBC_NO_HEAVY")) c->heavy_cap = 0;
     if (c->k_loc > 0 && c->workers == 0) {
         fail(c, DBC_ENOMEM, "not enough device memory for one worker (%zu bytes)", per_worker);
@@ -486,6 +495,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->help.gapp, nwk);
     AL(c->help.gU, wn);
     AL(c->help.roots_left, 1);
+    AL(c->help.low, nwk);
     c->help.nworkers = (int)nwk;
     if (const char *e = getenv("DBC_NO_HELP")) c->help_on = atoi(e) == 0;
     AL(c->next_slot, 2);
@@ -692,6 +702,7 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     a.merge = (c->flags & DBC_FLAG_NO_MERGE) ? 0 : 1;
     a.scen = nullptr;
     a.del = 0;
+    a.lowdeg = c->lowdeg && !getenv("DBC_NO_LOWDEG");
     if (c->scen_cap > 0) {  // Fig. 2 / Fig. 4 log: one job per (root, insertion)
         if (cnt > c->scen_cap)
             return fail(c, DBC_EINVAL, "batch of %lld exceeds the scenario log (%lld insertions)",
@@ -744,7 +755,9 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
                 std::vector<double> srt(c->root_ms);
                 std::nth_element(srt.begin(), srt.begin() + k / 2, srt.end());
                 const double med = srt[k / 2];
-                while (nh < c->heavy_cap && nh < k - 1 && c->root_ms[order[nh]] > 1.3 * med) ++nh;
+                double hf = c->block == 512 ? 1.8 : 1.3;  // "slow" = this many medians
+                if (const char *e = getenv("DBC_HEAVY_FACTOR")) hf = atof(e);
+                while (nh < c->heavy_cap && nh < k - 1 && c->root_ms[order[nh]] > hf * med) ++nh;
             }
             // slot list: normal slots (longest first), then the heavy ones
             std::vector<int32_t> list;
@@ -771,7 +784,9 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
                 h.slot_count = nh;
                 h.worker_base = c->workers;
                 h.next_slot = c->next_slot + 1;
-                if (c->hblock == 512)
+                if (c->hblock == 1024)
+                    launch_update_1024(h, nh, c->hstream);
+                else if (c->hblock == 512)
                     launch_update_512(h, nh, c->hstream);
                 else
                     launch_update_256(h, nh, c->hstream);
@@ -785,6 +800,8 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
                 launch_update_128(a, wl, c->stream);
             else if (c->block == 512)
                 (c->ub2 ? launch_update_512x2 : launch_update_512)(a, wl, c->stream);
+            else if (c->block == 1024)
+                launch_update_1024(a, wl, c->stream);
             else
                 launch_update_256(a, wl, c->stream);
             ++ulaunch;
@@ -800,6 +817,8 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
                     launch_update_128(a, c->workers, c->stream);
                 else if (c->block == 512)
                     (c->ub2 ? launch_update_512x2 : launch_update_512)(a, c->workers, c->stream);
+                else if (c->block == 1024)
+                    launch_update_1024(a, c->workers, c->stream);
                 else
                     launch_update_256(a, c->workers, c->stream);
                 ++ulaunch;
@@ -939,6 +958,7 @@ static dbc_status delete_host_ids(dbc_ctx *c, const int32_t *u, const int32_t *v
     a.help = HelpBoard{};
     a.merge = 0;
     a.del = 1;
+    a.lowdeg = c->lowdeg && !getenv("DBC_NO_LOWDEG");
     a.scen = nullptr;
     if (c->scen_cap > 0) {
         if (cnt > c->scen_cap)
@@ -960,6 +980,8 @@ static dbc_status delete_host_ids(dbc_ctx *c, const int32_t *u, const int32_t *v
                 launch_update_128(a, c->workers, c->stream);
             else if (c->block == 512)
                 (c->ub2 ? launch_update_512x2 : launch_update_512)(a, c->workers, c->stream);
+            else if (c->block == 1024)
+                launch_update_1024(a, c->workers, c->stream);
             else
                 launch_update_256(a, c->workers, c->stream);
             ++ulaunch;

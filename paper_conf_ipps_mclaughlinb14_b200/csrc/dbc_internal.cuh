@@ -343,7 +343,8 @@ __device__ __forceinline__ void big_entries(BigSmem &S, const GView &g, const Ro
 }
 
 // --- up phase: chunked flattened level pass ----------------------------------
-constexpr int kChunk = kBlock > 512 ? kBlock : 512;  // items per chunk (shared memory)
+constexpr int kChunk = 512;   // items per chunk (shared memory; one layout for every CTA width,
+                              // so owners and helpers of different widths share the help board)
 constexpr int kUcap = 1024;   // up-frontier entries kept in shared memory
 constexpr int kMetaUp = 1, kMetaNotPulled = 2, kMetaMask = 4;
 constexpr int kMetaNew = 8;  // down row with batch entries: its pushes check new_edge()
@@ -365,7 +366,7 @@ struct ChunkSmem {
 __device__ __forceinline__ void chunk_scan(int *off, int cnt) {
     __shared__ int ws[kWarps];
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-    constexpr int per = kChunk / kBlock;  // items per thread
+    constexpr int per = kChunk >= kBlock ? kChunk / kBlock : 1;  // items per thread
     int vals[per];
     int run = 0;
 #pragma unroll
@@ -401,7 +402,8 @@ __device__ __forceinline__ void chunk_scan(int *off, int cnt) {
 // calls f(t, y, d, sd, mark) (sd, mark gathered for want(d)); if acc != nullptr
 // the returned contribution is
 // summed into acc[t].  Ends with a barrier.
-template <bool kCG = false, class Want, class Col, class F>
+// kSd = false: sd is not gathered (f sees zeros), only mark.
+template <bool kCG = false, bool kSd = true, class Want, class Col, class F>
 __device__ __forceinline__ void flat_entries(const int *off, int cnt, int E, Col colf, const Root &st,
                                              const uint32_t *mk, Want want, double *acc, F f, int Ebeg = 0) {
     const int tid = threadIdx.x;
@@ -436,7 +438,7 @@ __device__ __forceinline__ void flat_entries(const int *off, int cnt, int E, Col
 #pragma unroll
         for (int u = 0; u < kFlatU; ++u) {
             const bool w = t[u] >= 0 && want(dy[u]);
-            q[u] = w ? (kCG ? __ldcg(st.sd + y[u]) : st.sd[y[u]]) : make_double2(0.0, 0.0);
+            q[u] = (kSd && w) ? (kCG ? __ldcg(st.sd + y[u]) : st.sd[y[u]]) : make_double2(0.0, 0.0);
             mm[u] = (mk && w) ? (kCG ? __ldcg(mk + y[u]) : mk[y[u]]) : 0u;
         }
 #pragma unroll
@@ -492,6 +494,9 @@ constexpr int kHelpMinBlocks = 3;      // publish only passes of >= 3 blocks
 struct HelpCtx {
     int root_slot, l, g0, lim, cnt, nblocks, E2;  // g0..lim: the job's insertions
     uint32_t E;  // epoch << 2 of the job
+    int kind;    // 0: C2 push pass of a published chunk; 1: a down-phase level
+    int lb;      // kind 1: the level's first position in D
+    int mvalid;  // kind 1: level-2 masks are maintained
 };
 struct HelpBoard {
     unsigned long long *word;  // [workers]
@@ -501,6 +506,7 @@ struct HelpBoard {
     int *gapp;                 // [workers] global append counters
     int32_t *gU;               // [workers][n] global append lists
     int *roots_left;           // [1] root chains not yet finished (both lanes)
+    int *low;                  // [workers] kind 1: a distance was lowered in the helped level
     int nworkers;
 };
 __device__ __forceinline__ unsigned long long help_pack(int open, int nblocks, int next, int seq) {
@@ -538,6 +544,7 @@ struct UpdateArgs {
     int32_t merge;                 // 1: a window of ws.wcap insertions per job; 0: one per insertion
     long long *scen;               // nullable: scenario log [batch insertion][k_loc] (merge == 0)
     int32_t del;                   // 1: ins_u/ins_v[ins_begin] is an edge DELETION (already tombstoned)
+    int32_t lowdeg;                // 1: rows are short: up levels of any size are walked in-lane
 };
 
 struct StaticArgs {
@@ -580,6 +587,7 @@ void launch_edge_update(const EdgeArgs &a, int workers, cudaStream_t s);
 
 void launch_update_256(const UpdateArgs &a, int workers, cudaStream_t s);
 void launch_update_512x2(const UpdateArgs &a, int workers, cudaStream_t s);  // 64 regs, 2 CTAs/SM
+void launch_update_1024(const UpdateArgs &a, int workers, cudaStream_t s);   // heavy lane, 64 regs
 void launch_update_128(const UpdateArgs &a, int workers, cudaStream_t s);
 void launch_update_512(const UpdateArgs &a, int workers, cudaStream_t s);
 void launch_static_256(const StaticArgs &a, int workers, cudaStream_t s);

@@ -60,15 +60,16 @@ __device__ __forceinline__ void help_push_entry(const GView &g, const ChunkSmem 
     if (dp != cx.l - 1) return;
     const uint32_t E = cx.E, mD = E | kDown, mU = E | kUp;
     const int meta = M.meta[t];
-    double dlt;
+    double dlt;  // Ddelta[p] / sigma[p] (the accumulator is sigma-factored)
     if (meta & kMetaUp) {
-        dlt = __dmul_rn(__ddiv_rn(sp, M.c0[t]), M.c1[t]);
+        dlt = __ddiv_rn(M.c1[t], M.c0[t]);
     } else {
         if (mp == mD) return;
-        dlt = __dmul_rn(__ddiv_rn(sp, M.c0[t]), 1.0 + M.acc[t]);
+        dlt = __ddiv_rn(1.0 + M.acc[t], M.c0[t]);
         if ((meta & kMetaNotPulled) && !((meta & kMetaNew) && new_edge(g, M.v[t], pp, cx.g0, cx.lim)))
-            dlt = __dsub_rn(dlt, __dmul_rn(__ddiv_rn(sp, M.c2[t]), 1.0 + M.c1[t]));
+            dlt = __dsub_rn(dlt, __ddiv_rn(1.0 + M.c1[t], M.c2[t]));
     }
+    (void)sp;
     atomicAdd(dacc + pp, dlt);
     bytes += 24;
     if (mp >= E) return;
@@ -83,7 +84,7 @@ __device__ __forceinline__ void help_run_block(const ChunkSmem &M, int e0, int e
                                                const Root &st, uint32_t *mark, double *dacc, int32_t *gU,
                                                int *gapp, const HelpCtx &cx, unsigned long long &bytes) {
     auto colf = [&](int t, int e) { return ldg_i(g.col + M.beg[t] + e - M.off[t]); };
-    flat_entries<kCG>(
+    flat_entries<kCG, false>(
         M.off, cx.cnt, e1, colf, st, mark, [&](int dp) { return dp == cx.l - 1; }, nullptr,
         [&](int t, int pp, int dp, double2 q, uint32_t mp) -> double {
             bytes += 8;
@@ -91,6 +92,169 @@ __device__ __forceinline__ void help_run_block(const ChunkSmem &M, int e0, int e
             return 0.0;
         },
         e0);
+}
+
+// ---------------------------------------------------------------------------
+// One level of the down phase (K3) over items [i0, i1) of the level -- the
+// owner's whole level, or one block of a helped level (owner or helper CTA).
+struct DownCtx {
+    GView g;
+    Root st;
+    uint32_t *mark;
+    unsigned long long *lowrec;
+    int32_t *Dv, *Dold;
+    double *Dsig;
+    uint32_t *mask;   // the root's level-2 predecessor masks
+    int32_t *err;
+    int *dcnt;        // D append counter (shared; global on a helped level)
+    int *lowflag;     // set when a distance is lowered (Case 3)
+    const int *adjs;  // the root's row (bit positions of the masks), dsr entries
+    int dsr, L, lb, lim, mvalid, del;
+    uint32_t epoch, mD;
+};
+constexpr int kDownBlock = 1024;    // items per block of a helped level
+constexpr int kHelpDownMin = 3072;  // levels of at least this many items are published
+
+__device__ __forceinline__ uint32_t dc_l1bit(const DownCtx &c, int y) {
+    for (int j = 0; j < c.dsr; ++j)
+        if (c.adjs[j] == y) return 1u << j;
+    return 0u;
+}
+
+// per-D-entry epilogue: record old d / sigma, store the new sigma (and, at
+// level 2, the vertex's level-1 predecessor mask)
+__device__ __forceinline__ void dc_finish(const DownCtx &c, int idx, int w, double sum, uint32_t m, bool ext,
+                                          unsigned long long &bytes) {
+    if (c.mvalid && c.L == 2) c.mask[w] = m;
+    const unsigned long long lr = c.lowrec[w];
+    const int od = ((uint32_t)(lr >> 32) == c.epoch) ? (int)(uint32_t)lr : c.L;
+    c.Dold[idx] = od | (ext ? kExtPred : 0);
+    c.Dsig[idx] = c.st.sd[w].x;
+    c.st.sd[w].x = sum;
+    if (!(sum <= 1.7976931348623157e308)) atomicOr(c.err, kErrNumeric);
+    bytes += 8 + 8 + 20;
+}
+
+// one neighbour y of a level-L vertex; returns sigma[y] if y is a predecessor
+__device__ __forceinline__ double dc_visit(const DownCtx &c, int y, int dy, double sy, unsigned long long &bytes) {
+    const int L = c.L;
+    if (dy == L - 1) {
+        bytes += 8;
+        return sy;
+    }
+    if (dy > L + 1) {  // Case 3 pull-up
+        const int old = atomicMin(c.st.d + y, L + 1);
+        if (old > L + 1 && !(c.del && (uint32_t)(c.lowrec[y] >> 32) == c.epoch)) {
+            c.lowrec[y] = ((unsigned long long)c.epoch << 32) | (uint32_t)old;
+            *c.lowflag = 1;
+            bytes += 4;
+        }
+        dy = L + 1;
+    }
+    if (dy == L + 1 && atomicMax(c.mark + y, c.mD) < c.mD) c.Dv[atomicAdd(c.dcnt, 1)] = y;
+    return 0.0;
+}
+
+// short rows of items [i0, i1) walked in-lane in canonical order (bit-exact
+// sigma); long rows handed to enq(item)
+template <class Enq>
+__device__ __forceinline__ void dc_small(const DownCtx &c, int i0, int i1, Enq enq, unsigned long long &bytes,
+                                         unsigned long long &scanned) {
+    const int L = c.L, mD = c.mD;
+    for (int i = i0 + (int)threadIdx.x; i < i1; i += kBlock) {
+        const int w = c.Dv[c.lb + i];
+        const int2 r = row_of(c.g, w, c.lim);
+        if (r.y - r.x > kSmallDeg) {
+            enq(i);
+            continue;
+        }
+        double sum = 0.0;  // canonical order: bit-exact
+        uint32_t m = 0u;
+        bool ext = false;
+        for (int j = r.x; j < r.y; j += kRowUnroll) {
+            int y[kRowUnroll], dy[kRowUnroll], om[kRowUnroll];
+            uint32_t oc[kRowUnroll], pm[kRowUnroll];
+            double sy[kRowUnroll];
+#pragma unroll
+            for (int u = 0; u < kRowUnroll; ++u) y[u] = (j + u < r.y) ? ldg_i(c.g.col + j + u) : -1;
+#pragma unroll
+            for (int u = 0; u < kRowUnroll; ++u) dy[u] = (y[u] >= 0) ? c.st.d[y[u]] : kInf;
+#pragma unroll
+            for (int u = 0; u < kRowUnroll; ++u) {
+                const bool pr = y[u] >= 0 && dy[u] == L - 1;
+                sy[u] = pr ? c.st.sd[y[u]].x : 0.0;
+                pm[u] = pr ? c.mark[y[u]] : (uint32_t)mD;
+            }
+            // issue every lowering and claim of the block, then consume
+#pragma unroll
+            for (int u = 0; u < kRowUnroll; ++u)
+                om[u] = (y[u] >= 0 && dy[u] > L + 1) ? atomicMin(c.st.d + y[u], L + 1) : 0;
+#pragma unroll
+            for (int u = 0; u < kRowUnroll; ++u) oc[u] = mD;
+#pragma unroll
+            for (int u = 0; u < kRowUnroll; ++u)
+                if (y[u] >= 0 && dy[u] >= L + 1) oc[u] = atomicMax(c.mark + y[u], (uint32_t)mD);
+#pragma unroll
+            for (int u = 0; u < kRowUnroll; ++u) {
+                if (y[u] < 0) continue;
+                if (dy[u] == L - 1) {  // predecessor: canonical-order sum
+                    sum += sy[u];
+                    ext |= pm[u] != (uint32_t)mD;
+                    bytes += 8;
+                    if (c.mvalid && L == 2) m |= dc_l1bit(c, y[u]);
+                }
+                if (dy[u] > L + 1 && om[u] > L + 1 &&  // first lowerer (Case 3)
+                    !(c.del && (uint32_t)(c.lowrec[y[u]] >> 32) == c.epoch)) {
+                    c.lowrec[y[u]] = ((unsigned long long)c.epoch << 32) | (uint32_t)om[u];
+                    *c.lowflag = 1;
+                    bytes += 4;
+                }
+                if (dy[u] >= L + 1 && oc[u] < (uint32_t)mD) c.Dv[atomicAdd(c.dcnt, 1)] = y[u];
+            }
+        }
+        bytes += 8 + 8ull * (r.y - r.x);
+        scanned += r.y - r.x;
+        dc_finish(c, c.lb + i, w, sum, m, ext, bytes);
+    }
+}
+
+// the long rows queued in Bq[0, nbig) (item indices), kBig per round through
+// S, entries flattened over the CTA.  Caller: barrier before (queue complete);
+// ends with a barrier.
+__device__ __forceinline__ void dc_big(const DownCtx &c, BigSmem &S, const int32_t *Bq, int nbig,
+                                       unsigned long long &bytes, unsigned long long &scanned) {
+    const int tid = threadIdx.x, L = c.L;
+    for (int r0 = 0; r0 < nbig; r0 += kBig) {
+        const int m = min(kBig, nbig - r0);
+        big_load(S, m, [&](int t) { return Bq[r0 + t]; }, [&](int i) { return c.Dv[c.lb + i]; }, c.g, c.lim);
+        if (tid < m) {
+            S.mk[tid] = 0u;
+            S.ext[tid] = 0;
+        }
+        __syncthreads();
+        big_entries(S, c.g, c.st, [&](int dy) { return dy == L - 1; }, [&](int t, int y, int dy, double2 q) {
+            bytes += 8;
+            scanned++;
+            if (c.mvalid && L == 2 && dy == 1) atomicOr(&S.mk[t], dc_l1bit(c, y));
+            if (dy == L - 1 && c.mark[y] != c.mD) S.ext[t] = 1;
+            return dc_visit(c, y, dy, q.x, bytes);
+        });
+        if (tid < m) {
+            double sum = S.acc[tid];
+            const int w = S.v[tid];
+            if (sum >= kExact) {  // order-dependent rounding: canonical sum
+                const int2 r = row_of(c.g, w, c.lim);
+                sum = 0.0;
+                for (int j = r.x; j < r.y; ++j) {
+                    const int y = ldg_i(c.g.col + j);
+                    if (c.st.dist(y) == L - 1) sum += c.st.sd[y].x;
+                }
+            }
+            bytes += 8;
+            dc_finish(c, c.lb + S.idx[tid], w, sum, S.mk[tid], S.ext[tid] != 0, bytes);
+        }
+        __syncthreads();
+    }
 }
 
 __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a) {
@@ -458,135 +622,95 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                 const int le0 = s_dcnt;
                 if (tid == 0) Doff[1] = le0;
                 const bool mvalid = mstate == 1;  // masks usable during this job's down phase
-                // bit of a level-1 vertex in the masks (its position in the root's row)
-                auto l1bit = [&](int y) -> uint32_t {
-                    for (int j = 0; j < dsr; ++j)
-                        if (s_adjs[j] == y) return 1u << j;
-                    return 0u;
-                };
 
                 tick(-1);
                 // ================= down phase (K3) =================
                 int L = L0, lb = 0, le = le0, nlev = 1;
-                // per-D-entry epilogue: record old d / sigma, store the new sigma
-                // (and, at level 2, the vertex's level-1 predecessor mask)
-                auto down_finish = [&](int idx, int w, double sum, uint32_t m, bool ext) {
-                    if (mvalid && L == 2) mask[w] = m;
-                    const unsigned long long lr = lowrec[w];
-                    const int od = ((uint32_t)(lr >> 32) == epoch) ? (int)(uint32_t)lr : L;
-                    Dold[idx] = od | (ext ? kExtPred : 0);
-                    Dsig[idx] = st.sd[w].x;
-                    st.sd[w].x = sum;
-                    if (!(sum <= 1.7976931348623157e308)) atomicOr(a.err, kErrNumeric);
-                    st_bytes += 8 + 8 + 20;
-                };
-                // one neighbour y of a level-L vertex; returns sigma[y] if y is a predecessor
-                auto down_visit = [&](int y, int dy, double sy) -> double {
-                    if (dy == L - 1) {
-                        st_bytes += 8;
-                        return sy;
-                    }
-                    if (dy > L + 1) {  // Case 3 pull-up
-                        const int old = atomicMin(st.d + y, L + 1);
-                        if (old > L + 1 && !(a.del && (uint32_t)(lowrec[y] >> 32) == epoch)) {
-                            lowrec[y] = ((unsigned long long)epoch << 32) | (uint32_t)old;
-                            s_job[3] = 1;
-                            st_bytes += 4;
-                        }
-                        dy = L + 1;
-                    }
-                    if (dy == L + 1 && atomicMax(mark + y, mD) < mD)
-                        Dv[atomicAdd(&s_dcnt, 1)] = y;
-                    return 0.0;
-                };
+                DownCtx dc;
+                dc.g = g;
+                dc.st = st;
+                dc.mark = mark;
+                dc.lowrec = lowrec;
+                dc.Dv = Dv;
+                dc.Dold = Dold;
+                dc.Dsig = Dsig;
+                dc.mask = mask;
+                dc.err = a.err;
+                dc.dcnt = &s_dcnt;
+                dc.lowflag = &s_job[3];
+                dc.adjs = s_adjs;
+                dc.dsr = dsr;
+                dc.lim = lim;
+                dc.mvalid = mvalid;
+                dc.del = a.del;
+                dc.epoch = epoch;
+                dc.mD = mD;
                 while (true) {
-                    split_pass(
-                        le - lb, g, lim, [&](int i, int &w) { w = Dv[lb + i]; return true; },
-                        [&](int i, int w, int2 r) {
-                            double sum = 0.0;  // canonical order: bit-exact
-                            uint32_t m = 0u;
-                            bool ext = false;
-                            for (int j = r.x; j < r.y; j += kRowUnroll) {
-                                int y[kRowUnroll], dy[kRowUnroll], om[kRowUnroll];
-                                uint32_t oc[kRowUnroll], pm[kRowUnroll];
-                                double sy[kRowUnroll];
-#pragma unroll
-                                for (int u = 0; u < kRowUnroll; ++u) y[u] = (j + u < r.y) ? ldg_i(g.col + j + u) : -1;
-#pragma unroll
-                                for (int u = 0; u < kRowUnroll; ++u) dy[u] = (y[u] >= 0) ? st.d[y[u]] : kInf;
-#pragma unroll
-                                for (int u = 0; u < kRowUnroll; ++u) {
-                                    const bool pr = y[u] >= 0 && dy[u] == L - 1;
-                                    sy[u] = pr ? st.sd[y[u]].x : 0.0;
-                                    pm[u] = pr ? mark[y[u]] : mD;
-                                }
-                                // issue every lowering and claim of the block, then consume
-#pragma unroll
-                                for (int u = 0; u < kRowUnroll; ++u)
-                                    om[u] = (y[u] >= 0 && dy[u] > L + 1) ? atomicMin(st.d + y[u], L + 1) : 0;
-#pragma unroll
-                                for (int u = 0; u < kRowUnroll; ++u)
-                                    oc[u] = mD;
-#pragma unroll
-                                for (int u = 0; u < kRowUnroll; ++u)
-                                    if (y[u] >= 0 && dy[u] >= L + 1) oc[u] = atomicMax(mark + y[u], mD);
-#pragma unroll
-                                for (int u = 0; u < kRowUnroll; ++u) {
-                                    if (y[u] < 0) continue;
-                                    if (dy[u] == L - 1) {  // predecessor: canonical-order sum
-                                        sum += sy[u];
-                                        ext |= pm[u] != mD;
-                                        st_bytes += 8;
-                                        if (mvalid && L == 2) m |= l1bit(y[u]);
-                                    }
-                                    if (dy[u] > L + 1 && om[u] > L + 1 &&  // first lowerer (Case 3)
-                                        !(a.del && (uint32_t)(lowrec[y[u]] >> 32) == epoch)) {
-                                        lowrec[y[u]] = ((unsigned long long)epoch << 32) | (uint32_t)om[u];
-                                        s_job[3] = 1;
-                                        st_bytes += 4;
-                                    }
-                                    if (dy[u] >= L + 1 && oc[u] < mD) Dv[atomicAdd(&s_dcnt, 1)] = y[u];
-                                }
+                    dc.L = L;
+                    dc.lb = lb;
+                    const int items = le - lb;
+                    if (a.help.word && items >= kHelpDownMin) {
+                        // a wide level: published, idle workers take blocks of items
+                        // (appends and the lowering flag go through global memory)
+                        const int nblk = (items + kDownBlock - 1) / kDownBlock;
+                        if (tid == 0) {
+                            HelpCtx cx;
+                            cx.root_slot = slot;
+                            cx.l = L;
+                            cx.g0 = g0;
+                            cx.lim = lim;
+                            cx.cnt = items;
+                            cx.nblocks = nblk;
+                            cx.E2 = 0;
+                            cx.E = E;
+                            cx.kind = 1;
+                            cx.lb = lb;
+                            cx.mvalid = mvalid;
+                            a.help.ctx[wk] = cx;
+                            a.help.done[wk] = 0;
+                            a.help.gapp[wk] = s_dcnt;
+                            a.help.low[wk] = 0;
+                            __threadfence();
+                            atomicAdd(a.stats + kStHelpReq, 1ull);
+                            atomicAdd(a.stats + kStHelpBlkAll, (unsigned long long)nblk);
+                            hseq = (hseq + 1) & 0xFFFF;
+                            atomicExch(a.help.word + wk, help_pack(1, nblk, 0, hseq));
+                        }
+                        DownCtx gd = dc;
+                        gd.dcnt = a.help.gapp + wk;
+                        gd.lowflag = a.help.low + wk;
+                        for (;;) {  // the owner takes blocks too
+                            if (tid == 0) {
+                                const unsigned long long w = atomicAdd(a.help.word + wk, 1ull << 16);
+                                s_hb = help_next(w) < nblk ? help_next(w) : -1;
                             }
-                            st_bytes += 8 + 8ull * (r.y - r.x);
-                            sc_down += r.y - r.x;
-                            down_finish(lb + i, w, sum, m, ext);
-                        },
-                        enq_front);
-                    __syncthreads();
-                    const int nbig = s_nbig;
-                    for (int r0 = 0; r0 < nbig; r0 += kBig) {
-                        const int m = min(kBig, nbig - r0);
-                        big_load(S, m, [&](int t) { return Bq[r0 + t]; }, [&](int i) { return Dv[lb + i]; },
-                                 g, lim);
-                        if (tid < m) {
-                            S.mk[tid] = 0u;
-                            S.ext[tid] = 0;
+                            __syncthreads();
+                            const int b = s_hb;
+                            __syncthreads();
+                            if (b < 0) break;
+                            dc_small(gd, b * kDownBlock, min(items, (b + 1) * kDownBlock), enq_front, st_bytes,
+                                     sc_down);
+                            __syncthreads();
+                            dc_big(gd, S, Bq, s_nbig, st_bytes, sc_down);
+                            if (tid == 0) {
+                                s_nbig = 0;
+                                __threadfence();
+                                atomicAdd(a.help.done + wk, 1);
+                            }
+                            __syncthreads();
+                        }
+                        if (tid == 0) {  // wait for the helpers' blocks, then close
+                            while (atomicAdd(a.help.done + wk, 0) < nblk) __nanosleep(256);
+                            atomicExch(a.help.word + wk, help_pack(0, 0, 0, hseq));
+                            __threadfence();
+                            s_dcnt = __ldcg(a.help.gapp + wk);
+                            if (__ldcg(a.help.low + wk)) s_job[3] = 1;
                         }
                         __syncthreads();
-                        big_entries(S, g, st, [&](int dy) { return dy == L - 1; },
-                                    [&](int t, int y, int dy, double2 q) {
-                                        st_bytes += 8;
-                                        sc_down++;
-                                        if (mvalid && L == 2 && dy == 1) atomicOr(&S.mk[t], l1bit(y));
-                                        if (dy == L - 1 && mark[y] != mD) S.ext[t] = 1;
-                                        return down_visit(y, dy, q.x);
-                                    });
-                        if (tid < m) {
-                            double sum = S.acc[tid];
-                            const int w = S.v[tid];
-                            if (sum >= kExact) {  // order-dependent rounding: canonical sum
-                                const int2 r = row_of(g, w, lim);
-                                sum = 0.0;
-                                for (int j = r.x; j < r.y; ++j) {
-                                    const int y = ldg_i(g.col + j);
-                                    if (st.dist(y) == L - 1) sum += st.sd[y].x;
-                                }
-                            }
-                            st_bytes += 8;
-                            down_finish(lb + S.idx[tid], w, sum, S.mk[tid], S.ext[tid] != 0);
-                        }
+                    } else {
+                        dc_small(dc, 0, items, enq_front, st_bytes, sc_down);
                         __syncthreads();
+                        dc_big(dc, S, Bq, s_nbig, st_bytes, sc_down);
                     }
                     if (L < Lseed) {  // seeds of the next level (claimed children stay once)
                         inject(L + 1);
@@ -639,7 +763,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                         const int uh = s_del[0];
                         const int dh = st.d[uh];
                         if (dh >= 1) {  // the root's delta is never used
-                            atomicAdd(dacc + uh, -__dmul_rn(__ddiv_rn(st.sd[uh].x, s_delsd[0]), 1.0 + s_delsd[1]));
+                            atomicAdd(dacc + uh, -__ddiv_rn(1.0 + s_delsd[1], s_delsd[0]));
                             if (atomicMax(mark + uh, mU) < E) {
                                 const int pos = atomicAdd(&s_rcnt, 1);
                                 Rv[pos] = uh;
@@ -660,7 +784,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                         if (dx != od - 1) return;
                         if (mark[x] == mD) return;
                         if (ldg_i(g.rp + w) < 0 && new_edge(g, w, x, g0, lim)) return;  // not an old predecessor
-                        atomicAdd(dacc + x, -__dmul_rn(__ddiv_rn(sx, osig), coef));
+                        atomicAdd(dacc + x, -__ddiv_rn(coef, osig));
+                        (void)sx;
                         st_bytes += 24;
                         if (atomicMax(mark + x, mU) < E) {
                             const int pos = atomicAdd(&s_rcnt, 1);
@@ -742,7 +867,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                     };
                     // up vertex x (not in D): push sigma[p]/sigma[x] * Ddelta[x] upwards
                     auto up_visit = [&](double gx, double sx, int pp, double sp, uint32_t mp) {
-                        atomicAdd(dacc + pp, __dmul_rn(__ddiv_rn(sp, sx), gx));
+                        (void)sp;
+                        atomicAdd(dacc + pp, __ddiv_rn(gx, sx));
                         st_bytes += 24;
                         claim_up(pp, mp);
                     };
@@ -761,9 +887,10 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                     auto dpush_visit = [&](int x, double sx, double dn, double odel, double osig,
                                            int meta, int pp, double sp, uint32_t mp) {
                         if (mp == mD) return;
-                        double dlt = __dmul_rn(__ddiv_rn(sp, sx), 1.0 + dn);
+                        (void)sp;
+                        double dlt = __ddiv_rn(1.0 + dn, sx);
                         if ((meta & kMetaNotPulled) && !((meta & kMetaNew) && new_edge(g, x, pp, g0, lim)))
-                            dlt = __dsub_rn(dlt, __dmul_rn(__ddiv_rn(sp, osig), 1.0 + odel));
+                            dlt = __dsub_rn(dlt, __ddiv_rn(1.0 + odel, osig));
                         atomicAdd(dacc + pp, dlt);
                         st_bytes += 24;
                         claim_up(pp, mp);
@@ -825,9 +952,10 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                         if (x < 0) return false;
                         // the dedup claim and the loads are issued together
                         const uint32_t prev = atomicMax(mark + x, E | kUpDone);
-                        const double gx = __ldcg(dacc + x);  // Ddelta (complete; helpers add via L2)
+                        const double gxs = __ldcg(dacc + x);  // Ddelta / sigma (complete; helpers add via L2)
                         const double2 s2 = st.sd[x];
                         const double sx = s2.x, odl = s2.y;
+                        const double gx = __dmul_rn(sx, gxs);
                         const bool usemask = l == 2 && mok;  // level-1 predecessors from the mask
                         const int2 rr = (push && !usemask) ? row_of(g, x, lim) : make_int2(0, 0);
                         mk = usemask ? mask[x] : 0u;
@@ -846,15 +974,15 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                         if (meta & kMetaMask) {  // level 2: predecessors = set bits (root's row order)
                             for (uint32_t b = mk; b; b &= b - 1) {
                                 const int pp = s_adjs[__ffs(b) - 1];
-                                up_visit(c1, c0, pp, st.sd[pp].x, mark[pp]);
+                                up_visit(c1, c0, pp, 0.0, mark[pp]);
                             }
                             up_finish(x, c1, c2);
                         } else if (meta & kMetaUp) {
                             if (wantpush) {
+                                const double wx = __ddiv_rn(c1, c0);  // Ddelta[x] / sigma[x]
                                 for (int j = r.x; j < r.y; j += kRowUnroll) {
                                     int y[kRowUnroll], dy[kRowUnroll];
                                     uint32_t mp[kRowUnroll], oc[kRowUnroll];
-                                    double sp[kRowUnroll];
 #pragma unroll
                                     for (int u = 0; u < kRowUnroll; ++u)
                                         y[u] = (j + u < r.y) ? ldg_i(g.col + j + u) : -1;
@@ -863,13 +991,12 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
 #pragma unroll
                                     for (int u = 0; u < kRowUnroll; ++u) {
                                         const bool pr = y[u] >= 0 && dy[u] == l - 1;
-                                        sp[u] = pr ? st.sd[y[u]].x : 0.0;
                                         mp[u] = pr ? mark[y[u]] : 0xffffffffu;
                                     }
 #pragma unroll
                                     for (int u = 0; u < kRowUnroll; ++u)
                                         if (y[u] >= 0 && dy[u] == l - 1) {
-                                            atomicAdd(dacc + y[u], __dmul_rn(__ddiv_rn(sp[u], c0), c1));
+                                            atomicAdd(dacc + y[u], wx);
                                             st_bytes += 24;
                                         }
 #pragma unroll
@@ -949,7 +1076,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                     // small levels (<= one item per thread): short rows in-lane;
                     // large levels: every row through the flattened pass, in chunks
                     const int total = nDl + ucnt + rcnt;
-                    const bool small_level = total <= kBlock;
+                    const bool small_level = total <= kBlock || a.lowdeg;
                     const int step = small_level ? total : kChunk;
                     bool first_barrier = true;
                     for (int cb = 0; cb < total; cb += step) {
@@ -1025,15 +1152,18 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                 cx.nblocks = nblk;
                                 cx.E2 = E2;
                                 cx.E = E;
+                                cx.kind = 0;
+                                cx.lb = 0;
+                                cx.mvalid = 0;
                                 if (tid == 0) {
                                     mir->off[0] = 0;
                                     a.help.ctx[wk] = cx;
                                     a.help.done[wk] = 0;
                                     a.help.gapp[wk] = 0;
                                 }
-                                __threadfence();
-                                __syncthreads();
+                                __syncthreads();  // the chunk is written; one release fence publishes it
                                 if (tid == 0) {
+                                    __threadfence();
                                     atomicAdd(a.stats + kStHelpReq, 1ull);
                                     atomicAdd(a.stats + kStHelpBlkAll, (unsigned long long)nblk);
                                     hseq = (hseq + 1) & 0xFFFF;
@@ -1052,9 +1182,11 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                     if (b < 0) break;
                                     help_run_block<false>(I, b * kHelpEntries, min(E2, (b + 1) * kHelpEntries), g,
                                                           st, mark, dacc, gU, gapp, cx, st_bytes);
-                                    __threadfence();
-                                    __syncthreads();
-                                    if (tid == 0) atomicAdd(a.help.done + wk, 1);
+                                    __syncthreads();  // (help_run_block ends with one too)
+                                    if (tid == 0) {   // release by one thread after the CTA barrier
+                                        __threadfence();
+                                        atomicAdd(a.help.done + wk, 1);
+                                    }
                                 }
                                 if (tid == 0) {  // wait for the helpers' blocks, then close
                                     while (atomicAdd(a.help.done + wk, 0) < nblk) __nanosleep(256);
@@ -1073,7 +1205,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                 }
                                 __syncthreads();
                             } else if (push && E2 > 0)
-                                flat_entries(
+                                flat_entries<false, false>(  // pushes need no sigma of the target
                                     I.off, nb, E2, colf, st, mark, [&](int dp) { return dp == l - 1; }, nullptr,
                                     [&](int t, int pp, int dp, double2 q, uint32_t mp) -> double {
                                         const double sp = q.x;
@@ -1118,7 +1250,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                     const double w = s_l1acc[j];
                                     if (w != 0.0) {
                                         const int pp = s_adjs[j];
-                                        atomicAdd(dacc + pp, __dmul_rn(st.sd[pp].x, w));
+                                        atomicAdd(dacc + pp, w);
                                         st_bytes += 24;
                                         claim_up(pp, mark[pp]);
                                     }
@@ -1227,10 +1359,20 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                     s_hctx.nblocks = __ldcg(&src->nblocks);
                     s_hctx.E2 = __ldcg(&src->E2);
                     s_hctx.E = __ldcg(&src->E);
+                    s_hctx.kind = __ldcg(&src->kind);
+                    s_hctx.lb = __ldcg(&src->lb);
+                    s_hctx.mvalid = __ldcg(&src->mvalid);
+                    __threadfence();  // acquire: drop stale L1 lines of the owner's state
                 }
                 __syncthreads();
                 const ChunkSmem *mir = a.help.mir + pick;
-                const int cnt = s_hctx.cnt;
+                const int cnt = s_hctx.kind == 0 ? s_hctx.cnt : 0;
+                if (s_hctx.kind == 1 && s_hctx.mvalid && tid < 32) {  // the root's row (mask bits)
+                    const int2 rs = row_of(g, a.roots[s_hctx.root_slot], s_hctx.lim);
+                    const int ds = rs.y - rs.x;
+                    if (tid < ds && ds <= kMaskDeg) s_adjs[tid] = ldg_i(g.col + rs.x + tid);
+                    if (tid == 0) s_job[5] = ds;
+                }
                 for (int t = tid; t < cnt; t += kBlock) {
                     I.v[t] = __ldcg(&mir->v[t]);
                     I.meta[t] = __ldcg(&mir->meta[t]);
@@ -1248,12 +1390,42 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
             }
             const HelpCtx cx = s_hctx;
             const Root ost{a.d + (size_t)cx.root_slot * n, a.sd + (size_t)cx.root_slot * n};
-            help_run_block<true>(I, b * kHelpEntries, min(cx.E2, (b + 1) * kHelpEntries), g, ost,
-                                 a.ws.mark + (size_t)pick * n, a.ws.dacc + (size_t)pick * n,
-                                 a.help.gU + (size_t)pick * n, a.help.gapp + pick, cx, st_bytes);
-            __threadfence();
+            if (cx.kind == 1) {  // a block of a published down-phase level
+                DownCtx hd;
+                hd.g = g;
+                hd.st = ost;
+                hd.mark = a.ws.mark + (size_t)pick * n;
+                hd.lowrec = a.ws.lowrec + (size_t)pick * n;
+                hd.Dv = a.ws.Dv + (size_t)pick * n;
+                hd.Dold = a.ws.Dold + (size_t)pick * n;
+                hd.Dsig = a.ws.Dsig + (size_t)pick * n;
+                hd.mask = a.l2mask + (size_t)cx.root_slot * n;
+                hd.err = a.err;
+                hd.dcnt = a.help.gapp + pick;
+                hd.lowflag = a.help.low + pick;
+                hd.adjs = s_adjs;
+                hd.dsr = s_job[5];
+                hd.L = cx.l;
+                hd.lb = cx.lb;
+                hd.lim = cx.lim;
+                hd.mvalid = cx.mvalid;
+                hd.del = a.del;
+                hd.epoch = cx.E >> 2;
+                hd.mD = cx.E | kDown;
+                int32_t *Bqh = a.ws.Bq + (size_t)wk * n;
+                dc_small(hd, b * kDownBlock, min(cx.cnt, (b + 1) * kDownBlock),
+                         [&](int idx) { Bqh[atomicAdd(&s_nbig, 1)] = idx; }, st_bytes, sc_down);
+                __syncthreads();
+                dc_big(hd, S, Bqh, s_nbig, st_bytes, sc_down);
+                if (tid == 0) s_nbig = 0;
+            } else {
+                help_run_block<true>(I, b * kHelpEntries, min(cx.E2, (b + 1) * kHelpEntries), g, ost,
+                                     a.ws.mark + (size_t)pick * n, a.ws.dacc + (size_t)pick * n,
+                                     a.help.gU + (size_t)pick * n, a.help.gapp + pick, cx, st_bytes);
+            }
             __syncthreads();
-            if (tid == 0) {
+            if (tid == 0) {  // release by one thread after the CTA barrier
+                __threadfence();
                 atomicAdd(a.help.done + pick, 1);
                 atomicAdd(a.stats + kStHelpBlk, 1ull);
             }

@@ -333,10 +333,13 @@ def test_block128_kernels_match_oracle(name, monkeypatch):
         check_all(dbc, ref.compute(), wl.roots.size)
 
 
-def test_heavy_lane_batches_match_oracle(monkeypatch):
+@pytest.mark.parametrize("block", ["256", "512"])
+def test_heavy_lane_batches_match_oracle(monkeypatch, block):
     """Several Mode-A batches so the adaptive heavy lane (2x-wide CTAs for the
-    slowest roots of the previous batch; 256-thread build) is exercised; d/sigma bit-exact."""
-    monkeypatch.setenv("DBC_BLOCK", "256")
+    slowest roots of the previous batch: 512 threads beside the 256-thread
+    build, 1024 beside the 512-thread one) is exercised; d/sigma bit-exact."""
+    monkeypatch.setenv("DBC_BLOCK", block)
+    monkeypatch.setenv("DBC_HEAVY_FACTOR", "1.0")  # any root slower than the median
     monkeypatch.setenv("DBC_WINDOW", "8")  # several jobs per root and batch
     wl = W.make_workload("rmat10", insertions=120)
     ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
