@@ -35,6 +35,7 @@ struct dbc_ctx {
     int block = 512;   // threads per update worker CTA (512, 256 or 128)
     bool ub2 = false;  // 512-thread CTAs built for two per SM (update_512x2)
     bool lowdeg = false;  // max degree <= 32 (mesh-like graphs)
+    int hd_min = 1024, hd_block = 512;  // helped down levels (update.cu)
     int sblock = 256, sworkers = 0;  // static kernel: its own CTA width and grid
     size_t nscratch = 0;             // worker scratch sets allocated
     // heavy lanes: the slowest root chains of the previous batch run on
@@ -408,6 +409,8 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     for (int32_t v = 0; v < n; ++v) maxdeg = std::max<int64_t>(maxdeg, row_ptr[v + 1] - row_ptr[v]);
     c->sblock = (c->k_loc > 2 * c->nsm && maxdeg <= 256) ? 128 : 256;  // hubs need the wide CTA
     c->lowdeg = maxdeg <= 32;  // every row walked by one lane: no chunked up levels
+    if (const char *e = getenv("DBC_HDMIN")) c->hd_min = std::max(1, atoi(e));
+    if (const char *e = getenv("DBC_HDBLK")) c->hd_block = std::max(32, atoi(e));
     c->block = 512;
     if (const char *eb = getenv("DBC_BLOCK"))
         c->block = atoi(eb) == 128 ? 128 : (atoi(eb) == 256 ? 256 : (atoi(eb) == 1024 ? 1024 : 512));
@@ -702,6 +705,8 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     a.merge = (c->flags & DBC_FLAG_NO_MERGE) ? 0 : 1;
     a.scen = nullptr;
     a.del = 0;
+    a.hd_min = c->hd_min;
+    a.hd_block = c->hd_block;
     a.lowdeg = c->lowdeg && !getenv("DBC_NO_LOWDEG");
     if (c->scen_cap > 0) {  // Fig. 2 / Fig. 4 log: one job per (root, insertion)
         if (cnt > c->scen_cap)
@@ -958,6 +963,8 @@ static dbc_status delete_host_ids(dbc_ctx *c, const int32_t *u, const int32_t *v
     a.help = HelpBoard{};
     a.merge = 0;
     a.del = 1;
+    a.hd_min = c->hd_min;
+    a.hd_block = c->hd_block;
     a.lowdeg = c->lowdeg && !getenv("DBC_NO_LOWDEG");
     a.scen = nullptr;
     if (c->scen_cap > 0) {

@@ -545,6 +545,7 @@ struct UpdateArgs {
     long long *scen;               // nullable: scenario log [batch insertion][k_loc] (merge == 0)
     int32_t del;                   // 1: ins_u/ins_v[ins_begin] is an edge DELETION (already tombstoned)
     int32_t lowdeg;                // 1: rows are short: up levels of any size are walked in-lane
+    int32_t hd_min, hd_block;      // down levels of >= hd_min items are published in hd_block blocks
 };
 
 struct StaticArgs {

@@ -112,8 +112,7 @@ struct DownCtx {
     int dsr, L, lb, lim, mvalid, del;
     uint32_t epoch, mD;
 };
-constexpr int kDownBlock = 1024;    // items per block of a helped level
-constexpr int kHelpDownMin = 3072;  // levels of at least this many items are published
+// helped down levels: UpdateArgs.hd_min items at least, hd_block items per block
 
 __device__ __forceinline__ uint32_t dc_l1bit(const DownCtx &c, int y) {
     for (int j = 0; j < c.dsr; ++j)
@@ -649,7 +648,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                     dc.L = L;
                     dc.lb = lb;
                     const int items = le - lb;
-                    if (a.help.word && items >= kHelpDownMin) {
+                    const int kDownBlock = a.hd_block;
+                    if (a.help.word && items >= a.hd_min) {
                         // a wide level: published, idle workers take blocks of items
                         // (appends and the lowering flag go through global memory)
                         const int nblk = (items + kDownBlock - 1) / kDownBlock;
@@ -1101,13 +1101,75 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                             auto colf = [&](int t, int e) { return ldg_i(g.col + I.beg[t] + e - I.off[t]); };
                             // --- C1: delta pull of the long down rows (Eq. (2)) ---
                             const int E1 = I.off[nDb];
-                            if (E1 > 0)
-                                flat_entries(I.off, nb, E1, colf, st, nullptr, [&](int dy) { return dy == l + 1; },
+                            auto c1_pass = [&](int e0, int e1) {
+                                flat_entries(I.off, nb, e1, colf, st, nullptr, [&](int dy) { return dy == l + 1; },
                                              I.acc, [&](int t, int, int dy, double2 q, uint32_t) {
                                                  sc_dpull++;
                                                  st_bytes += 8;
                                                  return dpull_visit(I.c0[t], dy, q.x, q.y);
-                                             });
+                                             }, e0);
+                            };
+                            const int nblk1 = (E1 + kHelpEntries - 1) / kHelpEntries;
+                            if (E1 > 0 && a.help.word && nblk1 >= kHelpMinBlocks) {
+                                // publish the pull rows; helpers add per-row partial sums
+                                // into the mirror's acc (delta: rounding order is free)
+                                ChunkSmem *mir = a.help.mir + wk;
+                                for (int t = tid; t < nDb; t += kBlock) {
+                                    mir->v[t] = I.v[t];
+                                    mir->meta[t] = I.meta[t];
+                                    mir->beg[t] = I.beg[t];
+                                    mir->off[t + 1] = I.off[t + 1];
+                                    mir->acc[t] = 0.0;
+                                    mir->c0[t] = I.c0[t];
+                                }
+                                if (tid == 0) {
+                                    HelpCtx cx;
+                                    cx.root_slot = slot;
+                                    cx.l = l;
+                                    cx.g0 = g0;
+                                    cx.lim = lim;
+                                    cx.cnt = nDb;
+                                    cx.nblocks = nblk1;
+                                    cx.E2 = E1;
+                                    cx.E = E;
+                                    cx.kind = 2;
+                                    cx.lb = 0;
+                                    cx.mvalid = 0;
+                                    mir->off[0] = 0;
+                                    a.help.ctx[wk] = cx;
+                                    a.help.done[wk] = 0;
+                                }
+                                __syncthreads();
+                                if (tid == 0) {
+                                    __threadfence();
+                                    atomicAdd(a.stats + kStHelpReq, 1ull);
+                                    atomicAdd(a.stats + kStHelpBlkAll, (unsigned long long)nblk1);
+                                    hseq = (hseq + 1) & 0xFFFF;
+                                    atomicExch(a.help.word + wk, help_pack(1, nblk1, 0, hseq));
+                                }
+                                for (;;) {  // the owner takes blocks too
+                                    if (tid == 0) {
+                                        const unsigned long long w = atomicAdd(a.help.word + wk, 1ull << 16);
+                                        s_hb = help_next(w) < nblk1 ? help_next(w) : -1;
+                                    }
+                                    __syncthreads();
+                                    const int b = s_hb;
+                                    __syncthreads();
+                                    if (b < 0) break;
+                                    c1_pass(b * kHelpEntries, min(E1, (b + 1) * kHelpEntries));  // ends with a barrier
+                                    if (tid == 0) atomicAdd(a.help.done + wk, 1);
+                                }
+                                if (tid == 0) {  // wait for the helpers' blocks, then close
+                                    while (atomicAdd(a.help.done + wk, 0) < nblk1) __nanosleep(256);
+                                    atomicExch(a.help.word + wk, help_pack(0, 0, 0, hseq));
+                                    __threadfence();
+                                }
+                                __syncthreads();
+                                for (int t = tid; t < nDb; t += kBlock) I.acc[t] += __ldcg(&mir->acc[t]);
+                                __syncthreads();
+                            } else if (E1 > 0) {
+                                c1_pass(0, E1);
+                            }
                             tick(8);
                             // --- C2: pushes towards level l-1 (down rows only if they have a
                             // predecessor outside D: drop the others from the offsets) ---
@@ -1366,7 +1428,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                 }
                 __syncthreads();
                 const ChunkSmem *mir = a.help.mir + pick;
-                const int cnt = s_hctx.kind == 0 ? s_hctx.cnt : 0;
+                const int cnt = s_hctx.kind != 1 ? s_hctx.cnt : 0;  // kinds 0 and 2 publish a chunk
                 if (s_hctx.kind == 1 && s_hctx.mvalid && tid < 32) {  // the root's row (mask bits)
                     const int2 rs = row_of(g, a.roots[s_hctx.root_slot], s_hctx.lim);
                     const int ds = rs.y - rs.x;
@@ -1391,6 +1453,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
             const HelpCtx cx = s_hctx;
             const Root ost{a.d + (size_t)cx.root_slot * n, a.sd + (size_t)cx.root_slot * n};
             if (cx.kind == 1) {  // a block of a published down-phase level
+                const int kDownBlock = a.hd_block;
                 DownCtx hd;
                 hd.g = g;
                 hd.st = ost;
@@ -1418,6 +1481,20 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                 __syncthreads();
                 dc_big(hd, S, Bqh, s_nbig, st_bytes, sc_down);
                 if (tid == 0) s_nbig = 0;
+            } else if (cx.kind == 2) {  // a block of a published delta-pull pass (C1)
+                const int e0 = b * kHelpEntries, e1 = min(cx.E2, (b + 1) * kHelpEntries);
+                for (int t = tid; t < cx.cnt; t += kBlock) I.acc[t] = 0.0;
+                __syncthreads();
+                auto colf = [&](int t, int e) { return ldg_i(g.col + I.beg[t] + e - I.off[t]); };
+                flat_entries<true>(I.off, cx.cnt, e1, colf, ost, nullptr, [&](int dy) { return dy == cx.l + 1; },
+                                   I.acc, [&](int t, int, int dy, double2 q, uint32_t) -> double {
+                                       st_bytes += 8;
+                                       if (dy != cx.l + 1) return 0.0;
+                                       return __dmul_rn(__ddiv_rn(I.c0[t], q.x), __dadd_rn(1.0, q.y));
+                                   }, e0);
+                ChunkSmem *mir = a.help.mir + pick;
+                for (int t = tid; t < cx.cnt; t += kBlock)
+                    if (I.acc[t] != 0.0) atomicAdd(&mir->acc[t], I.acc[t]);
             } else {
                 help_run_block<true>(I, b * kHelpEntries, min(cx.E2, (b + 1) * kHelpEntries), g, ost,
                                      a.ws.mark + (size_t)pick * n, a.ws.dacc + (size_t)pick * n,
