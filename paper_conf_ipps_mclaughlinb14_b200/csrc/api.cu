@@ -36,6 +36,7 @@ struct dbc_ctx {
     bool ub2 = false;  // 512-thread CTAs built for two per SM (update_512x2)
     bool lowdeg = false;  // max degree <= 32 (mesh-like graphs)
     int hd_min = 1024, hd_block = 512;  // helped down levels (update.cu)
+    int he_entries = 4096, he_min = 3;   // helped flattened passes (update.cu)
     int sblock = 256, sworkers = 0;  // static kernel: its own CTA width and grid
     size_t nscratch = 0;             // worker scratch sets allocated
     // heavy lanes: the slowest root chains of the previous batch run on
@@ -411,6 +412,8 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     c->lowdeg = maxdeg <= 32;  // every row walked by one lane: no chunked up levels
     if (const char *e = getenv("DBC_HDMIN")) c->hd_min = std::max(1, atoi(e));
     if (const char *e = getenv("DBC_HDBLK")) c->hd_block = std::max(32, atoi(e));
+    if (const char *e = getenv("DBC_HEENT")) c->he_entries = std::max(256, atoi(e));
+    if (const char *e = getenv("DBC_HEMIN")) c->he_min = std::max(1, atoi(e));
     c->block = 512;
     if (const char *eb = getenv("DBC_BLOCK"))
         c->block = atoi(eb) == 128 ? 128 : (atoi(eb) == 256 ? 256 : (atoi(eb) == 1024 ? 1024 : 512));
@@ -701,12 +704,17 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     a.slot_list = nullptr;
     a.slot_count = 0;
     a.worker_base = 0;
+    a.steal_list = nullptr;
+    a.steal_count = 0;
+    a.steal_next = nullptr;
     a.help = HelpBoard{};  // Mode S: no cooperative help
     a.merge = (c->flags & DBC_FLAG_NO_MERGE) ? 0 : 1;
     a.scen = nullptr;
     a.del = 0;
     a.hd_min = c->hd_min;
     a.hd_block = c->hd_block;
+    a.he_entries = c->he_entries;
+    a.he_min = c->he_min;
     a.lowdeg = c->lowdeg && !getenv("DBC_NO_LOWDEG");
     if (c->scen_cap > 0) {  // Fig. 2 / Fig. 4 log: one job per (root, insertion)
         if (cnt > c->scen_cap)
@@ -789,6 +797,9 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
                 h.slot_count = nh;
                 h.worker_base = c->workers;
                 h.next_slot = c->next_slot + 1;
+                h.steal_list = c->slots_d;  // heavy CTAs continue with normal roots
+                h.steal_count = k - nh;
+                h.steal_next = c->next_slot;
                 if (c->hblock == 1024)
                     launch_update_1024(h, nh, c->hstream);
                 else if (c->hblock == 512)
@@ -800,7 +811,17 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
             }
             a.slot_list = c->slots_d;
             a.slot_count = k - nh;
-            const int wl = std::min(c->workers, k - nh);
+            if (nh > 0) {  // normal CTAs take heavy roots the heavy lane has not started
+                a.steal_list = c->slots_d + (k - nh);
+                a.steal_count = nh;
+                a.steal_next = c->next_slot + 1;
+            }
+            // Co-residency: a heavy CTA needs a whole SM, and idle workers of either
+            // lane spin on the help board until every root chain is done -- so the
+            // normal lane must leave the heavy lane its SMs, or a normal grid that
+            // fills every SM first would wait forever for the heavy roots.
+            const int upb_n = c->block == 128 ? 4 : (c->block == 256 ? 2 : (c->ub2 ? 2 : 1));
+            const int wl = std::max(1, std::min(c->workers - nh * upb_n, k - nh));
             if (c->block == 128)
                 launch_update_128(a, wl, c->stream);
             else if (c->block == 512)
@@ -960,11 +981,16 @@ static dbc_status delete_host_ids(dbc_ctx *c, const int32_t *u, const int32_t *v
     a.slot_list = nullptr;
     a.slot_count = 0;
     a.worker_base = 0;
+    a.steal_list = nullptr;
+    a.steal_count = 0;
+    a.steal_next = nullptr;
     a.help = HelpBoard{};
     a.merge = 0;
     a.del = 1;
     a.hd_min = c->hd_min;
     a.hd_block = c->hd_block;
+    a.he_entries = c->he_entries;
+    a.he_min = c->he_min;
     a.lowdeg = c->lowdeg && !getenv("DBC_NO_LOWDEG");
     a.scen = nullptr;
     if (c->scen_cap > 0) {

@@ -489,8 +489,8 @@ __device__ __forceinline__ void build_l2masks(const GView &g, const Root &st, ui
 //   bit 63 open | bits 40..59 blocks | bits 16..35 next block | bits 0..15 seq
 // (helpers grab a block with one atomicAdd of 1 << 16), a done counter, the
 // job context, a global mirror of the chunk and a global append list.
-constexpr int kHelpEntries = 4096;     // entries per help block
-constexpr int kHelpMinBlocks = 3;      // publish only passes of >= 3 blocks
+// flattened passes (C1 pull, C2 push) are published when they have at least
+// UpdateArgs.he_min blocks of he_entries entries (defaults 3 x 4096)
 struct HelpCtx {
     int root_slot, l, g0, lim, cnt, nblocks, E2;  // g0..lim: the job's insertions
     uint32_t E;  // epoch << 2 of the job
@@ -540,12 +540,16 @@ struct UpdateArgs {
     const int32_t *slot_list;      // nullable: the slots this launch processes (else 0..k_loc-1)
     int32_t slot_count;            // entries of slot_list
     int32_t worker_base;           // scratch index of CTA 0
+    const int32_t *steal_list;     // nullable: the other lane's slots, taken once this list is done
+    int32_t steal_count;
+    int32_t *steal_next;           // the other lane's counter
     HelpBoard help;                // help.word == nullptr: no cooperative help
     int32_t merge;                 // 1: a window of ws.wcap insertions per job; 0: one per insertion
     long long *scen;               // nullable: scenario log [batch insertion][k_loc] (merge == 0)
     int32_t del;                   // 1: ins_u/ins_v[ins_begin] is an edge DELETION (already tombstoned)
     int32_t lowdeg;                // 1: rows are short: up levels of any size are walked in-lane
     int32_t hd_min, hd_block;      // down levels of >= hd_min items are published in hd_block blocks
+    int32_t he_entries, he_min;    // flattened passes: entries per help block, minimum blocks
 };
 
 struct StaticArgs {

@@ -331,6 +331,10 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
             const int q = atomicAdd(a.next_slot, 1);
             const int cnt = a.slot_list ? a.slot_count : a.k_loc;
             s_slot = q < cnt ? (a.slot_list ? a.slot_list[q] : q) : -1;
+            if (s_slot < 0 && a.steal_list) {  // the other lane's roots: no lane waits on the other's residency
+                const int q2 = atomicAdd(a.steal_next, 1);
+                s_slot = q2 < a.steal_count ? a.steal_list[q2] : -1;
+            }
         }
         __syncthreads();
         const int slot = s_slot;
@@ -1109,8 +1113,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                                  return dpull_visit(I.c0[t], dy, q.x, q.y);
                                              }, e0);
                             };
-                            const int nblk1 = (E1 + kHelpEntries - 1) / kHelpEntries;
-                            if (E1 > 0 && a.help.word && nblk1 >= kHelpMinBlocks) {
+                            const int nblk1 = (E1 + a.he_entries - 1) / a.he_entries;
+                            if (E1 > 0 && a.help.word && nblk1 >= a.he_min) {
                                 // publish the pull rows; helpers add per-row partial sums
                                 // into the mirror's acc (delta: rounding order is free)
                                 ChunkSmem *mir = a.help.mir + wk;
@@ -1156,7 +1160,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                     const int b = s_hb;
                                     __syncthreads();
                                     if (b < 0) break;
-                                    c1_pass(b * kHelpEntries, min(E1, (b + 1) * kHelpEntries));  // ends with a barrier
+                                    c1_pass(b * a.he_entries, min(E1, (b + 1) * a.he_entries));  // ends with a barrier
                                     if (tid == 0) atomicAdd(a.help.done + wk, 1);
                                 }
                                 if (tid == 0) {  // wait for the helpers' blocks, then close
@@ -1191,8 +1195,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                 chunk_scan(I.off, nb);
                             }
                             const int E2 = I.off[nb];
-                            const int nblk = (E2 + kHelpEntries - 1) / kHelpEntries;
-                            if (push && E2 > 0 && a.help.word && nblk >= kHelpMinBlocks) {
+                            const int nblk = (E2 + a.he_entries - 1) / a.he_entries;
+                            if (push && E2 > 0 && a.help.word && nblk >= a.he_min) {
                                 // publish the chunk; idle workers help block by block
                                 ChunkSmem *mir = a.help.mir + wk;
                                 for (int t = tid; t < nb; t += kBlock) {
@@ -1242,7 +1246,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                     const int b = s_hb;
                                     __syncthreads();
                                     if (b < 0) break;
-                                    help_run_block<false>(I, b * kHelpEntries, min(E2, (b + 1) * kHelpEntries), g,
+                                    help_run_block<false>(I, b * a.he_entries, min(E2, (b + 1) * a.he_entries), g,
                                                           st, mark, dacc, gU, gapp, cx, st_bytes);
                                     __syncthreads();  // (help_run_block ends with one too)
                                     if (tid == 0) {   // release by one thread after the CTA barrier
@@ -1482,7 +1486,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                 dc_big(hd, S, Bqh, s_nbig, st_bytes, sc_down);
                 if (tid == 0) s_nbig = 0;
             } else if (cx.kind == 2) {  // a block of a published delta-pull pass (C1)
-                const int e0 = b * kHelpEntries, e1 = min(cx.E2, (b + 1) * kHelpEntries);
+                const int e0 = b * a.he_entries, e1 = min(cx.E2, (b + 1) * a.he_entries);
                 for (int t = tid; t < cx.cnt; t += kBlock) I.acc[t] = 0.0;
                 __syncthreads();
                 auto colf = [&](int t, int e) { return ldg_i(g.col + I.beg[t] + e - I.off[t]); };
@@ -1496,7 +1500,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                 for (int t = tid; t < cx.cnt; t += kBlock)
                     if (I.acc[t] != 0.0) atomicAdd(&mir->acc[t], I.acc[t]);
             } else {
-                help_run_block<true>(I, b * kHelpEntries, min(cx.E2, (b + 1) * kHelpEntries), g, ost,
+                help_run_block<true>(I, b * a.he_entries, min(cx.E2, (b + 1) * a.he_entries), g, ost,
                                      a.ws.mark + (size_t)pick * n, a.ws.dacc + (size_t)pick * n,
                                      a.help.gU + (size_t)pick * n, a.help.gapp + pick, cx, st_bytes);
             }

@@ -678,3 +678,27 @@ def test_delete_rejects_bad_batches_atomically():
             with pytest.raises(DBCError):
                 dbc.delete_edges([p[0] for p in bad], [p[1] for p in bad])
         check_all(dbc, ref, roots.size)  # nothing changed
+
+
+@pytest.mark.timeout(240)
+@pytest.mark.parametrize("rep", range(3))
+def test_heavy_lane_with_help_completes_rmat16(rep):
+    """Heavy lane (1024-thread CTAs) beside the normal lane with the help board
+    on: a normal grid that fills every SM must not wait on heavy roots (the
+    lanes steal each other's roots).  Full-size R-MAT 16, several batches from
+    host arrays; d/sigma of sampled roots bit-exact vs the GPU's own recompute."""
+    from paper_conf_ipps_mclaughlinb14_b200 import DynamicBC
+
+    wl = W.make_workload("rmat16", insertions=4000, seed=1 + rep)
+    g = wl.graph
+    with DynamicBC(g.n, g.row_ptr, g.col, wl.roots) as dbc:
+        dbc.static_compute()
+        heavy = 0
+        for b in range(4):
+            dbc.insert_edges(wl.ins_u[1000 * b:1000 * (b + 1)], wl.ins_v[1000 * b:1000 * (b + 1)])
+            heavy = max(heavy, dbc.timings()["heavy_roots"])
+        dyn = [dbc.get_root_state(s)[:2] for s in range(0, wl.roots.size, 37)]
+        dbc.static_compute()
+        for i, s in enumerate(range(0, wl.roots.size, 37)):
+            d, sg, _ = dbc.get_root_state(s)
+            assert np.array_equal(d, dyn[i][0]) and np.array_equal(sg, dyn[i][1])
