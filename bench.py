@@ -135,14 +135,16 @@ def hbm_peak():
         return 6650.0, "fallback (B200_PROFILING.md)"
 
 
-def ncu_traffic(config, batch, mode):
-    """dram bytes per update-kernel launch from the committed ncu capture, if any."""
+def ncu_traffic(config, batch, mode, launches_per_batch):
+    """dram bytes per update-kernel launch from the committed ncu capture, if any
+    (the capture holds one batch's update in ONE launch; the timed run may split
+    it over the heavy and normal lanes, so it is divided like the algorithmic bytes)."""
     path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     try:
         with open(path) as f:
             t = json.load(f)
         e = t.get(f"{config}/b{batch}/{mode}")
-        return None if e is None else float(e["dram_bytes_per_launch"])
+        return None if e is None else float(e["dram_bytes_per_batch"]) / max(launches_per_batch, 1.0)
     except Exception:
         return None
 
@@ -468,7 +470,7 @@ def run_ours(args):
         },
         "roofline": {
             "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-            "frac": achieved / peak, "traffic": ncu_traffic(args.config, B, args.mode),
+            "frac": achieved / peak, "traffic": ncu_traffic(args.config, B, args.mode, launches / K),
             "kernel": "update_kernel", "peak_source": peak_src,
             "alg_bytes_per_launch": bytes_per_launch, "launch_ms": launch_ms,
             "share_of_step": upd_ms / ms if ms > 0 else None,

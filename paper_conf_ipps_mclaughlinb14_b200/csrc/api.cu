@@ -500,7 +500,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->help.mir, nwk);
     AL(c->help.gapp, nwk);
     AL(c->help.gU, wn);
-    AL(c->help.roots_left, 1);
+    AL(c->help.roots_left, 2);  // [0] live counter, [1] = k_loc (the per-batch reset source)
     AL(c->help.low, nwk);
     c->help.nworkers = (int)nwk;
     if (const char *e = getenv("DBC_NO_HELP")) c->help_on = atoi(e) == 0;
@@ -509,6 +509,11 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->stats, (size_t)kStCount);
     AL(c->err, 1);
     AL(c->root_prof, (size_t)6 * std::max(c->k_loc, 1));
+    {
+        const int kl[2] = {0, c->k_loc};
+        if (cudaMemcpy(c->help.roots_left, kl, sizeof(kl), cudaMemcpyHostToDevice) != cudaSuccess)
+            return bail(fail(c, DBC_ECUDA, "roots_left init"));
+    }
     if (c->flags & DBC_FLAG_EDGE_PARALLEL) {  // Table II comparison kernel: one 512-thread CTA per SM
         c->eworkers = std::max(0, std::min<int>({c->nsm, c->k_loc, (int)nwk}));
         AL(c->esrc, (size_t)c->col_cap);
@@ -785,9 +790,8 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
             if (c->help_on) {  // fresh board: all requests closed, every root chain pending
                 a.help = c->help;
                 CK(cudaMemsetAsync(c->help.word, 0, sizeof(unsigned long long) * c->help.nworkers, c->stream));
-                const int left = k;
-                CK(cudaMemcpyAsync(c->help.roots_left, &left, sizeof(int), cudaMemcpyHostToDevice, c->stream));
-                CK(cudaStreamSynchronize(c->stream));  // `left` is a host stack value
+                CK(cudaMemcpyAsync(c->help.roots_left, c->help.roots_left + 1, sizeof(int),
+                                   cudaMemcpyDeviceToDevice, c->stream));  // no host sync per batch
             }
             if (nh > 0) {  // heavy lane first, on the high-priority stream
                 CK(cudaEventRecord(c->ev_fork, c->stream));

@@ -505,7 +505,7 @@ struct HelpBoard {
     ChunkSmem *mir;            // [workers]
     int *gapp;                 // [workers] global append counters
     int32_t *gU;               // [workers][n] global append lists
-    int *roots_left;           // [1] root chains not yet finished (both lanes)
+    int *roots_left;           // [0] root chains not yet finished (both lanes), [1] = k_loc
     int *low;                  // [workers] kind 1: a distance was lowered in the helped level
     int nworkers;
 };
