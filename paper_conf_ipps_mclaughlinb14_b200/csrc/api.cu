@@ -37,6 +37,9 @@ struct dbc_ctx {
     bool lowdeg = false;  // max degree <= 32 (mesh-like graphs)
     int hd_min = 1024, hd_block = 512;  // helped down levels (update.cu)
     int he_entries = 4096, he_min = 3;   // helped flattened passes (update.cu)
+    int busy_help = 1;                   // blocks a busy worker takes at a level boundary
+    int busy_min = 32;                   // ... of passes of at least this many blocks
+    int dl_min = 16 * 4096;              // entry-balanced long rows of a down level from this many entries
     int sblock = 256, sworkers = 0;  // static kernel: its own CTA width and grid
     size_t nscratch = 0;             // worker scratch sets allocated
     // heavy lanes: the slowest root chains of the previous batch run on
@@ -414,6 +417,9 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     if (const char *e = getenv("DBC_HDBLK")) c->hd_block = std::max(32, atoi(e));
     if (const char *e = getenv("DBC_HEENT")) c->he_entries = std::max(256, atoi(e));
     if (const char *e = getenv("DBC_HEMIN")) c->he_min = std::max(1, atoi(e));
+    if (const char *e = getenv("DBC_BUSY_HELP")) c->busy_help = std::max(0, atoi(e));
+    if (const char *e = getenv("DBC_BUSY_MIN")) c->busy_min = std::max(1, atoi(e));
+    if (const char *e = getenv("DBC_DLMIN")) c->dl_min = std::max(1, atoi(e));
     c->block = 512;
     if (const char *eb = getenv("DBC_BLOCK"))
         c->block = atoi(eb) == 128 ? 128 : (atoi(eb) == 256 ? 256 : (atoi(eb) == 1024 ? 1024 : 512));
@@ -500,8 +506,9 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->help.mir, nwk);
     AL(c->help.gapp, nwk);
     AL(c->help.gU, wn);
-    AL(c->help.roots_left, 2);  // [0] live counter, [1] = k_loc (the per-batch reset source)
+    AL(c->help.roots_left, 4);  // [0] live counter, [1] open requests, [2..3] = {k_loc, 0}
     AL(c->help.low, nwk);
+    AL(c->help.gbig, 2 * nwk);
     c->help.nworkers = (int)nwk;
     if (const char *e = getenv("DBC_NO_HELP")) c->help_on = atoi(e) == 0;
     AL(c->next_slot, 2);
@@ -510,7 +517,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->err, 1);
     AL(c->root_prof, (size_t)6 * std::max(c->k_loc, 1));
     {
-        const int kl[2] = {0, c->k_loc};
+        const int kl[4] = {0, 0, c->k_loc, 0};
         if (cudaMemcpy(c->help.roots_left, kl, sizeof(kl), cudaMemcpyHostToDevice) != cudaSuccess)
             return bail(fail(c, DBC_ECUDA, "roots_left init"));
     }
@@ -720,6 +727,10 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     a.hd_block = c->hd_block;
     a.he_entries = c->he_entries;
     a.he_min = c->he_min;
+    a.busy_help = c->busy_help;
+    a.busy_min = c->busy_min;
+    a.dl_min = c->dl_min;
+    a.trace_slot = getenv("DBC_TRACE_SLOT") ? atoi(getenv("DBC_TRACE_SLOT")) : -1;
     a.lowdeg = c->lowdeg && !getenv("DBC_NO_LOWDEG");
     if (c->scen_cap > 0) {  // Fig. 2 / Fig. 4 log: one job per (root, insertion)
         if (cnt > c->scen_cap)
@@ -790,7 +801,7 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
             if (c->help_on) {  // fresh board: all requests closed, every root chain pending
                 a.help = c->help;
                 CK(cudaMemsetAsync(c->help.word, 0, sizeof(unsigned long long) * c->help.nworkers, c->stream));
-                CK(cudaMemcpyAsync(c->help.roots_left, c->help.roots_left + 1, sizeof(int),
+                CK(cudaMemcpyAsync(c->help.roots_left, c->help.roots_left + 2, 2 * sizeof(int),
                                    cudaMemcpyDeviceToDevice, c->stream));  // no host sync per batch
             }
             if (nh > 0) {  // heavy lane first, on the high-priority stream
@@ -995,6 +1006,10 @@ static dbc_status delete_host_ids(dbc_ctx *c, const int32_t *u, const int32_t *v
     a.hd_block = c->hd_block;
     a.he_entries = c->he_entries;
     a.he_min = c->he_min;
+    a.busy_help = c->busy_help;
+    a.busy_min = c->busy_min;
+    a.dl_min = c->dl_min;
+    a.trace_slot = getenv("DBC_TRACE_SLOT") ? atoi(getenv("DBC_TRACE_SLOT")) : -1;
     a.lowdeg = c->lowdeg && !getenv("DBC_NO_LOWDEG");
     a.scen = nullptr;
     if (c->scen_cap > 0) {

@@ -65,8 +65,12 @@ enum StatIdx : int {
     kStHelpBlkAll,               // all blocks of published passes
     kStGroups,                   // Case-2 group jobs (>= 2 insertions repaired together)
     kStGroupIns,                 // insertions in those group jobs
-    kStCount
+    kStBusyBlk,                  // help blocks run by busy workers (at their level boundaries)
+    kStTraceN,                   // -DDBC_PHASE_TIMERS: events of the traced slot (DBC_TRACE_SLOT)
+    kStTrace0,                   // kTraceCap (code, %globaltimer) pairs
+    kStCount = kStTrace0 + 2 * 1024
 };
+constexpr int kTraceCap = 1024;
 
 // The state of one root (pointers into the root-major arrays).
 struct Root {
@@ -494,7 +498,9 @@ __device__ __forceinline__ void build_l2masks(const GView &g, const Root &st, ui
 struct HelpCtx {
     int root_slot, l, g0, lim, cnt, nblocks, E2;  // g0..lim: the job's insertions
     uint32_t E;  // epoch << 2 of the job
-    int kind;    // 0: C2 push pass of a published chunk; 1: a down-phase level
+    int kind;    // 0: C2 push pass of a published chunk; 1: a down-phase level;
+                 // 2: C1 delta-pull pass of a chunk; 3: the Case-3 removal pass over D;
+                 // 4: the long rows of a down level, entry-balanced (E2 entries, cnt rows)
     int lb;      // kind 1: the level's first position in D
     int mvalid;  // kind 1: level-2 masks are maintained
 };
@@ -505,9 +511,12 @@ struct HelpBoard {
     ChunkSmem *mir;            // [workers]
     int *gapp;                 // [workers] global append counters
     int32_t *gU;               // [workers][n] global append lists
-    int *roots_left;           // [0] root chains not yet finished (both lanes), [1] = k_loc
-    int *low;                  // [workers] kind 1: a distance was lowered in the helped level
+    int *roots_left;           // [0] root chains not yet finished (both lanes), [1] open requests,
+                               // [2..3] = {k_loc, 0}: the per-batch reset source of [0..1]
+    int *low;                  // [workers] kind 1: a distance was lowered in the helped level;
+                               // kind 3: deepest removal-target level
     int nworkers;
+    int *gbig;                 // [workers][2] kind 1: long rows queued in the owner's Bq, their entries
 };
 __device__ __forceinline__ unsigned long long help_pack(int open, int nblocks, int next, int seq) {
     return ((unsigned long long)(open ? 1 : 0) << 63) | ((unsigned long long)(nblocks & 0xFFFFF) << 40) |
@@ -550,6 +559,10 @@ struct UpdateArgs {
     int32_t lowdeg;                // 1: rows are short: up levels of any size are walked in-lane
     int32_t hd_min, hd_block;      // down levels of >= hd_min items are published in hd_block blocks
     int32_t he_entries, he_min;    // flattened passes: entries per help block, minimum blocks
+    int32_t busy_help;             // blocks a busy worker takes per poll of the board (0: only idle workers help)
+    int32_t busy_min;              // busy workers take blocks of passes of at least this many blocks
+    int32_t dl_min;                // down levels whose long rows hold >= dl_min entries: entry-balanced pass
+    int32_t trace_slot;            // -DDBC_PHASE_TIMERS builds: time this slot only (-1: all)
 };
 
 struct StaticArgs {

@@ -155,7 +155,7 @@ __device__ __forceinline__ double dc_visit(const DownCtx &c, int y, int dy, doub
 }
 
 // short rows of items [i0, i1) walked in-lane in canonical order (bit-exact
-// sigma); long rows handed to enq(item)
+// sigma); long rows handed to enq(item, length)
 template <class Enq>
 __device__ __forceinline__ void dc_small(const DownCtx &c, int i0, int i1, Enq enq, unsigned long long &bytes,
                                          unsigned long long &scanned) {
@@ -164,7 +164,7 @@ __device__ __forceinline__ void dc_small(const DownCtx &c, int i0, int i1, Enq e
         const int w = c.Dv[c.lb + i];
         const int2 r = row_of(c.g, w, c.lim);
         if (r.y - r.x > kSmallDeg) {
-            enq(i);
+            enq(i, r.y - r.x);
             continue;
         }
         double sum = 0.0;  // canonical order: bit-exact
@@ -256,6 +256,248 @@ __device__ __forceinline__ void dc_big(const DownCtx &c, BigSmem &S, const int32
     }
 }
 
+// ---------------------------------------------------------------------------
+// (0) Case-3 removal pushes (A4 step 0) over D items [i0, i1): every pulled-up
+// w (finite old level od != d[w]) gives each old predecessor x outside D
+//   Ddelta[x] -= sigma[x] / sigma_old(w) * (1 + delta_old(w))
+// (the accumulator holds Ddelta / sigma: DESIGN.md Sec. 6), and x becomes an
+// up vertex of level od - 1.  The owner's whole pass, or one block of a helped
+// pass (then rcnt / rmax are the owner's global counters).  Ends with a barrier.
+struct RemCtx {
+    GView g;
+    Root st;
+    uint32_t *mark;
+    double *dacc;
+    const int32_t *Dv, *Dold;
+    const double *Dsig;
+    int32_t *Rv, *Rl;
+    int *rcnt, *rmax;
+    int g0, lim;
+    uint32_t E, mD, mU;
+};
+
+__device__ __forceinline__ void rem_visit(const RemCtx &c, int w, int od, double osig, double coef, int x,
+                                          int dx, unsigned long long &bytes) {
+    if (dx != od - 1) return;
+    if (c.mark[x] == c.mD) return;
+    if (ldg_i(c.g.rp + w) < 0 && new_edge(c.g, w, x, c.g0, c.lim)) return;  // not an old predecessor
+    atomicAdd(c.dacc + x, -__ddiv_rn(coef, osig));
+    bytes += 24;
+    if (atomicMax(c.mark + x, c.mU) < c.E) {
+        const int pos = atomicAdd(c.rcnt, 1);
+        c.Rv[pos] = x;
+        c.Rl[pos] = od - 1;
+        atomicMax(c.rmax, od - 1);
+    }
+}
+
+__device__ __forceinline__ void rem_range(const RemCtx &c, BigSmem &S, int *s_old, int32_t *Bq, int *nbig,
+                                          int i0, int i1, unsigned long long &bytes,
+                                          unsigned long long &scanned) {
+    const int tid = threadIdx.x;
+    split_pass(
+        i1 - i0, c.g, c.lim,
+        [&](int q, int &w) {
+            const int i = i0 + q;
+            const int od = c.Dold[i] & kOldMask;
+            w = c.Dv[i];
+            return od != kInf && od != c.st.dist(w);
+        },
+        [&](int q, int w, int2 r) {
+            const int i = i0 + q;
+            const int od = c.Dold[i] & kOldMask;
+            const double osig = c.Dsig[i];
+            const double coef = 1.0 + c.st.sd[w].y;  // delta still old
+            row_walk(c.g, c.st, nullptr, r, [&](int dx) { return dx == od - 1; },
+                     [&](int x, int dx, double2, uint32_t) { rem_visit(c, w, od, osig, coef, x, dx, bytes); });
+            bytes += 16 + 8ull * (r.y - r.x);
+            scanned += r.y - r.x;
+        },
+        [&](int q) { Bq[atomicAdd(nbig, 1)] = i0 + q; });
+    __syncthreads();
+    const int nb = *nbig;
+    for (int r0 = 0; r0 < nb; r0 += kBig) {
+        const int m = min(kBig, nb - r0);
+        big_load(S, m, [&](int t) { return Bq[r0 + t]; }, [&](int i) { return c.Dv[i]; }, c.g, c.lim);
+        if (tid < m) {
+            const int i = S.idx[tid];
+            S.c0[tid] = c.Dsig[i];
+            s_old[tid] = c.Dold[i] & kOldMask;  // old level of each row
+            bytes += 16;
+        }
+        __syncthreads();
+        big_entries(S, c.g, c.st, [](int) { return true; }, [&](int t, int x, int dx, double2) {
+            bytes += 8;
+            scanned++;
+            const int w = S.v[t];
+            rem_visit(c, w, s_old[t], S.c0[t], 1.0 + c.st.sd[w].y, x, dx, bytes);
+            return 0.0;
+        });
+    }
+    __syncthreads();
+    if (tid == 0) *nbig = 0;
+    __syncthreads();
+}
+
+// ---------------------------------------------------------------------------
+// Long rows of a down level, entry-balanced (a level's long rows can hold most
+// of its entries -- hub neighbourhoods -- so blocks of rows would not balance).
+// The owner queues the level's long rows (item indices) in Bq[0, nrows), builds
+// exclusive entry offsets Boff[0..nrows] (dl_offsets), then the entries are
+// processed in blocks of he_entries (dl_block, owner and helpers): per entry the
+// down-phase visit (lowering, claims), per row the predecessor-sigma partial sum
+// added into dacc[w] (sums of integer-valued sigma: exact in any order below
+// 2^53, else the owner re-sums the row in canonical order), the "predecessor
+// outside D" flag as bit 31 of Bq[t], and level-2 mask bits into mask[w].
+// dl_finish (owner) completes every row with dc_finish.
+constexpr uint32_t kBqExt = 0x80000000u;
+constexpr int kDlEntries = 32 * kBig;  // entries per block: spans <= kBig long rows (> kSmallDeg entries each)
+
+// owner: offsets of Bq[0, nrows) into Boff (uses I.off as scratch); returns the
+// entry total (every thread).  Ends with a barrier.
+__device__ __forceinline__ int dl_offsets(const DownCtx &c, int32_t *Bq, int32_t *Boff, int nrows, int *soff,
+                                          int *s_tot) {
+    const int tid = threadIdx.x;
+    if (tid == 0) *s_tot = 0;
+    __syncthreads();
+    for (int r0 = 0; r0 < nrows; r0 += kChunk) {
+        const int m = min(kChunk, nrows - r0);
+        for (int i = tid; i < m; i += kBlock) {
+            const int w = c.Dv[c.lb + Bq[r0 + i]];
+            const int2 r = row_of(c.g, w, c.lim);
+            soff[i + 1] = r.y - r.x;
+            if (c.mvalid && c.L == 2) c.mask[w] = 0u;
+        }
+        __syncthreads();
+        chunk_scan(soff, m);  // ends with a barrier
+        const int carry = *s_tot;
+        for (int i = tid; i < m; i += kBlock) Boff[r0 + i] = carry + soff[i];
+        __syncthreads();
+        if (tid == 0) *s_tot = carry + soff[m];
+        __syncthreads();
+    }
+    const int tot = *s_tot;
+    if (tid == 0) Boff[nrows] = tot;
+    return tot;
+}
+
+// entries [e0, e1) of the published long rows (owner or helper; kCG: read the
+// owner's lists through L2).  Ends with a barrier.
+template <bool kCG>
+__device__ __forceinline__ void dl_block(const DownCtx &c, BigSmem &S, int32_t *Bq, const int32_t *Boff,
+                                         int nrows, int e0, int e1, double *dacc, int *s_t0,
+                                         unsigned long long &bytes, unsigned long long &scanned) {
+    const int tid = threadIdx.x, L = c.L;
+    // first row: last t with Boff[t] <= e0 (two strided probes over the CTA)
+    if (tid == 0) *s_t0 = 0;
+    __syncthreads();
+    const int stride = (nrows + kBlock - 1) / kBlock;
+    {
+        const int t = tid * stride;
+        if (t < nrows && (kCG ? __ldcg(Boff + t) : Boff[t]) <= e0) atomicMax(s_t0, tid);
+    }
+    __syncthreads();
+    const int j0 = *s_t0 * stride;
+    __syncthreads();
+    if (tid < stride && j0 + tid < nrows && (kCG ? __ldcg(Boff + j0 + tid) : Boff[j0 + tid]) <= e0)
+        atomicMax(s_t0, j0 + tid);
+    __syncthreads();
+    const int t0 = *s_t0;
+    // rows t0 .. (at most kBig of them: long rows have > kSmallDeg entries)
+    if (tid < kBig) {
+        const int t = t0 + tid;
+        const int bo = (t < nrows) ? (kCG ? __ldcg(Boff + t) : Boff[t]) : e1;
+        if (bo < e1) {
+            const int idx = (int)((uint32_t)(kCG ? __ldcg(Bq + t) : Bq[t]) & ~kBqExt);
+            const int w = kCG ? __ldcg(c.Dv + c.lb + idx) : c.Dv[c.lb + idx];
+            const int2 r = row_of(c.g, w, c.lim);
+            S.v[tid] = w;
+            S.b[tid] = r.x;
+            S.off[tid] = bo;
+            S.acc[tid] = 0.0;
+            S.mk[tid] = 0u;
+            S.ext[tid] = 0;
+            S.idx[tid] = 1;
+        } else {
+            S.idx[tid] = 0;
+        }
+    }
+    __syncthreads();
+    if (tid < kBig && S.idx[tid] && (tid + 1 == kBig || !S.idx[tid + 1])) S.m = tid + 1;
+    __syncthreads();
+    const int m = S.m;
+    for (int base = e0; base < e1; base += kUnroll * kBlock) {
+        int t[kUnroll], y[kUnroll], dy[kUnroll];
+        double sy[kUnroll];
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u) {
+            const int e = base + u * kBlock + tid;
+            t[u] = -1;
+            y[u] = 0;
+            if (e < e1) {
+                int lo = 0, hi = m - 1;  // last row with off <= e
+                while (lo < hi) {
+                    const int mid = (lo + hi + 1) >> 1;
+                    if (S.off[mid] <= e) lo = mid; else hi = mid - 1;
+                }
+                t[u] = lo;
+                y[u] = ldg_i(c.g.col + S.b[lo] + (e - S.off[lo]));
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u) dy[u] = (t[u] >= 0) ? (kCG ? __ldcg(c.st.d + y[u]) : c.st.dist(y[u])) : kInf;
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u)
+            sy[u] = (t[u] >= 0 && dy[u] == L - 1) ? (kCG ? __ldcg(&c.st.sd[y[u]].x) : c.st.sd[y[u]].x) : 0.0;
+#pragma unroll
+        for (int u = 0; u < kUnroll; ++u) {
+            double cc = 0.0;
+            if (t[u] >= 0) {
+                bytes += 8;
+                scanned++;
+                if (dy[u] == L - 1) {
+                    if (c.mvalid && L == 2) atomicOr(&S.mk[t[u]], dc_l1bit(c, y[u]));
+                    if ((kCG ? __ldcg(c.mark + y[u]) : c.mark[y[u]]) != c.mD) S.ext[t[u]] = 1;
+                }
+                cc = dc_visit(c, y[u], dy[u], sy[u], bytes);
+            }
+            acc_add(S.acc, t[u], cc);
+        }
+    }
+    __syncthreads();
+    if (tid < m) {  // publish the block's per-row partials
+        const int w = S.v[tid];
+        if (S.acc[tid] != 0.0) atomicAdd(dacc + w, S.acc[tid]);
+        if (S.ext[tid]) atomicOr((uint32_t *)(Bq + t0 + tid), kBqExt);
+        if (S.mk[tid]) atomicOr(c.mask + w, S.mk[tid]);
+    }
+    __syncthreads();
+}
+
+// owner: complete the long rows after every block ran
+__device__ __forceinline__ void dl_finish(const DownCtx &c, const int32_t *Bq, int nrows, double *dacc,
+                                          unsigned long long &bytes) {
+    const int L = c.L;
+    for (int t = threadIdx.x; t < nrows; t += kBlock) {
+        const uint32_t q = (uint32_t)__ldcg(Bq + t);
+        const int idx = (int)(q & ~kBqExt);
+        const int w = c.Dv[c.lb + idx];
+        double sum = __ldcg(dacc + w);
+        dacc[w] = 0.0;
+        if (sum >= kExact) {  // order-dependent rounding: canonical sum
+            const int2 r = row_of(c.g, w, c.lim);
+            sum = 0.0;
+            for (int j = r.x; j < r.y; ++j) {
+                const int y = ldg_i(c.g.col + j);
+                if (c.st.dist(y) == L - 1) sum += c.st.sd[y].x;
+            }
+        }
+        const uint32_t m = (c.mvalid && L == 2) ? __ldcg(c.mask + w) : 0u;
+        dc_finish(c, c.lb + idx, w, sum, m, (q & kBqExt) != 0, bytes);
+    }
+    __syncthreads();
+}
+
 __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a) {
     __shared__ int s_slot;
     __shared__ int s_dcnt;     // |D| (absolute positions in Dv)
@@ -278,6 +520,9 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
     __shared__ int s_un[2][kUcap];       // up frontier ping-pong (overflow: U0 / U1)
     __shared__ int s_hb, s_hpick, s_hseq; // cooperative help: grabbed block, owner, request
     __shared__ HelpCtx s_hctx;
+    __shared__ int s_hadjs[kMaskDeg], s_hds;  // helped down level: the owner's root row (mask bits)
+    __shared__ int s_hopen;                   // open requests seen at the last level boundary
+    __shared__ int s_nent, s_tot, s_t0;        // long rows of a down level: entries, offsets total, first row
     __shared__ int s_del[6];     // deletion job: [0] u_high, [1] u_low, [2] |A|, [3] seeds, [4] candidates, [5] u_low keeps a predecessor
     __shared__ double s_delsd[2];  // deletion job: old sigma / delta of u_low
 
@@ -309,21 +554,223 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
     // per-phase wall time seen by thread 0 (diagnostic)
     unsigned long long tm_ph[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
     unsigned long long tclk = 0;
+    int tick_on = 1;  // DBC_TRACE_SLOT: time one root only
+    int own_blk = 0;  // blocks of a published pass the owner ran itself (trace)
+    // event trace of the traced slot: code = kind << 56 | level << 32 | items
+    auto trace = [&](int kind, int lev, int items) {
+        if (kPhaseTimers && tid == 0 && tick_on && a.trace_slot >= 0) {
+            unsigned long long t;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+            const unsigned long long q = atomicAdd(a.stats + kStTraceN, 1ull);
+            if (q < (unsigned long long)kTraceCap) {
+                a.stats[kStTrace0 + 2 * q] = ((unsigned long long)kind << 56) |
+                                             ((unsigned long long)(lev & 0xFFFFFF) << 32) | (uint32_t)items;
+                a.stats[kStTrace0 + 2 * q + 1] = t;
+            }
+        }
+    };
     auto tick = [&](int ph) {
-        if (kPhaseTimers && tid == 0) {
+        if (kPhaseTimers && tid == 0 && tick_on) {
             unsigned long long t;
             asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
             if (ph >= 0) tm_ph[ph] += t - tclk;
             tclk = t;
         }
     };
-    auto enq_front = [&](int idx) { Bq[atomicAdd(&s_nbig, 1)] = idx; };
+
+    // One help step: scan the board, claim one block of an open request of
+    // another worker and run it.  Idle workers (out of roots) loop on it; busy
+    // workers call it at their own level boundaries (only there: the block
+    // reuses S, I, Bq and s_nbig, which are free between levels).  (cur_owner,
+    // cur_seq) caches the chunk loaded into I -- valid only while this CTA runs
+    // nothing else.  Returns -2 when every root chain is done (idle), -1 when
+    // no block was taken, 1 after running one.
+    auto help_step = [&](bool idle, int &cur_owner, int &cur_seq) -> int {
+        // the whole CTA scans the board (one word per thread), first open one wins
+        // Priority: the request with the most blocks left (the widest pass of the
+        // slowest chain); busy workers only take passes of >= busy_min blocks.
+        const int nw = a.help.nworkers;
+        if (tid == 0) s_hpick = 0;
+        __syncthreads();
+        for (int i = tid; i < nw; i += kBlock) {
+            const int o = (wk + 1 + i) % nw;
+            const unsigned long long w = __ldcg(a.help.word + o);
+            const int left = help_nblocks(w) - help_next(w);
+            if (help_open(w) && left > 0 && (idle || help_nblocks(w) >= a.busy_min))
+                atomicMax((unsigned *)&s_hpick, ((unsigned)min(left, 0xFFFFF) << 12) | (unsigned)i);
+        }
+        __syncthreads();
+        if (tid == 0) {
+            int pick = -1, b = -1, sq = -1;
+            if (idle && atomicAdd(a.help.roots_left, 0) <= 0) {
+                pick = -2;
+            } else {
+                if (s_hpick != 0) pick = (wk + 1 + (s_hpick & 0xFFF)) % nw;
+                if (pick >= 0) {
+                    const unsigned long long w = atomicAdd(a.help.word + pick, 1ull << 16);
+                    if (help_open(w) && help_next(w) < help_nblocks(w)) {
+                        b = help_next(w);
+                        sq = help_seq(w);
+                    }
+                }
+            }
+            s_hpick = pick;
+            s_hb = b;
+            s_hseq = sq;
+        }
+        __syncthreads();
+        const int pick = s_hpick, b = s_hb, sq = s_hseq;
+        __syncthreads();
+        if (pick == -2) return -2;
+        if (b < 0) return -1;
+        if (pick != cur_owner || sq != cur_seq) {  // a new request: load its chunk
+            if (tid == 0) {
+                const HelpCtx *src = a.help.ctx + pick;
+                s_hctx.root_slot = __ldcg(&src->root_slot);
+                s_hctx.l = __ldcg(&src->l);
+                s_hctx.g0 = __ldcg(&src->g0);
+                s_hctx.lim = __ldcg(&src->lim);
+                s_hctx.cnt = __ldcg(&src->cnt);
+                s_hctx.nblocks = __ldcg(&src->nblocks);
+                s_hctx.E2 = __ldcg(&src->E2);
+                s_hctx.E = __ldcg(&src->E);
+                s_hctx.kind = __ldcg(&src->kind);
+                s_hctx.lb = __ldcg(&src->lb);
+                s_hctx.mvalid = __ldcg(&src->mvalid);
+                __threadfence();  // acquire: drop stale L1 lines of the owner's state
+            }
+            __syncthreads();
+            const ChunkSmem *mir = a.help.mir + pick;
+            const int cnt = (s_hctx.kind == 0 || s_hctx.kind == 2) ? s_hctx.cnt : 0;  // kinds 0 and 2 publish a chunk
+            if ((s_hctx.kind == 1 || s_hctx.kind == 4) && s_hctx.mvalid && tid < 32) {  // the root's row (mask bits)
+                const int2 rs = row_of(g, a.roots[s_hctx.root_slot], s_hctx.lim);
+                const int ds = rs.y - rs.x;
+                if (tid < ds && ds <= kMaskDeg) s_hadjs[tid] = ldg_i(g.col + rs.x + tid);
+                if (tid == 0) s_hds = ds;
+            }
+            for (int t = tid; t < cnt; t += kBlock) {
+                I.v[t] = __ldcg(&mir->v[t]);
+                I.meta[t] = __ldcg(&mir->meta[t]);
+                I.beg[t] = __ldcg(&mir->beg[t]);
+                I.off[t + 1] = __ldcg(&mir->off[t + 1]);
+                I.acc[t] = __ldcg(&mir->acc[t]);
+                I.c0[t] = __ldcg(&mir->c0[t]);
+                I.c1[t] = __ldcg(&mir->c1[t]);
+                I.c2[t] = __ldcg(&mir->c2[t]);
+            }
+            if (tid == 0) I.off[0] = 0;
+            __syncthreads();
+            cur_owner = pick;
+            cur_seq = sq;
+        }
+        const HelpCtx cx = s_hctx;
+        const Root ost{a.d + (size_t)cx.root_slot * n, a.sd + (size_t)cx.root_slot * n};
+        if (cx.kind == 1 || cx.kind == 4) {  // a block of a published down-phase level / its long rows
+            DownCtx hd;
+            hd.g = g;
+            hd.st = ost;
+            hd.mark = a.ws.mark + (size_t)pick * n;
+            hd.lowrec = a.ws.lowrec + (size_t)pick * n;
+            hd.Dv = a.ws.Dv + (size_t)pick * n;
+            hd.Dold = a.ws.Dold + (size_t)pick * n;
+            hd.Dsig = a.ws.Dsig + (size_t)pick * n;
+            hd.mask = a.l2mask + (size_t)cx.root_slot * n;
+            hd.err = a.err;
+            hd.dcnt = a.help.gapp + pick;
+            hd.lowflag = a.help.low + pick;
+            hd.adjs = s_hadjs;
+            hd.dsr = s_hds;
+            hd.L = cx.l;
+            hd.lb = cx.lb;
+            hd.lim = cx.lim;
+            hd.mvalid = cx.mvalid;
+            hd.del = a.del;
+            hd.epoch = cx.E >> 2;
+            hd.mD = cx.E | kDown;
+            int32_t *oBq = a.ws.Bq + (size_t)pick * n;  // the owner's long-row queue
+            if (cx.kind == 1) {
+                const int kDownBlock = a.hd_block;
+                int *gb = a.help.gbig + 2 * pick;
+                dc_small(hd, b * kDownBlock, min(cx.cnt, (b + 1) * kDownBlock),
+                         [&](int i, int len) {
+                             oBq[atomicAdd(gb, 1)] = i;
+                             atomicAdd(gb + 1, len);
+                         },
+                         st_bytes, sc_down);
+            } else {
+                dl_block<true>(hd, S, oBq, a.ws.U1 + (size_t)pick * n, cx.cnt, b * kDlEntries,
+                               min(cx.E2, (b + 1) * kDlEntries), a.ws.dacc + (size_t)pick * n, &s_t0, st_bytes,
+                               sc_down);
+            }
+        } else if (cx.kind == 3) {  // a block of a published removal pass (Case 3)
+            RemCtx hr;
+            hr.g = g;
+            hr.st = ost;
+            hr.mark = a.ws.mark + (size_t)pick * n;
+            hr.dacc = a.ws.dacc + (size_t)pick * n;
+            hr.Dv = a.ws.Dv + (size_t)pick * n;
+            hr.Dold = a.ws.Dold + (size_t)pick * n;
+            hr.Dsig = a.ws.Dsig + (size_t)pick * n;
+            hr.Rv = a.ws.Rv + (size_t)pick * n;
+            hr.Rl = a.ws.Rl + (size_t)pick * n;
+            hr.rcnt = a.help.gapp + pick;
+            hr.rmax = a.help.low + pick;
+            hr.g0 = cx.g0;
+            hr.lim = cx.lim;
+            hr.E = cx.E;
+            hr.mD = cx.E | kDown;
+            hr.mU = cx.E | kUp;
+            const int kRemBlock = a.hd_block;
+            rem_range(hr, S, s_l1, a.ws.Bq + (size_t)wk * n, &s_nbig, b * kRemBlock,
+                      min(cx.cnt, (b + 1) * kRemBlock), st_bytes, sc_rem);
+        } else if (cx.kind == 2) {  // a block of a published delta-pull pass (C1)
+            const int e0 = b * a.he_entries, e1 = min(cx.E2, (b + 1) * a.he_entries);
+            for (int t = tid; t < cx.cnt; t += kBlock) I.acc[t] = 0.0;
+            __syncthreads();
+            auto colf = [&](int t, int e) { return ldg_i(g.col + I.beg[t] + e - I.off[t]); };
+            flat_entries<true>(I.off, cx.cnt, e1, colf, ost, nullptr, [&](int dy) { return dy == cx.l + 1; },
+                               I.acc, [&](int t, int, int dy, double2 q, uint32_t) -> double {
+                                   st_bytes += 8;
+                                   if (dy != cx.l + 1) return 0.0;
+                                   return __dmul_rn(__ddiv_rn(I.c0[t], q.x), __dadd_rn(1.0, q.y));
+                               }, e0);
+            ChunkSmem *mir = a.help.mir + pick;
+            for (int t = tid; t < cx.cnt; t += kBlock)
+                if (I.acc[t] != 0.0) atomicAdd(&mir->acc[t], I.acc[t]);
+        } else {
+            help_run_block<true>(I, b * a.he_entries, min(cx.E2, (b + 1) * a.he_entries), g, ost,
+                                 a.ws.mark + (size_t)pick * n, a.ws.dacc + (size_t)pick * n,
+                                 a.help.gU + (size_t)pick * n, a.help.gapp + pick, cx, st_bytes);
+        }
+        __syncthreads();
+        if (tid == 0) {  // release by one thread after the CTA barrier
+            __threadfence();
+            atomicAdd(a.help.done + pick, 1);
+            atomicAdd(a.stats + kStHelpBlk, 1ull);
+        }
+        return 1;
+    };
+    // a busy worker at a level boundary: take up to a.busy_help blocks of other
+    // workers' open requests (the heavy chains' wide levels do not wait for
+    // idle workers).  s_hopen was sampled during the previous level; every
+    // thread reads the same value (written before a barrier).
+    auto busy_help = [&]() {
+        if (!a.help.word || a.busy_help <= 0 || s_hopen <= 0) return;
+        int co = -1, cs = -1;
+        for (int q = 0; q < a.busy_help; ++q) {
+            if (help_step(false, co, cs) < 0) break;
+            if (tid == 0) atomicAdd(a.stats + kStBusyBlk, 1ull);
+        }
+    };
+    auto sample_open = [&]() { return (tid == 0 && a.help.word) ? __ldcg(a.help.roots_left + 1) : 0; };
+
 
     if (tid == 0) {
         s_nbig = 0;
         s_nbigI = 0;
         s_nl1 = 0;
         s_noext = 0;
+        s_hopen = 0;
     }
 
     for (;;) {
@@ -342,6 +789,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
         if (slot < 0) break;
         const Root st{a.d + (size_t)slot * n, a.sd + (size_t)slot * n};
         const int sroot = a.roots[slot];
+        tick_on = a.trace_slot < 0 || a.trace_slot == slot;
         uint32_t *mask = a.l2mask + (size_t)slot * n;
         unsigned long long prof_t0 = 0, prof_jobs = 0, prof_touch0 = st_touched;
         const unsigned long long prof_sc0 = sc_down + sc_rem + sc_dpull + sc_dpush + sc_up2 + sc_up3;
@@ -649,13 +1097,20 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                 dc.epoch = epoch;
                 dc.mD = mD;
                 while (true) {
+                    busy_help();
+                    const int hopen_pf = sample_open();
+                    trace(1, L, le - lb);
                     dc.L = L;
                     dc.lb = lb;
                     const int items = le - lb;
                     const int kDownBlock = a.hd_block;
+                    DownCtx gd = dc;  // appends and the lowering flag through global memory (helped passes)
+                    gd.dcnt = a.help.gapp + wk;
+                    gd.lowflag = a.help.low + wk;
+                    int nrows = 0, nent = 0;  // the level's long rows (queued in Bq) and their entries
                     if (a.help.word && items >= a.hd_min) {
-                        // a wide level: published, idle workers take blocks of items
-                        // (appends and the lowering flag go through global memory)
+                        // a wide level: published, idle workers take blocks of items; their
+                        // long rows are queued in this worker's Bq for the entry-balanced pass
                         const int nblk = (items + kDownBlock - 1) / kDownBlock;
                         if (tid == 0) {
                             HelpCtx cx;
@@ -674,15 +1129,16 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                             a.help.done[wk] = 0;
                             a.help.gapp[wk] = s_dcnt;
                             a.help.low[wk] = 0;
+                            a.help.gbig[2 * wk] = 0;
+                            a.help.gbig[2 * wk + 1] = 0;
                             __threadfence();
                             atomicAdd(a.stats + kStHelpReq, 1ull);
                             atomicAdd(a.stats + kStHelpBlkAll, (unsigned long long)nblk);
                             hseq = (hseq + 1) & 0xFFFF;
                             atomicExch(a.help.word + wk, help_pack(1, nblk, 0, hseq));
+                            if (nblk >= a.busy_min) atomicAdd(a.help.roots_left + 1, 1);  // open wide requests
                         }
-                        DownCtx gd = dc;
-                        gd.dcnt = a.help.gapp + wk;
-                        gd.lowflag = a.help.low + wk;
+                        int *gb = a.help.gbig + 2 * wk;
                         for (;;) {  // the owner takes blocks too
                             if (tid == 0) {
                                 const unsigned long long w = atomicAdd(a.help.word + wk, 1ull << 16);
@@ -692,29 +1148,107 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                             const int b = s_hb;
                             __syncthreads();
                             if (b < 0) break;
-                            dc_small(gd, b * kDownBlock, min(items, (b + 1) * kDownBlock), enq_front, st_bytes,
-                                     sc_down);
+                            ++own_blk;
+                            dc_small(gd, b * kDownBlock, min(items, (b + 1) * kDownBlock),
+                                     [&](int i, int len) {
+                                         Bq[atomicAdd(gb, 1)] = i;
+                                         atomicAdd(gb + 1, len);
+                                     },
+                                     st_bytes, sc_down);
                             __syncthreads();
-                            dc_big(gd, S, Bq, s_nbig, st_bytes, sc_down);
                             if (tid == 0) {
-                                s_nbig = 0;
                                 __threadfence();
                                 atomicAdd(a.help.done + wk, 1);
                             }
-                            __syncthreads();
                         }
+                        trace(6, 1, own_blk | (nblk << 16));
+                        own_blk = 0;
                         if (tid == 0) {  // wait for the helpers' blocks, then close
                             while (atomicAdd(a.help.done + wk, 0) < nblk) __nanosleep(256);
                             atomicExch(a.help.word + wk, help_pack(0, 0, 0, hseq));
+                            if (nblk >= a.busy_min) atomicSub(a.help.roots_left + 1, 1);
+                            __threadfence();
+                            s_dcnt = __ldcg(a.help.gapp + wk);
+                            if (__ldcg(a.help.low + wk)) s_job[3] = 1;
+                            s_nbig = __ldcg(gb);
+                            s_nent = __ldcg(gb + 1);
+                        }
+                        __syncthreads();
+                    } else {
+                        if (tid == 0) s_nent = 0;
+                        __syncthreads();
+                        dc_small(dc, 0, items,
+                                 [&](int i, int len) {
+                                     Bq[atomicAdd(&s_nbig, 1)] = i;
+                                     atomicAdd(&s_nent, len);
+                                 },
+                                 st_bytes, sc_down);
+                        __syncthreads();
+                    }
+                    nrows = s_nbig;
+                    nent = s_nent;
+                    if (a.help.word && nent >= a.dl_min) {
+                        // long rows with many entries (hub neighbourhoods): entry-balanced
+                        // blocks, owner and helpers; per-row results completed by the owner
+                        int32_t *Boff = Ub;  // free during the down phase
+                        const int tot = dl_offsets(dc, Bq, Boff, nrows, I.off, &s_tot);
+                        const int nblk = (tot + kDlEntries - 1) / kDlEntries;
+                        trace(9, nrows, tot);
+                        if (tid == 0) {
+                            HelpCtx cx;
+                            cx.root_slot = slot;
+                            cx.l = L;
+                            cx.g0 = g0;
+                            cx.lim = lim;
+                            cx.cnt = nrows;
+                            cx.nblocks = nblk;
+                            cx.E2 = tot;
+                            cx.E = E;
+                            cx.kind = 4;
+                            cx.lb = lb;
+                            cx.mvalid = mvalid;
+                            a.help.ctx[wk] = cx;
+                            a.help.done[wk] = 0;
+                            a.help.gapp[wk] = s_dcnt;
+                            a.help.low[wk] = 0;
+                            __threadfence();
+                            atomicAdd(a.stats + kStHelpReq, 1ull);
+                            atomicAdd(a.stats + kStHelpBlkAll, (unsigned long long)nblk);
+                            hseq = (hseq + 1) & 0xFFFF;
+                            atomicExch(a.help.word + wk, help_pack(1, nblk, 0, hseq));
+                            if (nblk >= a.busy_min) atomicAdd(a.help.roots_left + 1, 1);
+                        }
+                        for (;;) {  // the owner takes blocks too
+                            if (tid == 0) {
+                                const unsigned long long w = atomicAdd(a.help.word + wk, 1ull << 16);
+                                s_hb = help_next(w) < nblk ? help_next(w) : -1;
+                            }
+                            __syncthreads();
+                            const int b = s_hb;
+                            __syncthreads();
+                            if (b < 0) break;
+                            ++own_blk;
+                            dl_block<false>(gd, S, Bq, Boff, nrows, b * kDlEntries, min(tot, (b + 1) * kDlEntries),
+                                            dacc, &s_t0, st_bytes, sc_down);  // ends with a barrier
+                            if (tid == 0) {
+                                __threadfence();
+                                atomicAdd(a.help.done + wk, 1);
+                            }
+                        }
+                        trace(6, 4, own_blk | (nblk << 16));
+                        own_blk = 0;
+                        if (tid == 0) {  // wait for the helpers' blocks, then close
+                            while (atomicAdd(a.help.done + wk, 0) < nblk) __nanosleep(256);
+                            atomicExch(a.help.word + wk, help_pack(0, 0, 0, hseq));
+                            if (nblk >= a.busy_min) atomicSub(a.help.roots_left + 1, 1);
                             __threadfence();
                             s_dcnt = __ldcg(a.help.gapp + wk);
                             if (__ldcg(a.help.low + wk)) s_job[3] = 1;
                         }
                         __syncthreads();
-                    } else {
-                        dc_small(dc, 0, items, enq_front, st_bytes, sc_down);
-                        __syncthreads();
-                        dc_big(dc, S, Bq, s_nbig, st_bytes, sc_down);
+                        dl_finish(dc, Bq, nrows, dacc, st_bytes);  // ends with a barrier
+                    } else if (nrows > 0) {
+                        dc_big(dc, S, Bq, nrows, st_bytes, sc_down);
                     }
                     if (L < Lseed) {  // seeds of the next level (claimed children stay once)
                         inject(L + 1);
@@ -724,6 +1258,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                     __syncthreads();  // everyone has read nbig / ne
                     if (tid == 0) {
                         s_nbig = 0;
+                        s_hopen = hopen_pf;
                         if (ne != le || L < Lseed) Doff[nlev + 1] = ne;
                     }
                     __syncthreads();  // reset visible before the next level enqueues
@@ -781,66 +1316,88 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
 
                 tick(0);
                 // ================= (0) Case-3 removal pushes =================
+                trace(3, 0, dtotal);
                 if (case3) {
-                    // a pulled-up w (finite old level od) loses its old predecessors x
-                    auto rem_visit = [&](int w, int od, double osig, double coef, int x, int dx,
-                                         double sx) {
-                        if (dx != od - 1) return;
-                        if (mark[x] == mD) return;
-                        if (ldg_i(g.rp + w) < 0 && new_edge(g, w, x, g0, lim)) return;  // not an old predecessor
-                        atomicAdd(dacc + x, -__ddiv_rn(coef, osig));
-                        (void)sx;
-                        st_bytes += 24;
-                        if (atomicMax(mark + x, mU) < E) {
-                            const int pos = atomicAdd(&s_rcnt, 1);
-                            Rv[pos] = x;
-                            Rl[pos] = od - 1;
-                            atomicMax(&s_rmax, od - 1);
+                    RemCtx rc;
+                    rc.g = g;
+                    rc.st = st;
+                    rc.mark = mark;
+                    rc.dacc = dacc;
+                    rc.Dv = Dv;
+                    rc.Dold = Dold;
+                    rc.Dsig = Dsig;
+                    rc.Rv = Rv;
+                    rc.Rl = Rl;
+                    rc.rcnt = &s_rcnt;
+                    rc.rmax = &s_rmax;
+                    rc.g0 = g0;
+                    rc.lim = lim;
+                    rc.E = E;
+                    rc.mD = mD;
+                    rc.mU = mU;
+                    const int kRemBlock = a.hd_block;
+                    if (a.help.word && dtotal >= a.hd_min) {
+                        // a wide pass: published, idle and busy workers take blocks of D
+                        // (appends to R and the deepest target level go through global memory)
+                        const int nblk = (dtotal + kRemBlock - 1) / kRemBlock;
+                        if (tid == 0) {
+                            HelpCtx cx;
+                            cx.root_slot = slot;
+                            cx.l = 0;
+                            cx.g0 = g0;
+                            cx.lim = lim;
+                            cx.cnt = dtotal;
+                            cx.nblocks = nblk;
+                            cx.E2 = 0;
+                            cx.E = E;
+                            cx.kind = 3;
+                            cx.lb = 0;
+                            cx.mvalid = 0;
+                            a.help.ctx[wk] = cx;
+                            a.help.done[wk] = 0;
+                            a.help.gapp[wk] = s_rcnt;
+                            a.help.low[wk] = s_rmax;
+                            __threadfence();
+                            atomicAdd(a.stats + kStHelpReq, 1ull);
+                            atomicAdd(a.stats + kStHelpBlkAll, (unsigned long long)nblk);
+                            hseq = (hseq + 1) & 0xFFFF;
+                            atomicExch(a.help.word + wk, help_pack(1, nblk, 0, hseq));
+                            if (nblk >= a.busy_min) atomicAdd(a.help.roots_left + 1, 1);  // open wide requests
                         }
-                    };
-                    split_pass(
-                        dtotal, g, lim,
-                        [&](int i, int &w) {
-                            const int od = Dold[i] & kOldMask;
-                            w = Dv[i];
-                            return od != kInf && od != st.dist(w);
-                        },
-                        [&](int i, int w, int2 r) {
-                            const int od = Dold[i] & kOldMask;
-                            const double osig = Dsig[i];
-                            const double coef = 1.0 + st.sd[w].y;  // delta still old
-                            row_walk(g, st, nullptr, r, [&](int dx) { return dx == od - 1; },
-                                     [&](int x, int dx, double2 q, uint32_t) {
-                                         rem_visit(w, od, osig, coef, x, dx, q.x);
-                                     });
-                            st_bytes += 16 + 8ull * (r.y - r.x);
-                            sc_rem += r.y - r.x;
-                        },
-                        enq_front);
-                    __syncthreads();
-                    const int nbig = s_nbig;
-                    for (int r0 = 0; r0 < nbig; r0 += kBig) {
-                        const int m = min(kBig, nbig - r0);
-                        big_load(S, m, [&](int t) { return Bq[r0 + t]; }, [&](int i) { return Dv[i]; },
-                                 g, lim);
-                        if (tid < m) {
-                            const int i = S.idx[tid];
-                            S.c0[tid] = Dsig[i];
-                            s_l1[tid] = Dold[i] & kOldMask;  // reused: old level of each row
-                            st_bytes += 16;
+                        RemCtx gr = rc;
+                        gr.rcnt = a.help.gapp + wk;
+                        gr.rmax = a.help.low + wk;
+                        for (;;) {  // the owner takes blocks too
+                            if (tid == 0) {
+                                const unsigned long long w = atomicAdd(a.help.word + wk, 1ull << 16);
+                                s_hb = help_next(w) < nblk ? help_next(w) : -1;
+                            }
+                            __syncthreads();
+                            const int b = s_hb;
+                            __syncthreads();
+                            if (b < 0) break;
+                            ++own_blk;
+                            rem_range(gr, S, s_l1, Bq, &s_nbig, b * kRemBlock, min(dtotal, (b + 1) * kRemBlock),
+                                      st_bytes, sc_rem);  // ends with a barrier
+                            if (tid == 0) {
+                                __threadfence();
+                                atomicAdd(a.help.done + wk, 1);
+                            }
+                        }
+                        trace(6, 3, own_blk | (nblk << 16));
+                        own_blk = 0;
+                        if (tid == 0) {  // wait for the helpers' blocks, then close
+                            while (atomicAdd(a.help.done + wk, 0) < nblk) __nanosleep(256);
+                            atomicExch(a.help.word + wk, help_pack(0, 0, 0, hseq));
+                            if (nblk >= a.busy_min) atomicSub(a.help.roots_left + 1, 1);
+                            __threadfence();
+                            s_rcnt = __ldcg(a.help.gapp + wk);
+                            s_rmax = __ldcg(a.help.low + wk);
                         }
                         __syncthreads();
-                        big_entries(S, g, st, [](int) { return true; }, [&](int t, int x, int dx, double2 q) {
-                            st_bytes += 8;
-                            sc_rem++;
-                            const int w = S.v[t];
-                            rem_visit(w, s_l1[t], S.c0[t], 1.0 + st.sd[w].y, x, dx, q.x);
-                            return 0.0;
-                        });
+                    } else {
+                        rem_range(rc, S, s_l1, Bq, &s_nbig, 0, dtotal, st_bytes, sc_rem);
                     }
-                    __syncthreads();
-                    if (tid == 0) s_nbig = 0;
-                    __syncthreads();
                 }
                 const int rcnt = s_rcnt;
                 // a deletion's removal targets can sit one level above the seeds (u_high)
@@ -855,6 +1412,9 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                 int ucnt = 0;
                 for (int l = Lmax; l >= 1; --l) {
                     if (l < Lstop && ucnt == 0) break;  // nothing left above the insertion
+                    busy_help();
+                    const int hopen_pf = sample_open();
+                    trace(2, l, ucnt + rcnt + ((l >= L0 && l <= LmaxD) ? Doff[l - L0 + 1] - Doff[l - L0] : 0));
                     const bool push = l >= 2;          // level-1 vertices only feed the root
                     ++st_lvu;
                     // queue p for level l-1 unless already queued: the prefetched mark
@@ -1150,6 +1710,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                     atomicAdd(a.stats + kStHelpBlkAll, (unsigned long long)nblk1);
                                     hseq = (hseq + 1) & 0xFFFF;
                                     atomicExch(a.help.word + wk, help_pack(1, nblk1, 0, hseq));
+                                    if (nblk1 >= a.busy_min) atomicAdd(a.help.roots_left + 1, 1);  // open wide requests
                                 }
                                 for (;;) {  // the owner takes blocks too
                                     if (tid == 0) {
@@ -1160,12 +1721,16 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                     const int b = s_hb;
                                     __syncthreads();
                                     if (b < 0) break;
+                                    ++own_blk;
                                     c1_pass(b * a.he_entries, min(E1, (b + 1) * a.he_entries));  // ends with a barrier
                                     if (tid == 0) atomicAdd(a.help.done + wk, 1);
                                 }
+                                trace(6, 2, own_blk | (nblk1 << 16));
+                                own_blk = 0;
                                 if (tid == 0) {  // wait for the helpers' blocks, then close
                                     while (atomicAdd(a.help.done + wk, 0) < nblk1) __nanosleep(256);
                                     atomicExch(a.help.word + wk, help_pack(0, 0, 0, hseq));
+                                    if (nblk1 >= a.busy_min) atomicSub(a.help.roots_left + 1, 1);
                                     __threadfence();
                                 }
                                 __syncthreads();
@@ -1234,6 +1799,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                     atomicAdd(a.stats + kStHelpBlkAll, (unsigned long long)nblk);
                                     hseq = (hseq + 1) & 0xFFFF;
                                     atomicExch(a.help.word + wk, help_pack(1, nblk, 0, hseq));
+                                    if (nblk >= a.busy_min) atomicAdd(a.help.roots_left + 1, 1);  // open wide requests
                                 }
                                 int32_t *gU = a.help.gU + (size_t)wk * n;
                                 int *gapp = a.help.gapp + wk;
@@ -1246,6 +1812,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                     const int b = s_hb;
                                     __syncthreads();
                                     if (b < 0) break;
+                                    ++own_blk;
                                     help_run_block<false>(I, b * a.he_entries, min(E2, (b + 1) * a.he_entries), g,
                                                           st, mark, dacc, gU, gapp, cx, st_bytes);
                                     __syncthreads();  // (help_run_block ends with one too)
@@ -1254,9 +1821,12 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                         atomicAdd(a.help.done + wk, 1);
                                     }
                                 }
+                                trace(6, 0, own_blk | (nblk << 16));
+                                own_blk = 0;
                                 if (tid == 0) {  // wait for the helpers' blocks, then close
                                     while (atomicAdd(a.help.done + wk, 0) < nblk) __nanosleep(256);
                                     atomicExch(a.help.word + wk, help_pack(0, 0, 0, hseq));
+                                    if (nblk >= a.busy_min) atomicSub(a.help.roots_left + 1, 1);
                                     __threadfence();
                                 }
                                 __syncthreads();
@@ -1337,6 +1907,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                             s_nbigI = 0;
                             s_nl1 = 0;
                             s_noext = 0;
+                            s_hopen = hopen_pf;
                         }
                         __syncthreads();
                     }  // chunks
@@ -1356,6 +1927,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                                                        ((st_touched - touch0) << 2) |
                                                                        (s_wcnt[1] ? 3u : 2u));
             }
+            trace(4, 0, 0);
             ins = wend;
             __syncthreads();  // the counters are reset by the next window
         }
@@ -1372,144 +1944,13 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
             rp4[5] = st_lvd + st_lvu - prof_lv0;
         }
     }
-    // ---- out of roots: help the C2 passes of workers still running ----
+    // ---- out of roots: help the passes of workers still running ----
     if (a.help.word) {
         int cur_owner = -1, cur_seq = -1;
         for (;;) {
-            // the whole CTA scans the board (one word per thread), first open one wins
-            if (tid == 0) s_hpick = INT32_MAX;
-            __syncthreads();
-            {
-                const int nw = a.help.nworkers;
-                for (int i = tid; i < nw; i += kBlock) {
-                    const int o = (wk + 1 + i) % nw;
-                    const unsigned long long w = __ldcg(a.help.word + o);
-                    if (help_open(w) && help_next(w) < help_nblocks(w)) atomicMin(&s_hpick, i);
-                }
-            }
-            __syncthreads();
-            if (tid == 0) {
-                int pick = -1, b = -1, sq = -1;
-                if (atomicAdd(a.help.roots_left, 0) <= 0) {
-                    pick = -2;
-                } else {
-                    if (s_hpick != INT32_MAX) pick = (wk + 1 + s_hpick) % a.help.nworkers;
-                    if (pick >= 0) {
-                        const unsigned long long w = atomicAdd(a.help.word + pick, 1ull << 16);
-                        if (help_open(w) && help_next(w) < help_nblocks(w)) {
-                            b = help_next(w);
-                            sq = help_seq(w);
-                        }
-                    }
-                }
-                s_hpick = pick;
-                s_hb = b;
-                s_hseq = sq;
-            }
-            __syncthreads();
-            const int pick = s_hpick, b = s_hb, sq = s_hseq;
-            __syncthreads();
-            if (pick == -2) break;
-            if (b < 0) {
-                __nanosleep(1000);
-                continue;
-            }
-            if (pick != cur_owner || sq != cur_seq) {  // a new request: load its chunk
-                if (tid == 0) {
-                    const HelpCtx *src = a.help.ctx + pick;
-                    s_hctx.root_slot = __ldcg(&src->root_slot);
-                    s_hctx.l = __ldcg(&src->l);
-                    s_hctx.g0 = __ldcg(&src->g0);
-                    s_hctx.lim = __ldcg(&src->lim);
-                    s_hctx.cnt = __ldcg(&src->cnt);
-                    s_hctx.nblocks = __ldcg(&src->nblocks);
-                    s_hctx.E2 = __ldcg(&src->E2);
-                    s_hctx.E = __ldcg(&src->E);
-                    s_hctx.kind = __ldcg(&src->kind);
-                    s_hctx.lb = __ldcg(&src->lb);
-                    s_hctx.mvalid = __ldcg(&src->mvalid);
-                    __threadfence();  // acquire: drop stale L1 lines of the owner's state
-                }
-                __syncthreads();
-                const ChunkSmem *mir = a.help.mir + pick;
-                const int cnt = s_hctx.kind != 1 ? s_hctx.cnt : 0;  // kinds 0 and 2 publish a chunk
-                if (s_hctx.kind == 1 && s_hctx.mvalid && tid < 32) {  // the root's row (mask bits)
-                    const int2 rs = row_of(g, a.roots[s_hctx.root_slot], s_hctx.lim);
-                    const int ds = rs.y - rs.x;
-                    if (tid < ds && ds <= kMaskDeg) s_adjs[tid] = ldg_i(g.col + rs.x + tid);
-                    if (tid == 0) s_job[5] = ds;
-                }
-                for (int t = tid; t < cnt; t += kBlock) {
-                    I.v[t] = __ldcg(&mir->v[t]);
-                    I.meta[t] = __ldcg(&mir->meta[t]);
-                    I.beg[t] = __ldcg(&mir->beg[t]);
-                    I.off[t + 1] = __ldcg(&mir->off[t + 1]);
-                    I.acc[t] = __ldcg(&mir->acc[t]);
-                    I.c0[t] = __ldcg(&mir->c0[t]);
-                    I.c1[t] = __ldcg(&mir->c1[t]);
-                    I.c2[t] = __ldcg(&mir->c2[t]);
-                }
-                if (tid == 0) I.off[0] = 0;
-                __syncthreads();
-                cur_owner = pick;
-                cur_seq = sq;
-            }
-            const HelpCtx cx = s_hctx;
-            const Root ost{a.d + (size_t)cx.root_slot * n, a.sd + (size_t)cx.root_slot * n};
-            if (cx.kind == 1) {  // a block of a published down-phase level
-                const int kDownBlock = a.hd_block;
-                DownCtx hd;
-                hd.g = g;
-                hd.st = ost;
-                hd.mark = a.ws.mark + (size_t)pick * n;
-                hd.lowrec = a.ws.lowrec + (size_t)pick * n;
-                hd.Dv = a.ws.Dv + (size_t)pick * n;
-                hd.Dold = a.ws.Dold + (size_t)pick * n;
-                hd.Dsig = a.ws.Dsig + (size_t)pick * n;
-                hd.mask = a.l2mask + (size_t)cx.root_slot * n;
-                hd.err = a.err;
-                hd.dcnt = a.help.gapp + pick;
-                hd.lowflag = a.help.low + pick;
-                hd.adjs = s_adjs;
-                hd.dsr = s_job[5];
-                hd.L = cx.l;
-                hd.lb = cx.lb;
-                hd.lim = cx.lim;
-                hd.mvalid = cx.mvalid;
-                hd.del = a.del;
-                hd.epoch = cx.E >> 2;
-                hd.mD = cx.E | kDown;
-                int32_t *Bqh = a.ws.Bq + (size_t)wk * n;
-                dc_small(hd, b * kDownBlock, min(cx.cnt, (b + 1) * kDownBlock),
-                         [&](int idx) { Bqh[atomicAdd(&s_nbig, 1)] = idx; }, st_bytes, sc_down);
-                __syncthreads();
-                dc_big(hd, S, Bqh, s_nbig, st_bytes, sc_down);
-                if (tid == 0) s_nbig = 0;
-            } else if (cx.kind == 2) {  // a block of a published delta-pull pass (C1)
-                const int e0 = b * a.he_entries, e1 = min(cx.E2, (b + 1) * a.he_entries);
-                for (int t = tid; t < cx.cnt; t += kBlock) I.acc[t] = 0.0;
-                __syncthreads();
-                auto colf = [&](int t, int e) { return ldg_i(g.col + I.beg[t] + e - I.off[t]); };
-                flat_entries<true>(I.off, cx.cnt, e1, colf, ost, nullptr, [&](int dy) { return dy == cx.l + 1; },
-                                   I.acc, [&](int t, int, int dy, double2 q, uint32_t) -> double {
-                                       st_bytes += 8;
-                                       if (dy != cx.l + 1) return 0.0;
-                                       return __dmul_rn(__ddiv_rn(I.c0[t], q.x), __dadd_rn(1.0, q.y));
-                                   }, e0);
-                ChunkSmem *mir = a.help.mir + pick;
-                for (int t = tid; t < cx.cnt; t += kBlock)
-                    if (I.acc[t] != 0.0) atomicAdd(&mir->acc[t], I.acc[t]);
-            } else {
-                help_run_block<true>(I, b * a.he_entries, min(cx.E2, (b + 1) * a.he_entries), g, ost,
-                                     a.ws.mark + (size_t)pick * n, a.ws.dacc + (size_t)pick * n,
-                                     a.help.gU + (size_t)pick * n, a.help.gapp + pick, cx, st_bytes);
-            }
-            __syncthreads();
-            if (tid == 0) {  // release by one thread after the CTA barrier
-                __threadfence();
-                atomicAdd(a.help.done + pick, 1);
-                atomicAdd(a.stats + kStHelpBlk, 1ull);
-            }
+            const int r = help_step(true, cur_owner, cur_seq);
+            if (r == -2) break;
+            if (r < 0) __nanosleep(1000);
         }
     }
     if (tid == 0) {

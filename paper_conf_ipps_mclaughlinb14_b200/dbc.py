@@ -271,10 +271,22 @@ class DynamicBC:
                  "ns_down", "ns_removal", "ns_up_setup", "ns_up_epi", "ns_up_l1pairs", "ns_up_end",
                  "ns_up_split", "ns_up_scan", "ns_up_pull", "ns_up_push", "levels_down", "levels_up",
                  "help_requests", "help_blocks_by_helpers", "help_blocks_all",
-                 "case2_groups", "case2_group_insertions"]
+                 "case2_groups", "case2_group_insertions", "help_blocks_busy"]
         out = np.zeros(len(names), dtype=np.int64)
         _check(self._ctx, self._lib.dbc_debug_counters(self._ctx, _np_ptr(out), out.size))
         return dict(zip(names, out.tolist()))
+
+    def debug_trace(self):
+        """Per-level event trace of the slot named by DBC_TRACE_SLOT (builds with
+        -DDBC_PHASE_TIMERS only): list of (kind, level, items, t_ns); kinds 1 down
+        level, 2 up level, 3 removal pass, 4 job end."""
+        base = 32  # kStTraceN (after the debug_counters names)
+        out = np.zeros(base + 1 + 2 * 1024, dtype=np.int64)
+        _check(self._ctx, self._lib.dbc_debug_counters(self._ctx, _np_ptr(out), out.size))
+        cnt = min(int(out[base]), 1024)
+        ev = out[base + 1: base + 1 + 2 * cnt].reshape(-1, 2).astype(np.uint64)
+        return [(int(c >> np.uint64(56)), int((c >> np.uint64(32)) & np.uint64(0xFFFFFF)),
+                 int(c & np.uint64(0xFFFFFFFF)), int(t)) for c, t in ev]
 
     def root_profile(self, enable=True, read=True):
         out = np.zeros((self.num_local_roots(), 6), dtype=np.int64) if read else None

@@ -1,0 +1,11 @@
+#!/bin/bash
+# helped removal pass (kind 3) + busy help: parity + bench
+O=gpurun_out/r24; mkdir -p $O
+timeout 900 python -m pytest tests -m gpu -q -x > $O/tests.log 2>&1; echo "rc=$?" >> $O/tests.log
+B="python bench.py --no-cpu-baseline --no-per-insertion --no-e2e --no-deletions"
+for bh in 1 4; do DBC_BUSY_HELP=$bh timeout 300 $B > $O/rmat16_bh$bh.json 2>> $O/err.txt; done
+timeout 300 $B --config delaunay18 > $O/del18.json 2>> $O/err.txt
+timeout 300 $B --config smallworld > $O/sw.json 2>> $O/err.txt
+timeout 600 $B --config kron20 --steps 3 --warmup 3 > $O/kron20.json 2>> $O/err.txt
+export DBC_LIB_PATH=$PWD/paper_conf_ipps_mclaughlinb14_b200/libdbc_timers.so
+DBC_TRACE_SLOT=38 PB_BATCHES=4 timeout 120 python -u tools/phase_breakdown.py rmat16 4000 > $O/pb_slot38.txt 2>&1

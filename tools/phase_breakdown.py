@@ -37,3 +37,13 @@ print("median root: slot", i, "deg", g.degree()[wl.roots[i]], "ms %.2f" % dur[i]
 print("jobs: median", np.median(prof[:,2]), "max", prof[:,2].max(), "touched/job median", np.median(prof[:,3]/np.maximum(prof[:,2],1)))
 st = (prof[:, 0] - prof[:, 0].min()) / 1e6
 print("root start ms: min %.2f median %.2f max %.2f; #late(>1ms) %d" % (st.min(), np.median(st), st.max(), (st > 1).sum()))
+if os.environ.get("DBC_TRACE_SLOT"):
+    ev = dbc.debug_trace()
+    t0 = None
+    last = None
+    for kind, lev, items, t in ev:
+        if t0 is None:
+            t0 = t
+        dt = (t - last) / 1e3 if last is not None else 0.0
+        print("trace +%8.1f us (at %8.1f) %s level %d items %d%s" % (dt, (t - t0) / 1e3, {1: "down", 2: "up", 3: "removal", 4: "job-end", 6: "owner-blocks(kind; own|total<<16)", 9: "long-rows(rows; entries)"}.get(kind, "?"), lev, items, (" own %d of %d" % (items & 0xFFFF, items >> 16)) if kind == 6 else ""))
+        last = t
