@@ -702,3 +702,32 @@ def test_heavy_lane_with_help_completes_rmat16(rep):
         for i, s in enumerate(range(0, wl.roots.size, 37)):
             d, sg, _ = dbc.get_root_state(s)
             assert np.array_equal(d, dyn[i][0]) and np.array_equal(sg, dyn[i][1])
+
+
+@pytest.mark.parametrize("name", ["rmat10", "delaunay12u", "smallworld"])
+def test_forced_help_paths_match_oracle(name, monkeypatch):
+    """Every cooperative path forced on at small sizes: helped down levels
+    (kind 1, 32-item blocks), entry-balanced long rows of every down level
+    (kind 4), the Case-3 removal pass as help blocks (kind 3), helped delta-pull
+    / push passes (kinds 2 / 0, 256-entry blocks), busy workers taking blocks of
+    any pass; several batches (heavy lanes).  d/sigma bit-exact vs the oracle,
+    BC within tolerance."""
+    for k, v in {"DBC_HDMIN": "1", "DBC_HDBLK": "32", "DBC_DLMIN": "1", "DBC_HEMIN": "1",
+                 "DBC_HEENT": "256", "DBC_BUSY_MIN": "1", "DBC_BUSY_HELP": "4",
+                 "DBC_HEAVY_FACTOR": "1.0"}.items():
+        monkeypatch.setenv(k, v)
+    wl = W.make_workload(name)
+    ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
+    with _dbc(wl.graph, wl.roots) as dbc:
+        dbc.static_compute()
+        c0 = dbc.debug_counters()
+        nb = 3
+        step = (wl.ins_u.size + nb - 1) // nb
+        for b in range(nb):
+            sl = slice(b * step, (b + 1) * step)
+            dbc.insert_edges(wl.ins_u[sl], wl.ins_v[sl])
+            for u, v in zip(wl.ins_u[sl], wl.ins_v[sl]):
+                ref.insert(u, v)
+        c1 = dbc.debug_counters()
+        check_all(dbc, ref.compute(), wl.roots.size)
+        assert c1["help_requests"] > c0["help_requests"]
