@@ -506,7 +506,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->help.mir, nwk);
     AL(c->help.gapp, nwk);
     AL(c->help.gU, wn);
-    AL(c->help.roots_left, 4);  // [0] live counter, [1] open requests, [2..3] = {k_loc, 0}
+    AL(c->help.roots_left, 6);  // [0] live counter, [1] open wide requests, [2] idle workers, [3..5] = {k_loc, 0, 0}
     AL(c->help.low, nwk);
     AL(c->help.gbig, 2 * nwk);
     c->help.nworkers = (int)nwk;
@@ -517,7 +517,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->err, 1);
     AL(c->root_prof, (size_t)6 * std::max(c->k_loc, 1));
     {
-        const int kl[4] = {0, 0, c->k_loc, 0};
+        const int kl[6] = {0, 0, 0, c->k_loc, 0, 0};
         if (cudaMemcpy(c->help.roots_left, kl, sizeof(kl), cudaMemcpyHostToDevice) != cudaSuccess)
             return bail(fail(c, DBC_ECUDA, "roots_left init"));
     }
@@ -801,7 +801,7 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
             if (c->help_on) {  // fresh board: all requests closed, every root chain pending
                 a.help = c->help;
                 CK(cudaMemsetAsync(c->help.word, 0, sizeof(unsigned long long) * c->help.nworkers, c->stream));
-                CK(cudaMemcpyAsync(c->help.roots_left, c->help.roots_left + 2, 2 * sizeof(int),
+                CK(cudaMemcpyAsync(c->help.roots_left, c->help.roots_left + 3, 3 * sizeof(int),
                                    cudaMemcpyDeviceToDevice, c->stream));  // no host sync per batch
             }
             if (nh > 0) {  // heavy lane first, on the high-priority stream

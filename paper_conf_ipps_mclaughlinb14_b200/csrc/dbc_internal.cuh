@@ -511,8 +511,8 @@ struct HelpBoard {
     ChunkSmem *mir;            // [workers]
     int *gapp;                 // [workers] global append counters
     int32_t *gU;               // [workers][n] global append lists
-    int *roots_left;           // [0] root chains not yet finished (both lanes), [1] open requests,
-                               // [2..3] = {k_loc, 0}: the per-batch reset source of [0..1]
+    int *roots_left;           // [0] root chains not yet finished (both lanes), [1] open wide requests,
+                               // [2] idle workers, [3..5] = {k_loc, 0, 0}: the per-batch reset source
     int *low;                  // [workers] kind 1: a distance was lowered in the helped level;
                                // kind 3: deepest removal-target level
     int nworkers;

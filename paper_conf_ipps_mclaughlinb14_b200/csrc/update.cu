@@ -56,7 +56,7 @@ constexpr int32_t kExtPred = INT32_MIN;
 __device__ __forceinline__ void help_push_entry(const GView &g, const ChunkSmem &M, int t, int pp, int dp,
                                                 double sp, uint32_t mp, const HelpCtx &cx, uint32_t *mark,
                                                 double *dacc, int32_t *gU, int *gapp,
-                                                unsigned long long &bytes) {
+                                                uint32_t &bytes) {
     if (dp != cx.l - 1) return;
     const uint32_t E = cx.E, mD = E | kDown, mU = E | kUp;
     const int meta = M.meta[t];
@@ -82,7 +82,7 @@ __device__ __forceinline__ void help_push_entry(const GView &g, const ChunkSmem 
 template <bool kCG>
 __device__ __forceinline__ void help_run_block(const ChunkSmem &M, int e0, int e1, const GView &g,
                                                const Root &st, uint32_t *mark, double *dacc, int32_t *gU,
-                                               int *gapp, const HelpCtx &cx, unsigned long long &bytes) {
+                                               int *gapp, const HelpCtx &cx, uint32_t &bytes) {
     auto colf = [&](int t, int e) { return ldg_i(g.col + M.beg[t] + e - M.off[t]); };
     flat_entries<kCG, false>(
         M.off, cx.cnt, e1, colf, st, mark, [&](int dp) { return dp == cx.l - 1; }, nullptr,
@@ -123,7 +123,7 @@ __device__ __forceinline__ uint32_t dc_l1bit(const DownCtx &c, int y) {
 // per-D-entry epilogue: record old d / sigma, store the new sigma (and, at
 // level 2, the vertex's level-1 predecessor mask)
 __device__ __forceinline__ void dc_finish(const DownCtx &c, int idx, int w, double sum, uint32_t m, bool ext,
-                                          unsigned long long &bytes) {
+                                          uint32_t &bytes) {
     if (c.mvalid && c.L == 2) c.mask[w] = m;
     const unsigned long long lr = c.lowrec[w];
     const int od = ((uint32_t)(lr >> 32) == c.epoch) ? (int)(uint32_t)lr : c.L;
@@ -135,7 +135,7 @@ __device__ __forceinline__ void dc_finish(const DownCtx &c, int idx, int w, doub
 }
 
 // one neighbour y of a level-L vertex; returns sigma[y] if y is a predecessor
-__device__ __forceinline__ double dc_visit(const DownCtx &c, int y, int dy, double sy, unsigned long long &bytes) {
+__device__ __forceinline__ double dc_visit(const DownCtx &c, int y, int dy, double sy, uint32_t &bytes) {
     const int L = c.L;
     if (dy == L - 1) {
         bytes += 8;
@@ -157,8 +157,8 @@ __device__ __forceinline__ double dc_visit(const DownCtx &c, int y, int dy, doub
 // short rows of items [i0, i1) walked in-lane in canonical order (bit-exact
 // sigma); long rows handed to enq(item, length)
 template <class Enq>
-__device__ __forceinline__ void dc_small(const DownCtx &c, int i0, int i1, Enq enq, unsigned long long &bytes,
-                                         unsigned long long &scanned) {
+__device__ __forceinline__ void dc_small(const DownCtx &c, int i0, int i1, Enq enq, uint32_t &bytes,
+                                         uint32_t &scanned) {
     const int L = c.L, mD = c.mD;
     for (int i = i0 + (int)threadIdx.x; i < i1; i += kBlock) {
         const int w = c.Dv[c.lb + i];
@@ -221,7 +221,7 @@ __device__ __forceinline__ void dc_small(const DownCtx &c, int i0, int i1, Enq e
 // S, entries flattened over the CTA.  Caller: barrier before (queue complete);
 // ends with a barrier.
 __device__ __forceinline__ void dc_big(const DownCtx &c, BigSmem &S, const int32_t *Bq, int nbig,
-                                       unsigned long long &bytes, unsigned long long &scanned) {
+                                       uint32_t &bytes, uint32_t &scanned) {
     const int tid = threadIdx.x, L = c.L;
     for (int r0 = 0; r0 < nbig; r0 += kBig) {
         const int m = min(kBig, nbig - r0);
@@ -277,7 +277,7 @@ struct RemCtx {
 };
 
 __device__ __forceinline__ void rem_visit(const RemCtx &c, int w, int od, double osig, double coef, int x,
-                                          int dx, unsigned long long &bytes) {
+                                          int dx, uint32_t &bytes) {
     if (dx != od - 1) return;
     if (c.mark[x] == c.mD) return;
     if (ldg_i(c.g.rp + w) < 0 && new_edge(c.g, w, x, c.g0, c.lim)) return;  // not an old predecessor
@@ -292,8 +292,8 @@ __device__ __forceinline__ void rem_visit(const RemCtx &c, int w, int od, double
 }
 
 __device__ __forceinline__ void rem_range(const RemCtx &c, BigSmem &S, int *s_old, int32_t *Bq, int *nbig,
-                                          int i0, int i1, unsigned long long &bytes,
-                                          unsigned long long &scanned) {
+                                          int i0, int i1, uint32_t &bytes,
+                                          uint32_t &scanned) {
     const int tid = threadIdx.x;
     split_pass(
         i1 - i0, c.g, c.lim,
@@ -386,7 +386,7 @@ __device__ __forceinline__ int dl_offsets(const DownCtx &c, int32_t *Bq, int32_t
 template <bool kCG>
 __device__ __forceinline__ void dl_block(const DownCtx &c, BigSmem &S, int32_t *Bq, const int32_t *Boff,
                                          int nrows, int e0, int e1, double *dacc, int *s_t0,
-                                         unsigned long long &bytes, unsigned long long &scanned) {
+                                         uint32_t &bytes, uint32_t &scanned) {
     const int tid = threadIdx.x, L = c.L;
     // first row: last t with Boff[t] <= e0 (two strided probes over the CTA)
     if (tid == 0) *s_t0 = 0;
@@ -476,7 +476,7 @@ __device__ __forceinline__ void dl_block(const DownCtx &c, BigSmem &S, int32_t *
 
 // owner: complete the long rows after every block ran
 __device__ __forceinline__ void dl_finish(const DownCtx &c, const int32_t *Bq, int nrows, double *dacc,
-                                          unsigned long long &bytes) {
+                                          uint32_t &bytes) {
     const int L = c.L;
     for (int t = threadIdx.x; t < nrows; t += kBlock) {
         const uint32_t q = (uint32_t)__ldcg(Bq + t);
@@ -523,6 +523,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
     __shared__ int s_hadjs[kMaskDeg], s_hds;  // helped down level: the owner's root row (mask bits)
     __shared__ int s_hopen;                   // open requests seen at the last level boundary
     __shared__ int s_nent, s_tot, s_t0;        // long rows of a down level: entries, offsets total, first row
+    __shared__ int s_stg[3];                  // helped down block: staged long rows, their entries, base
     __shared__ int s_del[6];     // deletion job: [0] u_high, [1] u_low, [2] |A|, [3] seeds, [4] candidates, [5] u_low keeps a predecessor
     __shared__ double s_delsd[2];  // deletion job: old sigma / delta of u_low
 
@@ -548,9 +549,16 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
     const GView &g = a.g;
     int hseq = 0;  // this worker's help-request sequence
 
-    unsigned long long st_bytes = 0, st_touched = 0, st_down = 0;
-    unsigned long long st_c1 = 0, st_c2 = 0, st_c3 = 0, st_lvd = 0, st_lvu = 0;
-    unsigned long long sc_down = 0, sc_rem = 0, sc_dpull = 0, sc_dpush = 0, sc_up2 = 0, sc_up3 = 0;
+    // diagnostic counters: per-thread bytes / entries scanned in 32 bits (one
+    // launch moves < 4 GB per thread), thread 0's tallies in shared memory --
+    // registers are the occupancy limit of this kernel
+    uint32_t st_bytes = 0;
+    uint32_t sc_down = 0, sc_rem = 0, sc_dpull = 0, sc_dpush = 0, sc_up2 = 0, sc_up3 = 0;
+    __shared__ unsigned long long s_st[7];    // touched, down, case 1/2/3, level steps down/up (thread 0)
+    __shared__ unsigned long long s_touch0;   // touched count at the job start (scenario log)
+    __shared__ unsigned long long s_prof[5];  // root profile: t0, jobs, touched0, scanned0, levels0 (thread 0)
+    if (tid == 0)
+        for (int q = 0; q < 7; ++q) s_st[q] = 0;
     // per-phase wall time seen by thread 0 (diagnostic)
     unsigned long long tm_ph[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
     unsigned long long tclk = 0;
@@ -585,6 +593,36 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
     // cur_seq) caches the chunk loaded into I -- valid only while this CTA runs
     // nothing else.  Returns -2 when every root chain is done (idle), -1 when
     // no block was taken, 1 after running one.
+    // one block of a helped down level (owner or helper): short rows in-lane;
+    // long rows staged in shared memory (I.v is free outside the up phase) and
+    // appended to the owner's queue oBq with one reservation per block
+    // (gb[0] rows, gb[1] their entries)
+    auto down_block = [&](const DownCtx &c, int i0, int i1, int32_t *oBq, int *gb) {
+        if (tid == 0) {
+            s_stg[0] = 0;
+            s_stg[1] = 0;
+        }
+        __syncthreads();
+        dc_small(c, i0, i1,
+                 [&](int i, int len) {
+                     const int q = atomicAdd(&s_stg[0], 1);
+                     if (q < kChunk)
+                         I.v[q] = i;
+                     else
+                         oBq[atomicAdd(gb, 1)] = i;
+                     atomicAdd(&s_stg[1], len);
+                 },
+                 st_bytes, sc_down);
+        __syncthreads();
+        const int m = min(s_stg[0], kChunk);
+        if (tid == 0) {
+            s_stg[2] = m ? atomicAdd(gb, m) : 0;
+            if (s_stg[1]) atomicAdd(gb + 1, s_stg[1]);
+        }
+        __syncthreads();
+        for (int i = tid; i < m; i += kBlock) oBq[s_stg[2] + i] = I.v[i];
+        __syncthreads();
+    };
     auto help_step = [&](bool idle, int &cur_owner, int &cur_seq) -> int {
         // the whole CTA scans the board (one word per thread), first open one wins
         // Priority: the request with the most blocks left (the widest pass of the
@@ -691,12 +729,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
             if (cx.kind == 1) {
                 const int kDownBlock = a.hd_block;
                 int *gb = a.help.gbig + 2 * pick;
-                dc_small(hd, b * kDownBlock, min(cx.cnt, (b + 1) * kDownBlock),
-                         [&](int i, int len) {
-                             oBq[atomicAdd(gb, 1)] = i;
-                             atomicAdd(gb + 1, len);
-                         },
-                         st_bytes, sc_down);
+                down_block(hd, b * kDownBlock, min(cx.cnt, (b + 1) * kDownBlock), oBq, gb);
             } else {
                 dl_block<true>(hd, S, oBq, a.ws.U1 + (size_t)pick * n, cx.cnt, b * kDlEntries,
                                min(cx.E2, (b + 1) * kDlEntries), a.ws.dacc + (size_t)pick * n, &s_t0, st_bytes,
@@ -755,14 +788,23 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
     // idle workers).  s_hopen was sampled during the previous level; every
     // thread reads the same value (written before a barrier).
     auto busy_help = [&]() {
-        if (!a.help.word || a.busy_help <= 0 || s_hopen <= 0) return;
+        if (!a.help.word || a.busy_help <= 0 || (s_hopen & 0xFFFF) == 0) return;
         int co = -1, cs = -1;
         for (int q = 0; q < a.busy_help; ++q) {
             if (help_step(false, co, cs) < 0) break;
             if (tid == 0) atomicAdd(a.stats + kStBusyBlk, 1ull);
         }
     };
-    auto sample_open = [&]() { return (tid == 0 && a.help.word) ? __ldcg(a.help.roots_left + 1) : 0; };
+    // sampled at a level start by thread 0, published at the level end:
+    // open wide requests (busy workers help) and idle workers (a pass is worth
+    // publishing only if someone can take its blocks)
+    auto sample_open = [&]() {
+        return (tid == 0 && a.help.word)
+                   ? min(__ldcg(a.help.roots_left + 1), 0xFFFF) | (min(__ldcg(a.help.roots_left + 2), 0x7FFF) << 16)
+                   : 0;
+    };
+    // publish a pass of nb blocks?  (idle helpers exist, or busy ones take passes this wide)
+    auto worth = [&](int nb) { return (s_hopen >> 16) > 0 || (a.busy_help > 0 && nb >= a.busy_min); };
 
 
     if (tid == 0) {
@@ -791,10 +833,15 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
         const int sroot = a.roots[slot];
         tick_on = a.trace_slot < 0 || a.trace_slot == slot;
         uint32_t *mask = a.l2mask + (size_t)slot * n;
-        unsigned long long prof_t0 = 0, prof_jobs = 0, prof_touch0 = st_touched;
-        const unsigned long long prof_sc0 = sc_down + sc_rem + sc_dpull + sc_dpush + sc_up2 + sc_up3;
-        const unsigned long long prof_lv0 = st_lvd + st_lvu;
-        if (a.root_prof && tid == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(prof_t0));
+        if (a.root_prof && tid == 0) {
+            unsigned long long t;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+            s_prof[0] = t;
+            s_prof[1] = 0;
+            s_prof[2] = s_st[0];
+            s_prof[3] = (unsigned long long)sc_down + sc_rem + sc_dpull + sc_dpush + sc_up2 + sc_up3;
+            s_prof[4] = s_st[5] + s_st[6];
+        }
 
         // Insertions are taken in windows (ws.wcap of them, or 1 with
         // DBC_FLAG_NO_MERGE).  A window is ONE job (R18): every
@@ -852,9 +899,9 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
             {
                 const int nw = s_wcnt[0], n3 = s_wcnt[1];
                 if (tid == 0) {
-                    st_c1 += nwin - nw;
-                    st_c2 += nw - n3;
-                    st_c3 += n3;
+                    s_st[2] += nwin - nw;
+                    s_st[3] += nw - n3;
+                    s_st[4] += n3;
                     st_bytes += 8ull * nwin;
                     if (nw > 1) {
                         atomicAdd(a.stats + kStGroups, 1ull);
@@ -871,8 +918,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
             {
                 if (a.del) ++epoch;  // deletion: one epoch for the affected-set search, one for the job
                 ++epoch;
-                ++prof_jobs;
-                const unsigned long long touch0 = st_touched;  // scenario log (thread 0's counter)
+                if (tid == 0) ++s_prof[1];
+                if (tid == 0) s_touch0 = s_st[0];  // scenario log (thread 0's counter)
                 const uint32_t E = epoch << 2;
                 const uint32_t mD = E | kDown, mU = E | kUp;
                 // the job's insertions and the graph as of lim; a deletion sees
@@ -946,8 +993,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                             s_del[2] = 1;
                             s_job[3] = 1;
                             s_wcnt[1] = 1;  // a distance changes: reported as Case 3
-                            --st_c2;
-                            ++st_c3;
+                            --s_st[3];
+                            ++s_st[4];
                         }
                         __syncthreads();
                         int fb = 0, fe = 1, la = Lul;
@@ -1097,7 +1144,9 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                 dc.epoch = epoch;
                 dc.mD = mD;
                 while (true) {
+#ifndef DBC_NO_BUSY_SITES
                     busy_help();
+#endif
                     const int hopen_pf = sample_open();
                     trace(1, L, le - lb);
                     dc.L = L;
@@ -1108,7 +1157,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                     gd.dcnt = a.help.gapp + wk;
                     gd.lowflag = a.help.low + wk;
                     int nrows = 0, nent = 0;  // the level's long rows (queued in Bq) and their entries
-                    if (a.help.word && items >= a.hd_min) {
+                    if (a.help.word && items >= a.hd_min && worth((items + kDownBlock - 1) / kDownBlock)) {
                         // a wide level: published, idle workers take blocks of items; their
                         // long rows are queued in this worker's Bq for the entry-balanced pass
                         const int nblk = (items + kDownBlock - 1) / kDownBlock;
@@ -1149,13 +1198,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                             __syncthreads();
                             if (b < 0) break;
                             ++own_blk;
-                            dc_small(gd, b * kDownBlock, min(items, (b + 1) * kDownBlock),
-                                     [&](int i, int len) {
-                                         Bq[atomicAdd(gb, 1)] = i;
-                                         atomicAdd(gb + 1, len);
-                                     },
-                                     st_bytes, sc_down);
-                            __syncthreads();
+                            down_block(gd, b * kDownBlock, min(items, (b + 1) * kDownBlock), Bq, gb);
                             if (tid == 0) {
                                 __threadfence();
                                 atomicAdd(a.help.done + wk, 1);
@@ -1187,7 +1230,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                     }
                     nrows = s_nbig;
                     nent = s_nent;
-                    if (a.help.word && nent >= a.dl_min) {
+                    if (a.help.word && nent >= a.dl_min && worth(nent / kDlEntries)) {
                         // long rows with many entries (hub neighbourhoods): entry-balanced
                         // blocks, owner and helpers; per-row results completed by the owner
                         int32_t *Boff = Ub;  // free during the down phase
@@ -1271,10 +1314,10 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                 // D levels: level L0 + j occupies Dv[Doff[j] .. Doff[j+1]), j < nlev
                 const int LmaxD = L0 + nlev - 1;
                 const int dtotal = le;
-                st_lvd += nlev;
+                if (tid == 0) s_st[5] += nlev;
                 if (tid == 0) {
-                    st_down += dtotal;
-                    st_touched += dtotal;
+                    s_st[1] += dtotal;
+                    s_st[0] += dtotal;
                 }
 
                 // the root gained a neighbour (Case 3 with u_high = root): rebuild its masks
@@ -1336,7 +1379,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                     rc.mD = mD;
                     rc.mU = mU;
                     const int kRemBlock = a.hd_block;
-                    if (a.help.word && dtotal >= a.hd_min) {
+                    if (a.help.word && dtotal >= a.hd_min && worth((dtotal + a.hd_block - 1) / a.hd_block)) {
                         // a wide pass: published, idle and busy workers take blocks of D
                         // (appends to R and the deepest target level go through global memory)
                         const int nblk = (dtotal + kRemBlock - 1) / kRemBlock;
@@ -1403,7 +1446,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                 // a deletion's removal targets can sit one level above the seeds (u_high)
                 const int Lstop = a.del ? min(L0, st.d[s_del[0]]) : L0;
                 const int Lmax = max(LmaxD, s_rmax);
-                if (tid == 0) st_touched += rcnt;
+                if (tid == 0) s_st[0] += rcnt;
 
                 tick(1);
                 // ================= up phase (K4 + Alg. 8) =================
@@ -1412,11 +1455,13 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                 int ucnt = 0;
                 for (int l = Lmax; l >= 1; --l) {
                     if (l < Lstop && ucnt == 0) break;  // nothing left above the insertion
+#ifndef DBC_NO_BUSY_SITES
                     busy_help();
+#endif
                     const int hopen_pf = sample_open();
                     trace(2, l, ucnt + rcnt + ((l >= L0 && l <= LmaxD) ? Doff[l - L0 + 1] - Doff[l - L0] : 0));
                     const bool push = l >= 2;          // level-1 vertices only feed the root
-                    ++st_lvu;
+                    if (tid == 0) ++s_st[6];
                     // queue p for level l-1 unless already queued: the prefetched mark
                     // filters the common case, the returning atomic elects one
                     // appender among concurrent pushers (no duplicates)
@@ -1658,10 +1703,12 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                             if (tid == 0) s_ucnt2[ucur_sel] = 0;
                         }
                         tick(6);
+                        trace(10, 0, min(s_nbigI, kChunk));  // chunk split done: long rows
                         const int nb = min(s_nbigI, kChunk);
                         if (nb > 0) {
                             chunk_scan(I.off, nb);  // off[0..nb], ends with a barrier
                             tick(7);
+                            trace(11, 0, I.off[nDb]);  // C1 entries
                             auto colf = [&](int t, int e) { return ldg_i(g.col + I.beg[t] + e - I.off[t]); };
                             // --- C1: delta pull of the long down rows (Eq. (2)) ---
                             const int E1 = I.off[nDb];
@@ -1674,7 +1721,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                              }, e0);
                             };
                             const int nblk1 = (E1 + a.he_entries - 1) / a.he_entries;
-                            if (E1 > 0 && a.help.word && nblk1 >= a.he_min) {
+                            if (E1 > 0 && a.help.word && nblk1 >= a.he_min && worth(nblk1)) {
                                 // publish the pull rows; helpers add per-row partial sums
                                 // into the mirror's acc (delta: rounding order is free)
                                 ChunkSmem *mir = a.help.mir + wk;
@@ -1740,6 +1787,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                 c1_pass(0, E1);
                             }
                             tick(8);
+                            trace(12, 0, I.off[nb]);  // C2 (before compaction)
                             // --- C2: pushes towards level l-1 (down rows only if they have a
                             // predecessor outside D: drop the others from the offsets) ---
                             if (push && s_noext) {
@@ -1761,7 +1809,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                             }
                             const int E2 = I.off[nb];
                             const int nblk = (E2 + a.he_entries - 1) / a.he_entries;
-                            if (push && E2 > 0 && a.help.word && nblk >= a.he_min) {
+                            if (push && E2 > 0 && a.help.word && nblk >= a.he_min && worth(nblk)) {
                                 // publish the chunk; idle workers help block by block
                                 ChunkSmem *mir = a.help.mir + wk;
                                 for (int t = tid; t < nb; t += kBlock) {
@@ -1857,6 +1905,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                         return 0.0;
                                     });
                             tick(9);
+                            trace(13, 0, s_nl1);
                             // --- C3: level-2 rows resolved against adj(root) ---
                             const int nl1 = s_nl1;
                             if (nl1 > 0) {
@@ -1894,6 +1943,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                 __syncthreads();
                             }
                             tick(4);
+                            trace(14, 0, nb);
                             // --- epilogue of the long rows (Alg. 8 fused) ---
                             for (int t = tid; t < nb; t += kBlock) {
                                 if (I.meta[t] & kMetaUp)
@@ -1914,7 +1964,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                     tick(3);
                     // the chunk loop ended with a barrier: every append of this level is in
                     ucnt = s_ucnt2[ucur_sel ^ 1];
-                    if (tid == 0) st_touched += ucnt;
+                    if (tid == 0) s_st[0] += ucnt;
                     int *t = Ucur;
                     Ucur = Unext;
                     Unext = t;
@@ -1924,7 +1974,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                 // any up vertices left at level 0 would be the root: never produced
                 if (a.scen && tid == 0)  // Fig. 2 / Fig. 4 record: case | touched << 2 | |D| << 33
                     a.scen[(size_t)ins * a.k_loc + slot] = (long long)(((unsigned long long)dtotal << 33) |
-                                                                       ((st_touched - touch0) << 2) |
+                                                                       ((s_st[0] - s_touch0) << 2) |
                                                                        (s_wcnt[1] ? 3u : 2u));
             }
             trace(4, 0, 0);
@@ -1936,17 +1986,18 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
             unsigned long long t1;
             asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t1));
             unsigned long long *rp4 = a.root_prof + 6 * (size_t)slot;
-            rp4[0] = prof_t0;
+            rp4[0] = s_prof[0];
             rp4[1] = t1;
-            rp4[2] = prof_jobs;
-            rp4[3] = st_touched - prof_touch0;
-            rp4[4] = sc_down + sc_rem + sc_dpull + sc_dpush + sc_up2 + sc_up3 - prof_sc0;
-            rp4[5] = st_lvd + st_lvu - prof_lv0;
+            rp4[2] = s_prof[1];
+            rp4[3] = s_st[0] - s_prof[2];
+            rp4[4] = (unsigned long long)sc_down + sc_rem + sc_dpull + sc_dpush + sc_up2 + sc_up3 - s_prof[3];
+            rp4[5] = s_st[5] + s_st[6] - s_prof[4];
         }
     }
     // ---- out of roots: help the passes of workers still running ----
     if (a.help.word) {
         int cur_owner = -1, cur_seq = -1;
+        if (tid == 0) atomicAdd(a.help.roots_left + 2, 1);  // one more idle worker
         for (;;) {
             const int r = help_step(true, cur_owner, cur_seq);
             if (r == -2) break;
@@ -1955,13 +2006,13 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
     }
     if (tid == 0) {
         a.ws.wepoch[wk] = epoch;
-        if (st_c1) atomicAdd(a.stats + kStCase1, st_c1);
-        if (st_c2) atomicAdd(a.stats + kStCase2, st_c2);
-        if (st_c3) atomicAdd(a.stats + kStCase3, st_c3);
-        if (st_touched) atomicAdd(a.stats + kStTouched, st_touched);
-        if (st_down) atomicAdd(a.stats + kStDown, st_down);
-        if (st_lvd) atomicAdd(a.stats + kStLevDown, st_lvd);
-        if (st_lvu) atomicAdd(a.stats + kStLevUp, st_lvu);
+        if (s_st[2]) atomicAdd(a.stats + kStCase1, s_st[2]);
+        if (s_st[3]) atomicAdd(a.stats + kStCase2, s_st[3]);
+        if (s_st[4]) atomicAdd(a.stats + kStCase3, s_st[4]);
+        if (s_st[0]) atomicAdd(a.stats + kStTouched, s_st[0]);
+        if (s_st[1]) atomicAdd(a.stats + kStDown, s_st[1]);
+        if (s_st[5]) atomicAdd(a.stats + kStLevDown, s_st[5]);
+        if (s_st[6]) atomicAdd(a.stats + kStLevUp, s_st[6]);
         for (int q = 0; q < 10; ++q)
             if (tm_ph[q]) atomicAdd(a.stats + kStTime0 + q, tm_ph[q]);
     }

@@ -45,5 +45,5 @@ if os.environ.get("DBC_TRACE_SLOT"):
         if t0 is None:
             t0 = t
         dt = (t - last) / 1e3 if last is not None else 0.0
-        print("trace +%8.1f us (at %8.1f) %s level %d items %d%s" % (dt, (t - t0) / 1e3, {1: "down", 2: "up", 3: "removal", 4: "job-end", 6: "owner-blocks(kind; own|total<<16)", 9: "long-rows(rows; entries)"}.get(kind, "?"), lev, items, (" own %d of %d" % (items & 0xFFFF, items >> 16)) if kind == 6 else ""))
+        print("trace +%8.1f us (at %8.1f) %s level %d items %d%s" % (dt, (t - t0) / 1e3, {1: "down", 2: "up", 3: "removal", 4: "job-end", 6: "owner-blocks(kind; own|total<<16)", 9: "long-rows(rows; entries)", 10: " chunk-split(long rows)", 11: " C1(entries)", 12: " C2(entries)", 13: " C3(l1 rows)", 14: " epilogue(rows)"}.get(kind, "?"), lev, items, (" own %d of %d" % (items & 0xFFFF, items >> 16)) if kind == 6 else ""))
         last = t
