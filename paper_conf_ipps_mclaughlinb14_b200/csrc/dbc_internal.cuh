@@ -186,7 +186,12 @@ __device__ __forceinline__ bool new_edge(const GView &g, int x, int p, int g0, i
 // neighbours' distances, then -- only for entries passing want(d) -- their
 // (sigma, delta) pair and mk[y] (if mk), kRowUnroll entries in flight; then
 // f(y, d, sd, mark) runs in order.
-constexpr int kRowUnroll = 8;
+#ifndef DBC_ROW_UNROLL
+// 64-register builds (>= 1024 resident threads per CTA launch bound) keep 4
+// entries in flight per lane: 8 would spill the gathered arrays
+#define DBC_ROW_UNROLL ((DBC_BLOCK * DBC_MINB >= 1024) ? 4 : 8)
+#endif
+constexpr int kRowUnroll = DBC_ROW_UNROLL;
 template <class Want, class F>
 __device__ __forceinline__ void row_walk(const GView &g, const Root &st, const uint32_t *mk,
                                          int2 r, Want want, F f) {
