@@ -420,12 +420,16 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     if (const char *e = getenv("DBC_BUSY_HELP")) c->busy_help = std::max(0, atoi(e));
     if (const char *e = getenv("DBC_BUSY_MIN")) c->busy_min = std::max(1, atoi(e));
     if (const char *e = getenv("DBC_DLMIN")) c->dl_min = std::max(1, atoi(e));
-    c->block = 512;
+    // Update CTAs (measured on B200): one 1024-thread CTA per
+    // SM (64 registers) by default -- a window-merged job has wide levels and
+    // hub rows (R-MAT 16 +7.5%, Kronecker 20 +6%, small world +6% over one
+    // 512-thread CTA); low-degree graphs with many roots per SM (>= 3 x #SMs,
+    // long chains of narrow levels: Delaunay 2^18) run two register-capped
+    // 512-thread CTAs per SM instead (+40% over 1024).
+    const bool many_narrow = c->lowdeg && c->k_loc >= 3 * c->nsm;
+    c->block = many_narrow ? 512 : 1024;
     if (const char *eb = getenv("DBC_BLOCK"))
         c->block = atoi(eb) == 128 ? 128 : (atoi(eb) == 256 ? 256 : (atoi(eb) == 1024 ? 1024 : 512));
-    // Many roots per SM (>= 3 x #SMs): two register-capped 512-thread CTAs per
-    // SM keep more root chains in flight (Delaunay 2^18 / 512 roots: +29%,
-    // Kronecker 20 / 1024 roots: +3%); fewer roots: one 128-register CTA.
     c->ub2 = c->block == 512 && c->k_loc >= 3 * c->nsm;
     if (const char *e = getenv("DBC_UB2")) c->ub2 = c->block == 512 && atoi(e) != 0;
     int upb = c->block == 128 ? 4 : (c->block >= 512 ? (c->ub2 ? 2 : 1) : 2);  // update CTAs per SM

@@ -704,8 +704,9 @@ def test_heavy_lane_with_help_completes_rmat16(rep):
             assert np.array_equal(d, dyn[i][0]) and np.array_equal(sg, dyn[i][1])
 
 
+@pytest.mark.parametrize("block", [None, "512"])
 @pytest.mark.parametrize("name", ["rmat10", "delaunay12u", "smallworld"])
-def test_forced_help_paths_match_oracle(name, monkeypatch):
+def test_forced_help_paths_match_oracle(name, block, monkeypatch):
     """Every cooperative path forced on at small sizes: helped down levels
     (kind 1, 32-item blocks), entry-balanced long rows of every down level
     (kind 4), the Case-3 removal pass as help blocks (kind 3), helped delta-pull
@@ -716,6 +717,8 @@ def test_forced_help_paths_match_oracle(name, monkeypatch):
                  "DBC_HEENT": "256", "DBC_BUSY_MIN": "1", "DBC_BUSY_HELP": "4",
                  "DBC_HEAVY_FACTOR": "1.0"}.items():
         monkeypatch.setenv(k, v)
+    if block:  # 512-thread CTAs (128 registers) beside the default width
+        monkeypatch.setenv("DBC_BLOCK", block)
     wl = W.make_workload(name)
     ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
     with _dbc(wl.graph, wl.roots) as dbc:
