@@ -40,6 +40,7 @@ struct dbc_ctx {
     int busy_help = 1;                   // blocks a busy worker takes at a level boundary
     int busy_min = 32;                   // ... of passes of at least this many blocks
     int dl_min = 16 * 4096;              // entry-balanced long rows of a down level from this many entries
+    int wide_inlane = -1;                // up levels of <= this many items per thread: short rows in-lane
     int sblock = 256, sworkers = 0;  // static kernel: its own CTA width and grid
     size_t nscratch = 0;             // worker scratch sets allocated
     // heavy lanes: the slowest root chains of the previous batch run on
@@ -420,6 +421,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     if (const char *e = getenv("DBC_BUSY_HELP")) c->busy_help = std::max(0, atoi(e));
     if (const char *e = getenv("DBC_BUSY_MIN")) c->busy_min = std::max(1, atoi(e));
     if (const char *e = getenv("DBC_DLMIN")) c->dl_min = std::max(1, atoi(e));
+    if (const char *e = getenv("DBC_WIDE_INLANE")) c->wide_inlane = std::max(0, atoi(e));
     // Update CTAs (measured on B200): one 1024-thread CTA per
     // SM (64 registers) by default -- a window-merged job has wide levels and
     // hub rows (R-MAT 16 +7.5%, Kronecker 20 +6%, small world +6% over one
@@ -437,6 +439,10 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     want = std::min(want, c->k_loc);
     int fit = (int)std::min<size_t>(budget / per_worker, 1 << 20);
     c->workers = std::max(0, std::min(want, fit));
+    // in-lane short rows on wide up levels: lower latency, less even work --
+    // worth it while the batch time is the slowest root chain (few roots per
+    // worker: R-MAT 16 +8%), not when every worker has many roots (Kronecker 20)
+    if (c->wide_inlane < 0) c->wide_inlane = c->k_loc <= 2 * std::max(c->workers, 1) ? 64 : 16;
     c->sworkers = std::max(0, std::min({opt.workers ? opt.workers : (c->sblock == 128 ? 4 : 2) * c->nsm,
                                         c->k_loc, fit}));
     c->hblock = c->block == 128 ? 256 : (c->block == 256 ? 512 : 1024);
@@ -499,6 +505,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->ws.Rv, wn);
     AL(c->ws.Rl, wn);
     AL(c->ws.Bq, wn);
+    AL(c->ws.X, nwk * (size_t)kXcap);
     AL(c->ws.wepoch, nwk);
     c->ws.wcap = kWindow;
     if (const char *e = getenv("DBC_WINDOW")) c->ws.wcap = std::max(1, atoi(e));
@@ -734,6 +741,7 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     a.busy_help = c->busy_help;
     a.busy_min = c->busy_min;
     a.dl_min = c->dl_min;
+    a.wide_inlane = c->wide_inlane;
     a.trace_slot = getenv("DBC_TRACE_SLOT") ? atoi(getenv("DBC_TRACE_SLOT")) : -1;
     a.lowdeg = c->lowdeg && !getenv("DBC_NO_LOWDEG");
     if (c->scen_cap > 0) {  // Fig. 2 / Fig. 4 log: one job per (root, insertion)
@@ -1013,6 +1021,7 @@ static dbc_status delete_host_ids(dbc_ctx *c, const int32_t *u, const int32_t *v
     a.busy_help = c->busy_help;
     a.busy_min = c->busy_min;
     a.dl_min = c->dl_min;
+    a.wide_inlane = c->wide_inlane;
     a.trace_slot = getenv("DBC_TRACE_SLOT") ? atoi(getenv("DBC_TRACE_SLOT")) : -1;
     a.lowdeg = c->lowdeg && !getenv("DBC_NO_LOWDEG");
     a.scen = nullptr;

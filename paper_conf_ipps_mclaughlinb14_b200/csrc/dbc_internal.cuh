@@ -66,6 +66,7 @@ enum StatIdx : int {
     kStGroups,                   // Case-2 group jobs (>= 2 insertions repaired together)
     kStGroupIns,                 // insertions in those group jobs
     kStBusyBlk,                  // help blocks run by busy workers (at their level boundaries)
+    kStDeferred,                 // long rows of wide up levels processed in deferred chunks
     kStTraceN,                   // -DDBC_PHASE_TIMERS: events of the traced slot (DBC_TRACE_SLOT)
     kStTrace0,                   // kTraceCap (code, %globaltimer) pairs
     kStCount = kStTrace0 + 2 * 1024
@@ -90,6 +91,16 @@ struct GView {
 
 // Scratch of the persistent workers (one CTA = one worker), each array
 // worker-major with stride n.
+// A resolved long row of a wide up level waiting for a later chunk (down rows
+// from the front of the per-worker array, up rows from the back).
+struct XRow {
+    int x, meta, beg, len;
+    double c0, c1, c2;
+    uint32_t mk;
+    int pad;
+};
+constexpr int kXcap = 16384;  // deferred long rows per worker (beyond: walked in-lane)
+
 struct Scratch {
     uint32_t *mark;            // epoch<<2 | state
     unsigned long long *lowrec;  // (epoch << 32) | old d, written by the lowering thread
@@ -101,6 +112,7 @@ struct Scratch {
     int32_t *U0, *U1;          // up frontier overflow ping-pong
     int32_t *Rv, *Rl;          // removal-push targets and their levels (Case 3)
     int32_t *Bq;               // long-row queue of the current level, n per worker
+    struct XRow *X;            // wide up levels: long rows beyond one chunk, kXcap per worker
     int32_t *Wul, *Wlev;       // window of insertions: u_low and seed level, wcap per worker
     int32_t wcap;              // window capacity (insertions per job)
     uint32_t *wepoch;          // per-worker epoch counter
@@ -567,6 +579,7 @@ struct UpdateArgs {
     int32_t busy_help;             // blocks a busy worker takes per poll of the board (0: only idle workers help)
     int32_t busy_min;              // busy workers take blocks of passes of at least this many blocks
     int32_t dl_min;                // down levels whose long rows hold >= dl_min entries: entry-balanced pass
+    int32_t wide_inlane;           // up levels of <= wide_inlane items per thread: short rows in-lane, long rows chunked
     int32_t trace_slot;            // -DDBC_PHASE_TIMERS builds: time this slot only (-1: all)
 };
 

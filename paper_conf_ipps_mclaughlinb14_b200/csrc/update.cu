@@ -524,6 +524,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
     __shared__ int s_hopen;                   // open requests seen at the last level boundary
     __shared__ int s_nent, s_tot, s_t0;        // long rows of a down level: entries, offsets total, first row
     __shared__ int s_stg[3];                  // helped down block: staged long rows, their entries, base
+    __shared__ int s_nx[2];                   // wide up level: deferred long down / up rows
     __shared__ int s_del[6];     // deletion job: [0] u_high, [1] u_low, [2] |A|, [3] seeds, [4] candidates, [5] u_low keeps a predecessor
     __shared__ double s_delsd[2];  // deletion job: old sigma / delta of u_low
 
@@ -813,6 +814,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
         s_nl1 = 0;
         s_noext = 0;
         s_hopen = 0;
+        s_nx[0] = 0;
+        s_nx[1] = 0;
     }
 
     for (;;) {
@@ -1643,7 +1646,32 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                             d_finish(x, dn, c1);
                         }
                     };
-                    auto split_range = [&](int q0, int q1, bool small_inlane) {
+                    // long row t of the chunk in I (level-2 rows resolved against adj(root)
+                    // carry no entries of their own)
+                    auto put_row = [&](int t, int x, int meta, double c0, double c1, double c2, int beg, int len,
+                                       uint32_t mk) {
+                        int elen = len;
+                        if (meta & kMetaMask) {  // level 2 via the mask
+                            if (mk) s_l1[atomicAdd(&s_nl1, 1)] = t;
+                            elen = 0;
+                        } else if ((meta & kMetaUp) && l == 2 && s_ds >= 0 && s_ds * (33 - __clz(len)) < len) {
+                            // level 2 without masks: resolve against adj(root) by search
+                            s_l1[atomicAdd(&s_nl1, 1)] = t;
+                            elen = 0;
+                        }
+                        if (!(meta & (kMetaUp | kMetaExt))) s_noext = 1;  // a down row without pushes
+                        I.mk[t] = mk;
+                        I.v[t] = x;
+                        I.meta[t] = meta;
+                        I.beg[t] = beg;
+                        I.off[t + 1] = elen;
+                        I.acc[t] = 0.0;
+                        I.c0[t] = c0;
+                        I.c1[t] = c1;
+                        I.c2[t] = c2;
+                    };
+                    XRow *Xw = a.ws.X + (size_t)wk * kXcap;
+                    auto split_range = [&](int q0, int q1, bool small_inlane, bool defer) {
                         for (int q = q0 + tid; q < q1; q += kBlock) {
                             int x, meta = 0;
                             double c0 = 0.0, c1 = 0.0, c2 = 0.0;
@@ -1656,47 +1684,46 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                 continue;
                             }
                             const int t = atomicAdd(&s_nbigI, 1);
-                            if (t >= kChunk) {  // shared list full: stay in-lane
-                                inlane(x, meta, c0, c1, c2, r, mk);
+                            if (t >= kChunk) {  // shared list full: a later chunk, or in-lane
+                                const bool up = (meta & kMetaUp) != 0;
+                                const int xi = defer ? atomicAdd(&s_nx[up ? 1 : 0], 1) : kXcap;
+                                if (xi < kXcap / 2) {  // down rows from the front, up rows from the back
+                                    XRow &w = Xw[up ? kXcap - 1 - xi : xi];
+                                    w.x = x;
+                                    w.meta = meta;
+                                    w.beg = r.x;
+                                    w.len = len;
+                                    w.c0 = c0;
+                                    w.c1 = c1;
+                                    w.c2 = c2;
+                                    w.mk = mk;
+                                } else {
+                                    inlane(x, meta, c0, c1, c2, r, mk);
+                                }
                                 continue;
                             }
-                            int elen = len;
-                            if (meta & kMetaMask) {  // level 2 via the mask
-                                if (mk) s_l1[atomicAdd(&s_nl1, 1)] = t;
-                                elen = 0;
-                            } else if ((meta & kMetaUp) && l == 2 && s_ds >= 0 &&
-                                       s_ds * (33 - __clz(len)) < len) {
-                                // level 2 without masks: resolve against adj(root) by search
-                                s_l1[atomicAdd(&s_nl1, 1)] = t;
-                                elen = 0;
-                            }
-                            if (!(meta & (kMetaUp | kMetaExt))) s_noext = 1;  // a down row without pushes
-                            I.mk[t] = mk;
-                            I.v[t] = x;
-                            I.meta[t] = meta;
-                            I.beg[t] = r.x;
-                            I.off[t + 1] = elen;
-                            I.acc[t] = 0.0;
-                            I.c0[t] = c0;
-                            I.c1[t] = c1;
-                            I.c2[t] = c2;
+                            put_row(t, x, meta, c0, c1, c2, r.x, len, mk);
                         }
                     };
                     // small levels (<= one item per thread): short rows in-lane;
                     // large levels: every row through the flattened pass, in chunks
                     const int total = nDl + ucnt + rcnt;
                     const bool small_level = total <= kBlock || a.lowdeg;
-                    const int step = small_level ? total : kChunk;
+                    // wide levels of up to wide_inlane items per thread: short rows in-lane
+                    // in one pass, long rows through chunks of kChunk (the first in I, the
+                    // rest deferred in Xw); wider levels: every row chunked
+                    const bool wide = !small_level && total <= a.wide_inlane * kBlock;
+                    const int step = (small_level || wide) ? total : kChunk;
                     bool first_barrier = true;
                     for (int cb = 0; cb < total; cb += step) {
                         const int ce = min(total, cb + step);
                         int nDb = 0;
                         if (cb < nDl) {  // down rows first: their pull precedes their push
-                            split_range(cb, min(ce, nDl), small_level);
+                            split_range(cb, min(ce, nDl), small_level || wide, wide);
                             __syncthreads();
                             nDb = min(s_nbigI, kChunk);
                         }
-                        split_range(max(cb, nDl), ce, small_level);
+                        split_range(max(cb, nDl), ce, small_level || wide, wide);
                         __syncthreads();
                         if (first_barrier) {  // the current list's count was read last level
                             first_barrier = false;
@@ -1704,7 +1731,9 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                         }
                         tick(6);
                         trace(10, 0, min(s_nbigI, kChunk));  // chunk split done: long rows
-                        const int nb = min(s_nbigI, kChunk);
+                        int nb = min(s_nbigI, kChunk);
+                        int xdn = 0, xun = 0;  // deferred down / up rows already loaded
+                        for (;;) {  // the chunk in I, then (wide levels) the deferred rows
                         if (nb > 0) {
                             chunk_scan(I.off, nb);  // off[0..nb], ends with a barrier
                             tick(7);
@@ -1958,6 +1987,26 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                             s_nl1 = 0;
                             s_noext = 0;
                             s_hopen = hopen_pf;
+                        }
+                        __syncthreads();
+                        if (!wide) break;
+                        const int nxd = min(s_nx[0], kXcap / 2), nxu = min(s_nx[1], kXcap / 2);
+                        const bool dn = xdn < nxd;  // deferred down rows first (own chunks: C1 then C2)
+                        if (!dn && xun >= nxu) break;
+                        const int m = dn ? min(kChunk, nxd - xdn) : min(kChunk, nxu - xun);
+                        for (int t = tid; t < m; t += kBlock) {
+                            const XRow &w = Xw[dn ? xdn + t : kXcap - 1 - (xun + t)];
+                            put_row(t, w.x, w.meta, w.c0, w.c1, w.c2, w.beg, w.len, w.mk);
+                        }
+                        if (dn) xdn += m; else xun += m;
+                        if (tid == 0) atomicAdd(a.stats + kStDeferred, (unsigned long long)m);
+                        nb = m;
+                        nDb = dn ? m : 0;
+                        __syncthreads();
+                        }  // deferred chunks
+                        if (wide && tid == 0) {
+                            s_nx[0] = 0;
+                            s_nx[1] = 0;
                         }
                         __syncthreads();
                     }  // chunks

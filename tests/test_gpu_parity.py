@@ -734,3 +734,26 @@ def test_forced_help_paths_match_oracle(name, block, monkeypatch):
         c1 = dbc.debug_counters()
         check_all(dbc, ref.compute(), wl.roots.size)
         assert c1["help_requests"] > c0["help_requests"]
+
+
+@pytest.mark.parametrize("block", [None, "512"])
+def test_wide_up_levels_deferred_chunks_match_oracle(block, monkeypatch):
+    """Wide up levels walked with short rows in-lane and long rows in chunks,
+    more than one chunk of them deferred (DBC_WIDE_INLANE forces the mode on
+    every level wider than a CTA): R-MAT 2^14 / edgefactor 16, 64 roots, 400
+    insertions in two batches; d/sigma bit-exact vs the oracle, BC in tolerance."""
+    monkeypatch.setenv("DBC_WIDE_INLANE", "100000")
+    if block:
+        monkeypatch.setenv("DBC_BLOCK", block)
+    wl = W.make_workload("rmat14")
+    ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
+    with _dbc(wl.graph, wl.roots) as dbc:
+        dbc.static_compute()
+        c0 = dbc.debug_counters()
+        for sl in (slice(0, 200), slice(200, 400)):
+            dbc.insert_edges(wl.ins_u[sl], wl.ins_v[sl])
+            for u, v in zip(wl.ins_u[sl], wl.ins_v[sl]):
+                ref.insert(u, v)
+        c1 = dbc.debug_counters()
+        check_all(dbc, ref.compute(), wl.roots.size)
+        assert c1["deferred_rows"] > c0["deferred_rows"]  # more than one chunk of long rows

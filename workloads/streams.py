@@ -105,6 +105,7 @@ CONFIGS = {
     "smallworld": dict(graph="ws", n=100_000, kk=10, p=0.1, k=256, insertions=100, mode="reinsert"),
     # small shapes of the same families for oracle-speed parity tests
     "rmat10": dict(graph="rmat", scale=10, ef=8, k=64, insertions=40, mode="reinsert"),
+    "rmat14": dict(graph="rmat", scale=14, ef=16, k=64, insertions=400, mode="reinsert"),
     "delaunay12": dict(graph="delaunay", npts=1 << 12, k=48, insertions=40, mode="reinsert"),
     "delaunay12u": dict(graph="delaunay", npts=1 << 12, k=48, insertions=40, mode="non_edges"),
 }
