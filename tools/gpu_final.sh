@@ -1,6 +1,6 @@
 #!/bin/bash
 # Round evidence: default bench line, launch list, ncu captures, per-config lines, paper figures.
-O=gpurun_out/final; mkdir -p $O
+O=gpurun_out/${FINAL_DIR:-final}; mkdir -p $O
 timeout 1500 python -m pytest tests -m gpu -q > $O/gpu_tests.log 2>&1; echo "rc=$?" >> $O/gpu_tests.log
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; echo "rc=$?" >> $O/smoke.log
 timeout 600 python bench.py > $O/bench_rmat16.json 2> $O/bench_rmat16.err
