@@ -406,13 +406,16 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     cudaMemGetInfo(&free_b, &total_b);
     const size_t state_b = (size_t)c->k_loc * n * 24 + (size_t)c->col_cap * 8 + (size_t)n * 40;
     size_t budget = free_b > state_b ? (free_b - state_b) / 2 : 0;
-    // Update: a job is a window of up to 4096 insertions whose levels are wide,
-    // so one 512-thread CTA per SM beats more, narrower CTAs.
-    // Static: more roots than two 256-thread CTAs per SM can hold and no hub
-    // rows -> 128-thread CTAs, four per SM, every root resident at once.
     int64_t maxdeg = 0;
     for (int32_t v = 0; v < n; ++v) maxdeg = std::max<int64_t>(maxdeg, row_ptr[v + 1] - row_ptr[v]);
-    c->sblock = (c->k_loc > 2 * c->nsm && maxdeg <= 256) ? 128 : 256;  // hubs need the wide CTA
+    // static kernel: one 1024-thread CTA per SM (64 registers) -- measured on
+    // B200 against 256 (2/SM), 512 and 128 (4/SM): R-MAT 16 5.8 vs 9.6 ms,
+    // Delaunay 2^18 22.3 vs 29.4 ms, Kronecker 20 0.85 vs 1.56 s
+    c->sblock = 1024;
+    if (const char *e = getenv("DBC_SBLOCK")) {
+        const int b = atoi(e);
+        c->sblock = (b == 128 || b == 512 || b == 1024) ? b : 256;
+    }
     c->lowdeg = maxdeg <= 32;  // every row walked by one lane: no chunked up levels
     if (const char *e = getenv("DBC_HDMIN")) c->hd_min = std::max(1, atoi(e));
     if (const char *e = getenv("DBC_HDBLK")) c->hd_block = std::max(32, atoi(e));
@@ -443,7 +446,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     // worth it while the batch time is the slowest root chain (few roots per
     // worker: R-MAT 16 +8%), not when every worker has many roots (Kronecker 20)
     if (c->wide_inlane < 0) c->wide_inlane = c->k_loc <= 2 * std::max(c->workers, 1) ? 64 : 16;
-    c->sworkers = std::max(0, std::min({opt.workers ? opt.workers : (c->sblock == 128 ? 4 : 2) * c->nsm,
+    c->sworkers = std::max(0, std::min({opt.workers ? opt.workers : (c->sblock == 128 ? 4 : (c->sblock >= 512 ? 1 : 2)) * c->nsm,
                                         c->k_loc, fit}));
     c->hblock = c->block == 128 ? 256 : (c->block == 256 ? 512 : 1024);
     // only hub-heavy graphs (256-thread build) have step-bound slow roots
@@ -633,6 +636,10 @@ extern "C" dbc_status dbc_static_compute(dbc_ctx *c) {
         a.err = c->err;
         if (c->sblock == 128)
             launch_static_128(a, c->sworkers, c->stream);
+        else if (c->sblock == 512)
+            launch_static_512(a, c->sworkers, c->stream);
+        else if (c->sblock == 1024)
+            launch_static_1024(a, c->sworkers, c->stream);
         else
             launch_static_256(a, c->sworkers, c->stream);
         CK(cudaGetLastError());

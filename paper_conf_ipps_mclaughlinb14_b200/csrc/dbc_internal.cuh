@@ -628,5 +628,7 @@ void launch_update_128(const UpdateArgs &a, int workers, cudaStream_t s);
 void launch_update_512(const UpdateArgs &a, int workers, cudaStream_t s);
 void launch_static_256(const StaticArgs &a, int workers, cudaStream_t s);
 void launch_static_128(const StaticArgs &a, int workers, cudaStream_t s);
+void launch_static_512(const StaticArgs &a, int workers, cudaStream_t s);   // 64 regs, 2 CTAs/SM
+void launch_static_1024(const StaticArgs &a, int workers, cudaStream_t s);  // 64 regs, 1 CTA/SM
 
 }  // namespace dbc

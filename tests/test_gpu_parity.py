@@ -71,6 +71,19 @@ def test_static_matches_oracle(name):
         check_all(dbc, ref, roots.size)
 
 
+@pytest.mark.parametrize("sblock", ["128", "256", "512"])
+@pytest.mark.parametrize("name", ["grid_big_sigma", "disconnected", "rmat10", "delaunay12", "hub"])
+def test_static_other_widths_match_oracle(name, sblock, monkeypatch):
+    """The static kernel at the non-default CTA widths (DBC_SBLOCK; default 1024)."""
+    monkeypatch.setenv("DBC_SBLOCK", sblock)
+    g, roots = STATIC_CASES[name]()
+    roots = np.asarray(roots, np.int32)
+    ref = oracle.brandes_csr(g, roots)
+    with _dbc(g, roots) as dbc:
+        dbc.static_compute()
+        check_all(dbc, ref, roots.size)
+
+
 def test_static_no_edges_and_zero_roots():
     g = W.csr_from_edges(5, [], [])
     with _dbc(g, np.array([0, 3], np.int32)) as dbc:
