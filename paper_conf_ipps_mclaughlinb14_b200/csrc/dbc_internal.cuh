@@ -67,6 +67,7 @@ enum StatIdx : int {
     kStGroupIns,                 // insertions in those group jobs
     kStBusyBlk,                  // help blocks run by busy workers (at their level boundaries)
     kStDeferred,                 // long rows of wide up levels processed in deferred chunks
+    kStUpPass,                   // in-lane passes of wide up levels published as help blocks (kind 5)
     kStTraceN,                   // -DDBC_PHASE_TIMERS: events of the traced slot (DBC_TRACE_SLOT)
     kStTrace0,                   // kTraceCap (code, %globaltimer) pairs
     kStCount = kStTrace0 + 2 * 1024
@@ -517,9 +518,11 @@ struct HelpCtx {
     uint32_t E;  // epoch << 2 of the job
     int kind;    // 0: C2 push pass of a published chunk; 1: a down-phase level;
                  // 2: C1 delta-pull pass of a chunk; 3: the Case-3 removal pass over D;
-                 // 4: the long rows of a down level, entry-balanced (E2 entries, cnt rows)
-    int lb;      // kind 1: the level's first position in D
+                 // 4: the long rows of a down level, entry-balanced (E2 entries, cnt rows);
+                 // 5: the in-lane item pass of a wide up level (cnt items, E2 = |down segment|)
+    int lb;      // kind 1: the level's first position in D; kind 5: b0
     int mvalid;  // kind 1: level-2 masks are maintained
+    int aux;     // kind 5: |up frontier| | (its overflow list is U1) << 30
 };
 struct HelpBoard {
     unsigned long long *word;  // [workers]

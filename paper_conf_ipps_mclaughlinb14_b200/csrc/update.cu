@@ -498,6 +498,172 @@ __device__ __forceinline__ void dl_finish(const DownCtx &c, const int32_t *Bq, i
     __syncthreads();
 }
 
+// ---------------------------------------------------------------------------
+// The in-lane item pass of a wide up level as help blocks (kind 5): items
+// [q0, q1) of level l -- the down segment Dv[b0, b0 + nDl), then the up
+// frontier (Ul / Uo), then removal targets of level l -- resolved and, for
+// short rows, processed in-lane exactly as the owner's inlane() does (delta
+// pull of down rows, Ddelta pushes to level l - 1, Alg. 8 epilogue); long rows
+// are deferred to the owner's X list (its chunks run after the pass).  Claimed
+// predecessors are appended to gU.  Owner and helpers run the same code.
+struct UpCtx {
+    GView g;
+    Root st;
+    uint32_t *mark;
+    double *dacc, *bc;
+    const uint32_t *mask;
+    const int32_t *Dv, *Dold, *Rv, *Rl, *Ul, *Uo;
+    const double *Dsig;
+    const int *adjs;  // the root's row (level-2 mask bits)
+    int32_t *gU;
+    int *gapp, *xcnt;
+    XRow *X;
+    int l, b0, nDl, ucnt, g0, lim, mok;
+    uint32_t E, mU, mD;
+};
+
+__device__ __forceinline__ void up_claim(const UpCtx &c, int y, uint32_t my) {
+    if (my >= c.E) return;
+    if (atomicMax(c.mark + y, c.mU) >= c.E) return;
+    c.gU[atomicAdd(c.gapp, 1)] = y;
+}
+
+__device__ __forceinline__ void up_block(const UpCtx &c, int q0, int q1, uint32_t &bytes, uint32_t &scanned) {
+    const int l = c.l;
+    const bool push = l >= 2;
+    for (int q = q0 + (int)threadIdx.x; q < q1; q += kBlock) {
+        // ---- resolve (as the owner's resolve())
+        int x, meta;
+        double c0, c1, c2;
+        int2 r;
+        uint32_t mk = 0u;
+        if (q < c.nDl) {
+            const int idx = c.b0 + q;
+            x = c.Dv[idx];
+            const double2 s2 = c.st.sd[x];
+            c0 = s2.x;
+            c1 = s2.y;
+            c2 = c.Dsig[idx];
+            const int od = c.Dold[idx];
+            meta = (((od & kOldMask) == l) ? kMetaNotPulled : 0) | ((od < 0) ? kMetaExt : 0) |
+                   ((ldg_i(c.g.rp + x) < 0) ? kMetaNew : 0);
+            r = row_of(c.g, x, c.lim);
+            bytes += 8 + 16 + 8 + 4;
+        } else {
+            const int qi = q - c.nDl;
+            x = -1;
+            if (qi < c.ucnt)
+                x = (qi < kUcap) ? c.Ul[qi] : c.Uo[qi - kUcap];
+            else if (c.Rl[qi - c.ucnt] == l)
+                x = c.Rv[qi - c.ucnt];
+            if (x < 0) continue;
+            const uint32_t prev = atomicMax(c.mark + x, c.E | kUpDone);
+            const double gxs = __ldcg(c.dacc + x);
+            const double2 s2 = c.st.sd[x];
+            const double sx = s2.x, odl = s2.y;
+            const double gx = __dmul_rn(sx, gxs);
+            const bool usemask = l == 2 && c.mok;
+            const int2 rr = (push && !usemask) ? row_of(c.g, x, c.lim) : make_int2(0, 0);
+            mk = usemask ? c.mask[x] : 0u;
+            if (prev != c.mU) continue;  // a duplicate: the first claimant processes
+            meta = kMetaUp | (usemask ? kMetaMask : 0);
+            c0 = sx;
+            c1 = gx;
+            c2 = odl;
+            bytes += 24 + (usemask ? 4 : 0);
+            r = (push && gx != 0.0) ? rr : make_int2(0, 0);
+            if (gx == 0.0) mk = 0u;
+        }
+        const int len = r.y - r.x;
+        if (len > kSmallDeg) {  // long row: a deferred chunk of the owner
+            const bool up = (meta & kMetaUp) != 0;
+            const int xi = atomicAdd(c.xcnt + (up ? 1 : 0), 1);
+            if (xi < kXcap / 2) {
+                XRow &w = c.X[up ? kXcap - 1 - xi : xi];
+                w.x = x;
+                w.meta = meta;
+                w.beg = r.x;
+                w.len = len;
+                w.c0 = c0;
+                w.c1 = c1;
+                w.c2 = c2;
+                w.mk = mk;
+                continue;
+            }
+            // list full: walk it here
+        }
+        // ---- in-lane (as the owner's inlane())
+        const bool wantpush = push && r.y > r.x;
+        if (meta & kMetaMask) {  // level 2: predecessors = set bits (root's row order)
+            for (uint32_t b = mk; b; b &= b - 1) {
+                const int pp = c.adjs[__ffs(b) - 1];
+                atomicAdd(c.dacc + pp, __ddiv_rn(c1, c0));
+                bytes += 24;
+                up_claim(c, pp, c.mark[pp]);
+            }
+        } else if (meta & kMetaUp) {
+            if (wantpush) {
+                const double wx = __ddiv_rn(c1, c0);  // Ddelta[x] / sigma[x]
+                for (int j = r.x; j < r.y; j += kRowUnroll) {
+                    int y[kRowUnroll], dy[kRowUnroll];
+                    uint32_t mp[kRowUnroll];
+#pragma unroll
+                    for (int u = 0; u < kRowUnroll; ++u) y[u] = (j + u < r.y) ? ldg_i(c.g.col + j + u) : -1;
+#pragma unroll
+                    for (int u = 0; u < kRowUnroll; ++u) dy[u] = (y[u] >= 0) ? c.st.d[y[u]] : kInf;
+#pragma unroll
+                    for (int u = 0; u < kRowUnroll; ++u) mp[u] = (y[u] >= 0 && dy[u] == l - 1) ? c.mark[y[u]] : 0xffffffffu;
+#pragma unroll
+                    for (int u = 0; u < kRowUnroll; ++u)
+                        if (y[u] >= 0 && dy[u] == l - 1) {
+                            atomicAdd(c.dacc + y[u], wx);
+                            bytes += 24;
+                            up_claim(c, y[u], mp[u]);
+                        }
+                }
+                scanned += r.y - r.x;
+                bytes += 8 + 8u * (r.y - r.x);
+            }
+        } else {
+            double dn = 0.0;
+            row_walk(c.g, c.st, nullptr, r, [&](int dy) { return dy == l + 1; },
+                     [&](int, int dy, double2 qq, uint32_t) {
+                         if (dy == l + 1) {
+                             bytes += 16;
+                             dn += __dmul_rn(__ddiv_rn(c0, qq.x), __dadd_rn(1.0, qq.y));
+                         }
+                     });
+            scanned += r.y - r.x;
+            bytes += 8u * (r.y - r.x);
+            if (wantpush && (meta & kMetaExt)) {  // some predecessor outside D
+                row_walk(c.g, c.st, c.mark, r, [&](int dp) { return dp == l - 1; },
+                         [&](int pp, int dp, double2, uint32_t mp) {
+                             if (dp != l - 1 || mp == c.mD) return;
+                             double dlt = __ddiv_rn(1.0 + dn, c0);
+                             if ((meta & kMetaNotPulled) &&
+                                 !((meta & kMetaNew) && new_edge(c.g, x, pp, c.g0, c.lim)))
+                                 dlt = __dsub_rn(dlt, __ddiv_rn(1.0 + c1, c2));
+                             atomicAdd(c.dacc + pp, dlt);
+                             bytes += 24;
+                             up_claim(c, pp, mp);
+                         });
+                scanned += r.y - r.x;
+                bytes += 8u * (r.y - r.x);
+            }
+            c.st.sd[x].y = dn;  // d_finish
+            atomicAdd(c.bc + x, dn - c1);
+            bytes += 40;
+            continue;
+        }
+        // up_finish
+        c.dacc[x] = 0.0;
+        c.st.sd[x].y = c2 + c1;
+        atomicAdd(c.bc + x, c1);
+        bytes += 48;
+    }
+    __syncthreads();
+}
+
 __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a) {
     __shared__ int s_slot;
     __shared__ int s_dcnt;     // |D| (absolute positions in Dv)
@@ -676,12 +842,13 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                 s_hctx.kind = __ldcg(&src->kind);
                 s_hctx.lb = __ldcg(&src->lb);
                 s_hctx.mvalid = __ldcg(&src->mvalid);
+                s_hctx.aux = __ldcg(&src->aux);
                 __threadfence();  // acquire: drop stale L1 lines of the owner's state
             }
             __syncthreads();
             const ChunkSmem *mir = a.help.mir + pick;
             const int cnt = (s_hctx.kind == 0 || s_hctx.kind == 2) ? s_hctx.cnt : 0;  // kinds 0 and 2 publish a chunk
-            if ((s_hctx.kind == 1 || s_hctx.kind == 4) && s_hctx.mvalid && tid < 32) {  // the root's row (mask bits)
+            if ((s_hctx.kind == 1 || s_hctx.kind == 4 || s_hctx.kind == 5) && s_hctx.mvalid && tid < 32) {  // the root's row (mask bits)
                 const int2 rs = row_of(g, a.roots[s_hctx.root_slot], s_hctx.lim);
                 const int ds = rs.y - rs.x;
                 if (tid < ds && ds <= kMaskDeg) s_hadjs[tid] = ldg_i(g.col + rs.x + tid);
@@ -736,6 +903,37 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                min(cx.E2, (b + 1) * kDlEntries), a.ws.dacc + (size_t)pick * n, &s_t0, st_bytes,
                                sc_down);
             }
+        } else if (cx.kind == 5) {  // a block of a published in-lane up-level pass
+            UpCtx uc;
+            uc.g = g;
+            uc.st = ost;
+            uc.mark = a.ws.mark + (size_t)pick * n;
+            uc.dacc = a.ws.dacc + (size_t)pick * n;
+            uc.bc = a.bc;
+            uc.mask = a.l2mask + (size_t)cx.root_slot * n;
+            uc.Dv = a.ws.Dv + (size_t)pick * n;
+            uc.Dold = a.ws.Dold + (size_t)pick * n;
+            uc.Rv = a.ws.Rv + (size_t)pick * n;
+            uc.Rl = a.ws.Rl + (size_t)pick * n;
+            uc.Ul = a.ws.Bq + (size_t)pick * n;
+            uc.Uo = ((cx.aux >> 30) & 1 ? a.ws.U1 : a.ws.U0) + (size_t)pick * n;
+            uc.Dsig = a.ws.Dsig + (size_t)pick * n;
+            uc.adjs = s_hadjs;
+            uc.gU = a.help.gU + (size_t)pick * n;
+            uc.gapp = a.help.gapp + pick;
+            uc.xcnt = a.help.gbig + 2 * pick;
+            uc.X = a.ws.X + (size_t)pick * kXcap;
+            uc.l = cx.l;
+            uc.b0 = cx.lb;
+            uc.nDl = cx.E2;
+            uc.ucnt = cx.aux & ((1 << 30) - 1);
+            uc.g0 = cx.g0;
+            uc.lim = cx.lim;
+            uc.mok = cx.mvalid;
+            uc.E = cx.E;
+            uc.mU = cx.E | kUp;
+            uc.mD = cx.E | kDown;
+            up_block(uc, b * a.hd_block, min(cx.cnt, (b + 1) * a.hd_block), st_bytes, sc_up3);
         } else if (cx.kind == 3) {  // a block of a published removal pass (Case 3)
             RemCtx hr;
             hr.g = g;
@@ -1718,13 +1916,119 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                     for (int cb = 0; cb < total; cb += step) {
                         const int ce = min(total, cb + step);
                         int nDb = 0;
-                        if (cb < nDl) {  // down rows first: their pull precedes their push
-                            split_range(cb, min(ce, nDl), small_level || wide, wide);
+                        const int nblk5 = (total + a.hd_block - 1) / a.hd_block;
+                        if (wide && a.help.word && nblk5 >= a.he_min && worth(nblk5)) {
+                            // the in-lane pass as help blocks (kind 5): every long row is
+                            // deferred to Xw (the owner's chunks below), appends via gU
+                            const int nl = min(ucnt, kUcap);
+                            for (int i = tid; i < nl; i += kBlock) Bq[i] = s_un[ucur_sel][i];
+                            UpCtx uc;
+                            uc.g = g;
+                            uc.st = st;
+                            uc.mark = mark;
+                            uc.dacc = dacc;
+                            uc.bc = a.bc;
+                            uc.mask = mask;
+                            uc.Dv = Dv;
+                            uc.Dold = Dold;
+                            uc.Rv = Rv;
+                            uc.Rl = Rl;
+                            uc.Ul = Bq;
+                            uc.Uo = Ucur;
+                            uc.Dsig = Dsig;
+                            uc.adjs = s_adjs;
+                            uc.gU = a.help.gU + (size_t)wk * n;
+                            uc.gapp = a.help.gapp + wk;
+                            uc.xcnt = a.help.gbig + 2 * wk;
+                            uc.X = Xw;
+                            uc.l = l;
+                            uc.b0 = b0;
+                            uc.nDl = nDl;
+                            uc.ucnt = ucnt;
+                            uc.g0 = g0;
+                            uc.lim = lim;
+                            uc.mok = mok;
+                            uc.E = E;
+                            uc.mU = mU;
+                            uc.mD = mD;
+                            if (tid == 0) {
+                                HelpCtx cx;
+                                cx.root_slot = slot;
+                                cx.l = l;
+                                cx.g0 = g0;
+                                cx.lim = lim;
+                                cx.cnt = total;
+                                cx.nblocks = nblk5;
+                                cx.E2 = nDl;
+                                cx.E = E;
+                                cx.kind = 5;
+                                cx.lb = b0;
+                                cx.mvalid = mok;
+                                cx.aux = ucnt | ((Ucur == Ub) ? (1 << 30) : 0);
+                                a.help.ctx[wk] = cx;
+                                a.help.done[wk] = 0;
+                                a.help.gapp[wk] = 0;
+                                a.help.gbig[2 * wk] = 0;
+                                a.help.gbig[2 * wk + 1] = 0;
+                            }
+                            __syncthreads();  // the frontier copy is written; one release fence publishes it
+                            if (tid == 0) {
+                                __threadfence();
+                                atomicAdd(a.stats + kStHelpReq, 1ull);
+                                atomicAdd(a.stats + kStHelpBlkAll, (unsigned long long)nblk5);
+                                atomicAdd(a.stats + kStUpPass, 1ull);
+                                hseq = (hseq + 1) & 0xFFFF;
+                                atomicExch(a.help.word + wk, help_pack(1, nblk5, 0, hseq));
+                                if (nblk5 >= a.busy_min) atomicAdd(a.help.roots_left + 1, 1);
+                            }
+                            for (;;) {  // the owner takes blocks too
+                                if (tid == 0) {
+                                    const unsigned long long w = atomicAdd(a.help.word + wk, 1ull << 16);
+                                    s_hb = help_next(w) < nblk5 ? help_next(w) : -1;
+                                }
+                                __syncthreads();
+                                const int b = s_hb;
+                                __syncthreads();
+                                if (b < 0) break;
+                                ++own_blk;
+                                up_block(uc, b * a.hd_block, min(total, (b + 1) * a.hd_block), st_bytes,
+                                         sc_up3);  // ends with a barrier
+                                if (tid == 0) {
+                                    __threadfence();
+                                    atomicAdd(a.help.done + wk, 1);
+                                }
+                            }
+                            trace(6, 5, own_blk | (nblk5 << 16));
+                            own_blk = 0;
+                            if (tid == 0) {  // wait for the helpers' blocks, then close
+                                while (atomicAdd(a.help.done + wk, 0) < nblk5) __nanosleep(256);
+                                atomicExch(a.help.word + wk, help_pack(0, 0, 0, hseq));
+                                if (nblk5 >= a.busy_min) atomicSub(a.help.roots_left + 1, 1);
+                                __threadfence();
+                                s_nx[0] = __ldcg(a.help.gbig + 2 * wk);
+                                s_nx[1] = __ldcg(a.help.gbig + 2 * wk + 1);
+                                s_nbigI = 0;
+                            }
                             __syncthreads();
-                            nDb = min(s_nbigI, kChunk);
+                            const int gc = __ldcg(a.help.gapp + wk);  // merge the global appends
+                            for (int i = tid; i < gc; i += kBlock) {
+                                const int y = __ldcg(uc.gU + i);
+                                const int pos = atomicAdd(&s_ucnt2[ucur_sel ^ 1], 1);
+                                if (pos < kUcap)
+                                    s_un[ucur_sel ^ 1][pos] = y;
+                                else
+                                    Unext[pos - kUcap] = y;
+                            }
+                            __syncthreads();
+                        } else {
+                            if (cb < nDl) {  // down rows first: their pull precedes their push
+                                split_range(cb, min(ce, nDl), small_level || wide, wide);
+                                __syncthreads();
+                                nDb = min(s_nbigI, kChunk);
+                            }
+                            split_range(max(cb, nDl), ce, small_level || wide, wide);
+                            __syncthreads();
                         }
-                        split_range(max(cb, nDl), ce, small_level || wide, wide);
-                        __syncthreads();
                         if (first_barrier) {  // the current list's count was read last level
                             first_barrier = false;
                             if (tid == 0) s_ucnt2[ucur_sel] = 0;

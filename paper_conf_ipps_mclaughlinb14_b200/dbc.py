@@ -271,7 +271,7 @@ class DynamicBC:
                  "ns_down", "ns_removal", "ns_up_setup", "ns_up_epi", "ns_up_l1pairs", "ns_up_end",
                  "ns_up_split", "ns_up_scan", "ns_up_pull", "ns_up_push", "levels_down", "levels_up",
                  "help_requests", "help_blocks_by_helpers", "help_blocks_all",
-                 "case2_groups", "case2_group_insertions", "help_blocks_busy", "deferred_rows"]
+                 "case2_groups", "case2_group_insertions", "help_blocks_busy", "deferred_rows", "up_passes_helped"]
         out = np.zeros(len(names), dtype=np.int64)
         _check(self._ctx, self._lib.dbc_debug_counters(self._ctx, _np_ptr(out), out.size))
         return dict(zip(names, out.tolist()))
@@ -280,7 +280,7 @@ class DynamicBC:
         """Per-level event trace of the slot named by DBC_TRACE_SLOT (builds with
         -DDBC_PHASE_TIMERS only): list of (kind, level, items, t_ns); kinds 1 down
         level, 2 up level, 3 removal pass, 4 job end."""
-        base = 33  # kStTraceN (after the debug_counters names)
+        base = 34  # kStTraceN (after the debug_counters names)
         out = np.zeros(base + 1 + 2 * 1024, dtype=np.int64)
         _check(self._ctx, self._lib.dbc_debug_counters(self._ctx, _np_ptr(out), out.size))
         cnt = min(int(out[base]), 1024)

@@ -751,11 +751,13 @@ def test_forced_help_paths_match_oracle(name, block, monkeypatch):
 
 @pytest.mark.parametrize("block", [None, "512"])
 def test_wide_up_levels_deferred_chunks_match_oracle(block, monkeypatch):
-    """Wide up levels walked with short rows in-lane and long rows in chunks,
-    more than one chunk of them deferred (DBC_WIDE_INLANE forces the mode on
-    every level wider than a CTA): R-MAT 2^14 / edgefactor 16, 64 roots, 400
-    insertions in two batches; d/sigma bit-exact vs the oracle, BC in tolerance."""
+    """Wide up levels walked with short rows in-lane (published as help blocks,
+    kind 5) and long rows in chunks, more than one chunk of them deferred
+    (DBC_WIDE_INLANE forces the mode on every level wider than a CTA): R-MAT
+    2^14 / edgefactor 16, 64 roots, 400 insertions in two batches; d/sigma
+    bit-exact vs the oracle, BC in tolerance."""
     monkeypatch.setenv("DBC_WIDE_INLANE", "100000")
+    monkeypatch.setenv("DBC_BUSY_MIN", "1")  # every pass worth publishing (kind-5 help blocks too)
     if block:
         monkeypatch.setenv("DBC_BLOCK", block)
     wl = W.make_workload("rmat14")
@@ -770,3 +772,4 @@ def test_wide_up_levels_deferred_chunks_match_oracle(block, monkeypatch):
         c1 = dbc.debug_counters()
         check_all(dbc, ref.compute(), wl.roots.size)
         assert c1["deferred_rows"] > c0["deferred_rows"]  # more than one chunk of long rows
+        assert c1["up_passes_helped"] > c0["up_passes_helped"]  # kind-5 help blocks ran
