@@ -773,3 +773,46 @@ def test_wide_up_levels_deferred_chunks_match_oracle(block, monkeypatch):
         check_all(dbc, ref.compute(), wl.roots.size)
         assert c1["deferred_rows"] > c0["deferred_rows"]  # more than one chunk of long rows
         assert c1["up_passes_helped"] > c0["up_passes_helped"]  # kind-5 help blocks ran
+
+
+def _sampled_bench_batch(name, sample, rank=0, world=1):
+    """A full-size config exactly as bench.py times it: the config's whole batch
+    in ONE Mode A launch (kron20: 1024 roots, 10,000 insertions; kron22: rank
+    `rank` of `world`'s root shard, 10,000 insertions), then sampled local roots'
+    d/sigma bit-exact and delta within tolerance vs the oracle's Brandes on the
+    final graph (P:440 semantics: the batch == its insertions one at a time)."""
+    from paper_conf_ipps_mclaughlinb14_b200 import DynamicBC
+
+    wl = W.make_workload(name)
+    g = wl.graph
+    with DynamicBC(g.n, g.row_ptr, g.col, wl.roots, rank=rank, world=world) as dbc:
+        k_loc = dbc.num_local_roots()
+        assert k_loc == len(range(rank, wl.roots.size, world))
+        dbc.static_compute()
+        st = dbc.insert_edges(wl.ins_u, wl.ins_v, stats=True)
+        assert st["case1"] + st["case2"] + st["case3"] == k_loc * wl.ins_u.size
+        ref = oracle.NaiveDynamicBC(g, wl.roots)
+        for u, v in zip(wl.ins_u, wl.ins_v):
+            ref.insert(u, v)
+        rp, col = ref.csr()
+        loc = np.linspace(0, k_loc - 1, sample).astype(np.int64)
+        slots = loc * world + rank  # global slots this rank owns (slot % world == rank)
+        _, d_ref, s_ref, dl_ref = oracle.brandes(g.n, rp, col, wl.roots[slots])
+        for i, slot in enumerate(slots):
+            d, s, dl = dbc.get_root_state(int(slot))
+            assert np.array_equal(d, d_ref[i]), f"d slot {slot}"
+            assert np.array_equal(s, s_ref[i]), f"sigma slot {slot}"
+            err = np.abs(dl - dl_ref[i]) / np.maximum(np.abs(dl_ref[i]), 1.0)
+            assert err.max() <= DELTA_TOL
+
+
+@pytest.mark.timeout(600)
+def test_kron20_bench_batch_sampled():
+    _sampled_bench_batch("kron20", 3)
+
+
+@pytest.mark.timeout(1200)
+def test_kron22_shard_bench_batch_sampled():
+    """BASELINE configs[4]'s per-GPU unit: rank 0 of 8 (512 roots, 51.5 GB of
+    d/sigma/delta on one B200), one 10,000-insertion batch."""
+    _sampled_bench_batch("kron22", 2, rank=0, world=8)
