@@ -702,7 +702,7 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     }
     const int nb = 1 - c->cur;
     launches += append_batch(c->ab, c->rp[c->cur], c->col[c->cur], c->scol[c->cur], c->rp[nb],
-                             c->col[nb], c->scol[nb], c->n, c->stream);
+                             c->col[nb], c->scol[nb], c->n, c->nnz, c->stream);
     CK(cudaGetLastError());
     c->cur = nb;
     c->nnz += 2 * cnt;

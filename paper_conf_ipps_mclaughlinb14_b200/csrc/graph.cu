@@ -206,50 +206,58 @@ __global__ void k_group_sort(const int32_t *xcnt, const int32_t *xoff, int32_t n
     xinfo[x] = make_int2(b, c);
 }
 
-// warp per vertex: copy the old row to its new place, append the batch group
-__global__ void k_copy_rows(const int32_t *rp_old, const int32_t *col_old, const int32_t *rp_new,
-                            int32_t *col_new, const int32_t *xcnt, const int32_t *xoff,
-                            const int32_t *gnbr, int32_t n) {
-    const int lane = threadIdx.x & 31;
-    const int64_t warps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t x = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; x < n; x += warps) {
-        const int ob = rp_old[x] & kMask, oe = rp_old[x + 1] & kMask, nb = rp_new[x];
-        for (int j = lane; j < oe - ob; j += 32) col_new[nb + j] = col_old[ob + j];
-        const int c = xcnt[x];
-        if (c) {
-            const int g0 = xoff[x], dst = nb + (oe - ob);
-            for (int j = lane; j < c; j += 32) col_new[dst + j] = gnbr[g0 + j];
+// Thread per old entry j (flat over all rows, so a hub row costs no more than
+// its share of the entries): its row x is found by binary search of rp_old.  The
+// canonical row keeps its order and moves to rp_new[x] (the batch group goes
+// after it, k_place_groups); in the sorted row the entry moves right by the
+// number of the group's neighbours smaller than it.
+__global__ void k_copy_entries(const int32_t *__restrict__ rp_old, const int32_t *__restrict__ col_old,
+                               const int32_t *__restrict__ scol_old, const int32_t *__restrict__ rp_new,
+                               int32_t *__restrict__ col_new, int32_t *__restrict__ scol_new,
+                               const int32_t *__restrict__ xcnt, const int32_t *__restrict__ xoff,
+                               const int32_t *__restrict__ gnbr, int32_t n, int64_t nnz_old) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < nnz_old; j += stride) {
+        int lo = 0, hi = n;  // rp_old[lo] <= j < rp_old[hi]: the row of j is the last such lo
+        while (hi - lo > 1) {
+            const int mid = (lo + hi) >> 1;
+            if ((__ldg(rp_old + mid) & kMask) <= j) lo = mid; else hi = mid;
         }
+        const int x = lo;
+        const int64_t off = j - (__ldg(rp_old + x) & kMask), nb = __ldg(rp_new + x);
+        col_new[nb + off] = __ldg(col_old + j);
+        const int val = __ldg(scol_old + j), c = __ldg(xcnt + x);
+        int less = 0;
+        if (c) {
+            const int g0 = __ldg(xoff + x);
+            for (int k = 0; k < c; ++k) less += __ldg(gnbr + g0 + k) < val;
+        }
+        scol_new[nb + off + less] = val;
     }
 }
 
-// warp per vertex: the sorted copy of each row -- old sorted row merged with
-// the batch group (both sides locate their slot by counting the other side)
-__global__ void k_copy_rows_sorted(const int32_t *rp_old, const int32_t *scol_old,
-                                   const int32_t *rp_new, int32_t *scol_new, const int32_t *xcnt,
-                                   const int32_t *xoff, const int32_t *gnbr, int32_t n) {
+// warp per vertex with a batch group (a hub can get hundreds of the batch's
+// edges): the group appended after the canonical row (P:440 order), and each
+// group neighbour placed in the sorted row (old entries below it by binary
+// search, group entries below it by counting)
+__global__ void k_place_groups(const int32_t *__restrict__ rp_old, const int32_t *__restrict__ scol_old,
+                               const int32_t *__restrict__ rp_new, int32_t *__restrict__ col_new,
+                               int32_t *__restrict__ scol_new, const int32_t *__restrict__ xcnt,
+                               const int32_t *__restrict__ xoff, const int32_t *__restrict__ gnbr,
+                               int32_t n) {
     const int lane = threadIdx.x & 31;
     const int64_t warps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     for (int64_t x = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; x < n; x += warps) {
-        const int ob = rp_old[x] & kMask, oe = rp_old[x + 1] & kMask, nb = rp_new[x];
         const int c = xcnt[x];
-        if (c == 0) {
-            for (int j = lane; j < oe - ob; j += 32) scol_new[nb + j] = scol_old[ob + j];
-            continue;
-        }
-        const int g0 = xoff[x];
-        for (int j = lane; j < oe - ob; j += 32) {
-            const int val = scol_old[ob + j];
-            int less = 0;
-            for (int k = 0; k < c; ++k) less += gnbr[g0 + k] < val;
-            scol_new[nb + j + less] = val;
-        }
+        if (c == 0) continue;
+        const int ob = rp_old[x] & kMask, len = (rp_old[x + 1] & kMask) - ob, nb = rp_new[x], g0 = xoff[x];
         for (int k = lane; k < c; k += 32) {
             const int val = gnbr[g0 + k];
-            int lo = 0, hi = oe - ob;  // old entries < val
+            col_new[nb + len + k] = val;
+            int lo = 0, hi = len;  // old entries < val
             while (lo < hi) {
                 const int mid = (lo + hi) >> 1;
-                if (scol_old[ob + mid] < val) lo = mid + 1; else hi = mid;
+                if (__ldg(scol_old + ob + mid) < val) lo = mid + 1; else hi = mid;
             }
             int less = 0;
             for (int q = 0; q < c; ++q) less += gnbr[g0 + q] < val;
@@ -298,16 +306,17 @@ int validate_batch(const AppendBufs &B, const GView &g, const int32_t *rp_old, i
 
 int append_batch(const AppendBufs &B, const int32_t *rp_old, const int32_t *col_old,
                  const int32_t *scol_old, int32_t *rp_new, int32_t *col_new, int32_t *scol_new,
-                 int32_t n, cudaStream_t s) {
+                 int32_t n, int64_t nnz_old, cudaStream_t s) {
     int launches = 0;
     k_degrees<<<blocks_for((int64_t)n + 1, 256), 256, 0, s>>>(rp_old, B.xcnt, n, B.deg);
     launches += 1 + scan_launch(B.deg, rp_new, (int64_t)n + 1, B.sums, s);
-    k_copy_rows<<<std::min<int64_t>(blocks_for((int64_t)n * 32, 256), 148 * 16), 256, 0, s>>>(
-        rp_old, col_old, rp_new, col_new, B.xcnt, B.xoff, B.gnbr, n);
-    k_copy_rows_sorted<<<std::min<int64_t>(blocks_for((int64_t)n * 32, 256), 148 * 16), 256, 0, s>>>(
-        rp_old, scol_old, rp_new, scol_new, B.xcnt, B.xoff, B.gnbr, n);
+    if (nnz_old > 0)
+        k_copy_entries<<<std::min<int64_t>(blocks_for(nnz_old, 256), 148 * 64), 256, 0, s>>>(
+            rp_old, col_old, scol_old, rp_new, col_new, scol_new, B.xcnt, B.xoff, B.gnbr, n, nnz_old);
+    k_place_groups<<<std::min<int64_t>(blocks_for((int64_t)n * 32, 256), 148 * 16), 256, 0, s>>>(
+        rp_old, scol_old, rp_new, col_new, scol_new, B.xcnt, B.xoff, B.gnbr, n);
     k_flag_rows<<<blocks_for(n, 256), 256, 0, s>>>(B.xcnt, n, rp_new);
-    return launches + 3;
+    return launches + 2 + (nnz_old > 0);
 }
 
 // external -> internal vertex ids of a batch (out-of-range ids are passed

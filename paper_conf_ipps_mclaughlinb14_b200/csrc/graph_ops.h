@@ -32,7 +32,7 @@ int tombstone_edge(const int32_t *rp, int32_t *col, int32_t *scol, const int32_t
                    int64_t i, cudaStream_t s);
 int append_batch(const AppendBufs &B, const int32_t *rp_old, const int32_t *col_old,
                  const int32_t *scol_old, int32_t *rp_new, int32_t *col_new, int32_t *scol_new,
-                 int32_t n, cudaStream_t s);
+                 int32_t n, int64_t nnz_old, cudaStream_t s);
 int map_ids(const int32_t *su, const int32_t *sv, int32_t *du, int32_t *dv, int64_t cnt,
             const int32_t *perm, int32_t n, cudaStream_t s);
 int gather_ext(const double *in, const int32_t *perm, int32_t n, double *out, cudaStream_t s);
