@@ -180,30 +180,53 @@ __global__ void k_group_scatter(const int32_t *u, const int32_t *v, int64_t cnt,
     gnbr[p] = a;
 }
 
-// per vertex with batch entries: order its group by insertion index (canonical
-// order), detect duplicate edges within the batch, publish xinfo.
+// warp per vertex with batch entries: order its group by insertion index
+// (canonical order), detect duplicate edges within the batch, publish xinfo.
+// Groups of up to 32 entries (all but the rarest hubs) are ranked in registers,
+// one entry per lane (ties broken by lane: a self loop's two entries -- the
+// batch is rejected anyway -- still land in distinct slots); larger groups are
+// insertion-sorted by lane 0.
 __global__ void k_group_sort(const int32_t *xcnt, const int32_t *xoff, int32_t n, int32_t *gtag,
                              int32_t *gnbr, int2 *xinfo, int32_t *bad) {
-    const int64_t x = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (x >= n) return;
-    const int c = xcnt[x];
-    if (c == 0) return;
-    const int b = xoff[x];
-    for (int i = 1; i < c; ++i) {  // insertion sort (groups are tiny)
-        const int t = gtag[b + i], nb = gnbr[b + i];
-        int j = i - 1;
-        while (j >= 0 && gtag[b + j] > t) {
-            gtag[b + j + 1] = gtag[b + j];
-            gnbr[b + j + 1] = gnbr[b + j];
-            --j;
+    const int lane = threadIdx.x & 31;
+    const int64_t warps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t x = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; x < n; x += warps) {
+        const int c = xcnt[x];
+        if (c == 0) continue;
+        const int b = xoff[x];
+        if (c <= 32) {
+            const int t = lane < c ? gtag[b + lane] : INT32_MAX, nb = lane < c ? gnbr[b + lane] : -1;
+            int rank = 0;
+            bool dup = false;
+            for (int j = 0; j < c; ++j) {
+                const int tj = __shfl_sync(kFull, t, j), nj = __shfl_sync(kFull, nb, j);
+                rank += (tj < t) || (tj == t && j < lane);
+                dup |= (j != lane) && (nj == nb);
+            }
+            __syncwarp();
+            if (lane < c) {
+                gtag[b + rank] = t;
+                gnbr[b + rank] = nb;
+                if (dup) atomicOr(bad, 4);
+            }
+        } else if (lane == 0) {
+            for (int i = 1; i < c; ++i) {  // insertion sort
+                const int t = gtag[b + i], nb = gnbr[b + i];
+                int j = i - 1;
+                while (j >= 0 && gtag[b + j] > t) {
+                    gtag[b + j + 1] = gtag[b + j];
+                    gnbr[b + j + 1] = gnbr[b + j];
+                    --j;
+                }
+                gtag[b + j + 1] = t;
+                gnbr[b + j + 1] = nb;
+            }
+            for (int i = 1; i < c; ++i)
+                for (int j = 0; j < i; ++j)
+                    if (gnbr[b + j] == gnbr[b + i]) atomicOr(bad, 4);
         }
-        gtag[b + j + 1] = t;
-        gnbr[b + j + 1] = nb;
+        if (lane == 0) xinfo[x] = make_int2(b, c);
     }
-    for (int i = 1; i < c; ++i)
-        for (int j = 0; j < i; ++j)
-            if (gnbr[b + j] == gnbr[b + i]) atomicOr(bad, 4);
-    xinfo[x] = make_int2(b, c);
 }
 
 // Thread per old entry j (flat over all rows, so a hub row costs no more than
@@ -296,8 +319,8 @@ int validate_batch(const AppendBufs &B, const GView &g, const int32_t *rp_old, i
     if (cnt) {
         k_group_scatter<<<blocks_for(cnt, 256), 256, 0, s>>>(u, v, cnt, n, B.xoff, B.slot, B.xtag,
                                                             B.gnbr);
-        k_group_sort<<<blocks_for(n, 256), 256, 0, s>>>(B.xcnt, B.xoff, n, B.xtag, B.gnbr, B.xinfo,
-                                                       B.bad);
+        k_group_sort<<<std::min<int64_t>(blocks_for((int64_t)n * 32, 256), 148 * 16), 256, 0, s>>>(
+            B.xcnt, B.xoff, n, B.xtag, B.gnbr, B.xinfo, B.bad);
         launches += 2;
     }
     (void)rp_old;
