@@ -106,6 +106,67 @@ def brandes_csr(g, roots, want_state=True):
     return brandes(g.n, g.row_ptr, g.col, roots, want_state)
 
 
+def host_threads() -> int:
+    """Host cores this process may use (the root-parallel leg's thread count)."""
+    try:
+        return max(1, len(os.sched_getaffinity(0)))
+    except AttributeError:  # pragma: no cover
+        return max(1, os.cpu_count() or 1)
+
+
+def brandes_parallel(n, row_ptr, col, roots, threads=None, state_slots=None):
+    """Root-parallel leg of `brandes` (SURVEY.md Sec. 8(d) oracle timing (ii)).
+
+    The SAME per-root computation (oracle_brandes called with one root, so
+    Alg. 1 / Eq. (2) run unchanged, in canonical order) is spread over host
+    threads; BC is then Eq. (3) summed in slot order -- bc = ((0 + delta_0) +
+    delta_1) + ..., one IEEE add per slot and vertex exactly as brandes.c does
+    (delta_s(s) = 0, so adding slot s's whole row equals skipping v = s).  The
+    result is therefore bit-identical to `brandes` (pinned in
+    tests/test_oracle.py).  Roots run in waves of `threads` so only
+    threads x n deltas are held at once.
+
+    state_slots: None -> no per-root state returned; an index array -> (d,
+    sigma, delta) of those slots (rows in the order given).
+    Returns (bc[n], d, sigma, delta)."""
+    from concurrent.futures import ThreadPoolExecutor
+
+    lib = _load()
+    row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
+    col = np.ascontiguousarray(col, dtype=np.int32)
+    roots = np.ascontiguousarray(roots, dtype=np.int32)
+    k = roots.size
+    T = max(1, int(threads or host_threads()))
+    want = {} if state_slots is None else {int(s): i for i, s in enumerate(state_slots)}
+    m = len(want)
+    d = np.empty((m, n), np.int32) if m else None
+    sig = np.empty((m, n), np.float64) if m else None
+    dl = np.empty((m, n), np.float64) if m else None
+    bc = np.zeros(n, dtype=np.float64)
+    wave = np.empty((min(T, max(k, 1)), n), np.float64)
+    rbuf = [np.empty(1, np.int32) for _ in range(wave.shape[0])]
+
+    def one(slot, j):
+        rbuf[j][0] = roots[slot]
+        i = want.get(slot)
+        rc = lib.oracle_brandes(n, _ptr(row_ptr), _ptr(col), _ptr(rbuf[j]), 1,
+                                None if i is None else _ptr(d[i]),
+                                None if i is None else _ptr(sig[i]),
+                                _ptr(wave[j]), None)
+        if rc != 0:
+            raise RuntimeError(f"oracle_brandes failed: {rc}")
+        if i is not None:
+            dl[i] = wave[j]
+
+    with ThreadPoolExecutor(max_workers=T) as ex:
+        for s0 in range(0, k, T):
+            s1 = min(k, s0 + T)
+            list(ex.map(lambda a: one(*a), [(s, s - s0) for s in range(s0, s1)]))
+            for s in range(s0, s1):  # Eq. (3) in slot order
+                bc += wave[s - s0]
+    return bc, d, sig, dl
+
+
 class NaiveDynamicBC:
     """Naive dynamic rule: keep the canonical adjacency, recompute after each insertion."""
 

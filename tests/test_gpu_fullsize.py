@@ -1,0 +1,178 @@
+"""Full-size GPU parity against the oracle (BASELINE.json configs 2-5, SURVEY.md
+Sec. 8(d) "parity check cadence"; "we compare the results of the
+baseline and our algorithms").
+
+Every check recomputes the FINAL graph with the oracle over ALL roots (the
+root-parallel leg, `oracle.brandes_parallel`, bit-identical to the
+single-thread oracle and run on every host core) and compares:
+  * BC of every vertex: |bc - ref| <= 1e-9 * max(|ref|, 1) (north star);
+  * d and sigma bit-exact, delta within 1e-12 * max(|ref|, 1)
+     on >= 64 sampled roots (all roots where the
+    config has fewer);
+  * GPU dynamic == GPU static recompute (bitwise d / sigma) on the sampled roots.
+Configs run in the launch configuration bench.py times (default flags, one
+batch of the config's size) and, where SURVEY.md Sec. 8(d) asks for a cadence,
+in batches of that cadence.
+"""
+
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+import oracle
+import workloads as W
+
+pytestmark = pytest.mark.gpu
+
+BC_TOL = 1e-9
+DELTA_TOL = 1e-12
+SAMPLE = 64
+
+
+def _bc_err(bc, ref):
+    return float((np.abs(bc - ref) / np.maximum(np.abs(ref), 1.0)).max(initial=0.0))
+
+
+class Ref:
+    """The naive rule (oracle.NaiveDynamicBC's canonical rows) + the root-parallel oracle."""
+
+    def __init__(self, wl, local_slots):
+        self.dyn = oracle.NaiveDynamicBC(wl.graph, wl.roots)
+        self.n = wl.graph.n
+        self.local = np.asarray(local_slots, np.int64)  # global slots of the context's roots
+        self.roots = wl.roots[self.local]
+
+    def insert(self, us, vs):
+        for u, v in zip(us, vs):
+            self.dyn.insert(int(u), int(v))
+
+    def compute(self, sample_local):
+        rp, col = self.dyn.csr()
+        return oracle.brandes_parallel(self.n, rp, col, self.roots, state_slots=sample_local)
+
+
+def check(dbc, ref: Ref, sample_local, what=""):
+    """BC over all of the context's roots + d/sigma/delta on sample_local (local indices)."""
+    bc_ref, d_ref, s_ref, dl_ref = ref.compute(sample_local)
+    bc = dbc.get_bc()
+    err = _bc_err(bc, bc_ref)
+    assert err <= BC_TOL, f"{what}: BC rel err {err}"
+    worst = 0.0
+    for i, li in enumerate(sample_local):
+        slot = int(ref.local[li])
+        d, s, dl = dbc.get_root_state(slot)
+        assert np.array_equal(d, d_ref[i]), f"{what}: d mismatch slot {slot}"
+        bad = np.nonzero(s != s_ref[i])[0]
+        assert bad.size == 0, f"{what}: sigma mismatch slot {slot} at {bad[:4]}"
+        e = float((np.abs(dl - dl_ref[i]) / np.maximum(np.abs(dl_ref[i]), 1.0)).max(initial=0.0))
+        worst = max(worst, e)
+        assert e <= DELTA_TOL, f"{what}: delta rel err {e} slot {slot}"
+    return err, worst
+
+
+def dynamic_equals_static(dbc, ref: Ref, sample_local):
+    dyn = {int(ref.local[li]): dbc.get_root_state(int(ref.local[li]))[:2] for li in sample_local}
+    dbc.static_compute()
+    for slot, (d0, s0) in dyn.items():
+        d1, s1, _ = dbc.get_root_state(slot)
+        assert np.array_equal(d0, d1) and np.array_equal(s0, s1), f"dynamic != static slot {slot}"
+
+
+def _sample(k_loc, m=SAMPLE):
+    return np.unique(np.linspace(0, k_loc - 1, min(m, k_loc)).astype(np.int64))
+
+
+def run_cadence(name, batch, flags=0, sample=SAMPLE, state_every=1, insertions=None):
+    """Insert the config's stream in batches of `batch`; after every batch BC over
+    all roots, and every `state_every` batches d/sigma/delta on the sample."""
+    from paper_conf_ipps_mclaughlinb14_b200 import DynamicBC
+
+    wl = W.make_workload(name, insertions=insertions)
+    g = wl.graph
+    k = wl.roots.size
+    ref = Ref(wl, np.arange(k))
+    smp = _sample(k, sample)
+    worst = [0.0, 0.0]
+    with DynamicBC(g.n, g.row_ptr, g.col, wl.roots, flags=flags) as dbc:
+        dbc.static_compute()
+        nb = (wl.ins_u.size + batch - 1) // batch
+        for b in range(nb):
+            sl = slice(b * batch, (b + 1) * batch)
+            dbc.insert_edges(wl.ins_u[sl], wl.ins_v[sl])
+            ref.insert(wl.ins_u[sl], wl.ins_v[sl])
+            full = (b + 1) % state_every == 0 or b == nb - 1
+            e = check(dbc, ref, smp if full else np.zeros(0, np.int64), f"{name} after {sl.stop}")
+            worst = [max(worst[0], e[0]), max(worst[1], e[1])]
+        dynamic_equals_static(dbc, ref, smp[:8])
+    print(f"{name} batch {batch} flags {flags:#x}: max BC rel err {worst[0]:.2e}, "
+          f"max delta rel err {worst[1]:.2e}")
+
+
+# ---------------------------------------------------------------- config 2 ----
+@pytest.mark.timeout(900)
+def test_rmat16_every_10th_insertion_all_roots():
+    """Config 2 at SURVEY.md Sec. 8(d)'s cadence: every 10th insertion, BC over
+    all 256 roots; all 256 roots' d/sigma/delta every 100th and at the end."""
+    run_cadence("rmat16", 10, sample=256, state_every=10)
+
+
+@pytest.mark.timeout(600)
+def test_rmat16_bench_batch_all_roots():
+    """Config 2 exactly as bench.py times it: one 1,000-insertion batch."""
+    run_cadence("rmat16", 1000, sample=256)
+
+
+# ---------------------------------------------------------------- config 3 ----
+@pytest.mark.timeout(900)
+def test_delaunay18_every_100th_all_roots():
+    """Config 3 (remove-then-reinsert): every 100th insertion, BC over all 512
+    roots, d/sigma/delta on 64 sampled roots (sigma reaches 2^100 here)."""
+    run_cadence("delaunay18", 100)
+
+
+@pytest.mark.timeout(900)
+def test_delaunay18_bench_batch_all_roots():
+    run_cadence("delaunay18", 1000)
+
+
+@pytest.mark.timeout(1500)
+def test_delaunay18_uniform_nonedge_stress_all_roots():
+    """Config 3's stress variant (uniform random non-edges: long-range Case-3
+    pull-ups), every 100th insertion, BC over all 512 roots."""
+    run_cadence("delaunay18u", 100)
+
+
+# ------------------------------------------------------------ configs 4, 5 ----
+def run_bench_batch(name, rank=0, world=1):
+    """The config's whole 10,000-insertion batch in ONE call (bench.py's launch
+    configuration), BC over all of this rank's roots (the rank's partial, Eq. (3)
+    over slots with slot % world == rank) and 64 sampled roots' state."""
+    from paper_conf_ipps_mclaughlinb14_b200 import DynamicBC
+
+    wl = W.make_workload(name)
+    g = wl.graph
+    local = np.arange(rank, wl.roots.size, world)
+    ref = Ref(wl, local)
+    with DynamicBC(g.n, g.row_ptr, g.col, wl.roots, rank=rank, world=world) as dbc:
+        assert dbc.num_local_roots() == local.size
+        dbc.static_compute()
+        st = dbc.insert_edges(wl.ins_u, wl.ins_v, stats=True)
+        assert st["case1"] + st["case2"] + st["case3"] == local.size * wl.ins_u.size
+        ref.insert(wl.ins_u, wl.ins_v)
+        smp = _sample(local.size)
+        e = check(dbc, ref, smp, name)
+        dynamic_equals_static(dbc, ref, smp[:4])
+    print(f"{name} rank {rank}/{world}: BC rel err {e[0]:.2e}, delta rel err {e[1]:.2e}")
+
+
+@pytest.mark.timeout(1800)
+def test_kron20_bench_batch_all_roots():
+    """Config 4 on one GPU: 1,024 roots, one 10,000-insertion batch."""
+    run_bench_batch("kron20")
+
+
+@pytest.mark.timeout(2400)
+def test_kron22_shard_bench_batch_all_local_roots():
+    """Config 5's per-GPU unit: rank 0 of 8 (512 roots, 51.5 GB of state)."""
+    run_bench_batch("kron22", rank=0, world=8)

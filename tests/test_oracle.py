@@ -470,3 +470,32 @@ def test_delete_keeps_row_order():
     assert col[rp[0]:rp[1]].tolist() == [1, 3]
     assert col[rp[1]:rp[2]].tolist() == [0, 2]
     assert col[rp[2]:rp[3]].tolist() == [1]
+
+
+# --------------------------------------------------------------------------
+# root-parallel leg (SURVEY.md Sec. 8(d) oracle timing (ii)): the same per-root
+# computation spread over host threads, Eq. (3) summed in slot order -- must be
+# bit-identical to the single-thread path (and so inherits all its pins)
+# --------------------------------------------------------------------------
+@pytest.mark.parametrize("name", ["karate", "rmat10", "delaunay12u", "grid", "multi"])
+@pytest.mark.parametrize("threads", [1, 3, 8])
+def test_brandes_parallel_bitwise_equals_single_thread(name, threads):
+    if name == "grid":
+        g = W.grid_graph(30, 30)
+        roots = np.array([0, 31, 450, 899, 17], np.int32)
+    elif name == "multi":
+        g = W.random_gnm(300, 280, 5)  # several components: INF rows
+        roots = np.arange(0, 300, 7, dtype=np.int32)
+    else:
+        wl = W.make_workload(name)
+        g, roots = wl.graph, wl.roots
+    bc, d, sig, dl = oracle.brandes(g.n, g.row_ptr, g.col, roots)
+    slots = np.array(sorted({0, roots.size - 1, roots.size // 2}), np.int64)
+    pbc, pd, psig, pdl = oracle.brandes_parallel(g.n, g.row_ptr, g.col, roots, threads=threads,
+                                                 state_slots=slots)
+    assert np.array_equal(pbc.view(np.int64), bc.view(np.int64))  # bitwise, incl. signed zeros
+    assert np.array_equal(pd, d[slots])
+    assert np.array_equal(psig.view(np.int64), sig[slots].view(np.int64))
+    assert np.array_equal(pdl.view(np.int64), dl[slots].view(np.int64))
+    pbc2, pd2, _, _ = oracle.brandes_parallel(g.n, g.row_ptr, g.col, roots, threads=threads)
+    assert pd2 is None and np.array_equal(pbc2.view(np.int64), bc.view(np.int64))

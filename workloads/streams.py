@@ -100,6 +100,9 @@ CONFIGS = {
     "karate": dict(graph="karate", k=34, insertions=10, mode="non_edges"),
     "rmat16": dict(graph="rmat", scale=16, ef=8, k=256, insertions=1000, mode="reinsert"),
     "delaunay18": dict(graph="delaunay", npts=1 << 18, k=512, insertions=1000, mode="reinsert"),
+    # config 3's stress variant: uniform random
+    # non-edges -- long-range Case-3 pull-ups on a high-diameter mesh
+    "delaunay18u": dict(graph="delaunay", npts=1 << 18, k=512, insertions=1000, mode="non_edges"),
     "kron20": dict(graph="rmat", scale=20, ef=16, k=1024, insertions=10000, mode="reinsert"),
     "kron22": dict(graph="rmat", scale=22, ef=16, k=4096, insertions=10000, mode="reinsert"),
     "smallworld": dict(graph="ws", n=100_000, kk=10, p=0.1, k=256, insertions=100, mode="reinsert"),
