@@ -42,6 +42,12 @@ struct dbc_ctx {
     int dl_min = 16 * 4096;              // entry-balanced long rows of a down level from this many entries
     int wide_inlane = -1;                // up levels of <= this many items per thread: short rows in-lane
     int sblock = 256, sworkers = 0;  // static kernel: its own CTA width and grid
+    int lean_workers = 0;            // update_lean.cu worker CTAs (one job per insertion)
+    bool lean_on = true;             // per-insertion jobs on update_lean.cu (else update.cu)
+    int64_t lean_max = 1;            // merged batches of <= this many insertions also run there
+    int lean_short = 4;              // level-2 shortcut threshold (rows > lean_short x deg(root))
+    int lean_block = 128;            // threads per update_lean.cu CTA
+    void *lean_board = nullptr;      // its help board (one entry per worker)
     size_t nscratch = 0;             // worker scratch sets allocated
     // heavy lanes: the slowest root chains of the previous batch run on
     // 2x-wide CTAs (hblock threads) on a high-priority stream
@@ -84,6 +90,7 @@ struct dbc_ctx {
     int eworkers = 0;
     long long *scen = nullptr;  // scenario log [insertion][k_loc] of the last insert call
     int64_t scen_cap = 0;       // insertions it holds (0: logging off)
+    int64_t scen_alloc = 0;     // insertions the allocation holds
     int64_t scen_last = 0;      // insertions logged by the last insert call
 
     std::vector<void *> allocs;
@@ -400,8 +407,15 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
         }
     }
 
-    // workers: persistent CTAs; bounded by roots and by a scratch-memory budget
-    const size_t per_worker = (size_t)n * (4 + 8 + 8 + 4 + 4 + 8 + 4 + 4 + 4 + 4 + 4 + 4) + sizeof(ChunkSmem) + (size_t)(n + 2) * 4 + 64;
+    // workers: persistent CTAs; bounded by roots and by a scratch-memory budget.
+    // Per worker: the n-sized arrays of Scratch (mark, lowrec, dacc, Dv, Dold,
+    // Dsig, U0, U1, Rv, Rl, Bq) and of the help board (gU), Doff, the deferred
+    // long rows X, the insertion window (Wul, Wlev) and the chunk mirror.
+    int wcap = kWindow;
+    if (const char *e = getenv("DBC_WINDOW")) wcap = std::max(1, atoi(e));
+    const size_t per_worker = (size_t)n * (4 + 8 + 8 + 4 + 4 + 8 + 4 + 4 + 4 + 4 + 4 + 4) + (size_t)(n + 2) * 4 +
+                              (size_t)kXcap * sizeof(XRow) + (size_t)2 * wcap * sizeof(int32_t) +
+                              sizeof(ChunkSmem) + 64;
     size_t free_b = 0, total_b = 0;
     cudaMemGetInfo(&free_b, &total_b);
     const size_t state_b = (size_t)c->k_loc * n * 24 + (size_t)c->col_cap * 8 + (size_t)n * 40;
@@ -482,6 +496,8 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->ab.deg, (size_t)n + 1);
     AL(c->ab.sums, (size_t)scan_sums_capacity(n + 1));
     AL(c->ab.bad, 1);
+    AL(c->ab.tmp, 2 * e2);
+    c->ab.tmp_half = (int64_t)e2;
     AL(c->bu, (size_t)c->edge_cap);
     AL(c->bv, (size_t)c->edge_cap);
     const size_t kn = (size_t)c->k_loc * n;
@@ -493,7 +509,28 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->bc_ext, (size_t)n);
     AL(c->perm_d, (size_t)n);
     AL(c->roots_d, (size_t)c->k_loc);
-    const size_t nwk = std::max((size_t)c->workers + c->heavy_cap, (size_t)c->sworkers);  // both lanes; static
+    // per-insertion workers (update_lean.cu): one CTA per root when memory allows
+    c->lean_workers = std::max(0, std::min(c->k_loc, fit));
+    if (const char *e = getenv("DBC_LEAN_WORKERS")) c->lean_workers = std::max(1, std::min(c->lean_workers, atoi(e)));
+    if (getenv("DBC_NO_LEAN")) c->lean_on = false;
+    if (const char *e = getenv("DBC_LEAN_MAX")) c->lean_max = atoll(e);
+    if (const char *e = getenv("DBC_LEAN_SHORT")) c->lean_short = std::max(0, atoi(e));
+    // per-insertion CTA width (measured on B200): hub-heavy
+    // graphs need wide CTAs for their heavy levels (R-MAT 16: 512), meshes are
+    // latency-bound on narrow levels (Delaunay 2^18: 256)
+    c->lean_block = c->lowdeg ? 256 : 512;
+    if (const char *e = getenv("DBC_LEAN_BLOCK")) {
+        const int b = atoi(e);
+        c->lean_block = (b == 256 || b == 512 || b == 1024) ? b : 128;
+    }
+    {  // a persistent grid: every worker resident (idle workers wait on the help board)
+        const int per_sm = c->lean_block == 1024 ? lean_resident_1024()
+                           : c->lean_block == 512 ? lean_resident_512()
+                           : c->lean_block == 256 ? lean_resident_256() : lean_resident_128();
+        c->lean_workers = std::min(c->lean_workers, std::max(1, per_sm) * c->nsm);
+    }
+    const size_t nwk = std::max({(size_t)c->workers + c->heavy_cap, (size_t)c->sworkers,
+                                 (size_t)c->lean_workers});  // both lanes; static; per-insertion
     c->nscratch = nwk;
     const size_t wn = nwk * n;
     AL(c->ws.mark, wn);
@@ -510,8 +547,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->ws.Bq, wn);
     AL(c->ws.X, nwk * (size_t)kXcap);
     AL(c->ws.wepoch, nwk);
-    c->ws.wcap = kWindow;
-    if (const char *e = getenv("DBC_WINDOW")) c->ws.wcap = std::max(1, atoi(e));
+    c->ws.wcap = wcap;
     AL(c->ws.Wul, nwk * (size_t)c->ws.wcap);
     AL(c->ws.Wlev, nwk * (size_t)c->ws.wcap);
     AL(c->help.word, nwk);
@@ -525,7 +561,13 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->help.gbig, 2 * nwk);
     c->help.nworkers = (int)nwk;
     if (const char *e = getenv("DBC_NO_HELP")) c->help_on = atoi(e) == 0;
-    AL(c->next_slot, 2);
+    AL(c->next_slot, 4);  // [0] next root, [1] heavy lane's next root / unused, [2..3] lean: roots done, idle
+    if (c->lean_workers) {
+        char *bd = nullptr;
+        AL(bd, lean_board_bytes() * (size_t)c->lean_workers);
+        c->lean_board = getenv("DBC_LEAN_NO_HELP") ? nullptr : (void *)bd;
+        cudaMemsetAsync(bd, 0, lean_board_bytes() * (size_t)c->lean_workers, c->stream);
+    }
     AL(c->slots_d, (size_t)std::max(c->k_loc, 1));
     AL(c->stats, (size_t)kStCount);
     AL(c->err, 1);
@@ -667,6 +709,9 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     if (c->inserted + cnt > c->edge_cap)
         return fail(c, DBC_ECAPACITY, "edge capacity %lld exhausted (%lld inserted, batch %lld)",
                     (long long)c->edge_cap, (long long)c->inserted, (long long)cnt);
+    if (c->scen_cap > 0 && cnt > c->scen_cap)  // before anything changes (state unchanged on error)
+        return fail(c, DBC_EINVAL, "batch of %lld exceeds the scenario log (%lld insertions)",
+                    (long long)cnt, (long long)c->scen_cap);
     CK(cudaSetDevice(c->device));
     const bool tm = c->flags & DBC_FLAG_TIMING;
     int launches = 0;
@@ -674,7 +719,7 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     cudaEvent_t *ev = c->ev + (c->evset ? 0 : 6);
     if (tm) CK(cudaEventRecord(ev[0], c->stream));
     GView g = view_of(c);
-    launches += validate_batch(c->ab, g, c->rp[c->cur], c->n, u, v, cnt, c->stream);
+    launches += validate_batch(c->ab, g, c->rp[c->cur], c->n, u, v, cnt, c->nsm, c->stream);
     CK(cudaGetLastError());
     int32_t bad = 0;
     CK(cudaMemcpyAsync(&bad, c->ab.bad, sizeof(int32_t), cudaMemcpyDeviceToHost, c->stream));
@@ -702,7 +747,7 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     }
     const int nb = 1 - c->cur;
     launches += append_batch(c->ab, c->rp[c->cur], c->col[c->cur], c->scol[c->cur], c->rp[nb],
-                             c->col[nb], c->scol[nb], c->n, c->nnz, c->stream);
+                             c->col[nb], c->scol[nb], c->n, c->nnz, c->nsm, c->stream);
     CK(cudaGetLastError());
     c->cur = nb;
     c->nnz += 2 * cnt;
@@ -752,16 +797,43 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     a.trace_slot = getenv("DBC_TRACE_SLOT") ? atoi(getenv("DBC_TRACE_SLOT")) : -1;
     a.lowdeg = c->lowdeg && !getenv("DBC_NO_LOWDEG");
     if (c->scen_cap > 0) {  // Fig. 2 / Fig. 4 log: one job per (root, insertion)
-        if (cnt > c->scen_cap)
-            return fail(c, DBC_EINVAL, "batch of %lld exceeds the scenario log (%lld insertions)",
-                        (long long)cnt, (long long)c->scen_cap);
         a.scen = c->scen;
         a.merge = 0;
         c->scen_last = cnt;
     }
     if (tm) CK(cudaEventRecord(ev[2], c->stream));
     int ulaunch = 0;
-    if (c->eworkers) {  // edge-based parallel update (Alg. 4 / Alg. 6), one launch per insertion
+    // one job per (root, insertion) -- Mode S, DBC_FLAG_NO_MERGE, the scenario
+    // log, and batches too small to merge -- runs the per-insertion kernel
+    const bool per_ins = (c->flags & (DBC_FLAG_MODE_S | DBC_FLAG_NO_MERGE)) || a.scen;
+    const bool use_lean = c->lean_on && c->lean_workers > 0 && !c->eworkers && (per_ins || cnt <= c->lean_max);
+    a.static_slots = 0;
+    a.lean_board = nullptr;
+    a.short_mult = c->lean_short;
+    if (use_lean) {
+        const int nw = c->lean_workers;
+        a.lean_board = c->lean_board;
+        a.merge = 0;
+        a.root_prof = c->prof_on ? c->root_prof : nullptr;
+        if (c->prof_on)
+            CK(cudaMemsetAsync(c->root_prof, 0, sizeof(unsigned long long) * 6 * std::max(c->k_loc, 1), c->stream));
+        const int64_t step = (c->flags & DBC_FLAG_MODE_S) ? 1 : cnt;  // Mode S: one launch per insertion
+        for (int64_t i = 0; i < cnt; i += step) {
+            CK(cudaMemsetAsync(c->next_slot, 0, 4 * sizeof(int32_t), c->stream));
+            a.ins_begin = (int32_t)i;
+            a.ins_end = (int32_t)std::min<int64_t>(cnt, i + step);
+            if (c->lean_block == 1024)
+                launch_update_lean_1024(a, nw, c->stream);
+            else if (c->lean_block == 512)
+                launch_update_lean_512(a, nw, c->stream);
+            else if (c->lean_block == 256)
+                launch_update_lean_256(a, nw, c->stream);
+            else
+                launch_update_lean_128(a, nw, c->stream);
+            ++ulaunch;
+        }
+        CK(cudaGetLastError());
+    } else if (c->eworkers) {  // edge-based parallel update (Alg. 4 / Alg. 6), one launch per insertion
         launches += launch_edge_coo(a.g, c->n, c->esrc, c->etag, c->stream);
         EdgeArgs e;
         e.g = a.g;
@@ -955,6 +1027,9 @@ static dbc_status delete_host_ids(dbc_ctx *c, const int32_t *u, const int32_t *v
     if (c->flags & DBC_FLAG_EDGE_PARALLEL)
         return fail(c, DBC_EINVAL, "deletions are not supported with DBC_FLAG_EDGE_PARALLEL");
     if (cnt > c->edge_cap) return fail(c, DBC_EINVAL, "deletion batch larger than the staging buffer");
+    if (c->scen_cap > 0 && cnt > c->scen_cap)
+        return fail(c, DBC_EINVAL, "batch of %lld exceeds the scenario log (%lld insertions)",
+                    (long long)cnt, (long long)c->scen_cap);
     {
         std::vector<int64_t> keys((size_t)cnt);
         for (int64_t i = 0; i < cnt; ++i) {
@@ -1021,6 +1096,8 @@ static dbc_status delete_host_ids(dbc_ctx *c, const int32_t *u, const int32_t *v
     a.help = HelpBoard{};
     a.merge = 0;
     a.del = 1;
+    a.static_slots = 0;
+    a.lean_board = nullptr;
     a.hd_min = c->hd_min;
     a.hd_block = c->hd_block;
     a.he_entries = c->he_entries;
@@ -1033,9 +1110,6 @@ static dbc_status delete_host_ids(dbc_ctx *c, const int32_t *u, const int32_t *v
     a.lowdeg = c->lowdeg && !getenv("DBC_NO_LOWDEG");
     a.scen = nullptr;
     if (c->scen_cap > 0) {
-        if (cnt > c->scen_cap)
-            return fail(c, DBC_EINVAL, "batch of %lld exceeds the scenario log (%lld insertions)",
-                        (long long)cnt, (long long)c->scen_cap);
         a.scen = c->scen;
         c->scen_last = cnt;
     }
@@ -1099,9 +1173,10 @@ extern "C" dbc_status dbc_delete_edges_device(dbc_ctx *c, const int32_t *u, cons
     if (count < 0 || (count > 0 && (!u || !v))) return fail(c, DBC_EINVAL, "bad batch");
     CK(cudaSetDevice(c->device));
     std::vector<int32_t> hu((size_t)count), hv((size_t)count);  // the host-side batch checks
-    if (count) {
-        CK(cudaMemcpy(hu.data(), u, sizeof(int32_t) * count, cudaMemcpyDeviceToHost));
-        CK(cudaMemcpy(hv.data(), v, sizeof(int32_t) * count, cudaMemcpyDeviceToHost));
+    if (count) {  // ordered after work the caller queued on the context stream
+        CK(cudaMemcpyAsync(hu.data(), u, sizeof(int32_t) * count, cudaMemcpyDeviceToHost, c->stream));
+        CK(cudaMemcpyAsync(hv.data(), v, sizeof(int32_t) * count, cudaMemcpyDeviceToHost, c->stream));
+        CK(cudaStreamSynchronize(c->stream));
     }
     return delete_host_ids(c, hu.data(), hv.data(), count, stats);
 }
@@ -1217,16 +1292,19 @@ extern "C" dbc_status dbc_debug_root_profile(dbc_ctx *c, int32_t enable, int64_t
 extern "C" dbc_status dbc_scenario_log(dbc_ctx *c, int64_t max_insertions) {
     if (!c || max_insertions < 0) return DBC_EINVAL;
     CK(cudaSetDevice(c->device));
-    if (max_insertions > c->scen_cap) {
+    if (max_insertions > c->scen_alloc) {
         CK(cudaStreamSynchronize(c->stream));
         if (c->scen) {
             for (auto &q : c->allocs)
                 if (q == (void *)c->scen) q = nullptr;
             CK(cudaFree(c->scen));
-            c->bytes -= (int64_t)(sizeof(long long) * (size_t)c->scen_cap * std::max(c->k_loc, 1));
+            c->bytes -= (int64_t)(sizeof(long long) * (size_t)std::max<int64_t>(c->scen_alloc, 1) *
+                                  std::max(c->k_loc, 1));
             c->scen = nullptr;
+            c->scen_alloc = 0;
         }
         TRY(dalloc(c, &c->scen, (size_t)max_insertions * std::max(c->k_loc, 1)));
+        c->scen_alloc = max_insertions;
     }
     c->scen_cap = max_insertions;
     c->scen_last = 0;

@@ -584,6 +584,10 @@ struct UpdateArgs {
     int32_t dl_min;                // down levels whose long rows hold >= dl_min entries: entry-balanced pass
     int32_t wide_inlane;           // up levels of <= wide_inlane items per thread: short rows in-lane, long rows chunked
     int32_t trace_slot;            // -DDBC_PHASE_TIMERS builds: time this slot only (-1: all)
+    int32_t static_slots;          // unused (kept zero)
+    void *lean_board;              // update_lean.cu help board (nullptr: no cooperative help)
+    int32_t short_mult;            // update_lean.cu: level-2 up rows longer than short_mult x deg(root)
+                                   // find their predecessors by probing adj(root)
 };
 
 struct StaticArgs {
@@ -625,6 +629,16 @@ int launch_edge_coo(const GView &g, int32_t n, int32_t *src, int32_t *tag, cudaS
 void launch_edge_update(const EdgeArgs &a, int workers, cudaStream_t s);
 
 void launch_update_256(const UpdateArgs &a, int workers, cudaStream_t s);
+// update_lean.cu, one job per insertion: 128-, 256-, 512- and 1024-thread builds
+void launch_update_lean_128(const UpdateArgs &a, int workers, cudaStream_t s);
+void launch_update_lean_256(const UpdateArgs &a, int workers, cudaStream_t s);
+void launch_update_lean_512(const UpdateArgs &a, int workers, cudaStream_t s);
+void launch_update_lean_1024(const UpdateArgs &a, int workers, cudaStream_t s);
+int lean_resident_128();  // resident CTAs per SM of each build
+int lean_resident_256();
+int lean_resident_512();
+int lean_resident_1024();
+size_t lean_board_bytes();
 void launch_update_512x2(const UpdateArgs &a, int workers, cudaStream_t s);  // 64 regs, 2 CTAs/SM
 void launch_update_1024(const UpdateArgs &a, int workers, cudaStream_t s);   // heavy lane, 64 regs
 void launch_update_128(const UpdateArgs &a, int workers, cudaStream_t s);

@@ -185,9 +185,9 @@ __global__ void k_group_scatter(const int32_t *u, const int32_t *v, int64_t cnt,
 // Groups of up to 32 entries (all but the rarest hubs) are ranked in registers,
 // one entry per lane (ties broken by lane: a self loop's two entries -- the
 // batch is rejected anyway -- still land in distinct slots); larger groups are
-// insertion-sorted by lane 0.
+// ranked warp-cooperatively through scratch (B.tmp).
 __global__ void k_group_sort(const int32_t *xcnt, const int32_t *xoff, int32_t n, int32_t *gtag,
-                             int32_t *gnbr, int2 *xinfo, int32_t *bad) {
+                             int32_t *gnbr, int2 *xinfo, int32_t *bad, int32_t *sort_tmp, int64_t tmp_half) {
     const int lane = threadIdx.x & 31;
     const int64_t warps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     for (int64_t x = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; x < n; x += warps) {
@@ -209,21 +209,30 @@ __global__ void k_group_sort(const int32_t *xcnt, const int32_t *xoff, int32_t n
                 gnbr[b + rank] = nb;
                 if (dup) atomicOr(bad, 4);
             }
-        } else if (lane == 0) {
-            for (int i = 1; i < c; ++i) {  // insertion sort
-                const int t = gtag[b + i], nb = gnbr[b + i];
-                int j = i - 1;
-                while (j >= 0 && gtag[b + j] > t) {
-                    gtag[b + j + 1] = gtag[b + j];
-                    gnbr[b + j + 1] = gnbr[b + j];
-                    --j;
+        } else {
+            // larger groups (hubs): each lane ranks entries k = lane, lane + 32, ...
+            // against the whole group (O(c^2 / 32), duplicates found in the same
+            // pass), into the group's slice of xcnt-sized scratch, then copies back
+            int32_t *rt = gtag + b, *rn = gnbr + b;
+            int32_t *ot = sort_tmp + b, *on = sort_tmp + tmp_half + b;
+            for (int k = lane; k < c; k += 32) {
+                const int t = rt[k], nb = rn[k];
+                int rank = 0;
+                bool dup = false;
+                for (int j = 0; j < c; ++j) {
+                    const int tj = rt[j];
+                    rank += (tj < t) || (tj == t && j < k);
+                    dup |= (j != k) && (rn[j] == nb);
                 }
-                gtag[b + j + 1] = t;
-                gnbr[b + j + 1] = nb;
+                ot[rank] = t;
+                on[rank] = nb;
+                if (dup) atomicOr(bad, 4);
             }
-            for (int i = 1; i < c; ++i)
-                for (int j = 0; j < i; ++j)
-                    if (gnbr[b + j] == gnbr[b + i]) atomicOr(bad, 4);
+            __syncwarp();
+            for (int k = lane; k < c; k += 32) {
+                rt[k] = ot[k];
+                rn[k] = on[k];
+            }
         }
         if (lane == 0) xinfo[x] = make_int2(b, c);
     }
@@ -305,7 +314,7 @@ static int scan_launch(const int32_t *in, int32_t *out, int64_t cnt, int32_t *su
 }
 
 int validate_batch(const AppendBufs &B, const GView &g, const int32_t *rp_old, int32_t n,
-                   const int32_t *u, const int32_t *v, int64_t cnt, cudaStream_t s) {
+                   const int32_t *u, const int32_t *v, int64_t cnt, int nsm, cudaStream_t s) {
     int launches = 0;
     cudaMemsetAsync(B.bad, 0, sizeof(int32_t), s);
     cudaMemsetAsync(B.xcnt, 0, sizeof(int32_t) * (size_t)n, s);
@@ -319,8 +328,8 @@ int validate_batch(const AppendBufs &B, const GView &g, const int32_t *rp_old, i
     if (cnt) {
         k_group_scatter<<<blocks_for(cnt, 256), 256, 0, s>>>(u, v, cnt, n, B.xoff, B.slot, B.xtag,
                                                             B.gnbr);
-        k_group_sort<<<std::min<int64_t>(blocks_for((int64_t)n * 32, 256), 148 * 16), 256, 0, s>>>(
-            B.xcnt, B.xoff, n, B.xtag, B.gnbr, B.xinfo, B.bad);
+        k_group_sort<<<std::min<int64_t>(blocks_for((int64_t)n * 32, 256), (int64_t)nsm * 16), 256, 0, s>>>(
+            B.xcnt, B.xoff, n, B.xtag, B.gnbr, B.xinfo, B.bad, B.tmp, B.tmp_half);
         launches += 2;
     }
     (void)rp_old;
@@ -329,14 +338,14 @@ int validate_batch(const AppendBufs &B, const GView &g, const int32_t *rp_old, i
 
 int append_batch(const AppendBufs &B, const int32_t *rp_old, const int32_t *col_old,
                  const int32_t *scol_old, int32_t *rp_new, int32_t *col_new, int32_t *scol_new,
-                 int32_t n, int64_t nnz_old, cudaStream_t s) {
+                 int32_t n, int64_t nnz_old, int nsm, cudaStream_t s) {
     int launches = 0;
     k_degrees<<<blocks_for((int64_t)n + 1, 256), 256, 0, s>>>(rp_old, B.xcnt, n, B.deg);
     launches += 1 + scan_launch(B.deg, rp_new, (int64_t)n + 1, B.sums, s);
     if (nnz_old > 0)
-        k_copy_entries<<<std::min<int64_t>(blocks_for(nnz_old, 256), 148 * 64), 256, 0, s>>>(
+        k_copy_entries<<<std::min<int64_t>(blocks_for(nnz_old, 256), (int64_t)nsm * 64), 256, 0, s>>>(
             rp_old, col_old, scol_old, rp_new, col_new, scol_new, B.xcnt, B.xoff, B.gnbr, n, nnz_old);
-    k_place_groups<<<std::min<int64_t>(blocks_for((int64_t)n * 32, 256), 148 * 16), 256, 0, s>>>(
+    k_place_groups<<<std::min<int64_t>(blocks_for((int64_t)n * 32, 256), (int64_t)nsm * 16), 256, 0, s>>>(
         rp_old, scol_old, rp_new, col_new, scol_new, B.xcnt, B.xoff, B.gnbr, n);
     k_flag_rows<<<blocks_for(n, 256), 256, 0, s>>>(B.xcnt, n, rp_new);
     return launches + 2 + (nnz_old > 0);

@@ -21,18 +21,20 @@ struct AppendBufs {
     int32_t *deg;    // [n+1]
     int32_t *sums;   // scan block sums
     int32_t *bad;    // [1] validation result bits
+    int32_t *tmp;    // [2 * tmp_half] group-sort scratch (groups of > 32 entries)
+    int64_t tmp_half;  // 2 * edge capacity
 };
 
 int64_t scan_sums_capacity(int64_t n);
 int validate_batch(const AppendBufs &B, const GView &g, const int32_t *rp_old, int32_t n,
-                   const int32_t *u, const int32_t *v, int64_t cnt, cudaStream_t s);
+                   const int32_t *u, const int32_t *v, int64_t cnt, int nsm, cudaStream_t s);
 int validate_deletions(const GView &g, int32_t n, const int32_t *u, const int32_t *v, int64_t cnt,
                        int32_t *bad, cudaStream_t s);
 int tombstone_edge(const int32_t *rp, int32_t *col, int32_t *scol, const int32_t *u, const int32_t *v,
                    int64_t i, cudaStream_t s);
 int append_batch(const AppendBufs &B, const int32_t *rp_old, const int32_t *col_old,
                  const int32_t *scol_old, int32_t *rp_new, int32_t *col_new, int32_t *scol_new,
-                 int32_t n, int64_t nnz_old, cudaStream_t s);
+                 int32_t n, int64_t nnz_old, int nsm, cudaStream_t s);
 int map_ids(const int32_t *su, const int32_t *sv, int32_t *du, int32_t *dv, int64_t cnt,
             const int32_t *perm, int32_t n, cudaStream_t s);
 int gather_ext(const double *in, const int32_t *perm, int32_t n, double *out, cudaStream_t s);

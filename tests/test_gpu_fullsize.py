@@ -52,7 +52,7 @@ class Ref:
         return oracle.brandes_parallel(self.n, rp, col, self.roots, state_slots=sample_local)
 
 
-def check(dbc, ref: Ref, sample_local, what=""):
+def check(dbc, ref: Ref, sample_local, what="", delta_tol=DELTA_TOL):
     """BC over all of the context's roots + d/sigma/delta on sample_local (local indices)."""
     bc_ref, d_ref, s_ref, dl_ref = ref.compute(sample_local)
     bc = dbc.get_bc()
@@ -67,7 +67,7 @@ def check(dbc, ref: Ref, sample_local, what=""):
         assert bad.size == 0, f"{what}: sigma mismatch slot {slot} at {bad[:4]}"
         e = float((np.abs(dl - dl_ref[i]) / np.maximum(np.abs(dl_ref[i]), 1.0)).max(initial=0.0))
         worst = max(worst, e)
-        assert e <= DELTA_TOL, f"{what}: delta rel err {e} slot {slot}"
+        assert e <= delta_tol, f"{what}: delta rel err {e} slot {slot}"
     return err, worst
 
 
@@ -83,7 +83,7 @@ def _sample(k_loc, m=SAMPLE):
     return np.unique(np.linspace(0, k_loc - 1, min(m, k_loc)).astype(np.int64))
 
 
-def run_cadence(name, batch, flags=0, sample=SAMPLE, state_every=1, insertions=None):
+def run_cadence(name, batch, flags=0, sample=SAMPLE, state_every=1, insertions=None, delta_tol=DELTA_TOL):
     """Insert the config's stream in batches of `batch`; after every batch BC over
     all roots, and every `state_every` batches d/sigma/delta on the sample."""
     from paper_conf_ipps_mclaughlinb14_b200 import DynamicBC
@@ -102,7 +102,8 @@ def run_cadence(name, batch, flags=0, sample=SAMPLE, state_every=1, insertions=N
             dbc.insert_edges(wl.ins_u[sl], wl.ins_v[sl])
             ref.insert(wl.ins_u[sl], wl.ins_v[sl])
             full = (b + 1) % state_every == 0 or b == nb - 1
-            e = check(dbc, ref, smp if full else np.zeros(0, np.int64), f"{name} after {sl.stop}")
+            e = check(dbc, ref, smp if full else np.zeros(0, np.int64), f"{name} after {sl.stop}",
+                      delta_tol)
             worst = [max(worst[0], e[0]), max(worst[1], e[1])]
         dynamic_equals_static(dbc, ref, smp[:8])
     print(f"{name} batch {batch} flags {flags:#x}: max BC rel err {worst[0]:.2e}, "
@@ -139,8 +140,16 @@ def test_delaunay18_bench_batch_all_roots():
 @pytest.mark.timeout(1500)
 def test_delaunay18_uniform_nonedge_stress_all_roots():
     """Config 3's stress variant (uniform random non-edges: long-range Case-3
-    pull-ups), every 100th insertion, BC over all 512 roots."""
-    run_cadence("delaunay18u", 100)
+    pull-ups), every 100th insertion, BC over all 512 roots.
+
+    delta tolerance: vertices outside D keep delta by the push-delta form
+    (delta += Ddelta), whose rounding accumulates over
+    the insertions that touch a vertex.  One such update contributes at most
+    ~depth * u relative (a chain of <= 220 levels on this mesh, u = 2^-53:
+    2.4e-14); 100 insertions that each pull up large parts of the mesh touch a
+    vertex up to 100 times: 2.4e-12 (measured 1.8e-12).  So 1e-11 here
+    (DESIGN.md Sec. 3); BC keeps the north star's 1e-9."""
+    run_cadence("delaunay18u", 100, delta_tol=1e-11)
 
 
 # ------------------------------------------------------------ configs 4, 5 ----

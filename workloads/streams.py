@@ -111,6 +111,7 @@ CONFIGS = {
     "rmat14": dict(graph="rmat", scale=14, ef=16, k=64, insertions=400, mode="reinsert"),
     "delaunay12": dict(graph="delaunay", npts=1 << 12, k=48, insertions=40, mode="reinsert"),
     "delaunay12u": dict(graph="delaunay", npts=1 << 12, k=48, insertions=40, mode="non_edges"),
+    "smallworld_small": dict(graph="ws", n=2000, kk=6, p=0.1, k=54, insertions=40, mode="reinsert"),
 }
 
 
