@@ -35,9 +35,12 @@
  *  - A context is not thread-safe.  Several contexts may coexist (e.g. one per
  *    GPU and rank).
  *  - Multi-GPU: every rank passes the FULL root list; rank r owns root slots
- *    with slot % world == r.  BC partials are summed
- *    across ranks by the caller (dbc_get_bc_partial_device + an NCCL
- *    all-reduce) -- the only cross-GPU exchange of the method.
+ *    with slot % world == r.  The per-rank BC partials
+ *    are summed across ranks -- the only cross-GPU exchange of the method
+ *     -- by dbc_get_bc itself, through the context's own NCCL
+ *    communicator (opt->nccl_id) or the caller's reduction callback
+ *    (opt->reduce); dbc_get_bc_partial_device exposes the partial for callers
+ *    that reduce it themselves.
  */
 #ifndef DBC_H
 #define DBC_H
@@ -50,7 +53,7 @@ extern "C" {
 #endif
 
 #define DBC_INF INT32_MAX
-#define DBC_ABI_VERSION 1
+#define DBC_ABI_VERSION 2
 
 typedef struct dbc_ctx dbc_ctx; /* opaque; owns all device memory it allocates */
 
@@ -59,7 +62,7 @@ typedef enum {
     DBC_EINVAL = -1,     /* bad argument (NULL, n < 1, bad CSR, bad slot, ...) */
     DBC_ENOMEM = -2,     /* device or host allocation failed */
     DBC_ECUDA = -3,      /* CUDA runtime error (message in dbc_last_error) */
-    DBC_ENCCL = -4,      /* reserved: collective failure */
+    DBC_ENCCL = -4,      /* NCCL missing or a collective failed (message in dbc_last_error) */
     DBC_ESTATE = -5,     /* call out of order, e.g. insert before static_compute */
     DBC_EEDGE = -6,      /* self loop, out-of-range vertex, edge already present,
                             or duplicate edge within a batch; batch not applied */
@@ -90,12 +93,66 @@ typedef enum {
                                   within rounding (the sum of the per-insertion
                                   changes telescopes)                            */
 
+#define DBC_FLAG_PULL_DELTA 0x40u /* debug mode: every vertex the update touches
+                                  (Alg. 2's t[v] != untouched) recomputes
+                                  delta by the pull of Eq. (2) in canonical order
+                                  instead of the push-delta form (SURVEY.md Sec.
+                                  8(c) item 14), and the static pass sums long
+                                  rows in canonical order too: delta is then
+                                  bit-identical to the oracle, and with
+                                  DBC_FLAG_EXACT_BC at world 1 so is BC.  Every
+                                  batch runs one job per insertion.  Not with
+                                  deletions or DBC_FLAG_EDGE_PARALLEL (EINVAL) */
+
 #define DBC_FLAG_EDGE_PARALLEL 0x20u /* edge-based parallel update (Alg. 4 / Alg. 6,
                                   P:278-356): one launch per insertion, every
                                   level a pass of one CTA per root over all
                                   edges -- the comparison kernel of Table II
                                   (P:458-478).  Same results as the default
                                   node-based kernel; slower by design        */
+
+/* Sum all-reduce of the BC partial across ranks, in place: bc_device is
+ * fp64[n] device memory of the context's device, stream its CUDA stream (the
+ * reduction must be complete, or ordered on that stream, when the callback
+ * returns).  Return 0 on success; anything else makes dbc_get_bc fail with
+ * DBC_ENCCL. */
+typedef int (*dbc_reduce_fn)(double *bc_device, int64_t n, void *stream, void *user);
+/* Device memory hooks (e.g. torch's caching allocator): return NULL on failure. */
+typedef void *(*dbc_alloc_fn)(size_t bytes, void *user);
+typedef void (*dbc_free_fn)(void *ptr, void *user);
+
+/* Tuning of the kernels' launch configuration.  Results
+ * never depend on it.  dbc_tuning_default sets every field to "automatic"
+ * (integers < 0, heavy_factor 0, disable 0); the automatic choices are the
+ * ones measured best on B200. */
+typedef struct {
+    int32_t update_block;    /* batch kernel CTA width: 128, 256, 512 or 1024            */
+    int32_t update_pair;     /* 512-thread batch CTAs built for two per SM: 0 / 1        */
+    int32_t static_block;    /* static Brandes CTA width: 128, 256, 512 or 1024          */
+    int32_t window;          /* insertions merged into one job per root (R18)  */
+    int32_t heavy_cap;       /* roots run on the wide heavy lane per batch (0: none)     */
+    float heavy_factor;      /* a root is heavy if its last chain took > this x median   */
+    int32_t help_down_min;   /* batch kernel: down levels of >= this many items are helped */
+    int32_t help_down_block; /* ... in blocks of this many items                         */
+    int32_t help_entries;    /* flattened passes: entries per help block                 */
+    int32_t help_min_blocks; /* ... published from this many blocks                      */
+    int32_t busy_help;       /* blocks a busy worker takes at a level boundary (0: none) */
+    int32_t busy_min;        /* ... of passes of at least this many blocks               */
+    int32_t down_long_min;   /* entry-balanced long rows of a down level from this many entries */
+    int32_t wide_inlane;     /* up levels of <= this many items per thread: short rows in-lane */
+    int32_t lean_block;      /* per-insertion kernel CTA width: 128, 256, 512 or 1024    */
+    int32_t lean_workers;    /* its worker CTAs (capped at the resident maximum)         */
+    int32_t lean_max_batch;  /* merged batches of <= this many insertions run per insertion */
+    int32_t lean_short;      /* level-2 rows longer than this x deg(root) probe adj(root) */
+    int32_t trace_slot;      /* -DDBC_PHASE_TIMERS builds: trace this root slot          */
+    uint32_t disable;        /* DBC_TUNE_* bits                                          */
+    uint32_t reserved[8];    /* must be zero                                             */
+} dbc_tuning;
+#define DBC_TUNE_NO_HELP      0x1u  /* batch kernel: no cooperative help          */
+#define DBC_TUNE_NO_HEAVY     0x2u  /* batch kernel: no heavy lane                */
+#define DBC_TUNE_NO_LEAN      0x4u  /* per-insertion jobs on the batch kernel     */
+#define DBC_TUNE_NO_LEAN_HELP 0x8u  /* per-insertion kernel: no cooperative help  */
+#define DBC_TUNE_NO_LOWDEG    0x10u /* batch kernel: no in-lane up levels on low-degree graphs */
 
 typedef struct {
     int32_t device;        /* CUDA device ordinal (default 0)                      */
@@ -107,7 +164,19 @@ typedef struct {
     void *stream;          /* cudaStream_t to run on; NULL = library-owned stream;
                               cudaStreamLegacy ((void*)1) = the legacy default stream */
     uint32_t flags;        /* DBC_FLAG_*                                           */
-    uint32_t reserved[7];  /* must be zero                                         */
+    uint32_t pad0;         /* must be zero                                         */
+    const dbc_tuning *tuning;  /* nullable: automatic; copied by dbc_create        */
+    const void *nccl_id;   /* nullable: 128-byte ncclUniqueId (dbc_nccl_unique_id on
+                              rank 0, shared with every rank).  dbc_create then
+                              joins an NCCL communicator of `world` ranks (a
+                              collective call: every rank must create) that
+                              dbc_get_bc uses for the BC all-reduce over NVLink  */
+    dbc_reduce_fn reduce;  /* nullable: the BC all-reduce as a callback instead   */
+    void *reduce_user;
+    dbc_alloc_fn dev_alloc;  /* nullable: device allocations through the caller    */
+    dbc_free_fn dev_free;    /* (both or neither)                                  */
+    void *alloc_user;
+    uint32_t reserved[4];  /* must be zero                                         */
 } dbc_options;
 
 /* Per-call counters.  Filled when a non-NULL pointer is passed (synchronises). */
@@ -140,6 +209,15 @@ typedef struct {
 
 /* Fills *opt with defaults (device 0, rank 0, world 1, automatic sizes). */
 void dbc_options_default(dbc_options *opt);
+
+/* Fills *t with "automatic" for every field. */
+void dbc_tuning_default(dbc_tuning *t);
+
+/* Writes a fresh 128-byte ncclUniqueId to out (rank 0 of a multi-GPU job; the
+ * caller distributes it to every rank's dbc_options.nccl_id).  NCCL is loaded
+ * at run time (libnccl.so.2; the copy PyTorch loaded, if any).
+ * Errors: DBC_EINVAL (out NULL), DBC_ENCCL (no NCCL, or NCCL failed). */
+dbc_status dbc_nccl_unique_id(void *out);
 
 /* Creates a context from an undirected graph in CSR form and a root set.
  *  n        number of vertices, >= 1
@@ -201,9 +279,13 @@ dbc_status dbc_delete_edges_device(dbc_ctx *c, const int32_t *u_device,
                                    const int32_t *v_device, int64_t count,
                                    dbc_insert_stats *stats);
 
-/* Copies this rank's BC partial (sum over LOCAL roots, Eq. (3)) to host
- * bc[n].  With world == 1 this is the global BC.  Synchronises.  Returns
- * DBC_ENUMERIC if an earlier update overflowed. */
+/* Copies the GLOBAL BC (Eq. (3) over every root of every rank) to host
+ * bc[n].  world == 1: this rank's sum.  world > 1: the per-rank partials are
+ * summed by an all-reduce -- the context's NCCL communicator (opt.nccl_id) or
+ * the opt.reduce callback; a collective call, every rank must make it.
+ * Synchronises.  Errors: DBC_ESTATE (world > 1 without nccl_id or reduce; use
+ * dbc_get_bc_partial_device), DBC_ENCCL (the reduction failed), DBC_ENUMERIC
+ * (an earlier update overflowed). */
 dbc_status dbc_get_bc(dbc_ctx *c, double *bc);
 
 /* Device pointer to this rank's BC partial, fp64[n] in the caller's vertex

@@ -11,11 +11,49 @@
 #include <thread>
 #include <vector>
 
+#include <dlfcn.h>
+#include <nccl.h>  // types only: NCCL is loaded at run time (dlopen), never linked
+
 #include "dbc.h"
 #include "dbc_internal.cuh"
 #include "graph_ops.h"
 
 using namespace dbc;
+
+// NCCL entry points, resolved from libnccl.so.2 at first use -- the copy
+// PyTorch already loaded into the process when there is one (same NCCL as its
+// process groups), else the system's.
+struct NcclApi {
+    bool ok = false;
+    std::string why;
+    ncclResult_t (*get_unique_id)(ncclUniqueId *) = nullptr;
+    ncclResult_t (*comm_init_rank)(ncclComm_t *, int, ncclUniqueId, int) = nullptr;
+    ncclResult_t (*all_reduce)(const void *, void *, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
+                               cudaStream_t) = nullptr;
+    ncclResult_t (*comm_destroy)(ncclComm_t) = nullptr;
+    const char *(*error_string)(ncclResult_t) = nullptr;
+};
+static NcclApi &nccl_api() {
+    static NcclApi api = [] {
+        NcclApi a;
+        void *h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
+        if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+        if (!h) {
+            const char *e = dlerror();
+            a.why = e ? e : "libnccl.so.2 not found";
+            return a;
+        }
+        a.get_unique_id = (decltype(a.get_unique_id))dlsym(h, "ncclGetUniqueId");
+        a.comm_init_rank = (decltype(a.comm_init_rank))dlsym(h, "ncclCommInitRank");
+        a.all_reduce = (decltype(a.all_reduce))dlsym(h, "ncclAllReduce");
+        a.comm_destroy = (decltype(a.comm_destroy))dlsym(h, "ncclCommDestroy");
+        a.error_string = (decltype(a.error_string))dlsym(h, "ncclGetErrorString");
+        a.ok = a.get_unique_id && a.comm_init_rank && a.all_reduce && a.comm_destroy && a.error_string;
+        if (!a.ok) a.why = "libnccl.so.2 lacks an entry point";
+        return a;
+    }();
+    return api;
+}
 
 struct dbc_ctx {
     int device = 0, rank = 0, world = 1;
@@ -95,6 +133,13 @@ struct dbc_ctx {
 
     std::vector<void *> allocs;
     int64_t bytes = 0;
+    dbc_alloc_fn dev_alloc = nullptr;  // caller's device allocator (nullable)
+    dbc_free_fn dev_free = nullptr;
+    void *alloc_user = nullptr;
+    dbc_tuning tune{};                 // launch configuration (dbc_tuning_default: automatic)
+    ncclComm_t comm = nullptr;         // BC all-reduce across ranks (opt.nccl_id)
+    dbc_reduce_fn reduce = nullptr;    // ... or the caller's callback (opt.reduce)
+    void *reduce_user = nullptr;
 
     cudaEvent_t ev[10] = {};  // [0..3]/[6..9]: insert-call sets A/B, [4..5]: static
     int evset = 0;            // set of the most recent insert call (0 -> ev[0..3], 1 -> ev[6..9])
@@ -133,15 +178,28 @@ template <class T>
 static dbc_status dalloc(dbc_ctx *c, T **p, size_t count) {
     size_t b = std::max<size_t>(count, 1) * sizeof(T);
     void *q = nullptr;
-    cudaError_t e = cudaMalloc(&q, b);
-    if (e != cudaSuccess) {
-        cudaGetLastError();
-        return fail(c, DBC_ENOMEM, "cudaMalloc(%zu bytes) failed: %s", b, cudaGetErrorString(e));
+    if (c->dev_alloc) {  // the caller's allocator (e.g. torch's caching allocator)
+        q = c->dev_alloc(b, c->alloc_user);
+        if (!q) return fail(c, DBC_ENOMEM, "dev_alloc(%zu bytes) failed", b);
+    } else {
+        cudaError_t e = cudaMalloc(&q, b);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return fail(c, DBC_ENOMEM, "cudaMalloc(%zu bytes) failed: %s", b, cudaGetErrorString(e));
+        }
     }
     c->allocs.push_back(q);
     c->bytes += (int64_t)b;
     *p = (T *)q;
     return DBC_OK;
+}
+
+static void dfree(dbc_ctx *c, void *p) {
+    if (!p) return;
+    if (c->dev_free)
+        c->dev_free(p, c->alloc_user);
+    else
+        cudaFree(p);
 }
 
 #define TRY(x)                          \
@@ -156,6 +214,34 @@ void dbc_options_default(dbc_options *opt) {
     if (!opt) return;
     std::memset(opt, 0, sizeof(*opt));
     opt->world = 1;
+}
+
+void dbc_tuning_default(dbc_tuning *t) {
+    if (!t) return;
+    std::memset(t, 0, sizeof(*t));
+    t->update_block = t->update_pair = t->static_block = t->window = t->heavy_cap = -1;
+    t->help_down_min = t->help_down_block = t->help_entries = t->help_min_blocks = -1;
+    t->busy_help = t->busy_min = t->down_long_min = t->wide_inlane = -1;
+    t->lean_block = t->lean_workers = t->lean_max_batch = t->lean_short = t->trace_slot = -1;
+    t->heavy_factor = 0.0f;
+}
+
+dbc_status dbc_nccl_unique_id(void *out) {
+    if (!out) return DBC_EINVAL;
+    NcclApi &nc = nccl_api();
+    if (!nc.ok) {
+        g_create_msg = "NCCL unavailable: " + nc.why;
+        return DBC_ENCCL;
+    }
+    ncclUniqueId id;
+    const ncclResult_t r = nc.get_unique_id(&id);
+    if (r != ncclSuccess) {
+        g_create_msg = std::string("ncclGetUniqueId: ") + nc.error_string(r);
+        return DBC_ENCCL;
+    }
+    static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId is 128 bytes");
+    std::memcpy(out, &id, sizeof id);
+    return DBC_OK;
 }
 
 int32_t dbc_abi_version(void) { return DBC_ABI_VERSION; }
@@ -181,7 +267,8 @@ void dbc_destroy(dbc_ctx *c) {
     if (!c) return;
     cudaSetDevice(c->device);
     if (c->stream) cudaStreamSynchronize(c->stream);
-    for (void *p : c->allocs) cudaFree(p);
+    if (c->comm) nccl_api().comm_destroy(c->comm);
+    for (void *p : c->allocs) dfree(c, p);
     if (c->ev_ok)
         for (auto &e : c->ev) cudaEventDestroy(e);
     if (c->ev_fork) cudaEventDestroy(c->ev_fork);
@@ -328,8 +415,16 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     if (opt.world < 1 || opt.rank < 0 || opt.rank >= opt.world)
         return fail(nullptr, DBC_EINVAL, "bad rank/world %d/%d", opt.rank, opt.world);
     if (opt.edge_capacity < 0 || opt.workers < 0) return fail(nullptr, DBC_EINVAL, "bad sizes");
-    for (int i = 0; i < 7; ++i)
+    for (int i = 0; i < 4; ++i)
         if (opt.reserved[i]) return fail(nullptr, DBC_EINVAL, "reserved fields must be zero");
+    if (opt.pad0) return fail(nullptr, DBC_EINVAL, "reserved fields must be zero");
+    if ((opt.dev_alloc == nullptr) != (opt.dev_free == nullptr))
+        return fail(nullptr, DBC_EINVAL, "dev_alloc and dev_free come together");
+    if (opt.tuning)
+        for (int i = 0; i < 8; ++i)
+            if (opt.tuning->reserved[i]) return fail(nullptr, DBC_EINVAL, "tuning reserved fields must be zero");
+    if ((opt.flags & DBC_FLAG_PULL_DELTA) && (opt.flags & DBC_FLAG_EDGE_PARALLEL))
+        return fail(nullptr, DBC_EINVAL, "DBC_FLAG_PULL_DELTA excludes DBC_FLAG_EDGE_PARALLEL");
     {
         std::string why;
         if (!validate_csr(n, row_ptr, col, why)) return fail(nullptr, DBC_EINVAL, "bad CSR: %s", why.c_str());
@@ -344,6 +439,16 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     }
 
     c = new dbc_ctx();
+    c->dev_alloc = opt.dev_alloc;
+    c->dev_free = opt.dev_free;
+    c->alloc_user = opt.alloc_user;
+    c->reduce = opt.reduce;
+    c->reduce_user = opt.reduce_user;
+    if (opt.tuning)
+        c->tune = *opt.tuning;
+    else
+        dbc_tuning_default(&c->tune);
+    const dbc_tuning &T = c->tune;
     c->device = opt.device;
     c->rank = opt.rank;
     c->world = opt.world;
@@ -411,8 +516,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     // Per worker: the n-sized arrays of Scratch (mark, lowrec, dacc, Dv, Dold,
     // Dsig, U0, U1, Rv, Rl, Bq) and of the help board (gU), Doff, the deferred
     // long rows X, the insertion window (Wul, Wlev) and the chunk mirror.
-    int wcap = kWindow;
-    if (const char *e = getenv("DBC_WINDOW")) wcap = std::max(1, atoi(e));
+    const int wcap = T.window > 0 ? T.window : kWindow;
     const size_t per_worker = (size_t)n * (4 + 8 + 8 + 4 + 4 + 8 + 4 + 4 + 4 + 4 + 4 + 4) + (size_t)(n + 2) * 4 +
                               (size_t)kXcap * sizeof(XRow) + (size_t)2 * wcap * sizeof(int32_t) +
                               sizeof(ChunkSmem) + 64;
@@ -426,19 +530,19 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     // B200 against 256 (2/SM), 512 and 128 (4/SM): R-MAT 16 5.8 vs 9.6 ms,
     // Delaunay 2^18 22.3 vs 29.4 ms, Kronecker 20 0.85 vs 1.56 s
     c->sblock = 1024;
-    if (const char *e = getenv("DBC_SBLOCK")) {
-        const int b = atoi(e);
+    if (T.static_block > 0) {
+        const int b = T.static_block;
         c->sblock = (b == 128 || b == 512 || b == 1024) ? b : 256;
     }
     c->lowdeg = maxdeg <= 32;  // every row walked by one lane: no chunked up levels
-    if (const char *e = getenv("DBC_HDMIN")) c->hd_min = std::max(1, atoi(e));
-    if (const char *e = getenv("DBC_HDBLK")) c->hd_block = std::max(32, atoi(e));
-    if (const char *e = getenv("DBC_HEENT")) c->he_entries = std::max(256, atoi(e));
-    if (const char *e = getenv("DBC_HEMIN")) c->he_min = std::max(1, atoi(e));
-    if (const char *e = getenv("DBC_BUSY_HELP")) c->busy_help = std::max(0, atoi(e));
-    if (const char *e = getenv("DBC_BUSY_MIN")) c->busy_min = std::max(1, atoi(e));
-    if (const char *e = getenv("DBC_DLMIN")) c->dl_min = std::max(1, atoi(e));
-    if (const char *e = getenv("DBC_WIDE_INLANE")) c->wide_inlane = std::max(0, atoi(e));
+    if (T.help_down_min >= 0) c->hd_min = std::max(1, T.help_down_min);
+    if (T.help_down_block >= 0) c->hd_block = std::max(32, T.help_down_block);
+    if (T.help_entries >= 0) c->he_entries = std::max(256, T.help_entries);
+    if (T.help_min_blocks >= 0) c->he_min = std::max(1, T.help_min_blocks);
+    if (T.busy_help >= 0) c->busy_help = T.busy_help;
+    if (T.busy_min >= 0) c->busy_min = std::max(1, T.busy_min);
+    if (T.down_long_min >= 0) c->dl_min = std::max(1, T.down_long_min);
+    if (T.wide_inlane >= 0) c->wide_inlane = T.wide_inlane;
     // Update CTAs (measured on B200): one 1024-thread CTA per
     // SM (64 registers) by default -- a window-merged job has wide levels and
     // hub rows (R-MAT 16 +7.5%, Kronecker 20 +6%, small world +6% over one
@@ -447,10 +551,12 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     // 512-thread CTAs per SM instead (+40% over 1024).
     const bool many_narrow = c->lowdeg && c->k_loc >= 3 * c->nsm;
     c->block = many_narrow ? 512 : 1024;
-    if (const char *eb = getenv("DBC_BLOCK"))
-        c->block = atoi(eb) == 128 ? 128 : (atoi(eb) == 256 ? 256 : (atoi(eb) == 1024 ? 1024 : 512));
+    if (T.update_block > 0) {
+        const int b = T.update_block;
+        c->block = b == 128 ? 128 : (b == 256 ? 256 : (b == 1024 ? 1024 : 512));
+    }
     c->ub2 = c->block == 512 && c->k_loc >= 3 * c->nsm;
-    if (const char *e = getenv("DBC_UB2")) c->ub2 = c->block == 512 && atoi(e) != 0;
+    if (T.update_pair >= 0) c->ub2 = c->block == 512 && T.update_pair != 0;
     int upb = c->block == 128 ? 4 : (c->block >= 512 ? (c->ub2 ? 2 : 1) : 2);  // update CTAs per SM
     int want = opt.workers ? opt.workers : upb * c->nsm;
     want = std::min(want, c->k_loc);
@@ -469,9 +575,8 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     // slowest chain); 512-thread builds use 1024-thread heavy CTAs
     c->heavy_cap = (c->block == 128 || c->block == 1024 || c->ub2 || opt.workers) ? 0
                    : std::max(0, std::min(c->block == 512 ? c->nsm / 8 : c->nsm / 4, (int)(fit - c->workers)));
-    if (const char *e = getenv("DBC_HEAVY_CAP"))
-        if (c->block != 1024) c->heavy_cap = std::max(0, std::min(atoi(e), (int)(fit - c->workers)));
-    if (getenv("DBC_NO_HEAVY")) c->heavy_cap = 0;
+    if (T.heavy_cap >= 0 && c->block != 1024) c->heavy_cap = std::max(0, std::min(T.heavy_cap, (int)(fit - c->workers)));
+    if (T.disable & DBC_TUNE_NO_HEAVY) c->heavy_cap = 0;
     if (c->k_loc > 0 && c->workers == 0) {
         fail(c, DBC_ENOMEM, "not enough device memory for one worker (%zu bytes)", per_worker);
         return bail(DBC_ENOMEM);
@@ -511,16 +616,16 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->roots_d, (size_t)c->k_loc);
     // per-insertion workers (update_lean.cu): one CTA per root when memory allows
     c->lean_workers = std::max(0, std::min(c->k_loc, fit));
-    if (const char *e = getenv("DBC_LEAN_WORKERS")) c->lean_workers = std::max(1, std::min(c->lean_workers, atoi(e)));
-    if (getenv("DBC_NO_LEAN")) c->lean_on = false;
-    if (const char *e = getenv("DBC_LEAN_MAX")) c->lean_max = atoll(e);
-    if (const char *e = getenv("DBC_LEAN_SHORT")) c->lean_short = std::max(0, atoi(e));
+    if (T.lean_workers > 0) c->lean_workers = std::max(1, std::min(c->lean_workers, T.lean_workers));
+    if (T.disable & DBC_TUNE_NO_LEAN) c->lean_on = false;
+    if (T.lean_max_batch >= 0) c->lean_max = T.lean_max_batch;
+    if (T.lean_short >= 0) c->lean_short = T.lean_short;
     // per-insertion CTA width (measured on B200): hub-heavy
     // graphs need wide CTAs for their heavy levels (R-MAT 16: 512), meshes are
     // latency-bound on narrow levels (Delaunay 2^18: 256)
     c->lean_block = c->lowdeg ? 256 : 512;
-    if (const char *e = getenv("DBC_LEAN_BLOCK")) {
-        const int b = atoi(e);
+    if (T.lean_block > 0) {
+        const int b = T.lean_block;
         c->lean_block = (b == 256 || b == 512 || b == 1024) ? b : 128;
     }
     {  // a persistent grid: every worker resident (idle workers wait on the help board)
@@ -560,12 +665,12 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->help.low, nwk);
     AL(c->help.gbig, 2 * nwk);
     c->help.nworkers = (int)nwk;
-    if (const char *e = getenv("DBC_NO_HELP")) c->help_on = atoi(e) == 0;
+    if (T.disable & DBC_TUNE_NO_HELP) c->help_on = false;
     AL(c->next_slot, 4);  // [0] next root, [1] heavy lane's next root / unused, [2..3] lean: roots done, idle
     if (c->lean_workers) {
         char *bd = nullptr;
         AL(bd, lean_board_bytes() * (size_t)c->lean_workers);
-        c->lean_board = getenv("DBC_LEAN_NO_HELP") ? nullptr : (void *)bd;
+        c->lean_board = (T.disable & DBC_TUNE_NO_LEAN_HELP) ? nullptr : (void *)bd;
         cudaMemsetAsync(bd, 0, lean_board_bytes() * (size_t)c->lean_workers, c->stream);
     }
     AL(c->slots_d, (size_t)std::max(c->k_loc, 1));
@@ -631,6 +736,21 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
         fail(c, DBC_ECUDA, "init failed: %s", cudaGetErrorString(cudaGetLastError()));
         return bail(DBC_ECUDA);
     }
+    if (opt.nccl_id) {  // the BC all-reduce's communicator: one rank per GPU
+        NcclApi &nc = nccl_api();
+        if (!nc.ok) {
+            fail(c, DBC_ENCCL, "NCCL unavailable: %s", nc.why.c_str());
+            return bail(DBC_ENCCL);
+        }
+        ncclUniqueId id;
+        std::memcpy(&id, opt.nccl_id, sizeof id);
+        const ncclResult_t r = nc.comm_init_rank(&c->comm, c->world, id, c->rank);
+        if (r != ncclSuccess) {
+            c->comm = nullptr;
+            fail(c, DBC_ENCCL, "ncclCommInitRank(%d of %d): %s", c->rank, c->world, nc.error_string(r));
+            return bail(DBC_ENCCL);
+        }
+    }
     *out = c;
     return DBC_OK;
 }
@@ -663,6 +783,7 @@ extern "C" dbc_status dbc_static_compute(dbc_ctx *c) {
     if (tm) CK(cudaEventRecord(c->ev[4], c->stream));
     if (c->workers) {
         StaticArgs a;
+        a.exact_delta = (c->flags & DBC_FLAG_PULL_DELTA) ? 1 : 0;
         a.g = view_of(c);
         a.n = c->n;
         a.k_loc = c->k_loc;
@@ -794,8 +915,8 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     a.busy_min = c->busy_min;
     a.dl_min = c->dl_min;
     a.wide_inlane = c->wide_inlane;
-    a.trace_slot = getenv("DBC_TRACE_SLOT") ? atoi(getenv("DBC_TRACE_SLOT")) : -1;
-    a.lowdeg = c->lowdeg && !getenv("DBC_NO_LOWDEG");
+    a.trace_slot = c->tune.trace_slot;
+    a.lowdeg = c->lowdeg && !(c->tune.disable & DBC_TUNE_NO_LOWDEG);
     if (c->scen_cap > 0) {  // Fig. 2 / Fig. 4 log: one job per (root, insertion)
         a.scen = c->scen;
         a.merge = 0;
@@ -805,14 +926,17 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     int ulaunch = 0;
     // one job per (root, insertion) -- Mode S, DBC_FLAG_NO_MERGE, the scenario
     // log, and batches too small to merge -- runs the per-insertion kernel
-    const bool per_ins = (c->flags & (DBC_FLAG_MODE_S | DBC_FLAG_NO_MERGE)) || a.scen;
-    const bool use_lean = c->lean_on && c->lean_workers > 0 && !c->eworkers && (per_ins || cnt <= c->lean_max);
+    const bool pull = c->flags & DBC_FLAG_PULL_DELTA;
+    const bool per_ins = (c->flags & (DBC_FLAG_MODE_S | DBC_FLAG_NO_MERGE)) || a.scen || pull;
+    const bool use_lean = c->lean_workers > 0 && !c->eworkers && (c->lean_on || pull) &&
+                          (per_ins || cnt <= c->lean_max);
     a.static_slots = 0;
     a.lean_board = nullptr;
+    a.pull_delta = pull ? 1 : 0;
     a.short_mult = c->lean_short;
     if (use_lean) {
         const int nw = c->lean_workers;
-        a.lean_board = c->lean_board;
+        a.lean_board = pull ? nullptr : c->lean_board;  // pull mode: every pass local
         a.merge = 0;
         a.root_prof = c->prof_on ? c->root_prof : nullptr;
         if (c->prof_on)
@@ -876,7 +1000,7 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
                 std::nth_element(srt.begin(), srt.begin() + k / 2, srt.end());
                 const double med = srt[k / 2];
                 double hf = c->block == 512 ? 1.8 : 1.3;  // "slow" = this many medians
-                if (const char *e = getenv("DBC_HEAVY_FACTOR")) hf = atof(e);
+                if (c->tune.heavy_factor > 0.0f) hf = c->tune.heavy_factor;
                 while (nh < c->heavy_cap && nh < k - 1 && c->root_ms[order[nh]] > hf * med) ++nh;
             }
             // slot list: normal slots (longest first), then the heavy ones
@@ -1024,8 +1148,8 @@ extern "C" dbc_status dbc_insert_edges(dbc_ctx *c, const int32_t *u, const int32
 static dbc_status delete_host_ids(dbc_ctx *c, const int32_t *u, const int32_t *v, int64_t cnt,
                                   dbc_insert_stats *stats) {
     if (!c->have_state) return fail(c, DBC_ESTATE, "dbc_static_compute must run before deletions");
-    if (c->flags & DBC_FLAG_EDGE_PARALLEL)
-        return fail(c, DBC_EINVAL, "deletions are not supported with DBC_FLAG_EDGE_PARALLEL");
+    if (c->flags & (DBC_FLAG_EDGE_PARALLEL | DBC_FLAG_PULL_DELTA))
+        return fail(c, DBC_EINVAL, "deletions are not supported with DBC_FLAG_EDGE_PARALLEL or DBC_FLAG_PULL_DELTA");
     if (cnt > c->edge_cap) return fail(c, DBC_EINVAL, "deletion batch larger than the staging buffer");
     if (c->scen_cap > 0 && cnt > c->scen_cap)
         return fail(c, DBC_EINVAL, "batch of %lld exceeds the scenario log (%lld insertions)",
@@ -1098,6 +1222,7 @@ static dbc_status delete_host_ids(dbc_ctx *c, const int32_t *u, const int32_t *v
     a.del = 1;
     a.static_slots = 0;
     a.lean_board = nullptr;
+    a.pull_delta = 0;
     a.hd_min = c->hd_min;
     a.hd_block = c->hd_block;
     a.he_entries = c->he_entries;
@@ -1106,8 +1231,8 @@ static dbc_status delete_host_ids(dbc_ctx *c, const int32_t *u, const int32_t *v
     a.busy_min = c->busy_min;
     a.dl_min = c->dl_min;
     a.wide_inlane = c->wide_inlane;
-    a.trace_slot = getenv("DBC_TRACE_SLOT") ? atoi(getenv("DBC_TRACE_SLOT")) : -1;
-    a.lowdeg = c->lowdeg && !getenv("DBC_NO_LOWDEG");
+    a.trace_slot = c->tune.trace_slot;
+    a.lowdeg = c->lowdeg && !(c->tune.disable & DBC_TUNE_NO_LOWDEG);
     a.scen = nullptr;
     if (c->scen_cap > 0) {
         a.scen = c->scen;
@@ -1213,8 +1338,21 @@ extern "C" dbc_status dbc_get_bc_partial_device(dbc_ctx *c, double **p) {
 extern "C" dbc_status dbc_get_bc(dbc_ctx *c, double *bc) {
     if (!c || !bc) return DBC_EINVAL;
     if (!c->have_state) return fail(c, DBC_ESTATE, "no state: call dbc_static_compute first");
+    if (c->world > 1 && !c->comm && !c->reduce)
+        return fail(c, DBC_ESTATE, "world %d: global BC needs opt.nccl_id or opt.reduce "
+                                   "(or reduce dbc_get_bc_partial_device yourself)", c->world);
     double *p = nullptr;
     TRY(dbc_get_bc_partial_device(c, &p));
+    // Eq. (3) over all roots: the per-rank partials summed across ranks, in
+    // place on the context stream (a copy: the library keeps its own partial)
+    if (c->comm) {
+        NcclApi &nc = nccl_api();
+        const ncclResult_t r = nc.all_reduce(p, p, (size_t)c->n, ncclFloat64, ncclSum, c->comm, c->stream);
+        if (r != ncclSuccess) return fail(c, DBC_ENCCL, "ncclAllReduce: %s", nc.error_string(r));
+    } else if (c->reduce && c->world > 1) {
+        const int r = c->reduce(p, (int64_t)c->n, (void *)c->stream, c->reduce_user);
+        if (r != 0) return fail(c, DBC_ENCCL, "reduce callback returned %d", r);
+    }
     CK(cudaMemcpyAsync(bc, p, sizeof(double) * c->n, cudaMemcpyDeviceToHost, c->stream));
     return check_err(c);
 }
@@ -1297,7 +1435,7 @@ extern "C" dbc_status dbc_scenario_log(dbc_ctx *c, int64_t max_insertions) {
         if (c->scen) {
             for (auto &q : c->allocs)
                 if (q == (void *)c->scen) q = nullptr;
-            CK(cudaFree(c->scen));
+            dfree(c, c->scen);
             c->bytes -= (int64_t)(sizeof(long long) * (size_t)std::max<int64_t>(c->scen_alloc, 1) *
                                   std::max(c->k_loc, 1));
             c->scen = nullptr;

@@ -586,11 +586,13 @@ struct UpdateArgs {
     int32_t trace_slot;            // -DDBC_PHASE_TIMERS builds: time this slot only (-1: all)
     int32_t static_slots;          // unused (kept zero)
     void *lean_board;              // update_lean.cu help board (nullptr: no cooperative help)
+    int32_t pull_delta;            // update_lean.cu: DBC_FLAG_PULL_DELTA (every touched vertex pulls delta)
     int32_t short_mult;            // update_lean.cu: level-2 up rows longer than short_mult x deg(root)
                                    // find their predecessors by probing adj(root)
 };
 
 struct StaticArgs {
+    int32_t exact_delta;  // DBC_FLAG_PULL_DELTA: long rows' delta re-summed in canonical order
     GView g;
     int32_t n;
     int32_t k_loc;

@@ -176,7 +176,22 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) static_kernel(StaticArgs a
                     bytes += 8;
                     return bwd_visit(S.c0[t], dy, q.x, q.y);
                 });
-                if (tid < m) bwd_finish(S.v[tid], S.acc[tid]);
+                if (tid < m) {
+                    double acc = S.acc[tid];
+                    if (a.exact_delta) {  // DBC_FLAG_PULL_DELTA: Eq. (2) left to right in canonical order
+                        const int v = S.v[tid];
+                        const int2 r = row_of(g, v, INT32_MAX);
+                        const double sv = S.c0[tid];
+                        acc = 0.0;
+                        for (int j = r.x; j < r.y; ++j) {
+                            const int y = ldg_i(g.col + j);
+                            if (st.dist(y) != lev + 1) continue;
+                            const double2 q = st.sd[y];
+                            acc = __dadd_rn(acc, __dmul_rn(__ddiv_rn(sv, q.x), __dadd_rn(1.0, q.y)));
+                        }
+                    }
+                    bwd_finish(S.v[tid], acc);
+                }
                 __syncthreads();
             }
             __syncthreads();

@@ -127,7 +127,8 @@ struct PassCtx {
     int *low, *rmin, *rmax;
     double *acc;                 // per-row sums (when ev == nullptr)
     double *ev;                  // per-entry contributions (a local pass of <= kLEnt entries)
-    bool full;                   // scenario log: claim even over a zero push (Alg. 2's touched set)
+    bool full;
+    bool pull;                   // DBC_FLAG_PULL_DELTA: targets are only claimed (they pull)                   // scenario log: claim even over a zero push (Alg. 2's touched set)
 };
 
 __device__ __forceinline__ int block_excl_scan(int x, int *total) {
@@ -231,7 +232,7 @@ __device__ __forceinline__ double pass_visit(const PassCtx &c, LeanSmem &S, int 
             return 0.0;
         case kPRem:  // an old predecessor outside D gets the old contribution back
             if (dy == S.aux[t] && mk != c.mD) {
-                atomicAdd(c.dacc + y, S.c0[t]);
+                if (!c.pull) atomicAdd(c.dacc + y, S.c0[t]);
                 bytes += 16;
                 if (mk < c.E && atomicMax(c.mark + y, c.mU) < c.E) {
                     const int p = atomicAdd(c.ctr, 1);
@@ -352,6 +353,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
     LeanBoard *mine = board ? board + wk : nullptr;
     int *live = a.next_slot + 2;                   // [0] roots finished, [1] idle workers
     const int total_roots = a.slot_list ? a.slot_count : a.k_loc;
+    const bool pull = a.pull_delta != 0;  // DBC_FLAG_PULL_DELTA (no help board then)
     int hseq = 0;
 
     // counters: thread-local bytes / scanned entries, thread 0's tallies
@@ -506,7 +508,8 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                 pc.rmax = &s_rmax;
                 pc.acc = S.acc;
                 pc.ev = nullptr;
-                pc.full = a.scen != nullptr;
+                pc.full = a.scen != nullptr || pull;
+                pc.pull = pull;
                 // ---- seed (A2) ----
                 if (tid == 0) {
                     const int dl = __ldcg(st.d + ul);
@@ -648,17 +651,22 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                     cp.l = l;
                     cp.list = Ul[cu ^ 1];
                     cp.ctr = &s_ucnt[cu ^ 1];
-                    // D vertices of the level: delta by pull, pushes to predecessors outside D
-                    for (int c = 0; c < nd; c += kLCap) {
-                        const int cnt = min(kLCap, nd - c);
+                    // D vertices of the level: delta by pull, pushes to predecessors
+                    // outside D.  DBC_FLAG_PULL_DELTA: the up vertices too (rows
+                    // nd.. of this loop, aux = -1): every touched vertex pulls
+                    // delta in canonical order, predecessors are only claimed.
+                    const int npull = nd + (pull ? nu : 0);
+                    for (int c = 0; c < npull; c += kLCap) {
+                        const int cnt = min(kLCap, npull - c);
                         if (tid == 0) s_nst = 0;
                         for (int t = tid; t < cnt; t += kBlock) {
-                            const int x = __ldcg(Dv + db + c + t);
+                            const int j = c + t;
+                            const int x = j < nd ? __ldcg(Dv + db + j) : __ldcg(Ul[cu] + j - nd);
                             const double2 q = __ldcg(st.sd + x);  // (sigma_new, delta_old)
                             const int2 r = row_of(g, x, lim);
                             S.v[t] = x;
                             S.beg[t] = r.x;
-                            S.aux[t] = db + c + t;
+                            S.aux[t] = j < nd ? db + j : -1;
                             S.c0[t] = q.x;
                             S.c1[t] = q.y;
                             S.off[t + 1] = r.y - r.x;
@@ -677,13 +685,26 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                             if (cd.ev) {  // Eq. (2) summed left to right in canonical order
                                 dn = 0.0;
                                 for (int e = S.off[t]; e < S.off[t + 1]; ++e) dn = __dadd_rn(dn, S.ev[e]);
+                            } else if (pull) {  // a chunk too wide for the entry buffer: re-sum in order
+                                const int2 r = row_of(g, x, lim);
+                                dn = 0.0;
+                                for (int e = r.x; e < r.y; ++e) {
+                                    const int y = ldg_i(g.col + e);
+                                    if (__ldcg(st.d + y) != l + 1) continue;
+                                    const double2 qy = __ldcg(st.sd + y);
+                                    dn = __dadd_rn(dn, __dmul_rn(__ddiv_rn(S.c0[t], qy.x), __dadd_rn(1.0, qy.y)));
+                                }
                             }
                             const double sn = S.c0[t], dold = S.c1[t];
-                            atomicAdd(a.bc + x, __dsub_rn(dn, dold));
-                            st.sd[x].y = dn;
-                            const bool lowered = __ldcg(Dold + di) != l;
-                            S.c0[t] = __ddiv_rn(__dadd_rn(1.0, dn), sn);
-                            S.c1[t] = lowered ? 0.0 : __ddiv_rn(__dadd_rn(1.0, dold), __ldcg(Dsig + di));
+                            if (dn != dold) {
+                                atomicAdd(a.bc + x, __dsub_rn(dn, dold));
+                                st.sd[x].y = dn;
+                            }
+                            if (di >= 0) {
+                                const bool lowered = __ldcg(Dold + di) != l;
+                                S.c0[t] = __ddiv_rn(__dadd_rn(1.0, dn), sn);
+                                S.c1[t] = lowered ? 0.0 : __ddiv_rn(__dadd_rn(1.0, dold), __ldcg(Dsig + di));
+                            }
                             my_bytes += 16 + 16;
                         }
                         __syncthreads();
@@ -691,6 +712,10 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                         if (nst <= kLStash) {
                             for (int j = tid; j < nst; j += kBlock) {
                                 const int t = S.st_t[j], pr = S.st_p[j], p = pr & INT32_MAX;
+                                if (pull) {  // the predecessor pulls its own delta at level l - 1
+                                    if (pr >= 0) claim_append(cp, p, mU);
+                                    continue;
+                                }
                                 const bool new_edge = S.v[t] == ul && p == uh;
                                 const double w = new_edge ? S.c0[t] : __dsub_rn(S.c0[t], S.c1[t]);
                                 if (w != 0.0) atomicAdd(dacc + p, w);
@@ -711,6 +736,10 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                                 }
                                 const int p = ldg_i(g.col + S.beg[lo] + (e - S.off[lo]));
                                 if (__ldcg(st.d + p) != l - 1 || __ldcg(mark + p) == mD) continue;
+                                if (pull) {
+                                    claim_append(cp, p, mU);
+                                    continue;
+                                }
                                 const bool new_edge = S.v[lo] == ul && p == uh;
                                 const double w = new_edge ? S.c0[lo] : __dsub_rn(S.c0[lo], S.c1[lo]);
                                 if (w != 0.0) atomicAdd(dacc + p, w);
@@ -721,7 +750,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                         __syncthreads();
                     }
                     // up vertices of the level: apply Ddelta, forward it to the predecessors
-                    for (int c = 0; c < nu; c += kLCap) {
+                    for (int c = 0; c < (pull ? 0 : nu); c += kLCap) {
                         const int cnt = min(kLCap, nu - c);
                         if (tid == 0) s_nsc = 0;
                         __syncthreads();
@@ -909,6 +938,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
             c.acc = ob->acc;
             c.ev = nullptr;
             c.full = a.scen != nullptr;
+            c.pull = false;
             uint32_t hscan = 0;
             lean_pass(c, S, &s_nst, g, cnt, b * kHelpBlk, min(Etot, (b + 1) * kHelpBlk), my_bytes, hscan);
             my_scan += hscan;

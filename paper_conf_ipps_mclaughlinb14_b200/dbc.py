@@ -24,6 +24,8 @@ FLAG_EXACT_BC = 0x4
 FLAG_NO_REORDER = 0x8
 FLAG_NO_MERGE = 0x10
 FLAG_EDGE_PARALLEL = 0x20
+FLAG_PULL_DELTA = 0x40
+TUNE_NO_HELP, TUNE_NO_HEAVY, TUNE_NO_LEAN, TUNE_NO_LEAN_HELP, TUNE_NO_LOWDEG = 0x1, 0x2, 0x4, 0x8, 0x10
 
 STATUS = {
     0: "DBC_OK", -1: "DBC_EINVAL", -2: "DBC_ENOMEM", -3: "DBC_ECUDA", -4: "DBC_ENCCL",
@@ -38,12 +40,34 @@ class DBCError(RuntimeError):
         self.name = STATUS.get(status, str(status))
 
 
+REDUCE_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_int64, ctypes.c_void_p, ctypes.c_void_p)
+ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p)
+FREE_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p)
+
+
+class Tuning(ctypes.Structure):
+    """dbc_tuning (include/dbc.h): launch configuration only, results never depend on it."""
+    _fields_ = [
+        ("update_block", ctypes.c_int32), ("update_pair", ctypes.c_int32),
+        ("static_block", ctypes.c_int32), ("window", ctypes.c_int32), ("heavy_cap", ctypes.c_int32),
+        ("heavy_factor", ctypes.c_float), ("help_down_min", ctypes.c_int32),
+        ("help_down_block", ctypes.c_int32), ("help_entries", ctypes.c_int32),
+        ("help_min_blocks", ctypes.c_int32), ("busy_help", ctypes.c_int32), ("busy_min", ctypes.c_int32),
+        ("down_long_min", ctypes.c_int32), ("wide_inlane", ctypes.c_int32), ("lean_block", ctypes.c_int32),
+        ("lean_workers", ctypes.c_int32), ("lean_max_batch", ctypes.c_int32), ("lean_short", ctypes.c_int32),
+        ("trace_slot", ctypes.c_int32), ("disable", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 8),
+    ]
+
+
 class Options(ctypes.Structure):
     _fields_ = [
         ("device", ctypes.c_int32), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
         ("workers", ctypes.c_int32), ("edge_capacity", ctypes.c_int64),
-        ("stream", ctypes.c_void_p), ("flags", ctypes.c_uint32),
-        ("reserved", ctypes.c_uint32 * 7),
+        ("stream", ctypes.c_void_p), ("flags", ctypes.c_uint32), ("pad0", ctypes.c_uint32),
+        ("tuning", ctypes.POINTER(Tuning)), ("nccl_id", ctypes.c_void_p),
+        ("reduce", REDUCE_FN), ("reduce_user", ctypes.c_void_p),
+        ("dev_alloc", ALLOC_FN), ("dev_free", FREE_FN), ("alloc_user", ctypes.c_void_p),
+        ("reserved", ctypes.c_uint32 * 4),
     ]
 
 
@@ -80,6 +104,8 @@ class Timings(ctypes.Structure):
 _P = ctypes.c_void_p
 SIGNATURES = {
     "dbc_options_default": (None, [_P]),
+    "dbc_tuning_default": (None, [_P]),
+    "dbc_nccl_unique_id": (ctypes.c_int, [_P]),
     "dbc_create": (ctypes.c_int, [_P, ctypes.c_int32, _P, _P, _P, ctypes.c_int32, _P]),
     "dbc_static_compute": (ctypes.c_int, [_P]),
     "dbc_insert_edges": (ctypes.c_int, [_P, _P, _P, ctypes.c_int64, _P]),
@@ -149,10 +175,18 @@ class DynamicBC:
     """
 
     def __init__(self, n, row_ptr, col, roots, *, device=0, rank=0, world=1, workers=0,
-                 edge_capacity=0, stream=None, flags=0):
+                 edge_capacity=0, stream=None, flags=0, tuning=None, nccl_id=None, reduce=None,
+                 allocator=None):
+        """tuning: dict of dbc_tuning fields (launch configuration only);
+        nccl_id: 128 bytes from nccl_unique_id() on rank 0 (the context then
+        owns an NCCL communicator and get_bc() returns the global BC);
+        reduce: python callable(ptr, n, stream) -> int summing the partial in
+        place across ranks (see torch_reducer); allocator: (alloc, free)
+        python callables, e.g. torch_allocator(device)."""
         lib = load_library()
         self._lib = lib
         self._ctx = None
+        self._keep = []  # ctypes objects the context points at
         self.n = int(n)
         self.k = int(np.asarray(roots).size)
         self.rank, self.world, self.device = int(rank), int(world), int(device)
@@ -163,6 +197,34 @@ class DynamicBC:
         lib.dbc_options_default(ctypes.byref(opt))
         opt.device, opt.rank, opt.world = self.device, self.rank, self.world
         opt.workers, opt.edge_capacity, opt.flags = int(workers), int(edge_capacity), int(flags)
+        if tuning:
+            t = Tuning()
+            lib.dbc_tuning_default(ctypes.byref(t))
+            for k, val in tuning.items():
+                if k not in dict(Tuning._fields_):
+                    raise KeyError(f"unknown tuning field {k}")
+                setattr(t, k, val)
+            self._keep.append(t)
+            opt.tuning = ctypes.pointer(t)
+        if nccl_id is not None:
+            buf = ctypes.create_string_buffer(bytes(nccl_id), 128)
+            self._keep.append(buf)
+            opt.nccl_id = ctypes.cast(buf, ctypes.c_void_p)
+        if reduce is not None:
+            def _red(ptr, cnt, strm, _user, _f=reduce):
+                try:
+                    return int(_f(int(ptr), int(cnt), strm))
+                except Exception:  # pragma: no cover - reported as DBC_ENCCL
+                    return 1
+            cb = REDUCE_FN(_red)
+            self._keep.append(cb)
+            opt.reduce = cb
+        if allocator is not None:
+            af, ff = allocator
+            ca = ALLOC_FN(lambda b, _u, _f=af: _f(int(b)) or None)
+            cf = FREE_FN(lambda p, _u, _f=ff: _f(int(p)))
+            self._keep += [ca, cf]
+            opt.dev_alloc, opt.dev_free = ca, cf
         if stream is None:
             try:
                 import torch
@@ -232,6 +294,13 @@ class DynamicBC:
         out = np.empty(self.n, dtype=np.float64) if out is None else out
         _check(self._ctx, self._lib.dbc_get_bc(self._ctx, _np_ptr(out)))
         return out
+
+    def get_bc_partial(self):
+        """This rank's BC partial (Eq. (3) over the local roots) on the host: a copy
+        of dbc_get_bc_partial_device's buffer."""
+        ptr = self.bc_partial_device_ptr()
+        self.synchronize()
+        return _wrap_device_f64(ptr, self.n, self.device).cpu().numpy().copy()
 
     def bc_partial_device_ptr(self) -> int:
         p = ctypes.c_void_p()
@@ -316,6 +385,53 @@ class DynamicBC:
         return b.value
 
 
+def nccl_unique_id() -> bytes:
+    """dbc_nccl_unique_id: 128 bytes for every rank's DynamicBC(nccl_id=...)."""
+    lib = load_library()
+    buf = ctypes.create_string_buffer(128)
+    _check(None, lib.dbc_nccl_unique_id(buf))
+    return buf.raw
+
+
+def torch_reducer(group=None):
+    """A `reduce` callback for DynamicBC: sums the BC partial across the ranks of a
+    torch.distributed group, in place -- NCCL groups reduce the device buffer
+    directly, gloo groups through a host copy.  The library's stream is
+    synchronised first, so the reduction sees the finished partial."""
+    import torch
+    import torch.distributed as dist
+
+    def red(ptr, n, stream):
+        dev = torch.cuda.current_device()
+        torch.cuda.synchronize()  # the partial is final on the library's stream
+        t = _wrap_device_f64(ptr, n, dev)
+        if dist.get_backend(group) == "nccl":
+            dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+            torch.cuda.synchronize()
+        else:
+            h = t.cpu()
+            dist.all_reduce(h, op=dist.ReduceOp.SUM, group=group)
+            t.copy_(h)
+            torch.cuda.synchronize()
+        return 0
+
+    return red
+
+
+def torch_allocator(device=0):
+    """(alloc, free) hooks routing the library's device memory through torch's
+    caching allocator (dbc_options.dev_alloc / dev_free)."""
+    import torch
+
+    def alloc(nbytes):
+        return int(torch.cuda.caching_allocator_alloc(nbytes, device))
+
+    def free(ptr):
+        torch.cuda.caching_allocator_delete(ptr)
+
+    return alloc, free
+
+
 def local_slots(k: int, rank: int, world: int):
     """Root slots owned by `rank` (slot % world == rank), SURVEY.md Sec. 8(e)."""
     return list(range(rank, k, world))
@@ -324,8 +440,9 @@ def local_slots(k: int, rank: int, world: int):
 def allreduce_bc(dbc: DynamicBC, group=None, force=False):
     """Sum the per-rank BC partials over torch.distributed (NCCL on GPUs) and
     return the global BC on the host -- the only cross-GPU exchange of the
-    method.  force=True runs the collective even for a
-    single rank (tests)."""
+    method -- for contexts created without nccl_id /
+    reduce (those return the global BC from get_bc() directly).  force=True
+    runs the collective even for a single rank (tests)."""
     import torch
     import torch.distributed as dist
 

@@ -62,7 +62,7 @@ def test_built_for_sm100a():
 
 
 def test_abi_version_and_strerror(lib):
-    assert lib.dbc_abi_version() == 1
+    assert lib.dbc_abi_version() == 2
     assert lib.dbc_strerror(-6) == b"invalid edge in batch"
     assert lib.dbc_strerror(0) == b"ok"
 
@@ -121,3 +121,30 @@ def test_product_never_imports_oracle():
                 txt = open(os.path.join(dirpath, f)).read()
                 assert "import oracle" not in txt and "from oracle" not in txt, f
                 assert "oracle/" not in txt.replace("oracle/ ", ""), f
+
+
+def test_binding_struct_layouts_match_the_header(tmp_path):
+    """dbc_options / dbc_tuning / dbc_insert_stats / dbc_timings: the ctypes
+    mirrors have the C sizes and field offsets (compiled against include/dbc.h)."""
+    import subprocess
+
+    from paper_conf_ipps_mclaughlinb14_b200 import dbc
+
+    structs = {"dbc_options": dbc.Options, "dbc_tuning": dbc.Tuning,
+               "dbc_insert_stats": dbc.InsertStats, "dbc_timings": dbc.Timings}
+    lines = ['#include <stdio.h>', '#include <stddef.h>', '#include "dbc.h"', "int main(void) {"]
+    for cname, py in structs.items():
+        lines.append(f'printf("{cname} size %zu\\n", sizeof({cname}));')
+        for fname, _ in py._fields_:
+            lines.append(f'printf("{cname} {fname} %zu\\n", offsetof({cname}, {fname}));')
+    lines.append("return 0; }")
+    src = tmp_path / "layout.c"
+    src.write_text("\n".join(lines))
+    exe = tmp_path / "layout"
+    subprocess.check_call(["gcc", "-I", os.path.join(ROOT, "include"), str(src), "-o", str(exe)])
+    out = subprocess.run([str(exe)], capture_output=True, text=True, check=True).stdout.split("\n")
+    got = {tuple(l.split()[:2]): int(l.split()[2]) for l in out if l}
+    for cname, py in structs.items():
+        assert got[(cname, "size")] == ctypes.sizeof(py), cname
+        for fname, _ in py._fields_:
+            assert got[(cname, fname)] == getattr(py, fname).offset, (cname, fname)

@@ -55,7 +55,7 @@ class Ref:
 def check(dbc, ref: Ref, sample_local, what="", delta_tol=DELTA_TOL):
     """BC over all of the context's roots + d/sigma/delta on sample_local (local indices)."""
     bc_ref, d_ref, s_ref, dl_ref = ref.compute(sample_local)
-    bc = dbc.get_bc()
+    bc = dbc.get_bc() if dbc.world == 1 else dbc.get_bc_partial()  # a rank's partial vs its roots
     err = _bc_err(bc, bc_ref)
     assert err <= BC_TOL, f"{what}: BC rel err {err}"
     worst = 0.0

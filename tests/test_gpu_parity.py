@@ -19,9 +19,22 @@ BC_TOL = 1e-9
 DELTA_TOL = 1e-12  # SURVEY.md Sec. 8(c) item 14 (hybrid delta, relative, floor 1)
 
 
+_TUNE: dict = {}
+
+
+@pytest.fixture
+def tune():
+    """dbc_tuning fields (launch configuration) for the contexts _dbc creates in a test."""
+    _TUNE.clear()
+    yield _TUNE
+    _TUNE.clear()
+
+
 def _dbc(g, roots, **kw):
     from paper_conf_ipps_mclaughlinb14_b200 import DynamicBC
 
+    if _TUNE:
+        kw.setdefault("tuning", dict(_TUNE))
     return DynamicBC(g.n, g.row_ptr, g.col, roots, **kw)
 
 
@@ -73,9 +86,9 @@ def test_static_matches_oracle(name):
 
 @pytest.mark.parametrize("sblock", ["128", "256", "512"])
 @pytest.mark.parametrize("name", ["grid_big_sigma", "disconnected", "rmat10", "delaunay12", "hub"])
-def test_static_other_widths_match_oracle(name, sblock, monkeypatch):
-    """The static kernel at the non-default CTA widths (DBC_SBLOCK; default 1024)."""
-    monkeypatch.setenv("DBC_SBLOCK", sblock)
+def test_static_other_widths_match_oracle(name, sblock, tune):
+    """The static kernel at the non-default CTA widths (tuning.static_block; default 1024)."""
+    tune["static_block"] = int(sblock)
     g, roots = STATIC_CASES[name]()
     roots = np.asarray(roots, np.int32)
     ref = oracle.brandes_csr(g, roots)
@@ -158,11 +171,11 @@ def test_grid_sigma_above_2p53_dynamic():
 @pytest.mark.parametrize("lean", [True, False])  # per-insertion jobs on update_lean.cu / update.cu
 @pytest.mark.parametrize("flags", [0, 1, 0x10])  # Mode A merged, Mode S, Mode A one job per insertion
 @pytest.mark.parametrize("name", ["karate", "rmat10", "delaunay12u"])
-def test_batch_modes_match_oracle(name, flags, lean, monkeypatch):
+def test_batch_modes_match_oracle(name, flags, lean, tune):
     if flags == 0 and not lean:
         pytest.skip("merged batches do not use the per-insertion kernel")
     if not lean:
-        monkeypatch.setenv("DBC_NO_LEAN", "1")
+        tune["disable"] = 0x4  # DBC_TUNE_NO_LEAN
     wl = W.make_workload(name)
     ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
     with _dbc(wl.graph, wl.roots, flags=flags) as dbc:
@@ -230,7 +243,7 @@ def test_fake_multi_gpu_shards_sum_to_single():
             with _dbc(wl.graph, wl.roots, rank=rank, world=world) as dbc:
                 dbc.static_compute()
                 dbc.insert_edges(wl.ins_u, wl.ins_v)
-                parts.append(dbc.get_bc())
+                parts.append(dbc.get_bc() if world == 1 else dbc.get_bc_partial())
                 assert dbc.num_local_roots() == len(range(rank, wl.roots.size, world))
         outs.append(np.sum(parts, axis=0))
     assert_bc(outs[1], outs[0], tol=1e-12)
@@ -337,9 +350,9 @@ def test_no_reorder_flag_matches_oracle(name):
 
 
 @pytest.mark.parametrize("name", ["karate", "rmat10", "delaunay12u"])
-def test_block128_kernels_match_oracle(name, monkeypatch):
+def test_block128_kernels_match_oracle(name, tune):
     """The 128-thread kernel build (chosen when there are more roots than 2 x SMs)."""
-    monkeypatch.setenv("DBC_BLOCK", "128")
+    tune["update_block"] = 128
     wl = W.make_workload(name)
     ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
     with _dbc(wl.graph, wl.roots) as dbc:
@@ -352,13 +365,13 @@ def test_block128_kernels_match_oracle(name, monkeypatch):
 
 
 @pytest.mark.parametrize("block", ["256", "512"])
-def test_heavy_lane_batches_match_oracle(monkeypatch, block):
+def test_heavy_lane_batches_match_oracle(tune, block):
     """Several Mode-A batches so the adaptive heavy lane (2x-wide CTAs for the
     slowest roots of the previous batch: 512 threads beside the 256-thread
     build, 1024 beside the 512-thread one) is exercised; d/sigma bit-exact."""
-    monkeypatch.setenv("DBC_BLOCK", block)
-    monkeypatch.setenv("DBC_HEAVY_FACTOR", "1.0")  # any root slower than the median
-    monkeypatch.setenv("DBC_WINDOW", "8")  # several jobs per root and batch
+    tune["update_block"] = int(block)
+    tune["heavy_factor"] = 1.0  # any root slower than the median
+    tune["window"] = 8  # several jobs per root and batch
     wl = W.make_workload("rmat10", insertions=120)
     ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
     with _dbc(wl.graph, wl.roots) as dbc:
@@ -424,14 +437,14 @@ def test_kron20_full_size_sampled():
     _sampled_full_size("kron20", 600, 3)
 
 
-def test_help_off_matches_help_on(monkeypatch):
-    """DBC_NO_HELP=1 (every C2 push done by its owner CTA) and the default
+def test_help_off_matches_help_on(tune):
+    """DBC_TUNE_NO_HELP (every C2 push done by its owner CTA) and the default
     cooperative path give bitwise-equal d/sigma and BC within tolerance."""
     wl = W.make_workload("rmat16", insertions=400)
     g = wl.graph
     outs = []
-    for off in ("1", "0"):
-        monkeypatch.setenv("DBC_NO_HELP", off)
+    for off in (1, 0):
+        tune["disable"] = off  # DBC_TUNE_NO_HELP
         with _dbc(g, wl.roots) as dbc:
             dbc.static_compute()
             dbc.insert_edges(wl.ins_u, wl.ins_v)
@@ -470,10 +483,10 @@ def test_case2_groups_match_oracle_and_no_merge(name):
 
 @pytest.mark.parametrize("window", ["2", "7", "64"])
 @pytest.mark.parametrize("name", ["rmat10", "delaunay12u"])
-def test_window_sizes_match_oracle(name, window, monkeypatch):
+def test_window_sizes_match_oracle(name, window, tune):
     """Jobs of `window` insertions (seed injection across several windows per
     batch, Case 3 inside windows): oracle d/sigma bit-exact, BC within tolerance."""
-    monkeypatch.setenv("DBC_WINDOW", window)
+    tune["window"] = int(window)
     wl = W.make_workload(name)
     ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
     for u, v in zip(wl.ins_u, wl.ins_v):
@@ -721,19 +734,17 @@ def test_heavy_lane_with_help_completes_rmat16(rep):
 
 @pytest.mark.parametrize("block", [None, "512"])
 @pytest.mark.parametrize("name", ["rmat10", "delaunay12u", "smallworld"])
-def test_forced_help_paths_match_oracle(name, block, monkeypatch):
+def test_forced_help_paths_match_oracle(name, block, tune):
     """Every cooperative path forced on at small sizes: helped down levels
     (kind 1, 32-item blocks), entry-balanced long rows of every down level
     (kind 4), the Case-3 removal pass as help blocks (kind 3), helped delta-pull
     / push passes (kinds 2 / 0, 256-entry blocks), busy workers taking blocks of
     any pass; several batches (heavy lanes).  d/sigma bit-exact vs the oracle,
     BC within tolerance."""
-    for k, v in {"DBC_HDMIN": "1", "DBC_HDBLK": "32", "DBC_DLMIN": "1", "DBC_HEMIN": "1",
-                 "DBC_HEENT": "256", "DBC_BUSY_MIN": "1", "DBC_BUSY_HELP": "4",
-                 "DBC_HEAVY_FACTOR": "1.0"}.items():
-        monkeypatch.setenv(k, v)
+    tune.update(help_down_min=1, help_down_block=32, down_long_min=1, help_min_blocks=1,
+                help_entries=256, busy_min=1, busy_help=4, heavy_factor=1.0)
     if block:  # 512-thread CTAs (128 registers) beside the default width
-        monkeypatch.setenv("DBC_BLOCK", block)
+        tune["update_block"] = int(block)
     wl = W.make_workload(name)
     ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
     with _dbc(wl.graph, wl.roots) as dbc:
@@ -752,16 +763,16 @@ def test_forced_help_paths_match_oracle(name, block, monkeypatch):
 
 
 @pytest.mark.parametrize("block", [None, "512"])
-def test_wide_up_levels_deferred_chunks_match_oracle(block, monkeypatch):
+def test_wide_up_levels_deferred_chunks_match_oracle(block, tune):
     """Wide up levels walked with short rows in-lane (published as help blocks,
     kind 5) and long rows in chunks, more than one chunk of them deferred
     (DBC_WIDE_INLANE forces the mode on every level wider than a CTA): R-MAT
     2^14 / edgefactor 16, 64 roots, 400 insertions in two batches; d/sigma
     bit-exact vs the oracle, BC in tolerance."""
-    monkeypatch.setenv("DBC_WIDE_INLANE", "100000")
-    monkeypatch.setenv("DBC_BUSY_MIN", "1")  # every pass worth publishing (kind-5 help blocks too)
+    tune["wide_inlane"] = 100000
+    tune["busy_min"] = 1  # every pass worth publishing (kind-5 help blocks too)
     if block:
-        monkeypatch.setenv("DBC_BLOCK", block)
+        tune["update_block"] = int(block)
     wl = W.make_workload("rmat14")
     ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
     with _dbc(wl.graph, wl.roots) as dbc:
@@ -780,10 +791,10 @@ def test_wide_up_levels_deferred_chunks_match_oracle(block, monkeypatch):
 
 # ------------------------------------------------ per-insertion kernel (update_lean.cu) ----
 @pytest.mark.parametrize("name", ["rmat10", "delaunay12u", "smallworld_small"])
-def test_lean_fewer_workers_than_roots(name, monkeypatch):
+def test_lean_fewer_workers_than_roots(name, tune):
     """Per-insertion jobs with 3 worker CTAs for all roots (dynamic root counter,
     several roots per worker and launch), one-job-per-insertion batch and Mode S."""
-    monkeypatch.setenv("DBC_LEAN_WORKERS", "3")
+    tune["lean_workers"] = 3
     wl = W.make_workload(name)
     ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
     for u, v in zip(wl.ins_u, wl.ins_v):
@@ -797,10 +808,10 @@ def test_lean_fewer_workers_than_roots(name, monkeypatch):
 
 
 @pytest.mark.parametrize("mult", ["0", "1"])
-def test_lean_level2_shortcut_forced(mult, monkeypatch):
+def test_lean_level2_shortcut_forced(mult, tune):
     """Level-2 up vertices resolved against adj(root) (probing the sorted rows)
     whenever the root's row is cached, on hub-heavy and mesh graphs."""
-    monkeypatch.setenv("DBC_LEAN_SHORT", mult)
+    tune["lean_short"] = int(mult)
     for name in ("rmat10", "rmat14", "delaunay12u"):
         wl = W.make_workload(name, insertions=60)
         ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
@@ -852,3 +863,87 @@ def test_lean_single_edge_calls_match_batch_kernel():
     for (d0, s0), (d1, s1) in zip(outs[0][:-1], outs[1][:-1]):
         assert np.array_equal(d0, d1) and np.array_equal(s0, s1)
     assert_bc(outs[0][-1], outs[1][-1])
+
+
+# ------------------------------------------------ DBC_FLAG_PULL_DELTA (bitwise delta) ----
+def _bitwise_state(dbc, ref_out, k, what):
+    bc_ref, d_ref, s_ref, dl_ref = ref_out
+    for slot in range(k):
+        d, s, dl = dbc.get_root_state(slot)
+        assert np.array_equal(d, d_ref[slot]), f"{what}: d slot {slot}"
+        assert np.array_equal(s.view(np.int64), s_ref[slot].view(np.int64)), f"{what}: sigma slot {slot}"
+        bad = np.nonzero(dl.view(np.int64) != dl_ref[slot].view(np.int64))[0]
+        assert bad.size == 0, f"{what}: delta slot {slot} at {bad[:4]}: {dl[bad[:4]]} vs {dl_ref[slot][bad[:4]]}"
+
+
+@pytest.mark.parametrize("name", ["karate", "rmat10", "delaunay12u", "grid60", "multi"])
+def test_pull_delta_mode_is_bitwise(name):
+    """DBC_FLAG_PULL_DELTA + DBC_FLAG_EXACT_BC at world 1 (SURVEY.md Sec. 8(c)
+    items 14-15): every touched vertex pulls delta in canonical order, so d,
+    sigma, delta AND BC are bit-identical to the oracle -- after the static pass
+    and after insertion batches (Case 3 heavy streams, sigma > 2^53, several
+    components included)."""
+    from paper_conf_ipps_mclaughlinb14_b200 import FLAG_EXACT_BC, FLAG_PULL_DELTA
+
+    if name == "grid60":
+        g = W.grid_graph(60, 60)
+        roots = np.array([0, 61, 1830, 3599, 29], np.int32)
+        rng = np.random.default_rng(3)
+        pairs = set()
+        while len(pairs) < 30:
+            a, b = (int(x) for x in rng.integers(0, g.n, 2))
+            if a != b and b not in set(g.col[g.row_ptr[a]:g.row_ptr[a + 1]].tolist()):
+                pairs.add((min(a, b), max(a, b)))
+        us = np.array([p[0] for p in pairs], np.int32)
+        vs = np.array([p[1] for p in pairs], np.int32)
+    elif name == "multi":
+        g = W.random_gnm(400, 380, 11)
+        roots = np.arange(0, 400, 9, dtype=np.int32)
+        rng = np.random.default_rng(5)
+        eu, ev = W.edges_of(g)
+        existing = set(zip(eu.tolist(), ev.tolist()))
+        pairs = []
+        while len(pairs) < 60:
+            a, b = sorted(int(x) for x in rng.integers(0, g.n, 2))
+            if a != b and (a, b) not in existing and (a, b) not in pairs:
+                pairs.append((a, b))
+        us = np.array([p[0] for p in pairs], np.int32)
+        vs = np.array([p[1] for p in pairs], np.int32)
+    else:
+        wl = W.make_workload(name)
+        g, roots, us, vs = wl.graph, wl.roots, wl.ins_u, wl.ins_v
+    ref = oracle.NaiveDynamicBC(g, roots)
+    with _dbc(g, roots, flags=FLAG_PULL_DELTA | FLAG_EXACT_BC) as dbc:
+        dbc.static_compute()
+        out = ref.compute()
+        _bitwise_state(dbc, out, roots.size, "static")
+        assert np.array_equal(dbc.get_bc().view(np.int64), out[0].view(np.int64))
+        half = us.size // 2
+        for sl in (slice(0, half), slice(half, None)):
+            dbc.insert_edges(us[sl], vs[sl])
+            for u, v in zip(us[sl], vs[sl]):
+                ref.insert(u, v)
+            out = ref.compute()
+            _bitwise_state(dbc, out, roots.size, f"after {sl.stop}")
+            assert np.array_equal(dbc.get_bc().view(np.int64), out[0].view(np.int64)), "BC not bitwise"
+    # without the rebase: BC incremental (within the north star's tolerance), delta still bitwise
+    ref2 = oracle.NaiveDynamicBC(g, roots)
+    with _dbc(g, roots, flags=FLAG_PULL_DELTA) as dbc:
+        dbc.static_compute()
+        dbc.insert_edges(us, vs)
+        for u, v in zip(us, vs):
+            ref2.insert(u, v)
+        out = ref2.compute()
+        _bitwise_state(dbc, out, roots.size, "incremental BC")
+        assert_bc(dbc.get_bc(), out[0])
+
+
+def test_pull_delta_rejects_deletions():
+    from paper_conf_ipps_mclaughlinb14_b200 import FLAG_PULL_DELTA, DBCError
+
+    g = W.cycle_graph(8)
+    with _dbc(g, np.array([0, 3], np.int32), flags=FLAG_PULL_DELTA) as dbc:
+        dbc.static_compute()
+        with pytest.raises(DBCError) as e:
+            dbc.delete_edges([0], [1])
+        assert e.value.name == "DBC_EINVAL"

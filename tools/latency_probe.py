@@ -1,5 +1,7 @@
 """Per-insertion latency probe (diagnostic): one-job-per-insertion batches,
-Mode S launches and single-edge calls on one config, for several CTA widths.
+Mode S launches and single-edge calls on one config, for several launch
+configurations (variants: comma-separated dbc_tuning fields, e.g.
+lean_block=512,disable=8; "default" = automatic).
 
     python tools/latency_probe.py [config] [variants...]   -> JSON lines
 """
@@ -26,18 +28,9 @@ stream = torch.cuda.Stream()
 torch.cuda.set_stream(stream)
 
 
-def ctx(flags, env):
-    old = {k: os.environ.get(k) for k in env}
-    os.environ.update(env)
-    try:
-        d = DynamicBC(g.n, g.row_ptr, g.col, wl.roots, flags=flags | FLAG_TIMING, stream=stream.cuda_stream,
-                      edge_capacity=NB + NS + N1 + 200)
-    finally:
-        for k, v in old.items():
-            if v is None:
-                os.environ.pop(k, None)
-            else:
-                os.environ[k] = v
+def ctx(flags, tuning):
+    d = DynamicBC(g.n, g.row_ptr, g.col, wl.roots, flags=flags | FLAG_TIMING, stream=stream.cuda_stream,
+                  edge_capacity=NB + NS + N1 + 200, tuning=tuning or None)
     d.static_compute()
     d.synchronize()
     return d
@@ -55,11 +48,11 @@ def dev_time(fn):
 
 
 for var in variants:
-    env = {}
+    env = {}  # dbc_tuning fields, e.g. lean_block=512,disable=8
     if var != "default":
         for kv in var.split(","):
             k, v = kv.split("=")
-            env[k] = v
+            env[k] = float(v) if k == "heavy_factor" else int(v)
     res = {"variant": var}
     u, v = wl.ins_u, wl.ins_v
     # one job per (root, insertion): 100 warm-up + a 1000 batch
