@@ -10,8 +10,10 @@ generated graph, the static state is built, and the removed edges are
 reinserted one at a time, B per batch.
 
     python bench.py [--gpus N --steps K --warmup W --config rmat16 --batch 1000]
-    torchrun --nproc-per-node N bench.py --gpus N ...   (roots sharded slot % N)
-    python bench.py --impl reference ...                (the CPU oracle arm)
+    torchrun --nproc-per-node N bench.py --gpus N ...   (roots sharded slot % N; the
+        library's own NCCL communicator all-reduces BC at the end of every batch;
+        default config kron20 at N = 2, 4 and kron22 at N = 8)
+    python bench.py --impl reference ...                (the CPU oracle arm, same workload)
 
 Prints ONE JSON line on rank 0.
 """
@@ -51,7 +53,9 @@ def parse():
     p.add_argument("--steps", type=int, default=5)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    p.add_argument("--config", default="rmat16", choices=sorted(W.CONFIGS))
+    p.add_argument("--config", default=None, choices=sorted(W.CONFIGS),
+                   help="default: rmat16 (BASELINE configs[1]) on 1 GPU, kron20 (configs[3]) on 2 or 4, "
+                        "kron22 (configs[4], 4,096 roots) on 8")
     p.add_argument("--batch", type=int, default=0, help="insertions per step (default: the config's)")
     p.add_argument("--roots", type=int, default=0, help="override k")
     p.add_argument("--mode", default="A", choices=["A", "S"])
@@ -62,12 +66,38 @@ def parse():
                    help="headline run with DBC_FLAG_NO_MERGE (one job per (root, insertion))")
     p.add_argument("--no-deletions", action="store_true", help="skip the edge-deletion side measurement")
     p.add_argument("--no-per-insertion", action="store_true",
-                   help="skip the side measurement with DBC_FLAG_NO_MERGE")
+                   help="skip the per-insertion side measurements (one job per insertion, Mode S, Table III)")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-budget-s", type=float, default=12.0)
+    p.add_argument("--side-insertions", type=int, default=1000,
+                   help="bound on the insertions of each side measurement")
     p.add_argument("--shard", default="", help="R/N: run rank R's root shard of an N-GPU job on this "
                    "single GPU (per-GPU view of configs that need N GPUs, e.g. kron22 on 8)")
-    return p.parse_args()
+    a = p.parse_args()
+    if a.config is None:
+        world = int(os.environ.get("WORLD_SIZE", str(a.gpus)))
+        a.config = "rmat16" if world <= 1 else ("kron22" if world >= 8 else "kron20")
+    return a
+
+
+METRIC = "edge insertions/sec"
+
+
+def n_batches(args, B):
+    """Insertion batches both arms build the workload for (same graph: the
+    remove-then-reinsert protocol removes B x n_batches edges)."""
+    return args.warmup + args.steps + (0 if args.no_e2e else args.warmup + args.steps)
+
+
+def cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for ln in f:
+                if ln.startswith("model name"):
+                    return ln.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
 
 
 # ----------------------------------------------------------------- clocks ----
@@ -151,26 +181,36 @@ def ncu_traffic(config, batch, mode, launches_per_batch):
 
 # ----------------------------------------------------------- CPU baseline ----
 def cpu_baseline(wl, k, budget_s):
-    """The oracle as it stands (single thread): the naive rule costs one k-root
-    recompute per insertion; time it on a bounded root sample and scale to k."""
+    """The oracle as it stands timed on this host (a reported baseline, not the
+    target): the naive rule costs one k-root recompute per insertion.  (ii) the
+    root-parallel leg on every host core (oracle.brandes_parallel, bit-identical
+    to the single-thread oracle) is the value; (i) the single-thread oracle
+    ("single-threaded CPU experiments") is reported beside it.  Both on a
+    bounded root sample of the same workload, scaled linearly to k."""
     import oracle
 
     g = wl.graph
-    r = 1
-    t_root = None
-    while True:
-        roots = wl.roots[:r]
-        t0 = time.perf_counter()
-        oracle.brandes(g.n, g.row_ptr, g.col, roots, want_state=False)
-        dt = time.perf_counter() - t0
-        t_root = dt / r
-        if dt > budget_s / 3 or r >= k:
-            break
-        r = min(k, max(r * 2, int(r * (budget_s / 3) / max(dt, 1e-6))))
-    per_ins = t_root * k
-    return {"value": 1.0 / per_ins, "unit": "insertions/s", "cores": 1, "kind": "oracle",
-            "sample": f"naive rule (recompute all k={k} roots per insertion): {r} of {k} roots "
-                      f"recomputed single-threaded, {t_root * 1e3:.2f} ms/root, scaled linearly to k"}
+    T = oracle.host_threads()
+    t0 = time.perf_counter()
+    oracle.brandes(g.n, g.row_ptr, g.col, wl.roots[:1], want_state=False)
+    t1 = max(time.perf_counter() - t0, 1e-6)
+    r = int(max(T, min(k, T * max(1, int((budget_s / 2) / t1)))))  # ~budget/2 of all-core work
+    r = min(r, k)
+    t0 = time.perf_counter()
+    oracle.brandes_parallel(g.n, g.row_ptr, g.col, wl.roots[:r], threads=T)
+    tp = time.perf_counter() - t0
+    per_ins = tp / r * k
+    r1 = int(max(1, min(k, (budget_s / 4) / t1)))
+    t0 = time.perf_counter()
+    oracle.brandes(g.n, g.row_ptr, g.col, wl.roots[:r1], want_state=False)
+    ts = (time.perf_counter() - t0) / r1 * k
+    return {"value": 1.0 / per_ins, "unit": "insertions/s", "cores": T, "kind": "oracle",
+            "cpu_model": cpu_model(), "nproc": os.cpu_count(),
+            "sample": f"naive rule (recompute all k={k} roots per insertion): {r} of {k} roots recomputed "
+                      f"root-parallel on {T} threads ({tp / r * 1e3:.2f} ms/root), scaled linearly to k",
+            "single_thread": {"value": 1.0 / ts, "cores": 1,
+                              "sample": f"{r1} of {k} roots single-threaded ({ts / k * 1e3:.2f} ms/root), "
+                                        f"scaled to k"}}
 
 
 def cpu_dynamic(wl, k, budget_s):
@@ -201,6 +241,10 @@ def cpu_dynamic(wl, k, budget_s):
 
 # -------------------------------------------------------------- reference ----
 def run_reference(args):
+    """The reference arm of this tier: the CPU oracle's naive rule (recompute
+    every root after each insertion) on the SAME workload our arm builds (same
+    config, seed, graph and stream), on every host core.  Each step times one
+    insertion's recompute over a bounded root sample and scales linearly to k."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
@@ -209,35 +253,40 @@ def run_reference(args):
     cfg = W.CONFIGS[args.config]
     B = args.batch or cfg["insertions"]
     k = args.roots or cfg["k"]
-    steps = args.warmup + args.steps
-    wl = W.make_workload(args.config, seed=args.seed, insertions=max(steps, 1), k=k)
+    wl = W.make_workload(args.config, seed=args.seed, insertions=B * n_batches(args, B), k=k)
     g = wl.graph
-    # bounded sample: r roots per naive-rule insertion, ~1-2 s per step
+    T = oracle.host_threads()
     t0 = time.perf_counter()
     oracle.brandes(g.n, g.row_ptr, g.col, wl.roots[:1], want_state=False)
     t_root = max(time.perf_counter() - t0, 1e-6)
-    r = int(max(1, min(k, 1.5 / t_root)))
+    r = int(max(1, min(k, T * max(1, int(1.0 / t_root)))))  # ~1 s of all-core work per step
     dyn = oracle.NaiveDynamicBC(g, wl.roots[:r])
     times = []
-    for i in range(steps):
+    for i in range(args.warmup + args.steps):
         dyn.insert(wl.ins_u[i], wl.ins_v[i])
+        rp, col = dyn.csr()
         t0 = time.perf_counter()
-        dyn.compute(want_state=False)
+        oracle.brandes_parallel(g.n, rp, col, wl.roots[:r], threads=T)
         dt = time.perf_counter() - t0
         if i >= args.warmup:
             times.append(dt)
     per_ins = (sum(times) / len(times)) * k / r
     value = 1.0 / per_ins
     line = {
-        "impl": "reference", "metric": "edge insertions/sec", "value": value,
+        "impl": "reference", "metric": METRIC, "value": value,
         "unit": "insertions/s", "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": per_ins * B * 1e3, "higher_is_better": True, "scaling": "strong",
         "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": args.config, "graph": GRAPH_DESC.get(args.config, args.config),
-                   "n": g.n, "m": g.m, "k": k, "batch": B, "seed": args.seed},
-        "cpu_baseline": {"value": value, "unit": "insertions/s", "cores": 1, "kind": "oracle",
-                         "sample": f"each step: one naive-rule insertion (recompute) over {r} of {k} "
-                                   f"roots, single thread, scaled linearly to k"},
+                   "n": g.n, "m": g.m, "k": k, "batch": B, "seed": args.seed,
+                   "protocol": "remove-then-reinsert (P:440)" if cfg["mode"] == "reinsert" else "uniform non-edges",
+                   "timing": "host wall clock of the oracle's recompute",
+                   "ms_per_step_extrapolated": f"one insertion timed per step on {r} of {k} roots, scaled to k "
+                                               f"roots and to the {B}-insertion batch"},
+        "cpu_baseline": {"value": value, "unit": "insertions/s", "cores": T, "kind": "oracle",
+                         "cpu_model": cpu_model(), "nproc": os.cpu_count(),
+                         "sample": f"each step: one naive-rule insertion (recompute) over {r} of {k} roots, "
+                                   f"root-parallel on {T} threads, scaled linearly to k"},
         "e2e": {"value": value, "unit": "insertions/s", "h2d_bytes_per_step": 0,
                 "d2h_bytes_per_step": 0},
     }
@@ -258,8 +307,14 @@ def run_ours(args):
         if world > 1:
             raise SystemExit("--shard emulates one rank on one GPU; do not combine with torchrun")
         shard_rank, shard_world = (int(x) for x in args.shard.split("/"))
+    nccl_log = None
     if world > 1:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        # NCCL's communicator lines (version, transports, NVLS) into a per-rank file
+        nccl_log = os.path.join("/tmp", f"dbc_nccl.{os.getpid()}.log")
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+        os.environ.setdefault("NCCL_DEBUG_FILE", nccl_log)
         torch.cuda.set_device(local)
         dist.init_process_group("nccl", device_id=torch.device(f"cuda:{local}"))
     else:
@@ -267,22 +322,32 @@ def run_ours(args):
     dev = torch.cuda.current_device()
 
     from paper_conf_ipps_mclaughlinb14_b200 import (FLAG_MODE_S, FLAG_NO_MERGE, FLAG_TIMING,
-                                                    DynamicBC, allreduce_bc)
+                                                    DynamicBC, nccl_unique_id)
 
     cfg = W.CONFIGS[args.config]
     B = args.batch or cfg["insertions"]
     k = args.roots or cfg["k"]
     Wm, K = args.warmup, args.steps
     e2e_steps = 0 if args.no_e2e else (Wm + K)
-    nb = Wm + K + e2e_steps
+    nb = n_batches(args, B)
     wl = W.make_workload(args.config, seed=args.seed, insertions=B * nb, k=k)
     g = wl.graph
     flags = FLAG_TIMING | (FLAG_MODE_S if args.mode == "S" else 0) | (FLAG_NO_MERGE if args.no_merge else 0)
     stream = torch.cuda.Stream(device=dev)  # the library and the timing events share it
     torch.cuda.set_stream(stream)
-    dbc = DynamicBC(g.n, g.row_ptr, g.col, wl.roots, device=dev, rank=shard_rank, world=shard_world,
-                    workers=args.workers, edge_capacity=B * nb, flags=flags,
-                    stream=stream.cuda_stream)
+    uid = None
+    if world > 1:  # the library's own NCCL communicator for the BC all-reduce (opt.nccl_id)
+        obj = [nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        uid = obj[0]
+    side_ok = world == 1  # side measurements on one GPU only (scaling runs stay short)
+
+    def make(fl):
+        return DynamicBC(g.n, g.row_ptr, g.col, wl.roots, device=dev, rank=shard_rank, world=shard_world,
+                         workers=args.workers, edge_capacity=B * nb, flags=fl, stream=stream.cuda_stream,
+                         nccl_id=uid)
+
+    dbc = make(flags)
 
     def max_over_ranks(x):
         if world == 1:
@@ -309,8 +374,13 @@ def run_ours(args):
     def batch(i):
         return ins_u[i * B:(i + 1) * B], ins_v[i * B:(i + 1) * B]
 
+    def step(d, i):
+        d.insert_edges(*batch(i))
+        if world > 1:  # the end-of-batch BC all-reduce over NVLink, inside T_dev
+            d.bc_device_ptr()
+
     for i in range(Wm):
-        dbc.insert_edges(*batch(i))
+        step(dbc, i)
     dbc.synchronize()
     dbc.reset_timings()
 
@@ -322,7 +392,7 @@ def run_ours(args):
     ev1 = torch.cuda.Event(enable_timing=True)
     ev0.record(stream)
     for i in range(Wm, Wm + K):
-        dbc.insert_edges(*batch(i))
+        step(dbc, i)
     ev1.record(stream)
     torch.cuda.synchronize()
     barrier()
@@ -338,8 +408,9 @@ def run_ours(args):
     launch_ms = upd_ms / launches
     achieved = bytes_per_launch / (launch_ms / 1e3) / 1e9 if launch_ms > 0 else 0.0
     peak, peak_src = hbm_peak()
+    gpu_launches = int(tm["kernel_launches_total"])
 
-    # end to end through the public host API: pinned H2D of each batch + D2H of BC
+    # end to end through the public host API: pinned H2D of each batch + D2H of the (global) BC
     e2e = None
     case_mix = None
     if e2e_steps:
@@ -358,10 +429,7 @@ def run_ours(args):
             torch.cuda.synchronize()
             t0 = time.perf_counter()
             st = dbc.insert_edges(u, v, stats=(j < Wm))
-            if world > 1:
-                outn[:] = allreduce_bc(dbc)
-            else:
-                dbc.get_bc(out=outn)
+            dbc.get_bc(out=outn)  # global BC (NCCL all-reduce inside at N > 1)
             dt = time.perf_counter() - t0
             if j >= Wm:
                 t_e2e += dt
@@ -374,9 +442,7 @@ def run_ours(args):
         ncase = max(tot["case1"] + tot["case2"] + tot["case3"], 1)
         case_mix = {"case1": tot["case1"] / ncase, "case2": tot["case2"] / ncase,
                     "case3": tot["case3"] / ncase,
-                    "touched_per_working_root": tot["touched"] / max(tot["case2"] + tot["case3"], 1),
-                    "scanned_per_working_root": tot["edges_scanned"] / max(tot["case2"] + tot["case3"], 1),
-                    "sample": f"{Wm} untimed e2e batches, this rank's roots"}
+                    "sample": f"{Wm} untimed e2e batches (window-merged jobs), this rank's roots"}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -386,60 +452,114 @@ def run_ours(args):
             cpu = {"value": None, "unit": "insertions/s", "cores": 1, "kind": "oracle",
                    "sample": f"unavailable: {ex}"}
 
-    # side measurement: deletions (decremental update, R20) -- the
-    # edges of the timed batches deleted again, B per step, one job per deletion
-    dels = None
-    if not args.no_deletions:
-        barrier()
-        torch.cuda.synchronize()
-        ev0.record(stream)
-        for i in range(Wm + K - 1, Wm - 1, -1):
-            dbc.delete_edges(wl.ins_u[i * B:(i + 1) * B], wl.ins_v[i * B:(i + 1) * B])
-        ev1.record(stream)
-        torch.cuda.synchronize()
-        barrier()
-        msd = max_over_ranks(ev0.elapsed_time(ev1))
-        dels = {"value": K * B / (msd / 1e3), "unit": "deletions/s", "ms_per_step": msd / K,
-                "what": "the K timed batches deleted again (B per step, newest first), one job per "
-                        "(root, deletion); host-side batch checks inside the timed region"}
+    S = min(args.side_insertions, B)  # side measurements are bounded
 
-    # side measurement: the same batches with one job per (root, insertion)
-    # (DBC_FLAG_NO_MERGE: the paper's one-insertion-at-a-time structure)
-    per_ins = None
-    if not (args.no_per_insertion or args.no_merge or args.mode == "S"):
-        dbc.close()
-        dbc = DynamicBC(g.n, g.row_ptr, g.col, wl.roots, device=dev, rank=shard_rank,
-                        world=shard_world, workers=args.workers, edge_capacity=B * nb,
-                        flags=flags | FLAG_NO_MERGE, stream=stream.cuda_stream)
-        dbc.static_compute()
-        for i in range(Wm):
-            dbc.insert_edges(*batch(i))
-        barrier()
+    # side measurement: deletions (decremental update, R20) -- S edges
+    # of the last timed batch deleted again (newest first), one job per deletion
+    dels = None
+    if side_ok and not args.no_deletions:
+        D = min(S, 200)
+        i = Wm + K - 1
+        du, dv = wl.ins_u[i * B:i * B + D][::-1].copy(), wl.ins_v[i * B:i * B + D][::-1].copy()
         torch.cuda.synchronize()
         ev0.record(stream)
-        for i in range(Wm, Wm + K):
-            dbc.insert_edges(*batch(i))
+        dbc.delete_edges(du, dv)
         ev1.record(stream)
         torch.cuda.synchronize()
-        barrier()
-        ms1 = max_over_ranks(ev0.elapsed_time(ev1))
-        per_ins = {"value": K * B / (ms1 / 1e3), "unit": "insertions/s", "ms_per_step": ms1 / K,
-                   "speedup_vs_static": (static_ms / 1e3) / (ms1 / 1e3 / (K * B)),
-                   "what": "same batches, DBC_FLAG_NO_MERGE: one job per (root, insertion), "
-                           "insertions applied one at a time as in P:440"}
+        msd = ev0.elapsed_time(ev1)
+        dels = {"value": D / (msd / 1e3), "unit": "deletions/s", "deletions": D,
+                "what": f"{D} edges of the last timed batch deleted again (newest first), one job per "
+                        f"(root, deletion); host-side batch checks inside the timed region"}
+    dbc.close()
+
+    # per-insertion side measurements (the paper's structure):
+    # one job per (root, insertion) on the same batches, Mode S launches, and
+    # Table III's single-edge calls -- all on update_lean.cu
+    per_ins = None
+    if side_ok and not (args.no_per_insertion or args.no_merge or args.mode == "S"):
+        per_ins = {}
+        d = make(flags | FLAG_NO_MERGE)
+        d.static_compute()
+        for i in range(min(Wm, 1)):
+            d.insert_edges(*batch(i))
+        d.synchronize()
+        d.reset_timings()
+        i0 = Wm
+        torch.cuda.synchronize()
+        ev0.record(stream)
+        d.insert_edges(ins_u[i0 * B:i0 * B + S], ins_v[i0 * B:i0 * B + S])
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        ms1 = ev0.elapsed_time(ev1)
+        t1 = d.timings()
+        v1 = S / (ms1 / 1e3)
+        l1 = max(t1["update_launches_total"], 1)
+        ach1 = (t1["alg_bytes_total"] / l1) / (t1["update_ms_total"] / l1 / 1e3) / 1e9 if t1["update_ms_total"] else 0
+        per_ins["jobs"] = {"value": v1, "unit": "insertions/s", "insertions": S,
+                           "speedup_vs_static": (static_ms / 1e3) / (ms1 / 1e3 / S),
+                           "roofline": {"bound": "hbm", "achieved": ach1, "peak": peak, "unit": "GB/s",
+                                        "frac": ach1 / peak, "kernel": "lean_kernel"},
+                           "what": "DBC_FLAG_NO_MERGE: one job per (root, insertion), insertions applied one "
+                                   "at a time as in P:440, one launch"}
+        # Mode S: one launch per insertion over all roots
+        NS = min(S, 200)
+        i0 = Wm + 1
+        dS = make(flags | FLAG_MODE_S)
+        dS.static_compute()
+        dS.synchronize()
+        torch.cuda.synchronize()
+        ev0.record(stream)
+        dS.insert_edges(ins_u[i0 * B:i0 * B + NS], ins_v[i0 * B:i0 * B + NS])
+        ev1.record(stream)
+        torch.cuda.synchronize()
+        ms2 = ev0.elapsed_time(ev1)
+        per_ins["mode_s"] = {"value": NS / (ms2 / 1e3), "unit": "insertions/s", "insertions": NS,
+                             "what": "Mode S: one per-insertion kernel launch over all roots per insertion "
+                                     "(P:244-252)"}
+        dS.close()
+        # Table III: single-edge calls, device time of each call's update
+        NT = min(S, 60)
+        per = []
+        for j in range(NT + 3):
+            idx = (Wm + 2) * B + j
+            d.insert_edges(ins_u[idx:idx + 1], ins_v[idx:idx + 1])
+            if j >= 3:
+                per.append(d.timings()["update_ms"])
+        per = np.array(per)
+        per_ins["table3"] = {"calls": NT, "static_ms": static_ms, "fastest_ms": float(per.min()),
+                             "average_ms": float(per.mean()), "slowest_ms": float(per.max()),
+                             "speedup_average": static_ms / float(per.mean()),
+                             "speedup_slowest": static_ms / float(per.max()),
+                             "speedup_fastest": static_ms / float(per.min()),
+                             "what": "device time of the update of single-edge dbc_insert_edges calls (graph "
+                                     "update neglected as in P:440) vs one static recompute over the same roots "
+                                     "(Table III, P:482-514)"}
+        d.close()
 
     cpu_dyn = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         try:
             cpu_dyn = cpu_dynamic(wl, k, args.cpu_budget_s)
-            cpu_dyn["gpu_speedup"] = value / cpu_dyn["value"]
+            ref_v = per_ins["jobs"]["value"] if per_ins else value
+            cpu_dyn["gpu_speedup_per_insertion"] = ref_v / cpu_dyn["value"]
+            cpu_dyn["gpu_speedup_merged"] = value / cpu_dyn["value"]
             cpu_dyn["paper"] = "110x max GPU-over-CPU dynamic on a GTX-class GPU (P:444-478), context only"
         except Exception as ex:
             cpu_dyn = {"value": None, "kind": "cpu_dynamic_alg2", "sample": f"unavailable: {ex}"}
 
+    nccl = None
+    if nccl_log and rank == 0:
+        try:
+            with open(nccl_log) as f:
+                lines = [ln.strip() for ln in f if ("NCCL version" in ln or "NVLS" in ln or "comm " in ln
+                                                      or "Init COMPLETE" in ln)]
+            nccl = {"log": nccl_log, "lines": lines[:8]}
+        except OSError:
+            nccl = {"log": nccl_log, "lines": []}
+
     state_mb = 24.0 * k * g.n / shard_world / 1e6
     line = {
-        "metric": "edge insertions/sec (device-timed)",
+        "metric": METRIC,
         "value": value,
         "unit": "insertions/s",
         "n_gpus": world,
@@ -456,6 +576,8 @@ def run_ours(args):
             "graph": GRAPH_DESC.get(args.config, args.config),
             "n": g.n, "m": g.m, "k": k, "batch": B, "mode": args.mode, "seed": args.seed,
             "protocol": "remove-then-reinsert (P:440)" if cfg["mode"] == "reinsert" else "uniform non-edges",
+            "timing": "device (CUDA events on the library stream), max over ranks"
+                      + ("; the end-of-batch BC all-reduce inside" if world > 1 else ""),
             "l2": f"inputs larger than L2: per-GPU d/sigma/delta state {state_mb:.0f} MB vs 126 MB L2",
             "static_recompute_ms": static_ms,
             "shard": (f"rank {shard_rank} of {shard_world} (roots slot % {shard_world} == {shard_rank}) "
@@ -465,24 +587,25 @@ def run_ours(args):
             "case_mix": case_mix,
             "merge": ("one job per (root, insertion)" if args.no_merge or args.mode == "S" else
                       "window-merged: one job per root per window of insertions (DESIGN.md R18)"),
-            "per_insertion_jobs": per_ins,
+            "per_insertion": per_ins,
             "deletions": dels,
+            "nccl": nccl,
         },
         "roofline": {
             "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
             "frac": achieved / peak, "traffic": ncu_traffic(args.config, B, args.mode, launches / K),
             "kernel": "update_kernel", "peak_source": peak_src,
             "alg_bytes_per_launch": bytes_per_launch, "launch_ms": launch_ms,
+            "byte_model": "SURVEY.md Sec. 8(d), counted per event in the kernel",
             "share_of_step": upd_ms / ms if ms > 0 else None,
             "static_kernel_GBps": (static_bytes / (static_ms / 1e3) / 1e9) if static_ms > 0 else None,
         },
         "cpu_baseline": cpu,
         "cpu_dynamic": cpu_dyn,
         "e2e": e2e,
-        "gpu_launches": int(tm["kernel_launches_total"]),
+        "gpu_launches": gpu_launches,
         "clocks": clk,
     }
-    dbc.close()
     if rank == 0:
         print(json.dumps(line), flush=True)
     if world > 1:

@@ -288,6 +288,12 @@ dbc_status dbc_delete_edges_device(dbc_ctx *c, const int32_t *u_device,
  * (an earlier update overflowed). */
 dbc_status dbc_get_bc(dbc_ctx *c, double *bc);
 
+/* The same global BC left in DEVICE memory (fp64[n], caller's vertex order,
+ * valid until the next call that returns a BC buffer, or destroy); the
+ * all-reduce is enqueued on the context stream (a reduce callback may
+ * synchronise).  A collective call at world > 1.  Errors as dbc_get_bc. */
+dbc_status dbc_get_bc_device(dbc_ctx *c, double **bc_device);
+
 /* Device pointer to this rank's BC partial, fp64[n] in the caller's vertex
  * order (a copy refreshed by this call, valid until the next call or destroy);
  * for a sum all-reduce across ranks.  Asynchronous on the context stream. */

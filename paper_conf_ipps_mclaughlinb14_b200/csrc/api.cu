@@ -1335,8 +1335,8 @@ extern "C" dbc_status dbc_get_bc_partial_device(dbc_ctx *c, double **p) {
     return DBC_OK;
 }
 
-extern "C" dbc_status dbc_get_bc(dbc_ctx *c, double *bc) {
-    if (!c || !bc) return DBC_EINVAL;
+extern "C" dbc_status dbc_get_bc_device(dbc_ctx *c, double **out) {
+    if (!c || !out) return DBC_EINVAL;
     if (!c->have_state) return fail(c, DBC_ESTATE, "no state: call dbc_static_compute first");
     if (c->world > 1 && !c->comm && !c->reduce)
         return fail(c, DBC_ESTATE, "world %d: global BC needs opt.nccl_id or opt.reduce "
@@ -1353,6 +1353,14 @@ extern "C" dbc_status dbc_get_bc(dbc_ctx *c, double *bc) {
         const int r = c->reduce(p, (int64_t)c->n, (void *)c->stream, c->reduce_user);
         if (r != 0) return fail(c, DBC_ENCCL, "reduce callback returned %d", r);
     }
+    *out = p;
+    return DBC_OK;
+}
+
+extern "C" dbc_status dbc_get_bc(dbc_ctx *c, double *bc) {
+    if (!c || !bc) return DBC_EINVAL;
+    double *p = nullptr;
+    TRY(dbc_get_bc_device(c, &p));
     CK(cudaMemcpyAsync(bc, p, sizeof(double) * c->n, cudaMemcpyDeviceToHost, c->stream));
     return check_err(c);
 }

@@ -87,7 +87,7 @@ __device__ __forceinline__ void help_run_block(const ChunkSmem &M, int e0, int e
     flat_entries<kCG, false>(
         M.off, cx.cnt, e1, colf, st, mark, [&](int dp) { return dp == cx.l - 1; }, nullptr,
         [&](int t, int pp, int dp, double2 q, uint32_t mp) -> double {
-            bytes += 8;
+            if (M.meta[t] & kMetaUp) bytes += 8;  // D rows: counted by their C1 pull
             help_push_entry(g, M, t, pp, dp, q.x, mp, cx, mark, dacc, gU, gapp, bytes);
             return 0.0;
         },
@@ -310,7 +310,7 @@ __device__ __forceinline__ void rem_range(const RemCtx &c, BigSmem &S, int *s_ol
             const double coef = 1.0 + c.st.sd[w].y;  // delta still old
             row_walk(c.g, c.st, nullptr, r, [&](int dx) { return dx == od - 1; },
                      [&](int x, int dx, double2, uint32_t) { rem_visit(c, w, od, osig, coef, x, dx, bytes); });
-            bytes += 16 + 8ull * (r.y - r.x);
+            bytes += 8 + 8ull * (r.y - r.x);
             scanned += r.y - r.x;
         },
         [&](int q) { Bq[atomicAdd(nbig, 1)] = i0 + q; });
@@ -323,7 +323,7 @@ __device__ __forceinline__ void rem_range(const RemCtx &c, BigSmem &S, int *s_ol
             const int i = S.idx[tid];
             S.c0[tid] = c.Dsig[i];
             s_old[tid] = c.Dold[i] & kOldMask;  // old level of each row
-            bytes += 16;
+            bytes += 8;
         }
         __syncthreads();
         big_entries(S, c.g, c.st, [](int) { return true; }, [&](int t, int x, int dx, double2) {
@@ -548,7 +548,7 @@ __device__ __forceinline__ void up_block(const UpCtx &c, int q0, int q1, uint32_
             meta = (((od & kOldMask) == l) ? kMetaNotPulled : 0) | ((od < 0) ? kMetaExt : 0) |
                    ((ldg_i(c.g.rp + x) < 0) ? kMetaNew : 0);
             r = row_of(c.g, x, c.lim);
-            bytes += 8 + 16 + 8 + 4;
+            bytes += 8 + 8;
         } else {
             const int qi = q - c.nDl;
             x = -1;
@@ -570,7 +570,7 @@ __device__ __forceinline__ void up_block(const UpCtx &c, int q0, int q1, uint32_
             c0 = sx;
             c1 = gx;
             c2 = odl;
-            bytes += 24 + (usemask ? 4 : 0);
+            bytes += 8 + (usemask ? 4 : 0);
             r = (push && gx != 0.0) ? rr : make_int2(0, 0);
             if (gx == 0.0) mk = 0u;
         }
@@ -648,18 +648,18 @@ __device__ __forceinline__ void up_block(const UpCtx &c, int q0, int q1, uint32_
                              up_claim(c, pp, mp);
                          });
                 scanned += r.y - r.x;
-                bytes += 8u * (r.y - r.x);
+                (void)0;  // the second walk of the row: one pass in the byte model
             }
             c.st.sd[x].y = dn;  // d_finish
             atomicAdd(c.bc + x, dn - c1);
-            bytes += 40;
+            bytes += 8 + 16;  // delta write, BC RMW
             continue;
         }
         // up_finish
         c.dacc[x] = 0.0;
         c.st.sd[x].y = c2 + c1;
         atomicAdd(c.bc + x, c1);
-        bytes += 48;
+        bytes += 16 + 16;  // delta RMW, BC RMW
     }
     __syncthreads();
 }
@@ -1686,7 +1686,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                         dacc[x] = 0.0;
                         st.sd[x].y = odel + gx;
                         atomicAdd(a.bc + x, gx);
-                        st_bytes += 8 + 8 + 16 + 16;
+                        st_bytes += 16 + 16;  // delta RMW, BC RMW (40 B per up vertex)
                     };
                     // down vertex x: pull delta (Eq. (2)), then push new-minus-old contributions
                     auto dpull_visit = [&](double sx, int dy, double sy, double dly) -> double {
@@ -1708,7 +1708,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                     auto d_finish = [&](int x, double dn, double odel) {
                         st.sd[x].y = dn;
                         atomicAdd(a.bc + x, dn - odel);
-                        st_bytes += 8 + 16 + 16;
+                        st_bytes += 8 + 16;  // delta write, BC RMW
                     };
 
                     int b0 = 0, b1 = 0;
@@ -1750,7 +1750,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                             meta = (((od & kOldMask) == l) ? kMetaNotPulled : 0) | ((od < 0) ? kMetaExt : 0) |
                                    ((ldg_i(g.rp + x) < 0) ? kMetaNew : 0);
                             r = row_of(g, x, lim);
-                            st_bytes += 8 + 16 + 8 + 4;
+                            st_bytes += 8 + 8;  // row bounds, delta read
                             return true;
                         }
                         const int qi = q - nDl;
@@ -1774,7 +1774,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                         c0 = sx;
                         c1 = gx;
                         c2 = odl;
-                        st_bytes += 24 + (usemask ? 4 : 0);
+                        st_bytes += 8 + (usemask ? 4 : 0);  // Ddelta read
                         r = (push && gx != 0.0) ? rr : make_int2(0, 0);
                         if (gx == 0.0) mk = 0u;
                         return true;
@@ -1839,7 +1839,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                                  dpush_visit(x, c0, dn, c1, c2, meta, pp, q.x, mp);
                                          });
                                 sc_dpush += r.y - r.x;
-                                st_bytes += 8ull * (r.y - r.x);
+                                (void)0;  // second walk of the same row: one pass in the byte model
                             }
                             d_finish(x, dn, c1);
                         }
@@ -2227,9 +2227,9 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                     [&](int t, int pp, int dp, double2 q, uint32_t mp) -> double {
                                         const double sp = q.x;
                                         (l == 2 ? sc_up2 : sc_up3)++;
-                                        st_bytes += 8;
-                                        if (dp != l - 1) return 0.0;
                                         const int meta = I.meta[t];
+                                        if (meta & kMetaUp) st_bytes += 8;  // D rows: counted by their C1 pull
+                                        if (dp != l - 1) return 0.0;
                                         if (meta & kMetaUp)
                                             up_visit(I.c1[t], I.c0[t], pp, sp, mp);
                                         else

@@ -114,6 +114,7 @@ SIGNATURES = {
     "dbc_delete_edges_device": (ctypes.c_int, [_P, _P, _P, ctypes.c_int64, _P]),
     "dbc_get_bc": (ctypes.c_int, [_P, _P]),
     "dbc_get_bc_partial_device": (ctypes.c_int, [_P, _P]),
+    "dbc_get_bc_device": (ctypes.c_int, [_P, _P]),
     "dbc_get_root_state": (ctypes.c_int, [_P, ctypes.c_int32, _P, _P, _P]),
     "dbc_num_local_roots": (ctypes.c_int, [_P, _P]),
     "dbc_synchronize": (ctypes.c_int, [_P]),
@@ -301,6 +302,13 @@ class DynamicBC:
         ptr = self.bc_partial_device_ptr()
         self.synchronize()
         return _wrap_device_f64(ptr, self.n, self.device).cpu().numpy().copy()
+
+    def bc_device_ptr(self) -> int:
+        """dbc_get_bc_device: the global BC in device memory (all-reduced across
+        ranks on the context stream); a collective call at world > 1."""
+        p = ctypes.c_void_p()
+        _check(self._ctx, self._lib.dbc_get_bc_device(self._ctx, ctypes.byref(p)))
+        return int(p.value)
 
     def bc_partial_device_ptr(self) -> int:
         p = ctypes.c_void_p()
