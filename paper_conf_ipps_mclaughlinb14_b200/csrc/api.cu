@@ -566,7 +566,8 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     // worth it while the batch time is the slowest root chain (few roots per
     // worker: R-MAT 16 +8%), not when every worker has many roots (Kronecker 20)
     if (c->wide_inlane < 0) c->wide_inlane = c->k_loc <= 2 * std::max(c->workers, 1) ? 64 : 16;
-    c->sworkers = std::max(0, std::min({opt.workers ? opt.workers : (c->sblock == 128 ? 4 : (c->sblock >= 512 ? 1 : 2)) * c->nsm,
+    const int spb = c->sblock == 128 ? 4 : (c->sblock == 256 ? 2 : 1);  // static CTAs per SM
+    c->sworkers = std::max(0, std::min({opt.workers ? opt.workers : spb * c->nsm,
                                         c->k_loc, fit}));
     c->hblock = c->block == 128 ? 256 : (c->block == 256 ? 512 : 1024);
     // only hub-heavy graphs (256-thread build) have step-bound slow roots

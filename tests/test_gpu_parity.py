@@ -60,7 +60,53 @@ def check_all(dbc, ref_out, k):
 
 
 # ---------------------------------------------------------------- static ----
+def _big_sigma_hub(fan=5000):
+    """A hub whose row (> 4,096 entries: a single-row chunk, row sums by shared
+    atomics) sums predecessors with sigma ~ 2^56 of two different values, so the
+    result above 2^53 depends on the order: it must be the canonical one."""
+    eu, ev = [], []
+    nxt = [1]
+
+    def new():
+        nxt[0] += 1
+        return nxt[0] - 1
+
+    def diamonds(src, k):  # k diamonds: sigma doubles per diamond
+        cur = src
+        for _ in range(k):
+            a, b, z = new(), new(), new()
+            eu.extend([cur, cur, a, b])
+            ev.extend([a, b, z, z])
+            cur = z
+        return cur
+
+    def path(src, k):
+        cur = src
+        for _ in range(k):
+            x = new()
+            eu.append(cur)
+            ev.append(x)
+            cur = x
+        return cur
+
+    s = 0
+    t = diamonds(s, 56)                 # level 112, sigma 2^56
+    t2 = path(diamonds(s, 5), 102)      # level 112, sigma 2^5
+    hub = new()
+    for i in range(fan):
+        a = new()
+        eu.extend([t, a])
+        ev.extend([a, hub])
+        if i % 2 == 0:
+            eu.append(t2)
+            ev.append(a)
+    g = W.csr_from_edges(nxt[0], eu, ev)
+    return g, np.array([0, 1, hub], np.int32)
+
+
 STATIC_CASES = {
+    "big_sigma_hub": _big_sigma_hub,
+    "star6k": lambda: (W.star_graph(6000), np.array([0, 1, 5999])),
     "karate": lambda: (W.karate(), np.arange(34)),
     "path9": lambda: (W.path_graph(9), np.arange(9)),
     "star12": lambda: (W.star_graph(12), np.arange(12)),
@@ -85,7 +131,7 @@ def test_static_matches_oracle(name):
 
 
 @pytest.mark.parametrize("sblock", ["128", "256", "512"])
-@pytest.mark.parametrize("name", ["grid_big_sigma", "disconnected", "rmat10", "delaunay12", "hub"])
+@pytest.mark.parametrize("name", ["grid_big_sigma", "disconnected", "rmat10", "delaunay12", "hub", "big_sigma_hub"])
 def test_static_other_widths_match_oracle(name, sblock, tune):
     """The static kernel at the non-default CTA widths (tuning.static_block; default 1024)."""
     tune["static_block"] = int(sblock)
