@@ -41,6 +41,7 @@ GRAPH_DESC = {
     "karate": "Zachary karate club (34 vertices, 78 edges)",
     "rmat16": "R-MAT/Graph500 Kronecker scale 16 edgefactor 8 (A,B,C=.57,.19,.19), undirected",
     "delaunay18": "Delaunay triangulation of 2^18 uniform points",
+    "delaunay18u": "Delaunay triangulation of 2^18 uniform points, uniform random non-edge insertions (stress)",
     "kron20": "Kronecker scale 20 edgefactor 16",
     "kron22": "Kronecker scale 22 edgefactor 16",
     "smallworld": "Watts-Strogatz n=100000 k=10 p=0.1",

@@ -1,17 +1,21 @@
 #!/bin/bash
-# Round evidence: default bench line, launch list, ncu captures, per-config lines, paper figures.
+# Round evidence: GPU tests, smoke, bench lines per config, reference arm, launch
+# list, ncu captures of the three kernel families, paper figures.
 O=gpurun_out/${FINAL_DIR:-final}; mkdir -p $O
-timeout 1500 python -m pytest tests -m gpu -q > $O/gpu_tests.log 2>&1; echo "rc=$?" >> $O/gpu_tests.log
+timeout 1500 python -m pytest tests -m gpu -q --durations=15 > $O/gpu_tests.log 2>&1; echo "rc=$?" >> $O/gpu_tests.log
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; echo "rc=$?" >> $O/smoke.log
-timeout 600 python bench.py > $O/bench_rmat16.json 2> $O/bench_rmat16.err
-timeout 600 python bench.py --impl reference > $O/bench_reference.json 2> $O/bench_reference.err
+timeout 900 python bench.py --steps 20 --warmup 5 > $O/bench_rmat16.json 2> $O/bench_rmat16.err
+timeout 900 python bench.py --impl reference --steps 20 --warmup 5 > $O/bench_reference.json 2> $O/bench_reference.err
 B="python bench.py --no-cpu-baseline"
 timeout 900 $B --config delaunay18 > $O/bench_delaunay18.json 2> $O/bench_delaunay18.err
+timeout 900 $B --config delaunay18u > $O/bench_delaunay18u.json 2> $O/bench_delaunay18u.err
 timeout 600 $B --config smallworld > $O/bench_smallworld.json 2> $O/bench_smallworld.err
-timeout 1200 $B --config kron20 --steps 3 --warmup 3 --no-e2e --no-per-insertion > $O/bench_kron20.json 2> $O/bench_kron20.err
+timeout 1500 $B --config kron20 --steps 3 --warmup 3 --no-e2e > $O/bench_kron20.json 2> $O/bench_kron20.err
 timeout 1500 $B --config kron22 --shard 0/8 --steps 2 --warmup 3 --no-e2e --no-per-insertion --no-deletions > $O/bench_kron22_shard0of8.json 2> $O/bench_kron22.err
-timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches.csv python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-per-insertion --no-e2e --no-deletions > $O/ncu_launches.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:update --launch-skip 3 --launch-count 1 -o $O/update_full python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-per-insertion --no-e2e --no-deletions > $O/ncu_update.log 2>&1
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:static --launch-count 1 -o $O/static_full python bench.py --steps 1 --warmup 3 --no-cpu-baseline --no-per-insertion --no-e2e --no-deletions > $O/ncu_static.log 2>&1
+N="python bench.py --no-cpu-baseline --no-per-insertion --no-e2e --no-deletions"
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches.csv $N --steps 2 --warmup 3 > $O/ncu_launches.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:update_kernel --launch-skip 3 --launch-count 1 -o $O/update_full $N --steps 1 --warmup 3 > $O/ncu_update.log 2>&1
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:static_kernel --launch-count 1 -o $O/static_full $N --steps 1 --warmup 3 > $O/ncu_static.log 2>&1
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:lean --launch-skip 20 --launch-count 1 -o $O/lean_full python tools/lean_ncu_target.py rmat16 40 > $O/ncu_lean.log 2>&1
 for c in rmat16 smallworld delaunay18; do timeout 900 python tools/paper_figures.py $c 100 > $O/fig_$c.json 2> $O/fig_$c.err; done
 ls -la $O

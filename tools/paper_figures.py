@@ -4,9 +4,9 @@
 
 * Fig. 2: distribution of the k x B scenarios over Case 1/2/3.
 * Fig. 4: fraction of the vertices touched
-  ({i | t[i] != untouched}) by every Case-2 scenario, sorted ascending (the
-  kernel's touched set: ancestors are reached through non-zero Delta-delta
-  only, a subset of Alg. 2's; R19).
+  ({i | t[i] != untouched}, Alg. 2's set: D and every ancestor, the root
+  excluded -- the scenario log counts it exactly, R19) by every
+  Case-2 scenario, sorted ascending.
 * Table III: per-insertion update time (fastest / average /
   slowest single-edge call) against one static recompute over the same roots.
 Inputs: the bench workload (remove-then-reinsert).  Diagnostics only:
