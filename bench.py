@@ -175,7 +175,8 @@ def ncu_traffic(config, batch, mode, launches_per_batch):
         with open(path) as f:
             t = json.load(f)
         e = t.get(f"{config}/b{batch}/{mode}")
-        return None if e is None else float(e["dram_bytes_per_batch"]) / max(launches_per_batch, 1.0)
+        return None if e is None else (float(e["dram_bytes_per_batch"]) / max(launches_per_batch, 1.0),
+                                       e.get("sectors_per_request"))
     except Exception:
         return None
 
@@ -558,6 +559,7 @@ def run_ours(args):
         except OSError:
             nccl = {"log": nccl_log, "lines": []}
 
+    traffic = ncu_traffic(args.config, B, args.mode, launches / K)
     state_mb = 24.0 * k * g.n / shard_world / 1e6
     line = {
         "metric": METRIC,
@@ -594,7 +596,11 @@ def run_ours(args):
         },
         "roofline": {
             "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-            "frac": achieved / peak, "traffic": ncu_traffic(args.config, B, args.mode, launches / K),
+            "frac": achieved / peak, "traffic": traffic[0] if traffic else None,
+            "dram_GBps": (traffic[0] / (launch_ms / 1e3) / 1e9) if traffic and launch_ms > 0 else None,
+            "sectors_per_request": traffic[1] if traffic else None,
+            "traffic_source": "committed ncu --set full capture of this config's batch (profiles/ncu_traffic.json)"
+                              if traffic else None,
             "kernel": "update_kernel", "peak_source": peak_src,
             "alg_bytes_per_launch": bytes_per_launch, "launch_ms": launch_ms,
             "byte_model": "SURVEY.md Sec. 8(d), counted per event in the kernel",

@@ -67,7 +67,7 @@ constexpr uint32_t kLD = 3u;      // mark: in D (t = down).  kLD > kLUp: an up c
 constexpr uint32_t kLUp = 1u;     // mark: up (t = up)        never overrides a D mark
 constexpr int kHelpBlk = 4096;    // entries per help block
 constexpr int kHelpMinBlk = 3;    // passes of at least this many blocks are published
-constexpr int kLEnt = 2048;       // entries whose contributions are kept for an in-order row sum
+constexpr int kLEnt = 1536;       // entries whose contributions are kept for an in-order row sum
 constexpr int kSpecEntries = 2 * kBlock * kLU;  // passes up to this size gather speculatively
 
 // pass kinds (entry visitors)
@@ -86,6 +86,8 @@ struct LeanSmem {
     double ev[kLEnt];    // per-entry contribution of a local pass (rows summed in canonical order)
     int adjs[kLAdj];
     int wul[kLWin], wlev[kLWin], wq[kLWin];
+    int nx[kLCap];       // the next down level's first kLCap vertices (mirror of Dv)
+    int um[2][kLCap];    // the up lists' first kLCap vertices (mirrors of U0 / U1)
 };
 
 // A pass published for help (global memory, one per worker).
@@ -124,6 +126,9 @@ struct PassCtx {
     double *dacc;
     int32_t *list, *list2;       // appends: Dv (down), an up list (up), Rv / Rl (removal)
     int *ctr;
+    int *mir;                    // nullable: shared mirror of the list's entries [mbase, mbase + kLCap)
+    int mbase;
+    int mirbit;                  // its s_mirbad bit
     int *low, *rmin, *rmax;
     double *acc;                 // per-row sums (when ev == nullptr)
     double *ev;                  // per-entry contributions (a local pass of <= kLEnt entries)
@@ -157,6 +162,24 @@ __device__ __forceinline__ int block_excl_scan(int x, int *total) {
 // Exclusive offsets of the chunk's row lengths (S.off[t+1] holds len t on
 // entry); returns the total.  Ends with a barrier.
 __device__ __forceinline__ int chunk_offsets(LeanSmem &S, int cnt) {
+    if (cnt <= 32) {  // a narrow level: warp 0 scans alone (one barrier instead of three)
+        __shared__ int s_tot;
+        if (threadIdx.x < 32) {
+            const int lane = threadIdx.x;
+            const int x = lane < cnt ? S.off[lane + 1] : 0;
+            int incl = x;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const int y = __shfl_up_sync(kFull, incl, o);
+                if (lane >= o) incl += y;
+            }
+            if (lane < cnt) S.off[lane + 1] = incl;
+            if (lane == 31) s_tot = incl;
+            if (lane == 0) S.off[0] = 0;
+        }
+        __syncthreads();
+        return s_tot;
+    }
     constexpr int per = kLCap / kBlock > 0 ? kLCap / kBlock : 1;
     int vals[per];
     int run = 0;
@@ -196,7 +219,11 @@ __device__ __forceinline__ int pass_spec(int kind) {
 }
 
 __device__ __forceinline__ void claim_append(const PassCtx &c, int y, uint32_t m) {
-    if (atomicMax(c.mark + y, m) < c.E) c.list[atomicAdd(c.ctr, 1)] = y;
+    if (atomicMax(c.mark + y, m) < c.E) {
+        const int p = atomicAdd(c.ctr, 1);
+        c.list[p] = y;
+        if (c.mir && p - c.mbase < kLCap) c.mir[p - c.mbase] = y;
+    }
 }
 
 // One entry (row t, neighbour y at distance dy; q / mk gathered per pass_sel).
@@ -332,6 +359,7 @@ __device__ __forceinline__ void lean_pass(const PassCtx &c, LeanSmem &S, int *s_
 __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs a) {
     __shared__ LeanSmem S;
     __shared__ int s_slot, s_nwork, s_dcnt, s_ucnt[2], s_rcnt, s_rmin, s_rmax, s_nst, s_nsc, s_low, s_ds;
+    __shared__ int s_mirbad;  // bit (L & 1): the down mirror of level L is incomplete; bit 2 + i: up list i's
     __shared__ int s_hb, s_hpick, s_hseq, s_hidle;
 
     const int tid = threadIdx.x;
@@ -415,6 +443,8 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
         gc.rmax = &mine->rmax;
         gc.acc = mine->acc;
         gc.ev = nullptr;
+        gc.mir = nullptr;  // helpers append to the list only: its mirror is incomplete
+        if (tid == 0 && c.mir) s_mirbad |= c.mirbit;
         for (;;) {  // the owner takes blocks too
             if (tid == 0) {
                 const unsigned long long w = atomicAdd(&mine->word, 1ull << 16);
@@ -510,6 +540,9 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                 pc.ev = nullptr;
                 pc.full = a.scen != nullptr || pull;
                 pc.pull = pull;
+                pc.mir = nullptr;
+                pc.mbase = 0;
+                pc.mirbit = 0;
                 // ---- seed (A2) ----
                 if (tid == 0) {
                     const int dl = __ldcg(st.d + ul);
@@ -524,6 +557,8 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                     s_low = c3;
                     mark[ul] = mD;
                     Dv[0] = ul;
+                    S.nx[0] = ul;
+                    s_mirbad = 0;
                     Doff[0] = 0;
                     Doff[1] = 1;
                     s_dcnt = 1;
@@ -538,10 +573,14 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                 // ---- down phase (K3) ----
                 int L = L0, lb = 0, le = 1, nlev = 0;
                 while (lb < le) {
+                    // the first kLCap vertices of this level come from the shared
+                    // mirror its producer pass filled (unless helpers appended)
+                    const bool mir_ok = !(s_mirbad & (1 << (L & 1)));
                     for (int c = lb; c < le; c += kLCap) {
                         const int cnt = min(kLCap, le - c);
+                        if (c == lb && tid == 0) s_mirbad &= ~(1 << ((L + 1) & 1));  // the next level's
                         for (int t = tid; t < cnt; t += kBlock) {
-                            const int w = __ldcg(Dv + c + t);
+                            const int w = (c == lb && mir_ok) ? S.nx[t] : __ldcg(Dv + c + t);
                             const int2 r = row_of(g, w, lim);
                             const unsigned long long lr = __ldcg(lowrec + w);
                             Dold[c + t] = ((lr >> 32) == epoch) ? (int)(uint32_t)lr : L;
@@ -559,6 +598,9 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                         cdn.l = L;
                         cdn.list = Dv;
                         cdn.ctr = &s_dcnt;
+                        cdn.mir = S.nx;
+                        cdn.mbase = le;
+                        cdn.mirbit = 1 << ((L + 1) & 1);
                         const bool in_acc = run_pass(cdn, cnt, Etot, slot, 0, sc_ph[0]);
                         for (int t = tid; t < cnt; t += kBlock) {
                             double sum;
@@ -632,13 +674,19 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                     // removal targets of this level join the up list
                     if (rcnt && l >= rmin && l <= rmax) {
                         for (int j = tid; j < rcnt; j += kBlock)
-                            if (__ldcg(Rl + j) == l) Ul[cu][atomicAdd(&s_ucnt[cu], 1)] = __ldcg(Rv + j);
+                            if (__ldcg(Rl + j) == l) {
+                                const int p = atomicAdd(&s_ucnt[cu], 1), x = __ldcg(Rv + j);
+                                Ul[cu][p] = x;
+                                if (p < kLCap) S.um[cu][p] = x;
+                            }
                     }
                     if (l == 2 && tid == 0) {  // the root's row: level-1 candidates of the shortcut
                         const int2 rs = row_of(g, sroot, lim);
                         s_ds = rs.y - rs.x <= kLAdj ? rs.y - rs.x : -1;
                     }
+                    if (tid == 0) s_mirbad &= ~(4 << (cu ^ 1));  // the list this level produces
                     __syncthreads();
+                    const bool umir_ok = !(s_mirbad & (4 << cu));  // its shared mirror is complete
                     if (l == 2 && s_ds > 0) {
                         const int2 rs = row_of(g, sroot, lim);
                         for (int j = tid; j < s_ds; j += kBlock) S.adjs[j] = ldg_i(g.col + rs.x + j);
@@ -651,6 +699,9 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                     cp.l = l;
                     cp.list = Ul[cu ^ 1];
                     cp.ctr = &s_ucnt[cu ^ 1];
+                    cp.mir = S.um[cu ^ 1];
+                    cp.mbase = 0;
+                    cp.mirbit = 4 << (cu ^ 1);
                     // D vertices of the level: delta by pull, pushes to predecessors
                     // outside D.  DBC_FLAG_PULL_DELTA: the up vertices too (rows
                     // nd.. of this loop, aux = -1): every touched vertex pulls
@@ -661,7 +712,8 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                         if (tid == 0) s_nst = 0;
                         for (int t = tid; t < cnt; t += kBlock) {
                             const int j = c + t;
-                            const int x = j < nd ? __ldcg(Dv + db + j) : __ldcg(Ul[cu] + j - nd);
+                            const int x = j < nd ? __ldcg(Dv + db + j)
+                                          : ((j - nd < kLCap && umir_ok) ? S.um[cu][j - nd] : __ldcg(Ul[cu] + j - nd));
                             const double2 q = __ldcg(st.sd + x);  // (sigma_new, delta_old)
                             const int2 r = row_of(g, x, lim);
                             S.v[t] = x;
@@ -755,7 +807,9 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                         if (tid == 0) s_nsc = 0;
                         __syncthreads();
                         for (int t = tid; t < cnt; t += kBlock) {
-                            const int x = __ldcg(Ul[cu] + c + t);
+                            const int x = (c + t < kLCap && umir_ok) ? S.um[cu][c + t] : __ldcg(Ul[cu] + c + t);
+                            // the row bounds are loaded with the accumulator (one round trip)
+                            const int rb0 = ldg_i(g.rp + x), re0 = ldg_i(g.rp + x + 1);
                             const double f = __ldcg(dacc + x);
                             const double2 q = __ldcg(st.sd + x);
                             const double gd = __dmul_rn(q.x, f);
@@ -769,7 +823,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                             S.c0[t] = f;
                             int len = 0;
                             if (l >= 2 && (f != 0.0 || cp.full)) {
-                                const int2 r = row_of(g, x, lim);
+                                const int2 r = rb0 >= 0 ? make_int2(rb0, re0 & kMask) : row_of(g, x, lim);
                                 if (l == 2 && ds > 0 && r.y - r.x > a.short_mult * ds) {
                                     S.sc_t[atomicAdd(&s_nsc, 1)] = t;  // level-1 predecessors = adj(s) n adj(x)
                                 } else {
@@ -939,6 +993,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
             c.ev = nullptr;
             c.full = a.scen != nullptr;
             c.pull = false;
+            c.mir = nullptr;
             uint32_t hscan = 0;
             lean_pass(c, S, &s_nst, g, cnt, b * kHelpBlk, min(Etot, (b + 1) * kHelpBlk), my_bytes, hscan);
             my_scan += hscan;
