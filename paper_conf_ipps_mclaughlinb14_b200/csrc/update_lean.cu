@@ -226,10 +226,15 @@ __device__ __forceinline__ void claim_append(const PassCtx &c, int y, uint32_t m
     }
 }
 
-// One entry (row t, neighbour y at distance dy; q / mk gathered per pass_sel).
-// Returns the row's contribution (sigma for down rows, the delta term for D rows).
+// One entry (row t, neighbour y at distance dy; q / mk gathered per pass_sel),
+// first half: the row's contribution (sigma for down rows, the delta term for
+// D rows) and fire-and-forget updates; the atomics whose result matters are
+// returned as requests -- *low: a lowering to l + 1 (Case 3), *claim: the mark
+// to claim y with -- and issued by lean_pass for all of a thread's entries
+// together (one round trip instead of one per entry).
 __device__ __forceinline__ double pass_visit(const PassCtx &c, LeanSmem &S, int *s_nst, int t, int y, int dy,
-                                             double2 q, uint32_t mk, uint32_t &bytes) {
+                                             double2 q, uint32_t mk, uint32_t &bytes, bool *low,
+                                             uint32_t *claim) {
     bytes += 8;
     switch (c.kind) {
         case kPDown:
@@ -237,16 +242,11 @@ __device__ __forceinline__ double pass_visit(const PassCtx &c, LeanSmem &S, int 
                 bytes += 8;
                 return q.x;
             }
-            if (dy > c.l + 1) {  // Case 3: pull y up to l + 1, the first lowerer records the old d
-                const int old = atomicMin(c.st.d + y, c.l + 1);
-                if (old > c.l + 1) {
-                    c.lowrec[y] = c.E64 | (uint32_t)old;
-                    *c.low = 1;
-                    bytes += 4;
-                }
-                claim_append(c, y, c.mD);
+            if (dy > c.l + 1) {  // Case 3: pull y up to l + 1 (the first lowerer records the old d)
+                *low = true;
+                *claim = c.mD;
             } else if (dy == c.l + 1 && mk < c.E) {  // successor: t[y] = down
-                claim_append(c, y, c.mD);
+                *claim = c.mD;
             }
             return 0.0;
         case kPUp:  // up vertex: Ddelta[p] += sigma[p] / sigma[x] * Ddelta[x] (factored)
@@ -254,20 +254,14 @@ __device__ __forceinline__ double pass_visit(const PassCtx &c, LeanSmem &S, int 
                 const double f = S.c0[t];
                 if (f != 0.0) atomicAdd(c.dacc + y, f);
                 bytes += 16;
-                if (mk < c.E) claim_append(c, y, c.mU);
+                if (mk < c.E) *claim = c.mU;
             }
             return 0.0;
         case kPRem:  // an old predecessor outside D gets the old contribution back
             if (dy == S.aux[t] && mk != c.mD) {
                 if (!c.pull) atomicAdd(c.dacc + y, S.c0[t]);
                 bytes += 16;
-                if (mk < c.E && atomicMax(c.mark + y, c.mU) < c.E) {
-                    const int p = atomicAdd(c.ctr, 1);
-                    c.list[p] = y;
-                    c.list2[p] = dy;
-                    atomicMin(c.rmin, dy);
-                    atomicMax(c.rmax, dy);
-                }
+                if (mk < c.E) *claim = c.mU;
             }
             return 0.0;
         default:  // kPDRow: delta by pull; predecessors outside D staged for pushes
@@ -288,7 +282,7 @@ __device__ __forceinline__ double pass_visit(const PassCtx &c, LeanSmem &S, int 
 
 // Flattened pass over entries [e_beg, e_end) of the chunk's rows (S.off holds
 // cnt + 1 exclusive offsets, S.beg the row starts).  Contributions are summed
-// into c.acc[t].  Ends with a barrier.
+// into c.acc[t] (or kept per entry in c.ev).  Ends with a barrier.
 __device__ __forceinline__ void lean_pass(const PassCtx &c, LeanSmem &S, int *s_nst, const GView &g, int cnt,
                                           int e_beg, int e_end, uint32_t &bytes, uint32_t &scanned) {
     const int tid = threadIdx.x;
@@ -337,16 +331,48 @@ __device__ __forceinline__ void lean_pass(const PassCtx &c, LeanSmem &S, int *s_
                 mk[u] = (s & 2) ? __ldcg(c.mark + y[u]) : 0u;
             }
         }
+        bool low[kLU];
+        uint32_t clm[kLU];
 #pragma unroll
         for (int u = 0; u < kLU; ++u) {
             double v = 0.0;
+            low[u] = false;
+            clm[u] = 0u;
             if (t[u] >= 0) {
                 ++scanned;
-                v = pass_visit(c, S, s_nst, t[u], y[u], dy[u], q[u], mk[u], bytes);
+                v = pass_visit(c, S, s_nst, t[u], y[u], dy[u], q[u], mk[u], bytes, &low[u], &clm[u]);
                 if (c.ev) c.ev[e0 + u] = v;
             }
             if (!c.ev) acc_add(c.acc, v != 0.0 ? t[u] : -1, v);
         }
+        // the requested atomics, all of this thread's entries in flight together
+        if (c.kind == kPDown) {
+            int old[kLU];
+#pragma unroll
+            for (int u = 0; u < kLU; ++u) old[u] = low[u] ? atomicMin(c.st.d + y[u], c.l + 1) : 0;
+#pragma unroll
+            for (int u = 0; u < kLU; ++u)
+                if (low[u] && old[u] > c.l + 1) {  // the first lowerer records the old d
+                    c.lowrec[y[u]] = c.E64 | (uint32_t)old[u];
+                    *c.low = 1;
+                    bytes += 4;
+                }
+        }
+        uint32_t prev[kLU];
+#pragma unroll
+        for (int u = 0; u < kLU; ++u) prev[u] = clm[u] ? atomicMax(c.mark + y[u], clm[u]) : 0xffffffffu;
+#pragma unroll
+        for (int u = 0; u < kLU; ++u)
+            if (prev[u] < c.E) {  // claimed: append to the pass's list
+                const int p = atomicAdd(c.ctr, 1);
+                c.list[p] = y[u];
+                if (c.mir && p - c.mbase < kLCap) c.mir[p - c.mbase] = y[u];
+                if (c.kind == kPRem) {  // removal targets keep their level
+                    c.list2[p] = dy[u];
+                    atomicMin(c.rmin, dy[u]);
+                    atomicMax(c.rmax, dy[u]);
+                }
+            }
     }
     __syncthreads();
 }
@@ -360,6 +386,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
     __shared__ LeanSmem S;
     __shared__ int s_slot, s_nwork, s_dcnt, s_ucnt[2], s_rcnt, s_rmin, s_rmax, s_nst, s_nsc, s_low, s_ds;
     __shared__ int s_mirbad;  // bit (L & 1): the down mirror of level L is incomplete; bit 2 + i: up list i's
+    __shared__ unsigned long long s_tph[10];  // tuning.trace_slot: SM cycles per phase of that root (thread 0)
     __shared__ int s_hb, s_hpick, s_hseq, s_hidle;
 
     const int tid = threadIdx.x;
@@ -384,6 +411,20 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
     const bool pull = a.pull_delta != 0;  // DBC_FLAG_PULL_DELTA (no help board then)
     int hseq = 0;
 
+    // phase clocks of one traced root (dbc_tuning.trace_slot; diagnostic): down
+    // item load / scan / pass / finalize, removal, up level setup, D rows, up
+    // item load / scan / pass
+    bool trace = false;
+    long long tclk = 0;
+    if (tid == 0)
+        for (int q = 0; q < 10; ++q) s_tph[q] = 0;
+    auto tick = [&](int ph) {
+        if (trace && tid == 0) {
+            const long long t = clock64();
+            if (ph >= 0) s_tph[ph] += (unsigned long long)(t - tclk);
+            tclk = t;
+        }
+    };
     // counters: thread-local bytes / scanned entries, thread 0's tallies
     uint32_t my_bytes = 0, my_scan = 0;
     uint32_t sc_ph[6] = {0, 0, 0, 0, 0, 0};  // scanned: down, removal, D rows, level-2 probes, up@2, up@>=3
@@ -487,6 +528,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
         if (slot < 0) break;
         const Root st{a.d + (size_t)slot * n, a.sd + (size_t)slot * n};
         const int sroot = a.roots[slot];
+        trace = slot == a.trace_slot;
         bool masks_dropped = false;
         // root profile (dbc_debug_root_profile): start, jobs, touched, levels (thread 0)
         unsigned long long pr_t0 = 0, pr_jobs = 0, pr_touch = c_touch, pr_lev = c_lev[0] + c_lev[1];
@@ -572,6 +614,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
 
                 // ---- down phase (K3) ----
                 int L = L0, lb = 0, le = 1, nlev = 0;
+                tick(-1);
                 while (lb < le) {
                     // the first kLCap vertices of this level come from the shared
                     // mirror its producer pass filled (unless helpers appended)
@@ -592,7 +635,9 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                             my_bytes += 8 + 20;
                         }
                         __syncthreads();
+                        tick(0);
                         const int Etot = chunk_offsets(S, cnt);
+                        tick(1);
                         PassCtx cdn = pc;
                         cdn.kind = kPDown;
                         cdn.l = L;
@@ -622,6 +667,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                         }
                         __syncthreads();
                     }
+                    tick(2);
                     lb = le;
                     le = s_dcnt;
                     ++nlev;
@@ -665,6 +711,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                 }
                 __syncthreads();
 
+                tick(4);
                 // ---- up phase (K4 + Alg. 8) ----
                 const int rcnt = s_rcnt, rmin = s_rmin, rmax = s_rmax;
                 int cu = 0;  // Ul[cu] holds the up vertices of the current level
@@ -687,6 +734,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                     if (tid == 0) s_mirbad &= ~(4 << (cu ^ 1));  // the list this level produces
                     __syncthreads();
                     const bool umir_ok = !(s_mirbad & (4 << cu));  // its shared mirror is complete
+                    tick(5);
                     if (l == 2 && s_ds > 0) {
                         const int2 rs = row_of(g, sroot, lim);
                         for (int j = tid; j < s_ds; j += kBlock) S.adjs[j] = ldg_i(g.col + rs.x + j);
@@ -801,6 +849,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                         }
                         __syncthreads();
                     }
+                    tick(6);
                     // up vertices of the level: apply Ddelta, forward it to the predecessors
                     for (int c = 0; c < (pull ? 0 : nu); c += kLCap) {
                         const int cnt = min(kLCap, nu - c);
@@ -835,10 +884,13 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                             S.off[t + 1] = len;
                         }
                         __syncthreads();
+                        tick(7);
                         const int Etot = chunk_offsets(S, cnt);
+                        tick(8);
                         PassCtx cu2 = cp;
                         cu2.kind = kPUp;
                         run_pass(cu2, cnt, Etot, slot, cu ^ 1, sc_ph[l == 2 ? 4 : 5]);
+                        tick(9);
                         const int nsc = s_nsc;
                         if (nsc) {
                             const int pairs = nsc * ds;
@@ -861,6 +913,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                     cu ^= 1;
                     ++c_lev[1];
                     __syncthreads();
+                    tick(3);
                 }
                 c_lev[0] += nlev;
                 c_down += dtotal;
@@ -1006,6 +1059,8 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
     }
 
     if (tid == 0) {
+        for (int q = 0; q < 10; ++q)
+            if (s_tph[q]) atomicAdd(a.stats + kStTime0 + q, s_tph[q]);
         a.ws.wepoch[wk] = epoch;
         if (c_case[1]) atomicAdd(a.stats + kStCase2, c_case[1]);
         if (c_case[2]) atomicAdd(a.stats + kStCase3, c_case[2]);
