@@ -74,6 +74,9 @@ def parse():
                    help="bound on the insertions of each side measurement")
     p.add_argument("--shard", default="", help="R/N: run rank R's root shard of an N-GPU job on this "
                    "single GPU (per-GPU view of configs that need N GPUs, e.g. kron22 on 8)")
+    p.add_argument("--dist-test-one-gpu", action="store_true",
+                   help="validation only: every torchrun rank on cuda:0, gloo process group and the "
+                        "library's reduce callback instead of NCCL (NCCL refuses two ranks on one GPU)")
     a = p.parse_args()
     if a.config is None:
         world = int(os.environ.get("WORLD_SIZE", str(a.gpus)))
@@ -310,7 +313,12 @@ def run_ours(args):
             raise SystemExit("--shard emulates one rank on one GPU; do not combine with torchrun")
         shard_rank, shard_world = (int(x) for x in args.shard.split("/"))
     nccl_log = None
-    if world > 1:
+    one_gpu = args.dist_test_one_gpu
+    if world > 1 and one_gpu:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        torch.cuda.set_device(0)
+        dist.init_process_group("gloo")
+    elif world > 1:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
         # NCCL's communicator lines (version, transports, NVLS) into a per-rank file
         nccl_log = os.path.join("/tmp", f"dbc_nccl.{os.getpid()}.log")
@@ -324,7 +332,7 @@ def run_ours(args):
     dev = torch.cuda.current_device()
 
     from paper_conf_ipps_mclaughlinb14_b200 import (FLAG_MODE_S, FLAG_NO_MERGE, FLAG_TIMING,
-                                                    DynamicBC, nccl_unique_id)
+                                                    DynamicBC, nccl_unique_id, torch_reducer)
 
     cfg = W.CONFIGS[args.config]
     B = args.batch or cfg["insertions"]
@@ -338,7 +346,8 @@ def run_ours(args):
     stream = torch.cuda.Stream(device=dev)  # the library and the timing events share it
     torch.cuda.set_stream(stream)
     uid = None
-    if world > 1:  # the library's own NCCL communicator for the BC all-reduce (opt.nccl_id)
+    reducer = torch_reducer() if (world > 1 and one_gpu) else None
+    if world > 1 and not one_gpu:  # the library's own NCCL communicator for the BC all-reduce (opt.nccl_id)
         obj = [nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         uid = obj[0]
@@ -347,14 +356,14 @@ def run_ours(args):
     def make(fl):
         return DynamicBC(g.n, g.row_ptr, g.col, wl.roots, device=dev, rank=shard_rank, world=shard_world,
                          workers=args.workers, edge_capacity=B * nb, flags=fl, stream=stream.cuda_stream,
-                         nccl_id=uid)
+                         nccl_id=uid, reduce=reducer)
 
     dbc = make(flags)
 
     def max_over_ranks(x):
         if world == 1:
             return x
-        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        t = torch.tensor([x], dtype=torch.float64, device="cpu" if one_gpu else dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
@@ -559,7 +568,8 @@ def run_ours(args):
         except OSError:
             nccl = {"log": nccl_log, "lines": []}
 
-    traffic = ncu_traffic(args.config, B, args.mode, launches / K)
+    # the committed capture is of one whole-root-set batch: only comparable at one rank
+    traffic = ncu_traffic(args.config, B, args.mode, launches / K) if shard_world == 1 else None
     state_mb = 24.0 * k * g.n / shard_world / 1e6
     line = {
         "metric": METRIC,
@@ -576,6 +586,8 @@ def run_ours(args):
         "data": "synthetic",
         "config": {
             "workload": args.config,
+            "dist_test_one_gpu": (f"{world} ranks on cuda:0 over gloo + the reduce callback: validates the "
+                                  f"multi-rank path, not a scaling number") if one_gpu else None,
             "graph": GRAPH_DESC.get(args.config, args.config),
             "n": g.n, "m": g.m, "k": k, "batch": B, "mode": args.mode, "seed": args.seed,
             "protocol": "remove-then-reinsert (P:440)" if cfg["mode"] == "reinsert" else "uniform non-edges",
