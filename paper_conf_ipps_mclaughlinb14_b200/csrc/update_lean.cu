@@ -71,7 +71,7 @@ constexpr int kLEnt = 1536;       // entries whose contributions are kept for an
 constexpr int kSpecEntries = 2 * kBlock * kLU;  // passes up to this size gather speculatively
 
 // pass kinds (entry visitors)
-enum : int { kPDown = 1, kPUp = 2, kPRem = 3, kPDRow = 4 };
+enum : int { kPDown = 1, kPUp = 2, kPRem = 3, kPDRow = 4, kPDPush = 5 };
 
 struct LeanSmem {
     int v[kLCap];
@@ -98,10 +98,12 @@ struct LeanBoard {
     int low, rmin, rmax;      // down: a distance was lowered; removal: target level range
     int kind, slot, l, cnt, Etot, sel;  // sel: which up list receives appends
     uint32_t E, epoch;
+    int ul, uh, pull;         // the job's insertion (D-row pushes skip the old term over it)
     int off[kLCap + 1];
     int beg[kLCap];
     int aux[kLCap];
-    double c0[kLCap];
+    int v[kLCap];
+    double c0[kLCap], c1[kLCap];
     double acc[kLCap];
 };
 
@@ -132,6 +134,8 @@ struct PassCtx {
     int *low, *rmin, *rmax;
     double *acc;                 // per-row sums (when ev == nullptr)
     double *ev;                  // per-entry contributions (a local pass of <= kLEnt entries)
+    int ul, uh;                  // the job's insertion
+    bool stash;                  // kPDRow: stage predecessors in shared memory (a local pass)
     bool full;
     bool pull;                   // DBC_FLAG_PULL_DELTA: targets are only claimed (they pull)                   // scenario log: claim even over a zero push (Alg. 2's touched set)
 };
@@ -209,13 +213,14 @@ __device__ __forceinline__ int pass_sel(const PassCtx &c, const LeanSmem &S, int
         case kPDown: return dy == c.l - 1 ? 1 : (dy == c.l + 1 ? 2 : 0);
         case kPUp: return dy == c.l - 1 ? 2 : 0;
         case kPRem: return dy == S.aux[t] ? 2 : 0;
+        case kPDPush: return dy == c.l - 1 ? 2 : 0;
         default: return (dy == c.l + 1 ? 1 : 0) | ((c.l >= 2 && dy == c.l - 1) ? 2 : 0);  // kPDRow
     }
 }
 
 // everything a pass kind may gather (speculative gathers of a narrow pass)
 __device__ __forceinline__ int pass_spec(int kind) {
-    return kind == kPDown ? 3 : (kind == kPDRow ? 3 : 2);
+    return kind == kPDown ? 3 : (kind == kPDRow ? 3 : 2);  // kPUp, kPRem, kPDPush: the flag
 }
 
 __device__ __forceinline__ void claim_append(const PassCtx &c, int y, uint32_t m) {
@@ -264,12 +269,25 @@ __device__ __forceinline__ double pass_visit(const PassCtx &c, LeanSmem &S, int 
                 if (mk < c.E) *claim = c.mU;
             }
             return 0.0;
+        case kPDPush:  // D row x: Ddelta[p] += sigma[p] * ((1 + delta_new) / sigma_new - old term)
+            if (dy == c.l - 1 && mk != c.mD) {
+                if (c.pull) {  // the predecessor pulls its own delta
+                    if (mk < c.E) *claim = c.mU;
+                    return 0.0;
+                }
+                const bool ne = S.v[t] == c.ul && y == c.uh;  // never an old term over the new edge
+                const double w = ne ? S.c0[t] : __dsub_rn(S.c0[t], S.c1[t]);
+                if (w != 0.0) atomicAdd(c.dacc + y, w);
+                bytes += 16;
+                if ((w != 0.0 || c.full) && mk < c.E) *claim = c.mU;
+            }
+            return 0.0;
         default:  // kPDRow: delta by pull; predecessors outside D staged for pushes
             if (dy == c.l + 1) {
                 bytes += 16;
                 return __dmul_rn(__ddiv_rn(S.c0[t], q.x), __dadd_rn(1.0, q.y));
             }
-            if (c.l >= 2 && dy == c.l - 1 && mk != c.mD) {
+            if (c.stash && c.l >= 2 && dy == c.l - 1 && mk != c.mD) {
                 const int p = atomicAdd(s_nst, 1);
                 if (p < kLStash) {
                     S.st_p[p] = mk < c.E ? y : (y | INT32_MIN);  // high bit: already claimed
@@ -433,8 +451,9 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
     // Run a pass over the chunk in S (cnt rows, Etot entries): locally, or
     // published on the board when it is wide and idle workers exist.  c holds
     // the local (shared-memory) counters; they are updated either way.
-    // Returns true when the per-row sums are in S.acc (else in S.ev, per entry).
-    auto run_pass = [&](PassCtx c, int cnt, int Etot, int slot, int sel, uint32_t &scan) -> bool {
+    // Returns bit 0: the per-row sums are in S.acc (else in S.ev, per entry);
+    // bit 1: the pass was published (helped).
+    auto run_pass = [&](PassCtx c, int cnt, int Etot, int slot, int sel, uint32_t &scan) -> int {
         const int nblk = (Etot + kHelpBlk - 1) / kHelpBlk;
         if (nblk >= kHelpMinBlk) {
             if (tid == 0) s_hidle = mine ? __ldcg(live + 1) : 0;
@@ -443,7 +462,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
         if (nblk < kHelpMinBlk || s_hidle <= 0) {
             c.ev = Etot <= kLEnt ? S.ev : nullptr;
             lean_pass(c, S, &s_nst, g, cnt, 0, Etot, my_bytes, scan);
-            return c.ev == nullptr;
+            return c.ev == nullptr ? 1 : 0;
         }
         // publish: chunk mirror + context (visible device-wide), then the word
         for (int t = tid; t < cnt; t += kBlock) {
@@ -451,6 +470,8 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
             mine->beg[t] = S.beg[t];
             mine->aux[t] = S.aux[t];
             mine->c0[t] = S.c0[t];
+            mine->c1[t] = S.c1[t];
+            mine->v[t] = S.v[t];
             mine->acc[t] = 0.0;
         }
         __threadfence();
@@ -470,6 +491,9 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
             mine->sel = sel;
             mine->E = c.E;
             mine->epoch = (uint32_t)(c.E64 >> 32);
+            mine->ul = c.ul;
+            mine->uh = c.uh;
+            mine->pull = c.pull ? 1 : 0;
             hseq = (hseq + 1) & 0xFFFF;
             __threadfence();
             atomicExch(&mine->word, hb_pack(1, nblk, 0, hseq));
@@ -484,6 +508,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
         gc.rmax = &mine->rmax;
         gc.acc = mine->acc;
         gc.ev = nullptr;
+        gc.stash = false;  // helpers' shared memory is their own: D-row pushes run as a kPDPush pass
         gc.mir = nullptr;  // helpers append to the list only: its mirror is incomplete
         if (tid == 0 && c.mir) s_mirbad |= c.mirbit;
         for (;;) {  // the owner takes blocks too
@@ -514,7 +539,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
         __syncthreads();
         for (int t = tid; t < cnt; t += kBlock) S.acc[t] = __ldcg(mine->acc + t);
         __syncthreads();
-        return true;
+        return 3;
     };
 
     for (;;) {
@@ -582,6 +607,9 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                 pc.ev = nullptr;
                 pc.full = a.scen != nullptr || pull;
                 pc.pull = pull;
+                pc.ul = ul;
+                pc.uh = uh;
+                pc.stash = false;
                 pc.mir = nullptr;
                 pc.mbase = 0;
                 pc.mirbit = 0;
@@ -646,7 +674,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                         cdn.mir = S.nx;
                         cdn.mbase = le;
                         cdn.mirbit = 1 << ((L + 1) & 1);
-                        const bool in_acc = run_pass(cdn, cnt, Etot, slot, 0, sc_ph[0]);
+                        const bool in_acc = run_pass(cdn, cnt, Etot, slot, 0, sc_ph[0]) & 1;
                         for (int t = tid; t < cnt; t += kBlock) {
                             double sum;
                             const int w = S.v[t];
@@ -777,12 +805,13 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                         const int Etot = chunk_offsets(S, cnt);
                         PassCtx cd = cp;
                         cd.kind = kPDRow;
-                        cd.ev = Etot <= kLEnt ? S.ev : nullptr;
-                        lean_pass(cd, S, &s_nst, g, cnt, 0, Etot, my_bytes, sc_ph[2]);
+                        cd.stash = true;
+                        const int how = run_pass(cd, cnt, Etot, slot, cu ^ 1, sc_ph[2]);
+                        const bool in_acc = how & 1, helped = how & 2;
                         for (int t = tid; t < cnt; t += kBlock) {  // delta, BC, the push coefficients
                             const int x = S.v[t], di = S.aux[t];
                             double dn = S.acc[t];
-                            if (cd.ev) {  // Eq. (2) summed left to right in canonical order
+                            if (!in_acc) {  // Eq. (2) summed left to right in canonical order
                                 dn = 0.0;
                                 for (int e = S.off[t]; e < S.off[t + 1]; ++e) dn = __dadd_rn(dn, S.ev[e]);
                             } else if (pull) {  // a chunk too wide for the entry buffer: re-sum in order
@@ -809,7 +838,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                         }
                         __syncthreads();
                         const int nst = s_nst;
-                        if (nst <= kLStash) {
+                        if (!helped && nst <= kLStash) {  // the staged predecessors
                             for (int j = tid; j < nst; j += kBlock) {
                                 const int t = S.st_t[j], pr = S.st_p[j], p = pr & INT32_MAX;
                                 if (pull) {  // the predecessor pulls its own delta at level l - 1
@@ -822,30 +851,10 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                                 my_bytes += 16;
                                 if ((w != 0.0 || cp.full) && pr >= 0) claim_append(cp, p, mU);
                             }
-                        } else {  // stash overflow: a second pass over the rows pushes
-                            for (int t = tid; t < cnt; t += kBlock) S.off[t + 1] = row_of(g, S.v[t], lim).y - S.beg[t];
-                            __syncthreads();
-                            const int E2 = chunk_offsets(S, cnt);
-                            for (int base = 0; base < E2; base += kBlock) {
-                                const int e = base + tid;
-                                if (e >= E2) continue;
-                                int lo = 0, hi = cnt - 1;
-                                while (lo < hi) {
-                                    const int mid = (lo + hi + 1) >> 1;
-                                    if (S.off[mid] <= e) lo = mid; else hi = mid - 1;
-                                }
-                                const int p = ldg_i(g.col + S.beg[lo] + (e - S.off[lo]));
-                                if (__ldcg(st.d + p) != l - 1 || __ldcg(mark + p) == mD) continue;
-                                if (pull) {
-                                    claim_append(cp, p, mU);
-                                    continue;
-                                }
-                                const bool new_edge = S.v[lo] == ul && p == uh;
-                                const double w = new_edge ? S.c0[lo] : __dsub_rn(S.c0[lo], S.c1[lo]);
-                                if (w != 0.0) atomicAdd(dacc + p, w);
-                                my_bytes += 16;
-                                if (w != 0.0 || cp.full) claim_append(cp, p, mU);
-                            }
+                        } else {  // stash overflow, or a helped pull: a push pass over the rows
+                            PassCtx cpu = cp;
+                            cpu.kind = kPDPush;
+                            run_pass(cpu, cnt, Etot, slot, cu ^ 1, sc_ph[3]);
                         }
                         __syncthreads();
                     }
@@ -1016,6 +1025,8 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                         S.beg[t] = __ldcg(ob->beg + t);
                         S.aux[t] = __ldcg(ob->aux + t);
                         S.c0[t] = __ldcg(ob->c0 + t);
+                        S.c1[t] = __ldcg(ob->c1 + t);
+                        S.v[t] = __ldcg(ob->v + t);
                     }
                 }
                 cur_owner = pick;
@@ -1045,7 +1056,10 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
             c.acc = ob->acc;
             c.ev = nullptr;
             c.full = a.scen != nullptr;
-            c.pull = false;
+            c.ul = __ldcg(&ob->ul);
+            c.uh = __ldcg(&ob->uh);
+            c.pull = __ldcg(&ob->pull) != 0;
+            c.stash = false;
             c.mir = nullptr;
             uint32_t hscan = 0;
             lean_pass(c, S, &s_nst, g, cnt, b * kHelpBlk, min(Etot, (b + 1) * kHelpBlk), my_bytes, hscan);

@@ -32,7 +32,7 @@ with DynamicBC(g.n, g.row_ptr, g.col, wl.roots, flags=FLAG_TIMING) as dbc:
         dt = (p[:, 1] - p[:, 0]) / 1e3  # us
         w = p[:, 2] > 0
         j = int(np.argmax(dt))
-        rows.append({"i": i, "update_us": t["update_ms"] * 1e3, "working": int(w.sum()),
+        rows.append({"i": i, "update_us": t["update_ms"] * 1e3, "working": int(w.sum()), "max_slot": j,
                      "max_us": float(dt[j]), "max_levels": int(p[j, 5]), "max_touched": int(p[j, 3]),
                      "max_scanned": int(p[j, 4]),
                      "median_working_us": float(np.median(dt[w])) if w.any() else 0.0,
