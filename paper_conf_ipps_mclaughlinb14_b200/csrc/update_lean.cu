@@ -136,6 +136,7 @@ struct PassCtx {
     double *ev;                  // per-entry contributions (a local pass of <= kLEnt entries)
     int ul, uh;                  // the job's insertion
     bool stash;                  // kPDRow: stage predecessors in shared memory (a local pass)
+    unsigned long long *ptr;     // -DDBC_LEAN_PTRACE builds: step clocks of the traced root's up passes
     bool full;
     bool pull;                   // DBC_FLAG_PULL_DELTA: targets are only claimed (they pull)                   // scenario log: claim even over a zero push (Alg. 2's touched set)
 };
@@ -208,8 +209,9 @@ __device__ __forceinline__ int chunk_offsets(LeanSmem &S, int cnt) {
 
 // what to gather for an entry with distance dy of row t: bit 0 (sigma, delta),
 // bit 1 the claim flag
+template <int K>
 __device__ __forceinline__ int pass_sel(const PassCtx &c, const LeanSmem &S, int t, int dy) {
-    switch (c.kind) {
+    switch (K) {
         case kPDown: return dy == c.l - 1 ? 1 : (dy == c.l + 1 ? 2 : 0);
         case kPUp: return dy == c.l - 1 ? 2 : 0;
         case kPRem: return dy == S.aux[t] ? 2 : 0;
@@ -219,8 +221,9 @@ __device__ __forceinline__ int pass_sel(const PassCtx &c, const LeanSmem &S, int
 }
 
 // everything a pass kind may gather (speculative gathers of a narrow pass)
-__device__ __forceinline__ int pass_spec(int kind) {
-    return kind == kPDown ? 3 : (kind == kPDRow ? 3 : 2);  // kPUp, kPRem, kPDPush: the flag
+template <int K>
+__device__ __forceinline__ constexpr int pass_spec() {
+    return K == kPDown ? 3 : (K == kPDRow ? 3 : 2);  // kPUp, kPRem, kPDPush: the flag
 }
 
 __device__ __forceinline__ void claim_append(const PassCtx &c, int y, uint32_t m) {
@@ -237,11 +240,12 @@ __device__ __forceinline__ void claim_append(const PassCtx &c, int y, uint32_t m
 // returned as requests -- *low: a lowering to l + 1 (Case 3), *claim: the mark
 // to claim y with -- and issued by lean_pass for all of a thread's entries
 // together (one round trip instead of one per entry).
+template <int K>
 __device__ __forceinline__ double pass_visit(const PassCtx &c, LeanSmem &S, int *s_nst, int t, int y, int dy,
                                              double2 q, uint32_t mk, uint32_t &bytes, bool *low,
                                              uint32_t *claim) {
     bytes += 8;
-    switch (c.kind) {
+    switch (K) {
         case kPDown:
             if (dy == c.l - 1) {  // predecessor: sigma (pull, Alg. 2 line 14 / P:238)
                 bytes += 8;
@@ -301,10 +305,23 @@ __device__ __forceinline__ double pass_visit(const PassCtx &c, LeanSmem &S, int 
 // Flattened pass over entries [e_beg, e_end) of the chunk's rows (S.off holds
 // cnt + 1 exclusive offsets, S.beg the row starts).  Contributions are summed
 // into c.acc[t] (or kept per entry in c.ev).  Ends with a barrier.
-__device__ __forceinline__ void lean_pass(const PassCtx &c, LeanSmem &S, int *s_nst, const GView &g, int cnt,
-                                          int e_beg, int e_end, uint32_t &bytes, uint32_t &scanned) {
+template <int K>
+__device__ __forceinline__ void lean_pass_k(const PassCtx &c, LeanSmem &S, int *s_nst, const GView &g, int cnt,
+                                            int e_beg, int e_end, uint32_t &bytes, uint32_t &scanned) {
     const int tid = threadIdx.x;
     const bool spec = e_end - e_beg <= kSpecEntries;
+#ifdef DBC_LEAN_PTRACE
+    long long pt = clock64();
+    auto ptick = [&](int q) {
+        if (K == kPUp && c.ptr && tid == 0) {
+            const long long t2 = clock64();
+            c.ptr[q] += (unsigned long long)(t2 - pt);
+            pt = t2;
+        }
+    };
+#else
+    auto ptick = [](int) {};
+#endif
     for (int base = e_beg; base < e_end; base += kBlock * kLU) {
         const int e0 = base + tid * kLU;
         int t[kLU], y[kLU], dy[kLU];
@@ -330,8 +347,9 @@ __device__ __forceinline__ void lean_pass(const PassCtx &c, LeanSmem &S, int *s_
                 y[u] = ldg_i(g.col + S.beg[cur] + (e - S.off[cur]));
             }
         }
+        ptick(0);
         if (spec) {  // narrow pass (latency-bound): gather d, (sigma, delta) and the flag together
-            const int s = pass_spec(c.kind);
+            constexpr int s = pass_spec<K>();
 #pragma unroll
             for (int u = 0; u < kLU; ++u) {
                 const bool on = t[u] >= 0;
@@ -344,11 +362,12 @@ __device__ __forceinline__ void lean_pass(const PassCtx &c, LeanSmem &S, int *s_
             for (int u = 0; u < kLU; ++u) dy[u] = t[u] >= 0 ? __ldcg(c.st.d + y[u]) : kInf;
 #pragma unroll
             for (int u = 0; u < kLU; ++u) {
-                const int s = t[u] >= 0 ? pass_sel(c, S, t[u], dy[u]) : 0;
+                const int s = t[u] >= 0 ? pass_sel<K>(c, S, t[u], dy[u]) : 0;
                 q[u] = (s & 1) ? __ldcg(c.st.sd + y[u]) : make_double2(0.0, 0.0);
                 mk[u] = (s & 2) ? __ldcg(c.mark + y[u]) : 0u;
             }
         }
+        ptick(1);
         bool low[kLU];
         uint32_t clm[kLU];
 #pragma unroll
@@ -358,13 +377,13 @@ __device__ __forceinline__ void lean_pass(const PassCtx &c, LeanSmem &S, int *s_
             clm[u] = 0u;
             if (t[u] >= 0) {
                 ++scanned;
-                v = pass_visit(c, S, s_nst, t[u], y[u], dy[u], q[u], mk[u], bytes, &low[u], &clm[u]);
+                v = pass_visit<K>(c, S, s_nst, t[u], y[u], dy[u], q[u], mk[u], bytes, &low[u], &clm[u]);
                 if (c.ev) c.ev[e0 + u] = v;
             }
             if (!c.ev) acc_add(c.acc, v != 0.0 ? t[u] : -1, v);
         }
         // the requested atomics, all of this thread's entries in flight together
-        if (c.kind == kPDown) {
+        if (K == kPDown) {
             int old[kLU];
 #pragma unroll
             for (int u = 0; u < kLU; ++u) old[u] = low[u] ? atomicMin(c.st.d + y[u], c.l + 1) : 0;
@@ -376,6 +395,7 @@ __device__ __forceinline__ void lean_pass(const PassCtx &c, LeanSmem &S, int *s_
                     bytes += 4;
                 }
         }
+        ptick(2);
         uint32_t prev[kLU];
 #pragma unroll
         for (int u = 0; u < kLU; ++u) prev[u] = clm[u] ? atomicMax(c.mark + y[u], clm[u]) : 0xffffffffu;
@@ -385,14 +405,31 @@ __device__ __forceinline__ void lean_pass(const PassCtx &c, LeanSmem &S, int *s_
                 const int p = atomicAdd(c.ctr, 1);
                 c.list[p] = y[u];
                 if (c.mir && p - c.mbase < kLCap) c.mir[p - c.mbase] = y[u];
-                if (c.kind == kPRem) {  // removal targets keep their level
+                if (K == kPRem) {  // removal targets keep their level
                     c.list2[p] = dy[u];
                     atomicMin(c.rmin, dy[u]);
                     atomicMax(c.rmax, dy[u]);
                 }
             }
+        ptick(3);
     }
     __syncthreads();
+    ptick(4);
+#ifdef DBC_LEAN_PTRACE
+    if (K == kPUp && c.ptr && tid == 0) c.ptr[5] += 1;
+#endif
+}
+
+// one specialised pass per kind (no kind switch in the entry loop)
+__device__ __forceinline__ void lean_pass(const PassCtx &c, LeanSmem &S, int *s_nst, const GView &g, int cnt,
+                                          int e_beg, int e_end, uint32_t &bytes, uint32_t &scanned) {
+    switch (c.kind) {
+        case kPDown: lean_pass_k<kPDown>(c, S, s_nst, g, cnt, e_beg, e_end, bytes, scanned); break;
+        case kPUp: lean_pass_k<kPUp>(c, S, s_nst, g, cnt, e_beg, e_end, bytes, scanned); break;
+        case kPRem: lean_pass_k<kPRem>(c, S, s_nst, g, cnt, e_beg, e_end, bytes, scanned); break;
+        case kPDPush: lean_pass_k<kPDPush>(c, S, s_nst, g, cnt, e_beg, e_end, bytes, scanned); break;
+        default: lean_pass_k<kPDRow>(c, S, s_nst, g, cnt, e_beg, e_end, bytes, scanned); break;
+    }
 }
 
 // resident CTAs per SM the registers are sized for: 128 registers at 128
@@ -610,6 +647,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                 pc.ul = ul;
                 pc.uh = uh;
                 pc.stash = false;
+                pc.ptr = trace ? a.stats + kStTrace0 : nullptr;
                 pc.mir = nullptr;
                 pc.mbase = 0;
                 pc.mirbit = 0;
@@ -1060,6 +1098,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
             c.uh = __ldcg(&ob->uh);
             c.pull = __ldcg(&ob->pull) != 0;
             c.stash = false;
+            c.ptr = nullptr;
             c.mir = nullptr;
             uint32_t hscan = 0;
             lean_pass(c, S, &s_nst, g, cnt, b * kHelpBlk, min(Etot, (b + 1) * kHelpBlk), my_bytes, hscan);
