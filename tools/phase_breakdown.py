@@ -8,7 +8,9 @@ wl = W.make_workload(name, insertions=B, k=int(sys.argv[3]) if len(sys.argv) > 3
 if len(sys.argv) > 4:  # explicit root list, e.g. 650960,3614
     wl.roots = np.array([int(x) for x in sys.argv[4].split(",")], dtype=np.int32)
 g = wl.graph
-dbc = DynamicBC(g.n, g.row_ptr, g.col, wl.roots, flags=FLAG_TIMING)
+tr = os.environ.get("DBC_TRACE_SLOT")  # traced root slot (dbc_tuning.trace_slot; -DDBC_PHASE_TIMERS builds)
+dbc = DynamicBC(g.n, g.row_ptr, g.col, wl.roots, flags=FLAG_TIMING,
+                tuning={"trace_slot": int(tr)} if tr else None)
 dbc.static_compute(); dbc.synchronize()
 c0 = dbc.debug_counters()
 dbc.root_profile(True, read=False)
