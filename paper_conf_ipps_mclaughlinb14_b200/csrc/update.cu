@@ -51,30 +51,78 @@ namespace {
 constexpr int32_t kOldMask = 0x7fffffff;
 constexpr int32_t kExtPred = INT32_MIN;
 
+// A C2 push pass: flat_entries (dbc_internal.cuh) whose visitor f(t, y, d, sd,
+// mark) returns the mark to claim y with (0: none); the claims of a thread's
+// kFlatU entries are issued together -- one atomic round trip instead of one
+// per entry -- and onclaim(y) runs for each vertex this thread claimed.
+template <bool kCG, class Want, class Col, class F, class OnClaim>
+__device__ __forceinline__ void flat_push(const int *off, int cnt, int E, Col colf, const Root &st,
+                                          uint32_t *mk, uint32_t Etag, Want want, F f, OnClaim onclaim,
+                                          int Ebeg = 0) {
+    const int tid = threadIdx.x;
+    for (int base = Ebeg; base < E; base += kBlock * kFlatU) {
+        const int e0 = base + tid * kFlatU;
+        int t[kFlatU], y[kFlatU], dy[kFlatU];
+        uint32_t mm[kFlatU], req[kFlatU];
+        int cur = -1;
+        if (e0 < E) {
+            int lo = 0, hi = cnt - 1;  // last row with off[row] <= e0
+            while (lo < hi) {
+                const int mid = (lo + hi + 1) >> 1;
+                if (off[mid] <= e0) lo = mid; else hi = mid - 1;
+            }
+            cur = lo;
+        }
+#pragma unroll
+        for (int u = 0; u < kFlatU; ++u) {
+            const int e = e0 + u;
+            t[u] = -1;
+            y[u] = 0;
+            if (e < E) {
+                while (off[cur + 1] <= e) ++cur;
+                t[u] = cur;
+                y[u] = colf(cur, e);
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < kFlatU; ++u)
+            dy[u] = (t[u] >= 0) ? (kCG ? __ldcg(st.d + y[u]) : st.dist(y[u])) : kInf;
+#pragma unroll
+        for (int u = 0; u < kFlatU; ++u)
+            mm[u] = (t[u] >= 0 && want(dy[u])) ? (kCG ? __ldcg(mk + y[u]) : mk[y[u]]) : 0u;
+#pragma unroll
+        for (int u = 0; u < kFlatU; ++u) req[u] = (t[u] >= 0) ? f(t[u], y[u], dy[u], mm[u]) : 0u;
+        uint32_t prev[kFlatU];
+#pragma unroll
+        for (int u = 0; u < kFlatU; ++u) prev[u] = req[u] ? atomicMax(mk + y[u], req[u]) : 0xffffffffu;
+#pragma unroll
+        for (int u = 0; u < kFlatU; ++u)
+            if (prev[u] < Etag) onclaim(y[u]);
+    }
+    __syncthreads();
+}
+
 // One push of a helped C2 pass (owner or helper): the same arithmetic as the
-// owner's up_visit / dpush_visit, with claims appended to the global list.
-__device__ __forceinline__ void help_push_entry(const GView &g, const ChunkSmem &M, int t, int pp, int dp,
-                                                double sp, uint32_t mp, const HelpCtx &cx, uint32_t *mark,
-                                                double *dacc, int32_t *gU, int *gapp,
-                                                uint32_t &bytes) {
-    if (dp != cx.l - 1) return;
+// owner's up_visit / dpush_visit; returns the claim request (flat_push issues
+// it and appends the claimed vertex to the global list).
+__device__ __forceinline__ uint32_t help_push_entry(const GView &g, const ChunkSmem &M, int t, int pp, int dp,
+                                                    uint32_t mp, const HelpCtx &cx, double *dacc,
+                                                    uint32_t &bytes) {
+    if (dp != cx.l - 1) return 0u;
     const uint32_t E = cx.E, mD = E | kDown, mU = E | kUp;
     const int meta = M.meta[t];
     double dlt;  // Ddelta[p] / sigma[p] (the accumulator is sigma-factored)
     if (meta & kMetaUp) {
         dlt = __ddiv_rn(M.c1[t], M.c0[t]);
     } else {
-        if (mp == mD) return;
+        if (mp == mD) return 0u;
         dlt = __ddiv_rn(1.0 + M.acc[t], M.c0[t]);
         if ((meta & kMetaNotPulled) && !((meta & kMetaNew) && new_edge(g, M.v[t], pp, cx.g0, cx.lim)))
             dlt = __dsub_rn(dlt, __ddiv_rn(1.0 + M.c1[t], M.c2[t]));
     }
-    (void)sp;
     atomicAdd(dacc + pp, dlt);
     bytes += 24;
-    if (mp >= E) return;
-    if (atomicMax(mark + pp, mU) >= E) return;
-    gU[atomicAdd(gapp, 1)] = pp;
+    return mp >= E ? 0u : mU;
 }
 
 // Entries [e0, e1) of a published chunk M (in this CTA's shared memory).
@@ -84,14 +132,13 @@ __device__ __forceinline__ void help_run_block(const ChunkSmem &M, int e0, int e
                                                const Root &st, uint32_t *mark, double *dacc, int32_t *gU,
                                                int *gapp, const HelpCtx &cx, uint32_t &bytes) {
     auto colf = [&](int t, int e) { return ldg_i(g.col + M.beg[t] + e - M.off[t]); };
-    flat_entries<kCG, false>(
-        M.off, cx.cnt, e1, colf, st, mark, [&](int dp) { return dp == cx.l - 1; }, nullptr,
-        [&](int t, int pp, int dp, double2 q, uint32_t mp) -> double {
+    flat_push<kCG>(
+        M.off, cx.cnt, e1, colf, st, mark, cx.E, [&](int dp) { return dp == cx.l - 1; },
+        [&](int t, int pp, int dp, uint32_t mp) -> uint32_t {
             if (M.meta[t] & kMetaUp) bytes += 8;  // D rows: counted by their C1 pull
-            help_push_entry(g, M, t, pp, dp, q.x, mp, cx, mark, dacc, gU, gapp, bytes);
-            return 0.0;
+            return help_push_entry(g, M, t, pp, dp, mp, cx, dacc, bytes);
         },
-        e0);
+        [&](int pp) { gU[atomicAdd(gapp, 1)] = pp; }, e0);
 }
 
 // ---------------------------------------------------------------------------
@@ -2222,20 +2269,33 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                 }
                                 __syncthreads();
                             } else if (push && E2 > 0)
-                                flat_entries<false, false>(  // pushes need no sigma of the target
-                                    I.off, nb, E2, colf, st, mark, [&](int dp) { return dp == l - 1; }, nullptr,
-                                    [&](int t, int pp, int dp, double2 q, uint32_t mp) -> double {
-                                        const double sp = q.x;
+                                flat_push<false>(  // pushes need no sigma of the target; claims batched
+                                    I.off, nb, E2, colf, st, mark, E, [&](int dp) { return dp == l - 1; },
+                                    [&](int t, int pp, int dp, uint32_t mp) -> uint32_t {
                                         (l == 2 ? sc_up2 : sc_up3)++;
                                         const int meta = I.meta[t];
                                         if (meta & kMetaUp) st_bytes += 8;  // D rows: counted by their C1 pull
-                                        if (dp != l - 1) return 0.0;
-                                        if (meta & kMetaUp)
-                                            up_visit(I.c1[t], I.c0[t], pp, sp, mp);
+                                        if (dp != l - 1) return 0u;
+                                        if (meta & kMetaUp) {
+                                            atomicAdd(dacc + pp, __ddiv_rn(I.c1[t], I.c0[t]));
+                                            st_bytes += 24;
+                                            return mp >= E ? 0u : mU;
+                                        }
+                                        if (mp == mD) return 0u;
+                                        double dlt = __ddiv_rn(1.0 + I.acc[t], I.c0[t]);
+                                        if ((meta & kMetaNotPulled) &&
+                                            !((meta & kMetaNew) && new_edge(g, I.v[t], pp, g0, lim)))
+                                            dlt = __dsub_rn(dlt, __ddiv_rn(1.0 + I.c1[t], I.c2[t]));
+                                        atomicAdd(dacc + pp, dlt);
+                                        st_bytes += 24;
+                                        return mp >= E ? 0u : mU;
+                                    },
+                                    [&](int y) {  // claimed: the next up frontier
+                                        const int pos = atomicAdd(&s_ucnt2[ucur_sel ^ 1], 1);
+                                        if (pos < kUcap)
+                                            s_un[ucur_sel ^ 1][pos] = y;
                                         else
-                                            dpush_visit(I.v[t], I.c0[t], I.acc[t], I.c1[t], I.c2[t], meta, pp, sp,
-                                                        mp);
-                                        return 0.0;
+                                            Unext[pos - kUcap] = y;
                                     });
                             tick(9);
                             trace(13, 0, s_nl1);
