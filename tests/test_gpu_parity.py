@@ -338,6 +338,59 @@ def test_error_paths_leave_state_unchanged():
         assert e.value.name == "DBC_ECAPACITY"
 
 
+def test_scenario_log_oversized_batch_leaves_state_unchanged():
+    """A batch larger than the scenario log is rejected before anything changes
+    (the live graph, d/sigma/delta, BC): a later insertion of the same edges
+    succeeds and matches the oracle."""
+    from paper_conf_ipps_mclaughlinb14_b200 import DBCError
+
+    wl = W.make_workload("karate")
+    with _dbc(wl.graph, wl.roots) as dbc:
+        dbc.static_compute()
+        bc0 = dbc.get_bc().copy()
+        st0 = [dbc.get_root_state(s) for s in (0, 5, 33)]
+        dbc.scenario_log(3)
+        with pytest.raises(DBCError) as e:
+            dbc.insert_edges(wl.ins_u[:5], wl.ins_v[:5])
+        assert e.value.name == "DBC_EINVAL"
+        assert np.array_equal(dbc.get_bc(), bc0)
+        for s, want in zip((0, 5, 33), st0):
+            for a, b in zip(dbc.get_root_state(s), want):
+                assert np.array_equal(a, b)
+        dbc.scenario_log(0)
+        dbc.insert_edges(wl.ins_u[:5], wl.ins_v[:5])  # not "already present": nothing was applied
+        ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
+        for u, v in zip(wl.ins_u[:5], wl.ins_v[:5]):
+            ref.insert(u, v)
+        check_all(dbc, ref.compute(), wl.roots.size)
+
+
+def test_device_deletions_ordered_on_the_context_stream():
+    """dbc_delete_edges_device reads a batch the caller wrote on the context
+    stream after work already queued there (the batch is read on that stream)."""
+    import torch
+
+    wl = W.make_workload("rmat10")
+    g = wl.graph
+    eu, ev = W.edges_of(g)
+    pick = np.random.default_rng(4).choice(eu.size, 6, replace=False)
+    du, dv = eu[pick].astype(np.int32), ev[pick].astype(np.int32)
+    stream = torch.cuda.Stream()
+    with torch.cuda.stream(stream):
+        with _dbc(g, wl.roots, stream=stream.cuda_stream) as dbc:
+            dbc.static_compute()
+            tu = torch.full((6,), -1, dtype=torch.int32, device="cuda")
+            tv = torch.full((6,), -1, dtype=torch.int32, device="cuda")
+            torch.cuda._sleep(50_000_000)  # keep the stream busy: the copies below land late
+            tu.copy_(torch.from_numpy(du).cuda(non_blocking=True))
+            tv.copy_(torch.from_numpy(dv).cuda(non_blocking=True))
+            dbc.delete_edges(tu, tv)
+            ref = oracle.NaiveDynamicBC(g, wl.roots)
+            for a, b in zip(du, dv):
+                ref.delete(int(a), int(b))
+            check_all(dbc, ref.compute(), wl.roots.size)
+
+
 # ------------------------------------------------- full size (configs[1]) ----
 def test_rmat16_full_size_batch_parity():
     """BASELINE configs[1] at full size, in the launch configuration bench.py times
