@@ -146,7 +146,13 @@ typedef struct {
     int32_t lean_short;      /* level-2 rows longer than this x deg(root) probe adj(root) */
     int32_t trace_slot;      /* -DDBC_PHASE_TIMERS builds: trace this root slot          */
     uint32_t disable;        /* DBC_TUNE_* bits                                          */
-    uint32_t reserved[8];    /* must be zero                                             */
+    int32_t static_ms;       /* static Brandes: 1 multi-source (32 roots per warp), 0 one
+                                root per CTA; automatic: multi-source on graphs of mean
+                                degree >= 8 (falls back to per-root when a BFS passes
+                                level 254 or its level lists overflow)                  */
+    int32_t static_groups;   /* multi-source: 32-root groups traversed together          */
+    int32_t static_chunk;    /* multi-source: row entries per warp task                  */
+    uint32_t reserved[5];    /* must be zero                                             */
 } dbc_tuning;
 #define DBC_TUNE_NO_HELP      0x1u  /* batch kernel: no cooperative help          */
 #define DBC_TUNE_NO_HEAVY     0x2u  /* batch kernel: no heavy lane                */

@@ -650,4 +650,36 @@ void launch_static_128(const StaticArgs &a, int workers, cudaStream_t s);
 void launch_static_512(const StaticArgs &a, int workers, cudaStream_t s);   // 64 regs, 2 CTAs/SM
 void launch_static_1024(const StaticArgs &a, int workers, cudaStream_t s);  // 64 regs, 1 CTA/SM
 
+// Multi-source static Brandes (msbrandes.cu): one wave of 32-root groups.
+struct MsArgs {
+    GView g;
+    int32_t n;
+    int32_t k_loc;
+    const int32_t *roots;
+    int32_t g0, ng;        // groups g0 .. g0 + ng - 1 (slots 32 g .. 32 g + 31)
+    double *sg;            // [ng][n][32] sigma, then q = (1 + delta) / sigma (zeroed)
+    uint32_t *vis;         // [ng][n] lanes that reached the vertex (zeroed)
+    uint32_t *nm;          // [ng][3][n] level masks, level j in array j % 3 (zeroed)
+    int32_t *vq;           // [ng][vcap] level lists (vertex)
+    uint32_t *vm;          // [ng][vcap] ... and its lanes at that level
+    int2 *tq;              // [ng][tcap] row-chunk tasks {vq index, chunk}
+    int32_t *toff;         // [ng][max levels + 3] first task of each level
+    int32_t *ctr;          // [ng] {vcount, tcount, overflow, pad} (zeroed)
+    unsigned *bar;         // grid barrier {count, generation} (zeroed)
+    int64_t vcap, tcap;
+    int32_t chunk;         // row entries per task
+    int32_t *d;            // root-major state (written for the wave's slots)
+    double2 *sd;
+    double *bc;
+    unsigned long long *stats;
+    int32_t *err;
+};
+int ms_static_threads();
+int ms_static_max_groups();
+int ms_static_max_levels();
+size_t ms_static_counter_bytes(int ng);
+int ms_static_resident(int nsm);
+cudaError_t launch_static_ms(const MsArgs &a, int grid, cudaStream_t s);
+void launch_static_l2mask(const StaticArgs &a, cudaStream_t s);
+
 }  // namespace dbc

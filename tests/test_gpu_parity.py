@@ -143,6 +143,91 @@ def test_static_other_widths_match_oracle(name, sblock, tune):
         check_all(dbc, ref, roots.size)
 
 
+MS_CASES = dict(STATIC_CASES)
+MS_CASES.update({
+    "smallworld_small": lambda: (W.make_workload("smallworld_small").graph,
+                                 W.make_workload("smallworld_small").roots),
+    "rmat10_all": lambda: (W.make_workload("rmat10").graph,
+                           np.arange(0, W.make_workload("rmat10").graph.n, 9, dtype=np.int32)),
+    "grid60_sigma": lambda: (W.grid_graph(60, 60), np.array([0, 61, 1830, 3599, 29], np.int32)),
+})
+
+
+@pytest.mark.parametrize("chunk", [None, "4"])
+@pytest.mark.parametrize("name", sorted(MS_CASES))
+def test_static_multisource_matches_oracle(name, chunk, tune):
+    """The multi-source static kernel (msbrandes.cu, 32 roots per warp) forced on
+    every graph: d and sigma bit-exact, delta 1e-12 (Eq. (2) regrouped as
+    sigma(w) * sum q(y)), BC 1e-9.  chunk 4 splits every row longer than 4
+    entries over several warp tasks (sigma partials added atomically, re-summed
+    in canonical order at or above 2^53: grid60 and big_sigma_hub reach 2^56
+    and more); one 32-root group per wave, so the roots of karate / rmat10_all
+    / disconnected run in several waves."""
+    tune["static_ms"] = 1
+    tune["static_groups"] = 1
+    if chunk:
+        tune["static_chunk"] = int(chunk)
+    g, roots = MS_CASES[name]()
+    roots = np.asarray(roots, np.int32)
+    ref = oracle.brandes_csr(g, roots)
+    with _dbc(g, roots) as dbc:
+        dbc.static_compute()
+        check_all(dbc, ref, roots.size)
+
+
+@pytest.mark.parametrize("chunk", [None, "4"])
+@pytest.mark.parametrize("name", ["rmat10_all", "grid60_sigma", "big_sigma_hub", "disconnected"])
+def test_static_multisource_pull_delta_is_bitwise(name, chunk, tune):
+    """DBC_FLAG_PULL_DELTA with the multi-source kernel requested: it regroups
+    Eq. (2), so the static pass falls back to the per-root kernel, whose delta
+    is bit-identical to the oracle."""
+    from paper_conf_ipps_mclaughlinb14_b200 import FLAG_PULL_DELTA
+
+    tune["static_ms"] = 1
+    if chunk:
+        tune["static_chunk"] = int(chunk)
+    g, roots = MS_CASES[name]()
+    roots = np.asarray(roots, np.int32)
+    bc_ref, d_ref, s_ref, dl_ref = oracle.brandes_csr(g, roots)
+    with _dbc(g, roots, flags=FLAG_PULL_DELTA) as dbc:
+        dbc.static_compute()
+        assert_bc(dbc.get_bc(), bc_ref)
+        for slot in range(roots.size):
+            d, s, dl = dbc.get_root_state(slot)
+            assert np.array_equal(d, d_ref[slot]) and np.array_equal(s, s_ref[slot])
+            assert np.array_equal(dl.view(np.int64), dl_ref[slot].view(np.int64)), f"delta slot {slot}"
+
+
+def test_static_multisource_deep_graph_falls_back(tune):
+    """A BFS deeper than 254 levels (byte levels) makes the multi-source kernel
+    give up; the per-root kernel recomputes and the result is still exact."""
+    tune["static_ms"] = 1
+    g = W.path_graph(600)
+    roots = np.array([0, 299, 599], np.int32)
+    ref = oracle.brandes_csr(g, roots)
+    with _dbc(g, roots) as dbc:
+        dbc.static_compute()
+        check_all(dbc, ref, roots.size)
+
+
+@pytest.mark.parametrize("name", ["rmat10", "smallworld_small"])
+def test_static_multisource_then_dynamic(name, tune):
+    """The multi-source state (and its level-2 masks) feeds the update kernels:
+    a stream of insertions after it matches the naive dynamic oracle."""
+    tune["static_ms"] = 1
+    wl = W.make_workload(name)
+    g, roots = wl.graph, wl.roots
+    ref = oracle.NaiveDynamicBC(g, roots)
+    with _dbc(g, roots) as dbc:
+        dbc.static_compute()
+        us, vs = wl.ins_u[:40], wl.ins_v[:40]
+        for b in range(0, 40, 10):
+            dbc.insert_edges(us[b:b + 10], vs[b:b + 10])
+            for u, v in zip(us[b:b + 10], vs[b:b + 10]):
+                ref.insert(int(u), int(v))
+        check_all(dbc, ref.compute(), roots.size)
+
+
 def test_static_no_edges_and_zero_roots():
     g = W.csr_from_edges(5, [], [])
     with _dbc(g, np.array([0, 3], np.int32)) as dbc:
