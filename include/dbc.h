@@ -152,7 +152,8 @@ typedef struct {
                                 level 254 or its level lists overflow)                  */
     int32_t static_groups;   /* multi-source: 32-root groups traversed together          */
     int32_t static_chunk;    /* multi-source: row entries per warp task                  */
-    uint32_t reserved[5];    /* must be zero                                             */
+    int32_t static_width;    /* multi-source: roots per group, 32 or 64 (two per lane)   */
+    uint32_t reserved[4];    /* must be zero                                             */
 } dbc_tuning;
 #define DBC_TUNE_NO_HELP      0x1u  /* batch kernel: no cooperative help          */
 #define DBC_TUNE_NO_HEAVY     0x2u  /* batch kernel: no heavy lane                */

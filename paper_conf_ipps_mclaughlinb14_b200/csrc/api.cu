@@ -236,7 +236,7 @@ void dbc_tuning_default(dbc_tuning *t) {
     t->help_down_min = t->help_down_block = t->help_entries = t->help_min_blocks = -1;
     t->busy_help = t->busy_min = t->down_long_min = t->wide_inlane = -1;
     t->lean_block = t->lean_workers = t->lean_max_batch = t->lean_short = t->trace_slot = -1;
-    t->static_ms = t->static_groups = t->static_chunk = -1;
+    t->static_ms = t->static_groups = t->static_chunk = t->static_width = -1;
     t->heavy_factor = 0.0f;
 }
 
@@ -828,14 +828,19 @@ static StaticArgs static_args(dbc_ctx *c) {
 static dbc_status static_ms(dbc_ctx *c, bool *done) {
     *done = false;
     const size_t n = (size_t)c->n;
-    const int ng_all = (c->k_loc + 31) / 32;
+    // roots per group: 64 (two per lane, one 64-bit mask) once there are more
+    // than 32 roots, else 32
+    const int R = c->tune.static_width == 32 ? 1 : c->tune.static_width == 64 ? 2 : (c->k_loc > 32 ? 2 : 1);
+    const int G = 32 * R;
+    const size_t mb = 4 * (size_t)R;  // bytes per mask
+    const int ng_all = (c->k_loc + G - 1) / G;
     if (ng_all == 0 || n == 0) return DBC_OK;
-    // row entries per task: 16 (R-MAT 16, mean degree 13), 32 from mean degree 24 (Kronecker 20)
-    const int T = c->tune.static_chunk > 0 ? c->tune.static_chunk : (c->nnz >= 24 * (int64_t)n ? 32 : 16);
+    // row entries per task: 16 (R-MAT 16, mean degree 13), 64 from mean degree 24 (Kronecker 20)
+    const int T = c->tune.static_chunk > 0 ? c->tune.static_chunk : (c->nnz >= 24 * (int64_t)n ? 64 : 16);
     const int64_t vcap = std::min<int64_t>((int64_t)n * 12, INT32_MAX / 2);
     const int64_t tcap = std::min<int64_t>(vcap + 12 * (c->nnz / T) + 1024, INT32_MAX / 2);
     const int nlev = ms_static_max_levels() + 3;
-    const size_t per_group = n * (256 + 4 + 12) + (size_t)vcap * 8 + (size_t)tcap * 8 +
+    const size_t per_group = n * (8 * G + 4 * mb) + (size_t)vcap * (4 + mb) + (size_t)tcap * 8 +
                              (size_t)nlev * 4 + ms_static_counter_bytes(1);
     int wave = std::min(ng_all, ms_static_max_groups());
     if (c->tune.static_groups > 0) {
@@ -845,7 +850,7 @@ static dbc_status static_ms(dbc_ctx *c, bool *done) {
         CK(cudaMemGetInfo(&fr, &tot));
         wave = (int)std::min<size_t>((size_t)wave, (fr / 2) / per_group);
     }
-    const int grid = ms_static_resident(c->nsm);
+    const int grid = ms_static_resident(c->nsm, R);
     if (wave < 1 || grid < 1) return DBC_OK;
     MsArgs m;
     m.g = view_of(c);
@@ -861,7 +866,7 @@ static dbc_status static_ms(dbc_ctx *c, bool *done) {
     m.stats = c->stats;
     m.err = c->err;
     const size_t W = (size_t)wave;
-    const size_t sz[] = {W * n * 32 * 8, W * n * 4, W * n * 12, W * (size_t)vcap * 4, W * (size_t)vcap * 4,
+    const size_t sz[] = {W * n * G * 8, W * n * mb, W * n * 3 * mb, W * (size_t)vcap * 4, W * (size_t)vcap * mb,
                          W * (size_t)tcap * 8, W * (size_t)nlev * 4, ms_static_counter_bytes(wave),
                          2 * sizeof(unsigned)};
     constexpr int kBufs = sizeof(sz) / sizeof(sz[0]);
@@ -875,10 +880,10 @@ static dbc_status static_ms(dbc_ctx *c, bool *done) {
             return DBC_OK;  // no room: the per-root kernel
         }
     m.sg = (double *)buf[0];
-    m.vis = (uint32_t *)buf[1];
-    m.nm = (uint32_t *)buf[2];
+    m.vis = buf[1];
+    m.nm = buf[2];
     m.vq = (int32_t *)buf[3];
-    m.vm = (uint32_t *)buf[4];
+    m.vm = buf[4];
     m.tq = (int2 *)buf[5];
     m.toff = (int32_t *)buf[6];
     m.ctr = (int32_t *)buf[7];
@@ -897,13 +902,13 @@ static dbc_status static_ms(dbc_ctx *c, bool *done) {
     for (int g0 = 0; g0 < ng_all && ok && e == cudaSuccess; g0 += wave) {
         m.g0 = g0;
         m.ng = std::min(wave, ng_all - g0);
-        const size_t G = (size_t)m.ng;
-        e = cudaMemsetAsync(m.sg, 0, G * n * 32 * 8, c->stream);
-        if (e == cudaSuccess) e = cudaMemsetAsync(m.vis, 0, G * n * 4, c->stream);
-        if (e == cudaSuccess) e = cudaMemsetAsync(m.nm, 0, G * n * 12, c->stream);
+        const size_t Gn = (size_t)m.ng;
+        e = cudaMemsetAsync(m.sg, 0, Gn * n * G * 8, c->stream);
+        if (e == cudaSuccess) e = cudaMemsetAsync(m.vis, 0, Gn * n * mb, c->stream);
+        if (e == cudaSuccess) e = cudaMemsetAsync(m.nm, 0, Gn * n * 3 * mb, c->stream);
         if (e == cudaSuccess) e = cudaMemsetAsync(m.ctr, 0, ms_static_counter_bytes(m.ng), c->stream);
         if (e == cudaSuccess) e = cudaMemsetAsync(m.bar, 0, 2 * sizeof(unsigned), c->stream);
-        if (e == cudaSuccess) e = launch_static_ms(m, grid, c->stream);
+        if (e == cudaSuccess) e = launch_static_ms(m, R, grid, c->stream);
         if (e == cudaSuccess)
             e = cudaMemcpyAsync(ctr.data(), m.ctr, ms_static_counter_bytes(m.ng), cudaMemcpyDeviceToHost,
                                 c->stream);

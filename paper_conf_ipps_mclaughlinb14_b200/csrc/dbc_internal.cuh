@@ -656,12 +656,13 @@ struct MsArgs {
     int32_t n;
     int32_t k_loc;
     const int32_t *roots;
-    int32_t g0, ng;        // groups g0 .. g0 + ng - 1 (slots 32 g .. 32 g + 31)
-    double *sg;            // [ng][n][32] sigma, then q = (1 + delta) / sigma (zeroed)
-    uint32_t *vis;         // [ng][n] lanes that reached the vertex (zeroed)
-    uint32_t *nm;          // [ng][3][n] level masks, level j in array j % 3 (zeroed)
+    int32_t g0, ng;        // groups g0 .. g0 + ng - 1 (slots 32 R g .. 32 R g + 32 R - 1)
+    double *sg;            // [ng][n][32 R] sigma, then q = (1 + delta) / sigma (zeroed)
+    // masks over the 32 R roots of a group (R = 1: uint32, R = 2: uint64)
+    void *vis;             // [ng][n] roots that reached the vertex (zeroed)
+    void *nm;              // [ng][3][n] level masks, level j in array j % 3 (zeroed)
     int32_t *vq;           // [ng][vcap] level lists (vertex)
-    uint32_t *vm;          // [ng][vcap] ... and its lanes at that level
+    void *vm;              // [ng][vcap] ... and its roots at that level
     int2 *tq;              // [ng][tcap] row-chunk tasks {vq index, chunk}
     int32_t *toff;         // [ng][max levels + 3] first task of each level
     int32_t *ctr;          // [ng] {vcount, tcount, overflow, pad} (zeroed)
@@ -674,12 +675,11 @@ struct MsArgs {
     unsigned long long *stats;
     int32_t *err;
 };
-int ms_static_threads();
 int ms_static_max_groups();
 int ms_static_max_levels();
 size_t ms_static_counter_bytes(int ng);
-int ms_static_resident(int nsm);
-cudaError_t launch_static_ms(const MsArgs &a, int grid, cudaStream_t s);
+int ms_static_resident(int nsm, int r);  // r = roots per lane (1 or 2)
+cudaError_t launch_static_ms(const MsArgs &a, int r, int grid, cudaStream_t s);
 void launch_static_l2mask(const StaticArgs &a, cudaStream_t s);
 
 }  // namespace dbc

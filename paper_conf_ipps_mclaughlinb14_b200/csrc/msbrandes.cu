@@ -44,6 +44,17 @@ constexpr int kMsMaxG = 64;      // groups per wave (lockstep)
 constexpr int kMsMaxLev = 254;   // deeper BFS: the per-root kernel
 constexpr int kMsUnroll = 8;     // contributing entries whose gathers are in flight together
 
+// R roots per lane (a group of 32 R roots): lane l holds roots l + 32 j, j < R;
+// a vertex's lanes at a level form one R * 32-bit mask.
+template <int R> struct MaskOf;
+template <> struct MaskOf<1> { using T = uint32_t; };
+template <> struct MaskOf<2> { using T = unsigned long long; };
+__device__ __forceinline__ int popc_m(uint32_t x) { return __popc(x); }
+__device__ __forceinline__ int popc_m(unsigned long long x) { return __popcll(x); }
+__device__ __forceinline__ int ffs_m(uint32_t x) { return __ffs(x); }
+__device__ __forceinline__ int ffs_m(unsigned long long x) { return __ffsll(x); }
+template <class Mk> __device__ __forceinline__ bool bit(Mk m, int b) { return (m >> b) & 1u; }
+
 struct MsGroup {  // per-group counters (device)
     int vcount, tcount, overflow, pad;
 };
@@ -89,22 +100,25 @@ __device__ __forceinline__ int2 full_row(const GView &g, int v) {
     return make_int2(ldg_i(g.rp + v) & kMask, ldg_i(g.rp + v + 1) & kMask);
 }
 
+template <int R>
 struct Ms {
+    using Mk = typename MaskOf<R>::T;
+    static constexpr int G = 32 * R;  // roots per group
     const MsArgs &a;
     size_t n;
     int lane, gw, W;
-    // sigma of (vertex, lane); after the vertex's delta is final: q = (1 + delta) / sigma
-    __device__ double *sg(int grp) const { return a.sg + (size_t)grp * n * 32; }
-    __device__ uint32_t *vis(int grp) const { return a.vis + (size_t)grp * n; }
-    // level masks: nm(grp, j)[v] = lanes whose root has v at level j (array j % 3)
-    __device__ uint32_t *nm(int grp, int j) const { return a.nm + ((size_t)grp * 3 + (j % 3)) * n; }
+    // sigma of (vertex, root); after the vertex's delta is final: q = (1 + delta) / sigma
+    __device__ double *sg(int grp) const { return a.sg + (size_t)grp * n * G; }
+    __device__ Mk *vis(int grp) const { return reinterpret_cast<Mk *>(a.vis) + (size_t)grp * n; }
+    // level masks: nm(grp, j)[v] = roots with v at level j (array j % 3)
+    __device__ Mk *nm(int grp, int j) const { return reinterpret_cast<Mk *>(a.nm) + ((size_t)grp * 3 + (j % 3)) * n; }
     __device__ int32_t *vq(int grp) const { return a.vq + (size_t)grp * a.vcap; }
-    __device__ uint32_t *vm(int grp) const { return a.vm + (size_t)grp * a.vcap; }
+    __device__ Mk *vm(int grp) const { return reinterpret_cast<Mk *>(a.vm) + (size_t)grp * a.vcap; }
     __device__ int2 *tq(int grp) const { return a.tq + (size_t)grp * a.tcap; }
     __device__ int32_t *toff(int grp) const { return a.toff + (size_t)grp * (kMsMaxLev + 3); }
     __device__ MsGroup *ctr(int grp) const { return reinterpret_cast<MsGroup *>(a.ctr) + grp; }
-    // root-major state index of lane r of group grp
-    __device__ size_t st(int grp, int r, int v) const { return (size_t)((a.g0 + grp) * 32 + r) * n + v; }
+    // root-major state index of root b of group grp
+    __device__ size_t st(int grp, int b, int v) const { return (size_t)((a.g0 + grp) * G + b) * n + v; }
 
     // append w (first claimer) to the next level: its vertex entry and its row chunks
     __device__ void append(int grp, int w) const {
@@ -138,15 +152,17 @@ __device__ __forceinline__ int group_of(const int *s_pref, int ng, int t) {
 
 // Lane i's task of the warp's batch of 32; off = exclusive prefix of the
 // chunk lengths (entry e of the batch belongs to the largest i with off_i <= e).
+template <class Mk>
 struct Task {
     int grp, vi, w, chunk, deg, beg, len, off;
-    uint32_t m;
+    Mk m;
     bool valid;
 };
 
-__device__ __forceinline__ Task load_task(const Ms &M, const int *s_pref, const int *s_lo, int ng, int t,
-                                          int total, int T) {
-    Task k{};
+template <int R>
+__device__ __forceinline__ Task<typename MaskOf<R>::T> load_task(const Ms<R> &M, const int *s_pref, const int *s_lo,
+                                                                 int ng, int t, int total, int T) {
+    Task<typename MaskOf<R>::T> k{};
     k.valid = t < total;
     if (k.valid) {
         k.grp = group_of(s_pref, ng, t);
@@ -162,7 +178,8 @@ __device__ __forceinline__ Task load_task(const Ms &M, const int *s_pref, const 
     return k;
 }
 
-__device__ __forceinline__ int scan_len(Task &k, int lane) {
+template <class Tk>
+__device__ __forceinline__ int scan_len(Tk &k, int lane) {
     int x = k.len;
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
@@ -184,7 +201,8 @@ __device__ __forceinline__ int task_of(int off, int e) {
 }
 
 // Block-wide: s_lo / s_pref over the groups for the tasks toff[j] .. toff[j+1].
-__device__ __forceinline__ void level_tasks(const Ms &M, int ng, int j, int *s_pref, int *s_lo) {
+template <class MsT>
+__device__ __forceinline__ void level_tasks(const MsT &M, int ng, int j, int *s_pref, int *s_lo) {
     if (threadIdx.x < ng) {
         const int *to = M.toff(threadIdx.x);
         s_lo[threadIdx.x] = __ldcg(to + j);
@@ -199,16 +217,17 @@ __device__ __forceinline__ void level_tasks(const Ms &M, int ng, int j, int *s_p
 }
 
 // nm(j)[v] = 0 for the vertices of level j (their chunk-0 tasks), all groups.
-__device__ __forceinline__ void clear_level(const Ms &M, int ng, int j) {
+template <class MsT>
+__device__ __forceinline__ void clear_level(const MsT &M, int ng, int j) {
     if (j < 0) return;
     const int tid = blockIdx.x * kMsThreads + threadIdx.x;
     const int nth = gridDim.x * kMsThreads;
     for (int grp = 0; grp < ng; ++grp) {
         const int lo = __ldcg(M.toff(grp) + j), hi = __ldcg(M.toff(grp) + j + 1);
-        uint32_t *nm = M.nm(grp, j);
+        auto *nm = M.nm(grp, j);
         for (int t = lo + tid; t < hi; t += nth) {
             const int2 tk = __ldcg(M.tq(grp) + t);
-            if (tk.y == 0) nm[__ldcg(M.vq(grp) + tk.x)] = 0u;
+            if (tk.y == 0) nm[__ldcg(M.vq(grp) + tk.x)] = 0;
         }
     }
 }
@@ -219,12 +238,16 @@ __device__ __forceinline__ double warp_sum(double x) {
     return x;
 }
 
+template <int R>
 __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
+    using Mk = typename MaskOf<R>::T;
+    constexpr int G = 32 * R;
+    constexpr int U = kMsUnroll / R;  // contributing entries in flight (R gathers each)
     __shared__ int s_pref[kMsMaxG + 1];
     __shared__ int s_lo[kMsMaxG];
     __shared__ int s_done;
-    Ms M{a, (size_t)a.n, (int)(threadIdx.x & 31), (int)((blockIdx.x * kMsThreads + threadIdx.x) >> 5),
-         (int)((gridDim.x * kMsThreads) >> 5)};
+    Ms<R> M{a, (size_t)a.n, (int)(threadIdx.x & 31), (int)((blockIdx.x * kMsThreads + threadIdx.x) >> 5),
+            (int)((gridDim.x * kMsThreads) >> 5)};
     const int lane = M.lane;
     const int ng = a.ng;
     const GView &g = a.g;
@@ -234,7 +257,7 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
 
     // ---- Alg. 1 lines 3-9: d = INF, sigma = delta = 0 for the wave's slots
     {
-        const int s0 = a.g0 * 32, s1 = min(a.k_loc, (a.g0 + ng) * 32);
+        const int s0 = a.g0 * G, s1 = min(a.k_loc, (a.g0 + ng) * G);
         const size_t tot = (size_t)(s1 - s0) * n;
         int32_t *d = a.d + (size_t)s0 * n;
         double2 *sd = a.sd + (size_t)s0 * n;
@@ -249,23 +272,27 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
     // ---- level 0: the roots (one warp per group)
     if (M.gw < ng) {
         const int grp = M.gw;
-        const int slot = (a.g0 + grp) * 32 + lane;
-        const bool valid = slot < a.k_loc;
-        const int s = valid ? a.roots[slot] : -1;
-        if (valid) {  // roots are distinct (dbc_create)
-            M.sg(grp)[(size_t)s * 32 + lane] = 1.0;
-            a.d[(size_t)slot * n + s] = 0;
-            a.sd[(size_t)slot * n + s] = make_double2(1.0, 0.0);
-            const int vi = atomicAdd(&M.ctr(grp)->vcount, 1);
-            M.vq(grp)[vi] = s;
-            M.vm(grp)[vi] = 1u << lane;
-            M.vis(grp)[s] = 1u << lane;
-            M.nm(grp, 0)[s] = 1u << lane;
-            const int2 r = full_row(g, s);
-            const int deg = r.y - r.x;
-            const int nch = deg > T ? (deg + T - 1) / T : 1;
-            const int ti = atomicAdd(&M.ctr(grp)->tcount, nch);
-            for (int k = 0; k < nch; ++k) M.tq(grp)[ti + k] = make_int2(vi, k);
+#pragma unroll
+        for (int j = 0; j < R; ++j) {
+            const int b = lane + 32 * j;
+            const int slot = (a.g0 + grp) * G + b;
+            if (slot < a.k_loc) {  // roots are distinct (dbc_create)
+                const int s = a.roots[slot];
+                M.sg(grp)[(size_t)s * G + b] = 1.0;
+                a.d[(size_t)slot * n + s] = 0;
+                a.sd[(size_t)slot * n + s] = make_double2(1.0, 0.0);
+                const Mk mb = (Mk)1 << b;
+                const int vi = atomicAdd(&M.ctr(grp)->vcount, 1);
+                M.vq(grp)[vi] = s;
+                M.vm(grp)[vi] = mb;
+                M.vis(grp)[s] = mb;
+                M.nm(grp, 0)[s] = mb;
+                const int2 r = full_row(g, s);
+                const int deg = r.y - r.x;
+                const int nch = deg > T ? (deg + T - 1) / T : 1;
+                const int ti = atomicAdd(&M.ctr(grp)->tcount, nch);
+                for (int k = 0; k < nch; ++k) M.tq(grp)[ti + k] = make_int2(vi, k);
+            }
         }
         __syncwarp();
         if (lane == 0) {
@@ -281,7 +308,7 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
         // ---- pass A: expand level L (tasks toff[L] .. toff[L+1])
         level_tasks(M, ng, L, s_pref, s_lo);
         for (int t0 = M.gw * 32; t0 < s_pref[ng]; t0 += M.W * 32) {
-            Task k = load_task(M, s_pref, s_lo, ng, t0 + lane, s_pref[ng], T);
+            auto k = load_task(M, s_pref, s_lo, ng, t0 + lane, s_pref[ng], T);
             if (k.valid) k.m = __ldcg(M.vm(k.grp) + k.vi);
             // sigma of a split row (chunk partials added atomically): exact below
             // 2^53; at or above it, re-summed in canonical order; then stored
@@ -290,24 +317,38 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
                 const int i = __ffs(fix) - 1;
                 fix &= fix - 1;
                 const int grp = __shfl_sync(kFull, k.grp, i), u = __shfl_sync(kFull, k.w, i);
-                const bool act = (__shfl_sync(kFull, k.m, i) >> lane) & 1u;
-                double *su = M.sg(grp) + (size_t)u * 32 + lane;
-                double sum = act ? __ldcg(su) : 0.0;
-                const bool big = act && sum >= kExact;
-                if (__any_sync(kFull, big)) {
-                    const int2 r = full_row(g, u);
-                    const uint32_t *pm = M.nm(grp, L - 1);
-                    double s2 = 0.0;
-                    for (int j = r.x; j < r.y; ++j) {
-                        const int x = ldg_i(g.col + j);
-                        if (big && ((__ldcg(pm + x) >> lane) & 1u)) s2 += __ldcg(M.sg(grp) + (size_t)x * 32 + lane);
-                    }
-                    if (big) {
-                        sum = s2;
-                        *su = sum;
-                    }
+                const Mk mu = __shfl_sync(kFull, k.m, i);
+                double sum[R];
+                bool big[R], anyb = false;
+#pragma unroll
+                for (int j = 0; j < R; ++j) {
+                    const int b = lane + 32 * j;
+                    sum[j] = bit(mu, b) ? __ldcg(M.sg(grp) + (size_t)u * G + b) : 0.0;
+                    big[j] = bit(mu, b) && sum[j] >= kExact;
+                    anyb |= big[j];
                 }
-                if (act) a.sd[M.st(grp, lane, u)].x = sum;
+                if (__any_sync(kFull, anyb)) {
+                    const int2 r = full_row(g, u);
+                    const Mk *pm = M.nm(grp, L - 1);
+                    double s2[R] = {};
+                    for (int jj = r.x; jj < r.y; ++jj) {
+                        const int x = ldg_i(g.col + jj);
+                        const Mk px = anyb ? __ldcg(pm + x) : (Mk)0;
+#pragma unroll
+                        for (int j = 0; j < R; ++j)
+                            if (big[j] && bit(px, lane + 32 * j))
+                                s2[j] += __ldcg(M.sg(grp) + (size_t)x * G + lane + 32 * j);
+                    }
+#pragma unroll
+                    for (int j = 0; j < R; ++j)
+                        if (big[j]) {
+                            sum[j] = s2[j];
+                            M.sg(grp)[(size_t)u * G + lane + 32 * j] = sum[j];
+                        }
+                }
+#pragma unroll
+                for (int j = 0; j < R; ++j)
+                    if (bit(mu, lane + 32 * j)) a.sd[M.st(grp, lane + 32 * j, u)].x = sum[j];
             }
             const int E = scan_len(k, lane);
             for (int base = 0; base < E; base += 32) {
@@ -315,13 +356,13 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
                 const int i = task_of(k.off, e);
                 const int gi = __shfl_sync(kFull, k.grp, i), bi = __shfl_sync(kFull, k.beg, i);
                 const int oi = __shfl_sync(kFull, k.off, i);
-                const uint32_t mi = __shfl_sync(kFull, k.m, i);
+                const Mk mi = __shfl_sync(kFull, k.m, i);
                 if (e < E) {
                     const int w = ldg_i(g.col + bi + e - oi);
-                    const uint32_t nmk = mi & ~__ldcg(M.vis(gi) + w);
+                    const Mk nmk = mi & ~__ldcg(M.vis(gi) + w);
                     if (nmk) {
-                        const uint32_t old = atomicOr(M.nm(gi, L + 1) + w, nmk);
-                        if (old == 0u) M.append(gi, w);
+                        const Mk old = atomicOr(M.nm(gi, L + 1) + w, nmk);
+                        if (old == 0) M.append(gi, w);
                     }
                 }
             }
@@ -356,33 +397,37 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
         // ---- pass B: sigma pull of level Lc from level L (canonical order)
         clear_level(M, ng, Lc - 2);  // nm(Lc - 2) is pass A(Lc)'s discovery array
         for (int t0 = M.gw * 32; t0 < s_pref[ng]; t0 += M.W * 32) {
-            Task k = load_task(M, s_pref, s_lo, ng, t0 + lane, s_pref[ng], T);
+            auto k = load_task(M, s_pref, s_lo, ng, t0 + lane, s_pref[ng], T);
             if (k.valid) {
                 k.m = __ldcg(M.nm(k.grp, Lc) + k.w);
-                bytes += (unsigned long long)__popc(k.m) * 8ull * k.len;  // col + d per entry
+                bytes += (unsigned long long)popc_m(k.m) * 8ull * k.len;  // col + d per entry
                 if (k.chunk == 0) {  // the vertex's level-Lc record
                     M.vm(k.grp)[k.vi] = k.m;
                     M.vis(k.grp)[k.w] = __ldcg(M.vis(k.grp) + k.w) | k.m;
-                    for (uint32_t b = k.m; b; b &= b - 1) a.d[M.st(k.grp, __ffs(b) - 1, k.w)] = Lc;
-                    bytes += (unsigned long long)__popc(k.m) * (16 + 4);  // row bounds, sigma and d writes
+                    for (Mk b = k.m; b; b &= b - 1) a.d[M.st(k.grp, ffs_m(b) - 1, k.w)] = Lc;
+                    bytes += (unsigned long long)popc_m(k.m) * (16 + 4);  // row bounds, sigma and d writes
                 }
             }
             const int E = scan_len(k, lane);
             int cur = -1;
-            double sum = 0.0;
+            double sum[R];
             auto flush = [&]() {  // sigma of task cur (uniform)
                 const int gc = __shfl_sync(kFull, k.grp, cur), wc = __shfl_sync(kFull, k.w, cur);
-                const uint32_t mc = __shfl_sync(kFull, k.m, cur);
+                const Mk mc = __shfl_sync(kFull, k.m, cur);
                 const bool split = __shfl_sync(kFull, k.deg, cur) > T;
-                if ((mc >> lane) & 1u) {
-                    double *sw = M.sg(gc) + (size_t)wc * 32 + lane;
-                    if (split) {
-                        atomicAdd(sw, sum);
-                    } else {
-                        *sw = sum;
-                        a.sd[M.st(gc, lane, wc)].x = sum;
+#pragma unroll
+                for (int j = 0; j < R; ++j) {
+                    const int b = lane + 32 * j;
+                    if (bit(mc, b)) {
+                        double *sw = M.sg(gc) + (size_t)wc * G + b;
+                        if (split) {
+                            atomicAdd(sw, sum[j]);
+                        } else {
+                            *sw = sum[j];
+                            a.sd[M.st(gc, b, wc)].x = sum[j];
+                        }
+                        if (!(sum[j] <= 1.7976931348623157e308)) atomicOr(a.err, kErrNumeric);
                     }
-                    if (!(sum <= 1.7976931348623157e308)) atomicOr(a.err, kErrNumeric);
                 }
             };
             for (int base = 0; base < E; base += 32) {
@@ -390,36 +435,39 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
                 const int i = task_of(k.off, e);
                 const int gi = __shfl_sync(kFull, k.grp, i), bi = __shfl_sync(kFull, k.beg, i);
                 const int oi = __shfl_sync(kFull, k.off, i);
-                const uint32_t mi = __shfl_sync(kFull, k.m, i);
+                const Mk mi = __shfl_sync(kFull, k.m, i);
                 const int x = e < E ? ldg_i(g.col + bi + e - oi) : 0;
-                const uint32_t pm = e < E ? (__ldcg(M.nm(gi, L) + x) & mi) : 0u;
-                uint32_t todo = __ballot_sync(kFull, pm != 0u);
+                const Mk pm = e < E ? (__ldcg(M.nm(gi, L) + x) & mi) : (Mk)0;
+                bytes += 8ull * popc_m(pm);  // sigma of a predecessor (per root)
+                uint32_t todo = __ballot_sync(kFull, pm != 0);
                 while (todo) {
-                    int ts[kMsUnroll];
-                    uint32_t bits[kMsUnroll];
-                    double sx[kMsUnroll];
+                    int ts[U];
+                    Mk bits[U];
+                    double sx[U][R];
 #pragma unroll
-                    for (int q = 0; q < kMsUnroll; ++q) {
+                    for (int q = 0; q < U; ++q) {
                         const int kk = __ffs(todo) - 1;  // -1: past the last one
                         todo &= todo - 1;
                         const int xs = __shfl_sync(kFull, x, kk & 31);
                         const int gs = __shfl_sync(kFull, gi, kk & 31);
                         ts[q] = kk < 0 ? -1 : __shfl_sync(kFull, i, kk & 31);
-                        bits[q] = kk < 0 ? 0u : __shfl_sync(kFull, pm, kk & 31);
-                        sx[q] = ((bits[q] >> lane) & 1u) ? __ldcg(M.sg(gs) + (size_t)xs * 32 + lane) : 0.0;
+                        bits[q] = kk < 0 ? (Mk)0 : __shfl_sync(kFull, pm, kk & 31);
+                        const double *sp = M.sg(gs) + (size_t)xs * G + lane;
+#pragma unroll
+                        for (int j = 0; j < R; ++j) sx[q][j] = bit(bits[q], lane + 32 * j) ? __ldcg(sp + 32 * j) : 0.0;
                     }
 #pragma unroll
-                    for (int q = 0; q < kMsUnroll; ++q) {
+                    for (int q = 0; q < U; ++q) {
                         if (ts[q] < 0) break;
                         if (ts[q] != cur) {
                             if (cur >= 0) flush();
                             cur = ts[q];
-                            sum = 0.0;
+#pragma unroll
+                            for (int j = 0; j < R; ++j) sum[j] = 0.0;
                         }
-                        if ((bits[q] >> lane) & 1u) {
-                            sum += sx[q];
-                            bytes += 8;
-                        }
+#pragma unroll
+                        for (int j = 0; j < R; ++j)
+                            if (bit(bits[q], lane + 32 * j)) sum[j] += sx[q][j];
                     }
                 }
             }
@@ -440,75 +488,86 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
         level_tasks(M, ng, Lc, s_pref, s_lo);
         if (Lc + 2 <= maxlev) clear_level(M, ng, Lc + 2);
         for (int t0 = M.gw * 32; t0 < s_pref[ng]; t0 += M.W * 32) {
-            Task k = load_task(M, s_pref, s_lo, ng, t0 + lane, s_pref[ng], T);
+            auto k = load_task(M, s_pref, s_lo, ng, t0 + lane, s_pref[ng], T);
             if (k.valid) {
                 k.m = __ldcg(M.vm(k.grp) + k.vi);
                 if (k.chunk == 0) M.nm(k.grp, Lc)[k.w] = k.m;
-                bytes += (unsigned long long)__popc(k.m) * (8ull * k.len + (k.chunk == 0 ? 48 : 0));
+                bytes += (unsigned long long)popc_m(k.m) * (8ull * k.len + (k.chunk == 0 ? 48 : 0));
             }
             const int E = scan_len(k, lane);
             int cur = -1;
             uint32_t seen = 0;  // tasks of the batch that had successors
-            double acc = 0.0, sv = 1.0;
+            double acc[R], sv[R];
             auto flush = [&]() {  // delta (and q) of task cur (uniform)
                 const int gc = __shfl_sync(kFull, k.grp, cur), wc = __shfl_sync(kFull, k.w, cur);
-                const uint32_t mc = __shfl_sync(kFull, k.m, cur);
+                const Mk mc = __shfl_sync(kFull, k.m, cur);
                 const bool split = __shfl_sync(kFull, k.deg, cur) > T;
-                const bool act = (mc >> lane) & 1u;
-                const double dl = act ? __dmul_rn(sv, acc) : 0.0;
-                if (split) {  // a chunk's partial: q and BC once the pass is over
-                    if (act && acc != 0.0) atomicAdd(&a.sd[M.st(gc, lane, wc)].y, dl);
-                } else {
-                    if (act) {
-                        a.sd[M.st(gc, lane, wc)].y = dl;
-                        M.sg(gc)[(size_t)wc * 32 + lane] = __ddiv_rn(__dadd_rn(1.0, dl), sv);
+                double bsum = 0.0;
+#pragma unroll
+                for (int j = 0; j < R; ++j) {
+                    const int b = lane + 32 * j;
+                    const bool act = bit(mc, b);
+                    const double dl = act ? __dmul_rn(sv[j], acc[j]) : 0.0;
+                    if (split) {  // a chunk's partial: q and BC once the pass is over
+                        if (act && acc[j] != 0.0) atomicAdd(&a.sd[M.st(gc, b, wc)].y, dl);
+                    } else if (act) {
+                        a.sd[M.st(gc, b, wc)].y = dl;
+                        M.sg(gc)[(size_t)wc * G + b] = __ddiv_rn(__dadd_rn(1.0, dl), sv[j]);
+                        bsum += dl;
                     }
-                    const double bsum = warp_sum(dl);
+                }
+                if (!split) {
+                    bsum = warp_sum(bsum);
                     if (lane == 0 && bsum != 0.0) atomicAdd(a.bc + wc, bsum);
                 }
             };
             auto begin = [&](int c) {  // task c becomes current: prefetch its sigma
                 cur = c;
-                acc = 0.0;
                 seen |= 1u << c;
                 const int gc = __shfl_sync(kFull, k.grp, c), wc = __shfl_sync(kFull, k.w, c);
-                const bool act = (__shfl_sync(kFull, k.m, c) >> lane) & 1u;
-                sv = act ? __ldcg(M.sg(gc) + (size_t)wc * 32 + lane) : 1.0;
+                const Mk mc = __shfl_sync(kFull, k.m, c);
+#pragma unroll
+                for (int j = 0; j < R; ++j) {
+                    acc[j] = 0.0;
+                    sv[j] = bit(mc, lane + 32 * j) ? __ldcg(M.sg(gc) + (size_t)wc * G + lane + 32 * j) : 1.0;
+                }
             };
             for (int base = 0; base < E; base += 32) {
                 const int e = base + lane;
                 const int i = task_of(k.off, e);
                 const int gi = __shfl_sync(kFull, k.grp, i), bi = __shfl_sync(kFull, k.beg, i);
                 const int oi = __shfl_sync(kFull, k.off, i);
-                const uint32_t mi = __shfl_sync(kFull, k.m, i);
+                const Mk mi = __shfl_sync(kFull, k.m, i);
                 const int y = e < E ? ldg_i(g.col + bi + e - oi) : 0;
-                const uint32_t pm = e < E ? (__ldcg(M.nm(gi, Lc + 1) + y) & mi) : 0u;
-                uint32_t todo = __ballot_sync(kFull, pm != 0u);
+                const Mk pm = e < E ? (__ldcg(M.nm(gi, Lc + 1) + y) & mi) : (Mk)0;
+                bytes += 16ull * popc_m(pm);  // sigma, delta of a successor (per root)
+                uint32_t todo = __ballot_sync(kFull, pm != 0);
                 while (todo) {
-                    int ts[kMsUnroll];
-                    uint32_t bits[kMsUnroll];
-                    double qy[kMsUnroll];
+                    int ts[U];
+                    Mk bits[U];
+                    double qy[U][R];
 #pragma unroll
-                    for (int q = 0; q < kMsUnroll; ++q) {
+                    for (int q = 0; q < U; ++q) {
                         const int kk = __ffs(todo) - 1;
                         todo &= todo - 1;
                         const int ys = __shfl_sync(kFull, y, kk & 31);
                         const int gs = __shfl_sync(kFull, gi, kk & 31);
                         ts[q] = kk < 0 ? -1 : __shfl_sync(kFull, i, kk & 31);
-                        bits[q] = kk < 0 ? 0u : __shfl_sync(kFull, pm, kk & 31);
-                        qy[q] = ((bits[q] >> lane) & 1u) ? __ldcg(M.sg(gs) + (size_t)ys * 32 + lane) : 0.0;
+                        bits[q] = kk < 0 ? (Mk)0 : __shfl_sync(kFull, pm, kk & 31);
+                        const double *qp = M.sg(gs) + (size_t)ys * G + lane;
+#pragma unroll
+                        for (int j = 0; j < R; ++j) qy[q][j] = bit(bits[q], lane + 32 * j) ? __ldcg(qp + 32 * j) : 0.0;
                     }
 #pragma unroll
-                    for (int q = 0; q < kMsUnroll; ++q) {
+                    for (int q = 0; q < U; ++q) {
                         if (ts[q] < 0) break;
                         if (ts[q] != cur) {
                             if (cur >= 0) flush();
                             begin(ts[q]);
                         }
-                        if ((bits[q] >> lane) & 1u) {
-                            acc += qy[q];
-                            bytes += 16;
-                        }
+#pragma unroll
+                        for (int j = 0; j < R; ++j)
+                            if (bit(bits[q], lane + 32 * j)) acc[j] += qy[q][j];
                     }
                 }
             }
@@ -528,7 +587,7 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
             const int t = t0 + lane;
             bool sp = false;
             int grp = 0, w = 0;
-            uint32_t m = 0;
+            Mk m = 0;
             if (t < s_pref[ng]) {
                 grp = group_of(s_pref, ng, t);
                 const int2 tk = __ldcg(M.tq(grp) + s_lo[grp] + t - s_pref[grp]);
@@ -546,14 +605,19 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
                 const int i = __ffs(todo) - 1;
                 todo &= todo - 1;
                 const int gc = __shfl_sync(kFull, grp, i), wc = __shfl_sync(kFull, w, i);
-                const bool act = (__shfl_sync(kFull, m, i) >> lane) & 1u;
-                double dl = 0.0;
-                if (act) {
-                    dl = __ldcg(&a.sd[M.st(gc, lane, wc)].y);
-                    double *q = M.sg(gc) + (size_t)wc * 32 + lane;
-                    *q = __ddiv_rn(__dadd_rn(1.0, dl), __ldcg(q));
+                const Mk mc = __shfl_sync(kFull, m, i);
+                double bsum = 0.0;
+#pragma unroll
+                for (int j = 0; j < R; ++j) {
+                    const int b = lane + 32 * j;
+                    if (bit(mc, b)) {
+                        const double dl = __ldcg(&a.sd[M.st(gc, b, wc)].y);
+                        double *q = M.sg(gc) + (size_t)wc * G + b;
+                        *q = __ddiv_rn(__dadd_rn(1.0, dl), __ldcg(q));
+                        bsum += dl;
+                    }
                 }
-                const double bsum = warp_sum(dl);
+                bsum = warp_sum(bsum);
                 if (lane == 0 && bsum != 0.0) atomicAdd(a.bc + wc, bsum);
             }
         }
@@ -581,21 +645,22 @@ __global__ void __launch_bounds__(kBlock) ms_l2mask_kernel(StaticArgs a) {
 
 }  // namespace
 
-int ms_static_threads() { return kMsThreads; }
 int ms_static_max_groups() { return kMsMaxG; }
 int ms_static_max_levels() { return kMsMaxLev; }
 size_t ms_static_counter_bytes(int ng) { return sizeof(MsGroup) * (size_t)ng; }
 
-int ms_static_resident(int nsm) {
+int ms_static_resident(int nsm, int r) {
     int per = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, ms_kernel, kMsThreads, 0) != cudaSuccess) return 0;
+    const void *k = r == 2 ? (const void *)ms_kernel<2> : (const void *)ms_kernel<1>;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k, kMsThreads, 0) != cudaSuccess) return 0;
     return per * nsm;
 }
 
-cudaError_t launch_static_ms(const MsArgs &a, int grid, cudaStream_t s) {
+cudaError_t launch_static_ms(const MsArgs &a, int r, int grid, cudaStream_t s) {
     MsArgs copy = a;
     void *args[] = {&copy};
-    return cudaLaunchCooperativeKernel((const void *)ms_kernel, dim3(grid), dim3(kMsThreads), args, 0, s);
+    const void *k = r == 2 ? (const void *)ms_kernel<2> : (const void *)ms_kernel<1>;
+    return cudaLaunchCooperativeKernel(k, dim3(grid), dim3(kMsThreads), args, 0, s);
 }
 
 void launch_static_l2mask(const StaticArgs &a, cudaStream_t s) {

@@ -56,7 +56,8 @@ class Tuning(ctypes.Structure):
         ("down_long_min", ctypes.c_int32), ("wide_inlane", ctypes.c_int32), ("lean_block", ctypes.c_int32),
         ("lean_workers", ctypes.c_int32), ("lean_max_batch", ctypes.c_int32), ("lean_short", ctypes.c_int32),
         ("trace_slot", ctypes.c_int32), ("disable", ctypes.c_uint32), ("static_ms", ctypes.c_int32),
-        ("static_groups", ctypes.c_int32), ("static_chunk", ctypes.c_int32), ("reserved", ctypes.c_uint32 * 5),
+        ("static_groups", ctypes.c_int32), ("static_chunk", ctypes.c_int32), ("static_width", ctypes.c_int32),
+        ("reserved", ctypes.c_uint32 * 4),
     ]
 
 

@@ -153,18 +153,21 @@ MS_CASES.update({
 })
 
 
+@pytest.mark.parametrize("width", ["32", "64"])
 @pytest.mark.parametrize("chunk", [None, "4"])
 @pytest.mark.parametrize("name", sorted(MS_CASES))
-def test_static_multisource_matches_oracle(name, chunk, tune):
+def test_static_multisource_matches_oracle(name, chunk, width, tune):
     """The multi-source static kernel (msbrandes.cu, 32 roots per warp) forced on
     every graph: d and sigma bit-exact, delta 1e-12 (Eq. (2) regrouped as
     sigma(w) * sum q(y)), BC 1e-9.  chunk 4 splits every row longer than 4
     entries over several warp tasks (sigma partials added atomically, re-summed
     in canonical order at or above 2^53: grid60 and big_sigma_hub reach 2^56
     and more); one 32-root group per wave, so the roots of karate / rmat10_all
-    / disconnected run in several waves."""
+    / disconnected run in several waves.  width 64: two roots per lane (64-bit
+    masks)."""
     tune["static_ms"] = 1
     tune["static_groups"] = 1
+    tune["static_width"] = int(width)
     if chunk:
         tune["static_chunk"] = int(chunk)
     g, roots = MS_CASES[name]()
