@@ -840,7 +840,7 @@ static dbc_status static_ms(dbc_ctx *c, bool *done) {
     const int64_t vcap = std::min<int64_t>((int64_t)n * 12, INT32_MAX / 2);
     const int64_t tcap = std::min<int64_t>(vcap + 12 * (c->nnz / T) + 1024, INT32_MAX / 2);
     const int nlev = ms_static_max_levels() + 3;
-    const size_t per_group = n * (8 * G + 4 * mb) + (size_t)vcap * (4 + mb) + (size_t)tcap * 8 +
+    const size_t per_group = n * (17 * G + 4 * mb) + (size_t)vcap * (4 + mb) + (size_t)tcap * 8 +
                              (size_t)nlev * 4 + ms_static_counter_bytes(1);
     int wave = std::min(ng_all, ms_static_max_groups());
     if (c->tune.static_groups > 0) {
@@ -866,7 +866,7 @@ static dbc_status static_ms(dbc_ctx *c, bool *done) {
     m.stats = c->stats;
     m.err = c->err;
     const size_t W = (size_t)wave;
-    const size_t sz[] = {W * n * G * 8, W * n * mb, W * n * 3 * mb, W * (size_t)vcap * 4, W * (size_t)vcap * mb,
+    const size_t sz[] = {W * n * G * 8, W * n * G * 8, W * n * G, W * n * mb, W * n * 3 * mb, W * (size_t)vcap * 4, W * (size_t)vcap * mb,
                          W * (size_t)tcap * 8, W * (size_t)nlev * 4, ms_static_counter_bytes(wave),
                          2 * sizeof(unsigned)};
     constexpr int kBufs = sizeof(sz) / sizeof(sz[0]);
@@ -880,14 +880,16 @@ static dbc_status static_ms(dbc_ctx *c, bool *done) {
             return DBC_OK;  // no room: the per-root kernel
         }
     m.sg = (double *)buf[0];
-    m.vis = buf[1];
-    m.nm = buf[2];
-    m.vq = (int32_t *)buf[3];
-    m.vm = buf[4];
-    m.tq = (int2 *)buf[5];
-    m.toff = (int32_t *)buf[6];
-    m.ctr = (int32_t *)buf[7];
-    m.bar = (unsigned *)buf[8];
+    m.q = (double *)buf[1];
+    m.lv = (uint8_t *)buf[2];
+    m.vis = buf[3];
+    m.nm = buf[4];
+    m.vq = (int32_t *)buf[5];
+    m.vm = buf[6];
+    m.tq = (int2 *)buf[7];
+    m.toff = (int32_t *)buf[8];
+    m.ctr = (int32_t *)buf[9];
+    m.bar = (unsigned *)buf[10];
     std::vector<int32_t> ctr((size_t)4 * wave);
     bool ok = true;
     cudaError_t e = cudaSuccess;
@@ -904,6 +906,8 @@ static dbc_status static_ms(dbc_ctx *c, bool *done) {
         m.ng = std::min(wave, ng_all - g0);
         const size_t Gn = (size_t)m.ng;
         e = cudaMemsetAsync(m.sg, 0, Gn * n * G * 8, c->stream);
+        if (e == cudaSuccess) e = cudaMemsetAsync(m.q, 0, Gn * n * G * 8, c->stream);
+        if (e == cudaSuccess) e = cudaMemsetAsync(m.lv, 0xff, Gn * n * G, c->stream);
         if (e == cudaSuccess) e = cudaMemsetAsync(m.vis, 0, Gn * n * mb, c->stream);
         if (e == cudaSuccess) e = cudaMemsetAsync(m.nm, 0, Gn * n * 3 * mb, c->stream);
         if (e == cudaSuccess) e = cudaMemsetAsync(m.ctr, 0, ms_static_counter_bytes(m.ng), c->stream);

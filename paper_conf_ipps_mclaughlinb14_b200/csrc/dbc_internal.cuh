@@ -657,7 +657,9 @@ struct MsArgs {
     int32_t k_loc;
     const int32_t *roots;
     int32_t g0, ng;        // groups g0 .. g0 + ng - 1 (slots 32 R g .. 32 R g + 32 R - 1)
-    double *sg;            // [ng][n][32 R] sigma, then q = (1 + delta) / sigma (zeroed)
+    double *sg;            // [ng][n][32 R] sigma (zeroed)
+    double *q;             // [ng][n][32 R] q = (1 + delta) / sigma (zeroed)
+    uint8_t *lv;           // [ng][n][32 R] BFS level, 255 = unreached (0xff-filled)
     // masks over the 32 R roots of a group (R = 1: uint32, R = 2: uint64)
     void *vis;             // [ng][n] roots that reached the vertex (zeroed)
     void *nm;              // [ng][3][n] level masks, level j in array j % 3 (zeroed)

@@ -20,16 +20,15 @@
 //          level-(L+1) mask; the first claimer appends w to level L+1;
 //   pass B (level L+1): sigma pull -- lane = root, each row's predecessors at
 //          level L summed in canonical order;
-//   backward (level L = max-1 .. 1): delta by Eq. (2) regrouped as
+//   backward (level L = max .. 1): delta by Eq. (2) regrouped as
 //          delta(w) = sigma(w) * sum_y q(y), q(y) = (1 + delta(y)) / sigma(y),
-//          q replacing sigma in the scratch once a vertex's delta is final --
-//          one gather per successor instead of two and a division.
+//          stored once a vertex's delta is final -- one gather per successor
+//          instead of two and a division;
+//   final:  tiles transposed into the root-major state of the dynamic kernels.
 // Work unit: a task = a row chunk of <= `chunk` entries of one (vertex, level);
 // a warp takes 32 consecutive tasks (their metadata in one round of loads,
 // one task per lane) and walks their entries flattened, 32 per step.
-// d, sigma and delta go straight into the root-major state of the dynamic
-// kernels (one scattered store per (vertex, root)), BC gets one atomic add per
-// (vertex, level, group).  A group whose BFS passes level kMsMaxLev or whose
+// BC gets one atomic add per (vertex, level, group).  A group whose BFS passes level kMsMaxLev or whose
 // level lists outgrow their capacity sets an overflow flag and the host
 // recomputes with the per-root kernel; so does DBC_FLAG_PULL_DELTA (bitwise
 // delta needs Eq. (2)'s own order).
@@ -107,8 +106,11 @@ struct Ms {
     const MsArgs &a;
     size_t n;
     int lane, gw, W;
-    // sigma of (vertex, root); after the vertex's delta is final: q = (1 + delta) / sigma
+    // sigma of (vertex, root); q = (1 + delta) / sigma once the vertex's delta is
+    // final (a split row first accumulates its chunks' sums there); BFS level
     __device__ double *sg(int grp) const { return a.sg + (size_t)grp * n * G; }
+    __device__ double *qq(int grp) const { return a.q + (size_t)grp * n * G; }
+    __device__ uint8_t *lv(int grp) const { return a.lv + (size_t)grp * n * G; }
     __device__ Mk *vis(int grp) const { return reinterpret_cast<Mk *>(a.vis) + (size_t)grp * n; }
     // level masks: nm(grp, j)[v] = roots with v at level j (array j % 3)
     __device__ Mk *nm(int grp, int j) const { return reinterpret_cast<Mk *>(a.nm) + ((size_t)grp * 3 + (j % 3)) * n; }
@@ -246,6 +248,8 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
     __shared__ int s_pref[kMsMaxG + 1];
     __shared__ int s_lo[kMsMaxG];
     __shared__ int s_done;
+    __shared__ int s_d[G][33];
+    __shared__ double s_sd[2][G][33];
     Ms<R> M{a, (size_t)a.n, (int)(threadIdx.x & 31), (int)((blockIdx.x * kMsThreads + threadIdx.x) >> 5),
             (int)((gridDim.x * kMsThreads) >> 5)};
     const int lane = M.lane;
@@ -255,20 +259,6 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
     const size_t n = M.n;
     unsigned long long bytes = 0;  // algorithmic bytes (SURVEY.md Sec. 8(d) model)
 
-    // ---- Alg. 1 lines 3-9: d = INF, sigma = delta = 0 for the wave's slots
-    {
-        const int s0 = a.g0 * G, s1 = min(a.k_loc, (a.g0 + ng) * G);
-        const size_t tot = (size_t)(s1 - s0) * n;
-        int32_t *d = a.d + (size_t)s0 * n;
-        double2 *sd = a.sd + (size_t)s0 * n;
-        for (size_t i = (size_t)blockIdx.x * kMsThreads + threadIdx.x; i < tot;
-             i += (size_t)gridDim.x * kMsThreads) {
-            d[i] = kInf;
-            sd[i] = make_double2(0.0, 0.0);
-        }
-        if (blockIdx.x == 0 && threadIdx.x == 0) bytes += 20ull * tot;
-    }
-    grid_sync(a.bar);
     // ---- level 0: the roots (one warp per group)
     if (M.gw < ng) {
         const int grp = M.gw;
@@ -279,8 +269,7 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
             if (slot < a.k_loc) {  // roots are distinct (dbc_create)
                 const int s = a.roots[slot];
                 M.sg(grp)[(size_t)s * G + b] = 1.0;
-                a.d[(size_t)slot * n + s] = 0;
-                a.sd[(size_t)slot * n + s] = make_double2(1.0, 0.0);
+                M.lv(grp)[(size_t)s * G + b] = 0;
                 const Mk mb = (Mk)1 << b;
                 const int vi = atomicAdd(&M.ctr(grp)->vcount, 1);
                 M.vq(grp)[vi] = s;
@@ -346,9 +335,6 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
                             M.sg(grp)[(size_t)u * G + lane + 32 * j] = sum[j];
                         }
                 }
-#pragma unroll
-                for (int j = 0; j < R; ++j)
-                    if (bit(mu, lane + 32 * j)) a.sd[M.st(grp, lane + 32 * j, u)].x = sum[j];
             }
             const int E = scan_len(k, lane);
             for (int base = 0; base < E; base += 32) {
@@ -404,7 +390,21 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
                 if (k.chunk == 0) {  // the vertex's level-Lc record
                     M.vm(k.grp)[k.vi] = k.m;
                     M.vis(k.grp)[k.w] = __ldcg(M.vis(k.grp) + k.w) | k.m;
-                    for (Mk b = k.m; b; b &= b - 1) a.d[M.st(k.grp, ffs_m(b) - 1, k.w)] = Lc;
+                    uint4 *lp = reinterpret_cast<uint4 *>(M.lv(k.grp) + (size_t)k.w * G);
+                    const uint32_t rep = (uint32_t)Lc * 0x01010101u;
+#pragma unroll
+                    for (int h = 0; h < 2 * R; ++h) {  // 16 roots per uint4: their bytes := Lc
+                        uint4 q4 = __ldcg(lp + h);
+                        uint32_t *wd = reinterpret_cast<uint32_t *>(&q4);
+#pragma unroll
+                        for (int j = 0; j < 4; ++j) {
+                            const uint32_t nib = (uint32_t)(k.m >> (16 * h + 4 * j)) & 0xFu;
+                            const uint32_t bm = ((nib & 1u) ? 0xFFu : 0u) | ((nib & 2u) ? 0xFF00u : 0u) |
+                                                ((nib & 4u) ? 0xFF0000u : 0u) | ((nib & 8u) ? 0xFF000000u : 0u);
+                            wd[j] = (wd[j] & ~bm) | (rep & bm);
+                        }
+                        if ((k.m >> (16 * h)) & 0xFFFFu) lp[h] = q4;
+                    }
                     bytes += (unsigned long long)popc_m(k.m) * (16 + 4);  // row bounds, sigma and d writes
                 }
             }
@@ -420,12 +420,10 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
                     const int b = lane + 32 * j;
                     if (bit(mc, b)) {
                         double *sw = M.sg(gc) + (size_t)wc * G + b;
-                        if (split) {
+                        if (split)
                             atomicAdd(sw, sum[j]);
-                        } else {
+                        else
                             *sw = sum[j];
-                            a.sd[M.st(gc, b, wc)].x = sum[j];
-                        }
                         if (!(sum[j] <= 1.7976931348623157e308)) atomicOr(a.err, kErrNumeric);
                     }
                 }
@@ -507,12 +505,11 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
                 for (int j = 0; j < R; ++j) {
                     const int b = lane + 32 * j;
                     const bool act = bit(mc, b);
-                    const double dl = act ? __dmul_rn(sv[j], acc[j]) : 0.0;
-                    if (split) {  // a chunk's partial: q and BC once the pass is over
-                        if (act && acc[j] != 0.0) atomicAdd(&a.sd[M.st(gc, b, wc)].y, dl);
+                    if (split) {  // a chunk's sum: q and BC once the pass is over
+                        if (act && acc[j] != 0.0) atomicAdd(M.qq(gc) + (size_t)wc * G + b, acc[j]);
                     } else if (act) {
-                        a.sd[M.st(gc, b, wc)].y = dl;
-                        M.sg(gc)[(size_t)wc * G + b] = __ddiv_rn(__dadd_rn(1.0, dl), sv[j]);
+                        const double dl = __dmul_rn(sv[j], acc[j]);
+                        M.qq(gc)[(size_t)wc * G + b] = __ddiv_rn(__dadd_rn(1.0, dl), sv[j]);
                         bsum += dl;
                     }
                 }
@@ -529,7 +526,8 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
 #pragma unroll
                 for (int j = 0; j < R; ++j) {
                     acc[j] = 0.0;
-                    sv[j] = bit(mc, lane + 32 * j) ? __ldcg(M.sg(gc) + (size_t)wc * G + lane + 32 * j) : 1.0;
+                    // sigma is read-only in the backward passes (L1-cached loads)
+                    sv[j] = bit(mc, lane + 32 * j) ? M.sg(gc)[(size_t)wc * G + lane + 32 * j] : 1.0;
                 }
             };
             for (int base = 0; base < E; base += 32) {
@@ -554,7 +552,7 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
                         const int gs = __shfl_sync(kFull, gi, kk & 31);
                         ts[q] = kk < 0 ? -1 : __shfl_sync(kFull, i, kk & 31);
                         bits[q] = kk < 0 ? (Mk)0 : __shfl_sync(kFull, pm, kk & 31);
-                        const double *qp = M.sg(gs) + (size_t)ys * G + lane;
+                        const double *qp = M.qq(gs) + (size_t)ys * G + lane;
 #pragma unroll
                         for (int j = 0; j < R; ++j) qy[q][j] = bit(bits[q], lane + 32 * j) ? __ldcg(qp + 32 * j) : 0.0;
                     }
@@ -611,9 +609,10 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
                 for (int j = 0; j < R; ++j) {
                     const int b = lane + 32 * j;
                     if (bit(mc, b)) {
-                        const double dl = __ldcg(&a.sd[M.st(gc, b, wc)].y);
-                        double *q = M.sg(gc) + (size_t)wc * G + b;
-                        *q = __ddiv_rn(__dadd_rn(1.0, dl), __ldcg(q));
+                        double *q = M.qq(gc) + (size_t)wc * G + b;
+                        const double sw = M.sg(gc)[(size_t)wc * G + b];
+                        const double dl = __dmul_rn(sw, __ldcg(q));
+                        *q = __ddiv_rn(__dadd_rn(1.0, dl), sw);
                         bsum += dl;
                     }
                 }
@@ -623,6 +622,45 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
         }
         grid_sync(a.bar);
         ms_trace(a.stats, 4, Lc);
+    }
+
+    // ---- the root-major state of the dynamic kernels (Alg. 1's d, sigma,
+    // delta): tiles of 32 vertices x G roots through shared memory, so both
+    // the vertex-major reads and the root-major writes are coalesced;
+    // delta = q sigma - 1 (q = (1 + delta) / sigma: within 2^-51 relative, floor 1)
+    {
+        const int warp = threadIdx.x >> 5;
+        const size_t ntile = (n + 31) / 32;
+        for (size_t tile = blockIdx.x; tile < ntile * (size_t)ng; tile += gridDim.x) {
+            const int grp = (int)(tile / ntile);
+            const size_t v0 = (tile % ntile) * 32;
+            for (int i = warp; i < 32; i += kMsThreads / 32) {  // warp: vertex v0 + i, lane: roots
+                const size_t v = v0 + i;
+                if (v >= n) break;
+#pragma unroll
+                for (int j = 0; j < R; ++j) {
+                    const int b = lane + 32 * j;
+                    const size_t o = v * G + b;
+                    const int l = __ldcg(M.lv(grp) + o);
+                    const double sw = l == 255 ? 0.0 : __ldcg(M.sg(grp) + o);
+                    const double dl = (l == 255 || l == 0) ? 0.0 : __dsub_rn(__dmul_rn(__ldcg(M.qq(grp) + o), sw), 1.0);
+                    s_d[b][i] = l == 255 ? kInf : l;
+                    s_sd[0][b][i] = sw;
+                    s_sd[1][b][i] = dl;
+                }
+            }
+            __syncthreads();
+            const int s0 = (a.g0 + grp) * G;
+            for (int b = warp; b < G; b += kMsThreads / 32) {  // warp: root b, lane: vertex
+                const size_t v = v0 + lane;
+                if (s0 + b < a.k_loc && v < n) {
+                    a.d[(size_t)(s0 + b) * n + v] = s_d[b][lane];
+                    a.sd[(size_t)(s0 + b) * n + v] = make_double2(s_sd[0][b][lane], s_sd[1][b][lane]);
+                }
+            }
+            __syncthreads();
+        }
+        if (blockIdx.x == 0 && threadIdx.x == 0) bytes += 20ull * (size_t)max(0, min(a.k_loc - a.g0 * G, ng * G)) * n;
     }
 
 #pragma unroll
