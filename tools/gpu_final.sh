@@ -15,7 +15,9 @@ timeout 1500 $B --config kron22 --shard 0/8 --steps 2 --warmup 3 --no-e2e --no-p
 N="python bench.py --no-cpu-baseline --no-per-insertion --no-e2e --no-deletions"
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches.csv $N --steps 2 --warmup 3 > $O/ncu_launches.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:update_kernel --launch-skip 3 --launch-count 1 -o $O/update_full $N --steps 1 --warmup 3 > $O/ncu_update.log 2>&1
-timeout 600 ncu --set full --clock-control none --import-source on -k regex:static_kernel --launch-count 1 -o $O/static_full $N --steps 1 --warmup 3 > $O/ncu_static.log 2>&1
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:"static_kernel|ms_kernel" --launch-count 1 -o $O/static_full $N --steps 1 --warmup 3 > $O/ncu_static.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:ms_kernel --launch-count 1 -o $O/ms_kron20_full python tools/static_probe.py kron20 default > $O/ncu_ms_kron20.log 2>&1
+for c in rmat16 kron20 smallworld delaunay18; do timeout 900 python tools/static_probe.py $c static_ms=0 static_ms=1 > $O/static_$c.jsonl 2>&1; done
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:lean --launch-skip 20 --launch-count 1 -o $O/lean_full python tools/lean_ncu_target.py rmat16 40 > $O/ncu_lean.log 2>&1
 for c in rmat16 smallworld delaunay18; do timeout 900 python tools/paper_figures.py $c 100 > $O/fig_$c.json 2> $O/fig_$c.err; done
 ls -la $O
