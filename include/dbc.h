@@ -339,6 +339,13 @@ dbc_status dbc_debug_counters(dbc_ctx *c, int64_t *out, int32_t count);
  * steps}.  Synchronises when out != NULL. */
 dbc_status dbc_debug_root_profile(dbc_ctx *c, int32_t enable, int64_t *out);
 
+/* Diagnostic: per worker CTA of the last per-insertion (update_lean) launch run
+ * with the root profile on, {entry, end of its root and help loops, exit}
+ * globaltimer ns; worker w at out[3w..3w+2], 0 for a CTA that was not
+ * launched.  *count receives the number of values (3 x scratch sets); out may
+ * be NULL to query it; capacity < *count -> DBC_EINVAL.  Synchronises. */
+dbc_status dbc_debug_cta_profile(dbc_ctx *c, int64_t *out, int64_t capacity, int64_t *count);
+
 /* Scenario log (Fig. 2 and Fig. 4).  max_insertions > 0
  * turns it on for later insert calls whose batch has at most that many
  * insertions (larger batches -> DBC_EINVAL); while it is on, every (root,

@@ -690,9 +690,9 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
         cudaMemsetAsync(bd, 0, lean_board_bytes() * (size_t)c->lean_workers, c->stream);
     }
     AL(c->slots_d, (size_t)std::max(c->k_loc, 1));
-    AL(c->stats, (size_t)kStCount);
+    AL(c->stats, (size_t)kStAlloc);
     AL(c->err, 1);
-    AL(c->root_prof, (size_t)6 * std::max(c->k_loc, 1));
+    AL(c->root_prof, (size_t)6 * std::max(c->k_loc, 1) + 3 * nwk);  // + per-CTA {entry, loop end, exit}
     {
         const int kl[6] = {0, 0, 0, c->k_loc, 0, 0};
         if (cudaMemcpy(c->help.roots_left, kl, sizeof(kl), cudaMemcpyHostToDevice) != cudaSuccess)
@@ -747,7 +747,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     if ((s = reset_epochs(c)) != DBC_OK) return bail(s);
     cudaMemsetAsync(c->bc, 0, sizeof(double) * n, c->stream);
     cudaMemsetAsync(c->err, 0, sizeof(int32_t), c->stream);
-    cudaMemsetAsync(c->stats, 0, sizeof(unsigned long long) * kStCount, c->stream);
+    cudaMemsetAsync(c->stats, 0, sizeof(unsigned long long) * kStAlloc, c->stream);
     if (cudaStreamSynchronize(c->stream) != cudaSuccess) {
         fail(c, DBC_ECUDA, "init failed: %s", cudaGetErrorString(cudaGetLastError()));
         return bail(DBC_ECUDA);
@@ -965,9 +965,14 @@ extern "C" dbc_status dbc_static_compute(dbc_ctx *c) {
 }
 
 static dbc_status read_stats(dbc_ctx *c, unsigned long long *h) {
-    CK(cudaMemcpyAsync(h, c->stats, sizeof(unsigned long long) * kStCount, cudaMemcpyDeviceToHost,
+    static_assert(kStAlloc > kStCount, "stats lanes");
+    std::vector<unsigned long long> all(kStAlloc);
+    CK(cudaMemcpyAsync(all.data(), c->stats, sizeof(unsigned long long) * kStAlloc, cudaMemcpyDeviceToHost,
                        c->stream));
     CK(cudaStreamSynchronize(c->stream));
+    std::memcpy(h, all.data(), sizeof(unsigned long long) * kStCount);
+    for (int l = 0; l < kStLanes; ++l)
+        for (int i = 0; i < kStTraceN; ++i) h[i] += all[kStCount + (size_t)l * kStTraceN + i];
     return DBC_OK;
 }
 
@@ -1089,7 +1094,9 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
         a.merge = 0;
         a.root_prof = c->prof_on ? c->root_prof : nullptr;
         if (c->prof_on)
-            CK(cudaMemsetAsync(c->root_prof, 0, sizeof(unsigned long long) * 6 * std::max(c->k_loc, 1), c->stream));
+            CK(cudaMemsetAsync(c->root_prof, 0,
+                               sizeof(unsigned long long) * (6 * std::max(c->k_loc, 1) + 3 * c->nscratch),
+                               c->stream));
         const int64_t step = (c->flags & DBC_FLAG_MODE_S) ? 1 : cnt;  // Mode S: one launch per insertion
         for (int64_t i = 0; i < cnt; i += step) {
             CK(cudaMemsetAsync(c->next_slot, 0, 4 * sizeof(int32_t), c->stream));
@@ -1579,6 +1586,19 @@ extern "C" dbc_status dbc_debug_root_profile(dbc_ctx *c, int32_t enable, int64_t
     if (out) {
         CK(cudaMemcpyAsync(out, c->root_prof, sizeof(int64_t) * 6 * c->k_loc, cudaMemcpyDeviceToHost,
                            c->stream));
+        CK(cudaStreamSynchronize(c->stream));
+    }
+    return DBC_OK;
+}
+
+extern "C" dbc_status dbc_debug_cta_profile(dbc_ctx *c, int64_t *out, int64_t capacity, int64_t *count) {
+    if (!c || !count) return DBC_EINVAL;
+    CK(cudaSetDevice(c->device));
+    *count = 3 * (int64_t)c->nscratch;
+    if (out) {
+        if (capacity < *count) return DBC_EINVAL;
+        CK(cudaMemcpyAsync(out, c->root_prof + 6 * std::max(c->k_loc, 1), sizeof(int64_t) * *count,
+                           cudaMemcpyDeviceToHost, c->stream));
         CK(cudaStreamSynchronize(c->stream));
     }
     return DBC_OK;

@@ -73,6 +73,20 @@ enum StatIdx : int {
     kStCount = kStTrace0 + 2 * 1024
 };
 constexpr int kTraceCap = 1024;
+// Contention-free copies of the counters below kStTraceN: kernels whose CTAs
+// all finish together (the per-insertion kernel) add into lane (CTA % kStLanes)
+// at stats + kStCount + lane * kStTraceN; read_stats folds the lanes in.
+constexpr int kStLanes = 64;
+constexpr int kStAlloc = kStCount + kStLanes * kStTraceN;
+__device__ __forceinline__ unsigned long long *stat_lane(unsigned long long *stats) {
+    return stats + kStCount + (size_t)(blockIdx.x % kStLanes) * kStTraceN;
+}
+// Sum of v over the warp added to counter idx of the CTA's lane (all 32 lanes must call).
+__device__ __forceinline__ void stat_add_warp(unsigned long long *stats, int idx, unsigned long long v) {
+#pragma unroll
+    for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    if ((threadIdx.x & 31) == 0 && v) atomicAdd(stat_lane(stats) + idx, v);
+}
 
 // The state of one root (pointers into the root-major arrays).
 struct Root {

@@ -232,11 +232,11 @@ __global__ void __launch_bounds__(kEB, 1) edge_kernel(EdgeArgs a) {
     }
     if (tid == 0) {
         a.ws.wepoch[wk] = epoch;
-        atomicAdd(a.stats + kStCase1, c1);
-        atomicAdd(a.stats + kStCase2, c2);
-        atomicAdd(a.stats + kStCase3, c3);
-        atomicAdd(a.stats + kStScanned, scanned);
-        atomicAdd(a.stats + kStBytes, bytes + scanned * 12ull);  // per visited entry: src, col, tag
+        atomicAdd(stat_lane(a.stats) + kStCase1, c1);
+        atomicAdd(stat_lane(a.stats) + kStCase2, c2);
+        atomicAdd(stat_lane(a.stats) + kStCase3, c3);
+        atomicAdd(stat_lane(a.stats) + kStScanned, scanned);
+        atomicAdd(stat_lane(a.stats) + kStBytes, bytes + scanned * 12ull);  // per visited entry: src, col, tag
     }
 }
 

@@ -665,7 +665,7 @@ __global__ void __launch_bounds__(kMsThreads, 3) ms_kernel(MsArgs a) {
 
 #pragma unroll
     for (int off = 16; off > 0; off >>= 1) bytes += __shfl_xor_sync(kFull, bytes, off);
-    if (lane == 0 && bytes) atomicAdd(a.stats + kStStaticBytes, bytes);
+    if (lane == 0 && bytes) atomicAdd(stat_lane(a.stats) + kStStaticBytes, bytes);
 }
 
 // Level-2 predecessor masks of roots with at most kMaskDeg neighbours (read by

@@ -199,7 +199,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) static_kernel(StaticArgs a
             __syncthreads();
         }
     }
-    if (bytes) atomicAdd(a.stats + kStStaticBytes, bytes);
+    stat_add_warp(a.stats, kStStaticBytes, bytes);
 }
 
 }  // namespace

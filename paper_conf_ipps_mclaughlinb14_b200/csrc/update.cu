@@ -1025,7 +1025,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
         if (tid == 0) {  // release by one thread after the CTA barrier
             __threadfence();
             atomicAdd(a.help.done + pick, 1);
-            atomicAdd(a.stats + kStHelpBlk, 1ull);
+            atomicAdd(stat_lane(a.stats) + kStHelpBlk, 1ull);
         }
         return 1;
     };
@@ -1038,7 +1038,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
         int co = -1, cs = -1;
         for (int q = 0; q < a.busy_help; ++q) {
             if (help_step(false, co, cs) < 0) break;
-            if (tid == 0) atomicAdd(a.stats + kStBusyBlk, 1ull);
+            if (tid == 0) atomicAdd(stat_lane(a.stats) + kStBusyBlk, 1ull);
         }
     };
     // sampled at a level start by thread 0, published at the level end:
@@ -1152,8 +1152,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                     s_st[4] += n3;
                     st_bytes += 8ull * nwin;
                     if (nw > 1) {
-                        atomicAdd(a.stats + kStGroups, 1ull);
-                        atomicAdd(a.stats + kStGroupIns, (unsigned long long)nw);
+                        atomicAdd(stat_lane(a.stats) + kStGroups, 1ull);
+                        atomicAdd(stat_lane(a.stats) + kStGroupIns, (unsigned long long)nw);
                     }
                 }
                 if (nw == 0) {  // Case 1 throughout: nothing changes
@@ -1429,8 +1429,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                             a.help.gbig[2 * wk] = 0;
                             a.help.gbig[2 * wk + 1] = 0;
                             __threadfence();
-                            atomicAdd(a.stats + kStHelpReq, 1ull);
-                            atomicAdd(a.stats + kStHelpBlkAll, (unsigned long long)nblk);
+                            atomicAdd(stat_lane(a.stats) + kStHelpReq, 1ull);
+                            atomicAdd(stat_lane(a.stats) + kStHelpBlkAll, (unsigned long long)nblk);
                             hseq = (hseq + 1) & 0xFFFF;
                             atomicExch(a.help.word + wk, help_pack(1, nblk, 0, hseq));
                             if (nblk >= a.busy_min) atomicAdd(a.help.roots_left + 1, 1);  // open wide requests
@@ -1503,8 +1503,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                             a.help.gapp[wk] = s_dcnt;
                             a.help.low[wk] = 0;
                             __threadfence();
-                            atomicAdd(a.stats + kStHelpReq, 1ull);
-                            atomicAdd(a.stats + kStHelpBlkAll, (unsigned long long)nblk);
+                            atomicAdd(stat_lane(a.stats) + kStHelpReq, 1ull);
+                            atomicAdd(stat_lane(a.stats) + kStHelpBlkAll, (unsigned long long)nblk);
                             hseq = (hseq + 1) & 0xFFFF;
                             atomicExch(a.help.word + wk, help_pack(1, nblk, 0, hseq));
                             if (nblk >= a.busy_min) atomicAdd(a.help.roots_left + 1, 1);
@@ -1649,8 +1649,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                             a.help.gapp[wk] = s_rcnt;
                             a.help.low[wk] = s_rmax;
                             __threadfence();
-                            atomicAdd(a.stats + kStHelpReq, 1ull);
-                            atomicAdd(a.stats + kStHelpBlkAll, (unsigned long long)nblk);
+                            atomicAdd(stat_lane(a.stats) + kStHelpReq, 1ull);
+                            atomicAdd(stat_lane(a.stats) + kStHelpBlkAll, (unsigned long long)nblk);
                             hseq = (hseq + 1) & 0xFFFF;
                             atomicExch(a.help.word + wk, help_pack(1, nblk, 0, hseq));
                             if (nblk >= a.busy_min) atomicAdd(a.help.roots_left + 1, 1);  // open wide requests
@@ -2021,9 +2021,9 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                             __syncthreads();  // the frontier copy is written; one release fence publishes it
                             if (tid == 0) {
                                 __threadfence();
-                                atomicAdd(a.stats + kStHelpReq, 1ull);
-                                atomicAdd(a.stats + kStHelpBlkAll, (unsigned long long)nblk5);
-                                atomicAdd(a.stats + kStUpPass, 1ull);
+                                atomicAdd(stat_lane(a.stats) + kStHelpReq, 1ull);
+                                atomicAdd(stat_lane(a.stats) + kStHelpBlkAll, (unsigned long long)nblk5);
+                                atomicAdd(stat_lane(a.stats) + kStUpPass, 1ull);
                                 hseq = (hseq + 1) & 0xFFFF;
                                 atomicExch(a.help.word + wk, help_pack(1, nblk5, 0, hseq));
                                 if (nblk5 >= a.busy_min) atomicAdd(a.help.roots_left + 1, 1);
@@ -2133,8 +2133,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                 __syncthreads();
                                 if (tid == 0) {
                                     __threadfence();
-                                    atomicAdd(a.stats + kStHelpReq, 1ull);
-                                    atomicAdd(a.stats + kStHelpBlkAll, (unsigned long long)nblk1);
+                                    atomicAdd(stat_lane(a.stats) + kStHelpReq, 1ull);
+                                    atomicAdd(stat_lane(a.stats) + kStHelpBlkAll, (unsigned long long)nblk1);
                                     hseq = (hseq + 1) & 0xFFFF;
                                     atomicExch(a.help.word + wk, help_pack(1, nblk1, 0, hseq));
                                     if (nblk1 >= a.busy_min) atomicAdd(a.help.roots_left + 1, 1);  // open wide requests
@@ -2223,8 +2223,8 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                                 __syncthreads();  // the chunk is written; one release fence publishes it
                                 if (tid == 0) {
                                     __threadfence();
-                                    atomicAdd(a.stats + kStHelpReq, 1ull);
-                                    atomicAdd(a.stats + kStHelpBlkAll, (unsigned long long)nblk);
+                                    atomicAdd(stat_lane(a.stats) + kStHelpReq, 1ull);
+                                    atomicAdd(stat_lane(a.stats) + kStHelpBlkAll, (unsigned long long)nblk);
                                     hseq = (hseq + 1) & 0xFFFF;
                                     atomicExch(a.help.word + wk, help_pack(1, nblk, 0, hseq));
                                     if (nblk >= a.busy_min) atomicAdd(a.help.roots_left + 1, 1);  // open wide requests
@@ -2363,7 +2363,7 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
                             put_row(t, w.x, w.meta, w.c0, w.c1, w.c2, w.beg, w.len, w.mk);
                         }
                         if (dn) xdn += m; else xun += m;
-                        if (tid == 0) atomicAdd(a.stats + kStDeferred, (unsigned long long)m);
+                        if (tid == 0) atomicAdd(stat_lane(a.stats) + kStDeferred, (unsigned long long)m);
                         nb = m;
                         nDb = dn ? m : 0;
                         __syncthreads();
@@ -2419,25 +2419,25 @@ __global__ void __launch_bounds__(kBlock, kMinBlocks) update_kernel(UpdateArgs a
     }
     if (tid == 0) {
         a.ws.wepoch[wk] = epoch;
-        if (s_st[2]) atomicAdd(a.stats + kStCase1, s_st[2]);
-        if (s_st[3]) atomicAdd(a.stats + kStCase2, s_st[3]);
-        if (s_st[4]) atomicAdd(a.stats + kStCase3, s_st[4]);
-        if (s_st[0]) atomicAdd(a.stats + kStTouched, s_st[0]);
-        if (s_st[1]) atomicAdd(a.stats + kStDown, s_st[1]);
-        if (s_st[5]) atomicAdd(a.stats + kStLevDown, s_st[5]);
-        if (s_st[6]) atomicAdd(a.stats + kStLevUp, s_st[6]);
+        if (s_st[2]) atomicAdd(stat_lane(a.stats) + kStCase1, s_st[2]);
+        if (s_st[3]) atomicAdd(stat_lane(a.stats) + kStCase2, s_st[3]);
+        if (s_st[4]) atomicAdd(stat_lane(a.stats) + kStCase3, s_st[4]);
+        if (s_st[0]) atomicAdd(stat_lane(a.stats) + kStTouched, s_st[0]);
+        if (s_st[1]) atomicAdd(stat_lane(a.stats) + kStDown, s_st[1]);
+        if (s_st[5]) atomicAdd(stat_lane(a.stats) + kStLevDown, s_st[5]);
+        if (s_st[6]) atomicAdd(stat_lane(a.stats) + kStLevUp, s_st[6]);
         for (int q = 0; q < 10; ++q)
-            if (tm_ph[q]) atomicAdd(a.stats + kStTime0 + q, tm_ph[q]);
+            if (tm_ph[q]) atomicAdd(stat_lane(a.stats) + kStTime0 + q, tm_ph[q]);
     }
     const unsigned long long sc[6] = {sc_down, sc_rem, sc_dpull, sc_dpush, sc_up2, sc_up3};
     unsigned long long tot = 0;
 #pragma unroll
     for (int q = 0; q < 6; ++q) {
         tot += sc[q];
-        if (sc[q]) atomicAdd(a.stats + kStPhase0 + q, sc[q]);
+        stat_add_warp(a.stats, kStPhase0 + q, sc[q]);
     }
-    if (tot) atomicAdd(a.stats + kStScanned, tot);
-    if (st_bytes) atomicAdd(a.stats + kStBytes, st_bytes);
+    stat_add_warp(a.stats, kStScanned, tot);
+    stat_add_warp(a.stats, kStBytes, st_bytes);
 }
 
 }  // namespace

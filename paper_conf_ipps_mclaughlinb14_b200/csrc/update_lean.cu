@@ -465,6 +465,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
     const int total_roots = a.slot_list ? a.slot_count : a.k_loc;
     const bool pull = a.pull_delta != 0;  // DBC_FLAG_PULL_DELTA (no help board then)
     int hseq = 0;
+    unsigned long long *stl = a.stats + kStCount + (size_t)(wk % kStLanes) * kStTraceN;  // this CTA's counter lane
 
     // phase clocks of one traced root (dbc_tuning.trace_slot; diagnostic): down
     // item load / scan / pass / finalize, removal, up level setup, D rows, up
@@ -473,6 +474,13 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
     long long tclk = 0;
     if (tid == 0)
         for (int q = 0; q < 10; ++q) s_tph[q] = 0;
+    // per-CTA record after the root records (dbc_debug_cta_profile): entry, end of the work loops, exit
+    unsigned long long *cta_prof = a.root_prof ? a.root_prof + 6 * (size_t)max(a.k_loc, 1) + 3 * (size_t)wk : nullptr;
+    if (cta_prof && tid == 0) {
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        cta_prof[0] = t;
+    }
     auto tick = [&](int ph) {
         if (trace && tid == 0) {
             const long long t = clock64();
@@ -535,8 +543,8 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
             __threadfence();
             atomicExch(&mine->word, hb_pack(1, nblk, 0, hseq));
             atomicAdd(a.next_slot + 1, 1);  // open requests (idle workers poll this word only)
-            atomicAdd(a.stats + kStHelpReq, 1ull);
-            atomicAdd(a.stats + kStHelpBlkAll, (unsigned long long)nblk);
+            atomicAdd(stl + kStHelpReq, 1ull);
+            atomicAdd(stl + kStHelpBlkAll, (unsigned long long)nblk);
         }
         PassCtx gc = c;
         gc.ctr = &mine->ctr;
@@ -1015,7 +1023,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                         break;
                     }
                     __nanosleep(backoff);
-                    backoff = min(backoff * 2, 2048);
+                    backoff = min(backoff * 2, 512);
                 }
             }
             __syncthreads();
@@ -1106,27 +1114,32 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
             if (tid == 0) {
                 __threadfence();
                 atomicAdd(&ob->done, 1);
-                atomicAdd(a.stats + kStHelpBlk, 1ull);
+                atomicAdd(stl + kStHelpBlk, 1ull);
             }
         }
     }
 
+    if (cta_prof && tid == 0) {
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        cta_prof[1] = t;
+    }
     if (tid == 0) {
         for (int q = 0; q < 10; ++q)
-            if (s_tph[q]) atomicAdd(a.stats + kStTime0 + q, s_tph[q]);
+            if (s_tph[q]) atomicAdd(stl + kStTime0 + q, s_tph[q]);
         a.ws.wepoch[wk] = epoch;
-        if (c_case[1]) atomicAdd(a.stats + kStCase2, c_case[1]);
-        if (c_case[2]) atomicAdd(a.stats + kStCase3, c_case[2]);
-        if (c_touch) atomicAdd(a.stats + kStTouched, c_touch);
-        if (c_down) atomicAdd(a.stats + kStDown, c_down);
-        if (c_lev[0]) atomicAdd(a.stats + kStLevDown, c_lev[0]);
-        if (c_lev[1]) atomicAdd(a.stats + kStLevUp, c_lev[1]);
+        if (c_case[1]) atomicAdd(stl + kStCase2, c_case[1]);
+        if (c_case[2]) atomicAdd(stl + kStCase3, c_case[2]);
+        if (c_touch) atomicAdd(stl + kStTouched, c_touch);
+        if (c_down) atomicAdd(stl + kStDown, c_down);
+        if (c_lev[0]) atomicAdd(stl + kStLevDown, c_lev[0]);
+        if (c_lev[1]) atomicAdd(stl + kStLevUp, c_lev[1]);
     }
     unsigned long long sc_all = 0;
 #pragma unroll
     for (int q = 0; q < 6; ++q) {
         sc_all += sc_ph[q];
-        if (sc_ph[q]) atomicAdd(a.stats + kStPhase0 + q, (unsigned long long)sc_ph[q]);
+        if (sc_ph[q]) atomicAdd(stl + kStPhase0 + q, (unsigned long long)sc_ph[q]);
     }
     sc_all += my_scan;
     unsigned long long c1 = c_case[0], by = my_bytes;
@@ -1136,10 +1149,24 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
         by += __shfl_xor_sync(kFull, by, o);
         sc_all += __shfl_xor_sync(kFull, sc_all, o);
     }
+    __shared__ unsigned long long s_red[3];
+    if (tid < 3) s_red[tid] = 0;
+    __syncthreads();
     if ((tid & 31) == 0) {
-        if (c1) atomicAdd(a.stats + kStCase1, c1);
-        if (by) atomicAdd(a.stats + kStBytes, by);
-        if (sc_all) atomicAdd(a.stats + kStScanned, sc_all);
+        if (c1) atomicAdd(s_red + 0, c1);
+        if (by) atomicAdd(s_red + 1, by);
+        if (sc_all) atomicAdd(s_red + 2, sc_all);
+    }
+    __syncthreads();
+    if (tid == 0) {
+        if (s_red[0]) atomicAdd(stl + kStCase1, s_red[0]);
+        if (s_red[1]) atomicAdd(stl + kStBytes, s_red[1]);
+        if (s_red[2]) atomicAdd(stl + kStScanned, s_red[2]);
+    }
+    if (cta_prof && tid == 0) {
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        cta_prof[2] = t;
     }
 }
 

@@ -124,6 +124,7 @@ SIGNATURES = {
     "dbc_reset_timings": (ctypes.c_int, [_P]),
     "dbc_debug_counters": (ctypes.c_int, [_P, _P, ctypes.c_int32]),
     "dbc_debug_root_profile": (ctypes.c_int, [_P, ctypes.c_int32, _P]),
+    "dbc_debug_cta_profile": (ctypes.c_int, [_P, _P, ctypes.c_int64, _P]),
     "dbc_device_bytes": (ctypes.c_int, [_P, _P]),
     "dbc_scenario_log": (ctypes.c_int, [_P, ctypes.c_int64]),
     "dbc_get_scenarios": (ctypes.c_int, [_P, _P, ctypes.c_int64, _P]),
@@ -372,6 +373,15 @@ class DynamicBC:
         _check(self._ctx, self._lib.dbc_debug_root_profile(
             self._ctx, int(enable), _np_ptr(out) if read else None))
         return out
+
+    def cta_profile(self):
+        """Per worker CTA of the last per-insertion launch (root profile on):
+        int64 [workers, 3] = {entry, end of work loops, exit} globaltimer ns."""
+        cnt = ctypes.c_int64()
+        _check(self._ctx, self._lib.dbc_debug_cta_profile(self._ctx, None, 0, ctypes.byref(cnt)))
+        out = np.zeros(cnt.value, dtype=np.int64)
+        _check(self._ctx, self._lib.dbc_debug_cta_profile(self._ctx, _np_ptr(out), out.size, ctypes.byref(cnt)))
+        return out.reshape(-1, 3)
 
     def scenario_log(self, max_insertions: int):
         """Record case and touched count of every (root, insertion) of later
