@@ -62,11 +62,20 @@ constexpr int kLCap = 512;        // items per chunk
 constexpr int kLStash = 512;      // D-row predecessor pushes staged per chunk
 constexpr int kLWin = kBlock < 256 ? kBlock : 256;  // insertions classified at once
 constexpr int kLAdj = 256;        // longest root row cached (level-2 shortcut)
-constexpr int kLU = 4;            // consecutive entries per thread per step
+#ifndef DBC_LEAN_LU
+#define DBC_LEAN_LU 4
+#endif
+#ifndef DBC_LEAN_HELPBLK
+#define DBC_LEAN_HELPBLK 2048
+#endif
+#ifndef DBC_LEAN_HELPMIN
+#define DBC_LEAN_HELPMIN 3
+#endif
+constexpr int kLU = DBC_LEAN_LU;  // consecutive entries per thread per step
 constexpr uint32_t kLD = 3u;      // mark: in D (t = down).  kLD > kLUp: an up claim
 constexpr uint32_t kLUp = 1u;     // mark: up (t = up)        never overrides a D mark
-constexpr int kHelpBlk = 4096;    // entries per help block
-constexpr int kHelpMinBlk = 3;    // passes of at least this many blocks are published
+constexpr int kHelpBlk = DBC_LEAN_HELPBLK;  // entries per help block
+constexpr int kHelpMinBlk = DBC_LEAN_HELPMIN;  // passes of at least this many blocks are published
 constexpr int kLEnt = 1536;       // entries whose contributions are kept for an in-order row sum
 constexpr int kSpecEntries = 2 * kBlock * kLU;  // passes up to this size gather speculatively
 
