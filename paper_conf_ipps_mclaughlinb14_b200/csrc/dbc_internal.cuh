@@ -401,7 +401,10 @@ constexpr int kUcap = 1024;   // up-frontier entries kept in shared memory
 constexpr int kMetaUp = 1, kMetaNotPulled = 2, kMetaMask = 4;
 constexpr int kMetaNew = 8;  // down row with batch entries: its pushes check new_edge()
 constexpr int kMetaExt = 16; // down row with a predecessor outside D: it has pushes to make
-constexpr int kFlatU = 4;     // contiguous entries per thread per step
+#ifndef DBC_FLAT_U
+#define DBC_FLAT_U 4
+#endif
+constexpr int kFlatU = DBC_FLAT_U;  // contiguous entries per thread per step
 constexpr int kWindow = 16384;  // default insertions per Mode-A job (DBC_WINDOW overrides)
 constexpr int kAdjCap = 256;  // longest root row kept in shared memory (level-2 shortcut)
 
