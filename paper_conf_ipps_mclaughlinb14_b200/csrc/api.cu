@@ -630,25 +630,6 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->bc_ext, (size_t)n);
     AL(c->perm_d, (size_t)n);
     AL(c->roots_d, (size_t)c->k_loc);
-#ifdef DBC_L2PERSIST
-    {  // experiment: keep the distance array (every neighbour gather's filter) resident in L2
-        int maxwin = 0, maxpers = 0;
-        cudaDeviceGetAttribute(&maxwin, cudaDevAttrMaxAccessPolicyWindowSize, c->device);
-        cudaDeviceGetAttribute(&maxpers, cudaDevAttrMaxPersistingL2CacheSize, c->device);
-        const size_t bytes = kn * sizeof(int32_t);
-        fprintf(stderr, "[dbc] L2 persist: window max %d, persisting max %d, d %zu bytes\n", maxwin, maxpers, bytes);
-        if (bytes <= (size_t)maxwin && maxpers > 0) {
-            cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, std::min(bytes, (size_t)maxpers));
-            cudaStreamAttrValue v = {};
-            v.accessPolicyWindow.base_ptr = c->d;
-            v.accessPolicyWindow.num_bytes = bytes;
-            v.accessPolicyWindow.hitRatio = std::min(1.0f, (float)maxpers / (float)bytes);
-            v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-            v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
-            cudaStreamSetAttribute(c->stream, cudaStreamAttributeAccessPolicyWindow, &v);
-        }
-    }
-#endif
     // per-insertion workers (update_lean.cu): one CTA per root when memory allows
     c->lean_workers = std::max(0, std::min(c->k_loc, fit));
     if (T.lean_workers > 0) c->lean_workers = std::max(1, std::min(c->lean_workers, T.lean_workers));
