@@ -9,6 +9,7 @@
 #include <cstring>
 #include <string>
 #include <thread>
+#include <unordered_set>
 #include <vector>
 
 #include <dlfcn.h>
@@ -142,6 +143,13 @@ struct dbc_ctx {
     dbc_reduce_fn reduce = nullptr;    // ... or the caller's callback (opt.reduce)
     void *reduce_user = nullptr;
 
+    // Host copy of the adjacency in caller ids: the original rows sorted, plus
+    // the edges inserted / original edges deleted since (key min << 32 | max).
+    // Host-array batches are validated against it (no device round trip).
+    std::vector<int64_t> h_rp;
+    std::vector<int32_t> h_scol;
+    std::unordered_set<uint64_t> h_ins, h_del;
+    cudaEvent_t ev_prof = nullptr;  // recorded after a batch whose chain times are pending
     cudaEvent_t ev[10] = {};  // [0..3]/[6..9]: insert-call sets A/B, [4..5]: static
     int evset = 0;            // set of the most recent insert call (0 -> ev[0..3], 1 -> ev[6..9])
     bool ev_ok = false;
@@ -286,6 +294,7 @@ void dbc_destroy(dbc_ctx *c) {
     if (c->ev_ok)
         for (auto &e : c->ev) cudaEventDestroy(e);
     if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+    if (c->ev_prof) cudaEventDestroy(c->ev_prof);
     if (c->ev_join) cudaEventDestroy(c->ev_join);
     if (c->hstream) cudaStreamDestroy(c->hstream);
     if (c->own_stream && c->stream) cudaStreamDestroy(c->stream);
@@ -295,7 +304,8 @@ void dbc_destroy(dbc_ctx *c) {
 }  // extern "C"
 
 // Host CSR validation: symmetric, no self loops, no duplicate entries.
-static bool validate_csr(int32_t n, const int64_t *rp, const int32_t *col, std::string &why) {
+static bool validate_csr(int32_t n, const int64_t *rp, const int32_t *col, std::string &why,
+                         std::vector<int32_t> *sorted_out) {
     if (rp[0] != 0) { why = "row_ptr[0] != 0"; return false; }
     for (int32_t v = 0; v < n; ++v)
         if (rp[v + 1] < rp[v]) { why = "row_ptr not non-decreasing"; return false; }
@@ -338,6 +348,7 @@ static bool validate_csr(int32_t n, const int64_t *rp, const int32_t *col, std::
     }
     for (unsigned t = 0; t < nt; ++t)
         if (!ok[t]) { why = whys[t]; return false; }
+    if (sorted_out) *sorted_out = std::move(srt);
     return true;
 }
 
@@ -439,9 +450,11 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
             if (opt.tuning->reserved[i]) return fail(nullptr, DBC_EINVAL, "tuning reserved fields must be zero");
     if ((opt.flags & DBC_FLAG_PULL_DELTA) && (opt.flags & DBC_FLAG_EDGE_PARALLEL))
         return fail(nullptr, DBC_EINVAL, "DBC_FLAG_PULL_DELTA excludes DBC_FLAG_EDGE_PARALLEL");
+    std::vector<int32_t> h_scol;  // the rows sorted (kept for host-side batch validation)
     {
         std::string why;
-        if (!validate_csr(n, row_ptr, col, why)) return fail(nullptr, DBC_EINVAL, "bad CSR: %s", why.c_str());
+        if (!validate_csr(n, row_ptr, col, why, &h_scol))
+            return fail(nullptr, DBC_EINVAL, "bad CSR: %s", why.c_str());
     }
     {
         std::vector<int32_t> r(roots, roots + k);
@@ -470,6 +483,8 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     c->n = n;
     c->k = k;
     c->nnz = c->nnz0 = row_ptr[n];
+    c->h_rp.assign(row_ptr, row_ptr + (size_t)n + 1);
+    c->h_scol = std::move(h_scol);
     const int64_t m = c->nnz0 / 2;
     c->edge_cap = opt.edge_capacity ? opt.edge_capacity : std::max<int64_t>(1 << 16, m / 4);
     c->col_cap = c->nnz0 + 2 * c->edge_cap;
@@ -520,6 +535,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
         cudaDeviceGetStreamPriorityRange(&lo, &hi);
         if (cudaStreamCreateWithPriority(&c->hstream, cudaStreamNonBlocking, hi) != cudaSuccess ||
             cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
+            cudaEventCreateWithFlags(&c->ev_prof, cudaEventDisableTiming) != cudaSuccess ||
             cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming) != cudaSuccess) {
             fail(c, DBC_ECUDA, "heavy-lane stream creation failed");
             return bail(DBC_ECUDA);
@@ -964,6 +980,51 @@ extern "C" dbc_status dbc_static_compute(dbc_ctx *c) {
     return DBC_OK;
 }
 
+// Host-side batch validation against the host copy of the adjacency (caller
+// ids): the same rules and error bits as the device validation (graph.cu):
+// 1 self loop / out of range, 2 edge already present, 4 duplicate in the batch.
+static inline uint64_t edge_key(int32_t a, int32_t b) {
+    return ((uint64_t)(uint32_t)std::min(a, b) << 32) | (uint32_t)std::max(a, b);
+}
+static bool host_present(const dbc_ctx *c, int32_t a, int32_t b) {
+    const uint64_t k = edge_key(a, b);
+    if (c->h_ins.count(k)) return true;
+    const int32_t lo = std::min(a, b), hi = std::max(a, b);
+    return std::binary_search(c->h_scol.begin() + c->h_rp[lo], c->h_scol.begin() + c->h_rp[lo + 1], hi) &&
+           !c->h_del.count(k);
+}
+static int host_validate(const dbc_ctx *c, const int32_t *u, const int32_t *v, int64_t cnt) {
+    int bad = 0;
+    std::vector<uint64_t> keys((size_t)cnt);
+    for (int64_t i = 0; i < cnt; ++i) {
+        const int32_t a = u[i], b = v[i];
+        if (a < 0 || a >= c->n || b < 0 || b >= c->n || a == b) {
+            bad |= 1;
+            keys[(size_t)i] = ~0ull - (uint64_t)i;  // distinct placeholder
+            continue;
+        }
+        if (host_present(c, a, b)) bad |= 2;
+        keys[(size_t)i] = edge_key(a, b);
+    }
+    std::sort(keys.begin(), keys.end());
+    if (std::adjacent_find(keys.begin(), keys.end()) != keys.end()) bad |= 4;
+    return bad;
+}
+static const char *bad_batch_why(int bad) {
+    return (bad & 1) ? "self loop or vertex out of range" : (bad & 2) ? "edge already present"
+                                                                      : "duplicate edge within the batch";
+}
+// the host copy follows the device graph: inserted edges join, deleted ones leave
+static void host_record_insert(dbc_ctx *c, const int32_t *u, const int32_t *v, int64_t cnt) {
+    for (int64_t i = 0; i < cnt; ++i) c->h_ins.insert(edge_key(u[i], v[i]));
+}
+static void host_record_delete(dbc_ctx *c, const int32_t *u, const int32_t *v, int64_t cnt) {
+    for (int64_t i = 0; i < cnt; ++i) {
+        const uint64_t k = edge_key(u[i], v[i]);
+        if (!c->h_ins.erase(k)) c->h_del.insert(k);
+    }
+}
+
 static dbc_status read_stats(dbc_ctx *c, unsigned long long *h) {
     static_assert(kStAlloc > kStCount, "stats lanes");
     std::vector<unsigned long long> all(kStAlloc);
@@ -976,8 +1037,11 @@ static dbc_status read_stats(dbc_ctx *c, unsigned long long *h) {
     return DBC_OK;
 }
 
+// host_validated: the batch passed host_validate (host-array calls): no device
+// validation and no synchronisation -- the append and the update are enqueued
+// behind whatever the stream is still running.
 static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, int64_t cnt,
-                                dbc_insert_stats *stats) {
+                                dbc_insert_stats *stats, bool host_validated) {
     if (!c->have_state) return fail(c, DBC_ESTATE, "dbc_static_compute must run before insertions");
     if (cnt < 0 || (cnt > 0 && (!u || !v))) return fail(c, DBC_EINVAL, "bad batch");
     if (cnt > INT32_MAX / 4) return fail(c, DBC_EINVAL, "batch too large");
@@ -994,13 +1058,21 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     cudaEvent_t *ev = c->ev + (c->evset ? 0 : 6);
     if (tm) CK(cudaEventRecord(ev[0], c->stream));
     GView g = view_of(c);
-    launches += validate_batch(c->ab, g, c->rp[c->cur], c->n, u, v, cnt, c->nsm, c->stream);
-    CK(cudaGetLastError());
     int32_t bad = 0;
-    CK(cudaMemcpyAsync(&bad, c->ab.bad, sizeof(int32_t), cudaMemcpyDeviceToHost, c->stream));
-    CK(cudaStreamSynchronize(c->stream));  // all earlier work is complete here
+    // the batch's per-vertex groups (and, unless validated on the host, its checks)
+    launches += validate_batch(c->ab, g, c->rp[c->cur], c->n, u, v, cnt, c->nsm, c->stream, !host_validated);
+    CK(cudaGetLastError());
+    if (!host_validated) {
+        CK(cudaMemcpyAsync(&bad, c->ab.bad, sizeof(int32_t), cudaMemcpyDeviceToHost, c->stream));
+        CK(cudaStreamSynchronize(c->stream));  // all earlier work is complete here
+    } else if (c->tm_pending) {  // DBC_FLAG_TIMING: the previous call's events must be complete
+        cudaEvent_t *pe = c->ev + (c->evset ? 6 : 0);
+        CK(cudaEventSynchronize(pe[3]));
+    }
     TRY(fold_timings(c));
-    if (c->prof_pending) {  // chain time per root of the previous batch (heavy-lane choice)
+    // chain time per root of the previous batch (longest-first order, heavy lanes):
+    // read once it is complete -- an unfinished batch leaves the older order
+    if (c->prof_pending && cudaEventQuery(c->ev_prof) == cudaSuccess) {
         std::vector<unsigned long long> pr((size_t)6 * c->k_loc);
         CK(cudaMemcpy(pr.data(), c->root_prof, sizeof(unsigned long long) * pr.size(),
                       cudaMemcpyDeviceToHost));
@@ -1008,12 +1080,8 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
         for (int i = 0; i < c->k_loc; ++i) c->root_ms[i] = (double)(pr[6 * i + 1] - pr[6 * i]) * 1e-6;
         c->prof_pending = false;
     }
-    if (bad) {
-        const char *why = (bad & 1) ? "self loop or vertex out of range"
-                          : (bad & 2) ? "edge already present"
-                                      : "duplicate edge within the batch";
-        return fail(c, DBC_EEDGE, "batch rejected: %s", why);
-    }
+    cudaGetLastError();  // cudaEventQuery's cudaErrorNotReady is not an error
+    if (bad) return fail(c, DBC_EEDGE, "batch rejected: %s", bad_batch_why(bad));
     unsigned long long h0[kStCount] = {};
     if (stats) TRY(read_stats(c, h0));
     if (cnt == 0) {
@@ -1218,6 +1286,7 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
                 launch_update_256(a, wl, c->stream);
             ++ulaunch;
             if (nh > 0) CK(cudaStreamWaitEvent(c->stream, c->ev_join, 0));
+            CK(cudaEventRecord(c->ev_prof, c->stream));
             c->prof_pending = true;
             c->tm.heavy_roots = nh;
         } else {
@@ -1273,9 +1342,16 @@ extern "C" dbc_status dbc_insert_edges_device(dbc_ctx *c, const int32_t *u, cons
                     (long long)c->edge_cap, (long long)c->inserted, (long long)count);
     if (!c->have_state) return fail(c, DBC_ESTATE, "dbc_static_compute must run before insertions");
     CK(cudaSetDevice(c->device));
+    std::vector<int32_t> hu((size_t)count), hv((size_t)count);  // for the host copy of the graph
+    if (count) {
+        CK(cudaMemcpyAsync(hu.data(), u, sizeof(int32_t) * count, cudaMemcpyDeviceToHost, c->stream));
+        CK(cudaMemcpyAsync(hv.data(), v, sizeof(int32_t) * count, cudaMemcpyDeviceToHost, c->stream));
+    }
     map_ids(u, v, c->bu, c->bv, count, c->perm_d, c->n, c->stream);  // caller's ids -> internal
     CK(cudaGetLastError());
-    return insert_device(c, c->bu, c->bv, count, stats);
+    const dbc_status s = insert_device(c, c->bu, c->bv, count, stats, false);  // validates, synchronises
+    if (s == DBC_OK) host_record_insert(c, hu.data(), hv.data(), count);
+    return s;
 }
 
 extern "C" dbc_status dbc_insert_edges(dbc_ctx *c, const int32_t *u, const int32_t *v, int64_t count,
@@ -1286,6 +1362,11 @@ extern "C" dbc_status dbc_insert_edges(dbc_ctx *c, const int32_t *u, const int32
         return fail(c, DBC_ECAPACITY, "edge capacity %lld exhausted (%lld inserted, batch %lld)",
                     (long long)c->edge_cap, (long long)c->inserted, (long long)count);
     if (!c->have_state) return fail(c, DBC_ESTATE, "dbc_static_compute must run before insertions");
+    if (c->scen_cap > 0 && count > c->scen_cap)  // before anything changes (state unchanged on error)
+        return fail(c, DBC_EINVAL, "batch of %lld exceeds the scenario log (%lld insertions)",
+                    (long long)count, (long long)c->scen_cap);
+    if (const int bad = host_validate(c, u, v, count))  // nothing has changed yet
+        return fail(c, DBC_EEDGE, "batch rejected: %s", bad_batch_why(bad));
     CK(cudaSetDevice(c->device));
     if (count) {
         CK(cudaMemcpyAsync(c->bu, u, sizeof(int32_t) * count, cudaMemcpyHostToDevice, c->stream));
@@ -1293,7 +1374,9 @@ extern "C" dbc_status dbc_insert_edges(dbc_ctx *c, const int32_t *u, const int32
         map_ids(c->bu, c->bv, c->bu, c->bv, count, c->perm_d, c->n, c->stream);
         CK(cudaGetLastError());
     }
-    return insert_device(c, c->bu, c->bv, count, stats);
+    const dbc_status s = insert_device(c, c->bu, c->bv, count, stats, true);
+    if (s == DBC_OK) host_record_insert(c, u, v, count);
+    return s;
 }
 
 // Edge deletions (decremental update, R20): validated as a whole
@@ -1422,6 +1505,7 @@ static dbc_status delete_host_ids(dbc_ctx *c, const int32_t *u, const int32_t *v
     }
     launches += ulaunch;
     c->deleted += cnt;
+    host_record_delete(c, u, v, cnt);
     c->tm.update_launches = ulaunch;
     c->tm.kernel_launches = launches;
     c->tm.update_launches_total += ulaunch;

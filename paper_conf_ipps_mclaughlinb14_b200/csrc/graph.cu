@@ -314,14 +314,17 @@ static int scan_launch(const int32_t *in, int32_t *out, int64_t cnt, int32_t *su
 }
 
 int validate_batch(const AppendBufs &B, const GView &g, const int32_t *rp_old, int32_t n,
-                   const int32_t *u, const int32_t *v, int64_t cnt, int nsm, cudaStream_t s) {
+                   const int32_t *u, const int32_t *v, int64_t cnt, int nsm, cudaStream_t s, bool check) {
     int launches = 0;
     cudaMemsetAsync(B.bad, 0, sizeof(int32_t), s);
     cudaMemsetAsync(B.xcnt, 0, sizeof(int32_t) * (size_t)n, s);
     if (cnt) {
-        k_validate_edges<<<blocks_for(cnt * 32, 256), 256, 0, s>>>(g, n, u, v, cnt, B.bad);
+        if (check) {  // host-validated batches skip the presence test
+            k_validate_edges<<<blocks_for(cnt * 32, 256), 256, 0, s>>>(g, n, u, v, cnt, B.bad);
+            ++launches;
+        }
         k_count<<<blocks_for(cnt, 256), 256, 0, s>>>(u, v, cnt, n, B.xcnt, B.slot);
-        launches += 2;
+        ++launches;
     }
     // xoff = exclusive scan of xcnt (group offsets)
     launches += scan_launch(B.xcnt, B.xoff, n, B.sums, s);

@@ -27,7 +27,7 @@ struct AppendBufs {
 
 int64_t scan_sums_capacity(int64_t n);
 int validate_batch(const AppendBufs &B, const GView &g, const int32_t *rp_old, int32_t n,
-                   const int32_t *u, const int32_t *v, int64_t cnt, int nsm, cudaStream_t s);
+                   const int32_t *u, const int32_t *v, int64_t cnt, int nsm, cudaStream_t s, bool check = true);
 int validate_deletions(const GView &g, int32_t n, const int32_t *u, const int32_t *v, int64_t cnt,
                        int32_t *bad, cudaStream_t s);
 int tombstone_edge(const int32_t *rp, int32_t *col, int32_t *scol, const int32_t *u, const int32_t *v,

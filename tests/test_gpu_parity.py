@@ -426,6 +426,59 @@ def test_error_paths_leave_state_unchanged():
         assert e.value.name == "DBC_ECAPACITY"
 
 
+def test_host_and_device_validation_agree():
+    """Host-array batches are validated on the host against the context's host
+    copy of the adjacency (no device round trip), device-array batches on the
+    device: the same batches get the same verdicts, and the host copy follows
+    insertions through either path and deletions (an inserted edge deleted and
+    re-inserted, an original edge deleted and re-inserted); the final state
+    matches the oracle after the same operations."""
+    import torch
+
+    from paper_conf_ipps_mclaughlinb14_b200 import DBCError
+
+    g = W.karate()
+    roots = np.arange(34, dtype=np.int32)
+    ref = oracle.NaiveDynamicBC(g, roots)
+
+    def dev(a):
+        return torch.tensor(a, dtype=torch.int32, device="cuda")
+
+    with _dbc(g, roots, edge_capacity=16) as dbc:
+        dbc.static_compute()
+
+        def verdict(u, v, device):
+            try:
+                if device:
+                    dbc.insert_edges(dev(u), dev(v))
+                else:
+                    dbc.insert_edges(np.array(u, np.int32), np.array(v, np.int32))
+                return "ok"
+            except DBCError as e:
+                return e.name
+
+        bad = [([3], [3]), ([0], [34]), ([-1], [2]), ([0], [1]), ([1], [0]), ([0, 9], [9, 0]),
+               ([0, 4], [9, 4]), ([0, 2], [9, 40])]
+        for u, v in bad:
+            assert verdict(u, v, False) == verdict(u, v, True) == "DBC_EEDGE", (u, v)
+        assert verdict([0], [9], True) == "ok"  # through the device path ...
+        ref.insert(0, 9)
+        assert verdict([9], [0], False) == "DBC_EEDGE"  # ... is present for the host path
+        assert verdict([14], [0], False) == "ok"
+        ref.insert(14, 0)
+        assert verdict([0], [14], True) == "DBC_EEDGE"
+        dbc.delete_edges([0], [1])  # an original edge
+        ref.delete(0, 1)
+        assert verdict([1], [0], False) == "ok"
+        ref.insert(1, 0)
+        dbc.delete_edges([9], [0])  # an inserted edge
+        ref.delete(9, 0)
+        assert verdict([0], [9], False) == "ok"
+        ref.insert(0, 9)
+        assert verdict([9], [0], False) == "DBC_EEDGE"
+        check_all(dbc, ref.compute(), roots.size)
+
+
 def test_scenario_log_oversized_batch_leaves_state_unchanged():
     """A batch larger than the scenario log is rejected before anything changes
     (the live graph, d/sigma/delta, BC): a later insertion of the same edges
