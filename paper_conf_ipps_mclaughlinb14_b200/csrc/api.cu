@@ -87,6 +87,7 @@ struct dbc_ctx {
     int64_t lean_max = 1;            // merged batches of <= this many insertions also run there
     int lean_short = 4;              // level-2 shortcut threshold (rows > lean_short x deg(root))
     int lean_block = 128;            // threads per update_lean.cu CTA
+    int lean_narrow = 0;             // > 0: 128-thread workers for multi-insertion launches (meshes)
     void *lean_board = nullptr;      // its help board (one entry per worker)
     size_t nscratch = 0;             // worker scratch sets allocated
     // heavy lanes: the slowest root chains of the previous batch run on
@@ -665,9 +666,18 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
                            : c->lean_block == 512 ? lean_resident_512()
                            : c->lean_block == 256 ? lean_resident_256() : lean_resident_128();
         c->lean_workers = std::min(c->lean_workers, std::max(1, per_sm) * c->nsm);
+        // meshes (narrow levels) with more roots than resident wide workers: a
+        // launch over many insertions (DBC_FLAG_NO_MERGE) runs 128-thread
+        // workers so every root has one (Delaunay 2^18, 512 roots: 296 -> 512
+        // workers, +50%); single-insertion launches keep the wide CTAs, whose
+        // heaviest job sets the launch time
+        if (c->lowdeg && T.lean_block <= 0 && c->lean_block > 128 && c->k_loc > c->lean_workers) {
+            const int w = std::min({c->k_loc, fit, std::max(1, lean_resident_128()) * c->nsm});
+            if (w > c->lean_workers) c->lean_narrow = w;
+        }
     }
     const size_t nwk = std::max({(size_t)c->workers + c->heavy_cap, (size_t)c->sworkers,
-                                 (size_t)c->lean_workers});  // both lanes; static; per-insertion
+                                 (size_t)c->lean_workers, (size_t)c->lean_narrow});  // both lanes; static; per-insertion
     c->nscratch = nwk;
     const size_t wn = nwk * n;
     AL(c->ws.mark, wn);
@@ -701,9 +711,10 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->next_slot, 4);  // [0] next root, [1] heavy lane's next root / unused, [2..3] lean: roots done, idle
     if (c->lean_workers) {
         char *bd = nullptr;
-        AL(bd, lean_board_bytes() * (size_t)c->lean_workers);
+        const size_t nlw = (size_t)std::max(c->lean_workers, c->lean_narrow);
+        AL(bd, lean_board_bytes() * nlw);
         c->lean_board = (T.disable & DBC_TUNE_NO_LEAN_HELP) ? nullptr : (void *)bd;
-        cudaMemsetAsync(bd, 0, lean_board_bytes() * (size_t)c->lean_workers, c->stream);
+        cudaMemsetAsync(bd, 0, lean_board_bytes() * nlw, c->stream);
     }
     AL(c->slots_d, (size_t)std::max(c->k_loc, 1));
     AL(c->stats, (size_t)kStAlloc);
@@ -1157,7 +1168,8 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     a.pull_delta = pull ? 1 : 0;
     a.short_mult = c->lean_short;
     if (use_lean) {
-        const int nw = c->lean_workers;
+        const bool narrow = c->lean_narrow > 0 && !(c->flags & DBC_FLAG_MODE_S) && cnt > 1;
+        const int nw = narrow ? c->lean_narrow : c->lean_workers;
         a.lean_board = pull ? nullptr : c->lean_board;  // pull mode: every pass local
         a.merge = 0;
         a.root_prof = c->prof_on ? c->root_prof : nullptr;
@@ -1170,7 +1182,9 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
             CK(cudaMemsetAsync(c->next_slot, 0, 4 * sizeof(int32_t), c->stream));
             a.ins_begin = (int32_t)i;
             a.ins_end = (int32_t)std::min<int64_t>(cnt, i + step);
-            if (c->lean_block == 1024)
+            if (narrow)
+                launch_update_lean_128(a, nw, c->stream);
+            else if (c->lean_block == 1024)
                 launch_update_lean_1024(a, nw, c->stream);
             else if (c->lean_block == 512)
                 launch_update_lean_512(a, nw, c->stream);

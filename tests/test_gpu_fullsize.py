@@ -125,6 +125,17 @@ def test_rmat16_bench_batch_all_roots():
 
 
 # ---------------------------------------------------------------- config 3 ----
+@pytest.mark.timeout(600)
+def test_delaunay18_no_merge_all_roots():
+    """Config 3 in the paper's one-job-per-insertion structure (DBC_FLAG_NO_MERGE:
+    the per-insertion kernel, which on this mesh runs 128-thread workers so all
+    512 roots are resident): batches of 100, BC over all roots after each, 64
+    sampled roots' d/sigma/delta."""
+    from paper_conf_ipps_mclaughlinb14_b200 import FLAG_NO_MERGE
+
+    run_cadence("delaunay18", 100, flags=FLAG_NO_MERGE, insertions=300)
+
+
 @pytest.mark.timeout(900)
 def test_delaunay18_every_100th_all_roots():
     """Config 3 (remove-then-reinsert): every 100th insertion, BC over all 512
