@@ -1076,9 +1076,9 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     if (!host_validated) {
         CK(cudaMemcpyAsync(&bad, c->ab.bad, sizeof(int32_t), cudaMemcpyDeviceToHost, c->stream));
         CK(cudaStreamSynchronize(c->stream));  // all earlier work is complete here
-    } else if (c->tm_pending) {  // DBC_FLAG_TIMING: the previous call's events must be complete
-        cudaEvent_t *pe = c->ev + (c->evset ? 6 : 0);
-        CK(cudaEventSynchronize(pe[3]));
+    } else {  // DBC_FLAG_TIMING: the events fold_timings reads must be complete
+        if (c->tm_pending) CK(cudaEventSynchronize((c->ev + (c->evset ? 6 : 0))[3]));
+        if (c->tm_static) CK(cudaEventSynchronize(c->ev[5]));
     }
     TRY(fold_timings(c));
     // chain time per root of the previous batch (longest-first order, heavy lanes):

@@ -479,6 +479,24 @@ def test_host_and_device_validation_agree():
         check_all(dbc, ref.compute(), roots.size)
 
 
+def test_async_host_inserts_with_timing():
+    """Host-array insertions do not synchronise: back-to-back calls right after
+    dbc_static_compute with DBC_FLAG_TIMING (whose events the next call folds)
+    must work and give the oracle's state; the timings are filled in."""
+    from paper_conf_ipps_mclaughlinb14_b200 import FLAG_TIMING
+
+    wl = W.make_workload("karate")
+    ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
+    with _dbc(wl.graph, wl.roots, flags=FLAG_TIMING) as dbc:
+        dbc.static_compute()  # no synchronize: the next call folds the static events
+        for u, v in zip(wl.ins_u.tolist(), wl.ins_v.tolist()):
+            dbc.insert_edges([u], [v])
+            ref.insert(u, v)
+        t = dbc.timings()
+        assert t["static_ms"] > 0 and t["update_ms"] > 0 and t["insertions_total"] == wl.ins_u.size
+        check_all(dbc, ref.compute(), wl.roots.size)
+
+
 def test_scenario_log_oversized_batch_leaves_state_unchanged():
     """A batch larger than the scenario log is rejected before anything changes
     (the live graph, d/sigma/delta, BC): a later insertion of the same edges
