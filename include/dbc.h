@@ -255,19 +255,22 @@ dbc_status dbc_static_compute(dbc_ctx *c);
  * "reinserted one at a time").  The whole batch is validated before anything
  * changes (self loop, range, already present, duplicate in batch ->
  * DBC_EEDGE; capacity -> DBC_ECAPACITY).  Requires a prior
- * dbc_static_compute (DBC_ESTATE).  The batch is validated on the host against
- * the context's host copy of the adjacency (caller ids: the original rows
- * sorted, plus the inserted and deleted edges), so the call does not wait for
- * the device: the append and the update are enqueued asynchronously behind
- * earlier work on the stream.  It synchronises only with DBC_FLAG_TIMING (on
- * the previous call's events) or when stats is non-NULL.  stats: nullable. */
+ * dbc_static_compute (DBC_ESTATE).  Batches of up to 64 edges are validated on
+ * the host against the context's host copy of the adjacency (caller ids: the
+ * original rows sorted, plus the inserted and deleted edges), so the call does
+ * not wait for the device: the append and the update are enqueued
+ * asynchronously behind earlier work on the stream (it synchronises only with
+ * DBC_FLAG_TIMING, on the previous call's events, or when stats is non-NULL).
+ * Larger batches are validated on the device and the call synchronises once
+ * after validation; the update itself is enqueued asynchronously.  stats:
+ * nullable. */
 dbc_status dbc_insert_edges(dbc_ctx *c, const int32_t *u, const int32_t *v,
                             int64_t count, dbc_insert_stats *stats);
 
 /* Same as dbc_insert_edges with u, v in DEVICE memory (int32[count] each),
  * read in order after the work queued on the context stream.  Validated on the
- * device; synchronises once after validation (and copies the batch to the host
- * for the host copy of the adjacency). */
+ * device; synchronises once after validation (and copies the batch, through
+ * pinned staging allocated on first use, to the host copy of the adjacency). */
 dbc_status dbc_insert_edges_device(dbc_ctx *c, const int32_t *u_device,
                                    const int32_t *v_device, int64_t count,
                                    dbc_insert_stats *stats);
