@@ -524,7 +524,14 @@ def run_ours(args):
         ev1.record(stream)
         torch.cuda.synchronize()
         ms2 = ev0.elapsed_time(ev1)
+        t2 = dS.timings()
+        l2 = max(t2["update_launches_total"], 1)
+        ach2 = (t2["alg_bytes_total"] / l2) / (t2["update_ms_total"] / l2 / 1e3) / 1e9 if t2["update_ms_total"] else 0
         per_ins["mode_s"] = {"value": NS / (ms2 / 1e3), "unit": "insertions/s", "insertions": NS,
+                             "speedup_vs_static": (static_ms / 1e3) / (ms2 / 1e3 / NS),
+                             "launches": int(t2["update_launches_total"]),
+                             "roofline": {"bound": "hbm", "achieved": ach2, "peak": peak, "unit": "GB/s",
+                                          "frac": ach2 / peak, "kernel": "lean_kernel"},
                              "what": "Mode S: one per-insertion kernel launch over all roots per insertion "
                                      "(P:244-252)"}
         dS.close()
