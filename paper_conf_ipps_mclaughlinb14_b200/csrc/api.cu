@@ -122,6 +122,7 @@ struct dbc_ctx {
 
     Scratch ws{};
     int32_t *next_slot = nullptr;
+    bool lean_clean = false;          // next_slot[0..4] zero: left so by the per-insertion kernel's last CTA
     unsigned long long *stats = nullptr;
     int32_t *err = nullptr;
     unsigned long long *root_prof = nullptr;  // [k_loc][4], filled when profiling is on
@@ -710,7 +711,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->help.gbig, 2 * nwk);
     c->help.nworkers = (int)nwk;
     if (T.disable & DBC_TUNE_NO_HELP) c->help_on = false;
-    AL(c->next_slot, 4);  // [0] next root, [1] heavy lane's next root / unused, [2..3] lean: roots done, idle
+    AL(c->next_slot, 8);  // [0] next root, [1] heavy lane's next root / unused, [2..3] lean: roots done, idle, [4] lean: CTAs out
     if (c->lean_workers) {
         char *bd = nullptr;
         const size_t nlw = (size_t)std::max(c->lean_workers, c->lean_narrow);
@@ -971,6 +972,7 @@ extern "C" dbc_status dbc_static_compute(dbc_ctx *c) {
         if (tm) CK(cudaEventRecord(c->ev[4], c->stream));
         CK(cudaMemsetAsync(c->bc, 0, sizeof(double) * c->n, c->stream));
         CK(cudaMemsetAsync(c->next_slot, 0, sizeof(int32_t), c->stream));
+        c->lean_clean = false;
         CK(cudaMemsetAsync(c->stats + kStStaticBytes, 0, sizeof(unsigned long long), c->stream));
     }
     if (c->workers && !ms_done) {
@@ -1182,7 +1184,9 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
                                c->stream));
         const int64_t step = (c->flags & DBC_FLAG_MODE_S) ? 1 : cnt;  // Mode S: one launch per insertion
         for (int64_t i = 0; i < cnt; i += step) {
-            CK(cudaMemsetAsync(c->next_slot, 0, 4 * sizeof(int32_t), c->stream));
+            if (!c->lean_clean)  // else the previous launch's last CTA left the counters at zero
+                CK(cudaMemsetAsync(c->next_slot, 0, 5 * sizeof(int32_t), c->stream));
+            c->lean_clean = true;
             a.ins_begin = (int32_t)i;
             a.ins_end = (int32_t)std::min<int64_t>(cnt, i + step);
             if (narrow)
@@ -1220,6 +1224,7 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
         e.next_slot = c->next_slot;
         for (int64_t i = 0; i < cnt; ++i) {
             CK(cudaMemsetAsync(c->next_slot, 0, sizeof(int32_t), c->stream));
+            c->lean_clean = false;
             e.ins = (int32_t)i;
             launch_edge_update(e, c->eworkers, c->stream);
             ++ulaunch;
@@ -1252,6 +1257,7 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
             CK(cudaMemcpyAsync(c->slots_d, list.data(), sizeof(int32_t) * k, cudaMemcpyHostToDevice,
                                c->stream));
             CK(cudaMemsetAsync(c->next_slot, 0, 2 * sizeof(int32_t), c->stream));
+            c->lean_clean = false;
             a.ins_begin = 0;
             a.ins_end = (int32_t)cnt;
             if (c->help_on) {  // fresh board: all requests closed, every root chain pending
@@ -1309,6 +1315,7 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
         } else {
             for (int64_t i = 0; i < cnt; ++i) {
                 CK(cudaMemsetAsync(c->next_slot, 0, sizeof(int32_t), c->stream));
+                c->lean_clean = false;
                 a.ins_begin = (int32_t)i;
                 a.ins_end = (int32_t)i + 1;
                 if (c->block == 128)
@@ -1510,6 +1517,7 @@ static dbc_status delete_host_ids(dbc_ctx *c, const int32_t *u, const int32_t *v
                                    c->stream);
         if (c->workers) {
             CK(cudaMemsetAsync(c->next_slot, 0, sizeof(int32_t), c->stream));
+            c->lean_clean = false;
             a.ins_begin = (int32_t)i;
             a.ins_end = (int32_t)i + 1;
             if (c->block == 128)

@@ -1172,6 +1172,13 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
         if (s_red[1]) atomicAdd(stl + kStBytes, s_red[1]);
         if (s_red[2]) atomicAdd(stl + kStScanned, s_red[2]);
     }
+    if (tid == 0) {  // the last CTA out zeroes the launch counters for the next launch (no memset)
+        __threadfence();
+        if (atomicAdd(a.next_slot + 4, 1) == (int)gridDim.x - 1) {
+            for (int q = 0; q < 5; ++q) a.next_slot[q] = 0;
+            __threadfence();
+        }
+    }
     if (cta_prof && tid == 0) {
         unsigned long long t;
         asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));

@@ -119,6 +119,18 @@ def test_rmat16_every_10th_insertion_all_roots():
 
 
 @pytest.mark.timeout(600)
+def test_rmat16_mode_s_and_single_edge_calls_all_roots():
+    """Config 2 through the per-insertion kernel at full size: Mode S (one launch
+    per insertion over all roots) in batches of 50, then single-edge calls;
+    BC over all 256 roots after each call, every root's d/sigma/delta at the
+    end of each batch."""
+    from paper_conf_ipps_mclaughlinb14_b200 import FLAG_MODE_S
+
+    run_cadence("rmat16", 50, flags=FLAG_MODE_S, sample=256, insertions=200)
+    run_cadence("rmat16", 1, sample=64, state_every=10, insertions=30)
+
+
+@pytest.mark.timeout(600)
 def test_rmat16_bench_batch_all_roots():
     """Config 2 exactly as bench.py times it: one 1,000-insertion batch."""
     run_cadence("rmat16", 1000, sample=256)
