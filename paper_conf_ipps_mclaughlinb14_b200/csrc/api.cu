@@ -657,9 +657,11 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     if (T.lean_max_batch >= 0) c->lean_max = T.lean_max_batch;
     if (T.lean_short >= 0) c->lean_short = T.lean_short;
     // per-insertion CTA width (measured on B200): hub-heavy
-    // graphs need wide CTAs for their heavy levels (R-MAT 16: 512), meshes are
+    // graphs need wide CTAs for their heavy levels (R-MAT 16: 512; Kronecker 20,
+    // 10^6 vertices, whose heaviest jobs set a single-edge launch: 1024, 2.13 ->
+    // 1.78 ms, Mode S and one job per insertion unchanged), meshes are
     // latency-bound on narrow levels (Delaunay 2^18: 256)
-    c->lean_block = c->lowdeg ? 256 : 512;
+    c->lean_block = c->lowdeg ? 256 : (c->n >= (1 << 20) ? 1024 : 512);
     if (T.lean_block > 0) {
         const int b = T.lean_block;
         c->lean_block = (b == 256 || b == 512 || b == 1024) ? b : 128;

@@ -1065,6 +1065,28 @@ def test_lean_fewer_workers_than_roots(name, tune):
             check_all(dbc, want, wl.roots.size)
 
 
+@pytest.mark.parametrize("width", [128, 256, 512, 1024])
+def test_lean_every_cta_width(width, tune):
+    """The per-insertion kernel at every CTA width (128/256/512/1024 threads:
+    meshes' multi-insertion launches, meshes, hub graphs, million-vertex hub
+    graphs), one-job-per-insertion batch, Mode S and single-edge calls."""
+    tune["lean_block"] = width
+    wl = W.make_workload("rmat10")
+    ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
+    for u, v in zip(wl.ins_u, wl.ins_v):
+        ref.insert(u, v)
+    want = ref.compute()
+    for flags in (0x10, 0x1, 0):
+        with _dbc(wl.graph, wl.roots, flags=flags) as dbc:
+            dbc.static_compute()
+            if flags:
+                dbc.insert_edges(wl.ins_u, wl.ins_v)
+            else:
+                for u, v in zip(wl.ins_u.tolist(), wl.ins_v.tolist()):
+                    dbc.insert_edges([u], [v])
+            check_all(dbc, want, wl.roots.size)
+
+
 @pytest.mark.parametrize("mult", ["0", "1"])
 def test_lean_level2_shortcut_forced(mult, tune):
     """Level-2 up vertices resolved against adj(root) (probing the sorted rows)
