@@ -76,8 +76,10 @@ struct dbc_ctx {
     bool lowdeg = false;  // max degree <= 32 (mesh-like graphs)
     int64_t maxdeg0 = 0;  // max degree of the initial graph
     int hd_min = 1024, hd_block = 512;  // helped down levels (update.cu)
-    int he_entries = 4096, he_min = 3;   // helped flattened passes (update.cu)
-    int busy_help = 1;                   // blocks a busy worker takes at a level boundary
+    int he_entries = 8192, he_min = 3;   // helped flattened passes (update.cu)
+    int busy_help = 4;                   // blocks a busy worker takes at a level boundary
+                                         // (re-tuned after the counter lanes, DESIGN.md Sec. 9:
+                                         // 1 -> 4 and 4096 -> 8192 entries, R-MAT 16 -8%)
     int busy_min = 32;                   // ... of passes of at least this many blocks
     int dl_min = 16 * 4096;              // entry-balanced long rows of a down level from this many entries
     int wide_inlane = -1;                // up levels of <= this many items per thread: short rows in-lane
