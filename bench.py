@@ -299,6 +299,33 @@ def run_reference(args):
     return 0
 
 
+def shared_workload(name, seed, insertions, k, world, rank):
+    """The seeded workload; under torchrun rank 0 builds it once and the other
+    ranks of the node load its arrays from /tmp (generating Kronecker 22 takes
+    ~100 s of host time per process; every rank needs the same replicated graph)."""
+    if world == 1:
+        return W.make_workload(name, seed=seed, insertions=insertions, k=k)
+    import torch.distributed as dist
+
+    tag = os.environ.get("TORCHELASTIC_RUN_ID", "") + os.environ.get("MASTER_PORT", "")
+    path = os.path.join("/tmp", f"dbc_wl_{name}_{seed}_{insertions}_{k}_{tag}.npz")
+    if rank == 0:
+        wl = W.make_workload(name, seed=seed, insertions=insertions, k=k)
+        tmp = path + f".{os.getpid()}.npz"
+        np.savez(tmp, n=np.int64(wl.graph.n), row_ptr=wl.graph.row_ptr, col=wl.graph.col, roots=wl.roots,
+                 ins_u=wl.ins_u, ins_v=wl.ins_v, meta=np.array(json.dumps(wl.meta, default=str)))
+        os.replace(tmp, path)
+    dist.barrier()
+    if rank != 0:
+        z = np.load(path)
+        g = W.CSR(int(z["n"]), z["row_ptr"], z["col"])
+        wl = W.Workload(name, g, z["roots"], z["ins_u"], z["ins_v"], json.loads(str(z["meta"])))
+    dist.barrier()
+    if rank == 0:
+        os.remove(path)
+    return wl
+
+
 # -------------------------------------------------------------------- ours ----
 def run_ours(args):
     import torch
@@ -340,7 +367,7 @@ def run_ours(args):
     Wm, K = args.warmup, args.steps
     e2e_steps = 0 if args.no_e2e else (Wm + K)
     nb = n_batches(args, B)
-    wl = W.make_workload(args.config, seed=args.seed, insertions=B * nb, k=k)
+    wl = shared_workload(args.config, args.seed, B * nb, k, world, rank)
     g = wl.graph
     flags = FLAG_TIMING | (FLAG_MODE_S if args.mode == "S" else 0) | (FLAG_NO_MERGE if args.no_merge else 0)
     stream = torch.cuda.Stream(device=dev)  # the library and the timing events share it
