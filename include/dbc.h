@@ -370,10 +370,11 @@ dbc_status dbc_scenario_log(dbc_ctx *c, int64_t max_insertions);
  * record [i * k_local + j] is insertion i of the batch seen by local root slot
  * j (local slot j = global slot j * world + rank), encoded as
  * case | (touched << 2) | (down << 33): case 1, 2 or 3;
- * touched = number of vertices the update touched (t[v] != untouched, P:512;
- * the root excluded; ancestors are reached only through non-zero
- * Delta-delta, so this is a subset of Alg. 2's touched set); down = |D|, the
- * vertices whose d/sigma were recomputed.  Both 0 for Case 1.
+ * touched = number of vertices the update touched, Alg. 2's
+ * {v : t[v] != untouched} with the root excluded -- with the log on,
+ * every DAG ancestor of a changed vertex is claimed even over a zero
+ * Delta-delta push (R19); down = |D|, the vertices whose d/sigma were
+ * recomputed.  Both 0 for Case 1.
  * *count receives the number of records; out may be NULL to query it.
  * capacity < *count -> DBC_EINVAL.  Synchronises. */
 dbc_status dbc_get_scenarios(dbc_ctx *c, int64_t *out, int64_t capacity, int64_t *count);
