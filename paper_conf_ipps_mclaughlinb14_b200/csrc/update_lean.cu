@@ -78,6 +78,11 @@ constexpr int kHelpBlk = DBC_LEAN_HELPBLK;  // entries per help block
 constexpr int kHelpMinBlk = DBC_LEAN_HELPMIN;  // passes of at least this many blocks are published
 constexpr int kLEnt = 1536;       // entries whose contributions are kept for an in-order row sum
 constexpr int kSpecEntries = 2 * kBlock * kLU;  // passes up to this size gather speculatively
+// Shared-memory copy of the job's D list (ids, old d, old sigma) for its first
+// kDMir entries: the up phase's D rows and the removal pass read them without a
+// global round trip.  Dynamic shared memory (kLDyn bytes).
+constexpr int kDMir = kBlock * 2 < 1024 ? kBlock * 2 : 1024;
+constexpr int kLDyn = kDMir * (int)(2 * sizeof(int) + sizeof(double));
 
 // pass kinds (entry visitors)
 enum : int { kPDown = 1, kPUp = 2, kPRem = 3, kPDRow = 4, kPDPush = 5 };
@@ -140,6 +145,7 @@ struct PassCtx {
     int *mir;                    // nullable: shared mirror of the list's entries [mbase, mbase + kLCap)
     int mbase;
     int mirbit;                  // its s_mirbad bit
+    int *dmir;                   // nullable: shared copy of the D list (down passes of the owner)
     int *low, *rmin, *rmax;
     double *acc;                 // per-row sums (when ev == nullptr)
     double *ev;                  // per-entry contributions (a local pass of <= kLEnt entries)
@@ -240,6 +246,7 @@ __device__ __forceinline__ void claim_append(const PassCtx &c, int y, uint32_t m
         const int p = atomicAdd(c.ctr, 1);
         c.list[p] = y;
         if (c.mir && p - c.mbase < kLCap) c.mir[p - c.mbase] = y;
+        if (c.dmir && p < kDMir) c.dmir[p] = y;
     }
 }
 
@@ -414,6 +421,7 @@ __device__ __forceinline__ void lean_pass_k(const PassCtx &c, LeanSmem &S, int *
                 const int p = atomicAdd(c.ctr, 1);
                 c.list[p] = y[u];
                 if (c.mir && p - c.mbase < kLCap) c.mir[p - c.mbase] = y[u];
+                if (c.dmir && p < kDMir) c.dmir[p] = y[u];
                 if (K == kPRem) {  // removal targets keep their level
                     c.list2[p] = dy[u];
                     atomicMin(c.rmin, dy[u]);
@@ -448,6 +456,10 @@ __device__ __forceinline__ void lean_pass(const PassCtx &c, LeanSmem &S, int *s_
 #endif
 __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs a) {
     __shared__ LeanSmem S;
+    extern __shared__ double s_dyn[];  // dynamic: D list copy (old sigma, then ids, then old d)
+    double *s_dsig = s_dyn;
+    int *s_dmir = reinterpret_cast<int *>(s_dyn + kDMir);
+    int *s_dold = s_dmir + kDMir;
     __shared__ int s_slot, s_nwork, s_dcnt, s_ucnt[2], s_rcnt, s_rmin, s_rmax, s_nst, s_nsc, s_low, s_ds;
     __shared__ int s_mirbad;  // bit (L & 1): the down mirror of level L is incomplete; bit 2 + i: up list i's
     __shared__ unsigned long long s_tph[10];  // tuning.trace_slot: SM cycles per phase of that root (thread 0)
@@ -564,7 +576,9 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
         gc.ev = nullptr;
         gc.stash = false;  // helpers' shared memory is their own: D-row pushes run as a kPDPush pass
         gc.mir = nullptr;  // helpers append to the list only: its mirror is incomplete
+        gc.dmir = nullptr;
         if (tid == 0 && c.mir) s_mirbad |= c.mirbit;
+        if (tid == 0 && c.dmir) s_mirbad |= 256;  // the D id mirror too
         for (;;) {  // the owner takes blocks too
             if (tid == 0) {
                 const unsigned long long w = atomicAdd(&mine->word, 1ull << 16);
@@ -666,6 +680,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                 pc.stash = false;
                 pc.ptr = trace ? a.stats + kStTrace0 : nullptr;
                 pc.mir = nullptr;
+                pc.dmir = nullptr;
                 pc.mbase = 0;
                 pc.mirbit = 0;
                 // ---- seed (A2) ----
@@ -682,6 +697,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                     s_low = c3;
                     mark[ul] = mD;
                     Dv[0] = ul;
+                    s_dmir[0] = ul;
                     S.nx[0] = ul;
                     s_mirbad = 0;
                     Doff[0] = 0;
@@ -709,8 +725,14 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                             const int w = (c == lb && mir_ok) ? S.nx[t] : __ldcg(Dv + c + t);
                             const int2 r = row_of(g, w, lim);
                             const unsigned long long lr = __ldcg(lowrec + w);
-                            Dold[c + t] = ((lr >> 32) == epoch) ? (int)(uint32_t)lr : L;
-                            Dsig[c + t] = __ldcg(&st.sd[w].x);
+                            const int od = ((lr >> 32) == epoch) ? (int)(uint32_t)lr : L;
+                            const double os = __ldcg(&st.sd[w].x);
+                            Dold[c + t] = od;
+                            Dsig[c + t] = os;
+                            if (c + t < kDMir) {
+                                s_dold[c + t] = od;
+                                s_dsig[c + t] = os;
+                            }
                             S.v[t] = w;
                             S.beg[t] = r.x;
                             S.off[t + 1] = r.y - r.x;
@@ -727,6 +749,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                         cdn.list = Dv;
                         cdn.ctr = &s_dcnt;
                         cdn.mir = S.nx;
+                        cdn.dmir = s_dmir;
                         cdn.mbase = le;
                         cdn.mirbit = 1 << ((L + 1) & 1);
                         const bool in_acc = run_pass(cdn, cnt, Etot, slot, 0, sc_ph[0]) & 1;
@@ -759,14 +782,16 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                 }
                 const int Lmax = L - 1;  // deepest D level
                 const int dtotal = le;
+                const bool dmir_ok = !(s_mirbad & 256);  // the D id copy is complete (no helped down pass)
 
                 // ---- removal pushes (A4 step 0, Case 3) ----
                 if (s_low) {
                     for (int c = 0; c < dtotal; c += kLCap) {
                         const int cnt = min(kLCap, dtotal - c);
                         for (int t = tid; t < cnt; t += kBlock) {
-                            const int w = __ldcg(Dv + c + t);
-                            const int od = __ldcg(Dold + c + t);
+                            const int j = c + t;
+                            const int w = (j < kDMir && dmir_ok) ? s_dmir[j] : __ldcg(Dv + j);
+                            const int od = j < kDMir ? s_dold[j] : __ldcg(Dold + j);
                             const int dw = __ldcg(st.d + w);
                             int len = 0;
                             if (od != dw && od != kInf) {
@@ -774,7 +799,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                                 len = r.y - r.x;
                                 S.beg[t] = r.x;
                                 const double dold = __ldcg(&st.sd[w].y);  // delta is still the old one
-                                S.c0[t] = -__ddiv_rn(__dadd_rn(1.0, dold), __ldcg(Dsig + c + t));
+                                S.c0[t] = -__ddiv_rn(__dadd_rn(1.0, dold), j < kDMir ? s_dsig[j] : __ldcg(Dsig + j));
                                 S.aux[t] = od - 1;
                                 my_bytes += 8 + 16;
                             }
@@ -843,7 +868,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                         if (tid == 0) s_nst = 0;
                         for (int t = tid; t < cnt; t += kBlock) {
                             const int j = c + t;
-                            const int x = j < nd ? __ldcg(Dv + db + j)
+                            const int x = j < nd ? ((db + j < kDMir && dmir_ok) ? s_dmir[db + j] : __ldcg(Dv + db + j))
                                           : ((j - nd < kLCap && umir_ok) ? S.um[cu][j - nd] : __ldcg(Ul[cu] + j - nd));
                             const double2 q = __ldcg(st.sd + x);  // (sigma_new, delta_old)
                             const int2 r = row_of(g, x, lim);
@@ -885,9 +910,9 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
                                 st.sd[x].y = dn;
                             }
                             if (di >= 0) {
-                                const bool lowered = __ldcg(Dold + di) != l;
+                                const bool lowered = (di < kDMir ? s_dold[di] : __ldcg(Dold + di)) != l;
                                 S.c0[t] = __ddiv_rn(__dadd_rn(1.0, dn), sn);
-                                S.c1[t] = lowered ? 0.0 : __ddiv_rn(__dadd_rn(1.0, dold), __ldcg(Dsig + di));
+                                S.c1[t] = lowered ? 0.0 : __ddiv_rn(__dadd_rn(1.0, dold), di < kDMir ? s_dsig[di] : __ldcg(Dsig + di));
                             }
                             my_bytes += 16 + 16;
                         }
@@ -1117,6 +1142,7 @@ __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs 
             c.stash = false;
             c.ptr = nullptr;
             c.mir = nullptr;
+            c.dmir = nullptr;
             uint32_t hscan = 0;
             lean_pass(c, S, &s_nst, g, cnt, b * kHelpBlk, min(Etot, (b + 1) * kHelpBlk), my_bytes, hscan);
             my_scan += hscan;
@@ -1195,12 +1221,18 @@ size_t lean_board_bytes() { return sizeof(LeanBoard); }
 #define DBC_CAT2(a, b) a##b
 #define DBC_CAT(a, b) DBC_CAT2(a, b)
 void DBC_CAT(launch_update_lean_, DBC_BLOCK)(const UpdateArgs &a, int workers, cudaStream_t s) {
-    lean_kernel<<<workers, kBlock, 0, s>>>(a);
+    static bool attr = false;
+    if (!attr) {
+        cudaFuncSetAttribute(lean_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kLDyn);
+        attr = true;
+    }
+    lean_kernel<<<workers, kBlock, kLDyn, s>>>(a);
 }
 
 int DBC_CAT(lean_resident_, DBC_BLOCK)() {
     int nb = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, lean_kernel, kBlock, 0);
+    cudaFuncSetAttribute(lean_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kLDyn);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, lean_kernel, kBlock, kLDyn);
     return nb;
 }
 
