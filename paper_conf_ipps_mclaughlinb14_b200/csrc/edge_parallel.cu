@@ -55,7 +55,7 @@ __device__ __forceinline__ void for_vertices(int n, F f) {
 }
 
 __global__ void __launch_bounds__(kEB, 1) edge_kernel(EdgeArgs a) {
-    __shared__ int s_slot, s_found, s_low, s_lmax;
+    __shared__ int s_slot, s_found, s_lmax;
     const int tid = threadIdx.x;
     const int wk = blockIdx.x;
     const int n = a.n;
@@ -87,7 +87,7 @@ __global__ void __launch_bounds__(kEB, 1) edge_kernel(EdgeArgs a) {
             ++c1;
             continue;
         }
-        const int uh = du < dv ? u : v, ul = du < dv ? v : u;
+        const int ul = du < dv ? v : u;
         const int L0 = min(du, dv) + 1;
         const bool case3 = max(du, dv) != L0;
         case3 ? ++c3 : ++c2;
@@ -108,7 +108,6 @@ __global__ void __launch_bounds__(kEB, 1) edge_kernel(EdgeArgs a) {
             odel[ul] = sd[ul].y;
             sd[ul] = make_double2(0.0, 0.0);
             s_found = 0;
-            s_low = case3;
             s_lmax = L0;
         }
         __syncthreads();

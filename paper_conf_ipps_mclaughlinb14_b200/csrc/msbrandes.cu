@@ -50,8 +50,6 @@ template <> struct MaskOf<1> { using T = uint32_t; };
 template <> struct MaskOf<2> { using T = unsigned long long; };
 __device__ __forceinline__ int popc_m(uint32_t x) { return __popc(x); }
 __device__ __forceinline__ int popc_m(unsigned long long x) { return __popcll(x); }
-__device__ __forceinline__ int ffs_m(uint32_t x) { return __ffs(x); }
-__device__ __forceinline__ int ffs_m(unsigned long long x) { return __ffsll(x); }
 template <class Mk> __device__ __forceinline__ bool bit(Mk m, int b) { return (m >> b) & 1u; }
 
 struct MsGroup {  // per-group counters (device)
