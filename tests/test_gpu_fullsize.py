@@ -130,6 +130,15 @@ def test_rmat16_mode_s_and_single_edge_calls_all_roots():
     run_cadence("rmat16", 1, sample=64, state_every=10, insertions=30)
 
 
+@pytest.mark.timeout(900)
+def test_rmat16_long_stream_all_roots():
+    """Config 2's graph over a 10x longer stream (10,000 insertions in 10 bench
+    batches): the incrementally updated BC (no DBC_FLAG_EXACT_BC rebase) stays
+    within 1e-9 of the oracle over all 256 roots after every batch -- no drift --
+    and every root's d/sigma/delta matches at the end."""
+    run_cadence("rmat16", 1000, sample=256, state_every=10, insertions=10000)
+
+
 @pytest.mark.timeout(600)
 def test_rmat16_bench_batch_all_roots():
     """Config 2 exactly as bench.py times it: one 1,000-insertion batch."""
