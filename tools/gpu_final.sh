@@ -20,4 +20,11 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:ms_k
 for c in rmat16 kron20 smallworld delaunay18; do timeout 900 python tools/static_probe.py $c static_ms=0 static_ms=1 > $O/static_$c.jsonl 2>&1; done
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:lean --launch-skip 20 --launch-count 1 -o $O/lean_full python tools/lean_ncu_target.py rmat16 40 > $O/ncu_lean.log 2>&1
 for c in rmat16 smallworld delaunay18; do timeout 900 python tools/paper_figures.py $c 100 > $O/fig_$c.json 2> $O/fig_$c.err; done
+# the batch kernel on the other configs (DRAM traffic for ncu_traffic.json)
+timeout 1200 ncu --set full --clock-control none -k regex:update_kernel --launch-skip 3 --launch-count 1 -o $O/upd_kron20 $N --config kron20 --steps 1 --warmup 3 > $O/ncu_upd_kron20.log 2>&1
+timeout 900 ncu --set full --clock-control none -k regex:update_kernel --launch-skip 3 --launch-count 1 -o $O/upd_delaunay18 $N --config delaunay18 --steps 1 --warmup 3 > $O/ncu_upd_del18.log 2>&1
+timeout 600 ncu --set full --clock-control none -k regex:update_kernel --launch-skip 3 --launch-count 1 -o $O/upd_smallworld $N --config smallworld --steps 1 --warmup 3 > $O/ncu_upd_sw.log 2>&1
+# per-insertion launch anatomy
+timeout 600 python tools/lean_anatomy.py rmat16 40 > $O/anatomy_rmat16.jsonl 2>&1
+timeout 600 python tools/batch_anatomy.py rmat16 6 > $O/batch_anatomy_rmat16.jsonl 2>&1
 ls -la $O
