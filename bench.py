@@ -374,10 +374,22 @@ def run_ours(args):
     torch.cuda.set_stream(stream)
     uid = None
     reducer = torch_reducer() if (world > 1 and one_gpu) else None
+    reduction = None
     if world > 1 and not one_gpu:  # the library's own NCCL communicator for the BC all-reduce (opt.nccl_id)
-        obj = [nccl_unique_id() if rank == 0 else None]
+        u0, why = None, None
+        if rank == 0:
+            try:
+                u0 = nccl_unique_id()
+            except Exception as ex:  # NCCL not loadable by the library: every rank falls back together
+                why = str(ex)
+        obj = [(u0, why)]
         dist.broadcast_object_list(obj, src=0)
-        uid = obj[0]
+        uid, why = obj[0]
+        if uid is None:
+            reducer = torch_reducer()  # torch.distributed's NCCL all-reduce as the reduce callback
+            reduction = f"torch.distributed all-reduce callback (library NCCL unavailable: {why})"
+        else:
+            reduction = "library NCCL communicator (dbc_options.nccl_id)"
     side_ok = world == 1  # side measurements on one GPU only (scaling runs stay short)
 
     def make(fl):
@@ -598,9 +610,9 @@ def run_ours(args):
             with open(nccl_log) as f:
                 lines = [ln.strip() for ln in f if ("NCCL version" in ln or "NVLS" in ln or "comm " in ln
                                                       or "Init COMPLETE" in ln)]
-            nccl = {"log": nccl_log, "lines": lines[:8]}
+            nccl = {"log": nccl_log, "lines": lines[:8], "bc_reduction": reduction}
         except OSError:
-            nccl = {"log": nccl_log, "lines": []}
+            nccl = {"log": nccl_log, "lines": [], "bc_reduction": reduction}
 
     # the committed capture is of one whole-root-set batch: only comparable at one rank
     traffic = ncu_traffic(args.config, B, args.mode, launches / K) if shard_world == 1 else None
