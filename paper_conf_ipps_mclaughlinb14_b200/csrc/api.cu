@@ -1516,6 +1516,19 @@ static dbc_status delete_host_ids(dbc_ctx *c, const int32_t *u, const int32_t *v
     }
     if (tm) CK(cudaEventRecord(ev[2], c->stream));
     int ulaunch = 0;
+    // One job per (root, deletion) is latency-bound like Mode S: 128-register
+    // CTAs -- 512 threads, one per SM; 256 threads, two per SM, where the batch
+    // runs two CTAs per SM (many roots, narrow levels: Delaunay) -- beat the
+    // batch configuration (R-MAT 16 2.55k -> 2.84k deletions/s, small world
+    // 3.17k -> 3.51k, Delaunay 2^18 353 -> 390/s).  An
+    // explicit dbc_tuning.update_block keeps the batch configuration.
+    int dblock = c->block, dworkers = c->workers;
+    bool dpair = c->ub2;
+    if (c->tune.update_block <= 0 && c->workers) {
+        dblock = c->ub2 ? 256 : 512;
+        dpair = false;
+        dworkers = std::max(1, std::min({c->k_loc, (c->ub2 ? 2 : 1) * c->nsm, (int)c->nscratch}));
+    }
     for (int64_t i = 0; i < cnt; ++i) {
         launches += tombstone_edge(c->rp[c->cur], c->col[c->cur], c->scol[c->cur], c->bu, c->bv, i,
                                    c->stream);
@@ -1524,14 +1537,14 @@ static dbc_status delete_host_ids(dbc_ctx *c, const int32_t *u, const int32_t *v
             c->lean_clean = false;
             a.ins_begin = (int32_t)i;
             a.ins_end = (int32_t)i + 1;
-            if (c->block == 128)
-                launch_update_128(a, c->workers, c->stream);
-            else if (c->block == 512)
-                (c->ub2 ? launch_update_512x2 : launch_update_512)(a, c->workers, c->stream);
-            else if (c->block == 1024)
-                launch_update_1024(a, c->workers, c->stream);
+            if (dblock == 128)
+                launch_update_128(a, dworkers, c->stream);
+            else if (dblock == 512)
+                (dpair ? launch_update_512x2 : launch_update_512)(a, dworkers, c->stream);
+            else if (dblock == 1024)
+                launch_update_1024(a, dworkers, c->stream);
             else
-                launch_update_256(a, c->workers, c->stream);
+                launch_update_256(a, dworkers, c->stream);
             ++ulaunch;
         }
     }
