@@ -449,10 +449,11 @@ __device__ __forceinline__ void lean_pass(const PassCtx &c, LeanSmem &S, int *s_
     }
 }
 
-// resident CTAs per SM the registers are sized for: 128 registers at 128
-// and 256 threads, 64 at 512 and 1024
+// resident CTAs per SM the registers are sized for: 128 registers at 128, 256
+// and 512 threads (one 512-thread CTA per SM: R-MAT 16 Mode S +9%, single-edge
+// update -10% against two 64-register CTAs), 64 at 1024
 #ifndef DBC_LEAN_MINB
-#define DBC_LEAN_MINB (kBlock <= 128 ? 4 : (kBlock == 256 ? 2 : 1024 / kBlock))
+#define DBC_LEAN_MINB (kBlock <= 128 ? 4 : (kBlock == 256 ? 2 : 1))
 #endif
 __global__ void __launch_bounds__(kBlock, DBC_LEAN_MINB) lean_kernel(UpdateArgs a) {
     __shared__ LeanSmem S;
