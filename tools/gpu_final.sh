@@ -28,3 +28,9 @@ timeout 600 ncu --set full --clock-control none -k regex:update_kernel --launch-
 timeout 600 python tools/lean_anatomy.py rmat16 40 > $O/anatomy_rmat16.jsonl 2>&1
 timeout 600 python tools/batch_anatomy.py rmat16 6 > $O/batch_anatomy_rmat16.jsonl 2>&1
 ls -la $O
+# summaries on the box (gpurun copies back <= 64 MiB): JSON per capture, then
+# only the R-MAT 16 batch-kernel report is kept
+for r in $O/*.ncu-rep; do python tools/ncu_summary.py raw $r > ${r%.ncu-rep}_summary.json 2>/dev/null; done
+python tools/ncu_summary.py launches $O/launches.csv > $O/launches_summary.json 2>/dev/null
+for r in $O/*.ncu-rep; do case $r in *update_full.ncu-rep) ;; *) rm -f $r ;; esac; done
+du -sh $O
