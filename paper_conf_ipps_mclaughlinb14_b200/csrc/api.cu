@@ -90,6 +90,8 @@ struct dbc_ctx {
     int lean_short = 4;              // level-2 shortcut threshold (rows > lean_short x deg(root))
     int lean_block = 128;            // threads per update_lean.cu CTA
     int lean_narrow = 0;             // > 0: 128-thread workers for multi-insertion launches (meshes)
+    int lean_pair = 0;               // > 0: 512-thread 64-register workers (two per SM) for
+                                     //      multi-insertion launches on hub graphs
     void *lean_board = nullptr;      // its help board (one entry per worker)
     size_t nscratch = 0;             // worker scratch sets allocated
     // heavy lanes: the slowest root chains of the previous batch run on
@@ -682,9 +684,19 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
             const int w = std::min({c->k_loc, fit, std::max(1, lean_resident_128()) * c->nsm});
             if (w > c->lean_workers) c->lean_narrow = w;
         }
+        // hub graphs: a single-insertion launch is set by its heaviest job, which
+        // wants one 128-register 512-thread CTA per SM; a launch over many
+        // insertions (DBC_FLAG_NO_MERGE) wants every root resident: two
+        // 64-register CTAs per SM (R-MAT 16: Mode S +9% / one job per
+        // insertion +12% against a single build)
+        if (T.lean_block <= 0 && c->lean_block == 512 && c->k_loc > c->lean_workers) {
+            const int w = std::min({c->k_loc, fit, std::max(1, lean_resident_512x2()) * c->nsm});
+            if (w > c->lean_workers) c->lean_pair = w;
+        }
     }
     const size_t nwk = std::max({(size_t)c->workers + c->heavy_cap, (size_t)c->sworkers,
-                                 (size_t)c->lean_workers, (size_t)c->lean_narrow});  // both lanes; static; per-insertion
+                                 (size_t)c->lean_workers, (size_t)c->lean_narrow,
+                                 (size_t)c->lean_pair});  // both lanes; static; per-insertion
     c->nscratch = nwk;
     const size_t wn = nwk * n;
     AL(c->ws.mark, wn);
@@ -718,7 +730,7 @@ extern "C" dbc_status dbc_create(dbc_ctx **out, int32_t n, const int64_t *row_pt
     AL(c->next_slot, 8);  // [0] next root, [1] heavy lane's next root / unused, [2..3] lean: roots done, idle, [4] lean: CTAs out
     if (c->lean_workers) {
         char *bd = nullptr;
-        const size_t nlw = (size_t)std::max(c->lean_workers, c->lean_narrow);
+        const size_t nlw = (size_t)std::max({c->lean_workers, c->lean_narrow, c->lean_pair});
         AL(bd, lean_board_bytes() * nlw);
         c->lean_board = (T.disable & DBC_TUNE_NO_LEAN_HELP) ? nullptr : (void *)bd;
         cudaMemsetAsync(bd, 0, lean_board_bytes() * nlw, c->stream);
@@ -1177,8 +1189,10 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
     a.pull_delta = pull ? 1 : 0;
     a.short_mult = c->lean_short;
     if (use_lean) {
-        const bool narrow = c->lean_narrow > 0 && !(c->flags & DBC_FLAG_MODE_S) && cnt > 1;
-        const int nw = narrow ? c->lean_narrow : c->lean_workers;
+        const bool many = !(c->flags & DBC_FLAG_MODE_S) && cnt > 1;  // one launch over many insertions
+        const bool narrow = c->lean_narrow > 0 && many;
+        const bool pair = c->lean_pair > 0 && many;
+        const int nw = narrow ? c->lean_narrow : (pair ? c->lean_pair : c->lean_workers);
         a.lean_board = pull ? nullptr : c->lean_board;  // pull mode: every pass local
         a.merge = 0;
         a.root_prof = c->prof_on ? c->root_prof : nullptr;
@@ -1195,6 +1209,8 @@ static dbc_status insert_device(dbc_ctx *c, const int32_t *u, const int32_t *v, 
             a.ins_end = (int32_t)std::min<int64_t>(cnt, i + step);
             if (narrow)
                 launch_update_lean_128(a, nw, c->stream);
+            else if (pair)
+                launch_update_lean_512x2(a, nw, c->stream);
             else if (c->lean_block == 1024)
                 launch_update_lean_1024(a, nw, c->stream);
             else if (c->lean_block == 512)

@@ -668,10 +668,12 @@ void launch_update_256(const UpdateArgs &a, int workers, cudaStream_t s);
 void launch_update_lean_128(const UpdateArgs &a, int workers, cudaStream_t s);
 void launch_update_lean_256(const UpdateArgs &a, int workers, cudaStream_t s);
 void launch_update_lean_512(const UpdateArgs &a, int workers, cudaStream_t s);
+void launch_update_lean_512x2(const UpdateArgs &a, int workers, cudaStream_t s);  // 64 registers, two per SM
 void launch_update_lean_1024(const UpdateArgs &a, int workers, cudaStream_t s);
 int lean_resident_128();  // resident CTAs per SM of each build
 int lean_resident_256();
 int lean_resident_512();
+int lean_resident_512x2();
 int lean_resident_1024();
 size_t lean_board_bytes();
 void launch_update_512x2(const UpdateArgs &a, int workers, cudaStream_t s);  // 64 regs, 2 CTAs/SM

@@ -1221,7 +1221,10 @@ size_t lean_board_bytes() { return sizeof(LeanBoard); }
 
 #define DBC_CAT2(a, b) a##b
 #define DBC_CAT(a, b) DBC_CAT2(a, b)
-void DBC_CAT(launch_update_lean_, DBC_BLOCK)(const UpdateArgs &a, int workers, cudaStream_t s) {
+#ifndef DBC_LEAN_SUFFIX
+#define DBC_LEAN_SUFFIX DBC_BLOCK
+#endif
+void DBC_CAT(launch_update_lean_, DBC_LEAN_SUFFIX)(const UpdateArgs &a, int workers, cudaStream_t s) {
     static bool attr = false;
     if (!attr) {
         cudaFuncSetAttribute(lean_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kLDyn);
@@ -1230,7 +1233,7 @@ void DBC_CAT(launch_update_lean_, DBC_BLOCK)(const UpdateArgs &a, int workers, c
     lean_kernel<<<workers, kBlock, kLDyn, s>>>(a);
 }
 
-int DBC_CAT(lean_resident_, DBC_BLOCK)() {
+int DBC_CAT(lean_resident_, DBC_LEAN_SUFFIX)() {
     int nb = 0;
     cudaFuncSetAttribute(lean_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kLDyn);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, lean_kernel, kBlock, kLDyn);

@@ -1065,6 +1065,25 @@ def test_lean_fewer_workers_than_roots(name, tune):
             check_all(dbc, want, wl.roots.size)
 
 
+def test_lean_two_builds_per_launch_kind():
+    """A hub graph with more roots than SMs: single-insertion launches run the
+    128-register 512-thread build (one per SM), a launch over many insertions
+    the 64-register build (two per SM, every root resident) -- both against the
+    oracle, and the two orders of use within one context."""
+    wl = W.make_workload("rmat10", k=300)
+    ref = oracle.NaiveDynamicBC(wl.graph, wl.roots)
+    for u, v in zip(wl.ins_u, wl.ins_v):
+        ref.insert(u, v)
+    want = ref.compute()
+    h = wl.ins_u.size // 2
+    with _dbc(wl.graph, wl.roots, flags=0x10) as dbc:  # DBC_FLAG_NO_MERGE
+        dbc.static_compute()
+        dbc.insert_edges(wl.ins_u[:h], wl.ins_v[:h])  # many insertions: two CTAs per SM
+        for u, v in zip(wl.ins_u[h:].tolist(), wl.ins_v[h:].tolist()):
+            dbc.insert_edges([u], [v])  # single insertions: one CTA per SM
+        check_all(dbc, want, wl.roots.size)
+
+
 @pytest.mark.parametrize("width", [128, 256, 512, 1024])
 def test_lean_every_cta_width(width, tune):
     """The per-insertion kernel at every CTA width (128/256/512/1024 threads:
